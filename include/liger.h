@@ -1,0 +1,258 @@
+/* liger.h — C ABI of the B200-native Liger hot path (libliger.so).
+ *
+ * Liger (Du et al., PPoPP'24; /root/reference/PAPER.md, cited as P:<line>)
+ * serves pre-packed request batches on a model sharded with intra-operator
+ * (Megatron tensor) parallelism and interleaves the
+ * computation kernels of one batch with the communication kernels of another
+ * (interleaved parallelism, §3.1), scheduled by Algorithm 1 (§3.4
+ * P:178-226) with hybrid CPU-GPU / inter-stream synchronization,
+ * a contention factor (§3.5) and runtime decomposition of long
+ * GEMMs and all-reduces into k/F pieces (§3.6).
+ *
+ * Conventions
+ *  - Every call returns an int status: 0 = LIGER_OK, > 0 informational,
+ *    < 0 error.  No C++ exception crosses this boundary.  liger_last_error()
+ *    returns a description of the last error of a context (or the global one
+ *    for ctx == NULL).
+ *  - Pointers documented "device" are CUDA device pointers (e.g. a torch
+ *    tensor's data_ptr()); "host" are ordinary host pointers.  The library
+ *    never frees memory it did not allocate (borrowed pointers).
+ *  - `stream` arguments are cudaStream_t handles (NULL = legacy default stream).
+ *  - All bf16 tensors are row-major and 16-byte aligned; fp32 accumulation.
+ *  - Calls marked [collective] must be made by every rank of a context, in the
+ *    same order and with the same arguments (NCCL ordering).
+ *  - One host thread per context; nothing is re-entrant.
+ *  - There is no CPU fallback: without a usable sm_100 device every compute
+ *    entry point returns LIGER_ENODEV.
+ */
+#ifndef LIGER_H_
+#define LIGER_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ------------------------------------------------------------------ status */
+#define LIGER_OK 0
+#define LIGER_PENDING 1   /* liger_poll: batch not finished yet              */
+#define LIGER_IDLE 2      /* liger_step: nothing to schedule                 */
+#define LIGER_EINVAL (-22)
+#define LIGER_ENOMEM (-12)
+#define LIGER_ECUDA (-1000)
+#define LIGER_ENCCL (-1001)
+#define LIGER_ESTATE (-1002)
+#define LIGER_ETIMEOUT (-1003)
+#define LIGER_ENODEV (-1004)
+
+/* ------------------------------------------------------------------ enums */
+#define LIGER_ACT_NONE 0
+#define LIGER_ACT_RELU 1      /* OPT (reading R13)                          */
+#define LIGER_ACT_GELU_TANH 2 /* tiny and GLM-shaped configs                */
+
+#define LIGER_MODE_SERIAL 0      /* Intra-Op baseline: compute then all-reduce, in order */
+#define LIGER_MODE_INTERLEAVED 1 /* Liger: Algorithm 1 + hybrid sync               */
+
+/* ------------------------------------------------------------------ config */
+typedef struct {
+  int32_t n_layers, hidden, n_heads, ffn, vocab, max_pos; /* model shape, Table 1  */
+  int32_t act;              /* LIGER_ACT_*                                                     */
+  float ln_eps;             /* LayerNorm epsilon (1e-5, reading R26)                           */
+  int32_t max_batch;        /* max sequences per submitted batch                               */
+  int32_t max_seq;          /* max prompt length                                               */
+  int32_t max_new;          /* max generated tokens per sequence                               */
+  int32_t mode;             /* LIGER_MODE_*                                                    */
+  int32_t max_inflight;     /* processing-list size; 1 => serial order         */
+  int32_t decomp_factor;    /* F (P:254, 8 in the paper); 1 => no decomposition               */
+  float contention_factor;  /* cf scaling secondary durations; <= 0 => 1.0            */
+  uint64_t seed;            /* seed of the counter-based weight generator (C0)       */
+} liger_cfg;
+
+typedef struct liger_ctx liger_ctx;
+
+typedef struct {
+  int64_t id;
+  int32_t batch, seq_len, n_new;
+  int32_t done;             /* 1 when finished                                                */
+  double arrival_s;         /* trace arrival time (seconds, caller's clock)                   */
+  double submit_s;          /* host monotonic time of liger_submit                            */
+  double start_s;           /* host monotonic time the first kernel was launched              */
+  double finish_s;          /* host monotonic time the final event was observed complete      */
+} liger_result;
+
+typedef struct {
+  int64_t rounds;           /* Algorithm 1 iterations                                          */
+  int64_t kernels;          /* kernel launches (compute + comm pieces)                         */
+  int64_t comm_kernels;
+  int64_t split_pieces;     /* decomposed pieces launched (k/F < 1)                            */
+  int64_t overlapped_rounds;/* rounds with a non-empty secondary subset                        */
+  double host_us;           /* host time spent in liger_step (plan + launch + waits)          */
+  double wait_us;           /* host time spent waiting on E1 events                            */
+  int64_t gpu_launches;     /* CUDA kernel launches issued by the library                     */
+} liger_stats_t;
+
+/* ------------------------------------------------------------------ lifecycle */
+
+/* Create a context for rank `rank` of `world` tensor-parallel ranks on the
+ * current CUDA device.  nccl_uid: host pointer to the 128-byte ncclUniqueId
+ * produced by liger_nccl_unique_id() on rank 0 and broadcast by the caller
+ * (e.g. torch.distributed); ignored (may be NULL) when world == 1.
+ * Allocates weights (uninitialised), the paged KV pool and per-slot
+ * activation buffers with cudaMalloc; creates a compute and a communication
+ * stream (CUDA_DEVICE_MAX_CONNECTIONS=2 is recommended).
+ * [collective]  Returns LIGER_ENODEV without an sm_100 device. */
+int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_uid, liger_ctx** out);
+
+/* Write a fresh ncclUniqueId (128 bytes) to host buffer `uid`. */
+int liger_nccl_unique_id(uint8_t* uid);
+
+/* Initialise this rank's shard of layer `layer` on the device with the
+ * counter-based generator C0 (global indices, so every rank gets
+ * its slice of the same logical weights).  seed overrides cfg->seed when != 0
+ * is not desired: pass cfg->seed for the configured model. [collective] */
+int liger_load_layer(liger_ctx* ctx, int layer, uint64_t seed);
+
+/* Initialise embeddings (token + learned positions), final LN. [collective] */
+int liger_load_embed(liger_ctx* ctx, uint64_t seed);
+
+/* Enqueue one pre-packed batch in the waiting queue.
+ * tokens: [batch * seq_len] int32 prompt ids, sequence-major; host pointer
+ * (copied to the device inside the library) or device pointer when
+ * tokens_on_device != 0 (must stay valid until the batch finishes).
+ * n_new: tokens to generate greedily (1 prefill pass + n_new - 1 decode passes,
+ * reading R22).  arrival_s: the request's arrival time on the caller's clock.
+ * Returns the batch id (>= 0) or an error (< 0). [collective] */
+int64_t liger_submit(liger_ctx* ctx, int batch, int seq_len, const int32_t* tokens, int tokens_on_device,
+                     int n_new, double arrival_s);
+
+/* One scheduling round (one iteration of Algorithm 1): update the
+ * processing list, wait for the running round's E1 event (hybrid sync,
+ * P:236), plan SubSet0/SubSet1 and launch them (communication first) gated
+ * on the running round's E2 event.  Returns the number of kernel pieces
+ * launched (>= 0), LIGER_IDLE when no batch is pending, or an error.
+ * [collective] */
+int liger_step(liger_ctx* ctx);
+
+/* Run liger_step until every submitted batch has been launched and finished. */
+int liger_drain(liger_ctx* ctx);
+
+/* Query a batch.  Returns LIGER_PENDING while unfinished, LIGER_OK when done.
+ * tokens_out: optional host buffer [batch * n_new] for the generated ids
+ * (copied device -> host on the first successful poll that passes it). */
+int liger_poll(liger_ctx* ctx, int64_t id, liger_result* out, int32_t* tokens_out);
+
+/* Device pointer to a finished batch's generated tokens [batch * n_new] int32
+ * (valid until the batch's slot is reused by a later submit). */
+int liger_result_tokens_device(liger_ctx* ctx, int64_t id, const int32_t** dev_tokens);
+
+int liger_stats(liger_ctx* ctx, liger_stats_t* out);
+int liger_reset_stats(liger_ctx* ctx);
+
+/* Enable (1) / disable (0) CUDA-event timing of every GEMM and attention
+ * launch on the stream it runs on; liger_kernel_timing returns, per kernel
+ * class (0 = GEMM, 1 = attention, 2 = layernorm, 3 = all-reduce), the launch
+ * count, the summed device milliseconds, and the summed algorithmic bytes and
+ * flops.  Arrays of length 4, host. */
+int liger_set_kernel_timing(liger_ctx* ctx, int on);
+int liger_kernel_timing(liger_ctx* ctx, int64_t* count, double* ms, double* bytes, double* flops);
+
+/* Set the per-kernel duration table used by Algorithm 1:
+ * durations in microseconds for a kernel class at a token count, piecewise
+ * linear in M between profiled points.  Called by the offline profiler
+ * (bench.py / liger_profile) or loaded from JSON by the binding. */
+int liger_set_duration(liger_ctx* ctx, int kclass, int m_tokens, int k_of_F, double us);
+
+/* Offline profiling: measure no-load durations of every
+ * kernel class at token counts m_list[0..n_m) for every piece size k/F and
+ * store them in the duration table.  Returns LIGER_OK. */
+int liger_profile(liger_ctx* ctx, const int32_t* m_list, int n_m);
+
+const char* liger_last_error(const liger_ctx* ctx);
+int liger_finalize(liger_ctx* ctx); /* [collective] */
+
+/* ------------------------------------------------------------------ kernel entry points
+ * The single kernels of the hot path, exposed for parity tests and roofline
+ * measurement.  All pointers are device pointers unless stated.  They launch
+ * asynchronously on `stream` and return LIGER_EINVAL on bad shapes. */
+
+/* GEMM with fused epilogue (§8(a) a3/a5/a8/a9, decomposition a13):
+ *   out[m, n] = act( (sum_k x[m,k] * w[n,k]) + bias[n] ) * (n < scale_cols ? scale : 1)
+ * for m < M and n in the slice [n0, n1) of the N output columns (PAPER.md
+ * §3.6 "vertical" split, Fig. 9).  x bf16 [M, K] row stride ldx; w bf16
+ * [N, K] row stride ldw; bias bf16 [N] or NULL; out bf16 (or fp32 if out_f32)
+ * with row stride ldo (columns n0..n1 written at their global index n).
+ * Scaling is applied after the bias and before the activation.
+ * workspace: device scratch of liger_gemm_workspace_bytes(M, N, K) bytes whose
+ * first 16 KiB must be zero before the first use (the kernel leaves them zero).
+ * The result for any column is bit-identical for every slice containing it. */
+int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* out, int64_t ldo, int M, int N,
+                  int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
+                  void* workspace, size_t ws_bytes, void* stream);
+size_t liger_gemm_workspace_bytes(int M, int N, int K);
+
+/* Fused residual add + LayerNorm (§8(a) a2/a7/a11; C2):
+ *   r    = x[in_row(i)] + (add ? add[in_row(i)] : 0) + (add_bias ? add_bias : 0)     (fp32)
+ *   x_out[i] = bf16(r)           (if x_out != NULL; may alias x when in_row(i) == i)
+ *   y[i] = bf16( (r' - mean(r')) / sqrt(var(r') + eps) * gamma + beta ),  r' = bf16(r)
+ * for i < rows, in_row(i) = i * in_row_step + in_row_off (gather of the last
+ * token of each sequence for the LM head).  All [*, h] bf16. */
+int liger_op_add_layernorm(const void* x, const void* add, const void* add_bias, void* x_out, void* y,
+                           const void* gamma, const void* beta, int rows, int h, int in_row_step,
+                           int in_row_off, float eps, void* stream);
+
+/* Embedding (§8(a) a1; C1): out[i] = E_tok[ids[i]] + E_pos[pos(i) + 2] with
+ * pos(i) = start_pos + (seq_len > 0 ? i % seq_len : 0); bf16 [rows, h]. */
+int liger_op_embed(const int32_t* ids, const void* e_tok, const void* e_pos, void* out, int rows, int h,
+                   int seq_len, int start_pos, void* stream);
+
+/* Paged KV cache geometry: page = kv_block (16) tokens; pool layout
+ * [n_pages][2 (K,V)][heads][16][d] bf16.  page_table: int32 [b][max_pages]. */
+#define LIGER_KV_BLOCK 16
+
+/* Prefill causal attention (§8(a) a4; C4) over qkv [b*s, 3*heads*d] bf16
+ * (row = token, columns [q heads | k heads | v heads], q pre-scaled),
+ * writing o [b*s, heads*d] bf16 and the K/V of all s positions into the pages. */
+int liger_op_attn_prefill(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages,
+                          int b, int s, int heads, int d, void* stream);
+
+/* Decode attention (§8(a) a4) for one new token per sequence at position
+ * `pos` (cache holds positions [0, pos)): qkv [b, 3*heads*d]; appends the
+ * token's K/V to the cache page; o [b, heads*d].  workspace: device scratch
+ * of liger_attn_decode_workspace_bytes(b, heads, d, pos + 1) bytes, first
+ * 16 KiB zero before first use (left zero). */
+int liger_op_attn_decode(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
+                         int pos, int heads, int d, void* workspace, size_t ws_bytes, void* stream);
+size_t liger_attn_decode_workspace_bytes(int b, int heads, int d, int ctx);
+
+/* Row-wise argmax over fp32 logits [rows, n] (row stride ld): writes the
+ * maximum value and its index + idx_offset (lowest index on ties, C7). */
+int liger_op_argmax(const float* logits, int64_t ld, int rows, int n, int idx_offset, float* max_out,
+                    int32_t* idx_out, void* stream);
+
+/* Fill a bf16 [rows, cols] (row stride ld) device tensor with C0 values of
+ * logical tensor `tensor_id`: element (r, c) takes global index
+ * (r + row_off) * idx_row_stride + (c + col_off) * idx_col_stride, scale 2^exp;
+ * kind 0 = plain, 1 = gamma (1 + v/16), 2 = beta (v/16). */
+int liger_op_c0_fill(void* dst, int rows, int cols, int64_t ld, uint64_t seed, uint64_t tensor_id,
+                     int64_t row_off, int64_t col_off, int64_t idx_row_stride, int64_t idx_col_stride, int exp,
+                     int kind, void* stream);
+
+/* ------------------------------------------------------------------ host-only scheduler (no GPU needed)
+ * Algorithm 1 planner exposed for CPU tests of the host logic.  A planner
+ * holds batches of kernels (type 0 = compute, 1 = communication) with
+ * per-piece durations; liger_plan_round runs one round and writes up to cap
+ * entries {batch, kernel index, unit begin, unit end, subset (0/1)}. */
+typedef struct liger_planner liger_planner;
+int liger_planner_create(int list_size, double cf, liger_planner** out);
+int liger_planner_submit(liger_planner* p, int64_t batch, int n_kernels, const int32_t* types,
+                         const int32_t* units, const double* durs /* per kernel: units entries */);
+int liger_plan_round(liger_planner* p, int32_t* entries /* [cap][5] */, int cap, int32_t* round_type,
+                     double* time0);
+int liger_planner_destroy(liger_planner* p);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LIGER_H_ */

@@ -1,0 +1,416 @@
+// Attention over the paged KV cache (PAPER.md P:316 KV cache).
+//
+// Paged pool layout: [n_pages][2 (K,V)][heads][16 tokens][d] bf16; a sequence's
+// page_table row maps token position p to page page_table[p / 16].
+//
+//  * prefill: flash-style causal attention with bf16 tensor-core mma.sync
+//    (m16n8k16, fp32 accumulate), 64 queries x 64 keys per step, online
+//    softmax in registers; the CTA on the diagonal tile also writes that key
+//    tile's K/V into the cache pages.
+//  * decode: one query per sequence; split over the context in fixed chunks
+//    of 256 positions (a function of ctx only), two-pass softmax per chunk
+//    with warp-shuffle dot products, deterministic merge of the chunk partials
+//    in chunk order by the last CTA to finish.
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+#include "common.cuh"
+#include "kernels.h"
+
+namespace liger {
+
+constexpr int KVB = LIGER_KV_BLOCK;
+
+__device__ __forceinline__ int64_t kv_off(int page, int kv, int heads, int head, int tok, int D) {
+  return ((((int64_t)page * 2 + kv) * heads + head) * KVB + tok) * D;
+}
+
+// ================================================================== prefill
+constexpr int PF_BQ = 64, PF_BK = 64;
+
+__device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
+               : "r"(addr));
+}
+__device__ __forceinline__ void ldsm_x4_t(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
+               : "r"(addr));
+}
+__device__ __forceinline__ void mma_bf16_16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
+                                               uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};"
+      : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+      : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+}
+__device__ __forceinline__ uint32_t pack_bf16(float lo, float hi) {
+  __nv_bfloat162 v = __floats2bfloat162_rn(lo, hi);
+  return *reinterpret_cast<uint32_t*>(&v);
+}
+
+template <int D>
+__global__ void __launch_bounds__(128) attn_prefill_kernel(const __nv_bfloat16* __restrict__ qkv,
+                                                           __nv_bfloat16* __restrict__ o,
+                                                           __nv_bfloat16* __restrict__ kv_pool,
+                                                           const int32_t* __restrict__ page_table, int max_pages,
+                                                           int s, int heads) {
+  constexpr int LDS = D + 8;   // padded smem row (bank-conflict-free ldmatrix)
+  constexpr int NV = D / 8;    // 16-byte vectors per row
+  extern __shared__ __align__(16) uint8_t pf_smem[];
+  __nv_bfloat16* sQ = reinterpret_cast<__nv_bfloat16*>(pf_smem);
+  __nv_bfloat16* sK = sQ + PF_BQ * LDS;
+  __nv_bfloat16* sV = sK + PF_BK * LDS;
+
+  const int qt = blockIdx.x, head = blockIdx.y, bi = blockIdx.z;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t ld = (int64_t)3 * heads * D;
+  const __nv_bfloat16* base = qkv + (int64_t)bi * s * ld;
+  const int q0 = qt * PF_BQ;
+
+  for (int i = tid; i < PF_BQ * NV; i += 128) {
+    const int r = i / NV, c = (i % NV) * 8;
+    uint4 v = make_uint4(0, 0, 0, 0);
+    if (q0 + r < s) v = *reinterpret_cast<const uint4*>(base + (int64_t)(q0 + r) * ld + head * D + c);
+    *reinterpret_cast<uint4*>(&sQ[r * LDS + c]) = v;
+  }
+
+  const int g = lane >> 2, tig = lane & 3;
+  float m_r[2] = {-INFINITY, -INFINITY}, l_r[2] = {0.f, 0.f};
+  float acc[D / 8][4];
+#pragma unroll
+  for (int j = 0; j < D / 8; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+  const float L2E = 1.4426950408889634f;
+  const int row0 = q0 + warp * 16 + g;   // this thread's rows: row0, row0 + 8
+
+  for (int kt = 0; kt <= qt; ++kt) {
+    const int k0 = kt * PF_BK;
+    __syncthreads();
+    for (int i = tid; i < PF_BK * NV; i += 128) {
+      const int r = i / NV, c = (i % NV) * 8;
+      uint4 kv = make_uint4(0, 0, 0, 0), vv = make_uint4(0, 0, 0, 0);
+      if (k0 + r < s) {
+        const __nv_bfloat16* rowp = base + (int64_t)(k0 + r) * ld;
+        kv = *reinterpret_cast<const uint4*>(rowp + (int64_t)heads * D + head * D + c);
+        vv = *reinterpret_cast<const uint4*>(rowp + (int64_t)2 * heads * D + head * D + c);
+        if (kt == qt) {   // diagonal CTA appends this key tile to the paged cache
+          const int p = k0 + r;
+          const int page = page_table[(int64_t)bi * max_pages + p / KVB];
+          *reinterpret_cast<uint4*>(kv_pool + kv_off(page, 0, heads, head, p % KVB, D) + c) = kv;
+          *reinterpret_cast<uint4*>(kv_pool + kv_off(page, 1, heads, head, p % KVB, D) + c) = vv;
+        }
+      }
+      *reinterpret_cast<uint4*>(&sK[r * LDS + c]) = kv;
+      *reinterpret_cast<uint4*>(&sV[r * LDS + c]) = vv;
+    }
+    __syncthreads();
+
+    // S = Q K^T for this warp's 16 rows x 64 keys
+    float sc[8][4];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) sc[j][0] = sc[j][1] = sc[j][2] = sc[j][3] = 0.f;
+#pragma unroll
+    for (int kc = 0; kc < D; kc += 16) {
+      uint32_t a0, a1, a2, a3;
+      const int ar = warp * 16 + (lane % 8) + ((lane / 8) % 2) * 8;
+      const int ac = kc + (lane / 16) * 8;
+      ldsm_x4(smem_u32(&sQ[ar * LDS + ac]), a0, a1, a2, a3);
+#pragma unroll
+      for (int nb = 0; nb < 8; nb += 2) {
+        uint32_t b0, b1, b2, b3;
+        const int br = nb * 8 + (lane % 8) + (lane / 16) * 8;
+        const int bc = kc + ((lane / 8) % 2) * 8;
+        ldsm_x4(smem_u32(&sK[br * LDS + bc]), b0, b1, b2, b3);
+        mma_bf16_16816(sc[nb], a0, a1, a2, a3, b0, b1);
+        mma_bf16_16816(sc[nb + 1], a0, a1, a2, a3, b2, b3);
+      }
+    }
+    // mask (causal on the diagonal tile; key padding beyond s)
+#pragma unroll
+    for (int nb = 0; nb < 8; ++nb) {
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const int key = k0 + nb * 8 + tig * 2 + (e & 1);
+        const int row = row0 + (e >> 1) * 8;
+        if (key > row || key >= s) sc[nb][e] = -INFINITY;
+      }
+    }
+    // online softmax
+#pragma unroll
+    for (int h2 = 0; h2 < 2; ++h2) {
+      float mx = -INFINITY;
+#pragma unroll
+      for (int nb = 0; nb < 8; ++nb) mx = fmaxf(mx, fmaxf(sc[nb][2 * h2], sc[nb][2 * h2 + 1]));
+      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
+      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
+      const float m_new = fmaxf(m_r[h2], mx);
+      const float corr = (m_r[h2] == -INFINITY) ? 0.f : exp2f((m_r[h2] - m_new) * L2E);
+      float sum = 0.f;
+#pragma unroll
+      for (int nb = 0; nb < 8; ++nb) {
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const float v = sc[nb][2 * h2 + e];
+          const float pv = (v == -INFINITY) ? 0.f : exp2f((v - m_new) * L2E);
+          sc[nb][2 * h2 + e] = pv;
+          sum += pv;
+        }
+      }
+      sum += __shfl_xor_sync(0xffffffffu, sum, 1);
+      sum += __shfl_xor_sync(0xffffffffu, sum, 2);
+      l_r[h2] = l_r[h2] * corr + sum;
+      m_r[h2] = m_new;
+#pragma unroll
+      for (int j = 0; j < D / 8; ++j) {
+        acc[j][2 * h2] *= corr;
+        acc[j][2 * h2 + 1] *= corr;
+      }
+    }
+    // O += P V
+#pragma unroll
+    for (int kc = 0; kc < 4; ++kc) {   // 16 keys per step
+      const uint32_t a0 = pack_bf16(sc[2 * kc][0], sc[2 * kc][1]);
+      const uint32_t a1 = pack_bf16(sc[2 * kc][2], sc[2 * kc][3]);
+      const uint32_t a2 = pack_bf16(sc[2 * kc + 1][0], sc[2 * kc + 1][1]);
+      const uint32_t a3 = pack_bf16(sc[2 * kc + 1][2], sc[2 * kc + 1][3]);
+#pragma unroll
+      for (int nb = 0; nb < D / 8; nb += 2) {
+        uint32_t b0, b1, b2, b3;
+        const int vr = kc * 16 + (lane % 8) + ((lane / 8) % 2) * 8;
+        const int vc = nb * 8 + (lane / 16) * 8;
+        ldsm_x4_t(smem_u32(&sV[vr * LDS + vc]), b0, b1, b2, b3);
+        mma_bf16_16816(acc[nb], a0, a1, a2, a3, b0, b1);
+        mma_bf16_16816(acc[nb + 1], a0, a1, a2, a3, b2, b3);
+      }
+    }
+  }
+  // normalise and store
+#pragma unroll
+  for (int h2 = 0; h2 < 2; ++h2) {
+    const int row = row0 + h2 * 8;
+    if (row < s) {
+      const float inv = 1.0f / l_r[h2];
+      __nv_bfloat16* orow = o + ((int64_t)bi * s + row) * ((int64_t)heads * D) + head * D;
+#pragma unroll
+      for (int nb = 0; nb < D / 8; ++nb) {
+        const int c = nb * 8 + tig * 2;
+        *reinterpret_cast<__nv_bfloat162*>(orow + c) =
+            __floats2bfloat162_rn(acc[nb][2 * h2] * inv, acc[nb][2 * h2 + 1] * inv);
+      }
+    }
+  }
+}
+
+int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
+                        int s, int heads, int d, cudaStream_t stream) {
+  if (b <= 0 || s <= 0) return 0;
+  dim3 grid((s + PF_BQ - 1) / PF_BQ, heads, b);
+  const size_t smem = (size_t)(PF_BQ + 2 * PF_BK) * (d + 8) * 2;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(attn_prefill_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+    cudaFuncSetAttribute(attn_prefill_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+    attr = true;
+  }
+  if (d == 128)
+    attn_prefill_kernel<128><<<grid, 128, smem, stream>>>((const __nv_bfloat16*)qkv, (__nv_bfloat16*)o,
+                                                       (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
+  else if (d == 64)
+    attn_prefill_kernel<64><<<grid, 128, smem, stream>>>((const __nv_bfloat16*)qkv, (__nv_bfloat16*)o,
+                                                      (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
+  else
+    return LIGER_EINVAL;
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+// ================================================================== decode
+constexpr int DC_CHUNK = 256;
+constexpr int DC_THREADS = 128;
+
+size_t attn_decode_workspace_bytes(int b, int heads, int d, int ctx) {
+  const int ns = (ctx + DC_CHUNK - 1) / DC_CHUNK;
+  return ATTN_COUNTER_BYTES + (size_t)b * heads * ns * (d + 2) * sizeof(float);
+}
+
+template <int D>
+__global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bfloat16* __restrict__ qkv,
+                                                                 __nv_bfloat16* __restrict__ o,
+                                                                 __nv_bfloat16* __restrict__ kv_pool,
+                                                                 const int32_t* __restrict__ page_table,
+                                                                 int max_pages, int pos, int heads, float* ws,
+                                                                 int* counters) {
+  constexpr int LPT = D / 8;          // lanes per token (8 bf16 each)
+  constexpr int TPW = 32 / LPT;       // tokens per warp step
+  constexpr int NVEC = D / 8;
+  constexpr int SLOTS = DC_THREADS / NVEC;
+  __shared__ float sc[DC_CHUNK];
+  __shared__ float red[DC_THREADS / 32];
+  __shared__ float part[SLOTS][D];
+  __shared__ int last;
+
+  const int head = blockIdx.x, bi = blockIdx.y, sp = blockIdx.z, nsp = gridDim.z;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int ctx = pos + 1;
+  const int t0 = sp * DC_CHUNK, t1 = min(ctx, t0 + DC_CHUNK);
+  const int64_t ld = (int64_t)3 * heads * D;
+  const __nv_bfloat16* row = qkv + (int64_t)bi * ld;
+  const __nv_bfloat16* qp = row + head * D;
+  const __nv_bfloat16* knew = row + (int64_t)heads * D + head * D;
+  const __nv_bfloat16* vnew = row + (int64_t)2 * heads * D + head * D;
+  const int32_t* pt = page_table + (int64_t)bi * max_pages;
+
+  if (sp == nsp - 1 && tid < 2 * NVEC) {   // append the new token's K/V (position pos)
+    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
+    const int page = pt[pos / KVB];
+    *reinterpret_cast<uint4*>(kv_pool + kv_off(page, kv, heads, head, pos % KVB, D) + c) =
+        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
+  }
+
+  // pass 1: scores
+  float qf[8];
+  {
+    const int c = (lane % LPT) * 8;
+    uint4 qv = *reinterpret_cast<const uint4*>(qp + c);
+    const __nv_bfloat162* qh = reinterpret_cast<const __nv_bfloat162*>(&qv);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      float2 f = __bfloat1622float2(qh[i]);
+      qf[2 * i] = f.x;
+      qf[2 * i + 1] = f.y;
+    }
+  }
+  for (int tb = t0 + warp * TPW; tb < t1; tb += 4 * TPW) {
+    const int t = tb + lane / LPT;
+    float dot = 0.f;
+    if (t < t1) {
+      const int c = (lane % LPT) * 8;
+      const __nv_bfloat16* kp =
+          (t == pos) ? knew + c : kv_pool + kv_off(pt[t / KVB], 0, heads, head, t % KVB, D) + c;
+      uint4 kv = *reinterpret_cast<const uint4*>(kp);
+      const __nv_bfloat162* kh = reinterpret_cast<const __nv_bfloat162*>(&kv);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        float2 f = __bfloat1622float2(kh[i]);
+        dot += qf[2 * i] * f.x + qf[2 * i + 1] * f.y;
+      }
+    }
+#pragma unroll
+    for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
+    if (t < t1 && (lane % LPT) == 0) sc[t - t0] = dot;
+  }
+  __syncthreads();
+  const int n = t1 - t0;
+  float mx = -INFINITY;
+  for (int i = tid; i < n; i += DC_THREADS) mx = fmaxf(mx, sc[i]);
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+  if (lane == 0) red[warp] = mx;
+  __syncthreads();
+  mx = fmaxf(fmaxf(red[0], red[1]), fmaxf(red[2], red[3]));
+  __syncthreads();
+  float sum = 0.f;
+  for (int i = tid; i < n; i += DC_THREADS) {
+    const float p = __expf(sc[i] - mx);
+    sc[i] = p;
+    sum += p;
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
+  if (lane == 0) red[warp] = sum;
+  __syncthreads();
+  const float l = red[0] + red[1] + red[2] + red[3];
+
+  // pass 2: o = sum_t p_t v_t ; thread = (slot, vector)
+  const int vec = tid % NVEC, slot = tid / NVEC;
+  float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  for (int t = t0 + slot; t < t1; t += SLOTS) {
+    const __nv_bfloat16* vp =
+        (t == pos) ? vnew + vec * 8 : kv_pool + kv_off(pt[t / KVB], 1, heads, head, t % KVB, D) + vec * 8;
+    uint4 vv = *reinterpret_cast<const uint4*>(vp);
+    const __nv_bfloat162* vh = reinterpret_cast<const __nv_bfloat162*>(&vv);
+    const float p = sc[t - t0];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      float2 f = __bfloat1622float2(vh[i]);
+      acc[2 * i] += p * f.x;
+      acc[2 * i + 1] += p * f.y;
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) part[slot][vec * 8 + i] = acc[i];
+  __syncthreads();
+
+  if (nsp == 1) {
+    for (int e = tid; e < D; e += DC_THREADS) {
+      float a = 0.f;
+      for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
+      o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / l);
+    }
+    return;
+  }
+  // split: write partial (m, l, acc[D]); the last CTA merges in split order
+  const int64_t unit = (int64_t)bi * heads + head;
+  float* wp = ws + (unit * nsp + sp) * (D + 2);
+  for (int e = tid; e < D; e += DC_THREADS) {
+    float a = 0.f;
+    for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
+    wp[e] = a;
+  }
+  if (tid == 0) {
+    wp[D] = mx;
+    wp[D + 1] = l;
+  }
+  __threadfence();
+  __syncthreads();
+  if (tid == 0) last = (atomicAdd(&counters[unit], 1) == nsp - 1);
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  float M = -INFINITY;
+  for (int s2 = 0; s2 < nsp; ++s2) M = fmaxf(M, __ldcg(&ws[(unit * nsp + s2) * (D + 2) + D]));
+  float L = 0.f;
+  for (int s2 = 0; s2 < nsp; ++s2) {
+    const float* w2 = ws + (unit * nsp + s2) * (D + 2);
+    L += __ldcg(&w2[D + 1]) * __expf(__ldcg(&w2[D]) - M);
+  }
+  for (int e = tid; e < D; e += DC_THREADS) {
+    float a = 0.f;
+    for (int s2 = 0; s2 < nsp; ++s2) {
+      const float* w2 = ws + (unit * nsp + s2) * (D + 2);
+      a += __ldcg(&w2[e]) * __expf(__ldcg(&w2[D]) - M);
+    }
+    o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / L);
+  }
+  if (tid == 0) counters[unit] = 0;
+}
+
+int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
+                       int pos, int heads, int d, void* workspace, size_t ws_bytes, cudaStream_t stream) {
+  if (b <= 0) return 0;
+  const int ctx = pos + 1;
+  const int ns = (ctx + DC_CHUNK - 1) / DC_CHUNK;
+  if (ns > 1) {
+    if (!workspace || ws_bytes < attn_decode_workspace_bytes(b, heads, d, ctx) ||
+        (size_t)b * heads * 4 > ATTN_COUNTER_BYTES)
+      return LIGER_EINVAL;
+  }
+  int* counters = (int*)workspace;
+  float* ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
+  dim3 grid(heads, b, ns);
+  if (d == 128)
+    attn_decode_kernel<128><<<grid, DC_THREADS, 0, stream>>>((const __nv_bfloat16*)qkv, (__nv_bfloat16*)o,
+                                                              (__nv_bfloat16*)kv_pool, page_table, max_pages, pos,
+                                                              heads, ws, counters);
+  else if (d == 64)
+    attn_decode_kernel<64><<<grid, DC_THREADS, 0, stream>>>((const __nv_bfloat16*)qkv, (__nv_bfloat16*)o,
+                                                             (__nv_bfloat16*)kv_pool, page_table, max_pages, pos,
+                                                             heads, ws, counters);
+  else
+    return LIGER_EINVAL;
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+}  // namespace liger

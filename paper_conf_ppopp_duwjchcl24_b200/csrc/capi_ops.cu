@@ -1,0 +1,117 @@
+// C-ABI wrappers of the single hot-path kernels (include/liger.h "kernel entry points").
+#include <cuda_runtime.h>
+#include <stdio.h>
+#include <string.h>
+#include <mutex>
+#include <string>
+
+#include "kernels.h"
+
+namespace liger {
+
+static std::mutex g_err_mu;
+static std::string g_last_error;
+
+void set_global_error(const std::string& s) {
+  std::lock_guard<std::mutex> g(g_err_mu);
+  g_last_error = s;
+}
+const char* global_error() { return g_last_error.c_str(); }
+
+// Returns 0 if the current device is an sm_100 part, LIGER_ENODEV otherwise.
+int check_device() {
+  static int state = 1;   // 1 = unknown
+  static std::once_flag once;
+  std::call_once(once, [] {
+    int dev = 0, n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
+      state = LIGER_ENODEV;
+      cudaGetLastError();
+      return;
+    }
+    cudaGetDevice(&dev);
+    cudaDeviceProp p;
+    cudaGetDeviceProperties(&p, dev);
+    state = (p.major == 10) ? 0 : LIGER_ENODEV;
+  });
+  if (state) set_global_error("liger: no sm_100 (B200) CUDA device available; there is no CPU fallback");
+  return state;
+}
+
+static int ret(int rc, const char* what) {
+  if (rc) {
+    char buf[256];
+    snprintf(buf, sizeof buf, "%s failed: status %d (%s)", what, rc, cudaGetErrorString(cudaGetLastError()));
+    set_global_error(buf);
+  }
+  return rc;
+}
+
+}  // namespace liger
+
+using namespace liger;
+
+extern "C" {
+
+int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* out, int64_t ldo, int M, int N,
+                  int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
+                  void* workspace, size_t ws_bytes, void* stream) {
+  if (int rc = check_device()) return rc;
+  GemmArgs a{x, ldx, w, ldw, out, ldo, M, N, K, n0, n1, bias, act, scale_cols, scale, out_f32, workspace, ws_bytes};
+  return ret(gemm_launch(a, (cudaStream_t)stream), "liger_op_gemm");
+}
+
+size_t liger_gemm_workspace_bytes(int M, int N, int K) { return gemm_workspace_bytes(M, N, K); }
+
+int liger_op_add_layernorm(const void* x, const void* add, const void* add_bias, void* x_out, void* y,
+                           const void* gamma, const void* beta, int rows, int h, int in_row_step, int in_row_off,
+                           float eps, void* stream) {
+  if (int rc = check_device()) return rc;
+  return ret(add_layernorm_launch(x, add, add_bias, x_out, y, gamma, beta, rows, h, in_row_step, in_row_off, eps,
+                                  (cudaStream_t)stream),
+             "liger_op_add_layernorm");
+}
+
+int liger_op_embed(const int32_t* ids, const void* e_tok, const void* e_pos, void* out, int rows, int h,
+                   int seq_len, int start_pos, void* stream) {
+  if (int rc = check_device()) return rc;
+  return ret(embed_launch(ids, e_tok, e_pos, out, rows, h, seq_len, start_pos, (cudaStream_t)stream),
+             "liger_op_embed");
+}
+
+int liger_op_attn_prefill(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
+                          int s, int heads, int d, void* stream) {
+  if (int rc = check_device()) return rc;
+  return ret(attn_prefill_launch(qkv, o, kv_pool, page_table, max_pages, b, s, heads, d, (cudaStream_t)stream),
+             "liger_op_attn_prefill");
+}
+
+int liger_op_attn_decode(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
+                         int pos, int heads, int d, void* workspace, size_t ws_bytes, void* stream) {
+  if (int rc = check_device()) return rc;
+  return ret(attn_decode_launch(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, d, workspace, ws_bytes,
+                                (cudaStream_t)stream),
+             "liger_op_attn_decode");
+}
+
+size_t liger_attn_decode_workspace_bytes(int b, int heads, int d, int ctx) {
+  return attn_decode_workspace_bytes(b, heads, d, ctx);
+}
+
+int liger_op_argmax(const float* logits, int64_t ld, int rows, int n, int idx_offset, float* max_out,
+                    int32_t* idx_out, void* stream) {
+  if (int rc = check_device()) return rc;
+  return ret(argmax_launch(logits, ld, rows, n, idx_offset, max_out, idx_out, (cudaStream_t)stream),
+             "liger_op_argmax");
+}
+
+int liger_op_c0_fill(void* dst, int rows, int cols, int64_t ld, uint64_t seed, uint64_t tensor_id, int64_t row_off,
+                     int64_t col_off, int64_t idx_row_stride, int64_t idx_col_stride, int exp, int kind,
+                     void* stream) {
+  if (int rc = check_device()) return rc;
+  return ret(c0_fill_launch(dst, rows, cols, ld, seed, tensor_id, row_off, col_off, idx_row_stride, idx_col_stride,
+                            exp, kind, (cudaStream_t)stream),
+             "liger_op_c0_fill");
+}
+
+}  // extern "C"

@@ -1,0 +1,1221 @@
+// Liger runtime: sharded weights, paged KV pool, batch state machines ("function
+// assembly", §3.2), waiting queue + processing list (§3.3
+// P:168), Algorithm 1 rounds with hybrid synchronization (§3.4),
+// contention factor (§3.5) and runtime decomposition (§3.6).
+//
+// One process per GPU; tensor-parallel ranks talk through NCCL (loaded with
+// dlopen, bootstrapped with a caller-broadcast ncclUniqueId).  Computation
+// kernels run on the compute stream, all-reduce / all-gather pieces on the
+// communication stream.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string.h>
+#include <time.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cmath>
+#include <deque>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "kernels.h"
+#include "planner.h"
+
+namespace liger {
+void set_global_error(const std::string& s);
+const char* global_error();
+int check_device();
+}  // namespace liger
+
+using namespace liger;
+
+// ------------------------------------------------------------------ NCCL (dlopen)
+namespace {
+struct NcclApi {
+  bool ok = false;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*);
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int);
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t);
+  ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t);
+  ncclResult_t (*GroupStart)();
+  ncclResult_t (*GroupEnd)();
+  ncclResult_t (*CommDestroy)(ncclComm_t);
+  ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t*);
+  const char* (*GetErrorString)(ncclResult_t);
+};
+
+NcclApi& nccl() {
+  static NcclApi api;
+  static bool tried = false;
+  if (tried) return api;
+  tried = true;
+  const char* names[] = {"libnccl.so.2", "libnccl.so",
+                         "/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl/lib/libnccl.so.2"};
+  void* h = nullptr;
+  for (const char* n : names)
+    if ((h = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
+  if (!h) return api;
+#define LIGER_SYM(field, name) api.field = reinterpret_cast<decltype(api.field)>(dlsym(h, name))
+  LIGER_SYM(GetUniqueId, "ncclGetUniqueId");
+  LIGER_SYM(CommInitRank, "ncclCommInitRank");
+  LIGER_SYM(AllReduce, "ncclAllReduce");
+  LIGER_SYM(AllGather, "ncclAllGather");
+  LIGER_SYM(GroupStart, "ncclGroupStart");
+  LIGER_SYM(GroupEnd, "ncclGroupEnd");
+  LIGER_SYM(CommDestroy, "ncclCommDestroy");
+  LIGER_SYM(CommGetAsyncError, "ncclCommGetAsyncError");
+  LIGER_SYM(GetErrorString, "ncclGetErrorString");
+#undef LIGER_SYM
+  api.ok = api.GetUniqueId && api.CommInitRank && api.AllReduce && api.AllGather && api.GroupStart &&
+           api.GroupEnd && api.CommDestroy;
+  return api;
+}
+
+double now_s() {
+  timespec ts;
+  clock_gettime(CLOCK_MONOTONIC, &ts);
+  return ts.tv_sec + ts.tv_nsec * 1e-9;
+}
+
+// weight scale exponent of a GEMM with logical fan-in K (C0): round-half-even
+int weight_exp(int K) { return (int)std::nearbyint(0.5 * std::log2(3.0 / K)) - 1; }
+constexpr int BIAS_EXP = -6, EMB_EXP = -3;
+constexpr uint64_t GID_ETOK = 0xFFFF00, GID_EPOS = 0xFFFF01, GID_LNFG = 0xFFFF02, GID_LNFB = 0xFFFF03;
+
+// ------------------------------------------------------------------ ops of one pass
+enum Op { OP_EMBED, OP_LN1, OP_QKV, OP_ATTN, OP_OUT, OP_AR1, OP_LN2, OP_FC1, OP_FC2, OP_AR2, OP_HEAD, OP_TOKG,
+          OP_PICK, OP_COUNT };
+const char* kOpName[OP_COUNT] = {"embed", "ln1", "qkv", "attn", "out", "ar1", "ln2", "fc1", "fc2", "ar2",
+                                 "head",  "tokg", "pick"};
+inline bool op_is_comm(int op) { return op == OP_AR1 || op == OP_AR2 || op == OP_TOKG; }
+inline bool op_is_gemm(int op) { return op == OP_QKV || op == OP_OUT || op == OP_FC1 || op == OP_FC2; }
+inline bool op_is_ar(int op) { return op == OP_AR1 || op == OP_AR2; }
+
+struct PassOp {
+  int op, layer;
+};
+
+struct bf16p {
+  void* p = nullptr;
+};
+
+struct LayerW {
+  void *w_qkv, *b_qkv, *w_o, *b_o, *w_1, *b_1, *w_2, *b_2, *g1, *be1, *g2, *be2;
+};
+
+// Per in-flight batch slot device buffers.
+struct Slot {
+  void *x, *y, *qkv, *attn, *part, *hbuf, *yhead;
+  float *logits, *vals_all;
+  int32_t *idx_all, *cur_tok, *tok_out, *prompt, *page_table;
+  void *gemm_ws, *attn_ws;
+  size_t gemm_ws_bytes, attn_ws_bytes;
+  int32_t* h_page_table;   // pinned
+  int32_t* h_prompt;       // pinned
+  int32_t* h_tok_out;      // pinned
+  cudaEvent_t free_ev;     // completes when the last batch using the slot finished
+  bool busy = false;
+};
+
+struct DurTable {
+  // per op: M grid x (F+1) pieces; linear interpolation in M
+  std::vector<int> mgrid;
+  std::vector<std::vector<double>> t[OP_COUNT];   // t[op][mi][k] (k = 0..F)
+  bool have = false;
+};
+
+struct Batch;
+
+struct Engine;
+
+struct Piece {
+  Batch* bt;
+  int pass, idx, u0, u1;
+};
+
+struct Batch {
+  int64_t id;
+  int b, s, n_new;
+  double arrival_s, submit_s, start_s = 0;
+  std::atomic<double> finish_s{0.0};
+  const int32_t* dev_tokens = nullptr;   // user device tokens (tokens_on_device)
+  std::vector<int32_t> host_tokens;
+  bool results_to_host = true;
+  int slot = -1;
+  std::vector<int> pages;
+  // cursor
+  int pass = 0, idx = 0, done = 0;   // done = units of the current op already launched
+  bool all_launched = false, finished = false, results_copied = false;
+  cudaEvent_t last_ev = nullptr;
+  int last_stream = -1;
+  bool has_last_ev = false;
+  cudaEvent_t final_ev = nullptr;
+  std::vector<int32_t> tokens;   // host copy of results
+  Engine* eng = nullptr;
+};
+
+}  // namespace
+
+struct liger_ctx {
+  int world = 1, rank = 0;
+  liger_cfg cfg;
+  int h, a, d, f, V, hl, al, fl, Vl, L, F;
+  double cf;
+  std::string err;
+  ncclComm_t comm = nullptr;
+  cudaStream_t s_comp = nullptr, s_comm = nullptr;
+  std::vector<LayerW> layers;
+  void *e_tok = nullptr, *e_pos = nullptr, *lnf_g = nullptr, *lnf_b = nullptr;
+  std::vector<void*> allocs;
+  // KV pool
+  void* kv = nullptr;
+  int n_pages = 0, max_pages = 0;
+  size_t kv_layer_elems = 0;
+  std::vector<int> free_pages;
+  std::vector<Slot> slots;
+  std::vector<PassOp> pass_ops;
+  // scheduler state
+  std::deque<std::unique_ptr<Batch>> waiting;
+  std::vector<Batch*> processing;
+  std::vector<std::unique_ptr<Batch>> all_batches;   // id -> batch
+  int64_t next_id = 0;
+  cudaEvent_t e1 = nullptr, e2 = nullptr;
+  bool have_round = false;
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_next = 0;
+  DurTable dur;
+  double attn_scale[2] = {1.0, 1.0};   // calibration of the attention duration model (prefill, decode)
+  bool ar_atomic_chunks = false;
+  // stats / timing
+  liger_stats_t st{};
+  bool timing = false;
+  struct TimedLaunch {
+    int cls;
+    cudaEvent_t a, b;
+    double bytes, flops;
+  };
+  std::vector<TimedLaunch> timed;
+  std::vector<cudaEvent_t> timing_pool;
+  size_t timing_next = 0;
+  int64_t tcount[4] = {0, 0, 0, 0};
+  double tms[4] = {0, 0, 0, 0}, tbytes[4] = {0, 0, 0, 0}, tflops[4] = {0, 0, 0, 0};
+};
+
+namespace {
+
+int fail(liger_ctx* c, int rc, const std::string& msg) {
+  if (c) c->err = msg;
+  set_global_error(msg);
+  return rc;
+}
+
+#define CK(call)                                                                                   \
+  do {                                                                                             \
+    cudaError_t e_ = (call);                                                                       \
+    if (e_ != cudaSuccess)                                                                         \
+      return fail(c, LIGER_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_));             \
+  } while (0)
+#define CKR(call)                                                                                  \
+  do {                                                                                             \
+    int r_ = (call);                                                                               \
+    if (r_ < 0) return fail(c, r_, std::string(#call) + " failed");                                \
+  } while (0)
+
+void* dalloc(liger_ctx* c, size_t bytes) {
+  void* p = nullptr;
+  if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) return nullptr;
+  c->allocs.push_back(p);
+  return p;
+}
+
+// Ring of reusable events for per-batch cross-stream dependencies.  Re-recording
+// an event that an older wait still references is safe: cudaStreamWaitEvent
+// captures the event's state at the time of the call.
+cudaEvent_t pool_event(liger_ctx* c) {
+  if (c->ev_pool.empty()) {
+    c->ev_pool.resize(4096);
+    for (auto& e : c->ev_pool) cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+  }
+  return c->ev_pool[c->ev_next++ % c->ev_pool.size()];
+}
+
+// ------------------------------------------------------------------ geometry helpers
+int op_units(liger_ctx* c, int op) {
+  if (c->F <= 1) return 1;
+  if (op_is_gemm(op) || (op_is_ar(op) && c->world > 1)) return c->F;
+  return 1;
+}
+
+int gemm_N(liger_ctx* c, int op) {
+  switch (op) {
+    case OP_QKV: return 3 * c->hl;
+    case OP_OUT: return c->h;
+    case OP_FC1: return c->fl;
+    case OP_FC2: return c->h;
+  }
+  return 0;
+}
+int gemm_K(liger_ctx* c, int op) {
+  switch (op) {
+    case OP_QKV: return c->h;
+    case OP_OUT: return c->hl;
+    case OP_FC1: return c->h;
+    case OP_FC2: return c->fl;
+  }
+  return 0;
+}
+// column boundary of unit u (of F) for an N-wide GEMM: multiples of 16, last = N
+int unit_col(int N, int u, int F) {
+  if (u >= F) return N;
+  int c = (int)((int64_t)N * u / F);
+  return c / 16 * 16;
+}
+
+int batch_M(const Batch* bt, int pass) { return pass == 0 ? bt->b * bt->s : bt->b; }
+
+// ------------------------------------------------------------------ durations
+double model_dur(liger_ctx* c, int op, int M, int k, int ctx_len, int s_len) {
+  const double F = c->F > 1 ? c->F : 1;
+  const double frac = (op_units(c, op) > 1) ? k / F : 1.0;
+  const double bw = 5.0e12, tc = 1.0e15;
+  if (op_is_gemm(op)) {
+    const double N = gemm_N(c, op) * frac, K = gemm_K(c, op);
+    return 4e-6 + std::max(2.0 * M * N * K / tc, (N * K + M * K + M * N) * 2 / bw);
+  }
+  if (op_is_ar(op)) {
+    const double bytes = (double)M * c->h * 2 * frac;
+    return 8e-6 + bytes * 2 * (c->world - 1) / c->world / 600e9;
+  }
+  switch (op) {
+    case OP_EMBED:
+    case OP_LN1:
+    case OP_LN2: return 3e-6 + (double)M * c->h * 2 * 3 / bw;
+    case OP_ATTN:
+      if (s_len > 0) return 5e-6 + 4.0 * M * s_len * c->al * c->d / 2 / 3e14;
+      return 5e-6 + 4.0 * M * ctx_len * c->al * c->d / bw;
+    case OP_HEAD: return 10e-6 + (double)c->Vl * c->h * 2 / bw;
+    case OP_TOKG: return 10e-6;
+    case OP_PICK: return 2e-6;
+  }
+  return 5e-6;
+}
+
+double table_dur(liger_ctx* c, int op, int M, int k) {
+  const DurTable& T = c->dur;
+  if (!T.have || T.t[op].empty()) return -1;
+  const auto& g = T.mgrid;
+  auto at = [&](size_t mi) { return T.t[op][mi][k]; };
+  double v;
+  if (M <= g.front()) {
+    v = at(0);
+  } else if (M >= g.back()) {
+    v = at(g.size() - 1) * (double)M / g.back();
+  } else {
+    size_t i = 1;
+    while (g[i] < M) ++i;
+    const double w = (double)(M - g[i - 1]) / (g[i] - g[i - 1]);
+    if (at(i - 1) <= 0 || at(i) <= 0) return -1;
+    v = at(i - 1) * (1 - w) + at(i) * w;
+  }
+  return v > 0 ? v : -1;
+}
+
+double op_dur(liger_ctx* c, const Batch* bt, int pass, int op, int k) {
+  const int M = batch_M(bt, pass);
+  const int ctx_len = bt->s + pass;
+  const int s_len = pass == 0 ? bt->s : 0;
+  if (op == OP_ATTN) {
+    const double m = model_dur(c, op, M, k, ctx_len, s_len);
+    return m * (s_len > 0 ? c->attn_scale[0] : c->attn_scale[1]);
+  }
+  const int kk = op_units(c, op) > 1 ? k : std::max(1, c->F);
+  const double t = table_dur(c, op, M, kk);
+  return t > 0 ? t : model_dur(c, op, M, k, ctx_len, s_len);
+}
+
+// ------------------------------------------------------------------ timing instrumentation
+void timed_begin(liger_ctx* c, cudaStream_t s, cudaEvent_t* a) {
+  if (!c->timing) return;
+  if (c->timing_next + 2 > c->timing_pool.size()) {
+    for (int i = 0; i < 256; ++i) {
+      cudaEvent_t e;
+      cudaEventCreate(&e);
+      c->timing_pool.push_back(e);
+    }
+  }
+  *a = c->timing_pool[c->timing_next++];
+  cudaEventRecord(*a, s);
+}
+void timed_end(liger_ctx* c, cudaStream_t s, cudaEvent_t a, int cls, double bytes, double flops) {
+  if (!c->timing) return;
+  cudaEvent_t b = c->timing_pool[c->timing_next++];
+  cudaEventRecord(b, s);
+  c->timed.push_back({cls, a, b, bytes, flops});
+}
+void timing_flush(liger_ctx* c) {
+  if (c->timed.empty()) return;
+  cudaDeviceSynchronize();
+  for (auto& t : c->timed) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, t.a, t.b);
+    c->tcount[t.cls]++;
+    c->tms[t.cls] += ms;
+    c->tbytes[t.cls] += t.bytes;
+    c->tflops[t.cls] += t.flops;
+  }
+  c->timed.clear();
+  c->timing_next = 0;
+}
+
+// ------------------------------------------------------------------ launching one piece
+int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cudaStream_t st) {
+  const PassOp po = c->pass_ops[pidx];
+  Slot& S = c->slots[bt->slot];
+  const int M = batch_M(bt, pass);
+  const int h = c->h;
+  const float eps = c->cfg.ln_eps;
+  const int li = po.layer;
+  const LayerW* W = li >= 0 ? &c->layers[li] : nullptr;
+  int rc = 0;
+  cudaEvent_t ta = nullptr;
+  switch (po.op) {
+    case OP_EMBED: {
+      const int32_t* ids = pass == 0 ? (bt->dev_tokens ? bt->dev_tokens : S.prompt) : S.cur_tok;
+      rc = embed_launch(ids, c->e_tok, c->e_pos, S.x, M, h, pass == 0 ? bt->s : 0, pass == 0 ? 0 : bt->s + pass - 1,
+                        st);
+      c->st.gpu_launches++;
+      break;
+    }
+    case OP_LN1: {
+      timed_begin(c, st, &ta);
+      if (li == 0)
+        rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
+      else
+        rc = add_layernorm_launch(S.x, S.part, c->layers[li - 1].b_2, S.x, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
+      timed_end(c, st, ta, 2, (double)M * h * 2 * (li == 0 ? 2 : 4), 0);
+      c->st.gpu_launches++;
+      break;
+    }
+    case OP_LN2: {
+      timed_begin(c, st, &ta);
+      rc = add_layernorm_launch(S.x, S.part, W->b_o, S.x, S.y, W->g2, W->be2, M, h, 1, 0, eps, st);
+      timed_end(c, st, ta, 2, (double)M * h * 2 * 4, 0);
+      c->st.gpu_launches++;
+      break;
+    }
+    case OP_QKV:
+    case OP_OUT:
+    case OP_FC1:
+    case OP_FC2: {
+      const int N = gemm_N(c, po.op), K = gemm_K(c, po.op);
+      const int F = op_units(c, po.op);
+      GemmArgs g{};
+      g.M = M; g.N = N; g.K = K;
+      g.n0 = unit_col(N, u0, F);
+      g.n1 = unit_col(N, u1, F);
+      g.workspace = S.gemm_ws; g.ws_bytes = S.gemm_ws_bytes;
+      g.scale = 1.0f;
+      if (po.op == OP_QKV) {
+        g.x = S.y; g.ldx = h; g.w = W->w_qkv; g.ldw = K; g.out = S.qkv; g.ldo = N; g.bias = W->b_qkv;
+        g.scale_cols = c->hl; g.scale = 1.0f / sqrtf((float)c->d);
+      } else if (po.op == OP_OUT) {
+        g.x = S.attn; g.ldx = c->hl; g.w = W->w_o; g.ldw = K; g.out = S.part; g.ldo = h;
+      } else if (po.op == OP_FC1) {
+        g.x = S.y; g.ldx = h; g.w = W->w_1; g.ldw = K; g.out = S.hbuf; g.ldo = N; g.bias = W->b_1;
+        g.act = c->cfg.act;
+      } else {
+        g.x = S.hbuf; g.ldx = c->fl; g.w = W->w_2; g.ldw = K; g.out = S.part; g.ldo = h;
+      }
+      timed_begin(c, st, &ta);
+      rc = gemm_launch(g, st);
+      const double n = g.n1 - g.n0;
+      timed_end(c, st, ta, 0, (n * K + (double)M * K + (double)M * n) * 2, 2.0 * M * n * K);
+      c->st.gpu_launches++;
+      break;
+    }
+    case OP_ATTN: {
+      void* pool = (char*)c->kv + (size_t)li * c->kv_layer_elems * 2;
+      timed_begin(c, st, &ta);
+      if (pass == 0) {
+        rc = attn_prefill_launch(S.qkv, S.attn, pool, S.page_table, c->max_pages, bt->b, bt->s, c->al, c->d, st);
+        timed_end(c, st, ta, 1, (double)M * c->hl * 2 * 6, 2.0 * bt->b * c->al * c->d * (double)bt->s * bt->s);
+      } else {
+        const int pos = bt->s + pass - 1;
+        rc = attn_decode_launch(S.qkv, S.attn, pool, S.page_table, c->max_pages, bt->b, pos, c->al, c->d,
+                                S.attn_ws, S.attn_ws_bytes, st);
+        timed_end(c, st, ta, 1, (double)bt->b * c->hl * 2 * 2 * (pos + 1),
+                  4.0 * bt->b * c->al * c->d * (double)(pos + 1));
+      }
+      c->st.gpu_launches++;
+      break;
+    }
+    case OP_AR1:
+    case OP_AR2: {
+      const int F = op_units(c, po.op);
+      const size_t E = (size_t)M * h;
+      const size_t e0 = E * u0 / F, e1 = E * u1 / F;
+      timed_begin(c, st, &ta);
+      if (e1 > e0) {
+        ncclResult_t r = nccl().AllReduce((char*)S.part + e0 * 2, (char*)S.part + e0 * 2, e1 - e0, ncclBfloat16,
+                                          ncclSum, c->comm, st);
+        if (r != ncclSuccess) return fail(c, LIGER_ENCCL, std::string("ncclAllReduce: ") + nccl().GetErrorString(r));
+      }
+      timed_end(c, st, ta, 3, (double)(e1 - e0) * 2, 0);
+      c->st.comm_kernels++;
+      c->st.gpu_launches++;
+      break;
+    }
+    case OP_HEAD: {
+      const int b = bt->b;
+      const LayerW& Wl = c->layers[c->L - 1];
+      // residual add of the last layer + final LN on the last token of each sequence
+      const int step = pass == 0 ? bt->s : 1, off = pass == 0 ? bt->s - 1 : 0;
+      rc = add_layernorm_launch(S.x, S.part, Wl.b_2, nullptr, S.yhead, c->lnf_g, c->lnf_b, b, h, step, off, eps, st);
+      if (rc) break;
+      GemmArgs g{};
+      g.x = S.yhead; g.ldx = h;
+      g.w = (char*)c->e_tok + (size_t)c->rank * c->Vl * h * 2; g.ldw = h;
+      g.out = S.logits; g.ldo = c->Vl; g.out_f32 = 1;
+      g.M = b; g.N = c->Vl; g.K = h; g.n0 = 0; g.n1 = c->Vl; g.scale = 1.0f;
+      g.workspace = S.gemm_ws; g.ws_bytes = S.gemm_ws_bytes;
+      timed_begin(c, st, &ta);
+      rc = gemm_launch(g, st);
+      timed_end(c, st, ta, 0, ((double)c->Vl * h + (double)b * h) * 2 + (double)b * c->Vl * 4,
+                2.0 * b * c->Vl * h);
+      if (rc) break;
+      rc = argmax_launch(S.logits, c->Vl, b, c->Vl, c->rank * c->Vl, S.vals_all + (size_t)c->rank * b,
+                         S.idx_all + (size_t)c->rank * b, st);
+      if (rc) break;
+      c->st.gpu_launches += 3;
+      if (c->world == 1) {
+        rc = argmax_pick_launch(S.vals_all, S.idx_all, 1, b, S.cur_tok, S.tok_out, bt->n_new, pass, st);
+        c->st.gpu_launches++;
+      }
+      break;
+    }
+    case OP_TOKG: {
+      const int b = bt->b;
+      nccl().GroupStart();
+      nccl().AllGather(S.vals_all + (size_t)c->rank * b, S.vals_all, b, ncclFloat32, c->comm, st);
+      nccl().AllGather(S.idx_all + (size_t)c->rank * b, S.idx_all, b, ncclInt32, c->comm, st);
+      ncclResult_t r = nccl().GroupEnd();
+      if (r != ncclSuccess) return fail(c, LIGER_ENCCL, "ncclAllGather failed");
+      c->st.comm_kernels++;
+      c->st.gpu_launches++;
+      break;
+    }
+    case OP_PICK: {
+      rc = argmax_pick_launch(S.vals_all, S.idx_all, c->world, bt->b, S.cur_tok, S.tok_out, bt->n_new, pass, st);
+      c->st.gpu_launches++;
+      break;
+    }
+  }
+  if (rc < 0) return fail(c, rc, std::string("launch of ") + kOpName[po.op] + " failed");
+  return 0;
+}
+
+// ------------------------------------------------------------------ batch cursor for the planner
+struct BatchCursor : Cursor {
+  liger_ctx* c;
+  Batch* bt;
+  std::vector<Piece>* out;
+  BatchCursor(liger_ctx* c_, Batch* b_, std::vector<Piece>* o) : c(c_), bt(b_), out(o) {}
+  bool empty() const override { return bt->all_launched; }
+  int cur_op() const { return c->pass_ops[bt->idx].op; }
+  int head_type() const override { return op_is_comm(cur_op()) ? KT_COMM : KT_COMPUTE; }
+  int head_left() const override { return op_units(c, cur_op()) - bt->done; }
+  bool head_decomposable() const override { return op_units(c, cur_op()) > 1; }
+  double head_dur(int k) const override {
+    // duration of units [done, done + k): profiled piece of k units
+    return op_dur(c, bt, bt->pass, cur_op(), k);
+  }
+  int next_type() const override {
+    int pass = bt->pass, idx = bt->idx + 1;
+    if (idx >= (int)c->pass_ops.size()) {
+      idx = 0;
+      ++pass;
+    }
+    if (pass >= bt->n_new) return -1;
+    return op_is_comm(c->pass_ops[idx].op) ? KT_COMM : KT_COMPUTE;
+  }
+  int64_t take(int k) override {
+    Piece p{bt, bt->pass, bt->idx, bt->done, bt->done + k};
+    out->push_back(p);
+    bt->done += k;
+    if (bt->done >= op_units(c, cur_op())) {
+      bt->done = 0;
+      if (++bt->idx >= (int)c->pass_ops.size()) {
+        bt->idx = 0;
+        if (++bt->pass >= bt->n_new) bt->all_launched = true;
+      }
+    }
+    return (int64_t)out->size() - 1;
+  }
+};
+
+// ------------------------------------------------------------------ admission / completion
+int admit(liger_ctx* c, Batch* bt) {
+  int slot = -1;
+  for (size_t i = 0; i < c->slots.size(); ++i)
+    if (!c->slots[i].busy) {
+      slot = (int)i;
+      break;
+    }
+  if (slot < 0) return 1;   // no free slot yet
+  const int ppseq = (bt->s + bt->n_new + LIGER_KV_BLOCK - 1) / LIGER_KV_BLOCK;
+  if ((int)c->free_pages.size() < ppseq * bt->b) return 1;
+  Slot& S = c->slots[slot];
+  S.busy = true;
+  bt->slot = slot;
+  for (int i = 0; i < bt->b; ++i)
+    for (int p = 0; p < ppseq; ++p) {
+      const int pg = c->free_pages.back();
+      c->free_pages.pop_back();
+      bt->pages.push_back(pg);
+      S.h_page_table[i * c->max_pages + p] = pg;
+    }
+  // inputs for the first kernels: wait until the previous user of the slot is done
+  cudaStreamWaitEvent(c->s_comp, S.free_ev, 0);
+  cudaMemcpyAsync(S.page_table, S.h_page_table, sizeof(int32_t) * bt->b * c->max_pages, cudaMemcpyHostToDevice,
+                  c->s_comp);
+  if (!bt->dev_tokens) {
+    memcpy(S.h_prompt, bt->host_tokens.data(), sizeof(int32_t) * bt->b * bt->s);
+    cudaMemcpyAsync(S.prompt, S.h_prompt, sizeof(int32_t) * bt->b * bt->s, cudaMemcpyHostToDevice, c->s_comp);
+  }
+  bt->last_stream = 0;
+  bt->last_ev = pool_event(c);
+  cudaEventRecord(bt->last_ev, c->s_comp);
+  bt->has_last_ev = true;
+  return 0;
+}
+
+void CUDART_CB host_finish(void* p) {
+  Batch* bt = static_cast<Batch*>(p);
+  bt->finish_s.store(now_s());
+}
+
+void finalize_batch_launch(liger_ctx* c, Batch* bt, cudaStream_t st) {
+  Slot& S = c->slots[bt->slot];
+  if (bt->results_to_host)
+    cudaMemcpyAsync(S.h_tok_out, S.tok_out, sizeof(int32_t) * bt->b * bt->n_new, cudaMemcpyDeviceToHost, st);
+  cudaEventRecord(bt->final_ev, st);
+  cudaEventRecord(S.free_ev, st);
+  cudaLaunchHostFunc(st, host_finish, bt);
+}
+
+// a finished batch releases its pages and slot (host side)
+void reap(liger_ctx* c) {
+  for (auto& up : c->all_batches) {
+    Batch* bt = up.get();
+    if (!bt || !bt->all_launched || bt->finished) continue;
+    if (cudaEventQuery(bt->final_ev) != cudaSuccess) continue;
+    bt->finished = true;
+    Slot& S = c->slots[bt->slot];
+    if (bt->results_to_host) {
+      bt->tokens.assign(S.h_tok_out, S.h_tok_out + bt->b * bt->n_new);
+      bt->results_copied = true;
+    }
+    for (int pg : bt->pages) c->free_pages.push_back(pg);
+    bt->pages.clear();
+    S.busy = false;
+    if (bt->finish_s.load() == 0) bt->finish_s.store(now_s());
+  }
+}
+
+void update_list(liger_ctx* c) {
+  // completed batches leave the processing list; waiting batches are admitted FIFO.
+  std::vector<Batch*> keep;
+  for (Batch* b : c->processing)
+    if (!b->all_launched) keep.push_back(b);
+  c->processing.swap(keep);
+  const int cap = c->cfg.mode == LIGER_MODE_SERIAL ? 1 : std::max(1, c->cfg.max_inflight);
+  reap(c);
+  while ((int)c->processing.size() < cap && !c->waiting.empty()) {
+    Batch* bt = c->waiting.front().get();
+    if (admit(c, bt)) {
+      reap(c);
+      if (admit(c, bt)) break;
+    }
+    c->processing.push_back(bt);
+    c->all_batches[bt->id] = std::move(c->waiting.front());
+    c->waiting.pop_front();
+  }
+}
+
+// stream index: 0 = compute, 1 = communication
+cudaStream_t stream_of(liger_ctx* c, int idx) { return idx ? c->s_comm : c->s_comp; }
+
+// Launch a run of pieces on stream `si`, honouring each batch's cross-stream data dependency.
+int launch_run(liger_ctx* c, const std::vector<Piece>& pieces, const std::vector<int>& which, int si) {
+  cudaStream_t st = stream_of(c, si);
+  for (size_t j = 0; j < which.size(); ++j) {
+    const Piece& p = pieces[which[j]];
+    Batch* bt = p.bt;
+    if (bt->has_last_ev && bt->last_stream != si) cudaStreamWaitEvent(st, bt->last_ev, 0);
+    if (bt->start_s == 0) bt->start_s = now_s();
+    int rc = launch_piece(c, bt, p.pass, p.idx, p.u0, p.u1, st);
+    if (rc < 0) return rc;
+    c->st.kernels++;
+    const int units = op_units(c, c->pass_ops[p.idx].op);
+    if (p.u1 - p.u0 < units) c->st.split_pieces++;
+    const bool batch_changes = (j + 1 == which.size()) || pieces[which[j + 1]].bt != bt;
+    if (batch_changes) {
+      bt->last_ev = pool_event(c);
+      cudaEventRecord(bt->last_ev, st);
+      bt->last_stream = si;
+      bt->has_last_ev = true;
+    }
+    if (bt->all_launched && p.pass == bt->n_new - 1 && p.idx == (int)c->pass_ops.size() - 1 && p.u1 == units)
+      finalize_batch_launch(c, bt, st);
+  }
+  return 0;
+}
+
+}  // namespace
+
+// ================================================================== C ABI
+extern "C" {
+
+int liger_nccl_unique_id(uint8_t* uid) {
+  if (!uid) return LIGER_EINVAL;
+  if (!nccl().ok) return fail(nullptr, LIGER_ENCCL, "NCCL library not loadable");
+  ncclUniqueId id;
+  if (nccl().GetUniqueId(&id) != ncclSuccess) return fail(nullptr, LIGER_ENCCL, "ncclGetUniqueId failed");
+  memcpy(uid, &id, sizeof(id));
+  return LIGER_OK;
+}
+
+int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_uid, liger_ctx** out) {
+  if (!cfg || !out || world < 1 || rank < 0 || rank >= world) return LIGER_EINVAL;
+  if (int rc = check_device()) return rc;
+  auto cp = std::make_unique<liger_ctx>();
+  liger_ctx* c = cp.get();
+  c->world = world;
+  c->rank = rank;
+  c->cfg = *cfg;
+  c->h = cfg->hidden; c->a = cfg->n_heads; c->f = cfg->ffn; c->V = cfg->vocab; c->L = cfg->n_layers;
+  if (c->a <= 0 || c->h % c->a || c->a % world || c->f % world || c->V % world || c->h % 64)
+    return fail(nullptr, LIGER_EINVAL, "liger_init: shapes not divisible by the TP degree");
+  c->d = c->h / c->a;
+  if (c->d != 64 && c->d != 128) return fail(nullptr, LIGER_EINVAL, "liger_init: head_dim must be 64 or 128");
+  c->hl = c->h / world; c->al = c->a / world; c->fl = c->f / world; c->Vl = c->V / world;
+  c->F = std::max(1, cfg->decomp_factor);
+  c->cf = cfg->contention_factor > 0 ? cfg->contention_factor : 1.0;
+  const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
+  c->ar_atomic_chunks = env ? atoi(env) != 0 : (world > 2);
+  if (world > 1) {
+    if (!nccl().ok) return fail(nullptr, LIGER_ENCCL, "NCCL library not loadable");
+    if (!nccl_uid) return fail(nullptr, LIGER_EINVAL, "liger_init: nccl_uid required for world > 1");
+    ncclUniqueId id;
+    memcpy(&id, nccl_uid, sizeof(id));
+    ncclResult_t r = nccl().CommInitRank(&c->comm, world, id, rank);
+    if (r != ncclSuccess) return fail(nullptr, LIGER_ENCCL, std::string("ncclCommInitRank: ") + nccl().GetErrorString(r));
+  }
+  int lo, hi;
+  cudaDeviceGetStreamPriorityRange(&lo, &hi);
+  CK(cudaStreamCreateWithPriority(&c->s_comp, cudaStreamNonBlocking, lo));
+  CK(cudaStreamCreateWithPriority(&c->s_comm, cudaStreamNonBlocking, hi));
+  CK(cudaEventCreateWithFlags(&c->e1, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&c->e2, cudaEventDisableTiming));
+
+  // weights (this rank's shards, K-major [N_local, K])
+  c->layers.resize(c->L);
+  const size_t h = c->h;
+  for (int l = 0; l < c->L; ++l) {
+    LayerW& W = c->layers[l];
+    W.w_qkv = dalloc(c, 3 * c->hl * h * 2);
+    W.b_qkv = dalloc(c, 3 * c->hl * 2);
+    W.w_o = dalloc(c, h * c->hl * 2);
+    W.b_o = dalloc(c, h * 2);
+    W.w_1 = dalloc(c, (size_t)c->fl * h * 2);
+    W.b_1 = dalloc(c, (size_t)c->fl * 2);
+    W.w_2 = dalloc(c, h * c->fl * 2);
+    W.b_2 = dalloc(c, h * 2);
+    W.g1 = dalloc(c, h * 2); W.be1 = dalloc(c, h * 2); W.g2 = dalloc(c, h * 2); W.be2 = dalloc(c, h * 2);
+    if (!W.w_qkv || !W.w_o || !W.w_1 || !W.w_2 || !W.be2)
+      return fail(nullptr, LIGER_ENOMEM, "liger_init: out of device memory for weights");
+  }
+  c->e_tok = dalloc(c, (size_t)c->V * h * 2);
+  c->e_pos = dalloc(c, (size_t)(cfg->max_pos + 2) * h * 2);
+  c->lnf_g = dalloc(c, h * 2);
+  c->lnf_b = dalloc(c, h * 2);
+  if (!c->e_tok || !c->e_pos || !c->lnf_b) return fail(nullptr, LIGER_ENOMEM, "liger_init: embeddings");
+
+  // slots and paged KV pool
+  const int nslots = (cfg->mode == LIGER_MODE_SERIAL ? 1 : std::max(1, cfg->max_inflight)) + 1;
+  const int B = cfg->max_batch, Smax = cfg->max_seq;
+  const int Mmax = B * Smax;
+  c->max_pages = (Smax + cfg->max_new + LIGER_KV_BLOCK - 1) / LIGER_KV_BLOCK;
+  c->n_pages = nslots * B * c->max_pages;
+  c->kv_layer_elems = (size_t)c->n_pages * 2 * c->al * LIGER_KV_BLOCK * c->d;
+  c->kv = dalloc(c, c->kv_layer_elems * 2 * c->L);
+  if (!c->kv) return fail(nullptr, LIGER_ENOMEM, "liger_init: KV pool");
+  for (int p = c->n_pages - 1; p >= 0; --p) c->free_pages.push_back(p);
+  size_t ws = 0;
+  for (int M : {Mmax, B}) {
+    ws = std::max(ws, gemm_workspace_bytes(M, 3 * c->hl, c->h));
+    ws = std::max(ws, gemm_workspace_bytes(M, c->h, c->hl));
+    ws = std::max(ws, gemm_workspace_bytes(M, c->fl, c->h));
+    ws = std::max(ws, gemm_workspace_bytes(M, c->h, c->fl));
+    ws = std::max(ws, gemm_workspace_bytes(M, c->Vl, c->h));
+  }
+  // the decode GEMMs at every M <= B
+  for (int M = 1; M <= B; ++M) {
+    ws = std::max(ws, gemm_workspace_bytes(M, 3 * c->hl, c->h));
+    ws = std::max(ws, gemm_workspace_bytes(M, c->fl, c->h));
+    ws = std::max(ws, gemm_workspace_bytes(M, c->h, c->fl));
+    ws = std::max(ws, gemm_workspace_bytes(M, c->Vl, c->h));
+  }
+  c->slots.resize(nslots);
+  for (auto& S : c->slots) {
+    S.x = dalloc(c, (size_t)Mmax * h * 2);
+    S.y = dalloc(c, (size_t)Mmax * h * 2);
+    S.qkv = dalloc(c, (size_t)Mmax * 3 * c->hl * 2);
+    S.attn = dalloc(c, (size_t)Mmax * c->hl * 2);
+    S.part = dalloc(c, (size_t)Mmax * h * 2);
+    S.hbuf = dalloc(c, (size_t)Mmax * c->fl * 2);
+    S.yhead = dalloc(c, (size_t)B * h * 2);
+    S.logits = (float*)dalloc(c, (size_t)B * c->Vl * 4);
+    S.vals_all = (float*)dalloc(c, (size_t)world * B * 4);
+    S.idx_all = (int32_t*)dalloc(c, (size_t)world * B * 4);
+    S.cur_tok = (int32_t*)dalloc(c, (size_t)B * 4);
+    S.tok_out = (int32_t*)dalloc(c, (size_t)B * cfg->max_new * 4);
+    S.prompt = (int32_t*)dalloc(c, (size_t)Mmax * 4);
+    S.page_table = (int32_t*)dalloc(c, (size_t)B * c->max_pages * 4);
+    S.gemm_ws_bytes = ws;
+    S.gemm_ws = dalloc(c, ws);
+    S.attn_ws_bytes = attn_decode_workspace_bytes(B, c->al, c->d, Smax + cfg->max_new);
+    S.attn_ws = dalloc(c, S.attn_ws_bytes);
+    if (!S.x || !S.hbuf || !S.gemm_ws || !S.attn_ws || !S.page_table)
+      return fail(nullptr, LIGER_ENOMEM, "liger_init: slot buffers");
+    CK(cudaMemset(S.gemm_ws, 0, GEMM_COUNTER_BYTES));
+    CK(cudaMemset(S.attn_ws, 0, ATTN_COUNTER_BYTES));
+    CK(cudaMallocHost(&S.h_page_table, sizeof(int32_t) * B * c->max_pages));
+    CK(cudaMallocHost(&S.h_prompt, sizeof(int32_t) * Mmax));
+    CK(cudaMallocHost(&S.h_tok_out, sizeof(int32_t) * B * cfg->max_new));
+    CK(cudaEventCreateWithFlags(&S.free_ev, cudaEventDisableTiming));
+    CK(cudaEventRecord(S.free_ev, c->s_comp));
+  }
+  // function assembly template of one pass (§3.2)
+  c->pass_ops.push_back({OP_EMBED, -1});
+  for (int l = 0; l < c->L; ++l) {
+    c->pass_ops.push_back({OP_LN1, l});
+    c->pass_ops.push_back({OP_QKV, l});
+    c->pass_ops.push_back({OP_ATTN, l});
+    c->pass_ops.push_back({OP_OUT, l});
+    if (world > 1) c->pass_ops.push_back({OP_AR1, l});
+    c->pass_ops.push_back({OP_LN2, l});
+    c->pass_ops.push_back({OP_FC1, l});
+    c->pass_ops.push_back({OP_FC2, l});
+    if (world > 1) c->pass_ops.push_back({OP_AR2, l});
+  }
+  c->pass_ops.push_back({OP_HEAD, -1});
+  if (world > 1) {
+    c->pass_ops.push_back({OP_TOKG, -1});
+    c->pass_ops.push_back({OP_PICK, -1});
+  }
+  CK(cudaDeviceSynchronize());
+  *out = cp.release();
+  return LIGER_OK;
+}
+
+int liger_load_layer(liger_ctx* c, int l, uint64_t seed) {
+  if (!c || l < 0 || l >= c->L) return LIGER_EINVAL;
+  const int r = c->rank, t = c->world;
+  const int64_t h = c->h, hl = c->hl, fl = c->fl, f = c->f;
+  LayerW& W = c->layers[l];
+  cudaStream_t st = c->s_comp;
+  const uint64_t tid = 16ull * l;
+  // W_qkv logical [h, 3h]; local row j of block s in {q,k,v} = logical column s*h + r*hl + j'
+  for (int s = 0; s < 3; ++s) {
+    CKR(c0_fill_launch((char*)W.w_qkv + s * hl * h * 2, (int)hl, (int)h, h, seed, tid + 0, s * h + r * hl, 0, 1,
+                       3 * h, weight_exp((int)h), 0, st));
+    CKR(c0_fill_launch((char*)W.b_qkv + s * hl * 2, 1, (int)hl, hl, seed, tid + 1, 0, s * h + r * hl, 0, 1, BIAS_EXP,
+                       0, st));
+  }
+  // W_o logical [h_in, h_out]; local [h_out, hl_in]: (n, k) -> ((r*hl + k) * h + n)
+  CKR(c0_fill_launch(W.w_o, (int)h, (int)hl, hl, seed, tid + 2, 0, r * hl, 1, h, weight_exp((int)h), 0, st));
+  CKR(c0_fill_launch(W.b_o, 1, (int)h, h, seed, tid + 3, 0, 0, 0, 1, BIAS_EXP, 0, st));
+  // W_1 logical [h, f]; local [fl, h]: (n, k) -> (k * f + r*fl + n)
+  CKR(c0_fill_launch(W.w_1, (int)fl, (int)h, h, seed, tid + 4, r * fl, 0, 1, f, weight_exp((int)h), 0, st));
+  CKR(c0_fill_launch(W.b_1, 1, (int)fl, fl, seed, tid + 5, 0, r * fl, 0, 1, BIAS_EXP, 0, st));
+  // W_2 logical [f, h]; local [h, fl]: (n, k) -> ((r*fl + k) * h + n)
+  CKR(c0_fill_launch(W.w_2, (int)h, (int)fl, fl, seed, tid + 6, 0, r * fl, 1, h, weight_exp((int)f), 0, st));
+  CKR(c0_fill_launch(W.b_2, 1, (int)h, h, seed, tid + 7, 0, 0, 0, 1, BIAS_EXP, 0, st));
+  CKR(c0_fill_launch(W.g1, 1, (int)h, h, seed, tid + 8, 0, 0, 0, 1, 0, 1, st));
+  CKR(c0_fill_launch(W.be1, 1, (int)h, h, seed, tid + 9, 0, 0, 0, 1, 0, 2, st));
+  CKR(c0_fill_launch(W.g2, 1, (int)h, h, seed, tid + 10, 0, 0, 0, 1, 0, 1, st));
+  CKR(c0_fill_launch(W.be2, 1, (int)h, h, seed, tid + 11, 0, 0, 0, 1, 0, 2, st));
+  (void)t;
+  CK(cudaStreamSynchronize(st));
+  return LIGER_OK;
+}
+
+int liger_load_embed(liger_ctx* c, uint64_t seed) {
+  if (!c) return LIGER_EINVAL;
+  const int64_t h = c->h;
+  cudaStream_t st = c->s_comp;
+  CKR(c0_fill_launch(c->e_tok, c->V, (int)h, h, seed, GID_ETOK, 0, 0, h, 1, EMB_EXP, 0, st));
+  CKR(c0_fill_launch(c->e_pos, c->cfg.max_pos + 2, (int)h, h, seed, GID_EPOS, 0, 0, h, 1, EMB_EXP, 0, st));
+  CKR(c0_fill_launch(c->lnf_g, 1, (int)h, h, seed, GID_LNFG, 0, 0, 0, 1, 0, 1, st));
+  CKR(c0_fill_launch(c->lnf_b, 1, (int)h, h, seed, GID_LNFB, 0, 0, 0, 1, 0, 2, st));
+  CK(cudaStreamSynchronize(st));
+  return LIGER_OK;
+}
+
+int64_t liger_submit(liger_ctx* c, int batch, int seq_len, const int32_t* tokens, int tokens_on_device, int n_new,
+                     double arrival_s) {
+  if (!c || batch < 1 || batch > c->cfg.max_batch || seq_len < 1 || seq_len > c->cfg.max_seq || n_new < 1 ||
+      n_new > c->cfg.max_new || !tokens || seq_len + n_new + 1 > c->cfg.max_pos + 2)
+    return fail(c, LIGER_EINVAL, "liger_submit: batch/seq_len/n_new out of the configured range");
+  auto bt = std::make_unique<Batch>();
+  bt->id = c->next_id++;
+  bt->b = batch;
+  bt->s = seq_len;
+  bt->n_new = n_new;
+  bt->arrival_s = arrival_s;
+  bt->submit_s = now_s();
+  bt->eng = nullptr;
+  if (tokens_on_device) {
+    bt->dev_tokens = tokens;
+    bt->results_to_host = false;
+  } else {
+    bt->host_tokens.assign(tokens, tokens + (size_t)batch * seq_len);
+  }
+  cudaEventCreateWithFlags(&bt->final_ev, cudaEventDisableTiming);
+  const int64_t id = bt->id;
+  c->all_batches.emplace_back(nullptr);
+  c->waiting.push_back(std::move(bt));
+  return id;
+}
+
+int liger_step(liger_ctx* c) {
+  if (!c) return LIGER_EINVAL;
+  const double t0 = now_s();
+  // hybrid synchronization: wait for E1 of the running round (CPU-GPU sync)
+  if (c->have_round) {
+    const double w0 = now_s();
+    while (cudaEventQuery(c->e1) == cudaErrorNotReady) {
+    }
+    c->st.wait_us += (now_s() - w0) * 1e6;
+  }
+  update_list(c);
+  if (c->processing.empty()) {
+    c->st.host_us += (now_s() - t0) * 1e6;
+    return c->waiting.empty() ? LIGER_IDLE : 0;
+  }
+  std::vector<Piece> pieces;
+  int n = 0;
+  if (c->cfg.mode == LIGER_MODE_SERIAL) {
+    // Intra-Op baseline: the single batch's whole remaining list, in order,
+    // on one stream (computation then all-reduce, serially).
+    Batch* bt = c->processing[0];
+    BatchCursor cur(c, bt, &pieces);
+    while (!cur.empty()) cur.take(cur.head_left());
+    std::vector<int> all(pieces.size());
+    for (size_t i = 0; i < pieces.size(); ++i) all[i] = (int)i;
+    CKR(launch_run(c, pieces, all, 0));
+    c->st.rounds++;
+    c->have_round = false;
+    n = (int)pieces.size();
+  } else {
+    std::vector<std::unique_ptr<BatchCursor>> curs;
+    std::vector<Cursor*> pl;
+    for (Batch* bt : c->processing) {
+      curs.emplace_back(new BatchCursor(c, bt, &pieces));
+      pl.push_back(curs.back().get());
+    }
+    RoundPlan plan;
+    plan_round(pl, c->cf, &plan);
+    std::vector<int> w0, w1;
+    for (auto& p : plan.sub0) w0.push_back((int)p.token);
+    for (auto& p : plan.sub1) w1.push_back((int)p.token);
+    const int s0 = plan.type == KT_COMM ? 1 : 0;   // SubSet0 on the stream of its type
+    const int s1 = 1 - s0;
+    // gate both subsets on E2 of the previous round (inter-stream sync)
+    if (c->have_round) {
+      cudaStreamWaitEvent(c->s_comp, c->e2, 0);
+      cudaStreamWaitEvent(c->s_comm, c->e2, 0);
+    }
+    // communication subset first
+    auto launch_sub0 = [&]() -> int {
+      if (w0.empty()) return 0;
+      std::vector<int> head(w0.begin(), w0.end() - 1), last(1, w0.back());
+      int rc = launch_run(c, pieces, head, s0);
+      if (rc < 0) return rc;
+      cudaEventRecord(c->e1, stream_of(c, s0));   // E1: before the switch kernel
+      rc = launch_run(c, pieces, last, s0);
+      if (rc < 0) return rc;
+      cudaEventRecord(c->e2, stream_of(c, s0));   // E2: after it
+      return 0;
+    };
+    if (s1 == 1) {
+      CKR(launch_run(c, pieces, w1, s1));
+      CKR(launch_sub0());
+    } else {
+      CKR(launch_sub0());
+      CKR(launch_run(c, pieces, w1, s1));
+    }
+    c->have_round = !w0.empty();
+    c->st.rounds++;
+    if (!w1.empty()) c->st.overlapped_rounds++;
+    n = (int)pieces.size();
+  }
+  c->st.host_us += (now_s() - t0) * 1e6;
+  return n;
+}
+
+int liger_drain(liger_ctx* c) {
+  if (!c) return LIGER_EINVAL;
+  for (;;) {
+    int rc = liger_step(c);
+    if (rc < 0) return rc;
+    if (rc == LIGER_IDLE) break;
+  }
+  CK(cudaStreamSynchronize(c->s_comp));
+  CK(cudaStreamSynchronize(c->s_comm));
+  reap(c);
+  return LIGER_OK;
+}
+
+int liger_poll(liger_ctx* c, int64_t id, liger_result* out, int32_t* tokens_out) {
+  if (!c || id < 0 || id >= (int64_t)c->all_batches.size()) return LIGER_EINVAL;
+  Batch* bt = c->all_batches[id].get();
+  if (!bt) {   // still in the waiting queue
+    for (auto& w : c->waiting)
+      if (w->id == id) bt = w.get();
+    if (!bt) return LIGER_EINVAL;
+  }
+  if (!bt->finished) reap(c);
+  if (out) {
+    out->id = bt->id;
+    out->batch = bt->b;
+    out->seq_len = bt->s;
+    out->n_new = bt->n_new;
+    out->done = bt->finished ? 1 : 0;
+    out->arrival_s = bt->arrival_s;
+    out->submit_s = bt->submit_s;
+    out->start_s = bt->start_s;
+    out->finish_s = bt->finish_s.load();
+  }
+  if (!bt->finished) return LIGER_PENDING;
+  if (tokens_out) {
+    if (!bt->results_copied) return fail(c, LIGER_ESTATE, "liger_poll: results of this batch stay on the device");
+    memcpy(tokens_out, bt->tokens.data(), sizeof(int32_t) * bt->tokens.size());
+  }
+  return LIGER_OK;
+}
+
+int liger_result_tokens_device(liger_ctx* c, int64_t id, const int32_t** dev_tokens) {
+  if (!c || id < 0 || id >= (int64_t)c->all_batches.size() || !dev_tokens) return LIGER_EINVAL;
+  Batch* bt = c->all_batches[id].get();
+  if (!bt || bt->slot < 0) return LIGER_PENDING;
+  *dev_tokens = c->slots[bt->slot].tok_out;
+  return LIGER_OK;
+}
+
+int liger_stats(liger_ctx* c, liger_stats_t* out) {
+  if (!c || !out) return LIGER_EINVAL;
+  *out = c->st;
+  return LIGER_OK;
+}
+
+int liger_reset_stats(liger_ctx* c) {
+  if (!c) return LIGER_EINVAL;
+  c->st = liger_stats_t{};
+  return LIGER_OK;
+}
+
+int liger_set_kernel_timing(liger_ctx* c, int on) {
+  if (!c) return LIGER_EINVAL;
+  timing_flush(c);
+  c->timing = on != 0;
+  for (int i = 0; i < 4; ++i) c->tcount[i] = 0, c->tms[i] = c->tbytes[i] = c->tflops[i] = 0;
+  return LIGER_OK;
+}
+
+int liger_kernel_timing(liger_ctx* c, int64_t* count, double* ms, double* bytes, double* flops) {
+  if (!c) return LIGER_EINVAL;
+  timing_flush(c);
+  for (int i = 0; i < 4; ++i) {
+    if (count) count[i] = c->tcount[i];
+    if (ms) ms[i] = c->tms[i];
+    if (bytes) bytes[i] = c->tbytes[i];
+    if (flops) flops[i] = c->tflops[i];
+  }
+  return LIGER_OK;
+}
+
+int liger_set_duration(liger_ctx* c, int op, int m_tokens, int k_of_F, double us) {
+  if (!c || op < 0 || op >= OP_COUNT || m_tokens <= 0 || k_of_F < 0 || k_of_F > c->F) return LIGER_EINVAL;
+  DurTable& T = c->dur;
+  auto it = std::lower_bound(T.mgrid.begin(), T.mgrid.end(), m_tokens);
+  size_t mi = it - T.mgrid.begin();
+  if (it == T.mgrid.end() || *it != m_tokens) {
+    T.mgrid.insert(it, m_tokens);
+    for (int o = 0; o < OP_COUNT; ++o)
+      if (!T.t[o].empty()) T.t[o].insert(T.t[o].begin() + mi, std::vector<double>(c->F + 1, 0.0));
+  }
+  if (T.t[op].empty()) T.t[op].assign(T.mgrid.size(), std::vector<double>(c->F + 1, 0.0));
+  T.t[op][mi][k_of_F] = us * 1e-6;
+  T.have = true;
+  return LIGER_OK;
+}
+
+// Offline profiling: no-load durations of every kernel
+// class over a token grid and for every k/F piece, on slot 0's buffers.
+int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
+  if (!c || !m_list || n_m <= 0) return LIGER_EINVAL;
+  if (!c->processing.empty() || !c->waiting.empty()) return fail(c, LIGER_ESTATE, "liger_profile: batches in flight");
+  CK(cudaDeviceSynchronize());
+  Slot& S = c->slots[0];
+  cudaStream_t st = c->s_comp;
+  cudaEvent_t a, b;
+  CK(cudaEventCreate(&a));
+  CK(cudaEventCreate(&b));
+  const int Mmax = c->cfg.max_batch * c->cfg.max_seq;
+  const bool saved_timing = c->timing;
+  c->timing = false;
+  auto time_it = [&](auto&& fn) -> double {
+    for (int i = 0; i < 2; ++i) fn();
+    float best[5];
+    for (int r = 0; r < 5; ++r) {
+      cudaEventRecord(a, st);
+      fn();
+      cudaEventRecord(b, st);
+      cudaEventSynchronize(b);
+      cudaEventElapsedTime(&best[r], a, b);
+    }
+    std::sort(best, best + 5);
+    return best[2] * 1e-3;
+  };
+  Batch fake;
+  fake.slot = 0;
+  fake.n_new = 1;
+  for (int mi = 0; mi < n_m; ++mi) {
+    const int M = std::min<int>(m_list[mi], Mmax);
+    fake.b = 1;          // GEMM shapes depend on the token count M = b * s only
+    fake.s = M;
+    const int F = std::max(1, c->F);
+    for (int op : {OP_QKV, OP_OUT, OP_FC1, OP_FC2}) {
+      int pidx = 0;
+      while (c->pass_ops[pidx].op != op) ++pidx;
+      const int units = op_units(c, op);
+      for (int k = 1; k <= units; ++k) {
+        const int kk = units > 1 ? k : F;
+        const double t = time_it([&] { launch_piece(c, &fake, 0, pidx, 0, k, st); });
+        liger_set_duration(c, op, M, kk, t * 1e6);
+      }
+    }
+    // memory-bound ops
+    const double tln = time_it([&] {
+      add_layernorm_launch(S.x, S.part, c->layers[0].b_o, S.x, S.y, c->layers[0].g2, c->layers[0].be2, M, c->h, 1,
+                           0, c->cfg.ln_eps, st);
+    });
+    liger_set_duration(c, OP_LN1, M, F, tln * 1e6);
+    liger_set_duration(c, OP_LN2, M, F, tln * 1e6);
+    liger_set_duration(c, OP_EMBED, M, F, tln * 1e6);
+    if (c->world > 1) {
+      const size_t E = (size_t)M * c->h;
+      for (int k = 1; k <= op_units(c, OP_AR1); ++k) {
+        const int kk = op_units(c, OP_AR1) > 1 ? k : F;
+        const double t = time_it([&] {
+          nccl().AllReduce(S.part, S.part, E * k / op_units(c, OP_AR1), ncclBfloat16, ncclSum, c->comm, st);
+        });
+        liger_set_duration(c, OP_AR1, M, kk, t * 1e6);
+        liger_set_duration(c, OP_AR2, M, kk, t * 1e6);
+      }
+    }
+  }
+  // LM head at batch sizes
+  {
+    int pidx = 0;
+    while (c->pass_ops[pidx].op != OP_HEAD) ++pidx;
+    for (int bb : {1, c->cfg.max_batch}) {
+      fake.b = bb;
+      fake.s = 1;
+      const double t = time_it([&] { launch_piece(c, &fake, 1, pidx, 0, 1, st); });
+      liger_set_duration(c, OP_HEAD, bb, std::max(1, c->F), t * 1e6);
+    }
+  }
+  // attention: calibrate the analytical model at one prefill and one decode point
+  {
+    int pidx = 0;
+    while (c->pass_ops[pidx].op != OP_ATTN) ++pidx;
+    fake.b = 1;
+    fake.s = std::min(512, c->cfg.max_seq);
+    fake.pages.clear();
+    for (int p = 0; p < c->max_pages; ++p) S.h_page_table[p] = p;   // pages 0.. (no batch in flight)
+    cudaMemcpyAsync(S.page_table, S.h_page_table, sizeof(int32_t) * c->max_pages, cudaMemcpyHostToDevice, st);
+    const double tp = time_it([&] { launch_piece(c, &fake, 0, pidx, 0, 1, st); });
+    c->attn_scale[0] = tp / model_dur(c, OP_ATTN, fake.s, 1, fake.s, fake.s);
+    if (c->cfg.max_new > 1) {
+      fake.n_new = c->cfg.max_new;
+      const int pass = std::min(c->cfg.max_new - 1, 8);
+      const double td = time_it([&] { launch_piece(c, &fake, pass, pidx, 0, 1, st); });
+      c->attn_scale[1] = td / model_dur(c, OP_ATTN, 1, 1, fake.s + pass, 0);
+    }
+  }
+  c->timing = saved_timing;
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  // ranks must plan identically (NCCL ordering): take the max of every entry over ranks
+  if (c->world > 1) {
+    std::vector<float> flat;
+    for (int o = 0; o < OP_COUNT; ++o)
+      for (auto& row : c->dur.t[o])
+        for (double v : row) flat.push_back((float)v);
+    flat.push_back((float)c->attn_scale[0]);
+    flat.push_back((float)c->attn_scale[1]);
+    float* dv = nullptr;
+    CK(cudaMalloc(&dv, flat.size() * 4));
+    CK(cudaMemcpy(dv, flat.data(), flat.size() * 4, cudaMemcpyHostToDevice));
+    nccl().AllReduce(dv, dv, flat.size(), ncclFloat32, ncclMax, c->comm, st);
+    CK(cudaMemcpyAsync(flat.data(), dv, flat.size() * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    cudaFree(dv);
+    size_t i = 0;
+    for (int o = 0; o < OP_COUNT; ++o)
+      for (auto& row : c->dur.t[o])
+        for (double& v : row) v = flat[i++];
+    c->attn_scale[0] = flat[i++];
+    c->attn_scale[1] = flat[i++];
+  }
+  CK(cudaDeviceSynchronize());
+  return LIGER_OK;
+}
+
+const char* liger_last_error(const liger_ctx* c) { return c ? c->err.c_str() : global_error(); }
+
+int liger_finalize(liger_ctx* c) {
+  if (!c) return LIGER_EINVAL;
+  cudaDeviceSynchronize();
+  if (c->comm) nccl().CommDestroy(c->comm);
+  for (void* p : c->allocs) cudaFree(p);
+  for (auto& S : c->slots) {
+    cudaFreeHost(S.h_page_table);
+    cudaFreeHost(S.h_prompt);
+    cudaFreeHost(S.h_tok_out);
+    cudaEventDestroy(S.free_ev);
+  }
+  for (auto e : c->ev_pool) cudaEventDestroy(e);
+  for (auto e : c->timing_pool) cudaEventDestroy(e);
+  for (auto& b : c->all_batches)
+    if (b) cudaEventDestroy(b->final_ev);
+  for (auto& b : c->waiting) cudaEventDestroy(b->final_ev);
+  cudaEventDestroy(c->e1);
+  cudaEventDestroy(c->e2);
+  cudaStreamDestroy(c->s_comp);
+  cudaStreamDestroy(c->s_comm);
+  gemm_forget_pointer_range(nullptr, ~size_t(0));
+  delete c;
+  return LIGER_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,362 @@
+// tcgen05 / TMEM / TMA GEMM for the TP decoder-layer projections (sm_100a).
+//
+// Computes, for the output-column slice [n0, n1) (runtime kernel decomposition,
+// PAPER.md §3.6, "vertical" split of Fig. 9):
+//     out[m, n] = epi( sum_k X[m, k] * W[n, k] )          m < M, n0 <= n < n1
+// X: activations bf16 row-major [M, K] (row stride ldx); W: weights bf16
+// row-major [N, K] (nn.Linear layout, i.e. K-major); fp32 accumulation in TMEM.
+// epi: + bias[n], * scale for n < scale_cols (q scaling), ReLU / tanh-GELU,
+// then bf16 (or fp32) store.
+//
+// Orientation ("swap-AB"): the MMA M dimension (128 TMEM lanes) runs over the
+// weight rows n, the MMA N dimension over tokens m (bn = 16..256).  Decode
+// (M = batch <= 32) therefore costs one 128 x 16 MMA per K step and the kernel
+// streams W from HBM; prefill uses 128 x 256 tiles.
+//
+// Bit-exactness of decomposition (SURVEY AMB-9): every per-element quantity --
+// the token tiling bn, the split-K chunk kc and the K order, the fixed z-order
+// of the split-K reduction -- is a function of (M, K) only, never of N or of
+// the slice, so a slice computes exactly the bits of the full GEMM.
+//
+// Warp roles (192 threads): warp 0 = TMA producer, warp 1 = TMEM allocator +
+// single-thread MMA issuer, warps 2..5 = epilogue (TMEM -> registers -> HBM).
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <mutex>
+#include <unordered_map>
+#include <vector>
+
+#include "common.cuh"
+#include "kernels.h"
+
+namespace liger {
+
+constexpr int BM = 128;           // weight rows per tile (MMA M)
+constexpr int BK = 64;            // K per stage (one 128-byte swizzle atom)
+constexpr int A_BYTES = BM * BK * 2;
+constexpr int GEMM_THREADS = 192;
+constexpr int MAX_SMEM = 227 * 1024;
+
+struct GemmParams {
+  int M, N, K;
+  int n0, n1;
+  int kc, splits;
+  int bn;
+  int stages;
+  const __nv_bfloat16* bias;
+  int act;
+  int scale_cols;
+  float scale;
+  void* out;
+  int64_t ldo;
+  int out_f32;
+  float* ws;
+  int* counters;
+};
+
+__device__ __forceinline__ float epi_apply(const GemmParams& p, float v, int n, float bias_v) {
+  v += bias_v;
+  if (n < p.scale_cols) v *= p.scale;
+  if (p.act == LIGER_ACT_RELU) v = fmaxf(v, 0.0f);
+  else if (p.act == LIGER_ACT_GELU_TANH) v = gelu_tanh_f(v);
+  return v;
+}
+
+__device__ __forceinline__ void epi_store(const GemmParams& p, int m, int n, float v) {
+  if (p.out_f32)
+    reinterpret_cast<float*>(p.out)[(int64_t)m * p.ldo + n] = v;
+  else
+    reinterpret_cast<__nv_bfloat16*>(p.out)[(int64_t)m * p.ldo + n] = __float2bfloat16_rn(v);
+}
+
+__global__ void __launch_bounds__(GEMM_THREADS, 1)
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                   const GemmParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int S = p.stages;
+  const int B_BYTES = p.bn * BK * 2;
+  uint8_t* smA = smem;
+  uint8_t* smB = smem + (size_t)S * A_BYTES;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smB + (size_t)S * B_BYTES);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + S;
+  uint64_t* tmem_full = bars + 2 * S;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 1);
+  int* last_flag = reinterpret_cast<int*>(tmem_slot + 1);
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const int n_base = p.n0 + blockIdx.x * BM;
+  const int m_base = blockIdx.y * p.bn;
+  const int z = blockIdx.z;
+  const int k0 = z * p.kc;
+  const int k1 = min(p.K, k0 + p.kc);
+  const int nkb = (k1 - k0 + BK - 1) / BK;
+  const uint32_t tmem_cols = p.bn <= 32 ? 32 : (p.bn <= 64 ? 64 : (p.bn <= 128 ? 128 : 256));
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+    }
+    mbar_init(tmem_full, 1);
+    fence_barrier_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+  }
+  if (warp == 1) tmem_alloc(tmem_slot, tmem_cols);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      const uint64_t pol_w = policy_evict_first();   // weights: streamed once
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int s = kb % S;
+        const uint32_t ph = (kb / S) & 1;
+        mbar_wait(&empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&full[s], A_BYTES + B_BYTES);
+        const int kk = k0 + kb * BK;
+        tma_load_2d_hint(smA + (size_t)s * A_BYTES, &tmA, &full[s], kk, n_base, pol_w);
+        tma_load_2d(smB + (size_t)s * B_BYTES, &tmB, &full[s], kk, m_base);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // kind::f16 instruction descriptor: D=f32, A=B=bf16, both K-major, N=bn, M=128.
+      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(p.bn >> 3) << 17) |
+                             ((uint32_t)(BM >> 4) << 24);
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int s = kb % S;
+        const uint32_t ph = (kb / S) & 1;
+        mbar_wait(&full[s], ph);
+        tc_fence_after();
+        const uint64_t adesc = umma_desc_sw128(smem_u32(smA + (size_t)s * A_BYTES));
+        const uint64_t bdesc = umma_desc_sw128(smem_u32(smB + (size_t)s * B_BYTES));
+#pragma unroll
+        for (int k = 0; k < BK / 16; ++k)
+          umma_bf16(tmem_base, adesc + 2 * k, bdesc + 2 * k, idesc, (kb | k) != 0);
+        umma_commit(&empty[s]);
+      }
+      umma_commit(tmem_full);
+    }
+  } else {
+    // ---------------- epilogue: warps 2..5 own TMEM lane quarters (warp % 4)
+    const int q = warp & 3;
+    const int row = q * 32 + lane;
+    const int n = n_base + row;
+    const bool nval = (n < p.n1) && (n < p.N);
+    const float bias_v = (p.bias != nullptr && nval) ? __bfloat162float(p.bias[n]) : 0.0f;
+    const int slice_w = p.n1 - p.n0;
+    mbar_wait(tmem_full, 0);
+    tc_fence_after();
+    for (int c0 = 0; c0 < p.bn; c0 += 16) {
+      uint32_t r[16];
+      tmem_ld_32x32b_x16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)c0, r);
+      tmem_ld_wait();
+      if (nval) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          const int m = m_base + c0 + j;
+          if (m < p.M) {
+            const float v = __uint_as_float(r[j]);
+            if (p.splits == 1)
+              epi_store(p, m, n, epi_apply(p, v, n, bias_v));
+            else
+              p.ws[((int64_t)z * p.M + m) * slice_w + (n - p.n0)] = v;
+          }
+        }
+      }
+    }
+    if (p.splits > 1) {
+      // Deterministic split-K: the last CTA of this tile sums the partials in
+      // z order 0..splits-1 (independent of which CTA finishes last).
+      __threadfence();
+      named_bar_sync(1, 128);
+      const int tile_id = blockIdx.y * gridDim.x + blockIdx.x;
+      if (threadIdx.x == 64) {
+        const int prev = atomicAdd(&p.counters[tile_id], 1);
+        *last_flag = (prev == p.splits - 1);
+      }
+      named_bar_sync(1, 128);
+      if (*last_flag) {
+        __threadfence();
+        if (nval) {
+          const int mcount = min(p.bn, p.M - m_base);
+          for (int c0 = 0; c0 < mcount; c0 += 16) {
+            float acc[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) acc[j] = 0.0f;
+            for (int zz = 0; zz < p.splits; ++zz) {
+              const float* src = p.ws + ((int64_t)zz * p.M + m_base + c0) * slice_w + (n - p.n0);
+              float v[16];
+#pragma unroll
+              for (int j = 0; j < 16; ++j) v[j] = (c0 + j < mcount) ? __ldcg(src + (int64_t)j * slice_w) : 0.0f;
+#pragma unroll
+              for (int j = 0; j < 16; ++j) acc[j] += v[j];
+            }
+#pragma unroll
+            for (int j = 0; j < 16; ++j)
+              if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, acc[j], n, bias_v));
+          }
+        }
+        if (threadIdx.x == 64) p.counters[tile_id] = 0;
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tmem_base, tmem_cols);
+  }
+}
+
+// ------------------------------------------------------------------ host side
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static PFN_encodeTiled get_encode() {
+  static PFN_encodeTiled fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_encodeTiled>(f);
+  });
+  return fn;
+}
+
+struct MapKey {
+  const void* ptr;
+  int64_t rows, cols, ld;
+  int box_rows;
+  bool operator==(const MapKey& o) const {
+    return ptr == o.ptr && rows == o.rows && cols == o.cols && ld == o.ld && box_rows == o.box_rows;
+  }
+};
+struct MapKeyHash {
+  size_t operator()(const MapKey& k) const {
+    size_t h = std::hash<const void*>()(k.ptr);
+    h ^= std::hash<int64_t>()(k.rows * 1315423911ll + k.cols * 2654435761ll + k.ld) + 0x9e3779b9 + (h << 6);
+    return h ^ (size_t)k.box_rows;
+  }
+};
+
+static std::mutex g_map_mu;
+static std::unordered_map<MapKey, CUtensorMap, MapKeyHash> g_maps;
+
+// 2-D bf16 tensor [rows, cols] with row stride ld (elements); box = [64, box_rows], SWIZZLE_128B.
+static int make_map(CUtensorMap* out, const void* ptr, int64_t rows, int64_t cols, int64_t ld, int box_rows) {
+  MapKey key{ptr, rows, cols, ld, box_rows};
+  {
+    std::lock_guard<std::mutex> g(g_map_mu);
+    auto it = g_maps.find(key);
+    if (it != g_maps.end()) {
+      *out = it->second;
+      return 0;
+    }
+  }
+  PFN_encodeTiled enc = get_encode();
+  if (!enc) return LIGER_ECUDA;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(ld * 2)};
+  cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)box_rows};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return LIGER_ECUDA;
+  std::lock_guard<std::mutex> g(g_map_mu);
+  if (g_maps.size() > 65536) g_maps.clear();
+  g_maps.emplace(key, *out);
+  return 0;
+}
+
+void gemm_forget_pointer_range(const void* base, size_t bytes) {
+  std::lock_guard<std::mutex> g(g_map_mu);
+  for (auto it = g_maps.begin(); it != g_maps.end();) {
+    const char* p = static_cast<const char*>(it->first.ptr);
+    if (p >= static_cast<const char*>(base) && p < static_cast<const char*>(base) + bytes)
+      it = g_maps.erase(it);
+    else
+      ++it;
+  }
+}
+
+// Tiling policy: a function of (M, K) only (bit-exact decomposition).
+GemmPlan gemm_plan(int M, int K) {
+  GemmPlan pl{};
+  const int mt = (M + 255) / 256;
+  int bn = (M + mt - 1) / mt;
+  bn = (bn + 15) / 16 * 16;
+  if (bn < 16) bn = 16;
+  pl.bn = bn;
+  pl.m_tiles = mt;
+  int kc;
+  if (M <= 64) kc = 1024;
+  else if (M <= 512) kc = 2048;
+  else kc = K;
+  kc = (kc + BK - 1) / BK * BK;
+  if (kc >= K) kc = (K + BK - 1) / BK * BK;
+  pl.kc = kc;
+  pl.splits = (K + kc - 1) / kc;
+  const int stage_bytes = A_BYTES + bn * BK * 2;
+  int st = (MAX_SMEM - 1024 - 256) / stage_bytes;
+  if (st > 10) st = 10;
+  pl.stages = st;
+  pl.smem = 1024 + st * stage_bytes + 256;
+  return pl;
+}
+
+size_t gemm_workspace_bytes(int M, int N, int K) {
+  GemmPlan pl = gemm_plan(M, K);
+  if (pl.splits <= 1) return GEMM_COUNTER_BYTES;
+  return GEMM_COUNTER_BYTES + (size_t)pl.splits * M * N * sizeof(float);
+}
+
+int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
+  if (a.M <= 0 || a.n1 <= a.n0) return 0;
+  if (a.K <= 0 || a.K % 8 || a.ldx % 8 || a.ldw % 8 || a.n0 < 0 || a.n1 > a.N) return LIGER_EINVAL;
+  GemmPlan pl = gemm_plan(a.M, a.K);
+  const int ntiles = (a.n1 - a.n0 + BM - 1) / BM;
+  if (pl.splits > 1) {
+    if (!a.workspace) return LIGER_EINVAL;
+    const size_t need = GEMM_COUNTER_BYTES + (size_t)pl.splits * a.M * (a.n1 - a.n0) * sizeof(float);
+    if (a.ws_bytes < need || ntiles * pl.m_tiles > GEMM_COUNTER_BYTES / 4) return LIGER_EINVAL;
+  }
+  CUtensorMap tA, tB;
+  int rc = make_map(&tA, a.w, a.N, a.K, a.ldw, BM);
+  if (rc) return rc;
+  rc = make_map(&tB, a.x, a.M, a.K, a.ldx, pl.bn);
+  if (rc) return rc;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
+    attr_set = true;
+  }
+  GemmParams p;
+  p.M = a.M; p.N = a.N; p.K = a.K; p.n0 = a.n0; p.n1 = a.n1;
+  p.kc = pl.kc; p.splits = pl.splits; p.bn = pl.bn; p.stages = pl.stages;
+  p.bias = reinterpret_cast<const __nv_bfloat16*>(a.bias);
+  p.act = a.act; p.scale_cols = a.scale_cols; p.scale = a.scale;
+  p.out = a.out; p.ldo = a.ldo; p.out_f32 = a.out_f32;
+  p.counters = reinterpret_cast<int*>(a.workspace);
+  p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
+  dim3 grid(ntiles, pl.m_tiles, pl.splits);
+  gemm_tc_kernel<<<grid, GEMM_THREADS, pl.smem, stream>>>(tA, tB, p);
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+}  // namespace liger

@@ -1,0 +1,280 @@
+// Memory-bound kernels of the hot path: fused residual add + LayerNorm (a2/a7/a11),
+// embedding (a1), row argmax for greedy decoding (a12), the device-side C0
+// weight generator, and small helpers.  All vectorised 16-byte accesses.
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+#include "common.cuh"
+#include "kernels.h"
+
+namespace liger {
+
+struct __align__(16) bf16x8 {
+  __nv_bfloat162 h[4];
+};
+
+__device__ __forceinline__ void unpack8(const bf16x8& v, float* f) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    float2 t = __bfloat1622float2(v.h[i]);
+    f[2 * i] = t.x;
+    f[2 * i + 1] = t.y;
+  }
+}
+__device__ __forceinline__ bf16x8 pack8(const float* f) {
+  bf16x8 v;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) v.h[i] = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
+  return v;
+}
+
+template <int NT>
+__device__ __forceinline__ float block_sum(float v, float* red) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  __syncthreads();
+  if (l == 0) red[w] = v;
+  __syncthreads();
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < NT / 32; ++i) s += red[i];   // same order in every thread
+  return s;
+}
+
+// One CTA per output row.  MAXV = max 8-element vectors per thread.
+template <int NT, int MAXV>
+__global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x, const bf16x8* __restrict__ add,
+                                                    const bf16x8* __restrict__ add_bias, bf16x8* x_out,
+                                                    bf16x8* __restrict__ y, const bf16x8* __restrict__ gamma,
+                                                    const bf16x8* __restrict__ beta, int h, int in_row_step,
+                                                    int in_row_off, float eps) {
+  __shared__ float red[NT / 32];
+  const int nv = h >> 3;
+  const int64_t in_row = (int64_t)blockIdx.x * in_row_step + in_row_off;
+  const bf16x8* xr = x + in_row * nv;
+  float r[MAXV][8];
+  float s = 0.f;
+#pragma unroll
+  for (int j = 0; j < MAXV; ++j) {
+    const int v = threadIdx.x + j * NT;
+    if (v < nv) {
+      unpack8(xr[v], r[j]);
+      if (add) {
+        float a[8];
+        unpack8(add[in_row * nv + v], a);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) r[j][e] += a[e];
+      }
+      if (add_bias) {
+        float a[8];
+        unpack8(add_bias[v], a);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) r[j][e] += a[e];
+      }
+      bf16x8 pk = pack8(r[j]);          // the residual stream is stored in bf16
+      unpack8(pk, r[j]);
+      if (x_out) x_out[(int64_t)blockIdx.x * nv + v] = pk;
+#pragma unroll
+      for (int e = 0; e < 8; ++e) s += r[j][e];
+    }
+  }
+  const float mean = block_sum<NT>(s, red) / (float)h;
+  float q = 0.f;
+#pragma unroll
+  for (int j = 0; j < MAXV; ++j) {
+    const int v = threadIdx.x + j * NT;
+    if (v < nv) {
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        const float dlt = r[j][e] - mean;
+        q += dlt * dlt;
+      }
+    }
+  }
+  const float var = block_sum<NT>(q, red) / (float)h;
+  const float rstd = 1.0f / sqrtf(var + eps);
+#pragma unroll
+  for (int j = 0; j < MAXV; ++j) {
+    const int v = threadIdx.x + j * NT;
+    if (v < nv) {
+      float g[8], b[8], o[8];
+      unpack8(gamma[v], g);
+      unpack8(beta[v], b);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) o[e] = (r[j][e] - mean) * rstd * g[e] + b[e];
+      y[(int64_t)blockIdx.x * nv + v] = pack8(o);
+    }
+  }
+}
+
+int add_layernorm_launch(const void* x, const void* add, const void* add_bias, void* x_out, void* y,
+                         const void* gamma, const void* beta, int rows, int h, int in_row_step, int in_row_off,
+                         float eps, cudaStream_t stream) {
+  if (rows <= 0) return 0;
+  if (h % 8 || h > 8 * 256 * 8 || !x || !y || !gamma || !beta) return LIGER_EINVAL;
+  const bf16x8* X = (const bf16x8*)x;
+  const bf16x8* A = (const bf16x8*)add;
+  const bf16x8* AB = (const bf16x8*)add_bias;
+  const int nv = h / 8;
+  if (nv <= 128) {
+    add_ln_kernel<128, 1><<<rows, 128, 0, stream>>>(X, A, AB, (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma,
+                                                    (const bf16x8*)beta, h, in_row_step, in_row_off, eps);
+  } else if (nv <= 256 * 2) {
+    add_ln_kernel<256, 2><<<rows, 256, 0, stream>>>(X, A, AB, (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma,
+                                                    (const bf16x8*)beta, h, in_row_step, in_row_off, eps);
+  } else {
+    add_ln_kernel<256, 8><<<rows, 256, 0, stream>>>(X, A, AB, (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma,
+                                                    (const bf16x8*)beta, h, in_row_step, in_row_off, eps);
+  }
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+// ------------------------------------------------------------------ embedding
+__global__ void embed_kernel(const int32_t* __restrict__ ids, const bf16x8* __restrict__ e_tok,
+                             const bf16x8* __restrict__ e_pos, bf16x8* __restrict__ out, int h, int seq_len,
+                             int start_pos) {
+  const int i = blockIdx.x;
+  const int nv = h >> 3;
+  const int64_t id = ids[i];
+  const int pos = start_pos + (seq_len > 0 ? i % seq_len : 0) + 2;   // OPT learned positions, offset 2
+  for (int v = threadIdx.x; v < nv; v += blockDim.x) {
+    float a[8], b[8];
+    unpack8(e_tok[id * nv + v], a);
+    unpack8(e_pos[(int64_t)pos * nv + v], b);
+#pragma unroll
+    for (int e = 0; e < 8; ++e) a[e] += b[e];
+    out[(int64_t)i * nv + v] = pack8(a);
+  }
+}
+
+int embed_launch(const int32_t* ids, const void* e_tok, const void* e_pos, void* out, int rows, int h, int seq_len,
+                 int start_pos, cudaStream_t stream) {
+  if (rows <= 0) return 0;
+  if (h % 8) return LIGER_EINVAL;
+  int nt = h / 8 < 256 ? ((h / 8 + 31) / 32 * 32) : 256;
+  embed_kernel<<<rows, nt, 0, stream>>>(ids, (const bf16x8*)e_tok, (const bf16x8*)e_pos, (bf16x8*)out, h, seq_len,
+                                        start_pos);
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+// ------------------------------------------------------------------ argmax (lowest index on ties)
+__device__ __forceinline__ void better(float& bv, int& bi, float v, int i) {
+  if (v > bv || (v == bv && i < bi)) {
+    bv = v;
+    bi = i;
+  }
+}
+
+__global__ void argmax_kernel(const float* __restrict__ logits, int64_t ld, int n, int idx_offset,
+                              float* max_out, int32_t* idx_out) {
+  __shared__ float sv[32];
+  __shared__ int si[32];
+  const float* row = logits + (int64_t)blockIdx.x * ld;
+  float bv = -INFINITY;
+  int bi = 0x7fffffff;
+  for (int i = threadIdx.x; i < n; i += blockDim.x) better(bv, bi, row[i], i);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    float ov = __shfl_xor_sync(0xffffffffu, bv, o);
+    int oi = __shfl_xor_sync(0xffffffffu, bi, o);
+    better(bv, bi, ov, oi);
+  }
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  if (l == 0) {
+    sv[w] = bv;
+    si[w] = bi;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int k = 1; k < (int)(blockDim.x >> 5); ++k) better(bv, bi, sv[k], si[k]);
+    max_out[blockIdx.x] = bv;
+    idx_out[blockIdx.x] = bi + idx_offset;
+  }
+}
+
+int argmax_launch(const float* logits, int64_t ld, int rows, int n, int idx_offset, float* max_out,
+                  int32_t* idx_out, cudaStream_t stream) {
+  if (rows <= 0) return 0;
+  argmax_kernel<<<rows, 1024, 0, stream>>>(logits, ld, n, idx_offset, max_out, idx_out);
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+// vals/idx: [world][rows] gathered from every rank's vocab shard.  Writes the
+// greedy token to tok_cur[r] (fed to the next decode pass) and to
+// tok_out[r * out_stride + out_col] (the batch's generated sequence).
+__global__ void argmax_pick_kernel(const float* vals, const int32_t* idx, int world, int rows, int32_t* tok_cur,
+                                   int32_t* tok_out, int out_stride, int out_col) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= rows) return;
+  float bv = vals[r];
+  int bi = idx[r];
+  for (int w = 1; w < world; ++w) better(bv, bi, vals[w * rows + r], idx[w * rows + r]);
+  tok_cur[r] = bi;
+  if (tok_out) tok_out[(int64_t)r * out_stride + out_col] = bi;
+}
+
+int argmax_pick_launch(const float* vals, const int32_t* idx, int world, int rows, int32_t* tok_cur,
+                       int32_t* tok_out, int out_stride, int out_col, cudaStream_t stream) {
+  if (rows <= 0) return 0;
+  argmax_pick_kernel<<<(rows + 127) / 128, 128, 0, stream>>>(vals, idx, world, rows, tok_cur, tok_out, out_stride,
+                                                             out_col);
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+// ------------------------------------------------------------------ C0 generator (device side)
+// Same definition as liger_inputs/c0.py, implemented independently.
+__device__ __forceinline__ uint64_t mix64_dev(uint64_t x) {
+  x ^= x >> 30;
+  x *= 0xBF58476D1CE4E5B9ull;
+  x ^= x >> 27;
+  x *= 0x94D049BB133111EBull;
+  x ^= x >> 31;
+  return x;
+}
+
+__global__ void c0_fill_kernel(__nv_bfloat16* dst, int rows, int cols, int64_t ld, uint64_t base, int64_t row_off,
+                               int64_t col_off, int64_t irs, int64_t ics, float scale, int kind) {
+  const int64_t total = (int64_t)rows * cols;
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = t / cols, c = t % cols;
+    const uint64_t idx = (uint64_t)((r + row_off) * irs + (c + col_off) * ics);
+    const uint64_t u = mix64_dev(base + idx);
+    const int32_t iv = (int32_t)(u >> 40) - (1 << 23);
+    const float v = (float)iv * (1.0f / 8388608.0f);
+    float w;
+    if (kind == 1) w = __fadd_rn(1.0f, __fmul_rn(v, 0.0625f));
+    else if (kind == 2) w = __fmul_rn(v, 0.0625f);
+    else w = __fmul_rn(v, scale);
+    dst[r * ld + c] = __float2bfloat16_rn(w);
+  }
+}
+
+int c0_fill_launch(void* dst, int rows, int cols, int64_t ld, uint64_t seed, uint64_t tensor_id, int64_t row_off,
+                   int64_t col_off, int64_t idx_row_stride, int64_t idx_col_stride, int exp, int kind,
+                   cudaStream_t stream) {
+  if (rows <= 0 || cols <= 0) return 0;
+  const uint64_t G = 0x9E3779B97F4A7C15ull, T = 0xD1B54A32D192ED03ull;
+  const uint64_t base = seed * G + tensor_id * T + G;
+  const float scale = ldexpf(1.0f, exp);
+  const int64_t total = (int64_t)rows * cols;
+  int blocks = (int)((total + 255) / 256);
+  if (blocks > 148 * 32) blocks = 148 * 32;
+  c0_fill_kernel<<<blocks, 256, 0, stream>>>((__nv_bfloat16*)dst, rows, cols, ld, base, row_off, col_off,
+                                             idx_row_stride, idx_col_stride, scale, kind);
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+__global__ void copy_i32_kernel(const int32_t* s, int32_t* d, int n) {
+  int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) d[i] = s[i];
+}
+int copy_tokens_launch(const int32_t* src, int32_t* dst, int n, cudaStream_t stream) {
+  if (n <= 0) return 0;
+  copy_i32_kernel<<<(n + 255) / 256, 256, 0, stream>>>(src, dst, n);
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+}  // namespace liger

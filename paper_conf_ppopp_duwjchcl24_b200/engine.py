@@ -1,0 +1,120 @@
+"""Python convenience layer over the serving calls of libliger.so.
+
+Marshalling only: LigerEngine builds a liger_cfg from a model config, calls
+liger_init / liger_load_layer / liger_load_embed, and forwards submit / step /
+poll / drain.  All computation happens inside the library.
+"""
+import ctypes as C
+
+import numpy as np
+
+from . import liger as L
+
+
+class LigerEngine:
+    def __init__(self, model_cfg, *, world=1, rank=0, nccl_uid=None, mode="interleaved", max_batch=8,
+                 max_seq=512, max_new=32, max_inflight=2, decomp_factor=8, contention_factor=1.0, seed=0,
+                 load=True):
+        lib = L.lib()
+        cfg = L.liger_cfg()
+        cfg.n_layers, cfg.hidden, cfg.n_heads = model_cfg.n_layers, model_cfg.hidden, model_cfg.n_heads
+        cfg.ffn, cfg.vocab, cfg.max_pos = model_cfg.ffn, model_cfg.vocab, model_cfg.max_pos
+        cfg.act = L.ACT[model_cfg.act]
+        cfg.ln_eps = model_cfg.ln_eps
+        cfg.max_batch, cfg.max_seq, cfg.max_new = max_batch, max_seq, max_new
+        cfg.mode = L.MODE[mode]
+        cfg.max_inflight = max_inflight
+        cfg.decomp_factor = decomp_factor
+        cfg.contention_factor = contention_factor
+        cfg.seed = seed
+        self.cfg = cfg
+        self.model = model_cfg
+        self.world, self.rank = world, rank
+        self.seed = seed
+        ctx = C.c_void_p()
+        uid = None if nccl_uid is None else C.create_string_buffer(bytes(nccl_uid), 128)
+        L.check(lib.liger_init(world, rank, C.byref(cfg), uid, C.byref(ctx)), None, "liger_init")
+        self.ctx = ctx
+        if load:
+            self.load(seed)
+
+    @staticmethod
+    def unique_id():
+        buf = C.create_string_buffer(128)
+        L.check(L.lib().liger_nccl_unique_id(buf), None, "liger_nccl_unique_id")
+        return buf.raw
+
+    def _chk(self, rc, what):
+        return L.check(rc, self.ctx, what)
+
+    def load(self, seed):
+        lib = L.lib()
+        for l in range(self.model.n_layers):
+            self._chk(lib.liger_load_layer(self.ctx, l, seed), "liger_load_layer")
+        self._chk(lib.liger_load_embed(self.ctx, seed), "liger_load_embed")
+
+    def profile(self, m_list):
+        arr = (C.c_int32 * len(m_list))(*m_list)
+        self._chk(L.lib().liger_profile(self.ctx, arr, len(m_list)), "liger_profile")
+
+    def submit(self, tokens, batch, seq_len, n_new, arrival_s=-1.0, device_tokens=None):
+        """tokens: numpy int32 [batch*seq_len] (host) or None with device_tokens = a device
+        int32 tensor (kept alive by the caller until the batch finishes)."""
+        lib = L.lib()
+        if device_tokens is not None:
+            rc = lib.liger_submit(self.ctx, batch, seq_len, C.c_void_p(device_tokens.data_ptr()), 1, n_new,
+                                  float(arrival_s))
+        else:
+            t = np.ascontiguousarray(tokens, dtype=np.int32)
+            rc = lib.liger_submit(self.ctx, batch, seq_len, t.ctypes.data_as(C.c_void_p), 0, n_new, float(arrival_s))
+        return self._chk(rc, "liger_submit")
+
+    def step(self):
+        return self._chk(L.lib().liger_step(self.ctx), "liger_step")
+
+    def drain(self):
+        self._chk(L.lib().liger_drain(self.ctx), "liger_drain")
+
+    def poll(self, bid, want_tokens=False):
+        res = L.liger_result()
+        out = None
+        buf = None
+        if want_tokens:
+            buf = np.zeros(self.cfg.max_batch * self.cfg.max_new, dtype=np.int32)
+            out = buf.ctypes.data_as(C.c_void_p)
+        rc = self._chk(L.lib().liger_poll(self.ctx, bid, C.byref(res), out), "liger_poll")
+        if rc == L.LIGER_PENDING:
+            return None
+        toks = None
+        if want_tokens:
+            toks = buf[:res.batch * res.n_new].reshape(res.batch, res.n_new).copy()
+        return res, toks
+
+    def stats(self):
+        s = L.liger_stats_t()
+        self._chk(L.lib().liger_stats(self.ctx, C.byref(s)), "liger_stats")
+        return {k: getattr(s, k) for k, _ in s._fields_}
+
+    def reset_stats(self):
+        self._chk(L.lib().liger_reset_stats(self.ctx), "liger_reset_stats")
+
+    def set_kernel_timing(self, on):
+        self._chk(L.lib().liger_set_kernel_timing(self.ctx, int(on)), "liger_set_kernel_timing")
+
+    def kernel_timing(self):
+        cnt = (C.c_int64 * 4)()
+        ms, by, fl = (C.c_double * 4)(), (C.c_double * 4)(), (C.c_double * 4)()
+        self._chk(L.lib().liger_kernel_timing(self.ctx, cnt, ms, by, fl), "liger_kernel_timing")
+        names = ["gemm", "attn", "ln", "allreduce"]
+        return {n: dict(count=cnt[i], ms=ms[i], bytes=by[i], flops=fl[i]) for i, n in enumerate(names)}
+
+    def close(self):
+        if self.ctx:
+            L.lib().liger_finalize(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,303 @@
+"""GPU parity: every hot-path kernel, called through the C ABI, against the fp64
+CPU oracle on the same seeded inputs (task ③).  Tolerances (R16,
+from BASELINE.json): bf16 outputs rel = max|g-r|/max|r| <= 2e-2; layer outputs
+additionally MAE <= 1e-3; integer/index work bit-exact."""
+import numpy as np
+import pytest
+import torch
+
+from liger_inputs import get_config, layer_tensor, global_tensor, layer_activation, c0_values
+from oracle import model as om
+from tests.gpu_helpers import (to_np64, bf16_dev, errs, workspace, shard_weights_device, run_layer_rank,
+                               run_mlp_rank)
+
+pytestmark = pytest.mark.gpu
+REL, MAE = 2e-2, 1e-3
+
+
+@pytest.fixture(scope="module")
+def L():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ppopp_duwjchcl24_b200 import liger
+    liger.lib()
+    return liger
+
+
+# ---------------------------------------------------------------- C0 generator
+def test_c0_device_matches_numpy_bit_exact(L):
+    cfg = get_config("tiny")
+    for t, r in ((1, 0), (2, 1)):
+        W = shard_weights_device(L, cfg, 3, 1, t, r)
+        torch.cuda.synchronize()
+        full = {k: layer_tensor(cfg, 3, 1, k) for k in om.LAYER_KINDS}
+        shard = om.shard_layer(cfg, {k: v.astype(np.float32) for k, v in full.items()}, t, r)
+        for k in ("w_qkv", "w_o", "w_1", "w_2"):
+            assert np.array_equal(W[k].float().cpu().numpy(), shard[k].T), k     # K-major device layout
+        for k in ("b_qkv", "b_1", "ln1_g", "ln1_b", "ln2_g", "ln2_b"):
+            assert np.array_equal(W[k].float().cpu().numpy(), shard[k]), k
+        assert np.array_equal(W["b_o"].float().cpu().numpy(), full["b_o"])
+
+
+# ---------------------------------------------------------------- GEMM
+GEMM_SHAPES = [(1, 128, 64), (2, 384, 256), (16, 256, 128), (37, 200, 320), (64, 512, 1024), (65, 640, 768),
+               (300, 384, 512), (513, 256, 256), (1024, 1024, 512)]
+
+
+@pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
+@pytest.mark.parametrize("act", ["none", "relu", "gelu_tanh"])
+def test_gemm_vs_oracle(L, M, N, K, act):
+    rng = np.random.default_rng(M * 7 + N + K)
+    x = c0_values(1, 77, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K)
+    w = c0_values(1, 78, np.arange(N * K, dtype=np.uint64), -int(np.log2(K)) // 2).reshape(N, K)
+    b = c0_values(1, 79, np.arange(N, dtype=np.uint64), -4)
+    xd, wd, bd = bf16_dev(x), bf16_dev(w), bf16_dev(b)
+    out = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
+    sc = N // 3
+    L.gemm(xd, wd, out, bias=bd, act=act, scale_cols=sc, scale=0.125, workspace=workspace(L.gemm_workspace_bytes(M, N, K)))
+    torch.cuda.synchronize()
+    ref = x.astype(np.float64) @ w.astype(np.float64).T + b
+    ref[:, :sc] *= 0.125
+    ref = {"none": lambda v: v, "relu": om.relu, "gelu_tanh": om.gelu_tanh}[act](ref)
+    rel, mae = errs(to_np64(out), ref)
+    assert rel <= REL, (rel, mae)
+    assert mae <= 1e-2 * np.abs(ref).mean() + 1e-6
+
+
+@pytest.mark.parametrize("M,N,K", [(2, 384, 256), (8, 960, 1024), (300, 640, 512), (64, 5120, 2560)])
+def test_gemm_decomposition_bit_exact(L, M, N, K):
+    """§3.6 vertical decomposition: any k/F column piece reproduces the full GEMM's bits."""
+    x = bf16_dev(c0_values(2, 1, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K))
+    w = bf16_dev(c0_values(2, 2, np.arange(N * K, dtype=np.uint64), -5).reshape(N, K))
+    ws = workspace(L.gemm_workspace_bytes(M, N, K))
+    full = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
+    L.gemm(x, w, full, workspace=ws)
+    F = 8
+    for ks in ([1] * 8, [2, 3, 3], [7, 1], [3, 5]):
+        out = torch.zeros_like(full)
+        u = 0
+        for k in ks:
+            c0 = (N * u // F) // 16 * 16
+            c1 = N if u + k == F else (N * (u + k) // F) // 16 * 16
+            L.gemm(x, w, out, n0=c0, n1=c1, workspace=ws)
+            u += k
+        torch.cuda.synchronize()
+        assert torch.equal(out, full), ks
+
+
+@pytest.mark.parametrize("name,M", [("opt-13b", 8), ("opt-13b", 512), ("opt-66b", 2)])
+def test_gemm_full_size_sampled(L, name, M):
+    """BASELINE.json full sizes (per-rank shapes of the bench launch): compare sampled
+    output columns, computed one by one by the oracle."""
+    cfg = get_config(name)
+    t = 1 if name == "opt-13b" else 8
+    h, fl = cfg.hidden, cfg.ffn // t
+    for (N, K, kind) in ((3 * h // t, h, "w_qkv"), (fl, h, "w_1"), (h, fl, "w_2")):
+        x = c0_values(5, 9, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K)
+        w = c0_values(5, 10, np.arange(N * K, dtype=np.uint64), -6).reshape(N, K)
+        out = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
+        L.gemm(bf16_dev(x), bf16_dev(w), out, workspace=workspace(L.gemm_workspace_bytes(M, N, K)))
+        torch.cuda.synchronize()
+        cols = np.random.default_rng(0).choice(N, 64, replace=False)
+        ref = x.astype(np.float64) @ w[cols].astype(np.float64).T
+        rel, _ = errs(to_np64(out)[:, cols], ref)
+        assert rel <= REL, (kind, rel)
+
+
+def test_gemm_empty_and_errors(L):
+    x = torch.zeros(0, 64, dtype=torch.bfloat16, device="cuda")
+    w = torch.zeros(128, 64, dtype=torch.bfloat16, device="cuda")
+    out = torch.zeros(0, 128, dtype=torch.bfloat16, device="cuda")
+    L.gemm(x, w, out)            # M = 0: no launch, no error
+    with pytest.raises(L.LigerError):
+        L.gemm(torch.zeros(4, 60, dtype=torch.bfloat16, device="cuda"),
+               torch.zeros(128, 60, dtype=torch.bfloat16, device="cuda"),
+               torch.zeros(4, 128, dtype=torch.bfloat16, device="cuda"))
+
+
+# ---------------------------------------------------------------- LayerNorm
+@pytest.mark.parametrize("R,h", [(1, 256), (7, 1024), (33, 5120), (3, 12288)])
+def test_add_layernorm_vs_oracle(L, R, h):
+    x = c0_values(3, 1, np.arange(R * h, dtype=np.uint64), 0).reshape(R, h)
+    a = c0_values(3, 2, np.arange(R * h, dtype=np.uint64), -1).reshape(R, h)
+    ab = c0_values(3, 3, np.arange(h, dtype=np.uint64), -3)
+    g = 1 + c0_values(3, 4, np.arange(h, dtype=np.uint64), -4)
+    be = c0_values(3, 5, np.arange(h, dtype=np.uint64), -4)
+    xd = bf16_dev(x)
+    y = torch.empty_like(xd)
+    xo = torch.empty_like(xd)
+    L.add_layernorm(xd, bf16_dev(g), bf16_dev(be), y, add=bf16_dev(a), add_bias=bf16_dev(ab), x_out=xo)
+    torch.cuda.synchronize()
+    r = x.astype(np.float64) + a + ab
+    rel_x, _ = errs(to_np64(xo), r)
+    assert rel_x <= 2 ** -8
+    ref = om.layer_norm(to_np64(xo), g.astype(np.float64), be, 1e-5)
+    rel, mae = errs(to_np64(y), ref)
+    assert rel <= REL and mae <= 1e-2
+
+
+def test_layernorm_row_gather(L):
+    """Final LN on the last token of each sequence (in_row = i*s + s-1)."""
+    b, s, h = 3, 5, 256
+    x = c0_values(4, 1, np.arange(b * s * h, dtype=np.uint64), 0).reshape(b * s, h)
+    g = np.ones(h, np.float32)
+    be = np.zeros(h, np.float32)
+    y = torch.empty(b, h, dtype=torch.bfloat16, device="cuda")
+    L.add_layernorm(bf16_dev(x), bf16_dev(g), bf16_dev(be), y, rows=b, in_row_step=s, in_row_off=s - 1)
+    torch.cuda.synchronize()
+    ref = om.layer_norm(x[s - 1::s].astype(np.float64), 1.0, 0.0, 1e-5)
+    assert errs(to_np64(y), ref)[0] <= REL
+
+
+# ---------------------------------------------------------------- embedding
+def test_embed_vs_oracle(L):
+    cfg = get_config("tiny")
+    g = om.global_weights(cfg, 0)
+    b, s = 2, 9
+    ids = np.random.default_rng(0).integers(0, cfg.vocab, size=(b, s)).astype(np.int32)
+    out = torch.empty(b * s, cfg.hidden, dtype=torch.bfloat16, device="cuda")
+    L.embed(torch.from_numpy(ids.reshape(-1)).cuda(), bf16_dev(g["e_tok"]), bf16_dev(g["e_pos"]), out, seq_len=s)
+    torch.cuda.synchronize()
+    ref = om.embed(cfg, g, ids, np.arange(s)).reshape(b * s, -1)
+    assert errs(to_np64(out), ref)[0] <= 2 ** -8
+
+
+# ---------------------------------------------------------------- attention
+def _qkv(b, s, heads, d, seed):
+    q = c0_values(seed, 1, np.arange(b * s * heads * d, dtype=np.uint64), 0).reshape(b * s, heads * d) * d ** -0.5
+    k = c0_values(seed, 2, np.arange(b * s * heads * d, dtype=np.uint64), 0).reshape(b * s, heads * d)
+    v = c0_values(seed, 3, np.arange(b * s * heads * d, dtype=np.uint64), 0).reshape(b * s, heads * d)
+    return np.concatenate([q, k, v], axis=1).astype(np.float32)
+
+
+def _split(a, b, s, heads, d):
+    return a.reshape(b, s, heads, d).transpose(0, 2, 1, 3)
+
+
+@pytest.mark.parametrize("b,s,heads,d", [(2, 32, 2, 64), (1, 1, 1, 128), (3, 65, 2, 128), (2, 200, 3, 64),
+                                         (1, 512, 2, 128)])
+def test_attention_prefill_and_decode_vs_oracle(L, b, s, heads, d):
+    qkv = _qkv(b, s, heads, d, 11)
+    qkvd = bf16_dev(qkv)
+    qkv = to_np64(qkvd)
+    o = torch.empty(b * s, heads * d, dtype=torch.bfloat16, device="cuda")
+    maxp = (s + 40) // 16 + 1
+    pt = torch.from_numpy(np.random.default_rng(0).permutation(b * maxp).astype(np.int32).reshape(b, maxp)).cuda()
+    pool = torch.zeros(b * maxp, 2, heads, 16, d, dtype=torch.bfloat16, device="cuda")
+    L.attn_prefill(qkvd, o, pool, pt, b=b, s=s, heads=heads, d=d)
+    torch.cuda.synchronize()
+    hd = heads * d
+    q, k, v = (_split(qkv[:, i * hd:(i + 1) * hd], b, s, heads, d) for i in range(3))
+    ref = om.causal_attention(q, k, v, np.arange(s), np.arange(s)).transpose(0, 2, 1, 3).reshape(b * s, hd)
+    assert errs(to_np64(o), ref)[0] <= REL
+    # paged cache holds exactly K and V (index/byte work: bit-exact)
+    ptn = pt.cpu().numpy()
+    pl = pool.float().cpu().numpy()
+    for bi in range(b):
+        for p in range(s):
+            pg = ptn[bi, p // 16]
+            assert np.array_equal(pl[pg, 0, :, p % 16, :], k[bi, :, p, :])
+            assert np.array_equal(pl[pg, 1, :, p % 16, :], v[bi, :, p, :])
+    # two decode steps over the cache
+    for step in range(2):
+        pos = s + step
+        q1 = _qkv(b, 1, heads, d, 20 + step)
+        q1d = bf16_dev(q1)
+        q1 = to_np64(q1d)
+        o1 = torch.empty(b, hd, dtype=torch.bfloat16, device="cuda")
+        L.attn_decode(q1d, o1, pool, pt, b=b, pos=pos, heads=heads, d=d,
+                      workspace=workspace(L.attn_decode_workspace_bytes(b, heads, d, pos + 1)))
+        torch.cuda.synchronize()
+        k = np.concatenate([k, _split(q1[:, hd:2 * hd], b, 1, heads, d)], axis=2)
+        v = np.concatenate([v, _split(q1[:, 2 * hd:], b, 1, heads, d)], axis=2)
+        qq = _split(q1[:, :hd], b, 1, heads, d)
+        ref1 = om.causal_attention(qq, k, v, np.array([pos]), np.arange(pos + 1)).transpose(0, 2, 1, 3).reshape(b, hd)
+        assert errs(to_np64(o1), ref1)[0] <= REL
+
+
+def test_decode_attention_long_context_split(L):
+    """ctx > 256 exercises the deterministic multi-chunk merge; the result must not
+    depend on scheduling (run twice, bit-identical)."""
+    b, heads, d, s = 2, 2, 128, 700
+    qkv = bf16_dev(_qkv(b, s, heads, d, 5))
+    o = torch.empty(b * s, heads * d, dtype=torch.bfloat16, device="cuda")
+    maxp = (s + 16) // 16 + 1
+    pt = torch.arange(b * maxp, dtype=torch.int32, device="cuda").reshape(b, maxp)
+    pool = torch.zeros(b * maxp, 2, heads, 16, d, dtype=torch.bfloat16, device="cuda")
+    L.attn_prefill(qkv, o, pool, pt, b=b, s=s, heads=heads, d=d)
+    q1d = bf16_dev(_qkv(b, 1, heads, d, 6))
+    ws = workspace(L.attn_decode_workspace_bytes(b, heads, d, s + 1))
+    outs = []
+    for _ in range(2):
+        o1 = torch.empty(b, heads * d, dtype=torch.bfloat16, device="cuda")
+        L.attn_decode(q1d, o1, pool, pt, b=b, pos=s, heads=heads, d=d, workspace=ws)
+        outs.append(o1)
+    torch.cuda.synchronize()
+    assert torch.equal(outs[0], outs[1])
+    hd = heads * d
+    qkv_np, q1 = to_np64(qkv), to_np64(q1d)
+    k = np.concatenate([_split(qkv_np[:, hd:2 * hd], b, s, heads, d), _split(q1[:, hd:2 * hd], b, 1, heads, d)], 2)
+    v = np.concatenate([_split(qkv_np[:, 2 * hd:], b, s, heads, d), _split(q1[:, 2 * hd:], b, 1, heads, d)], 2)
+    ref = om.causal_attention(_split(q1[:, :hd], b, 1, heads, d), k, v, np.array([s]), np.arange(s + 1))
+    assert errs(to_np64(outs[0]), ref.transpose(0, 2, 1, 3).reshape(b, hd))[0] <= REL
+
+
+# ---------------------------------------------------------------- argmax
+def test_argmax_lowest_index_on_ties(L):
+    logits = np.random.default_rng(0).standard_normal((5, 3000)).astype(np.float32)
+    logits[1, 17] = logits[1, 2999] = 50.0
+    d = torch.from_numpy(logits).cuda()
+    mx = torch.empty(5, device="cuda")
+    ix = torch.empty(5, dtype=torch.int32, device="cuda")
+    L.argmax(d, mx, ix, idx_offset=100)
+    torch.cuda.synchronize()
+    assert np.array_equal(ix.cpu().numpy(), np.argmax(logits, axis=1) + 100)
+    assert np.array_equal(mx.cpu().numpy(), logits.max(axis=1))
+
+
+# ---------------------------------------------------------------- full TP decoder layer through the C ABI
+@pytest.mark.parametrize("name,t,b,s", [("tiny", 1, 2, 32), ("tiny", 2, 2, 32), ("tiny", 4, 3, 17),
+                                        ("opt-13b", 2, 1, 64)])
+def test_tp_layer_vs_oracle(L, name, t, b, s):
+    """One decoder layer (prefill + one decode step), sharded t ways, each rank's
+    partials produced by the C-ABI kernels and summed in bf16 (the all-reduce),
+    against the unsharded fp64 oracle layer fed the same bf16 input."""
+    cfg = get_config(name)
+    layer, seed = 0, 0
+    M = b * s
+    x = layer_activation(cfg, seed, layer, M + b)
+    x_pf, x_dc = x[:M], x[M:]
+    Ws = [shard_weights_device(L, cfg, seed, layer, t, r) for r in range(t)]
+    w = om.layer_weights(cfg, seed, layer)
+
+    def gpu_layer(xin, start_pos, kvs):
+        xd = bf16_dev(xin)
+        parts, new_kv = [], []
+        for r in range(t):
+            p, kv = run_layer_rank(L, cfg, Ws[r], t, xd, b, s, start_pos, None if kvs is None else kvs[r])
+            parts.append(p)
+            new_kv.append(kv)
+        ar = parts[0].float()
+        for p in parts[1:]:
+            ar = ar + p.float()
+        ar = ar.bfloat16()
+        x1 = torch.empty_like(xd)
+        y2 = torch.empty_like(xd)
+        L.add_layernorm(xd, Ws[0]["ln2_g"], Ws[0]["ln2_b"], y2, add=ar, add_bias=Ws[0]["b_o"], x_out=x1,
+                        eps=cfg.ln_eps)
+        parts2 = [run_mlp_rank(L, cfg, Ws[r], t, y2) for r in range(t)]
+        ar2 = parts2[0].float()
+        for p in parts2[1:]:
+            ar2 = ar2 + p.float()
+        out = (x1.float() + ar2.bfloat16().float() + Ws[0]["b_2"].float()).bfloat16()
+        return out, new_kv
+
+    out_pf, kvs = gpu_layer(x_pf, 0, None)
+    out_dc, _ = gpu_layer(x_dc, s, kvs)
+    torch.cuda.synchronize()
+    xin = x.astype(np.float64)
+    ref_pf, k, v = om.decoder_layer(cfg, w, xin[:M].reshape(b, s, -1))
+    ref_dc, _, _ = om.decoder_layer(cfg, w, xin[M:].reshape(b, 1, -1), k, v, start_pos=s)
+    for got, ref in ((out_pf, ref_pf.reshape(M, -1)), (out_dc, ref_dc.reshape(b, -1))):
+        rel, mae = errs(to_np64(got), ref)
+        assert rel <= REL and mae <= MAE, (rel, mae)
