@@ -150,11 +150,18 @@ int liger_result_tokens_device(liger_ctx* ctx, int64_t id, const int32_t** dev_t
 int liger_stats(liger_ctx* ctx, liger_stats_t* out);
 int liger_reset_stats(liger_ctx* ctx);
 
-/* Enable (1) / disable (0) CUDA-event timing of every GEMM and attention
- * launch on the stream it runs on; liger_kernel_timing returns, per kernel
- * class (0 = GEMM, 1 = attention, 2 = layernorm, 3 = all-reduce), the launch
+/* Enable (1) / disable (0) CUDA-event timing of every GEMM, attention,
+ * layernorm and all-reduce launch on the stream it runs on;
+ * liger_kernel_timing returns, per kernel class (LIGER_KT_*), the launch
  * count, the summed device milliseconds, and the summed algorithmic bytes and
- * flops.  Arrays of length 4, host. */
+ * flops.  Host arrays of LIGER_KT_CLASSES. */
+#define LIGER_KT_GEMM_DECODE 0   /* projection GEMMs with M <= 64 tokens (HBM-bound) */
+#define LIGER_KT_ATTN 1
+#define LIGER_KT_LN 2
+#define LIGER_KT_ALLREDUCE 3
+#define LIGER_KT_GEMM_PREFILL 4  /* projection GEMMs with M > 64 tokens (tensor-bound) */
+#define LIGER_KT_LMHEAD 5
+#define LIGER_KT_CLASSES 6
 int liger_set_kernel_timing(liger_ctx* ctx, int on);
 int liger_kernel_timing(liger_ctx* ctx, int64_t* count, double* ms, double* bytes, double* flops);
 

@@ -203,8 +203,8 @@ struct liger_ctx {
   std::vector<TimedLaunch> timed;
   std::vector<cudaEvent_t> timing_pool;
   size_t timing_next = 0;
-  int64_t tcount[4] = {0, 0, 0, 0};
-  double tms[4] = {0, 0, 0, 0}, tbytes[4] = {0, 0, 0, 0}, tflops[4] = {0, 0, 0, 0};
+  int64_t tcount[LIGER_KT_CLASSES] = {};
+  double tms[LIGER_KT_CLASSES] = {}, tbytes[LIGER_KT_CLASSES] = {}, tflops[LIGER_KT_CLASSES] = {};
 };
 
 namespace {
@@ -398,14 +398,14 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
         rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
       else
         rc = add_layernorm_launch(S.x, S.part, c->layers[li - 1].b_2, S.x, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
-      timed_end(c, st, ta, 2, (double)M * h * 2 * (li == 0 ? 2 : 4), 0);
+      timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * (li == 0 ? 2 : 4), 0);
       c->st.gpu_launches++;
       break;
     }
     case OP_LN2: {
       timed_begin(c, st, &ta);
       rc = add_layernorm_launch(S.x, S.part, W->b_o, S.x, S.y, W->g2, W->be2, M, h, 1, 0, eps, st);
-      timed_end(c, st, ta, 2, (double)M * h * 2 * 4, 0);
+      timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * 4, 0);
       c->st.gpu_launches++;
       break;
     }
@@ -435,7 +435,8 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       timed_begin(c, st, &ta);
       rc = gemm_launch(g, st);
       const double n = g.n1 - g.n0;
-      timed_end(c, st, ta, 0, (n * K + (double)M * K + (double)M * n) * 2, 2.0 * M * n * K);
+      timed_end(c, st, ta, M <= 64 ? LIGER_KT_GEMM_DECODE : LIGER_KT_GEMM_PREFILL,
+                (n * K + (double)M * K + (double)M * n) * 2, 2.0 * M * n * K);
       c->st.gpu_launches++;
       break;
     }
@@ -444,12 +445,12 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       timed_begin(c, st, &ta);
       if (pass == 0) {
         rc = attn_prefill_launch(S.qkv, S.attn, pool, S.page_table, c->max_pages, bt->b, bt->s, c->al, c->d, st);
-        timed_end(c, st, ta, 1, (double)M * c->hl * 2 * 6, 2.0 * bt->b * c->al * c->d * (double)bt->s * bt->s);
+        timed_end(c, st, ta, LIGER_KT_ATTN, (double)M * c->hl * 2 * 6, 2.0 * bt->b * c->al * c->d * (double)bt->s * bt->s);
       } else {
         const int pos = bt->s + pass - 1;
         rc = attn_decode_launch(S.qkv, S.attn, pool, S.page_table, c->max_pages, bt->b, pos, c->al, c->d,
                                 S.attn_ws, S.attn_ws_bytes, st);
-        timed_end(c, st, ta, 1, (double)bt->b * c->hl * 2 * 2 * (pos + 1),
+        timed_end(c, st, ta, LIGER_KT_ATTN, (double)bt->b * c->hl * 2 * 2 * (pos + 1),
                   4.0 * bt->b * c->al * c->d * (double)(pos + 1));
       }
       c->st.gpu_launches++;
@@ -466,7 +467,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
                                           ncclSum, c->comm, st);
         if (r != ncclSuccess) return fail(c, LIGER_ENCCL, std::string("ncclAllReduce: ") + nccl().GetErrorString(r));
       }
-      timed_end(c, st, ta, 3, (double)(e1 - e0) * 2, 0);
+      timed_end(c, st, ta, LIGER_KT_ALLREDUCE, (double)(e1 - e0) * 2, 0);
       c->st.comm_kernels++;
       c->st.gpu_launches++;
       break;
@@ -486,7 +487,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       g.workspace = S.gemm_ws; g.ws_bytes = S.gemm_ws_bytes;
       timed_begin(c, st, &ta);
       rc = gemm_launch(g, st);
-      timed_end(c, st, ta, 0, ((double)c->Vl * h + (double)b * h) * 2 + (double)b * c->Vl * 4,
+      timed_end(c, st, ta, LIGER_KT_LMHEAD, ((double)c->Vl * h + (double)b * h) * 2 + (double)b * c->Vl * 4,
                 2.0 * b * c->Vl * h);
       if (rc) break;
       rc = argmax_launch(S.logits, c->Vl, b, c->Vl, c->rank * c->Vl, S.vals_all + (size_t)c->rank * b,
@@ -1036,14 +1037,14 @@ int liger_set_kernel_timing(liger_ctx* c, int on) {
   if (!c) return LIGER_EINVAL;
   timing_flush(c);
   c->timing = on != 0;
-  for (int i = 0; i < 4; ++i) c->tcount[i] = 0, c->tms[i] = c->tbytes[i] = c->tflops[i] = 0;
+  for (int i = 0; i < LIGER_KT_CLASSES; ++i) c->tcount[i] = 0, c->tms[i] = c->tbytes[i] = c->tflops[i] = 0;
   return LIGER_OK;
 }
 
 int liger_kernel_timing(liger_ctx* c, int64_t* count, double* ms, double* bytes, double* flops) {
   if (!c) return LIGER_EINVAL;
   timing_flush(c);
-  for (int i = 0; i < 4; ++i) {
+  for (int i = 0; i < LIGER_KT_CLASSES; ++i) {
     if (count) count[i] = c->tcount[i];
     if (ms) ms[i] = c->tms[i];
     if (bytes) bytes[i] = c->tbytes[i];

@@ -102,10 +102,11 @@ class LigerEngine:
         self._chk(L.lib().liger_set_kernel_timing(self.ctx, int(on)), "liger_set_kernel_timing")
 
     def kernel_timing(self):
-        cnt = (C.c_int64 * 4)()
-        ms, by, fl = (C.c_double * 4)(), (C.c_double * 4)(), (C.c_double * 4)()
+        n = len(L.KT_NAMES)
+        cnt = (C.c_int64 * n)()
+        ms, by, fl = (C.c_double * n)(), (C.c_double * n)(), (C.c_double * n)()
         self._chk(L.lib().liger_kernel_timing(self.ctx, cnt, ms, by, fl), "liger_kernel_timing")
-        names = ["gemm", "attn", "ln", "allreduce"]
+        names = L.KT_NAMES
         return {n: dict(count=cnt[i], ms=ms[i], bytes=by[i], flops=fl[i]) for i, n in enumerate(names)}
 
     def close(self):

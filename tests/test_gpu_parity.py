@@ -8,7 +8,7 @@ import torch
 
 from liger_inputs import get_config, layer_tensor, global_tensor, layer_activation, c0_values
 from oracle import model as om
-from tests.gpu_helpers import (to_np64, bf16_dev, errs, workspace, shard_weights_device, run_layer_rank,
+from gpu_helpers import (to_np64, bf16_dev, errs, workspace, shard_weights_device, run_layer_rank,
                                run_mlp_rank)
 
 pytestmark = pytest.mark.gpu
