@@ -17,7 +17,9 @@ its elements from their global indices.
 
 Scales (reading R16, chosen to keep per-layer output RMS well below
 1 so that bf16 output rounding stays inside BASELINE.json's MAE bound):
-  GEMM weight with fan-in K : e = round(0.5*log2(3/K)) - 1
+  GEMM weight with fan-in K : e = round(0.5*log2(3/K)) - 1   (W_qkv, W_1)
+                              e = round(0.5*log2(3/K)) - 2   (output projections W_o, W_2,
+                                  halving the residual-branch gain, as GPT-2 scales them)
   bias                      : e = -6
   embeddings E_tok, E_pos   : e = -3
   layer-input activations   : e = -2   (layer-level parity tests only)
@@ -73,8 +75,12 @@ def bf16_rne(f: np.ndarray) -> np.ndarray:
     return u.view(np.float32)
 
 
-def weight_exp(k_in: int) -> int:
-    return int(round(0.5 * math.log2(3.0 / k_in))) - 1
+OUT_PROJ = ("w_o", "w_2")
+
+
+def weight_exp(k_in: int, kind: str = "w_qkv") -> int:
+    """Round half to even (Python round); the CUDA side uses nearbyint."""
+    return int(round(0.5 * math.log2(3.0 / k_in))) - (2 if kind in OUT_PROJ else 1)
 
 
 def c0_values(seed: int, tensor_id: int, idx: np.ndarray, exp: int) -> np.ndarray:
@@ -113,7 +119,7 @@ def layer_tensor(cfg, seed: int, layer: int, kind: str, cols=None, rows=None) ->
         r = np.arange(K, dtype=np.uint64) if rows is None else np.asarray(rows, dtype=np.uint64)
         c = np.arange(N, dtype=np.uint64) if cols is None else np.asarray(cols, dtype=np.uint64)
         idx = r[:, None] * np.uint64(N) + c[None, :]
-        return c0_values(seed, tid, idx, weight_exp(K))
+        return c0_values(seed, tid, idx, weight_exp(K, kind))
     n = shape[0]
     idx = np.arange(n, dtype=np.uint64) if cols is None else np.asarray(cols, dtype=np.uint64)
     if kind.endswith("_g"):

@@ -83,8 +83,11 @@ double now_s() {
   return ts.tv_sec + ts.tv_nsec * 1e-9;
 }
 
-// weight scale exponent of a GEMM with logical fan-in K (C0): round-half-even
-int weight_exp(int K) { return (int)std::nearbyint(0.5 * std::log2(3.0 / K)) - 1; }
+// weight scale exponent of a GEMM with logical fan-in K (C0): round-half-even;
+// output projections (W_o, W_2) get one more halving.
+int weight_exp(int K, bool out_proj = false) {
+  return (int)std::nearbyint(0.5 * std::log2(3.0 / K)) - (out_proj ? 2 : 1);
+}
 constexpr int BIAS_EXP = -6, EMB_EXP = -3;
 constexpr uint64_t GID_ETOK = 0xFFFF00, GID_EPOS = 0xFFFF01, GID_LNFG = 0xFFFF02, GID_LNFB = 0xFFFF03;
 
@@ -758,20 +761,14 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   c->kv = dalloc(c, c->kv_layer_elems * 2 * c->L);
   if (!c->kv) return fail(nullptr, LIGER_ENOMEM, "liger_init: KV pool");
   for (int p = c->n_pages - 1; p >= 0; --p) c->free_pages.push_back(p);
+  // split-K workspace: the maximum over every token count a pass can have
   size_t ws = 0;
-  for (int M : {Mmax, B}) {
+  for (int M = 1; M <= Mmax; ++M) {
     ws = std::max(ws, gemm_workspace_bytes(M, 3 * c->hl, c->h));
     ws = std::max(ws, gemm_workspace_bytes(M, c->h, c->hl));
     ws = std::max(ws, gemm_workspace_bytes(M, c->fl, c->h));
     ws = std::max(ws, gemm_workspace_bytes(M, c->h, c->fl));
-    ws = std::max(ws, gemm_workspace_bytes(M, c->Vl, c->h));
-  }
-  // the decode GEMMs at every M <= B
-  for (int M = 1; M <= B; ++M) {
-    ws = std::max(ws, gemm_workspace_bytes(M, 3 * c->hl, c->h));
-    ws = std::max(ws, gemm_workspace_bytes(M, c->fl, c->h));
-    ws = std::max(ws, gemm_workspace_bytes(M, c->h, c->fl));
-    ws = std::max(ws, gemm_workspace_bytes(M, c->Vl, c->h));
+    if (M <= B) ws = std::max(ws, gemm_workspace_bytes(M, c->Vl, c->h));
   }
   c->slots.resize(nslots);
   for (auto& S : c->slots) {
@@ -841,13 +838,13 @@ int liger_load_layer(liger_ctx* c, int l, uint64_t seed) {
                        0, st));
   }
   // W_o logical [h_in, h_out]; local [h_out, hl_in]: (n, k) -> ((r*hl + k) * h + n)
-  CKR(c0_fill_launch(W.w_o, (int)h, (int)hl, hl, seed, tid + 2, 0, r * hl, 1, h, weight_exp((int)h), 0, st));
+  CKR(c0_fill_launch(W.w_o, (int)h, (int)hl, hl, seed, tid + 2, 0, r * hl, 1, h, weight_exp((int)h, true), 0, st));
   CKR(c0_fill_launch(W.b_o, 1, (int)h, h, seed, tid + 3, 0, 0, 0, 1, BIAS_EXP, 0, st));
   // W_1 logical [h, f]; local [fl, h]: (n, k) -> (k * f + r*fl + n)
   CKR(c0_fill_launch(W.w_1, (int)fl, (int)h, h, seed, tid + 4, r * fl, 0, 1, f, weight_exp((int)h), 0, st));
   CKR(c0_fill_launch(W.b_1, 1, (int)fl, fl, seed, tid + 5, 0, r * fl, 0, 1, BIAS_EXP, 0, st));
   // W_2 logical [f, h]; local [h, fl]: (n, k) -> ((r*fl + k) * h + n)
-  CKR(c0_fill_launch(W.w_2, (int)h, (int)fl, fl, seed, tid + 6, 0, r * fl, 1, h, weight_exp((int)f), 0, st));
+  CKR(c0_fill_launch(W.w_2, (int)h, (int)fl, fl, seed, tid + 6, 0, r * fl, 1, h, weight_exp((int)f, true), 0, st));
   CKR(c0_fill_launch(W.b_2, 1, (int)h, h, seed, tid + 7, 0, 0, 0, 1, BIAS_EXP, 0, st));
   CKR(c0_fill_launch(W.g1, 1, (int)h, h, seed, tid + 8, 0, 0, 0, 1, 0, 1, st));
   CKR(c0_fill_launch(W.be1, 1, (int)h, h, seed, tid + 9, 0, 0, 0, 1, 0, 2, st));

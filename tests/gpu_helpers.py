@@ -42,13 +42,13 @@ def shard_weights_device(L, cfg, seed, layer, t, r, dev="cuda"):
         L.c0_fill(W["b_qkv"][:, s * hl:(s + 1) * hl], seed=seed, tensor_id=tid + KIND["b_qkv"],
                   col_off=s * h + r * hl, idx_row_stride=0, exp=BIAS_EXP)
     L.c0_fill(W["w_o"], seed=seed, tensor_id=tid + KIND["w_o"], col_off=r * hl, idx_row_stride=1,
-              idx_col_stride=h, exp=weight_exp(h))
+              idx_col_stride=h, exp=weight_exp(h, "w_o"))
     L.c0_fill(W["b_o"], seed=seed, tensor_id=tid + KIND["b_o"], idx_row_stride=0, exp=BIAS_EXP)
     L.c0_fill(W["w_1"], seed=seed, tensor_id=tid + KIND["w_1"], row_off=r * fl, idx_row_stride=1,
               idx_col_stride=f, exp=weight_exp(h))
     L.c0_fill(W["b_1"], seed=seed, tensor_id=tid + KIND["b_1"], col_off=r * fl, idx_row_stride=0, exp=BIAS_EXP)
     L.c0_fill(W["w_2"], seed=seed, tensor_id=tid + KIND["w_2"], col_off=r * fl, idx_row_stride=1,
-              idx_col_stride=h, exp=weight_exp(f))
+              idx_col_stride=h, exp=weight_exp(f, "w_2"))
     L.c0_fill(W["b_2"], seed=seed, tensor_id=tid + KIND["b_2"], idx_row_stride=0, exp=BIAS_EXP)
     for k, kind in (("ln1_g", 1), ("ln1_b", 2), ("ln2_g", 1), ("ln2_b", 2)):
         L.c0_fill(W[k], seed=seed, tensor_id=tid + KIND[k], idx_row_stride=0, kind=kind)
