@@ -227,12 +227,28 @@ int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* 
 }
 
 // ================================================================== decode
-constexpr int DC_CHUNK = 256;
+// CTA = (head, sequence, chunk of DC_CHUNK positions).  Phase 1: warp w scores
+// positions [w*32, w*32+32) of the chunk; a token's K row (d bf16) is spread over
+// LPT = d/8 lanes (16 B each) and every lane issues all of its K loads before the
+// first shuffle reduction (memory-level parallelism instead of a latency chain).
+// Phase 2: thread (slot, vec) accumulates p_t * V[t, vec*8 .. +8] over the
+// positions t = slot (mod SLOTS), again loading all V vectors first.
+constexpr int DC_CHUNK = 128;
 constexpr int DC_THREADS = 128;
 
 size_t attn_decode_workspace_bytes(int b, int heads, int d, int ctx) {
   const int ns = (ctx + DC_CHUNK - 1) / DC_CHUNK;
   return ATTN_COUNTER_BYTES + (size_t)b * heads * ns * (d + 2) * sizeof(float);
+}
+
+__device__ __forceinline__ void bf16x8_to_f32(const uint4& v, float* f) {
+  const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&v);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    float2 t = __bfloat1622float2(h[i]);
+    f[2 * i] = t.x;
+    f[2 * i + 1] = t.y;
+  }
 }
 
 template <int D>
@@ -242,13 +258,17 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
                                                                  const int32_t* __restrict__ page_table,
                                                                  int max_pages, int pos, int heads, float* ws,
                                                                  int* counters) {
-  constexpr int LPT = D / 8;          // lanes per token (8 bf16 each)
-  constexpr int TPW = 32 / LPT;       // tokens per warp step
+  constexpr int LPT = D / 8;            // lanes per token
+  constexpr int TPW = 32 / LPT;         // tokens per warp step
+  constexpr int STEPS = 32 / TPW;       // steps for the warp's 32 positions
   constexpr int NVEC = D / 8;
   constexpr int SLOTS = DC_THREADS / NVEC;
+  constexpr int PER = DC_CHUNK / SLOTS; // positions per thread in phase 2
+  constexpr int NPG = DC_CHUNK / KVB;   // pages per chunk
   __shared__ float sc[DC_CHUNK];
   __shared__ float red[DC_THREADS / 32];
   __shared__ float part[SLOTS][D];
+  __shared__ int pg[NPG];
   __shared__ int last;
 
   const int head = blockIdx.x, bi = blockIdx.y, sp = blockIdx.z, nsp = gridDim.z;
@@ -262,81 +282,91 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   const __nv_bfloat16* vnew = row + (int64_t)2 * heads * D + head * D;
   const int32_t* pt = page_table + (int64_t)bi * max_pages;
 
+  if (tid < NPG) pg[tid] = (t0 + tid * KVB < ctx) ? pt[(t0 >> 4) + tid] : 0;
   if (sp == nsp - 1 && tid < 2 * NVEC) {   // append the new token's K/V (position pos)
     const int kv = tid / NVEC, c = (tid % NVEC) * 8;
     const int page = pt[pos / KVB];
     *reinterpret_cast<uint4*>(kv_pool + kv_off(page, kv, heads, head, pos % KVB, D) + c) =
         *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
   }
-
-  // pass 1: scores
   float qf[8];
   {
-    const int c = (lane % LPT) * 8;
-    uint4 qv = *reinterpret_cast<const uint4*>(qp + c);
-    const __nv_bfloat162* qh = reinterpret_cast<const __nv_bfloat162*>(&qv);
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      float2 f = __bfloat1622float2(qh[i]);
-      qf[2 * i] = f.x;
-      qf[2 * i + 1] = f.y;
-    }
+    uint4 qv = *reinterpret_cast<const uint4*>(qp + (lane % LPT) * 8);
+    bf16x8_to_f32(qv, qf);
   }
-  for (int tb = t0 + warp * TPW; tb < t1; tb += 4 * TPW) {
-    const int t = tb + lane / LPT;
-    float dot = 0.f;
-    if (t < t1) {
-      const int c = (lane % LPT) * 8;
-      const __nv_bfloat16* kp =
-          (t == pos) ? knew + c : kv_pool + kv_off(pt[t / KVB], 0, heads, head, t % KVB, D) + c;
-      uint4 kv = *reinterpret_cast<const uint4*>(kp);
-      const __nv_bfloat162* kh = reinterpret_cast<const __nv_bfloat162*>(&kv);
+  __syncthreads();
+
+  // ---- phase 1: scores for positions [t0 + warp*32, +32)
+  {
+    const int c = (lane % LPT) * 8;
+    uint4 kr[STEPS];
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        float2 f = __bfloat1622float2(kh[i]);
-        dot += qf[2 * i] * f.x + qf[2 * i + 1] * f.y;
+    for (int st = 0; st < STEPS; ++st) {
+      const int t = t0 + warp * 32 + st * TPW + lane / LPT;
+      kr[st] = make_uint4(0, 0, 0, 0);
+      if (t < t1) {
+        const __nv_bfloat16* kp =
+            (t == pos) ? knew + c : kv_pool + kv_off(pg[(t - t0) >> 4], 0, heads, head, t % KVB, D) + c;
+        kr[st] = *reinterpret_cast<const uint4*>(kp);
       }
     }
 #pragma unroll
-    for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
-    if (t < t1 && (lane % LPT) == 0) sc[t - t0] = dot;
+    for (int st = 0; st < STEPS; ++st) {
+      float f[8];
+      bf16x8_to_f32(kr[st], f);
+      float dot = 0.f;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) dot += qf[i] * f[i];
+#pragma unroll
+      for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
+      const int t = t0 + warp * 32 + st * TPW + lane / LPT;
+      if (t < t1 && (lane % LPT) == 0) sc[t - t0] = dot;
+    }
   }
   __syncthreads();
   const int n = t1 - t0;
-  float mx = -INFINITY;
-  for (int i = tid; i < n; i += DC_THREADS) mx = fmaxf(mx, sc[i]);
+  float mx = (tid < n) ? sc[tid] : -INFINITY;
 #pragma unroll
   for (int off = 16; off > 0; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
   if (lane == 0) red[warp] = mx;
   __syncthreads();
   mx = fmaxf(fmaxf(red[0], red[1]), fmaxf(red[2], red[3]));
   __syncthreads();
-  float sum = 0.f;
-  for (int i = tid; i < n; i += DC_THREADS) {
-    const float p = __expf(sc[i] - mx);
-    sc[i] = p;
-    sum += p;
+  float p_t = 0.f;
+  if (tid < n) {
+    p_t = __expf(sc[tid] - mx);
+    sc[tid] = p_t;
   }
+  float sum = p_t;
 #pragma unroll
   for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
   if (lane == 0) red[warp] = sum;
   __syncthreads();
   const float l = red[0] + red[1] + red[2] + red[3];
 
-  // pass 2: o = sum_t p_t v_t ; thread = (slot, vector)
+  // ---- phase 2: o = sum_t p_t v_t
   const int vec = tid % NVEC, slot = tid / NVEC;
   float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-  for (int t = t0 + slot; t < t1; t += SLOTS) {
-    const __nv_bfloat16* vp =
-        (t == pos) ? vnew + vec * 8 : kv_pool + kv_off(pt[t / KVB], 1, heads, head, t % KVB, D) + vec * 8;
-    uint4 vv = *reinterpret_cast<const uint4*>(vp);
-    const __nv_bfloat162* vh = reinterpret_cast<const __nv_bfloat162*>(&vv);
-    const float p = sc[t - t0];
+  {
+    uint4 vr[PER];
 #pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      float2 f = __bfloat1622float2(vh[i]);
-      acc[2 * i] += p * f.x;
-      acc[2 * i + 1] += p * f.y;
+    for (int i = 0; i < PER; ++i) {
+      const int t = t0 + slot + i * SLOTS;
+      vr[i] = make_uint4(0, 0, 0, 0);
+      if (t < t1) {
+        const __nv_bfloat16* vp =
+            (t == pos) ? vnew + vec * 8 : kv_pool + kv_off(pg[(t - t0) >> 4], 1, heads, head, t % KVB, D) + vec * 8;
+        vr[i] = *reinterpret_cast<const uint4*>(vp);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < PER; ++i) {
+      const int t = t0 + slot + i * SLOTS;
+      const float pw = (t < t1) ? sc[t - t0] : 0.f;
+      float f[8];
+      bf16x8_to_f32(vr[i], f);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] += pw * f[e];
     }
   }
 #pragma unroll
@@ -346,16 +376,18 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   if (nsp == 1) {
     for (int e = tid; e < D; e += DC_THREADS) {
       float a = 0.f;
+#pragma unroll
       for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
       o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / l);
     }
     return;
   }
-  // split: write partial (m, l, acc[D]); the last CTA merges in split order
+  // split: write partial (m, l, acc[D]); the last CTA merges in chunk order
   const int64_t unit = (int64_t)bi * heads + head;
   float* wp = ws + (unit * nsp + sp) * (D + 2);
   for (int e = tid; e < D; e += DC_THREADS) {
     float a = 0.f;
+#pragma unroll
     for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
     wp[e] = a;
   }

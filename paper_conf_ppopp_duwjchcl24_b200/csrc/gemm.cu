@@ -46,6 +46,8 @@ struct GemmParams {
   int kc, splits;
   int bn;
   int stages;
+  int n_tiles, m_tiles;
+  int units;            // n_tiles * m_tiles * splits
   const __nv_bfloat16* bias;
   int act;
   int scale_cols;
@@ -72,6 +74,22 @@ __device__ __forceinline__ void epi_store(const GemmParams& p, int m, int n, flo
     reinterpret_cast<__nv_bfloat16*>(p.out)[(int64_t)m * p.ldo + n] = __float2bfloat16_rn(v);
 }
 
+// Work unit u -> (n tile, m tile, K chunk).  m is the inner tile index so that the
+// CTAs running concurrently (units i, i+G, ...) share weight tiles through L2;
+// chunks of one tile are adjacent.
+struct Unit {
+  int nt, mt, z;
+};
+__device__ __forceinline__ Unit unit_of(const GemmParams& p, int u) {
+  Unit r;
+  r.z = u % p.splits;
+  const int t = u / p.splits;
+  r.mt = t % p.m_tiles;
+  r.nt = t / p.m_tiles;
+  return r;
+}
+
+// Persistent: one CTA per SM, CTA i processes units i, i + G, i + 2G, ...
 __global__ void __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmParams p) {
@@ -84,26 +102,26 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   uint64_t* bars = reinterpret_cast<uint64_t*>(smB + (size_t)S * B_BYTES);
   uint64_t* full = bars;
   uint64_t* empty = bars + S;
-  uint64_t* tmem_full = bars + 2 * S;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 1);
+  uint64_t* tmem_full = bars + 2 * S;       // [2]
+  uint64_t* tmem_empty = bars + 2 * S + 2;  // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 4);
   int* last_flag = reinterpret_cast<int*>(tmem_slot + 1);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
-  const int n_base = p.n0 + blockIdx.x * BM;
-  const int m_base = blockIdx.y * p.bn;
-  const int z = blockIdx.z;
-  const int k0 = z * p.kc;
-  const int k1 = min(p.K, k0 + p.kc);
-  const int nkb = (k1 - k0 + BK - 1) / BK;
-  const uint32_t tmem_cols = p.bn <= 32 ? 32 : (p.bn <= 64 ? 64 : (p.bn <= 128 ? 128 : 256));
+  const int G = gridDim.x;
+  const uint32_t acc_cols = p.bn <= 32 ? 32 : (p.bn <= 64 ? 64 : (p.bn <= 128 ? 128 : 256));
+  const uint32_t tmem_cols = 2 * acc_cols;
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);
       mbar_init(&empty[i], 1);
     }
-    mbar_init(tmem_full, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&tmem_full[i], 1);
+      mbar_init(&tmem_empty[i], 4);   // one arrive per epilogue warp
+    }
     fence_barrier_init();
   }
   if (warp == 0 && lane == 0) {
@@ -118,15 +136,22 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
 
   if (warp == 0) {
     if (lane == 0) {
-      const uint64_t pol_w = policy_evict_first();   // weights: streamed once
-      for (int kb = 0; kb < nkb; ++kb) {
-        const int s = kb % S;
-        const uint32_t ph = (kb / S) & 1;
-        mbar_wait(&empty[s], ph ^ 1);
-        mbar_arrive_expect_tx(&full[s], A_BYTES + B_BYTES);
-        const int kk = k0 + kb * BK;
-        tma_load_2d_hint(smA + (size_t)s * A_BYTES, &tmA, &full[s], kk, n_base, pol_w);
-        tma_load_2d(smB + (size_t)s * B_BYTES, &tmB, &full[s], kk, m_base);
+      const uint64_t pol_w = policy_evict_first();   // weights: streamed once per tile
+      int it = 0;
+      for (int u = blockIdx.x; u < p.units; u += G) {
+        const Unit w = unit_of(p, u);
+        const int k0 = w.z * p.kc;
+        const int nkb = (min(p.K, k0 + p.kc) - k0 + BK - 1) / BK;
+        const int n_base = p.n0 + w.nt * BM, m_base = w.mt * p.bn;
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const int s = it % S;
+          const uint32_t ph = (it / S) & 1;
+          mbar_wait(&empty[s], ph ^ 1);
+          mbar_arrive_expect_tx(&full[s], A_BYTES + B_BYTES);
+          const int kk = k0 + kb * BK;
+          tma_load_2d_hint(smA + (size_t)s * A_BYTES, &tmA, &full[s], kk, n_base, pol_w);
+          tma_load_2d(smB + (size_t)s * B_BYTES, &tmB, &full[s], kk, m_base);
+        }
       }
     }
   } else if (warp == 1) {
@@ -134,81 +159,106 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       // kind::f16 instruction descriptor: D=f32, A=B=bf16, both K-major, N=bn, M=128.
       const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(p.bn >> 3) << 17) |
                              ((uint32_t)(BM >> 4) << 24);
-      for (int kb = 0; kb < nkb; ++kb) {
-        const int s = kb % S;
-        const uint32_t ph = (kb / S) & 1;
-        mbar_wait(&full[s], ph);
+      int it = 0, lu = 0;
+      for (int u = blockIdx.x; u < p.units; u += G, ++lu) {
+        const Unit w = unit_of(p, u);
+        const int k0 = w.z * p.kc;
+        const int nkb = (min(p.K, k0 + p.kc) - k0 + BK - 1) / BK;
+        const int acc = lu & 1;
+        const uint32_t acc_ph = (lu >> 1) & 1;
+        mbar_wait(&tmem_empty[acc], acc_ph ^ 1);
         tc_fence_after();
-        const uint64_t adesc = umma_desc_sw128(smem_u32(smA + (size_t)s * A_BYTES));
-        const uint64_t bdesc = umma_desc_sw128(smem_u32(smB + (size_t)s * B_BYTES));
+        const uint32_t tacc = tmem_base + (uint32_t)acc * acc_cols;
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const int s = it % S;
+          const uint32_t ph = (it / S) & 1;
+          mbar_wait(&full[s], ph);
+          tc_fence_after();
+          const uint64_t adesc = umma_desc_sw128(smem_u32(smA + (size_t)s * A_BYTES));
+          const uint64_t bdesc = umma_desc_sw128(smem_u32(smB + (size_t)s * B_BYTES));
 #pragma unroll
-        for (int k = 0; k < BK / 16; ++k)
-          umma_bf16(tmem_base, adesc + 2 * k, bdesc + 2 * k, idesc, (kb | k) != 0);
-        umma_commit(&empty[s]);
+          for (int k = 0; k < BK / 16; ++k)
+            umma_bf16(tacc, adesc + 2 * k, bdesc + 2 * k, idesc, (kb | k) != 0);
+          umma_commit(&empty[s]);
+        }
+        umma_commit(&tmem_full[acc]);
       }
-      umma_commit(tmem_full);
     }
   } else {
     // ---------------- epilogue: warps 2..5 own TMEM lane quarters (warp % 4)
     const int q = warp & 3;
     const int row = q * 32 + lane;
-    const int n = n_base + row;
-    const bool nval = (n < p.n1) && (n < p.N);
-    const float bias_v = (p.bias != nullptr && nval) ? __bfloat162float(p.bias[n]) : 0.0f;
     const int slice_w = p.n1 - p.n0;
-    mbar_wait(tmem_full, 0);
-    tc_fence_after();
-    for (int c0 = 0; c0 < p.bn; c0 += 16) {
-      uint32_t r[16];
-      tmem_ld_32x32b_x16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)c0, r);
-      tmem_ld_wait();
-      if (nval) {
-#pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const int m = m_base + c0 + j;
-          if (m < p.M) {
-            const float v = __uint_as_float(r[j]);
-            if (p.splits == 1)
-              epi_store(p, m, n, epi_apply(p, v, n, bias_v));
-            else
-              p.ws[((int64_t)z * p.M + m) * slice_w + (n - p.n0)] = v;
-          }
-        }
-      }
-    }
-    if (p.splits > 1) {
-      // Deterministic split-K: the last CTA of this tile sums the partials in
-      // z order 0..splits-1 (independent of which CTA finishes last).
-      __threadfence();
-      named_bar_sync(1, 128);
-      const int tile_id = blockIdx.y * gridDim.x + blockIdx.x;
-      if (threadIdx.x == 64) {
-        const int prev = atomicAdd(&p.counters[tile_id], 1);
-        *last_flag = (prev == p.splits - 1);
-      }
-      named_bar_sync(1, 128);
-      if (*last_flag) {
-        __threadfence();
+    int lu = 0;
+    for (int u = blockIdx.x; u < p.units; u += G, ++lu) {
+      const Unit w = unit_of(p, u);
+      const int n_base = p.n0 + w.nt * BM, m_base = w.mt * p.bn;
+      const int n = n_base + row;
+      const bool nval = (n < p.n1) && (n < p.N);
+      const float bias_v = (p.bias != nullptr && nval) ? __bfloat162float(p.bias[n]) : 0.0f;
+      const int acc = lu & 1;
+      const uint32_t acc_ph = (lu >> 1) & 1;
+      const int mcount = min(p.bn, p.M - m_base);
+      mbar_wait(&tmem_full[acc], acc_ph);
+      tc_fence_after();
+      const uint32_t tacc = tmem_base + (uint32_t)acc * acc_cols + ((uint32_t)(q * 32) << 16);
+      for (int c0 = 0; c0 < p.bn; c0 += 16) {
+        if (c0 >= mcount) break;   // warp-uniform
+        uint32_t r[16];
+        tmem_ld_32x32b_x16(tacc + (uint32_t)c0, r);
+        tmem_ld_wait();
         if (nval) {
-          const int mcount = min(p.bn, p.M - m_base);
-          for (int c0 = 0; c0 < mcount; c0 += 16) {
-            float acc[16];
 #pragma unroll
-            for (int j = 0; j < 16; ++j) acc[j] = 0.0f;
-            for (int zz = 0; zz < p.splits; ++zz) {
-              const float* src = p.ws + ((int64_t)zz * p.M + m_base + c0) * slice_w + (n - p.n0);
-              float v[16];
-#pragma unroll
-              for (int j = 0; j < 16; ++j) v[j] = (c0 + j < mcount) ? __ldcg(src + (int64_t)j * slice_w) : 0.0f;
-#pragma unroll
-              for (int j = 0; j < 16; ++j) acc[j] += v[j];
+          for (int j = 0; j < 16; ++j) {
+            if (c0 + j < mcount) {
+              const int m = m_base + c0 + j;
+              const float v = __uint_as_float(r[j]);
+              if (p.splits == 1)
+                epi_store(p, m, n, epi_apply(p, v, n, bias_v));
+              else
+                p.ws[((int64_t)w.z * p.M + m) * slice_w + (n - p.n0)] = v;
             }
-#pragma unroll
-            for (int j = 0; j < 16; ++j)
-              if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, acc[j], n, bias_v));
           }
         }
-        if (threadIdx.x == 64) p.counters[tile_id] = 0;
+      }
+      // accumulator drained: hand the TMEM buffer back to the MMA warp
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tmem_empty[acc]);
+      if (p.splits > 1) {
+        // Deterministic split-K: the last CTA to finish a tile's chunks sums the
+        // partials in chunk order 0..splits-1 (independent of who is last).
+        __threadfence();
+        named_bar_sync(1, 128);
+        const int tile_id = w.nt * p.m_tiles + w.mt;
+        if (threadIdx.x == 64) {
+          const int prev = atomicAdd(&p.counters[tile_id], 1);
+          *last_flag = (prev == p.splits - 1);
+        }
+        named_bar_sync(1, 128);
+        if (*last_flag) {
+          __threadfence();
+          if (nval) {
+            for (int c0 = 0; c0 < mcount; c0 += 16) {
+              float accv[16];
+#pragma unroll
+              for (int j = 0; j < 16; ++j) accv[j] = 0.0f;
+              for (int zz = 0; zz < p.splits; ++zz) {
+                const float* src = p.ws + ((int64_t)zz * p.M + m_base + c0) * slice_w + (n - p.n0);
+                float v[16];
+#pragma unroll
+                for (int j = 0; j < 16; ++j) v[j] = (c0 + j < mcount) ? __ldcg(src + (int64_t)j * slice_w) : 0.0f;
+#pragma unroll
+                for (int j = 0; j < 16; ++j) accv[j] += v[j];
+              }
+#pragma unroll
+              for (int j = 0; j < 16; ++j)
+                if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, accv[j], n, bias_v));
+            }
+          }
+          if (threadIdx.x == 64) p.counters[tile_id] = 0;
+        }
+        named_bar_sync(1, 128);   // last_flag is reused by the next unit
       }
     }
   }
@@ -295,6 +345,17 @@ void gemm_forget_pointer_range(const void* base, size_t bytes) {
   }
 }
 
+static int num_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
 // Tiling policy: a function of (M, K) only (bit-exact decomposition).
 GemmPlan gemm_plan(int M, int K) {
   GemmPlan pl{};
@@ -305,7 +366,7 @@ GemmPlan gemm_plan(int M, int K) {
   pl.bn = bn;
   pl.m_tiles = mt;
   int kc;
-  if (M <= 64) kc = 1024;
+  if (M <= 64) kc = 512;
   else if (M <= 512) kc = 2048;
   else kc = K;
   kc = (kc + BK - 1) / BK * BK;
@@ -314,7 +375,7 @@ GemmPlan gemm_plan(int M, int K) {
   pl.splits = (K + kc - 1) / kc;
   const int stage_bytes = A_BYTES + bn * BK * 2;
   int st = (MAX_SMEM - 1024 - 256) / stage_bytes;
-  if (st > 10) st = 10;
+  if (st > 12) st = 12;
   pl.stages = st;
   pl.smem = 1024 + st * stage_bytes + 256;
   return pl;
@@ -354,7 +415,10 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.out = a.out; p.ldo = a.ldo; p.out_f32 = a.out_f32;
   p.counters = reinterpret_cast<int*>(a.workspace);
   p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
-  dim3 grid(ntiles, pl.m_tiles, pl.splits);
+  p.n_tiles = ntiles;
+  p.m_tiles = pl.m_tiles;
+  p.units = ntiles * pl.m_tiles * pl.splits;
+  const int grid = p.units < num_sms() ? p.units : num_sms();
   gemm_tc_kernel<<<grid, GEMM_THREADS, pl.smem, stream>>>(tA, tB, p);
   return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
 }

@@ -43,7 +43,9 @@ __device__ __forceinline__ float block_sum(float v, float* red) {
   return s;
 }
 
-// One CTA per output row.  MAXV = max 8-element vectors per thread.
+// One CTA per output row; each thread owns up to MAXV 8-element vectors.  All
+// global loads of a row (x, add, bias, gamma, beta) are issued before any use so
+// the kernel pays one memory round trip (decode rows are latency-bound).
 template <int NT, int MAXV>
 __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x, const bf16x8* __restrict__ add,
                                                     const bf16x8* __restrict__ add_bias, bf16x8* x_out,
@@ -54,22 +56,34 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
   const int nv = h >> 3;
   const int64_t in_row = (int64_t)blockIdx.x * in_row_step + in_row_off;
   const bf16x8* xr = x + in_row * nv;
+  bf16x8 vx[MAXV], va[MAXV], vb[MAXV], vg[MAXV], vbe[MAXV];
+#pragma unroll
+  for (int j = 0; j < MAXV; ++j) {
+    const int v = threadIdx.x + j * NT;
+    if (v < nv) {
+      vx[j] = xr[v];
+      if (add) va[j] = add[in_row * nv + v];
+      if (add_bias) vb[j] = add_bias[v];
+      vg[j] = gamma[v];
+      vbe[j] = beta[v];
+    }
+  }
   float r[MAXV][8];
   float s = 0.f;
 #pragma unroll
   for (int j = 0; j < MAXV; ++j) {
     const int v = threadIdx.x + j * NT;
     if (v < nv) {
-      unpack8(xr[v], r[j]);
+      unpack8(vx[j], r[j]);
       if (add) {
         float a[8];
-        unpack8(add[in_row * nv + v], a);
+        unpack8(va[j], a);
 #pragma unroll
         for (int e = 0; e < 8; ++e) r[j][e] += a[e];
       }
       if (add_bias) {
         float a[8];
-        unpack8(add_bias[v], a);
+        unpack8(vb[j], a);
 #pragma unroll
         for (int e = 0; e < 8; ++e) r[j][e] += a[e];
       }
@@ -100,8 +114,8 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
     const int v = threadIdx.x + j * NT;
     if (v < nv) {
       float g[8], b[8], o[8];
-      unpack8(gamma[v], g);
-      unpack8(beta[v], b);
+      unpack8(vg[j], g);
+      unpack8(vbe[j], b);
 #pragma unroll
       for (int e = 0; e < 8; ++e) o[e] = (r[j][e] - mean) * rstd * g[e] + b[e];
       y[(int64_t)blockIdx.x * nv + v] = pack8(o);
@@ -113,21 +127,19 @@ int add_layernorm_launch(const void* x, const void* add, const void* add_bias, v
                          const void* gamma, const void* beta, int rows, int h, int in_row_step, int in_row_off,
                          float eps, cudaStream_t stream) {
   if (rows <= 0) return 0;
-  if (h % 8 || h > 8 * 256 * 8 || !x || !y || !gamma || !beta) return LIGER_EINVAL;
+  if (h % 8 || h > 16384 || !x || !y || !gamma || !beta) return LIGER_EINVAL;
   const bf16x8* X = (const bf16x8*)x;
   const bf16x8* A = (const bf16x8*)add;
   const bf16x8* AB = (const bf16x8*)add_bias;
   const int nv = h / 8;
-  if (nv <= 128) {
-    add_ln_kernel<128, 1><<<rows, 128, 0, stream>>>(X, A, AB, (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma,
-                                                    (const bf16x8*)beta, h, in_row_step, in_row_off, eps);
-  } else if (nv <= 256 * 2) {
-    add_ln_kernel<256, 2><<<rows, 256, 0, stream>>>(X, A, AB, (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma,
-                                                    (const bf16x8*)beta, h, in_row_step, in_row_off, eps);
-  } else {
-    add_ln_kernel<256, 8><<<rows, 256, 0, stream>>>(X, A, AB, (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma,
-                                                    (const bf16x8*)beta, h, in_row_step, in_row_off, eps);
-  }
+#define LIGER_LN(NT, MV)                                                                                   \
+  add_ln_kernel<NT, MV><<<rows, NT, 0, stream>>>(X, A, AB, (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma, \
+                                                 (const bf16x8*)beta, h, in_row_step, in_row_off, eps)
+  if (nv <= 128) LIGER_LN(128, 1);
+  else if (nv <= 512) LIGER_LN(128, 4);
+  else if (nv <= 1024) LIGER_LN(256, 4);
+  else LIGER_LN(512, 4);
+#undef LIGER_LN
   return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
 }
 
