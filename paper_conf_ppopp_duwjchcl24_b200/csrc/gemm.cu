@@ -40,6 +40,17 @@ constexpr int A_BYTES = BM * BK * 2;
 constexpr int GEMM_THREADS = 192;
 constexpr int MAX_SMEM = 227 * 1024;
 
+static int num_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
 struct GemmParams {
   int M, N, K;
   int n0, n1;
@@ -188,7 +199,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     // ---------------- epilogue: warps 2..5 own TMEM lane quarters (warp % 4)
     const int q = warp & 3;
     const int row = q * 32 + lane;
-    const int slice_w = p.n1 - p.n0;
+    const int tiles = p.n_tiles * p.m_tiles;
     int lu = 0;
     for (int u = blockIdx.x; u < p.units; u += G, ++lu) {
       const Unit w = unit_of(p, u);
@@ -199,6 +210,10 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       const int acc = lu & 1;
       const uint32_t acc_ph = (lu >> 1) & 1;
       const int mcount = min(p.bn, p.M - m_base);
+      const int tile_id = w.nt * p.m_tiles + w.mt;
+      // fp32 partial of (chunk z, tile): [128 rows][bn] row-major, 16-byte vectors
+      float* my_ws = p.splits > 1 ? p.ws + ((int64_t)w.z * tiles + tile_id) * (BM * p.bn) + (int64_t)row * p.bn
+                                  : nullptr;
       mbar_wait(&tmem_full[acc], acc_ph);
       tc_fence_after();
       const uint32_t tacc = tmem_base + (uint32_t)acc * acc_cols + ((uint32_t)(q * 32) << 16);
@@ -207,18 +222,19 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         uint32_t r[16];
         tmem_ld_32x32b_x16(tacc + (uint32_t)c0, r);
         tmem_ld_wait();
-        if (nval) {
+        if (p.splits == 1) {
+          if (nval) {
 #pragma unroll
-          for (int j = 0; j < 16; ++j) {
-            if (c0 + j < mcount) {
-              const int m = m_base + c0 + j;
-              const float v = __uint_as_float(r[j]);
-              if (p.splits == 1)
-                epi_store(p, m, n, epi_apply(p, v, n, bias_v));
-              else
-                p.ws[((int64_t)w.z * p.M + m) * slice_w + (n - p.n0)] = v;
-            }
+            for (int j = 0; j < 16; ++j)
+              if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, __uint_as_float(r[j]), n, bias_v));
           }
+        } else {
+          float4* dst = reinterpret_cast<float4*>(my_ws + c0);
+#pragma unroll
+          for (int v = 0; v < 4; ++v)
+            if (c0 + 4 * v < mcount)
+              __stcg(dst + v, make_float4(__uint_as_float(r[4 * v]), __uint_as_float(r[4 * v + 1]),
+                                          __uint_as_float(r[4 * v + 2]), __uint_as_float(r[4 * v + 3])));
         }
       }
       // accumulator drained: hand the TMEM buffer back to the MMA warp
@@ -228,32 +244,50 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       if (p.splits > 1) {
         // Deterministic split-K: the last CTA to finish a tile's chunks sums the
         // partials in chunk order 0..splits-1 (independent of who is last).
-        __threadfence();
+        // Release: CTA barrier, then one gpu-scope fence + atomic (cumulative).
         named_bar_sync(1, 128);
-        const int tile_id = w.nt * p.m_tiles + w.mt;
         if (threadIdx.x == 64) {
+          __threadfence();
           const int prev = atomicAdd(&p.counters[tile_id], 1);
           *last_flag = (prev == p.splits - 1);
+          if (*last_flag) __threadfence();   // acquire side
         }
         named_bar_sync(1, 128);
         if (*last_flag) {
-          __threadfence();
           if (nval) {
+            const float* base = p.ws + (int64_t)tile_id * (BM * p.bn) + (int64_t)row * p.bn;
+            const int64_t zstride = (int64_t)tiles * (BM * p.bn);
             for (int c0 = 0; c0 < mcount; c0 += 16) {
-              float accv[16];
+              const int nv4 = min(4, (mcount - c0 + 3) / 4);
+              float4 accv[4];
 #pragma unroll
-              for (int j = 0; j < 16; ++j) accv[j] = 0.0f;
-              for (int zz = 0; zz < p.splits; ++zz) {
-                const float* src = p.ws + ((int64_t)zz * p.M + m_base + c0) * slice_w + (n - p.n0);
-                float v[16];
+              for (int v = 0; v < 4; ++v) accv[v] = make_float4(0.f, 0.f, 0.f, 0.f);
+              constexpr int UNR = 4;
+              for (int z0 = 0; z0 < p.splits; z0 += UNR) {
+                float4 ld[UNR][4];
 #pragma unroll
-                for (int j = 0; j < 16; ++j) v[j] = (c0 + j < mcount) ? __ldcg(src + (int64_t)j * slice_w) : 0.0f;
+                for (int zz = 0; zz < UNR; ++zz)
 #pragma unroll
-                for (int j = 0; j < 16; ++j) accv[j] += v[j];
+                  for (int v = 0; v < 4; ++v)
+                    ld[zz][v] = (z0 + zz < p.splits && v < nv4)
+                                    ? __ldcg(reinterpret_cast<const float4*>(base + (z0 + zz) * zstride + c0) + v)
+                                    : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+                for (int zz = 0; zz < UNR; ++zz)
+#pragma unroll
+                  for (int v = 0; v < 4; ++v) {
+                    if (z0 + zz < p.splits) {     // sum in chunk order
+                      accv[v].x += ld[zz][v].x;
+                      accv[v].y += ld[zz][v].y;
+                      accv[v].z += ld[zz][v].z;
+                      accv[v].w += ld[zz][v].w;
+                    }
+                  }
               }
+              const float* a = reinterpret_cast<const float*>(accv);
 #pragma unroll
               for (int j = 0; j < 16; ++j)
-                if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, accv[j], n, bias_v));
+                if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, a[j], n, bias_v));
             }
           }
           if (threadIdx.x == 64) p.counters[tile_id] = 0;
@@ -345,35 +379,50 @@ void gemm_forget_pointer_range(const void* base, size_t bytes) {
   }
 }
 
-static int num_sms() {
-  static int n = 0;
-  if (!n) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-    if (n <= 0) n = 148;
-  }
-  return n;
-}
 
-// Tiling policy: a function of (M, K) only (bit-exact decomposition).
-GemmPlan gemm_plan(int M, int K) {
+// Tiling policy.  A decomposition piece of a GEMM (a column slice [n0, n1)) keeps
+// the full GEMM's (M, N, K), so every per-element quantity -- the token tiling
+// bn, the split-K chunk kc, the K order inside a chunk and the z-order of the
+// split reduction -- is a function of (M, N, K) and identical for the full GEMM
+// and all of its slices: slices are bit-exact.  The split count is chosen by a
+// small cost model that balances units over the SMs.
+GemmPlan gemm_plan(int M, int N, int K) {
   GemmPlan pl{};
-  const int mt = (M + 255) / 256;
-  int bn = (M + mt - 1) / mt;
-  bn = (bn + 15) / 16 * 16;
-  if (bn < 16) bn = 16;
-  pl.bn = bn;
-  pl.m_tiles = mt;
-  int kc;
-  if (M <= 64) kc = 512;
-  else if (M <= 512) kc = 2048;
-  else kc = K;
-  kc = (kc + BK - 1) / BK * BK;
-  if (kc >= K) kc = (K + BK - 1) / BK * BK;
-  pl.kc = kc;
-  pl.splits = (K + kc - 1) / kc;
-  const int stage_bytes = A_BYTES + bn * BK * 2;
+  const int G = num_sms();
+  const int n_tiles = (N + BM - 1) / BM;
+  const int nkb_total = (K + BK - 1) / BK;
+  double best = 1e30;
+  const int bn_opts[3] = {256, 128, 64};
+  for (int bi = 0; bi < 3; ++bi) {
+    const int bcap = bn_opts[bi];
+    if (bi > 0 && M <= bcap) break;           // smaller caps only when they create more tiles
+    const int mt = (M + bcap - 1) / bcap;
+    int bn = (M + mt - 1) / mt;
+    bn = (bn + 15) / 16 * 16;
+    if (bn < 16) bn = 16;
+    const int tiles = n_tiles * mt;
+    // per-k-block cost (cycles): MMA 4 x (2 bn) vs operand load (16 KB + 128 bn B) at ~64 B/clk
+    const double kb_cost = fmax(8.0 * bn, (A_BYTES + 128.0 * bn) / 64.0);
+    const int smax = nkb_total >= 8 ? nkb_total / 4 : 1;   // chunks of >= 256 K
+    for (int sp = 1; sp <= smax; ++sp) {
+      const int kcb = (nkb_total + sp - 1) / sp;            // k-blocks per chunk
+      const int S = (nkb_total + kcb - 1) / kcb;
+      if (S != sp) continue;
+      const int units = tiles * S;
+      const int per_cta = (units + G - 1) / G;
+      double cost = per_cta * (kcb * kb_cost + 600.0);     // + per-unit epilogue hand-off
+      if (S > 1) cost += 1500.0 + 40.0 * S * bn / 16;       // partial write/reduce
+      cost += (tiles > 4096 / 1 && S > 1) ? 1e30 : 0;       // counter capacity
+      if (cost < best - 1e-9) {
+        best = cost;
+        pl.bn = bn;
+        pl.m_tiles = mt;
+        pl.kc = kcb * BK;
+        pl.splits = S;
+      }
+    }
+  }
+  const int stage_bytes = A_BYTES + pl.bn * BK * 2;
   int st = (MAX_SMEM - 1024 - 256) / stage_bytes;
   if (st > 12) st = 12;
   pl.stages = st;
@@ -382,20 +431,21 @@ GemmPlan gemm_plan(int M, int K) {
 }
 
 size_t gemm_workspace_bytes(int M, int N, int K) {
-  GemmPlan pl = gemm_plan(M, K);
+  GemmPlan pl = gemm_plan(M, N, K);
   if (pl.splits <= 1) return GEMM_COUNTER_BYTES;
-  return GEMM_COUNTER_BYTES + (size_t)pl.splits * M * N * sizeof(float);
+  const size_t tiles = (size_t)((N + BM - 1) / BM + 1) * pl.m_tiles;   // +1: unaligned slices
+  return GEMM_COUNTER_BYTES + (size_t)pl.splits * tiles * BM * pl.bn * sizeof(float);
 }
 
 int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (a.M <= 0 || a.n1 <= a.n0) return 0;
   if (a.K <= 0 || a.K % 8 || a.ldx % 8 || a.ldw % 8 || a.n0 < 0 || a.n1 > a.N) return LIGER_EINVAL;
-  GemmPlan pl = gemm_plan(a.M, a.K);
+  GemmPlan pl = gemm_plan(a.M, a.N, a.K);
   const int ntiles = (a.n1 - a.n0 + BM - 1) / BM;
   if (pl.splits > 1) {
     if (!a.workspace) return LIGER_EINVAL;
-    const size_t need = GEMM_COUNTER_BYTES + (size_t)pl.splits * a.M * (a.n1 - a.n0) * sizeof(float);
-    if (a.ws_bytes < need || ntiles * pl.m_tiles > GEMM_COUNTER_BYTES / 4) return LIGER_EINVAL;
+    const size_t need = GEMM_COUNTER_BYTES + (size_t)pl.splits * ntiles * pl.m_tiles * BM * pl.bn * sizeof(float);
+    if (a.ws_bytes < need || ntiles * pl.m_tiles > (int)(GEMM_COUNTER_BYTES / 4)) return LIGER_EINVAL;
   }
   CUtensorMap tA, tB;
   int rc = make_map(&tA, a.w, a.N, a.K, a.ldw, BM);

@@ -32,7 +32,7 @@ struct GemmArgs {
   size_t ws_bytes;
 };
 
-GemmPlan gemm_plan(int M, int K);
+GemmPlan gemm_plan(int M, int N, int K);
 size_t gemm_workspace_bytes(int M, int N, int K);
 int gemm_launch(const GemmArgs& a, cudaStream_t stream);
 void gemm_forget_pointer_range(const void* base, size_t bytes);
