@@ -198,6 +198,10 @@ int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* 
                   int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
                   void* workspace, size_t ws_bytes, void* stream);
 size_t liger_gemm_workspace_bytes(int M, int N, int K);
+/* The tiling plan liger_op_gemm uses for a GEMM of full size (M, N, K) (host
+ * only; a function of (M, N, K), identical for every column slice):
+ * out[5] = {token tile bn, m tiles, split-K chunk kc, splits, pipeline stages}. */
+int liger_gemm_plan(int M, int N, int K, int32_t* out);
 
 /* Fused residual add + LayerNorm (§8(a) a2/a7/a11; C2):
  *   r    = x[in_row(i)] + (add ? add[in_row(i)] : 0) + (add_bias ? add_bias : 0)     (fp32)

@@ -63,6 +63,13 @@ int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* 
 
 size_t liger_gemm_workspace_bytes(int M, int N, int K) { return gemm_workspace_bytes(M, N, K); }
 
+int liger_gemm_plan(int M, int N, int K, int32_t* out) {
+  if (!out || M <= 0 || N <= 0 || K <= 0) return LIGER_EINVAL;
+  GemmPlan pl = gemm_plan(M, N, K);
+  out[0] = pl.bn; out[1] = pl.m_tiles; out[2] = pl.kc; out[3] = pl.splits; out[4] = pl.stages;
+  return LIGER_OK;
+}
+
 int liger_op_add_layernorm(const void* x, const void* add, const void* add_bias, void* x_out, void* y,
                            const void* gamma, const void* beta, int rows, int h, int in_row_step, int in_row_off,
                            float eps, void* stream) {

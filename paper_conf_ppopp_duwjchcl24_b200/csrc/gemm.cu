@@ -25,6 +25,7 @@
 #include <cuda_bf16.h>
 #include <stdint.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <mutex>
 #include <unordered_map>
 #include <vector>
@@ -390,38 +391,38 @@ GemmPlan gemm_plan(int M, int N, int K) {
   GemmPlan pl{};
   const int G = num_sms();
   const int n_tiles = (N + BM - 1) / BM;
-  const int nkb_total = (K + BK - 1) / BK;
-  double best = 1e30;
-  const int bn_opts[3] = {256, 128, 64};
-  for (int bi = 0; bi < 3; ++bi) {
-    const int bcap = bn_opts[bi];
-    if (bi > 0 && M <= bcap) break;           // smaller caps only when they create more tiles
-    const int mt = (M + bcap - 1) / bcap;
-    int bn = (M + mt - 1) / mt;
-    bn = (bn + 15) / 16 * 16;
-    if (bn < 16) bn = 16;
-    const int tiles = n_tiles * mt;
-    // per-k-block cost (cycles): MMA 4 x (2 bn) vs operand load (16 KB + 128 bn B) at ~64 B/clk
-    const double kb_cost = fmax(8.0 * bn, (A_BYTES + 128.0 * bn) / 64.0);
-    const int smax = nkb_total >= 8 ? nkb_total / 4 : 1;   // chunks of >= 256 K
-    for (int sp = 1; sp <= smax; ++sp) {
-      const int kcb = (nkb_total + sp - 1) / sp;            // k-blocks per chunk
-      const int S = (nkb_total + kcb - 1) / kcb;
+  const int nkb = (K + BK - 1) / BK;
+  const int mt = (M + 255) / 256;
+  int bn = (M + mt - 1) / mt;
+  bn = (bn + 15) / 16 * 16;
+  if (bn < 16) bn = 16;
+  const int tiles = n_tiles * mt;
+  // Split K only when the tiles alone leave SMs idle.  Cost = (units per CTA) x
+  // (k-blocks per unit + a fixed per-unit overhead), chunks of >= 4 k-blocks.
+  const double ovh = M <= 64 ? 4.0 : 12.0;
+  int best_s = 1;
+  double best = (double)((tiles + G - 1) / G) * (nkb + ovh);
+  if ((tiles < G || M <= 64) && tiles <= (int)(GEMM_COUNTER_BYTES / 4)) {
+    for (int sp = 2; sp <= nkb / 4; ++sp) {
+      const int kcb = (nkb + sp - 1) / sp;
+      const int S = (nkb + kcb - 1) / kcb;
       if (S != sp) continue;
-      const int units = tiles * S;
-      const int per_cta = (units + G - 1) / G;
-      double cost = per_cta * (kcb * kb_cost + 600.0);     // + per-unit epilogue hand-off
-      if (S > 1) cost += 1500.0 + 40.0 * S * bn / 16;       // partial write/reduce
-      cost += (tiles > 4096 / 1 && S > 1) ? 1e30 : 0;       // counter capacity
+      const double cost = (double)((tiles * S + G - 1) / G) * (kcb + ovh) + (M <= 64 ? 1.0 : 4.0) * S;
       if (cost < best - 1e-9) {
         best = cost;
-        pl.bn = bn;
-        pl.m_tiles = mt;
-        pl.kc = kcb * BK;
-        pl.splits = S;
+        best_s = S;
       }
     }
   }
+  if (const char* e = getenv("LIGER_GEMM_FORCE_SPLITS")) {   // experiments only
+    const int f = atoi(e);
+    if (f >= 1 && f <= nkb) best_s = f;
+  }
+  const int kcb = (nkb + best_s - 1) / best_s;
+  pl.bn = bn;
+  pl.m_tiles = mt;
+  pl.kc = kcb * BK;
+  pl.splits = (nkb + kcb - 1) / kcb;
   const int stage_bytes = A_BYTES + pl.bn * BK * 2;
   int st = (MAX_SMEM - 1024 - 256) / stage_bytes;
   if (st > 12) st = 12;

@@ -63,6 +63,7 @@ _SIGS = {
     "liger_finalize": (_I, [_P]),
     "liger_op_gemm": (_I, [_P, _I64, _P, _I64, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),
     "liger_gemm_workspace_bytes": (_SZ, [_I, _I, _I]),
+    "liger_gemm_plan": (_I, [_I, _I, _I, _P]),
     "liger_op_add_layernorm": (_I, [_P, _P, _P, _P, _P, _P, _P, _I, _I, _I, _I, _F, _P]),
     "liger_op_embed": (_I, [_P, _P, _P, _P, _I, _I, _I, _I, _P]),
     "liger_op_attn_prefill": (_I, [_P, _P, _P, _P, _I, _I, _I, _I, _I, _P]),
@@ -133,6 +134,12 @@ def gemm(x, w, out, *, n0=0, n1=None, bias=None, act="none", scale_cols=0, scale
 
 def gemm_workspace_bytes(M, N, K):
     return lib().liger_gemm_workspace_bytes(M, N, K)
+
+
+def gemm_plan(M, N, K):
+    out = (C.c_int32 * 5)()
+    check(lib().liger_gemm_plan(M, N, K, out), what="liger_gemm_plan")
+    return dict(zip(("bn", "m_tiles", "kc", "splits", "stages"), list(out)))
 
 
 def add_layernorm(x, gamma, beta, y, *, add=None, add_bias=None, x_out=None, rows=None, in_row_step=1,
