@@ -65,6 +65,7 @@ __global__ void __launch_bounds__(128) attn_prefill_kernel(const __nv_bfloat16* 
   __nv_bfloat16* sK = sQ + PF_BQ * LDS;
   __nv_bfloat16* sV = sK + PF_BK * LDS;
 
+  pdl_enter();
   const int qt = blockIdx.x, head = blockIdx.y, bi = blockIdx.z;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t ld = (int64_t)3 * heads * D;
@@ -215,15 +216,16 @@ int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* 
     cudaFuncSetAttribute(attn_prefill_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
     attr = true;
   }
+  int rc;
   if (d == 128)
-    attn_prefill_kernel<128><<<grid, 128, smem, stream>>>((const __nv_bfloat16*)qkv, (__nv_bfloat16*)o,
-                                                       (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
+    rc = launch_pdl(attn_prefill_kernel<128>, grid, dim3(128), smem, stream, (const __nv_bfloat16*)qkv,
+                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
   else if (d == 64)
-    attn_prefill_kernel<64><<<grid, 128, smem, stream>>>((const __nv_bfloat16*)qkv, (__nv_bfloat16*)o,
-                                                      (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
+    rc = launch_pdl(attn_prefill_kernel<64>, grid, dim3(128), smem, stream, (const __nv_bfloat16*)qkv,
+                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
   else
     return LIGER_EINVAL;
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  return rc ? LIGER_ECUDA : 0;
 }
 
 // ================================================================== decode
@@ -271,6 +273,7 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   __shared__ int pg[NPG];
   __shared__ int last;
 
+  pdl_enter();
   const int head = blockIdx.x, bi = blockIdx.y, sp = blockIdx.z, nsp = gridDim.z;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ctx = pos + 1;
@@ -432,17 +435,16 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   int* counters = (int*)workspace;
   float* ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
   dim3 grid(heads, b, ns);
+  int rc;
   if (d == 128)
-    attn_decode_kernel<128><<<grid, DC_THREADS, 0, stream>>>((const __nv_bfloat16*)qkv, (__nv_bfloat16*)o,
-                                                              (__nv_bfloat16*)kv_pool, page_table, max_pages, pos,
-                                                              heads, ws, counters);
+    rc = launch_pdl(attn_decode_kernel<128>, grid, dim3(DC_THREADS), 0, stream, (const __nv_bfloat16*)qkv,
+                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads, ws, counters);
   else if (d == 64)
-    attn_decode_kernel<64><<<grid, DC_THREADS, 0, stream>>>((const __nv_bfloat16*)qkv, (__nv_bfloat16*)o,
-                                                             (__nv_bfloat16*)kv_pool, page_table, max_pages, pos,
-                                                             heads, ws, counters);
+    rc = launch_pdl(attn_decode_kernel<64>, grid, dim3(DC_THREADS), 0, stream, (const __nv_bfloat16*)qkv,
+                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads, ws, counters);
   else
     return LIGER_EINVAL;
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  return rc ? LIGER_ECUDA : 0;
 }
 
 }  // namespace liger

@@ -4,6 +4,8 @@
 #include <cuda_bf16.h>
 #include <stdint.h>
 
+#include <utility>
+
 #define LIGER_DEV __device__ __forceinline__
 
 namespace liger {
@@ -127,11 +129,43 @@ LIGER_DEV void named_bar_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
+// Programmatic dependent launch: wait for the preceding grid in the stream
+// (no-op when launched without the PDL attribute).
+LIGER_DEV void grid_dependency_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+// Allow the next PDL kernel in the stream to be scheduled (its CTAs wait in
+// grid_dependency_wait until this grid has completed).
+LIGER_DEV void grid_dependency_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+// Both, for kernels whose whole body depends on upstream data.
+LIGER_DEV void pdl_enter() {
+  grid_dependency_trigger();
+  grid_dependency_wait();
+}
+
 LIGER_DEV float bf16_bits_to_f32(uint16_t b) { return __uint_as_float(((uint32_t)b) << 16); }
 
 LIGER_DEV float gelu_tanh_f(float x) {
   const float k0 = 0.7978845608028654f, k1 = 0.044715f;
   return 0.5f * x * (1.0f + tanhf(k0 * (x + k1 * x * x * x)));
+}
+
+// Launch with programmatic stream serialization so the kernel's prologue overlaps
+// the tail of the previous kernel on the stream (the kernel calls
+// grid_dependency_wait() before touching data produced or consumed upstream).
+template <typename... KArgs, typename... Args>
+inline int launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
+                      Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+  return e == cudaSuccess ? 0 : -1000;
 }
 
 }  // namespace liger

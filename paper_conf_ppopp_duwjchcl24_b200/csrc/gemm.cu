@@ -114,29 +114,31 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   uint64_t* bars = reinterpret_cast<uint64_t*>(smB + (size_t)S * B_BYTES);
   uint64_t* full = bars;
   uint64_t* empty = bars + S;
-  uint64_t* tmem_full = bars + 2 * S;       // [2]
-  uint64_t* tmem_empty = bars + 2 * S + 2;  // [2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 4);
-  int* last_flag = reinterpret_cast<int*>(tmem_slot + 1);
+  uint64_t* tmem_full = bars + 2 * S;       // [TS]
+  uint64_t* tmem_empty = bars + 2 * S + 4;  // [TS]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 8);
+  int* last_flag = reinterpret_cast<int*>(tmem_slot + 1);   // [2], alternating per unit
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const int G = gridDim.x;
   const uint32_t acc_cols = p.bn <= 32 ? 32 : (p.bn <= 64 ? 64 : (p.bn <= 128 ? 128 : 256));
-  const uint32_t tmem_cols = 2 * acc_cols;
+  const int TS = acc_cols >= 256 ? 2 : 4;          // TMEM accumulator stages (epilogue slack)
+  const uint32_t tmem_cols = (uint32_t)TS * acc_cols;
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);
       mbar_init(&empty[i], 1);
     }
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < TS; ++i) {
       mbar_init(&tmem_full[i], 1);
       mbar_init(&tmem_empty[i], 4);   // one arrive per epilogue warp
     }
     fence_barrier_init();
   }
   if (warp == 0 && lane == 0) {
+    grid_dependency_trigger();
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
   }
@@ -149,6 +151,24 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   if (warp == 0) {
     if (lane == 0) {
       const uint64_t pol_w = policy_evict_first();   // weights: streamed once per tile
+      // Programmatic dependent launch: the weight tiles of the first S stages do
+      // not depend on the previous kernel, so they are requested before
+      // griddepcontrol.wait; activation tiles only after it.
+      int pre = 0;
+      {
+        int it = 0;
+        for (int u = blockIdx.x; u < p.units && it < S; u += G) {
+          const Unit w = unit_of(p, u);
+          const int k0 = w.z * p.kc;
+          const int nkb = (min(p.K, k0 + p.kc) - k0 + BK - 1) / BK;
+          for (int kb = 0; kb < nkb && it < S; ++kb, ++it) {
+            mbar_arrive_expect_tx(&full[it], A_BYTES + B_BYTES);
+            tma_load_2d_hint(smA + (size_t)it * A_BYTES, &tmA, &full[it], k0 + kb * BK, p.n0 + w.nt * BM, pol_w);
+          }
+        }
+        pre = it;
+      }
+      grid_dependency_wait();
       int it = 0;
       for (int u = blockIdx.x; u < p.units; u += G) {
         const Unit w = unit_of(p, u);
@@ -158,10 +178,12 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         for (int kb = 0; kb < nkb; ++kb, ++it) {
           const int s = it % S;
           const uint32_t ph = (it / S) & 1;
-          mbar_wait(&empty[s], ph ^ 1);
-          mbar_arrive_expect_tx(&full[s], A_BYTES + B_BYTES);
           const int kk = k0 + kb * BK;
-          tma_load_2d_hint(smA + (size_t)s * A_BYTES, &tmA, &full[s], kk, n_base, pol_w);
+          if (it >= pre) {
+            mbar_wait(&empty[s], ph ^ 1);
+            mbar_arrive_expect_tx(&full[s], A_BYTES + B_BYTES);
+            tma_load_2d_hint(smA + (size_t)s * A_BYTES, &tmA, &full[s], kk, n_base, pol_w);
+          }
           tma_load_2d(smB + (size_t)s * B_BYTES, &tmB, &full[s], kk, m_base);
         }
       }
@@ -176,8 +198,8 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         const Unit w = unit_of(p, u);
         const int k0 = w.z * p.kc;
         const int nkb = (min(p.K, k0 + p.kc) - k0 + BK - 1) / BK;
-        const int acc = lu & 1;
-        const uint32_t acc_ph = (lu >> 1) & 1;
+        const int acc = lu % TS;
+        const uint32_t acc_ph = (lu / TS) & 1;
         mbar_wait(&tmem_empty[acc], acc_ph ^ 1);
         tc_fence_after();
         const uint32_t tacc = tmem_base + (uint32_t)acc * acc_cols;
@@ -208,13 +230,12 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       const int n = n_base + row;
       const bool nval = (n < p.n1) && (n < p.N);
       const float bias_v = (p.bias != nullptr && nval) ? __bfloat162float(p.bias[n]) : 0.0f;
-      const int acc = lu & 1;
-      const uint32_t acc_ph = (lu >> 1) & 1;
+      const int acc = lu % TS;
+      const uint32_t acc_ph = (lu / TS) & 1;
       const int mcount = min(p.bn, p.M - m_base);
       const int tile_id = w.nt * p.m_tiles + w.mt;
-      // fp32 partial of (chunk z, tile): [128 rows][bn] row-major, 16-byte vectors
-      float* my_ws = p.splits > 1 ? p.ws + ((int64_t)w.z * tiles + tile_id) * (BM * p.bn) + (int64_t)row * p.bn
-                                  : nullptr;
+      // fp32 partial of (chunk z, tile): [bn cols][128 rows] (a warp writes 128 B per column)
+      float* my_ws = p.splits > 1 ? p.ws + ((int64_t)w.z * tiles + tile_id) * (BM * p.bn) + row : nullptr;
       mbar_wait(&tmem_full[acc], acc_ph);
       tc_fence_after();
       const uint32_t tacc = tmem_base + (uint32_t)acc * acc_cols + ((uint32_t)(q * 32) << 16);
@@ -230,12 +251,9 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
               if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, __uint_as_float(r[j]), n, bias_v));
           }
         } else {
-          float4* dst = reinterpret_cast<float4*>(my_ws + c0);
 #pragma unroll
-          for (int v = 0; v < 4; ++v)
-            if (c0 + 4 * v < mcount)
-              __stcg(dst + v, make_float4(__uint_as_float(r[4 * v]), __uint_as_float(r[4 * v + 1]),
-                                          __uint_as_float(r[4 * v + 2]), __uint_as_float(r[4 * v + 3])));
+          for (int j = 0; j < 16; ++j)
+            if (c0 + j < mcount) __stcg(my_ws + (int64_t)(c0 + j) * BM, __uint_as_float(r[j]));
         }
       }
       // accumulator drained: hand the TMEM buffer back to the MMA warp
@@ -247,53 +265,46 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         // partials in chunk order 0..splits-1 (independent of who is last).
         // Release: CTA barrier, then one gpu-scope fence + atomic (cumulative).
         named_bar_sync(1, 128);
+        int* flag = last_flag + (lu & 1);
         if (threadIdx.x == 64) {
           __threadfence();
           const int prev = atomicAdd(&p.counters[tile_id], 1);
-          *last_flag = (prev == p.splits - 1);
-          if (*last_flag) __threadfence();   // acquire side
+          *flag = (prev == p.splits - 1);
+          if (*flag) __threadfence();   // acquire side
         }
         named_bar_sync(1, 128);
-        if (*last_flag) {
+        if (*flag) {
           if (nval) {
-            const float* base = p.ws + (int64_t)tile_id * (BM * p.bn) + (int64_t)row * p.bn;
+            const float* base = p.ws + (int64_t)tile_id * (BM * p.bn) + row;
             const int64_t zstride = (int64_t)tiles * (BM * p.bn);
             for (int c0 = 0; c0 < mcount; c0 += 16) {
-              const int nv4 = min(4, (mcount - c0 + 3) / 4);
-              float4 accv[4];
+              float accv[16];
 #pragma unroll
-              for (int v = 0; v < 4; ++v) accv[v] = make_float4(0.f, 0.f, 0.f, 0.f);
+              for (int j = 0; j < 16; ++j) accv[j] = 0.f;
               constexpr int UNR = 4;
               for (int z0 = 0; z0 < p.splits; z0 += UNR) {
-                float4 ld[UNR][4];
+                float ld[UNR][16];
 #pragma unroll
                 for (int zz = 0; zz < UNR; ++zz)
 #pragma unroll
-                  for (int v = 0; v < 4; ++v)
-                    ld[zz][v] = (z0 + zz < p.splits && v < nv4)
-                                    ? __ldcg(reinterpret_cast<const float4*>(base + (z0 + zz) * zstride + c0) + v)
-                                    : make_float4(0.f, 0.f, 0.f, 0.f);
+                  for (int j = 0; j < 16; ++j)
+                    ld[zz][j] = (z0 + zz < p.splits && c0 + j < mcount)
+                                    ? __ldcg(base + (z0 + zz) * zstride + (int64_t)(c0 + j) * BM)
+                                    : 0.f;
 #pragma unroll
                 for (int zz = 0; zz < UNR; ++zz)
+                  if (z0 + zz < p.splits) {   // sum in chunk order
 #pragma unroll
-                  for (int v = 0; v < 4; ++v) {
-                    if (z0 + zz < p.splits) {     // sum in chunk order
-                      accv[v].x += ld[zz][v].x;
-                      accv[v].y += ld[zz][v].y;
-                      accv[v].z += ld[zz][v].z;
-                      accv[v].w += ld[zz][v].w;
-                    }
+                    for (int j = 0; j < 16; ++j) accv[j] += ld[zz][j];
                   }
               }
-              const float* a = reinterpret_cast<const float*>(accv);
 #pragma unroll
               for (int j = 0; j < 16; ++j)
-                if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, a[j], n, bias_v));
+                if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, accv[j], n, bias_v));
             }
           }
           if (threadIdx.x == 64) p.counters[tile_id] = 0;
         }
-        named_bar_sync(1, 128);   // last_flag is reused by the next unit
       }
     }
   }
@@ -424,10 +435,10 @@ GemmPlan gemm_plan(int M, int N, int K) {
   pl.kc = kcb * BK;
   pl.splits = (nkb + kcb - 1) / kcb;
   const int stage_bytes = A_BYTES + pl.bn * BK * 2;
-  int st = (MAX_SMEM - 1024 - 256) / stage_bytes;
+  int st = (MAX_SMEM - 1024 - 512) / stage_bytes;
   if (st > 12) st = 12;
   pl.stages = st;
-  pl.smem = 1024 + st * stage_bytes + 256;
+  pl.smem = 1024 + st * stage_bytes + 512;
   return pl;
 }
 
@@ -470,8 +481,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.m_tiles = pl.m_tiles;
   p.units = ntiles * pl.m_tiles * pl.splits;
   const int grid = p.units < num_sms() ? p.units : num_sms();
-  gemm_tc_kernel<<<grid, GEMM_THREADS, pl.smem, stream>>>(tA, tB, p);
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  return launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
 }
 
 }  // namespace liger

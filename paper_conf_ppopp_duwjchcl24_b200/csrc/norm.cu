@@ -53,6 +53,7 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
                                                     const bf16x8* __restrict__ beta, int h, int in_row_step,
                                                     int in_row_off, float eps) {
   __shared__ float red[NT / 32];
+  pdl_enter();
   const int nv = h >> 3;
   const int64_t in_row = (int64_t)blockIdx.x * in_row_step + in_row_off;
   const bf16x8* xr = x + in_row * nv;
@@ -132,21 +133,23 @@ int add_layernorm_launch(const void* x, const void* add, const void* add_bias, v
   const bf16x8* A = (const bf16x8*)add;
   const bf16x8* AB = (const bf16x8*)add_bias;
   const int nv = h / 8;
-#define LIGER_LN(NT, MV)                                                                                   \
-  add_ln_kernel<NT, MV><<<rows, NT, 0, stream>>>(X, A, AB, (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma, \
-                                                 (const bf16x8*)beta, h, in_row_step, in_row_off, eps)
-  if (nv <= 128) LIGER_LN(128, 1);
-  else if (nv <= 512) LIGER_LN(128, 4);
-  else if (nv <= 1024) LIGER_LN(256, 4);
-  else LIGER_LN(512, 4);
+#define LIGER_LN(NT, MV)                                                                                     \
+  launch_pdl(add_ln_kernel<NT, MV>, dim3(rows), dim3(NT), 0, stream, X, A, AB, (bf16x8*)x_out, (bf16x8*)y, \
+             (const bf16x8*)gamma, (const bf16x8*)beta, h, in_row_step, in_row_off, eps)
+  int rc;
+  if (nv <= 128) rc = LIGER_LN(128, 1);
+  else if (nv <= 512) rc = LIGER_LN(128, 4);
+  else if (nv <= 1024) rc = LIGER_LN(256, 4);
+  else rc = LIGER_LN(512, 4);
 #undef LIGER_LN
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  return rc ? LIGER_ECUDA : 0;
 }
 
 // ------------------------------------------------------------------ embedding
 __global__ void embed_kernel(const int32_t* __restrict__ ids, const bf16x8* __restrict__ e_tok,
                              const bf16x8* __restrict__ e_pos, bf16x8* __restrict__ out, int h, int seq_len,
                              int start_pos) {
+  pdl_enter();
   const int i = blockIdx.x;
   const int nv = h >> 3;
   const int64_t id = ids[i];
@@ -166,9 +169,10 @@ int embed_launch(const int32_t* ids, const void* e_tok, const void* e_pos, void*
   if (rows <= 0) return 0;
   if (h % 8) return LIGER_EINVAL;
   int nt = h / 8 < 256 ? ((h / 8 + 31) / 32 * 32) : 256;
-  embed_kernel<<<rows, nt, 0, stream>>>(ids, (const bf16x8*)e_tok, (const bf16x8*)e_pos, (bf16x8*)out, h, seq_len,
-                                        start_pos);
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  return launch_pdl(embed_kernel, dim3(rows), dim3(nt), 0, stream, ids, (const bf16x8*)e_tok, (const bf16x8*)e_pos,
+                    (bf16x8*)out, h, seq_len, start_pos)
+             ? LIGER_ECUDA
+             : 0;
 }
 
 // ------------------------------------------------------------------ argmax (lowest index on ties)
@@ -183,6 +187,7 @@ __global__ void argmax_kernel(const float* __restrict__ logits, int64_t ld, int 
                               float* max_out, int32_t* idx_out) {
   __shared__ float sv[32];
   __shared__ int si[32];
+  pdl_enter();
   const float* row = logits + (int64_t)blockIdx.x * ld;
   float bv = -INFINITY;
   int bi = 0x7fffffff;
@@ -209,8 +214,9 @@ __global__ void argmax_kernel(const float* __restrict__ logits, int64_t ld, int 
 int argmax_launch(const float* logits, int64_t ld, int rows, int n, int idx_offset, float* max_out,
                   int32_t* idx_out, cudaStream_t stream) {
   if (rows <= 0) return 0;
-  argmax_kernel<<<rows, 1024, 0, stream>>>(logits, ld, n, idx_offset, max_out, idx_out);
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  return launch_pdl(argmax_kernel, dim3(rows), dim3(1024), 0, stream, logits, ld, n, idx_offset, max_out, idx_out)
+             ? LIGER_ECUDA
+             : 0;
 }
 
 // vals/idx: [world][rows] gathered from every rank's vocab shard.  Writes the
@@ -218,6 +224,7 @@ int argmax_launch(const float* logits, int64_t ld, int rows, int n, int idx_offs
 // tok_out[r * out_stride + out_col] (the batch's generated sequence).
 __global__ void argmax_pick_kernel(const float* vals, const int32_t* idx, int world, int rows, int32_t* tok_cur,
                                    int32_t* tok_out, int out_stride, int out_col) {
+  pdl_enter();
   const int r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= rows) return;
   float bv = vals[r];
@@ -230,9 +237,10 @@ __global__ void argmax_pick_kernel(const float* vals, const int32_t* idx, int wo
 int argmax_pick_launch(const float* vals, const int32_t* idx, int world, int rows, int32_t* tok_cur,
                        int32_t* tok_out, int out_stride, int out_col, cudaStream_t stream) {
   if (rows <= 0) return 0;
-  argmax_pick_kernel<<<(rows + 127) / 128, 128, 0, stream>>>(vals, idx, world, rows, tok_cur, tok_out, out_stride,
-                                                             out_col);
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  return launch_pdl(argmax_pick_kernel, dim3((rows + 127) / 128), dim3(128), 0, stream, vals, idx, world, rows,
+                    tok_cur, tok_out, out_stride, out_col)
+             ? LIGER_ECUDA
+             : 0;
 }
 
 // ------------------------------------------------------------------ C0 generator (device side)
