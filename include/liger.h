@@ -197,6 +197,15 @@ int liger_finalize(liger_ctx* ctx); /* [collective] */
 int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* out, int64_t ldo, int M, int N,
                   int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
                   void* workspace, size_t ws_bytes, void* stream);
+/* Same, with W in the tiled layout liger_load_layer uses for the projection
+ * weights: [ceil(N/128)][K/64][128][64] bf16 (every 16 KiB TMA box contiguous in
+ * HBM); requires K % 64 == 0 and n0 % 128 == 0. */
+int liger_op_gemm_tiled(const void* x, int64_t ldx, const void* w_tiled, void* out, int64_t ldo, int M, int N,
+                        int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
+                        void* workspace, size_t ws_bytes, void* stream);
+/* Convert a row-major bf16 W [N, K] (row stride ld) to the tiled layout
+ * (dst holds ceil(N/128)*128*K elements; padding rows are zero). */
+int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K, void* stream);
 size_t liger_gemm_workspace_bytes(int M, int N, int K);
 /* The tiling plan liger_op_gemm uses for a GEMM of full size (M, N, K) (host
  * only; a function of (M, N, K), identical for every column slice):
@@ -245,7 +254,10 @@ int liger_op_argmax(const float* logits, int64_t ld, int rows, int n, int idx_of
 /* Fill a bf16 [rows, cols] (row stride ld) device tensor with C0 values of
  * logical tensor `tensor_id`: element (r, c) takes global index
  * (r + row_off) * idx_row_stride + (c + col_off) * idx_col_stride, scale 2^exp;
- * kind 0 = plain, 1 = gamma (1 + v/16), 2 = beta (v/16). */
+ * kind 0 = plain, 1 = gamma (1 + v/16), 2 = beta (v/16); kind | LIGER_C0_TILED writes
+ * element (r, c) as row ld + r, column c of a tiled-layout matrix with K = cols
+ * (see liger_op_gemm_tiled; ld then means "first destination row"). */
+#define LIGER_C0_TILED 16
 int liger_op_c0_fill(void* dst, int rows, int cols, int64_t ld, uint64_t seed, uint64_t tensor_id,
                      int64_t row_off, int64_t col_off, int64_t idx_row_stride, int64_t idx_col_stride, int exp,
                      int kind, void* stream);

@@ -57,8 +57,21 @@ int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* 
                   int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
                   void* workspace, size_t ws_bytes, void* stream) {
   if (int rc = check_device()) return rc;
-  GemmArgs a{x, ldx, w, ldw, out, ldo, M, N, K, n0, n1, bias, act, scale_cols, scale, out_f32, workspace, ws_bytes};
+  GemmArgs a{x, ldx, w, ldw, out, ldo, M, N, K, n0, n1, bias, act, scale_cols, scale, out_f32, workspace, ws_bytes, 0};
   return ret(gemm_launch(a, (cudaStream_t)stream), "liger_op_gemm");
+}
+
+int liger_op_gemm_tiled(const void* x, int64_t ldx, const void* w, void* out, int64_t ldo, int M, int N, int K,
+                        int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
+                        void* workspace, size_t ws_bytes, void* stream) {
+  if (int rc = check_device()) return rc;
+  GemmArgs a{x, ldx, w, 64, out, ldo, M, N, K, n0, n1, bias, act, scale_cols, scale, out_f32, workspace, ws_bytes, 1};
+  return ret(gemm_launch(a, (cudaStream_t)stream), "liger_op_gemm_tiled");
+}
+
+int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K, void* stream) {
+  if (int rc = check_device()) return rc;
+  return ret(tile_weight_launch(w, ld, w_tiled, N, K, (cudaStream_t)stream), "liger_op_tile_weight");
 }
 
 size_t liger_gemm_workspace_bytes(int M, int N, int K) { return gemm_workspace_bytes(M, N, K); }

@@ -273,12 +273,14 @@ int gemm_K(liger_ctx* c, int op) {
   }
   return 0;
 }
-// column boundary of unit u (of F) for an N-wide GEMM: multiples of 16, last = N
+// column boundary of unit u (of F) for an N-wide GEMM: multiples of 128 (the
+// tiled weight layout's row tile), last = N.  Small GEMMs may get empty pieces.
 int unit_col(int N, int u, int F) {
   if (u >= F) return N;
   int c = (int)((int64_t)N * u / F);
-  return c / 16 * 16;
+  return c / 128 * 128;
 }
+int pad128(int n) { return (n + 127) / 128 * 128; }
 
 int batch_M(const Batch* bt, int pass) { return pass == 0 ? bt->b * bt->s : bt->b; }
 
@@ -424,6 +426,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       g.n1 = unit_col(N, u1, F);
       g.workspace = S.gemm_ws; g.ws_bytes = S.gemm_ws_bytes;
       g.scale = 1.0f;
+      g.w_tiled = 1;
       if (po.op == OP_QKV) {
         g.x = S.y; g.ldx = h; g.w = W->w_qkv; g.ldw = K; g.out = S.qkv; g.ldo = N; g.bias = W->b_qkv;
         g.scale_cols = c->hl; g.scale = 1.0f / sqrtf((float)c->d);
@@ -733,13 +736,13 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   const size_t h = c->h;
   for (int l = 0; l < c->L; ++l) {
     LayerW& W = c->layers[l];
-    W.w_qkv = dalloc(c, 3 * c->hl * h * 2);
+    W.w_qkv = dalloc(c, (size_t)pad128(3 * c->hl) * h * 2);
     W.b_qkv = dalloc(c, 3 * c->hl * 2);
-    W.w_o = dalloc(c, h * c->hl * 2);
+    W.w_o = dalloc(c, (size_t)pad128(c->h) * c->hl * 2);
     W.b_o = dalloc(c, h * 2);
-    W.w_1 = dalloc(c, (size_t)c->fl * h * 2);
+    W.w_1 = dalloc(c, (size_t)pad128(c->fl) * h * 2);
     W.b_1 = dalloc(c, (size_t)c->fl * 2);
-    W.w_2 = dalloc(c, h * c->fl * 2);
+    W.w_2 = dalloc(c, (size_t)pad128(c->h) * c->fl * 2);
     W.b_2 = dalloc(c, h * 2);
     W.g1 = dalloc(c, h * 2); W.be1 = dalloc(c, h * 2); W.g2 = dalloc(c, h * 2); W.be2 = dalloc(c, h * 2);
     if (!W.w_qkv || !W.w_o || !W.w_1 || !W.w_2 || !W.be2)
@@ -830,21 +833,27 @@ int liger_load_layer(liger_ctx* c, int l, uint64_t seed) {
   LayerW& W = c->layers[l];
   cudaStream_t st = c->s_comp;
   const uint64_t tid = 16ull * l;
-  // W_qkv logical [h, 3h]; local row j of block s in {q,k,v} = logical column s*h + r*hl + j'
+  // Projection weights are stored K-major in the tiled layout [N/128][K/64][128][64]
+  // (LIGER_C0_TILED; the `ld` argument is then the first destination row).
+  const int T = LIGER_C0_TILED;
+  if (hl % 64 || fl % 64) return fail(c, LIGER_EINVAL, "liger_load_layer: h/t and 4h/t must be multiples of 64");
+  CK(cudaMemsetAsync(W.w_qkv, 0, (size_t)pad128(3 * (int)hl) * h * 2, st));
+  CK(cudaMemsetAsync(W.w_1, 0, (size_t)pad128((int)fl) * h * 2, st));
+  // W_qkv logical [h, 3h]; local row j of block s in {q,k,v} = logical column s*h + r*hl + j
   for (int s = 0; s < 3; ++s) {
-    CKR(c0_fill_launch((char*)W.w_qkv + s * hl * h * 2, (int)hl, (int)h, h, seed, tid + 0, s * h + r * hl, 0, 1,
-                       3 * h, weight_exp((int)h), 0, st));
+    CKR(c0_fill_launch(W.w_qkv, (int)hl, (int)h, s * hl, seed, tid + 0, s * h + r * hl, 0, 1, 3 * h,
+                       weight_exp((int)h), T, st));
     CKR(c0_fill_launch((char*)W.b_qkv + s * hl * 2, 1, (int)hl, hl, seed, tid + 1, 0, s * h + r * hl, 0, 1, BIAS_EXP,
                        0, st));
   }
   // W_o logical [h_in, h_out]; local [h_out, hl_in]: (n, k) -> ((r*hl + k) * h + n)
-  CKR(c0_fill_launch(W.w_o, (int)h, (int)hl, hl, seed, tid + 2, 0, r * hl, 1, h, weight_exp((int)h, true), 0, st));
+  CKR(c0_fill_launch(W.w_o, (int)h, (int)hl, 0, seed, tid + 2, 0, r * hl, 1, h, weight_exp((int)h, true), T, st));
   CKR(c0_fill_launch(W.b_o, 1, (int)h, h, seed, tid + 3, 0, 0, 0, 1, BIAS_EXP, 0, st));
   // W_1 logical [h, f]; local [fl, h]: (n, k) -> (k * f + r*fl + n)
-  CKR(c0_fill_launch(W.w_1, (int)fl, (int)h, h, seed, tid + 4, r * fl, 0, 1, f, weight_exp((int)h), 0, st));
+  CKR(c0_fill_launch(W.w_1, (int)fl, (int)h, 0, seed, tid + 4, r * fl, 0, 1, f, weight_exp((int)h), T, st));
   CKR(c0_fill_launch(W.b_1, 1, (int)fl, fl, seed, tid + 5, 0, r * fl, 0, 1, BIAS_EXP, 0, st));
   // W_2 logical [f, h]; local [h, fl]: (n, k) -> ((r*fl + k) * h + n)
-  CKR(c0_fill_launch(W.w_2, (int)h, (int)fl, fl, seed, tid + 6, 0, r * fl, 1, h, weight_exp((int)f, true), 0, st));
+  CKR(c0_fill_launch(W.w_2, (int)h, (int)fl, 0, seed, tid + 6, 0, r * fl, 1, h, weight_exp((int)f, true), T, st));
   CKR(c0_fill_launch(W.b_2, 1, (int)h, h, seed, tid + 7, 0, 0, 0, 1, BIAS_EXP, 0, st));
   CKR(c0_fill_launch(W.g1, 1, (int)h, h, seed, tid + 8, 0, 0, 0, 1, 0, 1, st));
   CKR(c0_fill_launch(W.be1, 1, (int)h, h, seed, tid + 9, 0, 0, 0, 1, 0, 2, st));

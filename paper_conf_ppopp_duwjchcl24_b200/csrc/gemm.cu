@@ -60,6 +60,8 @@ struct GemmParams {
   int stages;
   int n_tiles, m_tiles;
   int units;            // n_tiles * m_tiles * splits
+  int w_tiled;          // W stored as [N/128][K/64][128][64] (each TMA box contiguous)
+  int nkb_total;        // K / 64
   const __nv_bfloat16* bias;
   int act;
   int scale_cols;
@@ -163,7 +165,9 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
           const int nkb = (min(p.K, k0 + p.kc) - k0 + BK - 1) / BK;
           for (int kb = 0; kb < nkb && it < S; ++kb, ++it) {
             mbar_arrive_expect_tx(&full[it], A_BYTES + B_BYTES);
-            tma_load_2d_hint(smA + (size_t)it * A_BYTES, &tmA, &full[it], k0 + kb * BK, p.n0 + w.nt * BM, pol_w);
+            const int kk = k0 + kb * BK, nb = p.n0 + w.nt * BM;
+            tma_load_2d_hint(smA + (size_t)it * A_BYTES, &tmA, &full[it], p.w_tiled ? 0 : kk,
+                             p.w_tiled ? ((nb / BM) * p.nkb_total + kk / BK) * BM : nb, pol_w);
           }
         }
         pre = it;
@@ -182,7 +186,8 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
           if (it >= pre) {
             mbar_wait(&empty[s], ph ^ 1);
             mbar_arrive_expect_tx(&full[s], A_BYTES + B_BYTES);
-            tma_load_2d_hint(smA + (size_t)s * A_BYTES, &tmA, &full[s], kk, n_base, pol_w);
+            tma_load_2d_hint(smA + (size_t)s * A_BYTES, &tmA, &full[s], p.w_tiled ? 0 : kk,
+                             p.w_tiled ? ((n_base / BM) * p.nkb_total + kk / BK) * BM : n_base, pol_w);
           }
           tma_load_2d(smB + (size_t)s * B_BYTES, &tmB, &full[s], kk, m_base);
         }
@@ -267,10 +272,12 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         named_bar_sync(1, 128);
         int* flag = last_flag + (lu & 1);
         if (threadIdx.x == 64) {
-          __threadfence();
-          const int prev = atomicAdd(&p.counters[tile_id], 1);
+          // acq_rel atomic: releases this CTA's partial stores (ordered before it by
+          // the barrier; PTX release is cumulative) and acquires the other CTAs'.
+          int prev;
+          asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&p.counters[tile_id])
+                       : "memory");
           *flag = (prev == p.splits - 1);
-          if (*flag) __threadfence();   // acquire side
         }
         named_bar_sync(1, 128);
         if (*flag) {
@@ -451,7 +458,7 @@ size_t gemm_workspace_bytes(int M, int N, int K) {
 
 int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (a.M <= 0 || a.n1 <= a.n0) return 0;
-  if (a.K <= 0 || a.K % 8 || a.ldx % 8 || a.ldw % 8 || a.n0 < 0 || a.n1 > a.N) return LIGER_EINVAL;
+  if (a.K <= 0 || a.K % 8 || a.ldx % 8 || (!a.w_tiled && a.ldw % 8) || a.n0 < 0 || a.n1 > a.N) return LIGER_EINVAL;
   GemmPlan pl = gemm_plan(a.M, a.N, a.K);
   const int ntiles = (a.n1 - a.n0 + BM - 1) / BM;
   if (pl.splits > 1) {
@@ -460,7 +467,14 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
     if (a.ws_bytes < need || ntiles * pl.m_tiles > (int)(GEMM_COUNTER_BYTES / 4)) return LIGER_EINVAL;
   }
   CUtensorMap tA, tB;
-  int rc = make_map(&tA, a.w, a.N, a.K, a.ldw, BM);
+  int rc;
+  if (a.w_tiled) {
+    if (a.K % BK || a.n0 % BM) return LIGER_EINVAL;
+    const int64_t rows = (int64_t)((a.N + BM - 1) / BM) * (a.K / BK) * BM;
+    rc = make_map(&tA, a.w, rows, BK, BK, BM);
+  } else {
+    rc = make_map(&tA, a.w, a.N, a.K, a.ldw, BM);
+  }
   if (rc) return rc;
   rc = make_map(&tB, a.x, a.M, a.K, a.ldx, pl.bn);
   if (rc) return rc;
@@ -477,6 +491,8 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.out = a.out; p.ldo = a.ldo; p.out_f32 = a.out_f32;
   p.counters = reinterpret_cast<int*>(a.workspace);
   p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
+  p.w_tiled = a.w_tiled;
+  p.nkb_total = (a.K + BK - 1) / BK;
   p.n_tiles = ntiles;
   p.m_tiles = pl.m_tiles;
   p.units = ntiles * pl.m_tiles * pl.splits;

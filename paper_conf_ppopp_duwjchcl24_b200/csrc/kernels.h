@@ -30,6 +30,7 @@ struct GemmArgs {
   int out_f32;
   void* workspace;
   size_t ws_bytes;
+  int w_tiled;   // 0: W row-major [N, K] (row stride ldw); 1: tiled [ceil(N/128)][K/64][128][64]
 };
 
 GemmPlan gemm_plan(int M, int N, int K);
@@ -55,5 +56,10 @@ int c0_fill_launch(void* dst, int rows, int cols, int64_t ld, uint64_t seed, uin
                    int64_t col_off, int64_t idx_row_stride, int64_t idx_col_stride, int exp, int kind,
                    cudaStream_t stream);
 int copy_tokens_launch(const int32_t* src, int32_t* dst, int n, cudaStream_t stream);
+int tile_weight_launch(const void* src, int64_t ld, void* dst, int N, int K, cudaStream_t stream);
+// storage offset (elements) of logical W[n, k] in the tiled layout
+inline __host__ __device__ int64_t tiled_offset(int n, int k, int K) {
+  return (((int64_t)(n >> 7) * (K >> 6) + (k >> 6)) << 13) + ((n & 127) << 6) + (k & 63);
+}
 
 }  // namespace liger

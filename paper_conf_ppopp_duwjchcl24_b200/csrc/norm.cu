@@ -255,12 +255,13 @@ __device__ __forceinline__ uint64_t mix64_dev(uint64_t x) {
 }
 
 __global__ void c0_fill_kernel(__nv_bfloat16* dst, int rows, int cols, int64_t ld, uint64_t base, int64_t row_off,
-                               int64_t col_off, int64_t irs, int64_t ics, float scale, int kind) {
+                               int64_t col_off, int64_t irs, int64_t ics, float scale, int kind, int tiled) {
   const int64_t total = (int64_t)rows * cols;
   for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
        t += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = t / cols, c = t % cols;
     const uint64_t idx = (uint64_t)((r + row_off) * irs + (c + col_off) * ics);
+    const int64_t dpos = tiled ? tiled_offset((int)(r + ld), (int)c, cols) : r * ld + c;   // tiled: ld = first row
     const uint64_t u = mix64_dev(base + idx);
     const int32_t iv = (int32_t)(u >> 40) - (1 << 23);
     const float v = (float)iv * (1.0f / 8388608.0f);
@@ -268,7 +269,7 @@ __global__ void c0_fill_kernel(__nv_bfloat16* dst, int rows, int cols, int64_t l
     if (kind == 1) w = __fadd_rn(1.0f, __fmul_rn(v, 0.0625f));
     else if (kind == 2) w = __fmul_rn(v, 0.0625f);
     else w = __fmul_rn(v, scale);
-    dst[r * ld + c] = __float2bfloat16_rn(w);
+    dst[dpos] = __float2bfloat16_rn(w);
   }
 }
 
@@ -282,8 +283,25 @@ int c0_fill_launch(void* dst, int rows, int cols, int64_t ld, uint64_t seed, uin
   const int64_t total = (int64_t)rows * cols;
   int blocks = (int)((total + 255) / 256);
   if (blocks > 148 * 32) blocks = 148 * 32;
+  const int tiled = (kind & LIGER_C0_TILED) ? 1 : 0;   // dst in the tiled GEMM weight layout
+  if (tiled && cols % 64) return LIGER_EINVAL;
   c0_fill_kernel<<<blocks, 256, 0, stream>>>((__nv_bfloat16*)dst, rows, cols, ld, base, row_off, col_off,
-                                             idx_row_stride, idx_col_stride, scale, kind);
+                                             idx_row_stride, idx_col_stride, scale, kind & 3, tiled);
+  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
+// row-major [N, K] (row stride ld) -> tiled [ceil(N/128)][K/64][128][64] (padding rows zero)
+__global__ void tile_weight_kernel(const __nv_bfloat16* src, int64_t ld, __nv_bfloat16* dst, int N, int K) {
+  const int64_t npad = (int64_t)(N + 127) / 128 * 128;
+  const int64_t total = npad * K;
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int n = (int)(t / K), k = (int)(t % K);
+    dst[tiled_offset(n, k, K)] = n < N ? src[(int64_t)n * ld + k] : __float2bfloat16_rn(0.f);
+  }
+}
+int tile_weight_launch(const void* src, int64_t ld, void* dst, int N, int K, cudaStream_t stream) {
+  if (K % 64 || N <= 0) return LIGER_EINVAL;
+  tile_weight_kernel<<<148 * 8, 256, 0, stream>>>((const __nv_bfloat16*)src, ld, (__nv_bfloat16*)dst, N, K);
   return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
 }
 

@@ -62,6 +62,8 @@ _SIGS = {
     "liger_last_error": (C.c_char_p, [_P]),
     "liger_finalize": (_I, [_P]),
     "liger_op_gemm": (_I, [_P, _I64, _P, _I64, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),
+    "liger_op_gemm_tiled": (_I, [_P, _I64, _P, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),
+    "liger_op_tile_weight": (_I, [_P, _I64, _P, _I, _I, _P]),
     "liger_gemm_workspace_bytes": (_SZ, [_I, _I, _I]),
     "liger_gemm_plan": (_I, [_I, _I, _I, _P]),
     "liger_op_add_layernorm": (_I, [_P, _P, _P, _P, _P, _P, _P, _I, _I, _I, _I, _F, _P]),
@@ -130,6 +132,27 @@ def gemm(x, w, out, *, n0=0, n1=None, bias=None, act="none", scale_cols=0, scale
     check(lib().liger_op_gemm(_p(x), x.stride(0), _p(w), w.stride(0), _p(out), out.stride(0), M, N, K, n0, n1,
                               _p(bias), ACT[act], scale_cols, scale, out_f32, _p(workspace), ws_b, _s(stream)),
           what="liger_op_gemm")
+
+
+def gemm_tiled(x, w_tiled, out, *, N, n0=0, n1=None, bias=None, act="none", scale_cols=0, scale=1.0,
+               workspace=None, stream=None):
+    """W given in the tiled layout (see tile_weight)."""
+    M, K = x.shape
+    n1 = N if n1 is None else n1
+    out_f32 = 1 if out.element_size() == 4 else 0
+    ws_b = workspace.numel() * workspace.element_size() if workspace is not None else 0
+    check(lib().liger_op_gemm_tiled(_p(x), x.stride(0), _p(w_tiled), _p(out), out.stride(0), M, N, K, n0, n1,
+                                    _p(bias), ACT[act], scale_cols, scale, out_f32, _p(workspace), ws_b,
+                                    _s(stream)), what="liger_op_gemm_tiled")
+
+
+def tile_weight(w, w_tiled, stream=None):
+    N, K = w.shape
+    check(lib().liger_op_tile_weight(_p(w), w.stride(0), _p(w_tiled), N, K, _s(stream)), what="liger_op_tile_weight")
+
+
+def tiled_numel(N, K):
+    return (N + 127) // 128 * 128 * K
 
 
 def gemm_workspace_bytes(M, N, K):

@@ -104,6 +104,41 @@ def test_gemm_full_size_sampled(L, name, M):
         assert rel <= REL, (kind, rel)
 
 
+@pytest.mark.parametrize("M,N,K", [(2, 384, 256), (8, 1280, 1024), (300, 640, 512), (16, 5120, 2560)])
+def test_gemm_tiled_layout_bit_exact(L, M, N, K):
+    """The tiled weight layout (each 128x64 TMA box contiguous) computes exactly the
+    bits of the row-major layout, for the full GEMM and for 128-aligned slices."""
+    x = bf16_dev(c0_values(6, 1, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K))
+    w = bf16_dev(c0_values(6, 2, np.arange(N * K, dtype=np.uint64), -5).reshape(N, K))
+    b = bf16_dev(c0_values(6, 3, np.arange(N, dtype=np.uint64), -4))
+    wt = torch.empty(L.tiled_numel(N, K), dtype=torch.bfloat16, device="cuda")
+    L.tile_weight(w, wt)
+    ws = workspace(L.gemm_workspace_bytes(M, N, K))
+    ref = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
+    L.gemm(x, w, ref, bias=b, act="relu", workspace=ws)
+    got = torch.zeros_like(ref)
+    L.gemm_tiled(x, wt, got, N=N, bias=b, act="relu", workspace=ws)
+    sl = torch.zeros_like(ref)
+    for c0 in range(0, N, 256):
+        L.gemm_tiled(x, wt, sl, N=N, n0=c0, n1=min(N, c0 + 256), bias=b, act="relu", workspace=ws)
+    torch.cuda.synchronize()
+    assert torch.equal(got, ref) and torch.equal(sl, ref)
+
+
+def test_c0_tiled_fill_matches_tile_weight(L):
+    from liger_inputs import weight_exp
+    N, K = 384, 256
+    rm = torch.empty(N, K, dtype=torch.bfloat16, device="cuda")
+    L.c0_fill(rm, seed=1, tensor_id=5, idx_row_stride=1, idx_col_stride=N, exp=weight_exp(K))
+    t1 = torch.empty(L.tiled_numel(N, K), dtype=torch.bfloat16, device="cuda")
+    L.tile_weight(rm, t1)
+    t2 = torch.zeros_like(t1)
+    for r0 in (0, 128, 256):     # fill in three row blocks (first destination row r0)
+        L.lib().liger_op_c0_fill(L._p(t2), 128, K, r0, 1, 5, r0, 0, 1, N, weight_exp(K), 16, None)
+    torch.cuda.synchronize()
+    assert torch.equal(t1, t2)
+
+
 def test_gemm_empty_and_errors(L):
     x = torch.zeros(0, 64, dtype=torch.bfloat16, device="cuda")
     w = torch.zeros(128, 64, dtype=torch.bfloat16, device="cuda")

@@ -20,13 +20,19 @@ h, f = 5120, 20480
 for M in (2, 8, 32, 256, 512, 1024, 4096):
     for (N, K, name) in ((3 * h, h, "qkv"), (h, h, "out"), (f, h, "fc1"), (h, f, "fc2")):
         copies = max(1, int(600e6 // (N * K * 2)))
-        ws_ = [(torch.randn(N, K, device=dev) / K ** 0.5).bfloat16() for _ in range(copies)]
+        ws_ = []
+        for _ in range(copies):
+            w = (torch.randn(N, K, device=dev) / K ** 0.5).bfloat16()
+            wt = torch.empty(L.tiled_numel(N, K), dtype=torch.bfloat16, device=dev)
+            L.tile_weight(w, wt)
+            ws_.append(wt)
+            del w
         x = torch.randn(M, K, device=dev).bfloat16()
         out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
         wsp = torch.zeros(max(L.gemm_workspace_bytes(M, N, K), 16384) // 4 + 16, dtype=torch.int32, device=dev)
         i = [0]
         def fn():
-            L.gemm(x, ws_[i[0] % copies], out, workspace=wsp); i[0] += 1
+            L.gemm_tiled(x, ws_[i[0] % copies], out, N=N, workspace=wsp); i[0] += 1
         t = timeit(fn)
         by = (N * K + M * K + M * N) * 2
         print(f"gemm {name:4s} M={M:5d} N={N:6d} K={K:6d}: {t*1e6:8.1f} us  {by/t/1e9:7.0f} GB/s ({by/t/1e9/HBM*100:4.1f}%)  {2*M*N*K/t/1e12:7.1f} TF/s ({2*M*N*K/t/1e12/TC*100:4.1f}%)")
