@@ -62,6 +62,7 @@ struct GemmParams {
   int units;            // n_tiles * m_tiles * splits
   int w_tiled;          // W stored as [N/128][K/64][128][64] (each TMA box contiguous)
   int nkb_total;        // K / 64
+
   const __nv_bfloat16* bias;
   int act;
   int scale_cols;
@@ -119,7 +120,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   uint64_t* tmem_full = bars + 2 * S;       // [TS]
   uint64_t* tmem_empty = bars + 2 * S + 4;  // [TS]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 8);
-  int* last_flag = reinterpret_cast<int*>(tmem_slot + 1);   // [2], alternating per unit
+
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -265,54 +266,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tmem_empty[acc]);
-      if (p.splits > 1) {
-        // Deterministic split-K: the last CTA to finish a tile's chunks sums the
-        // partials in chunk order 0..splits-1 (independent of who is last).
-        // Release: CTA barrier, then one gpu-scope fence + atomic (cumulative).
-        named_bar_sync(1, 128);
-        int* flag = last_flag + (lu & 1);
-        if (threadIdx.x == 64) {
-          // acq_rel atomic: releases this CTA's partial stores (ordered before it by
-          // the barrier; PTX release is cumulative) and acquires the other CTAs'.
-          int prev;
-          asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&p.counters[tile_id])
-                       : "memory");
-          *flag = (prev == p.splits - 1);
-        }
-        named_bar_sync(1, 128);
-        if (*flag) {
-          if (nval) {
-            const float* base = p.ws + (int64_t)tile_id * (BM * p.bn) + row;
-            const int64_t zstride = (int64_t)tiles * (BM * p.bn);
-            for (int c0 = 0; c0 < mcount; c0 += 16) {
-              float accv[16];
-#pragma unroll
-              for (int j = 0; j < 16; ++j) accv[j] = 0.f;
-              constexpr int UNR = 4;
-              for (int z0 = 0; z0 < p.splits; z0 += UNR) {
-                float ld[UNR][16];
-#pragma unroll
-                for (int zz = 0; zz < UNR; ++zz)
-#pragma unroll
-                  for (int j = 0; j < 16; ++j)
-                    ld[zz][j] = (z0 + zz < p.splits && c0 + j < mcount)
-                                    ? __ldcg(base + (z0 + zz) * zstride + (int64_t)(c0 + j) * BM)
-                                    : 0.f;
-#pragma unroll
-                for (int zz = 0; zz < UNR; ++zz)
-                  if (z0 + zz < p.splits) {   // sum in chunk order
-#pragma unroll
-                    for (int j = 0; j < 16; ++j) accv[j] += ld[zz][j];
-                  }
-              }
-#pragma unroll
-              for (int j = 0; j < 16; ++j)
-                if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, accv[j], n, bias_v));
-            }
-          }
-          if (threadIdx.x == 64) p.counters[tile_id] = 0;
-        }
-      }
     }
   }
   tc_fence_before();
@@ -320,6 +273,45 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc(tmem_base, tmem_cols);
+  }
+}
+
+// Split-K fixup: out[m, n] = epi( sum_{z=0..S-1} partial[z] ) in chunk order (the
+// same bits whatever slice or CTA produced each chunk).  One thread per (m, 4 rows n),
+// reading the column-major per-tile partials coalesced.
+__global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) {
+  grid_dependency_trigger();
+  grid_dependency_wait();
+  const int tiles = p.n_tiles * p.m_tiles;
+  const int64_t zstride = (int64_t)tiles * (BM * p.bn);
+  const int slice_w = p.n1 - p.n0;
+  const int64_t total = (int64_t)p.M * (BM / 4) * p.n_tiles;   // (m, tile row group of 4)
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int rq = (int)(t % (BM / 4));
+    const int64_t t2 = t / (BM / 4);
+    const int nt = (int)(t2 % p.n_tiles);
+    const int m = (int)(t2 / p.n_tiles);
+    const int mt = m / p.bn, col = m % p.bn;
+    const int tile_id = nt * p.m_tiles + mt;
+    const float4* src = reinterpret_cast<const float4*>(p.ws + (int64_t)tile_id * (BM * p.bn) + (int64_t)col * BM) + rq;
+    float4 acc = __ldcg(src);
+    for (int z = 1; z < p.splits; ++z) {
+      const float4 v = __ldcg(reinterpret_cast<const float4*>(reinterpret_cast<const float*>(src) + z * zstride));
+      acc.x += v.x;
+      acc.y += v.y;
+      acc.z += v.z;
+      acc.w += v.w;
+    }
+    const float a[4] = {acc.x, acc.y, acc.z, acc.w};
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int row = rq * 4 + i;
+      const int n = p.n0 + nt * BM + row;
+      if (nt * BM + row < slice_w && n < p.N) {
+        const float bias_v = p.bias ? __bfloat162float(p.bias[n]) : 0.0f;
+        epi_store(p, m, n, epi_apply(p, a[i], n, bias_v));
+      }
+    }
   }
 }
 
@@ -415,21 +407,22 @@ GemmPlan gemm_plan(int M, int N, int K) {
   bn = (bn + 15) / 16 * 16;
   if (bn < 16) bn = 16;
   const int tiles = n_tiles * mt;
-  // Split K only when the tiles alone leave SMs idle.  Cost = (units per CTA) x
-  // (k-blocks per unit + a fixed per-unit overhead), chunks of >= 4 k-blocks.
-  const double ovh = M <= 64 ? 4.0 : 12.0;
+  // Cost model in SM cycles: a k-block costs max(MMA = 8 bn, weight stream at
+  // ~23 B/clk/SM + activation tile from L2 at ~64 B/clk); a unit adds 300; a
+  // split adds the fixup kernel (launch + S*M*N*4 B of partial traffic x 2).
+  const double kb_time = fmax(8.0 * bn, A_BYTES / 23.0 + 128.0 * bn / 64.0);
   int best_s = 1;
-  double best = (double)((tiles + G - 1) / G) * (nkb + ovh);
-  if ((tiles < G || M <= 64) && tiles <= (int)(GEMM_COUNTER_BYTES / 4)) {
-    for (int sp = 2; sp <= nkb / 4; ++sp) {
-      const int kcb = (nkb + sp - 1) / sp;
-      const int S = (nkb + kcb - 1) / kcb;
-      if (S != sp) continue;
-      const double cost = (double)((tiles * S + G - 1) / G) * (kcb + ovh) + (M <= 64 ? 1.0 : 4.0) * S;
-      if (cost < best - 1e-9) {
-        best = cost;
-        best_s = S;
-      }
+  double best = 1e300;
+  for (int sp = 1; sp <= (nkb >= 8 ? nkb / 4 : 1); ++sp) {
+    const int kcb = (nkb + sp - 1) / sp;
+    const int S = (nkb + kcb - 1) / kcb;
+    if (S != sp) continue;
+    const double units = (double)tiles * S;
+    double cost = ceil(units / G) * (kcb * kb_time + 300.0);
+    if (S > 1) cost += 3000.0 + (double)S * M * N * 8.0 / 2600.0;
+    if (cost < best - 1e-9) {
+      best = cost;
+      best_s = S;
     }
   }
   if (const char* e = getenv("LIGER_GEMM_FORCE_SPLITS")) {   // experiments only
@@ -464,7 +457,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (pl.splits > 1) {
     if (!a.workspace) return LIGER_EINVAL;
     const size_t need = GEMM_COUNTER_BYTES + (size_t)pl.splits * ntiles * pl.m_tiles * BM * pl.bn * sizeof(float);
-    if (a.ws_bytes < need || ntiles * pl.m_tiles > (int)(GEMM_COUNTER_BYTES / 4)) return LIGER_EINVAL;
+    if (a.ws_bytes < need) return LIGER_EINVAL;
   }
   CUtensorMap tA, tB;
   int rc;
@@ -492,12 +485,18 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.counters = reinterpret_cast<int*>(a.workspace);
   p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
   p.w_tiled = a.w_tiled;
+
   p.nkb_total = (a.K + BK - 1) / BK;
   p.n_tiles = ntiles;
   p.m_tiles = pl.m_tiles;
   p.units = ntiles * pl.m_tiles * pl.splits;
   const int grid = p.units < num_sms() ? p.units : num_sms();
-  return launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
+  int rc2 = launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
+  if (rc2 || p.splits == 1) return rc2 ? LIGER_ECUDA : 0;
+  const int64_t work = (int64_t)p.M * (BM / 4) * p.n_tiles;
+  int rblocks = (int)((work + 255) / 256);
+  if (rblocks > num_sms() * 8) rblocks = num_sms() * 8;
+  return launch_pdl(splitk_reduce_kernel, dim3(rblocks), dim3(256), 0, stream, p) ? LIGER_ECUDA : 0;
 }
 
 }  // namespace liger
