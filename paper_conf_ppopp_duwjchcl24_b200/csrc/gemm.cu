@@ -413,7 +413,10 @@ GemmPlan gemm_plan(int M, int N, int K) {
   const double kb_time = fmax(8.0 * bn, A_BYTES / 23.0 + 128.0 * bn / 64.0);
   int best_s = 1;
   double best = 1e300;
-  for (int sp = 1; sp <= (nkb >= 8 ? nkb / 4 : 1); ++sp) {
+  // Prefill GEMMs that already fill the SMs are not split (their fp32 partials
+  // would exceed L2); decode GEMMs always consider it.
+  const int smax = (M > 64 && tiles >= G) ? 1 : (nkb >= 8 ? nkb / 4 : 1);
+  for (int sp = 1; sp <= smax; ++sp) {
     const int kcb = (nkb + sp - 1) / sp;
     const int S = (nkb + kcb - 1) / kcb;
     if (S != sp) continue;
