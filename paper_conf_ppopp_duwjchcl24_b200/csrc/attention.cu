@@ -229,12 +229,16 @@ int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* 
 }
 
 // ================================================================== decode
-// CTA = (head, sequence, chunk of DC_CHUNK positions).  Phase 1: warp w scores
-// positions [w*32, w*32+32) of the chunk; a token's K row (d bf16) is spread over
-// LPT = d/8 lanes (16 B each) and every lane issues all of its K loads before the
-// first shuffle reduction (memory-level parallelism instead of a latency chain).
-// Phase 2: thread (slot, vec) accumulates p_t * V[t, vec*8 .. +8] over the
-// positions t = slot (mod SLOTS), again loading all V vectors first.
+// CTA = (head, sequence, chunk of DC_CHUNK positions), 128 threads.  Thread 0
+// stages the chunk's K and V page blocks (16 tokens x d bf16 = 4 KiB each,
+// contiguous in the paged pool) into shared memory with cp.async.bulk (TMA bulk
+// engine), all issued at once on one mbarrier, so a CTA pays one DRAM round
+// trip.  The new token (position pos) is taken from the qkv buffer (and
+// appended to its page by the last chunk's CTA).  Phase 1: warp w scores
+// positions [32w, 32w+32) (a token row spread over d/8 lanes, shuffle dot
+// products); two-pass softmax over the chunk; phase 2: thread (slot, vec)
+// accumulates p_t V[t] over positions t = slot (mod SLOTS).  Chunks of one
+// (sequence, head) are merged in chunk order by the last CTA (deterministic).
 constexpr int DC_CHUNK = 128;
 constexpr int DC_THREADS = 128;
 
@@ -267,13 +271,15 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   constexpr int SLOTS = DC_THREADS / NVEC;
   constexpr int PER = DC_CHUNK / SLOTS; // positions per thread in phase 2
   constexpr int NPG = DC_CHUNK / KVB;   // pages per chunk
+  extern __shared__ __align__(128) uint8_t dsm[];
+  __nv_bfloat16* sK = reinterpret_cast<__nv_bfloat16*>(dsm);
+  __nv_bfloat16* sV = sK + DC_CHUNK * D;
   __shared__ float sc[DC_CHUNK];
   __shared__ float red[DC_THREADS / 32];
   __shared__ float part[SLOTS][D];
-  __shared__ int pg[NPG];
+  __shared__ __align__(8) uint64_t bar;
   __shared__ int last;
 
-  pdl_enter();
   const int head = blockIdx.x, bi = blockIdx.y, sp = blockIdx.z, nsp = gridDim.z;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ctx = pos + 1;
@@ -284,46 +290,60 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   const __nv_bfloat16* knew = row + (int64_t)heads * D + head * D;
   const __nv_bfloat16* vnew = row + (int64_t)2 * heads * D + head * D;
   const int32_t* pt = page_table + (int64_t)bi * max_pages;
+  // cached positions of this chunk: [t0, min(t1, pos)) -- pages touching them
+  const int tc1 = min(t1, pos);
+  const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
 
-  if (tid < NPG) pg[tid] = (t0 + tid * KVB < ctx) ? pt[(t0 >> 4) + tid] : 0;
-  if (sp == nsp - 1 && tid < 2 * NVEC) {   // append the new token's K/V (position pos)
-    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
-    const int page = pt[pos / KVB];
-    *reinterpret_cast<uint4*>(kv_pool + kv_off(page, kv, heads, head, pos % KVB, D) + c) =
-        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
+  if (tid == 0) {
+    mbar_init(&bar, 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  pdl_enter();
+  if (tid == 0) {
+    mbar_arrive_expect_tx(&bar, (uint32_t)npg * 2 * KVB * D * 2);
+    for (int g = 0; g < npg; ++g) {
+      const int page = pt[(t0 >> 4) + g];
+      bulk_load(sK + g * KVB * D, kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &bar);
+      bulk_load(sV + g * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &bar);
+    }
   }
   float qf[8];
   {
     uint4 qv = *reinterpret_cast<const uint4*>(qp + (lane % LPT) * 8);
     bf16x8_to_f32(qv, qf);
   }
+  const bool has_new = (t0 <= pos && pos < t1);
+  if (has_new && tid < 2 * NVEC) {   // append the new token's K/V (position pos) to its page
+    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
+    const int page = pt[pos / KVB];
+    *reinterpret_cast<uint4*>(kv_pool + kv_off(page, kv, heads, head, pos % KVB, D) + c) =
+        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
+  }
+  mbar_wait(&bar, 0);
+  if (has_new && tid < 2 * NVEC) {   // ... and into the staged chunk (the bulk copy may predate it)
+    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
+    *reinterpret_cast<uint4*>((kv ? sV : sK) + (pos - t0) * D + c) =
+        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
+  }
   __syncthreads();
 
   // ---- phase 1: scores for positions [t0 + warp*32, +32)
   {
     const int c = (lane % LPT) * 8;
-    uint4 kr[STEPS];
 #pragma unroll
     for (int st = 0; st < STEPS; ++st) {
-      const int t = t0 + warp * 32 + st * TPW + lane / LPT;
-      kr[st] = make_uint4(0, 0, 0, 0);
-      if (t < t1) {
-        const __nv_bfloat16* kp =
-            (t == pos) ? knew + c : kv_pool + kv_off(pg[(t - t0) >> 4], 0, heads, head, t % KVB, D) + c;
-        kr[st] = *reinterpret_cast<const uint4*>(kp);
-      }
-    }
-#pragma unroll
-    for (int st = 0; st < STEPS; ++st) {
-      float f[8];
-      bf16x8_to_f32(kr[st], f);
+      const int lt = warp * 32 + st * TPW + lane / LPT;   // local position
       float dot = 0.f;
+      if (t0 + lt < t1) {
+        float f[8];
+        bf16x8_to_f32(*reinterpret_cast<const uint4*>(sK + lt * D + c), f);
 #pragma unroll
-      for (int i = 0; i < 8; ++i) dot += qf[i] * f[i];
+        for (int i = 0; i < 8; ++i) dot += qf[i] * f[i];
+      }
 #pragma unroll
       for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
-      const int t = t0 + warp * 32 + st * TPW + lane / LPT;
-      if (t < t1 && (lane % LPT) == 0) sc[t - t0] = dot;
+      if (t0 + lt < t1 && (lane % LPT) == 0) sc[lt] = dot;
     }
   }
   __syncthreads();
@@ -350,24 +370,13 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   // ---- phase 2: o = sum_t p_t v_t
   const int vec = tid % NVEC, slot = tid / NVEC;
   float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-  {
-    uint4 vr[PER];
-#pragma unroll
-    for (int i = 0; i < PER; ++i) {
-      const int t = t0 + slot + i * SLOTS;
-      vr[i] = make_uint4(0, 0, 0, 0);
-      if (t < t1) {
-        const __nv_bfloat16* vp =
-            (t == pos) ? vnew + vec * 8 : kv_pool + kv_off(pg[(t - t0) >> 4], 1, heads, head, t % KVB, D) + vec * 8;
-        vr[i] = *reinterpret_cast<const uint4*>(vp);
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < PER; ++i) {
-      const int t = t0 + slot + i * SLOTS;
-      const float pw = (t < t1) ? sc[t - t0] : 0.f;
+#pragma unroll 4
+  for (int i = 0; i < PER; ++i) {
+    const int lt = slot + i * SLOTS;
+    if (t0 + lt < t1) {
+      const float pw = sc[lt];
       float f[8];
-      bf16x8_to_f32(vr[i], f);
+      bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + vec * 8), f);
 #pragma unroll
       for (int e = 0; e < 8; ++e) acc[e] += pw * f[e];
     }
@@ -398,12 +407,14 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
     wp[D] = mx;
     wp[D + 1] = l;
   }
-  __threadfence();
   __syncthreads();
-  if (tid == 0) last = (atomicAdd(&counters[unit], 1) == nsp - 1);
+  if (tid == 0) {
+    int prev;
+    asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&counters[unit]) : "memory");
+    last = (prev == nsp - 1);
+  }
   __syncthreads();
   if (!last) return;
-  __threadfence();
   float M = -INFINITY;
   for (int s2 = 0; s2 < nsp; ++s2) M = fmaxf(M, __ldcg(&ws[(unit * nsp + s2) * (D + 2) + D]));
   float L = 0.f;
@@ -436,11 +447,18 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   float* ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
   dim3 grid(heads, b, ns);
   int rc;
+  const size_t dsmem = (size_t)2 * DC_CHUNK * d * 2;
+  static bool attr_dc = false;
+  if (!attr_dc) {
+    cudaFuncSetAttribute(attn_decode_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * DC_CHUNK * 128 * 2);
+    cudaFuncSetAttribute(attn_decode_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * DC_CHUNK * 64 * 2);
+    attr_dc = true;
+  }
   if (d == 128)
-    rc = launch_pdl(attn_decode_kernel<128>, grid, dim3(DC_THREADS), 0, stream, (const __nv_bfloat16*)qkv,
+    rc = launch_pdl(attn_decode_kernel<128>, grid, dim3(DC_THREADS), dsmem, stream, (const __nv_bfloat16*)qkv,
                     (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads, ws, counters);
   else if (d == 64)
-    rc = launch_pdl(attn_decode_kernel<64>, grid, dim3(DC_THREADS), 0, stream, (const __nv_bfloat16*)qkv,
+    rc = launch_pdl(attn_decode_kernel<64>, grid, dim3(DC_THREADS), dsmem, stream, (const __nv_bfloat16*)qkv,
                     (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads, ws, counters);
   else
     return LIGER_EINVAL;
