@@ -300,12 +300,13 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   }
   __syncthreads();
   pdl_enter();
-  if (tid == 0) {
-    mbar_arrive_expect_tx(&bar, (uint32_t)npg * 2 * KVB * D * 2);
-    for (int g = 0; g < npg; ++g) {
-      const int page = pt[(t0 >> 4) + g];
-      bulk_load(sK + g * KVB * D, kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &bar);
-      bulk_load(sV + g * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &bar);
+  if (warp == 0) {   // lane g stages page g (page ids loaded in parallel, not a serial chain)
+    if (lane == 0) mbar_arrive_expect_tx(&bar, (uint32_t)npg * 2 * KVB * D * 2);
+    __syncwarp();
+    if (lane < npg) {
+      const int page = pt[(t0 >> 4) + lane];
+      bulk_load(sK + lane * KVB * D, kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &bar);
+      bulk_load(sV + lane * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &bar);
     }
   }
   float qf[8];
