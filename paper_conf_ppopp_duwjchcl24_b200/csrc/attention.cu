@@ -239,7 +239,7 @@ int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* 
 // products); two-pass softmax over the chunk; phase 2: thread (slot, vec)
 // accumulates p_t V[t] over positions t = slot (mod SLOTS).  Chunks of one
 // (sequence, head) are merged in chunk order by the last CTA (deterministic).
-constexpr int DC_CHUNK = 128;
+constexpr int DC_CHUNK = 64;    // positions per CTA (32 KiB of K+V staged for d = 128)
 constexpr int DC_THREADS = 128;
 
 size_t attn_decode_workspace_bytes(int b, int heads, int d, int ctx) {
@@ -258,198 +258,181 @@ __device__ __forceinline__ void bf16x8_to_f32(const uint4& v, float* f) {
 }
 
 template <int D>
-struct DecodeSmem {
-  __nv_bfloat16 k[2][DC_CHUNK * D];
-  __nv_bfloat16 v[2][DC_CHUNK * D];
-};
-
-// Persistent: CTA i processes units i, i+G, ... where unit = (sequence, head,
-// chunk); two shared-memory stages, the K/V pages of unit j+1 are in flight
-// (TMA bulk) while unit j is computed.
-template <int D>
 __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bfloat16* __restrict__ qkv,
                                                                  __nv_bfloat16* __restrict__ o,
                                                                  __nv_bfloat16* __restrict__ kv_pool,
                                                                  const int32_t* __restrict__ page_table,
-                                                                 int max_pages, int pos, int heads, int b, int nsp,
-                                                                 float* ws, int* counters) {
+                                                                 int max_pages, int pos, int heads, float* ws,
+                                                                 int* counters) {
   constexpr int LPT = D / 8;            // lanes per token
   constexpr int TPW = 32 / LPT;         // tokens per warp step
-  constexpr int STEPS = 32 / TPW;       // steps for the warp's 32 positions
+  constexpr int WPOS = DC_CHUNK / 4;    // positions per warp in phase 1
+  constexpr int STEPS = WPOS / TPW;     // steps for the warp's positions
   constexpr int NVEC = D / 8;
   constexpr int SLOTS = DC_THREADS / NVEC;
   constexpr int PER = DC_CHUNK / SLOTS; // positions per thread in phase 2
+  constexpr int NPG = DC_CHUNK / KVB;   // pages per chunk
   extern __shared__ __align__(128) uint8_t dsm[];
-  DecodeSmem<D>& S = *reinterpret_cast<DecodeSmem<D>*>(dsm);
+  __nv_bfloat16* sK = reinterpret_cast<__nv_bfloat16*>(dsm);
+  __nv_bfloat16* sV = sK + DC_CHUNK * D;
   __shared__ float sc[DC_CHUNK];
   __shared__ float red[DC_THREADS / 32];
   __shared__ float part[SLOTS][D];
-  __shared__ __align__(8) uint64_t bar[2];
+  __shared__ __align__(8) uint64_t bar;
   __shared__ int last;
 
+  const int head = blockIdx.x, bi = blockIdx.y, sp = blockIdx.z, nsp = gridDim.z;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ctx = pos + 1;
-  const int units = b * heads * nsp;
-  const int G = gridDim.x;
+  const int t0 = sp * DC_CHUNK, t1 = min(ctx, t0 + DC_CHUNK);
   const int64_t ld = (int64_t)3 * heads * D;
+  const __nv_bfloat16* row = qkv + (int64_t)bi * ld;
+  const __nv_bfloat16* qp = row + head * D;
+  const __nv_bfloat16* knew = row + (int64_t)heads * D + head * D;
+  const __nv_bfloat16* vnew = row + (int64_t)2 * heads * D + head * D;
+  const int32_t* pt = page_table + (int64_t)bi * max_pages;
+  // cached positions of this chunk: [t0, min(t1, pos)) -- pages touching them
+  const int tc1 = min(t1, pos);
+  const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
 
   if (tid == 0) {
-    mbar_init(&bar[0], 1);
-    mbar_init(&bar[1], 1);
+    mbar_init(&bar, 1);
     fence_barrier_init();
   }
   __syncthreads();
   pdl_enter();
-
-  // stage the cached K/V pages of unit u into buffer st (warp 0; lane g -> page g)
-  auto issue = [&](int u, int st) {
-    const int sp = u % nsp, hb = u / nsp, head = hb % heads, bi = hb / heads;
-    const int t0 = sp * DC_CHUNK, tc1 = min(min(ctx, t0 + DC_CHUNK), pos);
-    const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
-    if (lane == 0) mbar_arrive_expect_tx(&bar[st], (uint32_t)npg * 2 * KVB * D * 2);
+  if (warp == 0) {   // lane g stages page g (page ids loaded in parallel, not a serial chain)
+    if (lane == 0) mbar_arrive_expect_tx(&bar, (uint32_t)npg * 2 * KVB * D * 2);
     __syncwarp();
     if (lane < npg) {
-      const int page = page_table[(int64_t)bi * max_pages + (t0 >> 4) + lane];
-      bulk_load(S.k[st] + lane * KVB * D, kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &bar[st]);
-      bulk_load(S.v[st] + lane * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &bar[st]);
+      const int page = pt[(t0 >> 4) + lane];
+      bulk_load(sK + lane * KVB * D, kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &bar);
+      bulk_load(sV + lane * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &bar);
     }
-  };
-  if (warp == 0 && (int)blockIdx.x < units) issue(blockIdx.x, 0);
-
-  int j = 0;
-  for (int u = blockIdx.x; u < units; u += G, ++j) {
-    const int st = j & 1;
-    const uint32_t ph = (j >> 1) & 1;
-    if (warp == 0 && u + G < units) issue(u + G, st ^ 1);   // prefetch the next unit
-    const int sp = u % nsp, hb = u / nsp, head = hb % heads, bi = hb / heads;
-    const int t0 = sp * DC_CHUNK, t1 = min(ctx, t0 + DC_CHUNK);
-    const __nv_bfloat16* row = qkv + (int64_t)bi * ld;
-    const __nv_bfloat16* knew = row + (int64_t)heads * D + head * D;
-    const __nv_bfloat16* vnew = row + (int64_t)2 * heads * D + head * D;
-    __nv_bfloat16* sK = S.k[st];
-    __nv_bfloat16* sV = S.v[st];
-    float qf[8];
-    bf16x8_to_f32(*reinterpret_cast<const uint4*>(row + head * D + (lane % LPT) * 8), qf);
-    const bool has_new = (t0 <= pos && pos < t1);
-    if (has_new && tid < 2 * NVEC) {   // append the new token's K/V (position pos) to its page
-      const int kv = tid / NVEC, c = (tid % NVEC) * 8;
-      const int page = page_table[(int64_t)bi * max_pages + pos / KVB];
-      *reinterpret_cast<uint4*>(kv_pool + kv_off(page, kv, heads, head, pos % KVB, D) + c) =
-          *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
-    }
-    mbar_wait(&bar[st], ph);
-    if (has_new && tid < 2 * NVEC) {   // ... and into the staged chunk
-      const int kv = tid / NVEC, c = (tid % NVEC) * 8;
-      *reinterpret_cast<uint4*>((kv ? sV : sK) + (pos - t0) * D + c) =
-          *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
-    }
-    __syncthreads();
-    // ---- phase 1: scores
-    {
-      const int c = (lane % LPT) * 8;
-#pragma unroll
-      for (int stp = 0; stp < STEPS; ++stp) {
-        const int lt = warp * 32 + stp * TPW + lane / LPT;
-        float dot = 0.f;
-        if (t0 + lt < t1) {
-          float f[8];
-          bf16x8_to_f32(*reinterpret_cast<const uint4*>(sK + lt * D + c), f);
-#pragma unroll
-          for (int i = 0; i < 8; ++i) dot += qf[i] * f[i];
-        }
-#pragma unroll
-        for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
-        if (t0 + lt < t1 && (lane % LPT) == 0) sc[lt] = dot;
-      }
-    }
-    __syncthreads();
-    const int n = t1 - t0;
-    float mx = (tid < n) ? sc[tid] : -INFINITY;
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
-    if (lane == 0) red[warp] = mx;
-    __syncthreads();
-    mx = fmaxf(fmaxf(red[0], red[1]), fmaxf(red[2], red[3]));
-    __syncthreads();
-    float p_t = 0.f;
-    if (tid < n) {
-      p_t = __expf(sc[tid] - mx);
-      sc[tid] = p_t;
-    }
-    float sum = p_t;
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
-    if (lane == 0) red[warp] = sum;
-    __syncthreads();
-    const float l = red[0] + red[1] + red[2] + red[3];
-    // ---- phase 2: o = sum_t p_t v_t
-    const int vec = tid % NVEC, slot = tid / NVEC;
-    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-#pragma unroll 4
-    for (int i = 0; i < PER; ++i) {
-      const int lt = slot + i * SLOTS;
-      if (t0 + lt < t1) {
-        const float pw = sc[lt];
-        float f[8];
-        bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + vec * 8), f);
-#pragma unroll
-        for (int e = 0; e < 8; ++e) acc[e] += pw * f[e];
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < 8; ++i) part[slot][vec * 8 + i] = acc[i];
-    __syncthreads();
-    // stage st is free again (its data has been read into registers / part)
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    if (nsp == 1) {
-      for (int e = tid; e < D; e += DC_THREADS) {
-        float a = 0.f;
-#pragma unroll
-        for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
-        o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / l);
-      }
-    } else {
-      // partial (m, l, acc[D]); the last CTA of this (sequence, head) merges in chunk order
-      const int64_t un = (int64_t)bi * heads + head;
-      float* wp = ws + (un * nsp + sp) * (D + 2);
-      for (int e = tid; e < D; e += DC_THREADS) {
-        float a = 0.f;
-#pragma unroll
-        for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
-        wp[e] = a;
-      }
-      if (tid == 0) {
-        wp[D] = mx;
-        wp[D + 1] = l;
-      }
-      __syncthreads();
-      if (tid == 0) {
-        int prev;
-        asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&counters[un]) : "memory");
-        last = (prev == nsp - 1);
-      }
-      __syncthreads();
-      if (last) {
-        float M = -INFINITY;
-        for (int s2 = 0; s2 < nsp; ++s2) M = fmaxf(M, __ldcg(&ws[(un * nsp + s2) * (D + 2) + D]));
-        float L = 0.f;
-        for (int s2 = 0; s2 < nsp; ++s2) {
-          const float* w2 = ws + (un * nsp + s2) * (D + 2);
-          L += __ldcg(&w2[D + 1]) * __expf(__ldcg(&w2[D]) - M);
-        }
-        for (int e = tid; e < D; e += DC_THREADS) {
-          float a = 0.f;
-          for (int s2 = 0; s2 < nsp; ++s2) {
-            const float* w2 = ws + (un * nsp + s2) * (D + 2);
-            a += __ldcg(&w2[e]) * __expf(__ldcg(&w2[D]) - M);
-          }
-          o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / L);
-        }
-        if (tid == 0) counters[un] = 0;
-      }
-    }
-    __syncthreads();   // sc / part / last reused by the next unit
   }
+  float qf[8];
+  {
+    uint4 qv = *reinterpret_cast<const uint4*>(qp + (lane % LPT) * 8);
+    bf16x8_to_f32(qv, qf);
+  }
+  const bool has_new = (t0 <= pos && pos < t1);
+  if (has_new && tid < 2 * NVEC) {   // append the new token's K/V (position pos) to its page
+    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
+    const int page = pt[pos / KVB];
+    *reinterpret_cast<uint4*>(kv_pool + kv_off(page, kv, heads, head, pos % KVB, D) + c) =
+        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
+  }
+  mbar_wait(&bar, 0);
+  if (has_new && tid < 2 * NVEC) {   // ... and into the staged chunk (the bulk copy may predate it)
+    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
+    *reinterpret_cast<uint4*>((kv ? sV : sK) + (pos - t0) * D + c) =
+        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
+  }
+  __syncthreads();
+
+  // ---- phase 1: scores for positions [t0 + warp*WPOS, +WPOS)
+  {
+    const int c = (lane % LPT) * 8;
+#pragma unroll
+    for (int st = 0; st < STEPS; ++st) {
+      const int lt = warp * WPOS + st * TPW + lane / LPT;   // local position
+      float dot = 0.f;
+      if (t0 + lt < t1) {
+        float f[8];
+        bf16x8_to_f32(*reinterpret_cast<const uint4*>(sK + lt * D + c), f);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) dot += qf[i] * f[i];
+      }
+#pragma unroll
+      for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
+      if (t0 + lt < t1 && (lane % LPT) == 0) sc[lt] = dot;
+    }
+  }
+  __syncthreads();
+  const int n = t1 - t0;
+  float mx = (tid < n) ? sc[tid] : -INFINITY;   // n <= DC_CHUNK <= DC_THREADS
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+  if (lane == 0) red[warp] = mx;
+  __syncthreads();
+  mx = fmaxf(fmaxf(red[0], red[1]), fmaxf(red[2], red[3]));
+  __syncthreads();
+  float p_t = 0.f;
+  if (tid < n) {
+    p_t = __expf(sc[tid] - mx);
+    sc[tid] = p_t;
+  }
+  float sum = p_t;
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
+  if (lane == 0) red[warp] = sum;
+  __syncthreads();
+  const float l = red[0] + red[1] + red[2] + red[3];
+
+  // ---- phase 2: o = sum_t p_t v_t
+  const int vec = tid % NVEC, slot = tid / NVEC;
+  float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll 4
+  for (int i = 0; i < PER; ++i) {
+    const int lt = slot + i * SLOTS;
+    if (t0 + lt < t1) {
+      const float pw = sc[lt];
+      float f[8];
+      bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + vec * 8), f);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] += pw * f[e];
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) part[slot][vec * 8 + i] = acc[i];
+  __syncthreads();
+
+  if (nsp == 1) {
+    for (int e = tid; e < D; e += DC_THREADS) {
+      float a = 0.f;
+#pragma unroll
+      for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
+      o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / l);
+    }
+    return;
+  }
+  // split: write partial (m, l, acc[D]); the last CTA merges in chunk order
+  const int64_t unit = (int64_t)bi * heads + head;
+  float* wp = ws + (unit * nsp + sp) * (D + 2);
+  for (int e = tid; e < D; e += DC_THREADS) {
+    float a = 0.f;
+#pragma unroll
+    for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
+    wp[e] = a;
+  }
+  if (tid == 0) {
+    wp[D] = mx;
+    wp[D + 1] = l;
+  }
+  __syncthreads();
+  if (tid == 0) {
+    int prev;
+    asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&counters[unit]) : "memory");
+    last = (prev == nsp - 1);
+  }
+  __syncthreads();
+  if (!last) return;
+  float M = -INFINITY;
+  for (int s2 = 0; s2 < nsp; ++s2) M = fmaxf(M, __ldcg(&ws[(unit * nsp + s2) * (D + 2) + D]));
+  float L = 0.f;
+  for (int s2 = 0; s2 < nsp; ++s2) {
+    const float* w2 = ws + (unit * nsp + s2) * (D + 2);
+    L += __ldcg(&w2[D + 1]) * __expf(__ldcg(&w2[D]) - M);
+  }
+  for (int e = tid; e < D; e += DC_THREADS) {
+    float a = 0.f;
+    for (int s2 = 0; s2 < nsp; ++s2) {
+      const float* w2 = ws + (unit * nsp + s2) * (D + 2);
+      a += __ldcg(&w2[e]) * __expf(__ldcg(&w2[D]) - M);
+    }
+    o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / L);
+  }
+  if (tid == 0) counters[unit] = 0;
 }
 
 int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
@@ -464,31 +447,21 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   }
   int* counters = (int*)workspace;
   float* ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
-  static int nsm = 0;
-  if (!nsm) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  }
-  const int units = b * heads * ns;
-  const size_t dsmem = (size_t)2 * 2 * DC_CHUNK * d * 2;   // 2 stages x (K, V)
+  dim3 grid(heads, b, ns);
+  int rc;
+  const size_t dsmem = (size_t)2 * DC_CHUNK * d * 2;
   static bool attr_dc = false;
   if (!attr_dc) {
-    cudaFuncSetAttribute(attn_decode_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * DC_CHUNK * 128 * 2);
-    cudaFuncSetAttribute(attn_decode_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * DC_CHUNK * 64 * 2);
+    cudaFuncSetAttribute(attn_decode_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * DC_CHUNK * 128 * 2);
+    cudaFuncSetAttribute(attn_decode_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * DC_CHUNK * 64 * 2);
     attr_dc = true;
   }
-  const int per_sm = d == 128 ? 1 : 3;
-  const int grid = units < nsm * per_sm ? units : nsm * per_sm;
-  int rc;
   if (d == 128)
-    rc = launch_pdl(attn_decode_kernel<128>, dim3(grid), dim3(DC_THREADS), dsmem, stream, (const __nv_bfloat16*)qkv,
-                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads, b, ns, ws,
-                    counters);
+    rc = launch_pdl(attn_decode_kernel<128>, grid, dim3(DC_THREADS), dsmem, stream, (const __nv_bfloat16*)qkv,
+                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads, ws, counters);
   else if (d == 64)
-    rc = launch_pdl(attn_decode_kernel<64>, dim3(grid), dim3(DC_THREADS), dsmem, stream, (const __nv_bfloat16*)qkv,
-                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads, b, ns, ws,
-                    counters);
+    rc = launch_pdl(attn_decode_kernel<64>, grid, dim3(DC_THREADS), dsmem, stream, (const __nv_bfloat16*)qkv,
+                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads, ws, counters);
   else
     return LIGER_EINVAL;
   return rc ? LIGER_ECUDA : 0;
