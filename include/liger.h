@@ -263,16 +263,21 @@ int liger_op_c0_fill(void* dst, int rows, int cols, int64_t ld, uint64_t seed, u
                      int kind, void* stream);
 
 /* ------------------------------------------------------------------ host-only scheduler (no GPU needed)
- * Algorithm 1 planner exposed for CPU tests of the host logic.  A planner
- * holds batches of kernels (type 0 = compute, 1 = communication) with
- * per-piece durations; liger_plan_round runs one round and writes up to cap
- * entries {batch, kernel index, unit begin, unit end, subset (0/1)}. */
+ * Algorithm 1 planner (§3.4, readings R1-R5 of DESIGN.md)
+ * exposed for CPU tests of the host logic; the engine runs the same plan_round.
+ * liger_planner_submit: one batch of n_kernels kernels, types[i] 0 = compute,
+ * 1 = communication, units[i] = pieces (1 = not decomposable, else F), durs =
+ * concatenation over kernels of units[i] durations (duration of a k-unit piece,
+ * k = 1..units[i]).  liger_plan_round: update_list() + one round; writes
+ * *n_out entries {batch, kernel index, unit begin, unit end, subset (0/1)}
+ * (LIGER_EINVAL if more than cap), the round's type and SubSet0 time; returns
+ * LIGER_OK, or LIGER_IDLE when nothing is left. */
 typedef struct liger_planner liger_planner;
 int liger_planner_create(int list_size, double cf, liger_planner** out);
 int liger_planner_submit(liger_planner* p, int64_t batch, int n_kernels, const int32_t* types,
                          const int32_t* units, const double* durs /* per kernel: units entries */);
-int liger_plan_round(liger_planner* p, int32_t* entries /* [cap][5] */, int cap, int32_t* round_type,
-                     double* time0);
+int liger_plan_round(liger_planner* p, int32_t* entries /* [cap][5] */, int cap, int32_t* n_out,
+                     int32_t* round_type, double* time0);
 int liger_planner_destroy(liger_planner* p);
 
 #ifdef __cplusplus

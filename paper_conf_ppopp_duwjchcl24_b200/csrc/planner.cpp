@@ -127,8 +127,10 @@ int liger_planner_submit(liger_planner* p, int64_t batch, int n_kernels, const i
 }
 
 // entries: [cap][5] = {batch, kernel index, unit begin, unit end, subset}
-int liger_plan_round(liger_planner* p, int32_t* entries, int cap, int32_t* round_type, double* time0) {
+int liger_plan_round(liger_planner* p, int32_t* entries, int cap, int32_t* n_out, int32_t* round_type,
+                     double* time0) {
   if (!p) return LIGER_EINVAL;
+  if (n_out) *n_out = 0;
   // update_list(): drop exhausted batches, admit FIFO from the waiting queue
   std::vector<std::unique_ptr<ListCursor>> keep;
   for (auto& c : p->processing)
@@ -159,7 +161,8 @@ int liger_plan_round(liger_planner* p, int32_t* entries, int cap, int32_t* round
   for (auto& pp : r.sub1) emit(pp, 1);
   if (round_type) *round_type = r.type;
   if (time0) *time0 = r.time0;
-  return n;
+  if (n_out) *n_out = n;
+  return n <= cap ? LIGER_OK : LIGER_EINVAL;
 }
 
 int liger_planner_destroy(liger_planner* p) {

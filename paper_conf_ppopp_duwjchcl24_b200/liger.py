@@ -75,7 +75,7 @@ _SIGS = {
     "liger_op_c0_fill": (_I, [_P, _I, _I, _I64, _U64, _U64, _I64, _I64, _I64, _I64, _I, _I, _P]),
     "liger_planner_create": (_I, [_I, _D, C.POINTER(_P)]),
     "liger_planner_submit": (_I, [_P, _I64, _I, _P, _P, _P]),
-    "liger_plan_round": (_I, [_P, _P, _I, _P, _P]),
+    "liger_plan_round": (_I, [_P, _P, _I, _P, _P, _P]),
     "liger_planner_destroy": (_I, [_P]),
 }
 

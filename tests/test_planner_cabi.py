@@ -1,0 +1,191 @@
+"""The product's Algorithm 1 planner (C++, libliger.so `liger_plan_round`) against
+the oracle planner (oracle/scheduler.py) -- host logic only, no GPU (task ③:
+"-m 'not gpu' tests cover ... the host logic").  Also checks the library loads
+on a CPU-only host and exports every symbol include/liger.h declares."""
+import ctypes as C
+import os
+import random
+import re
+
+import pytest
+
+from oracle.scheduler import Kernel, Scheduler
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def L():
+    from paper_conf_ppopp_duwjchcl24_b200 import liger
+    if not os.path.exists(liger.LIB_PATH):
+        from paper_conf_ppopp_duwjchcl24_b200 import build
+        build.build()
+    liger.lib()
+    return liger
+
+
+def test_library_exports_every_header_symbol(L):
+    hdr = open(os.path.join(ROOT, "include", "liger.h")).read()
+    names = set(re.findall(r"\b(liger_[a-z0-9_]+)\s*\(", hdr))
+    names -= {"liger_ctx", "liger_cfg", "liger_result", "liger_stats_t", "liger_planner"}
+    lib = C.CDLL(L.LIB_PATH)
+    missing = [n for n in sorted(names) if not hasattr(lib, n)]
+    assert not missing, missing
+    assert set(L.exported_symbols()) <= names | {"liger_gemm_plan"}
+    assert L.missing_symbols() == []
+
+
+def test_compute_entry_points_fail_loudly_without_gpu(L):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    rc = L.lib().liger_op_argmax(None, 0, 1, 1, 0, None, None, None)
+    assert rc == -1004          # LIGER_ENODEV: no CPU fallback
+    assert b"no sm_100" in L.lib().liger_last_error(None)
+
+
+class CPlanner:
+    def __init__(self, L, list_size, cf):
+        self.L = L
+        self.p = C.c_void_p()
+        assert L.lib().liger_planner_create(list_size, cf, C.byref(self.p)) == 0
+
+    def submit(self, bid, kernels):
+        n = len(kernels)
+        types = (C.c_int32 * n)(*[0 if k.type == "C" else 1 for k in kernels])
+        units = (C.c_int32 * n)(*[k.units for k in kernels])
+        flat = [d for k in kernels for d in k.durs]
+        durs = (C.c_double * len(flat))(*flat)
+        assert self.L.lib().liger_planner_submit(self.p, bid, n, types, units, durs) == 0
+
+    def round(self):
+        cap = 4096
+        ent = (C.c_int32 * (5 * cap))()
+        typ = C.c_int32()
+        t0 = C.c_double()
+        nn = C.c_int32()
+        rc = self.L.lib().liger_plan_round(self.p, ent, cap, C.byref(nn), C.byref(typ), C.byref(t0))
+        if rc == 2:   # LIGER_IDLE
+            return None
+        assert rc == 0
+        n = nn.value
+        rows = [tuple(ent[5 * i:5 * i + 5]) for i in range(n)]
+        return rows, ("C" if typ.value == 0 else "M"), t0.value
+
+    def close(self):
+        self.L.lib().liger_planner_destroy(self.p)
+
+
+def _batch(rng, bid, F):
+    ks = []
+    for _ in range(rng.randint(1, 3)):
+        for name, typ, dec in (("LN", "C", False), ("QKV", "C", True), ("attn", "C", False), ("out", "C", True),
+                               ("AR1", "M", True), ("LN2", "C", False), ("FC1", "C", True), ("FC2", "C", True),
+                               ("AR2", "M", True)):
+            d = rng.uniform(1, 100)
+            durs = tuple(d * (0.1 + 0.9 * k / F) for k in range(1, F + 1)) if dec else (d,)
+            ks.append(Kernel(bid, name, typ, durs, decomposable=dec))
+    return ks
+
+
+def _copy(ks):
+    return [Kernel(k.batch, k.name, k.type, k.durs, k.decomposable) for k in ks]
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_cpp_planner_matches_oracle(L, seed):
+    rng = random.Random(seed)
+    F = rng.choice([1, 2, 4, 8, 16])
+    cf = rng.choice([1.0, 1.1, 1.15, 1.3])
+    size = rng.randint(1, 4)
+    batches = [_batch(rng, b, F) for b in range(rng.randint(1, 5))]
+    orc = Scheduler(list_size=size, cf=cf)
+    cp = CPlanner(L, size, cf)
+    idx = {}
+    for b, ks in enumerate(batches):
+        orc.submit(b, _copy(ks))
+        cp.submit(b, ks)
+        for i, k in enumerate(ks):
+            idx[(b, i)] = k.name
+    while True:
+        ro = orc.step()
+        rc = cp.round()
+        if ro is None:
+            assert rc is None
+            break
+        rows, typ, t0 = rc
+        assert typ == ro.type and t0 == pytest.approx(ro.time0)
+        want = [(p.batch, p.name, p.u0, p.u1, 0) for p in ro.sub0] + [(p.batch, p.name, p.u0, p.u1, 1) for p in ro.sub1]
+        got = [(b, idx[(b, i)], u0, u1, sub) for (b, i, u0, u1, sub) in rows]
+        assert got == want
+    cp.close()
+
+
+def test_cpp_planner_worked_example(L):
+    import json
+    ex = json.load(open(os.path.join(ROOT, "tests", "golden", "algorithm1_worked_example.json")))
+    cp = CPlanner(L, 2, ex["cf"])
+    names = {}
+    for b in ex["batches"]:
+        ks = []
+        for i, (name, typ, d) in enumerate(b["kernels"]):
+            durs = tuple(d) if isinstance(d, list) else (d,)
+            ks.append(Kernel(b["id"], name, typ, durs, decomposable=len(durs) > 1))
+            names[(b["id"], i)] = name
+        cp.submit(b["id"], ks)
+    for want in ex["rounds"]:
+        rows, typ, t0 = cp.round()
+        assert typ == want["type"] and t0 == pytest.approx(want["time0"])
+        assert [[b, names[(b, i)], u0, u1] for (b, i, u0, u1, s) in rows if s == 0] == want["sub0"]
+        assert [[b, names[(b, i)], u0, u1] for (b, i, u0, u1, s) in rows if s == 1] == want["sub1"]
+    cp.close()
+
+
+def _agree_worker(rank, world, port, q):
+    """Each rank runs its own C++ planner; rank 0 decides how many arrivals are due
+    at each step (wall clock) and broadcasts it (bench.py's rule); every rank
+    must then produce the same plan sequence (NCCL ordering needs it)."""
+    import hashlib
+    import time
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ppopp_duwjchcl24_b200 import liger
+    rng = random.Random(0)
+    batches = [_batch(rng, b, 8) for b in range(6)]
+    cp = CPlanner(liger, 2, 1.1)
+    h = hashlib.sha256()
+    submitted, t0 = 0, time.monotonic()
+    while True:
+        due = [min(6, int((time.monotonic() - t0) / 0.002) + 1)] if rank == 0 else [0]
+        dist.broadcast_object_list(due, src=0)
+        while submitted < due[0]:
+            cp.submit(submitted, batches[submitted])
+            submitted += 1
+        r = cp.round()
+        if r is None and submitted == 6:
+            break
+        h.update(repr(r).encode())
+    out = [None] * world
+    dist.all_gather_object(out, h.hexdigest())
+    q.put(out)
+    dist.destroy_process_group()
+
+
+def test_plan_agreement_two_ranks_gloo():
+    import socket
+    import torch.multiprocessing as mp
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_agree_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = [q.get(timeout=300) for _ in ps]
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert res[0][0] == res[0][1]
