@@ -194,6 +194,7 @@ struct liger_ctx {
   size_t ev_next = 0;
   DurTable dur;
   double attn_scale[2] = {1.0, 1.0};   // calibration of the attention duration model (prefill, decode)
+  bool no_ln_fuse = false;             // LIGER_NO_LN_FUSE=1 disables the fused fixup + LN
   bool ar_atomic_chunks = false;
   // stats / timing
   liger_stats_t st{};
@@ -250,7 +251,8 @@ cudaEvent_t pool_event(liger_ctx* c) {
 
 // ------------------------------------------------------------------ geometry helpers
 int op_units(liger_ctx* c, int op) {
-  if (c->F <= 1) return 1;
+  // decomposition exists to fill a communication window; at t = 1 there is none
+  if (c->F <= 1 || c->world == 1) return 1;
   if (op_is_gemm(op) || (op_is_ar(op) && c->world > 1)) return c->F;
   return 1;
 }
@@ -283,6 +285,15 @@ int unit_col(int N, int u, int F) {
 int pad128(int n) { return (n + 127) / 128 * 128; }
 
 int batch_M(const Batch* bt, int pass) { return pass == 0 ? bt->b * bt->s : bt->b; }
+
+// Is the residual add + LayerNorm after row-parallel GEMM `gemm_op` of `layer`
+// fused into that GEMM's split-K fixup?  (t = 1 only: at t > 1 the all-reduce
+// sits between them.  The last layer's FC2 feeds the LM head's own LN.)
+bool ln_fused(liger_ctx* c, const Batch* bt, int pass, int gemm_op, int layer) {
+  if (c->world != 1 || c->no_ln_fuse) return false;
+  if (gemm_op == OP_FC2 && layer == c->L - 1) return false;
+  return gemm_can_fuse_ln(batch_M(bt, pass), c->h, gemm_K(c, gemm_op));
+}
 
 // ------------------------------------------------------------------ durations
 double model_dur(liger_ctx* c, int op, int M, int k, int ctx_len, int s_len) {
@@ -398,6 +409,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_LN1: {
+      if (li > 0 && ln_fused(c, bt, pass, OP_FC2, li - 1)) break;   // done in FC2's fixup
       timed_begin(c, st, &ta);
       if (li == 0)
         rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
@@ -408,6 +420,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_LN2: {
+      if (ln_fused(c, bt, pass, OP_OUT, li)) break;                 // done in out-proj's fixup
       timed_begin(c, st, &ta);
       rc = add_layernorm_launch(S.x, S.part, W->b_o, S.x, S.y, W->g2, W->be2, M, h, 1, 0, eps, st);
       timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * 4, 0);
@@ -432,11 +445,20 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
         g.scale_cols = c->hl; g.scale = 1.0f / sqrtf((float)c->d);
       } else if (po.op == OP_OUT) {
         g.x = S.attn; g.ldx = c->hl; g.w = W->w_o; g.ldw = K; g.out = S.part; g.ldo = h;
+        if (ln_fused(c, bt, pass, OP_OUT, li) && g.n0 == 0 && g.n1 == N) {
+          g.ln_x = S.x; g.ln_xout = S.x; g.ln_add_bias = W->b_o; g.ln_g = W->g2; g.ln_b = W->be2; g.ln_y = S.y;
+          g.ln_eps = eps;
+        }
       } else if (po.op == OP_FC1) {
         g.x = S.y; g.ldx = h; g.w = W->w_1; g.ldw = K; g.out = S.hbuf; g.ldo = N; g.bias = W->b_1;
         g.act = c->cfg.act;
       } else {
         g.x = S.hbuf; g.ldx = c->fl; g.w = W->w_2; g.ldw = K; g.out = S.part; g.ldo = h;
+        if (ln_fused(c, bt, pass, OP_FC2, li) && g.n0 == 0 && g.n1 == N) {
+          const LayerW& Wn = c->layers[li + 1];
+          g.ln_x = S.x; g.ln_xout = S.x; g.ln_add_bias = W->b_2; g.ln_g = Wn.g1; g.ln_b = Wn.be1; g.ln_y = S.y;
+          g.ln_eps = eps;
+        }
       }
       timed_begin(c, st, &ta);
       rc = gemm_launch(g, st);
@@ -714,6 +736,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   c->hl = c->h / world; c->al = c->a / world; c->fl = c->f / world; c->Vl = c->V / world;
   c->F = std::max(1, cfg->decomp_factor);
   c->cf = cfg->contention_factor > 0 ? cfg->contention_factor : 1.0;
+  c->no_ln_fuse = getenv("LIGER_NO_LN_FUSE") != nullptr;
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (world > 2);
   if (world > 1) {

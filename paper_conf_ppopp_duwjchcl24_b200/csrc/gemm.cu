@@ -315,6 +315,100 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
   }
 }
 
+// Split-K fixup fused with the residual add and LayerNorm that follow the
+// row-parallel projections (decode, t = 1):
+//   part = bf16(sum_z partial[z]);  r = bf16(x + part + add_bias);  y = LN(r)
+// A cluster of LN_FUSE_CLUSTER CTAs owns one row m; each CTA sums its column
+// block, and the row statistics are reduced over the cluster through DSMEM in
+// rank order (deterministic).  Same bits as the unfused GEMM -> add_ln path.
+struct LnFuseParams {
+  const __nv_bfloat16* x;
+  __nv_bfloat16* x_out;
+  const __nv_bfloat16* add_bias;
+  const __nv_bfloat16* g;
+  const __nv_bfloat16* b;
+  __nv_bfloat16* y;
+  float eps;
+};
+
+__device__ __forceinline__ float cluster_sum(float v, float* slot, float* red) {
+  // CTA-level sum (warp shuffles + smem), then over the cluster's CTAs in rank order
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  if (l == 0) red[w] = v;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float s = 0.f;
+    for (int i = 0; i < (int)(blockDim.x >> 5); ++i) s += red[i];
+    *slot = s;
+  }
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+  float tot = 0.f;
+  for (int r = 0; r < LN_FUSE_CLUSTER; ++r) {
+    uint32_t remote;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(smem_u32(slot)), "r"(r));
+    float x;
+    asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(x) : "r"(remote) : "memory");
+    tot += x;
+  }
+  return tot;
+}
+
+constexpr int LNF_THREADS = 256, LNF_MAXC = 8;
+
+__global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const GemmParams p, const LnFuseParams q) {
+  __shared__ float red[LNF_THREADS / 32];
+  __shared__ float slot[2];
+  grid_dependency_trigger();
+  grid_dependency_wait();
+  const int m = blockIdx.y;
+  const int rank = blockIdx.x;   // == %cluster_ctarank for cluster dims (LN_FUSE_CLUSTER, 1, 1)
+  const int cw = p.N / LN_FUSE_CLUSTER;
+  const int n_begin = rank * cw;
+  const int tiles = p.n_tiles * p.m_tiles;
+  const int64_t zstride = (int64_t)tiles * (BM * p.bn);
+  const int mt = m / p.bn, col = m % p.bn;
+  float r[LNF_MAXC];
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < LNF_MAXC; ++i) {
+    const int c = threadIdx.x + i * LNF_THREADS;
+    r[i] = 0.f;
+    if (c < cw) {
+      const int n = n_begin + c;
+      const float* src = p.ws + (int64_t)((n / BM) * p.m_tiles + mt) * (BM * p.bn) + (int64_t)col * BM + (n % BM);
+      float acc = __ldcg(src);
+      for (int z = 1; z < p.splits; ++z) acc += __ldcg(src + z * zstride);
+      const float part = __bfloat162float(__float2bfloat16_rn(acc));
+      float v = __bfloat162float(q.x[(int64_t)m * p.N + n]) + part;
+      if (q.add_bias) v += __bfloat162float(q.add_bias[n]);
+      v = __bfloat162float(__float2bfloat16_rn(v));   // residual stream is bf16
+      r[i] = v;
+      s += v;
+    }
+  }
+  const float mean = cluster_sum(s, &slot[0], red) / (float)p.N;
+  float sq = 0.f;
+#pragma unroll
+  for (int i = 0; i < LNF_MAXC; ++i)
+    if (threadIdx.x + i * LNF_THREADS < cw) sq += (r[i] - mean) * (r[i] - mean);
+  const float var = cluster_sum(sq, &slot[1], red) / (float)p.N;
+  const float rstd = 1.0f / sqrtf(var + q.eps);
+#pragma unroll
+  for (int i = 0; i < LNF_MAXC; ++i) {
+    const int c = threadIdx.x + i * LNF_THREADS;
+    if (c < cw) {
+      const int n = n_begin + c;
+      q.x_out[(int64_t)m * p.N + n] = __float2bfloat16_rn(r[i]);
+      q.y[(int64_t)m * p.N + n] =
+          __float2bfloat16_rn((r[i] - mean) * rstd * __bfloat162float(q.g[n]) + __bfloat162float(q.b[n]));
+    }
+  }
+  // keep this CTA's shared slots alive until every CTA of the cluster has read them
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 // ------------------------------------------------------------------ host side
 typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                     const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
@@ -445,6 +539,10 @@ GemmPlan gemm_plan(int M, int N, int K) {
   return pl;
 }
 
+bool gemm_can_fuse_ln(int M, int N, int K) {
+  return gemm_plan(M, N, K).splits > 1 && N % LN_FUSE_CLUSTER == 0 && N / LN_FUSE_CLUSTER <= LNF_THREADS * LNF_MAXC;
+}
+
 size_t gemm_workspace_bytes(int M, int N, int K) {
   GemmPlan pl = gemm_plan(M, N, K);
   if (pl.splits <= 1) return GEMM_COUNTER_BYTES;
@@ -496,6 +594,26 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   const int grid = p.units < num_sms() ? p.units : num_sms();
   int rc2 = launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
   if (rc2 || p.splits == 1) return rc2 ? LIGER_ECUDA : 0;
+  if (a.ln_y) {
+    if (a.n0 != 0 || a.n1 != a.N || !gemm_can_fuse_ln(a.M, a.N, a.K) || !a.ln_x || !a.ln_xout || !a.ln_g || !a.ln_b)
+      return LIGER_EINVAL;
+    LnFuseParams q{(const __nv_bfloat16*)a.ln_x, (__nv_bfloat16*)a.ln_xout, (const __nv_bfloat16*)a.ln_add_bias,
+                   (const __nv_bfloat16*)a.ln_g, (const __nv_bfloat16*)a.ln_b, (__nv_bfloat16*)a.ln_y, a.ln_eps};
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(LN_FUSE_CLUSTER, a.M);
+    cfg.blockDim = dim3(LNF_THREADS);
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[2];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = LN_FUSE_CLUSTER;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = getenv("LIGER_NO_PDL") ? 0 : 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 2;
+    return cudaLaunchKernelEx(&cfg, splitk_reduce_ln_kernel, p, q) == cudaSuccess ? 0 : LIGER_ECUDA;
+  }
   const int64_t work = (int64_t)p.M * (BM / 4) * p.n_tiles;
   int rblocks = (int)((work + 255) / 256);
   if (rblocks > num_sms() * 8) rblocks = num_sms() * 8;

@@ -125,6 +125,34 @@ def test_gemm_tiled_layout_bit_exact(L, M, N, K):
     assert torch.equal(got, ref) and torch.equal(sl, ref)
 
 
+@pytest.mark.parametrize("M,N,K", [(2, 5120, 5120), (8, 5120, 20480), (5, 1024, 4096)])
+def test_fused_fixup_add_ln_bit_exact(L, M, N, K):
+    """Decode row-parallel GEMM with the residual add + LN fused into its split-K
+    fixup = the GEMM followed by liger_op_add_layernorm, bit for bit; and against
+    the oracle."""
+    assert L.gemm_can_fuse_ln(M, N, K)
+    x = bf16_dev(c0_values(7, 1, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K))
+    w = bf16_dev(c0_values(7, 2, np.arange(N * K, dtype=np.uint64), -7).reshape(N, K))
+    res = bf16_dev(c0_values(7, 3, np.arange(M * N, dtype=np.uint64), -2).reshape(M, N))
+    ab = bf16_dev(c0_values(7, 4, np.arange(N, dtype=np.uint64), -6))
+    g = bf16_dev(1 + c0_values(7, 5, np.arange(N, dtype=np.uint64), -4))
+    be = bf16_dev(c0_values(7, 6, np.arange(N, dtype=np.uint64), -4))
+    wt = torch.empty(L.tiled_numel(N, K), dtype=torch.bfloat16, device="cuda")
+    L.tile_weight(w, wt)
+    ws = workspace(L.gemm_workspace_bytes(M, N, K))
+    part = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+    L.gemm_tiled(x, wt, part, N=N, workspace=ws)
+    r1, y1 = torch.empty_like(res), torch.empty_like(res)
+    L.add_layernorm(res, g, be, y1, add=part, add_bias=ab, x_out=r1)
+    r2, y2 = torch.empty_like(res), torch.empty_like(res)
+    L.gemm_tiled_add_ln(x, wt, N=N, resid=res, resid_out=r2, add_bias=ab, gamma=g, beta=be, y=y2, workspace=ws)
+    torch.cuda.synchronize()
+    assert torch.equal(r1, r2) and torch.equal(y1, y2)
+    ref_r = to_np64(res) + to_np64(x) @ to_np64(w).T + to_np64(ab)
+    assert errs(to_np64(r2), ref_r)[0] <= REL
+    assert errs(to_np64(y2), om.layer_norm(to_np64(r2), to_np64(g), to_np64(be), 1e-5))[0] <= REL
+
+
 def test_c0_tiled_fill_matches_tile_weight(L):
     from liger_inputs import weight_exp
     N, K = 384, 256
