@@ -276,6 +276,20 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   }
 }
 
+// sum_{z=0..S-1} src[z * zstride] in chunk order, 8 loads in flight
+__device__ __forceinline__ float sum_partials(const float* src, int64_t zstride, int S) {
+  float acc = __ldcg(src);
+  for (int z0 = 1; z0 < S; z0 += 8) {
+    float v[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = (z0 + i < S) ? __ldcg(src + (z0 + i) * zstride) : 0.f;
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+      if (z0 + i < S) acc += v[i];
+  }
+  return acc;
+}
+
 // Split-K fixup: out[m, n] = epi( sum_{z=0..S-1} partial[z] ) in chunk order (the
 // same bits whatever slice or CTA produced each chunk).  One thread per (m, 4 rows n),
 // reading the column-major per-tile partials coalesced.
@@ -295,12 +309,22 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
     const int tile_id = nt * p.m_tiles + mt;
     const float4* src = reinterpret_cast<const float4*>(p.ws + (int64_t)tile_id * (BM * p.bn) + (int64_t)col * BM) + rq;
     float4 acc = __ldcg(src);
-    for (int z = 1; z < p.splits; ++z) {
-      const float4 v = __ldcg(reinterpret_cast<const float4*>(reinterpret_cast<const float*>(src) + z * zstride));
-      acc.x += v.x;
-      acc.y += v.y;
-      acc.z += v.z;
-      acc.w += v.w;
+    // chunk order z = 1..S-1; the loads of a group of 8 are all in flight before the adds
+    for (int z0 = 1; z0 < p.splits; z0 += 8) {
+      float4 v[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        v[i] = (z0 + i < p.splits)
+                   ? __ldcg(reinterpret_cast<const float4*>(reinterpret_cast<const float*>(src) + (z0 + i) * zstride))
+                   : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        if (z0 + i < p.splits) {
+          acc.x += v[i].x;
+          acc.y += v[i].y;
+          acc.z += v[i].z;
+          acc.w += v[i].w;
+        }
     }
     const float a[4] = {acc.x, acc.y, acc.z, acc.w};
 #pragma unroll
@@ -378,8 +402,7 @@ __global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const Gem
     if (c < cw) {
       const int n = n_begin + c;
       const float* src = p.ws + (int64_t)((n / BM) * p.m_tiles + mt) * (BM * p.bn) + (int64_t)col * BM + (n % BM);
-      float acc = __ldcg(src);
-      for (int z = 1; z < p.splits; ++z) acc += __ldcg(src + z * zstride);
+      const float acc = sum_partials(src, zstride, p.splits);
       const float part = __bfloat162float(__float2bfloat16_rn(acc));
       float v = __bfloat162float(q.x[(int64_t)m * p.N + n]) + part;
       if (q.add_bias) v += __bfloat162float(q.add_bias[n]);
