@@ -163,7 +163,7 @@ def main():
     ap.add_argument("--mode", default="interleaved", choices=["interleaved", "serial"])
     ap.add_argument("--inflight", type=int, default=2)
     ap.add_argument("--F", type=int, default=8)
-    ap.add_argument("--cf", type=float, default=1.1)
+    ap.add_argument("--cf", type=float, default=1.1, help="contention factor; <= 0: use the calibrated one")
     ap.add_argument("--n-new", type=int, default=32)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-latency", action="store_true")
@@ -192,6 +192,8 @@ def main():
                       max_new=args.n_new, max_inflight=args.inflight, decomp_factor=args.F,
                       contention_factor=args.cf, seed=args.seed)
     eng.profile([8, 64, 256, 512, 1024, 2048, 4096])
+    # contention factor: measured GEMM || all-reduce slowdown (1-rank proxy at N=1)
+    cf_cal, _ = eng.calibrate_cf([8, 256, 1024], set_cf=args.cf <= 0)
 
     def barrier():
         if world > 1:
@@ -276,10 +278,18 @@ def main():
                           per_launch_bytes=v["bytes"] / v["count"], per_launch_flops=v["flops"] / v["count"])
     dom = max(classes, key=lambda k: shares[k]) if classes else None
     roof = None
+    traffic = {}
+    try:   # dram bytes per launch of each kernel class from the committed `ncu --set full` capture
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            traffic = json.load(f)
+    except Exception:
+        pass
     if dom:
         c = classes[dom]
         roof = {"kernel": dom, "bound": c["bound"], "achieved": round(c["achieved"], 2), "peak": c["peak"],
-                "unit": c["unit"], "frac": round(c["frac"], 4), "traffic": None, "peak_source": peak_src,
+                "unit": c["unit"], "frac": round(c["frac"], 4),
+                "traffic": traffic.get(dom, {}).get("dram_bytes_per_launch"),
+                "traffic_source": traffic.get(dom, {}).get("source"), "peak_source": peak_src,
                 "share_of_kernel_time": round(c["share"], 4)}
 
     # ---- latency at a fixed request rate (Poisson, 0.5 x capacity)
@@ -330,7 +340,9 @@ def main():
                                    f"U[128,512], {args.n_new} generated tokens, all {len(timed)} batches offered "
                                    f"at once (capacity)", "model": cfg.name, "tp": world,
                        "mode": args.mode, "max_inflight": args.inflight, "decomp_factor": args.F,
-                       "contention_factor": args.cf, "sequences": seqs, "batches": len(timed),
+                       "contention_factor": args.cf if args.cf > 0 else cf_cal,
+                       "contention_factor_calibrated": round(cf_cal, 4),
+                       "sequences": seqs, "batches": len(timed),
                        "l2": "inputs larger than L2 (weights 26 GB per TP=1 rank)"},
             "latency": lat,
             "e2e": {"value": round(seqs / e2e_s, 3), "unit": "req/s", "h2d_bytes_per_step": int(h2d),

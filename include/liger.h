@@ -176,6 +176,17 @@ int liger_set_duration(liger_ctx* ctx, int kclass, int m_tokens, int k_of_F, dou
  * store them in the duration table.  Returns LIGER_OK. */
 int liger_profile(liger_ctx* ctx, const int32_t* m_list, int n_m);
 
+/* Contention-factor calibration (§8(a) a16): run each projection
+ * GEMM at token counts m_list concurrently with an all-reduce of the matching
+ * [M, h] partial on the communication stream, and return in *cf_out the
+ * maximum slowdown of either kernel versus its no-load duration (ranks agree
+ * by max).  detail (optional, host [n_m][4][2]): slowdowns (GEMM, all-reduce)
+ * per token count and GEMM (QKV, out, FC1, FC2).  At world == 1 a 1-rank NCCL
+ * all-reduce (a local copy kernel of the same bytes) is the proxy.
+ * set_cf != 0 installs the result as the scheduler's cf. [collective] */
+int liger_calibrate_cf(liger_ctx* ctx, const int32_t* m_list, int n_m, int set_cf, double* cf_out,
+                       double* detail);
+
 const char* liger_last_error(const liger_ctx* ctx);
 int liger_finalize(liger_ctx* ctx); /* [collective] */
 

@@ -1098,6 +1098,104 @@ int liger_set_duration(liger_ctx* c, int op, int m_tokens, int k_of_F, double us
   return LIGER_OK;
 }
 
+// Contention-factor calibration (§3.5): profile the lengthy
+// computation kernels (the projection GEMMs at the given token counts) running
+// concurrently with communication kernels (all-reduces of the matching
+// [M, h] partial) on the two streams, with different inputs, and take the
+// maximum slowdown of either side relative to its no-load duration (reading
+// R4).  At t = 1 there is no tensor-parallel all-reduce; the calibration then
+// uses a 1-rank NCCL communicator whose all-reduce kernel moves the same bytes
+// locally (a proxy, reported as such).  Sets the context's cf when set_cf != 0.
+int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf, double* cf_out,
+                       double* detail /* [n_m][4][2] slowdowns (gemm, ar) or NULL */) {
+  if (!c || !m_list || n_m <= 0) return LIGER_EINVAL;
+  if (!c->processing.empty() || !c->waiting.empty()) return fail(c, LIGER_ESTATE, "liger_calibrate_cf: batches in flight");
+  if (!nccl().ok) return fail(c, LIGER_ENCCL, "NCCL library not loadable");
+  ncclComm_t comm = c->comm, own = nullptr;
+  if (!comm) {
+    ncclUniqueId id;
+    if (nccl().GetUniqueId(&id) != ncclSuccess || nccl().CommInitRank(&own, 1, id, 0) != ncclSuccess)
+      return fail(c, LIGER_ENCCL, "liger_calibrate_cf: 1-rank NCCL communicator");
+    comm = own;
+  }
+  CK(cudaDeviceSynchronize());
+  Slot& S = c->slots[0];
+  const int Mmax = c->cfg.max_batch * c->cfg.max_seq;
+  cudaEvent_t ev[4];
+  for (auto& e : ev) CK(cudaEventCreate(&e));
+  const bool saved_timing = c->timing;
+  c->timing = false;
+  Batch fake;
+  fake.slot = 0;
+  fake.n_new = 1;
+  fake.b = 1;
+  double cf = 1.0;
+  auto ar = [&](size_t elems) {
+    nccl().AllReduce(S.part, S.part, elems, ncclBfloat16, ncclSum, comm, c->s_comm);
+  };
+  for (int mi = 0; mi < n_m; ++mi) {
+    const int M = std::min<int>(m_list[mi], Mmax);
+    fake.s = M;
+    int oi = 0;
+    for (int op : {OP_QKV, OP_OUT, OP_FC1, OP_FC2}) {
+      int pidx = 0;
+      while (c->pass_ops[pidx].op != op) ++pidx;
+      const size_t elems = (size_t)M * c->h;
+      auto gemm = [&] { launch_piece(c, &fake, 0, pidx, 0, op_units(c, op), c->s_comp); };
+      float tg = 1e30f, ta = 1e30f, tgc = 1e30f, tac = 1e30f;
+      for (int rep = 0; rep < 4; ++rep) {
+        float x;
+        cudaEventRecord(ev[0], c->s_comp); gemm(); cudaEventRecord(ev[1], c->s_comp);
+        cudaEventSynchronize(ev[1]); cudaEventElapsedTime(&x, ev[0], ev[1]); if (rep) tg = std::min(tg, x);
+        cudaEventRecord(ev[2], c->s_comm); ar(elems); cudaEventRecord(ev[3], c->s_comm);
+        cudaEventSynchronize(ev[3]); cudaEventElapsedTime(&x, ev[2], ev[3]); if (rep) ta = std::min(ta, x);
+        // concurrent: both streams released together
+        cudaEventRecord(ev[0], c->s_comp);
+        cudaStreamWaitEvent(c->s_comm, ev[0], 0);
+        cudaEventRecord(ev[2], c->s_comm);
+        ar(elems);
+        cudaEventRecord(ev[3], c->s_comm);
+        gemm();
+        cudaEventRecord(ev[1], c->s_comp);
+        cudaEventSynchronize(ev[1]);
+        cudaEventSynchronize(ev[3]);
+        float g2, a2;
+        cudaEventElapsedTime(&g2, ev[0], ev[1]);
+        cudaEventElapsedTime(&a2, ev[2], ev[3]);
+        if (rep) {
+          tgc = std::min(tgc, g2);
+          tac = std::min(tac, a2);
+        }
+      }
+      const double sg = tgc / tg, sa = tac / ta;
+      if (detail) {
+        detail[(mi * 4 + oi) * 2 + 0] = sg;
+        detail[(mi * 4 + oi) * 2 + 1] = sa;
+      }
+      cf = std::max(cf, std::max(sg, sa));
+      ++oi;
+    }
+  }
+  c->timing = saved_timing;
+  for (auto& e : ev) cudaEventDestroy(e);
+  if (own) nccl().CommDestroy(own);
+  if (c->world > 1) {   // all ranks must use the same cf (identical plans)
+    float* dv = nullptr;
+    float v = (float)cf;
+    CK(cudaMalloc(&dv, 4));
+    CK(cudaMemcpy(dv, &v, 4, cudaMemcpyHostToDevice));
+    nccl().AllReduce(dv, dv, 1, ncclFloat32, ncclMax, c->comm, c->s_comp);
+    CK(cudaMemcpyAsync(&v, dv, 4, cudaMemcpyDeviceToHost, c->s_comp));
+    CK(cudaStreamSynchronize(c->s_comp));
+    cudaFree(dv);
+    cf = v;
+  }
+  if (set_cf) c->cf = cf;
+  if (cf_out) *cf_out = cf;
+  CK(cudaDeviceSynchronize());
+  return LIGER_OK;
+}
+
 // Offline profiling: no-load durations of every kernel
 // class over a token grid and for every k/F piece, on slot 0's buffers.
 int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {

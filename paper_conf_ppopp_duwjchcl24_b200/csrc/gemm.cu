@@ -539,7 +539,7 @@ GemmPlan gemm_plan(int M, int N, int K) {
     if (S != sp) continue;
     const double units = (double)tiles * S;
     double cost = ceil(units / G) * (kcb * kb_time + 300.0);
-    if (S > 1) cost += 3000.0 + (double)S * M * N * 8.0 / 2600.0;
+    if (S > 1) cost += 6000.0 + (double)S * M * N * 8.0 / 2600.0;   // fixup launch + partial traffic
     if (cost < best - 1e-9) {
       best = cost;
       best_s = S;
@@ -557,6 +557,11 @@ GemmPlan gemm_plan(int M, int N, int K) {
   const int stage_bytes = A_BYTES + pl.bn * BK * 2;
   int st = (MAX_SMEM - 1024 - 512) / stage_bytes;
   if (st > 12) st = 12;
+  if (pl.bn <= 32 && st > 6) st = 6;   // decode: 96 KiB of weights in flight suffices (measured)
+  if (const char* e = getenv("LIGER_GEMM_STAGES")) {   // experiments only
+    const int f = atoi(e);
+    if (f >= 2 && f < st) st = f;
+  }
   pl.stages = st;
   pl.smem = 1024 + st * stage_bytes + 512;
   return pl;

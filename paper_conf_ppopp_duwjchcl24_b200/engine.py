@@ -57,6 +57,17 @@ class LigerEngine:
         arr = (C.c_int32 * len(m_list))(*m_list)
         self._chk(L.lib().liger_profile(self.ctx, arr, len(m_list)), "liger_profile")
 
+    def calibrate_cf(self, m_list, set_cf=True):
+        arr = (C.c_int32 * len(m_list))(*m_list)
+        cf = C.c_double()
+        det = (C.c_double * (len(m_list) * 8))()
+        self._chk(L.lib().liger_calibrate_cf(self.ctx, arr, len(m_list), int(set_cf), C.byref(cf), det),
+                  "liger_calibrate_cf")
+        names = ["qkv", "out", "fc1", "fc2"]
+        detail = {m: {n: (det[(i * 4 + j) * 2], det[(i * 4 + j) * 2 + 1]) for j, n in enumerate(names)}
+                  for i, m in enumerate(m_list)}
+        return cf.value, detail
+
     def submit(self, tokens, batch, seq_len, n_new, arrival_s=-1.0, device_tokens=None):
         """tokens: numpy int32 [batch*seq_len] (host) or None with device_tokens = a device
         int32 tensor (kept alive by the caller until the batch finishes)."""

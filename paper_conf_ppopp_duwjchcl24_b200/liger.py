@@ -59,6 +59,7 @@ _SIGS = {
     "liger_kernel_timing": (_I, [_P, _P, _P, _P, _P]),
     "liger_set_duration": (_I, [_P, _I, _I, _I, _D]),
     "liger_profile": (_I, [_P, _P, _I]),
+    "liger_calibrate_cf": (_I, [_P, _P, _I, _I, _P, _P]),
     "liger_last_error": (C.c_char_p, [_P]),
     "liger_finalize": (_I, [_P]),
     "liger_op_gemm": (_I, [_P, _I64, _P, _I64, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),

@@ -112,3 +112,13 @@ def test_fused_ln_path_bit_exact_with_unfused(E):
             os.environ.pop("LIGER_NO_LN_FUSE", None)
     for a, b in zip(*outs):
         assert np.array_equal(a, b)
+
+
+def test_contention_factor_calibration(E):
+    """cf = max slowdown of GEMM / all-reduce run concurrently (>= 1)."""
+    cfg = get_config("tiny")
+    eng = E(cfg, max_batch=2, max_seq=32, max_new=4, seed=0)
+    cf, detail = eng.calibrate_cf([16, 64])
+    eng.close()
+    assert 1.0 <= cf < 10.0
+    assert set(detail) == {16, 64} and all(len(v) == 4 for v in detail.values())
