@@ -30,6 +30,7 @@ import numpy as np
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
+os.environ["NCCL_DEBUG"] = "WARN"   # keep NCCL's version banner off stdout (one JSON line)
 
 from liger_inputs import get_config, make_trace  # noqa: E402
 
@@ -289,6 +290,7 @@ def main():
         roof = {"kernel": dom, "bound": c["bound"], "achieved": round(c["achieved"], 2), "peak": c["peak"],
                 "unit": c["unit"], "frac": round(c["frac"], 4),
                 "traffic": traffic.get(dom, {}).get("dram_bytes_per_launch"),
+                "traffic_algorithmic_bytes": traffic.get(dom, {}).get("algorithmic_bytes_per_launch"),
                 "traffic_source": traffic.get(dom, {}).get("source"), "peak_source": peak_src,
                 "share_of_kernel_time": round(c["share"], 4)}
 
