@@ -229,19 +229,23 @@ int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* 
 }
 
 // ================================================================== decode
-// One CTA per (head, sequence), 256 threads, streaming the sequence's cached
-// K/V through a DC_STAGES-deep ring of shared-memory chunks (DC_CHUNK positions
-// each).  Warp 0 stages a chunk's page blocks (16 tokens x d bf16 = 4 KiB,
-// contiguous in the paged pool) with cp.async.bulk (TMA bulk engine) on the
-// stage's mbarrier; the CTA computes the chunk with an online softmax (running
-// max / sum / accumulator, rescaled per chunk) while the next chunks are in
-// flight.  The new token (position pos) comes from the qkv buffer and is
-// appended to its page.  No cross-CTA merge: the result is produced by one CTA.
-constexpr int DC_CHUNK = 64;
-constexpr int DC_STAGES = 2;
-constexpr int DC_THREADS = 256;
+// CTA = (head, sequence, chunk of DC_CHUNK positions), 128 threads.  Thread 0
+// stages the chunk's K and V page blocks (16 tokens x d bf16 = 4 KiB each,
+// contiguous in the paged pool) into shared memory with cp.async.bulk (TMA bulk
+// engine), all issued at once on one mbarrier, so a CTA pays one DRAM round
+// trip.  The new token (position pos) is taken from the qkv buffer (and
+// appended to its page by the last chunk's CTA).  Phase 1: warp w scores
+// positions [32w, 32w+32) (a token row spread over d/8 lanes, shuffle dot
+// products); two-pass softmax over the chunk; phase 2: thread (slot, vec)
+// accumulates p_t V[t] over positions t = slot (mod SLOTS).  Chunks of one
+// (sequence, head) are merged in chunk order by the last CTA (deterministic).
+constexpr int DC_CHUNK_MIN = 32;   // positions per CTA: 32 or 64 (template), chosen per launch
+constexpr int DC_THREADS = 128;
 
-size_t attn_decode_workspace_bytes(int, int, int, int) { return ATTN_COUNTER_BYTES; }   // unused scratch (API stable)
+size_t attn_decode_workspace_bytes(int b, int heads, int d, int ctx) {
+  const int ns = (ctx + DC_CHUNK_MIN - 1) / DC_CHUNK_MIN;   // worst case (32-position chunks)
+  return ATTN_COUNTER_BYTES + (size_t)b * heads * ns * (d + 2) * sizeof(float);
+}
 
 __device__ __forceinline__ void bf16x8_to_f32(const uint4& v, float* f) {
   const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&v);
@@ -253,182 +257,221 @@ __device__ __forceinline__ void bf16x8_to_f32(const uint4& v, float* f) {
   }
 }
 
-template <int D>
+template <int D, int DC_CHUNK>
 __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bfloat16* __restrict__ qkv,
                                                                  __nv_bfloat16* __restrict__ o,
                                                                  __nv_bfloat16* __restrict__ kv_pool,
                                                                  const int32_t* __restrict__ page_table,
-                                                                 int max_pages, int pos, int heads) {
-  constexpr int NW = DC_THREADS / 32;
-  constexpr int LPT = D / 8;              // lanes per token in phase 1
-  constexpr int TPW = 32 / LPT;           // tokens per warp step
-  constexpr int WPOS = DC_CHUNK / NW;     // positions per warp per chunk
-  constexpr int STEPS = WPOS / TPW;
+                                                                 int max_pages, int pos, int heads, float* ws,
+                                                                 int* counters) {
+  constexpr int LPT = D / 8;            // lanes per token
+  constexpr int TPW = 32 / LPT;         // tokens per warp step
+  constexpr int WPOS = DC_CHUNK / 4;    // positions per warp in phase 1
+  constexpr int STEPS = WPOS / TPW;     // steps for the warp's positions
   constexpr int NVEC = D / 8;
   constexpr int SLOTS = DC_THREADS / NVEC;
-  constexpr int PER = DC_CHUNK / SLOTS;   // positions per thread per chunk in phase 2
-  constexpr int CH_ELEMS = DC_CHUNK * D;
-  static_assert(STEPS >= 1 && PER >= 1, "chunk too small");
+  constexpr int PER = DC_CHUNK / SLOTS; // positions per thread in phase 2
+  constexpr int NPG = DC_CHUNK / KVB;   // pages per chunk
   extern __shared__ __align__(128) uint8_t dsm[];
-  __nv_bfloat16* sK = reinterpret_cast<__nv_bfloat16*>(dsm);            // [DC_STAGES][DC_CHUNK][D]
-  __nv_bfloat16* sV = sK + DC_STAGES * CH_ELEMS;                          // [DC_STAGES][DC_CHUNK][D]
+  __nv_bfloat16* sK = reinterpret_cast<__nv_bfloat16*>(dsm);
+  __nv_bfloat16* sV = sK + DC_CHUNK * D;
   __shared__ float sc[DC_CHUNK];
-  __shared__ float red[NW];
-  __shared__ float part[SLOTS][D + 1];
-  __shared__ __align__(8) uint64_t bar[DC_STAGES];
+  __shared__ float red[DC_THREADS / 32];
+  __shared__ float part[SLOTS][D];
+  __shared__ __align__(8) uint64_t bar;
+  __shared__ int last;
 
-  const int head = blockIdx.x, bi = blockIdx.y;
+  const int head = blockIdx.x, bi = blockIdx.y, sp = blockIdx.z, nsp = gridDim.z;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int ctx = pos + 1;
-  const int nch = (ctx + DC_CHUNK - 1) / DC_CHUNK;
+  const int t0 = sp * DC_CHUNK, t1 = min(ctx, t0 + DC_CHUNK);
   const int64_t ld = (int64_t)3 * heads * D;
   const __nv_bfloat16* row = qkv + (int64_t)bi * ld;
+  const __nv_bfloat16* qp = row + head * D;
   const __nv_bfloat16* knew = row + (int64_t)heads * D + head * D;
   const __nv_bfloat16* vnew = row + (int64_t)2 * heads * D + head * D;
   const int32_t* pt = page_table + (int64_t)bi * max_pages;
+  // cached positions of this chunk: [t0, min(t1, pos)) -- pages touching them
+  const int tc1 = min(t1, pos);
+  const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
 
   if (tid == 0) {
-    for (int i = 0; i < DC_STAGES; ++i) mbar_init(&bar[i], 1);
+    mbar_init(&bar, 1);
     fence_barrier_init();
   }
   __syncthreads();
   pdl_enter();
-
-  // warp 0: stage the cached positions of chunk c (those < pos) into ring slot c % DC_STAGES
-  auto issue = [&](int c) {
-    const int st = c % DC_STAGES;
-    const int t0 = c * DC_CHUNK, tc1 = min(t0 + DC_CHUNK, pos);
-    const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
-    if (lane == 0) mbar_arrive_expect_tx(&bar[st], (uint32_t)npg * 2 * KVB * D * 2);
+  if (warp == 0) {   // lane g stages page g (page ids loaded in parallel, not a serial chain)
+    if (lane == 0) mbar_arrive_expect_tx(&bar, (uint32_t)npg * 2 * KVB * D * 2);
     __syncwarp();
     if (lane < npg) {
       const int page = pt[(t0 >> 4) + lane];
-      bulk_load(sK + st * CH_ELEMS + lane * KVB * D, kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2,
-                &bar[st]);
-      bulk_load(sV + st * CH_ELEMS + lane * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2,
-                &bar[st]);
+      bulk_load(sK + lane * KVB * D, kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &bar);
+      bulk_load(sV + lane * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &bar);
     }
-  };
-  if (warp == 0)
-    for (int c = 0; c < DC_STAGES && c < nch; ++c) issue(c);
-
+  }
   float qf[8];
-  bf16x8_to_f32(*reinterpret_cast<const uint4*>(row + head * D + (lane % LPT) * 8), qf);
-  if (tid < 2 * NVEC) {   // append the new token's K/V to its page
+  {
+    uint4 qv = *reinterpret_cast<const uint4*>(qp + (lane % LPT) * 8);
+    bf16x8_to_f32(qv, qf);
+  }
+  const bool has_new = (t0 <= pos && pos < t1);
+  if (has_new && tid < 2 * NVEC) {   // append the new token's K/V (position pos) to its page
     const int kv = tid / NVEC, c = (tid % NVEC) * 8;
-    *reinterpret_cast<uint4*>(kv_pool + kv_off(pt[pos / KVB], kv, heads, head, pos % KVB, D) + c) =
+    const int page = pt[pos / KVB];
+    *reinterpret_cast<uint4*>(kv_pool + kv_off(page, kv, heads, head, pos % KVB, D) + c) =
         *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
   }
-
-  const int vec = tid % NVEC, slot = tid / NVEC;
-  float m_run = -INFINITY, l_run = 0.f;
-  float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-  for (int c = 0; c < nch; ++c) {
-    const int st = c % DC_STAGES;
-    const int t0 = c * DC_CHUNK, n = min(DC_CHUNK, ctx - t0);
-    __nv_bfloat16* cK = sK + st * CH_ELEMS;
-    __nv_bfloat16* cV = sV + st * CH_ELEMS;
-    mbar_wait(&bar[st], (c / DC_STAGES) & 1);
-    if (t0 <= pos && pos < t0 + DC_CHUNK && tid < 2 * NVEC) {   // the new token into the staged chunk
-      const int kv = tid / NVEC, cc = (tid % NVEC) * 8;
-      *reinterpret_cast<uint4*>((kv ? cV : cK) + (pos - t0) * D + cc) =
-          *reinterpret_cast<const uint4*>((kv ? vnew : knew) + cc);
-    }
-    __syncthreads();
-    // phase 1: scores of this chunk
-    {
-      const int cc = (lane % LPT) * 8;
-#pragma unroll
-      for (int stp = 0; stp < STEPS; ++stp) {
-        const int lt = warp * WPOS + stp * TPW + lane / LPT;
-        float dot = 0.f;
-        if (lt < n) {
-          float f[8];
-          bf16x8_to_f32(*reinterpret_cast<const uint4*>(cK + lt * D + cc), f);
-#pragma unroll
-          for (int i = 0; i < 8; ++i) dot += qf[i] * f[i];
-        }
-#pragma unroll
-        for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
-        if ((lane % LPT) == 0) sc[lt] = lt < n ? dot : -INFINITY;
-      }
-    }
-    __syncthreads();
-    // chunk max (64 scores: warps 0-1)
-    float cm = tid < DC_CHUNK ? sc[tid] : -INFINITY;
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) cm = fmaxf(cm, __shfl_xor_sync(0xffffffffu, cm, off));
-    if (lane == 0) red[warp] = cm;
-    __syncthreads();
-    cm = red[0];
-#pragma unroll
-    for (int w = 1; w < NW; ++w) cm = fmaxf(cm, red[w]);
-    const float m_new = fmaxf(m_run, cm);
-    const float scale = __expf(m_run - m_new);   // exp(-inf) = 0 on the first chunk
-    // phase 2: p_t = exp(s_t - m_new); l, acc rescaled by `scale`
-    float lsum = 0.f;
-#pragma unroll
-    for (int e = 0; e < 8; ++e) acc[e] *= scale;
-#pragma unroll
-    for (int i = 0; i < PER; ++i) {
-      const int lt = slot + i * SLOTS;
-      if (lt < n) {
-        const float pw = __expf(sc[lt] - m_new);
-        if (vec == 0) lsum += pw;
-        float f[8];
-        bf16x8_to_f32(*reinterpret_cast<const uint4*>(cV + lt * D + vec * 8), f);
-#pragma unroll
-        for (int e = 0; e < 8; ++e) acc[e] += pw * f[e];
-      }
-    }
-    // l over the chunk: lsum lives in the vec == 0 thread of each slot
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) lsum += __shfl_xor_sync(0xffffffffu, lsum, off);
-    __syncthreads();                     // sc / red reads done; ring slot st fully consumed
-    if (lane == 0) red[warp] = lsum;
-    if (warp == 0 && c + DC_STAGES < nch) {
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      issue(c + DC_STAGES);
-    }
-    __syncthreads();
-    float ls = 0.f;
-#pragma unroll
-    for (int w = 0; w < NW; ++w) ls += red[w];
-    l_run = l_run * scale + ls;
-    m_run = m_new;
+  mbar_wait(&bar, 0);
+  if (has_new && tid < 2 * NVEC) {   // ... and into the staged chunk (the bulk copy may predate it)
+    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
+    *reinterpret_cast<uint4*>((kv ? sV : sK) + (pos - t0) * D + c) =
+        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
   }
-  // combine the SLOTS partial accumulators
-#pragma unroll
-  for (int e = 0; e < 8; ++e) part[slot][vec * 8 + e] = acc[e];
   __syncthreads();
+
+  // ---- phase 1: scores for positions [t0 + warp*WPOS, +WPOS)
+  {
+    const int c = (lane % LPT) * 8;
+#pragma unroll
+    for (int st = 0; st < STEPS; ++st) {
+      const int lt = warp * WPOS + st * TPW + lane / LPT;   // local position
+      float dot = 0.f;
+      if (t0 + lt < t1) {
+        float f[8];
+        bf16x8_to_f32(*reinterpret_cast<const uint4*>(sK + lt * D + c), f);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) dot += qf[i] * f[i];
+      }
+#pragma unroll
+      for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
+      if (t0 + lt < t1 && (lane % LPT) == 0) sc[lt] = dot;
+    }
+  }
+  __syncthreads();
+  const int n = t1 - t0;
+  float mx = (tid < n) ? sc[tid] : -INFINITY;   // n <= DC_CHUNK <= DC_THREADS
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+  if (lane == 0) red[warp] = mx;
+  __syncthreads();
+  mx = fmaxf(fmaxf(red[0], red[1]), fmaxf(red[2], red[3]));
+  __syncthreads();
+  float p_t = 0.f;
+  if (tid < n) {
+    p_t = __expf(sc[tid] - mx);
+    sc[tid] = p_t;
+  }
+  float sum = p_t;
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
+  if (lane == 0) red[warp] = sum;
+  __syncthreads();
+  const float l = red[0] + red[1] + red[2] + red[3];
+
+  // ---- phase 2: o = sum_t p_t v_t
+  const int vec = tid % NVEC, slot = tid / NVEC;
+  float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll 4
+  for (int i = 0; i < PER; ++i) {
+    const int lt = slot + i * SLOTS;
+    if (t0 + lt < t1) {
+      const float pw = sc[lt];
+      float f[8];
+      bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + vec * 8), f);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) acc[e] += pw * f[e];
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) part[slot][vec * 8 + i] = acc[i];
+  __syncthreads();
+
+  if (nsp == 1) {
+    for (int e = tid; e < D; e += DC_THREADS) {
+      float a = 0.f;
+#pragma unroll
+      for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
+      o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / l);
+    }
+    return;
+  }
+  // split: write partial (m, l, acc[D]); the last CTA merges in chunk order
+  const int64_t unit = (int64_t)bi * heads + head;
+  float* wp = ws + (unit * nsp + sp) * (D + 2);
   for (int e = tid; e < D; e += DC_THREADS) {
     float a = 0.f;
 #pragma unroll
     for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
-    o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / l_run);
+    wp[e] = a;
   }
+  if (tid == 0) {
+    wp[D] = mx;
+    wp[D + 1] = l;
+  }
+  __syncthreads();
+  if (tid == 0) {
+    int prev;
+    asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&counters[unit]) : "memory");
+    last = (prev == nsp - 1);
+  }
+  __syncthreads();
+  if (!last) return;
+  float M = -INFINITY;
+  for (int s2 = 0; s2 < nsp; ++s2) M = fmaxf(M, __ldcg(&ws[(unit * nsp + s2) * (D + 2) + D]));
+  float L = 0.f;
+  for (int s2 = 0; s2 < nsp; ++s2) {
+    const float* w2 = ws + (unit * nsp + s2) * (D + 2);
+    L += __ldcg(&w2[D + 1]) * __expf(__ldcg(&w2[D]) - M);
+  }
+  for (int e = tid; e < D; e += DC_THREADS) {
+    float a = 0.f;
+    for (int s2 = 0; s2 < nsp; ++s2) {
+      const float* w2 = ws + (unit * nsp + s2) * (D + 2);
+      a += __ldcg(&w2[e]) * __expf(__ldcg(&w2[D]) - M);
+    }
+    o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / L);
+  }
+  if (tid == 0) counters[unit] = 0;
+}
+
+template <int D, int CH>
+static int launch_decode(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
+                         int pos, int heads, float* ws, int* counters, cudaStream_t stream) {
+  const int ns = (pos + 1 + CH - 1) / CH;
+  const size_t dsmem = (size_t)2 * CH * D * 2;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(attn_decode_kernel<D, CH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
+    attr = true;
+  }
+  return launch_pdl(attn_decode_kernel<D, CH>, dim3(heads, b, ns), dim3(DC_THREADS), dsmem, stream,
+                    (const __nv_bfloat16*)qkv, (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages,
+                    pos, heads, ws, counters);
 }
 
 int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
-                       int pos, int heads, int d, void*, size_t, cudaStream_t stream) {
+                       int pos, int heads, int d, void* workspace, size_t ws_bytes, cudaStream_t stream) {
   if (b <= 0) return 0;
-  const size_t dsmem = (size_t)2 * DC_STAGES * DC_CHUNK * d * 2;
-  static bool attr_dc = false;
-  if (!attr_dc) {
-    cudaFuncSetAttribute(attn_decode_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         2 * DC_STAGES * DC_CHUNK * 128 * 2);
-    cudaFuncSetAttribute(attn_decode_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         2 * DC_STAGES * DC_CHUNK * 64 * 2);
-    attr_dc = true;
+  const int ctx = pos + 1;
+  // 32-position chunks when 64-position ones would leave SMs without ~6 resident CTAs
+  const bool small = (size_t)b * heads * ((ctx + 63) / 64) < (size_t)148 * 6;
+  const int CH = small ? 32 : 64;
+  const int ns = (ctx + CH - 1) / CH;
+  if (ns > 1) {
+    if (!workspace || ws_bytes < attn_decode_workspace_bytes(b, heads, d, ctx) ||
+        (size_t)b * heads * 4 > ATTN_COUNTER_BYTES)
+      return LIGER_EINVAL;
   }
-  dim3 grid(heads, b);
+  int* counters = (int*)workspace;
+  float* ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
   int rc;
   if (d == 128)
-    rc = launch_pdl(attn_decode_kernel<128>, grid, dim3(DC_THREADS), dsmem, stream, (const __nv_bfloat16*)qkv,
-                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads);
+    rc = small ? launch_decode<128, 32>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream)
+               : launch_decode<128, 64>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream);
   else if (d == 64)
-    rc = launch_pdl(attn_decode_kernel<64>, grid, dim3(DC_THREADS), dsmem, stream, (const __nv_bfloat16*)qkv,
-                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, pos, heads);
+    rc = small ? launch_decode<64, 32>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream)
+               : launch_decode<64, 64>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream);
   else
     return LIGER_EINVAL;
   return rc ? LIGER_ECUDA : 0;
