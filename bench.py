@@ -30,7 +30,21 @@ import numpy as np
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
-os.environ["NCCL_DEBUG"] = "WARN"   # keep NCCL's version banner off stdout (one JSON line)
+# stdout carries exactly one JSON line: NCCL prints a version banner at NCCL_DEBUG=WARN/VERSION
+os.environ["NCCL_DEBUG"] = "NONE"
+_JSON_FD = None
+
+
+def emit(line):
+    """Write the result line to the real stdout (C-level stdout is redirected to stderr)."""
+    os.write(_JSON_FD if _JSON_FD is not None else 1, (json.dumps(line) + "\n").encode())
+
+
+def _redirect_stdout():
+    global _JSON_FD
+    sys.stdout.flush()
+    _JSON_FD = os.dup(1)
+    os.dup2(2, 1)
 
 from liger_inputs import get_config, make_trace  # noqa: E402
 
@@ -148,7 +162,7 @@ def run_reference(args):
                        "model": args.config},
             "cpu_baseline": {**{k: r[k] for k in ("unit", "cores", "kind", "sample")}, "value": v},
             "e2e": {"value": v, "unit": "req/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    emit(line)
     return 0
 
 
@@ -170,6 +184,7 @@ def main():
     ap.add_argument("--no-latency", action="store_true")
     ap.add_argument("--seed", type=int, default=0)
     args = ap.parse_args()
+    _redirect_stdout()
     if args.impl == "reference":
         return run_reference(args)
 
@@ -358,7 +373,7 @@ def main():
             "host": {"wall_s": round(wall_s, 3), "host_us": round(st["host_us"], 1),
                      "rounds": st["rounds"], "kernels": st["kernels"]},
         }
-        print(json.dumps(line), flush=True)
+        emit(line)
     eng.close()
     if world > 1:
         dist.destroy_process_group()
