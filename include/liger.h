@@ -108,6 +108,14 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
 /* Write a fresh ncclUniqueId (128 bytes) to host buffer `uid`. */
 int liger_nccl_unique_id(uint8_t* uid);
 
+/* Write a 128-byte id selecting the LOOPBACK communicator: the `world` ranks
+ * are threads of one process sharing the current GPU (each calls liger_init
+ * with this id and its rank from its own host thread); collectives are a host
+ * rendezvous plus rank-ordered device reductions.  A test vehicle that runs
+ * the complete t > 1 path (comm stream, Algorithm 1 secondaries,
+ * decomposition, hybrid sync, token all-gather) on a single GPU; world <= 8. */
+int liger_loopback_unique_id(uint8_t* uid);
+
 /* Initialise this rank's shard of layer `layer` on the device with the
  * counter-based generator C0 (global indices, so every rank gets
  * its slice of the same logical weights).  seed overrides cfg->seed when != 0

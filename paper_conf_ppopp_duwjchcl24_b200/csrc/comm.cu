@@ -1,0 +1,318 @@
+// Communication backends of the tensor-parallel ranks.
+//
+//  * NcclComm: NCCL over NVLink/NVSwitch (the product path; libnccl is loaded with
+//    dlopen and bootstrapped with a caller-broadcast ncclUniqueId).
+//  * LoopbackComm: the ranks of a group are threads of ONE process sharing one
+//    GPU; a collective is a host rendezvous plus device kernels that read every
+//    rank's buffer (rank order, deterministic).  It exists so the whole t > 1
+//    path -- communication stream, Algorithm 1 rounds with real secondary
+//    subsets, decomposition, hybrid E1/E2 sync, token all-gather -- can be run
+//    and checked on a single GPU.  Selected by a uid from
+//    liger_loopback_unique_id().
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <dlfcn.h>
+#include <nccl.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <condition_variable>
+#include <map>
+#include <mutex>
+#include <random>
+#include <string>
+#include <vector>
+
+#include "comm.h"
+#include "common.cuh"
+#include "kernels.h"
+
+namespace liger {
+
+// ------------------------------------------------------------------ NCCL (dlopen)
+NcclApi& nccl() {
+  static NcclApi api;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    const char* names[] = {"libnccl.so.2", "libnccl.so",
+                           "/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl/lib/libnccl.so.2"};
+    void* h = nullptr;
+    for (const char* n : names)
+      if ((h = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
+    if (!h) return;
+#define LIGER_SYM(field, name) api.field = reinterpret_cast<decltype(api.field)>(dlsym(h, name))
+    LIGER_SYM(GetUniqueId, "ncclGetUniqueId");
+    LIGER_SYM(CommInitRank, "ncclCommInitRank");
+    LIGER_SYM(AllReduce, "ncclAllReduce");
+    LIGER_SYM(AllGather, "ncclAllGather");
+    LIGER_SYM(GroupStart, "ncclGroupStart");
+    LIGER_SYM(GroupEnd, "ncclGroupEnd");
+    LIGER_SYM(CommDestroy, "ncclCommDestroy");
+    LIGER_SYM(CommGetAsyncError, "ncclCommGetAsyncError");
+    LIGER_SYM(GetErrorString, "ncclGetErrorString");
+#undef LIGER_SYM
+    api.ok = api.GetUniqueId && api.CommInitRank && api.AllReduce && api.AllGather && api.GroupStart &&
+             api.GroupEnd && api.CommDestroy && api.GetErrorString;
+  });
+  return api;
+}
+
+static ncclDataType_t nccl_dt(CommDType d) {
+  return d == CD_BF16 ? ncclBfloat16 : d == CD_F32 ? ncclFloat32 : ncclInt32;
+}
+static size_t dt_size(CommDType d) { return d == CD_BF16 ? 2 : 4; }
+
+struct NcclComm : Comm {
+  ncclComm_t comm = nullptr;
+  ~NcclComm() override {
+    if (comm) nccl().CommDestroy(comm);
+  }
+  int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
+    if (!count) return 0;
+    ncclResult_t r = nccl().AllReduce(buf, buf, count, nccl_dt(dt), op == CO_SUM ? ncclSum : ncclMax, comm, st);
+    if (r != ncclSuccess) {
+      err = std::string("ncclAllReduce: ") + nccl().GetErrorString(r);
+      return LIGER_ENCCL;
+    }
+    return 0;
+  }
+  int allgather2(const void* s0, void* r0, size_t n0, CommDType d0, const void* s1, void* r1, size_t n1,
+                 CommDType d1, cudaStream_t st) override {
+    nccl().GroupStart();
+    nccl().AllGather(s0, r0, n0, nccl_dt(d0), comm, st);
+    nccl().AllGather(s1, r1, n1, nccl_dt(d1), comm, st);
+    ncclResult_t r = nccl().GroupEnd();
+    if (r != ncclSuccess) {
+      err = std::string("ncclAllGather: ") + nccl().GetErrorString(r);
+      return LIGER_ENCCL;
+    }
+    return 0;
+  }
+  int check_async() override {
+    if (!nccl().CommGetAsyncError) return 0;
+    ncclResult_t a = ncclSuccess;
+    nccl().CommGetAsyncError(comm, &a);
+    if (a != ncclSuccess && a != ncclInProgress) {
+      err = std::string("NCCL async error: ") + nccl().GetErrorString(a);
+      return LIGER_ENCCL;
+    }
+    return 0;
+  }
+};
+
+// ------------------------------------------------------------------ loopback (ranks = threads, one GPU)
+struct LoopGroup {
+  int world;
+  std::mutex mu;
+  std::condition_variable cv;
+  int arrived = 0;
+  uint64_t gen = 0;
+  // per-rank operands, double-buffered by generation parity: a rank can deposit
+  // for generation g+1 while slower ranks still read generation g, and cannot
+  // reach g+2 before every rank has left g.
+  std::vector<const void*> a[2], b[2];
+  std::vector<cudaEvent_t> ev[2];
+  int members = 0;
+};
+
+static std::mutex g_groups_mu;
+static std::map<std::string, LoopGroup*> g_groups;
+
+constexpr int LOOP_MAX_WORLD = 8;
+template <typename T>
+struct RankPtrs {
+  const T* p[LOOP_MAX_WORLD];
+};
+
+// out[i] = reduce over ranks q = 0..world-1 (in order) of in_q[i]
+template <typename T, bool MAX>
+__global__ void loop_reduce_kernel(const RankPtrs<T> in, int world, T* out, size_t n) {
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    float acc = (float)in.p[0][i];
+    for (int q = 1; q < world; ++q) acc = MAX ? fmaxf(acc, (float)in.p[q][i]) : acc + (float)in.p[q][i];
+    out[i] = (T)acc;
+  }
+}
+template <bool MAX>
+__global__ void loop_reduce_bf16_kernel(const RankPtrs<__nv_bfloat16> in, int world, __nv_bfloat16* out, size_t n) {
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    float acc = __bfloat162float(in.p[0][i]);
+    for (int q = 1; q < world; ++q) {
+      const float v = __bfloat162float(in.p[q][i]);
+      acc = MAX ? fmaxf(acc, v) : acc + v;
+    }
+    out[i] = __float2bfloat16_rn(acc);
+  }
+}
+
+struct LoopbackComm : Comm {
+  LoopGroup* g = nullptr;
+  std::string key;
+  int world = 1, rank = 0;
+  cudaEvent_t ev_ready = nullptr, ev_done = nullptr;
+  void* scratch = nullptr;
+  size_t scratch_bytes = 0;
+  ~LoopbackComm() override {
+    cudaDeviceSynchronize();
+    if (ev_ready) cudaEventDestroy(ev_ready);
+    if (ev_done) cudaEventDestroy(ev_done);
+    if (scratch) cudaFree(scratch);
+    std::lock_guard<std::mutex> l(g_groups_mu);
+    if (g && --g->members == 0) {
+      g_groups.erase(key);
+      delete g;
+    }
+  }
+  // host rendezvous: deposit (x, y, e) for this rank, wait for all ranks, return everyone's
+  void rendezvous(const void* x, const void* y, cudaEvent_t e, std::vector<const void*>* xs,
+                  std::vector<const void*>* ys, std::vector<cudaEvent_t>* es) {
+    std::unique_lock<std::mutex> l(g->mu);
+    const uint64_t my_gen = g->gen;
+    const int par = (int)(my_gen & 1);
+    g->a[par][rank] = x;
+    g->b[par][rank] = y;
+    g->ev[par][rank] = e;
+    if (++g->arrived == world) {
+      g->arrived = 0;
+      ++g->gen;
+      g->cv.notify_all();
+    } else {
+      g->cv.wait(l, [&] { return g->gen != my_gen; });
+    }
+    *xs = g->a[par];
+    *ys = g->b[par];
+    *es = g->ev[par];
+  }
+  void wait_all(const std::vector<cudaEvent_t>& es, cudaStream_t st) {
+    for (int q = 0; q < world; ++q) cudaStreamWaitEvent(st, es[q], 0);
+  }
+  int ensure_scratch(size_t bytes) {
+    if (bytes <= scratch_bytes) return 0;
+    cudaDeviceSynchronize();
+    if (scratch) cudaFree(scratch);
+    if (cudaMalloc(&scratch, bytes) != cudaSuccess) return LIGER_ENOMEM;
+    scratch_bytes = bytes;
+    return 0;
+  }
+  int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
+    if (!count) return 0;
+    const size_t bytes = count * dt_size(dt);
+    if (int rc = ensure_scratch(bytes)) return rc;
+    std::vector<const void*> xs, ys;
+    std::vector<cudaEvent_t> es;
+    cudaEventRecord(ev_ready, st);
+    rendezvous(buf, nullptr, ev_ready, &xs, &ys, &es);
+    wait_all(es, st);
+    const int blocks = (int)std::min<size_t>((count + 255) / 256, 148 * 8);
+    if (dt == CD_BF16) {
+      RankPtrs<__nv_bfloat16> in{};
+      for (int q = 0; q < world; ++q) in.p[q] = (const __nv_bfloat16*)xs[q];
+      if (op == CO_SUM)
+        loop_reduce_bf16_kernel<false><<<blocks, 256, 0, st>>>(in, world, (__nv_bfloat16*)scratch, count);
+      else
+        loop_reduce_bf16_kernel<true><<<blocks, 256, 0, st>>>(in, world, (__nv_bfloat16*)scratch, count);
+    } else if (dt == CD_F32) {
+      RankPtrs<float> in{};
+      for (int q = 0; q < world; ++q) in.p[q] = (const float*)xs[q];
+      if (op == CO_SUM)
+        loop_reduce_kernel<float, false><<<blocks, 256, 0, st>>>(in, world, (float*)scratch, count);
+      else
+        loop_reduce_kernel<float, true><<<blocks, 256, 0, st>>>(in, world, (float*)scratch, count);
+    } else {
+      return LIGER_EINVAL;
+    }
+    // every rank has read every input before anyone overwrites its buffer
+    cudaEventRecord(ev_done, st);
+    rendezvous(nullptr, nullptr, ev_done, &xs, &ys, &es);
+    wait_all(es, st);
+    cudaMemcpyAsync(buf, scratch, bytes, cudaMemcpyDeviceToDevice, st);
+    return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  }
+  int allgather2(const void* s0, void* r0, size_t n0, CommDType d0, const void* s1, void* r1, size_t n1,
+                 CommDType d1, cudaStream_t st) override {
+    std::vector<const void*> xs, ys;
+    std::vector<cudaEvent_t> es;
+    cudaEventRecord(ev_ready, st);
+    rendezvous(s0, s1, ev_ready, &xs, &ys, &es);
+    wait_all(es, st);
+    const size_t b0 = n0 * dt_size(d0), b1 = n1 * dt_size(d1);
+    for (int q = 0; q < world; ++q) {
+      if (xs[q] != (char*)r0 + q * b0) cudaMemcpyAsync((char*)r0 + q * b0, xs[q], b0, cudaMemcpyDeviceToDevice, st);
+      if (ys[q] != (char*)r1 + q * b1) cudaMemcpyAsync((char*)r1 + q * b1, ys[q], b1, cudaMemcpyDeviceToDevice, st);
+    }
+    cudaEventRecord(ev_done, st);
+    rendezvous(nullptr, nullptr, ev_done, &xs, &ys, &es);
+    wait_all(es, st);
+    return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  }
+  int check_async() override { return 0; }
+};
+
+static const char kLoopMagic[16] = {'L', 'I', 'G', 'E', 'R', '-', 'L', 'O', 'O', 'P', 'B', 'A', 'C', 'K', ':', 0};
+
+bool uid_is_loopback(const uint8_t* uid) { return uid && memcmp(uid, kLoopMagic, 16) == 0; }
+
+void make_loopback_uid(uint8_t* uid) {
+  memset(uid, 0, 128);
+  memcpy(uid, kLoopMagic, 16);
+  std::random_device rd;
+  for (int i = 16; i < 48; ++i) uid[i] = (uint8_t)(rd() & 0xff);
+}
+
+Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err) {
+  if (uid_is_loopback(uid)) {
+    auto* c = new LoopbackComm();
+    c->world = world;
+    c->rank = rank;
+    c->key.assign((const char*)uid, 48);
+    {
+      std::lock_guard<std::mutex> l(g_groups_mu);
+      LoopGroup*& g = g_groups[c->key];
+      if (!g) {
+        g = new LoopGroup();
+        g->world = world;
+        for (int i = 0; i < 2; ++i) {
+          g->a[i].assign(world, nullptr);
+          g->b[i].assign(world, nullptr);
+          g->ev[i].assign(world, nullptr);
+        }
+      }
+      if (g->world != world) {
+        *err = "loopback group world size mismatch";
+        delete c;
+        return nullptr;
+      }
+      ++g->members;
+      c->g = g;
+    }
+    if (world > LOOP_MAX_WORLD) {
+      *err = "loopback communicator: at most 8 ranks";
+      delete c;
+      return nullptr;
+    }
+    if (cudaEventCreateWithFlags(&c->ev_ready, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->ev_done, cudaEventDisableTiming) != cudaSuccess) {
+      *err = "loopback communicator: CUDA allocation failed";
+      delete c;
+      return nullptr;
+    }
+    return c;
+  }
+  if (!nccl().ok) {
+    *err = "NCCL library not loadable";
+    return nullptr;
+  }
+  ncclUniqueId id;
+  memcpy(&id, uid, sizeof(id));
+  auto* c = new NcclComm();
+  ncclResult_t r = nccl().CommInitRank(&c->comm, world, id, rank);
+  if (r != ncclSuccess) {
+    *err = std::string("ncclCommInitRank: ") + nccl().GetErrorString(r);
+    c->comm = nullptr;
+    delete c;
+    return nullptr;
+  }
+  return c;
+}
+
+}  // namespace liger

@@ -1,0 +1,45 @@
+// Communication backend interface of the tensor-parallel ranks (see comm.cu).
+#pragma once
+#include <cuda_runtime.h>
+#include <nccl.h>
+#include <stddef.h>
+#include <stdint.h>
+
+#include <string>
+
+namespace liger {
+
+struct NcclApi {
+  bool ok = false;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t*) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+NcclApi& nccl();
+
+enum CommDType { CD_BF16, CD_F32, CD_I32 };
+enum CommOp { CO_SUM, CO_MAX };
+
+struct Comm {
+  std::string err;
+  virtual ~Comm() {}
+  // in-place all-reduce of `count` elements
+  virtual int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) = 0;
+  // two all-gathers issued as one group: recv[q * n + i] = send_q[i]
+  virtual int allgather2(const void* s0, void* r0, size_t n0, CommDType d0, const void* s1, void* r1, size_t n1,
+                         CommDType d1, cudaStream_t st) = 0;
+  virtual int check_async() = 0;
+};
+
+Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err);
+bool uid_is_loopback(const uint8_t* uid);
+void make_loopback_uid(uint8_t* uid);
+
+}  // namespace liger

@@ -24,6 +24,7 @@
 #include <string>
 #include <vector>
 
+#include "comm.h"
 #include "kernels.h"
 #include "planner.h"
 
@@ -35,47 +36,7 @@ int check_device();
 
 using namespace liger;
 
-// ------------------------------------------------------------------ NCCL (dlopen)
 namespace {
-struct NcclApi {
-  bool ok = false;
-  ncclResult_t (*GetUniqueId)(ncclUniqueId*);
-  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int);
-  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t);
-  ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t);
-  ncclResult_t (*GroupStart)();
-  ncclResult_t (*GroupEnd)();
-  ncclResult_t (*CommDestroy)(ncclComm_t);
-  ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t*);
-  const char* (*GetErrorString)(ncclResult_t);
-};
-
-NcclApi& nccl() {
-  static NcclApi api;
-  static bool tried = false;
-  if (tried) return api;
-  tried = true;
-  const char* names[] = {"libnccl.so.2", "libnccl.so",
-                         "/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl/lib/libnccl.so.2"};
-  void* h = nullptr;
-  for (const char* n : names)
-    if ((h = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
-  if (!h) return api;
-#define LIGER_SYM(field, name) api.field = reinterpret_cast<decltype(api.field)>(dlsym(h, name))
-  LIGER_SYM(GetUniqueId, "ncclGetUniqueId");
-  LIGER_SYM(CommInitRank, "ncclCommInitRank");
-  LIGER_SYM(AllReduce, "ncclAllReduce");
-  LIGER_SYM(AllGather, "ncclAllGather");
-  LIGER_SYM(GroupStart, "ncclGroupStart");
-  LIGER_SYM(GroupEnd, "ncclGroupEnd");
-  LIGER_SYM(CommDestroy, "ncclCommDestroy");
-  LIGER_SYM(CommGetAsyncError, "ncclCommGetAsyncError");
-  LIGER_SYM(GetErrorString, "ncclGetErrorString");
-#undef LIGER_SYM
-  api.ok = api.GetUniqueId && api.CommInitRank && api.AllReduce && api.AllGather && api.GroupStart &&
-           api.GroupEnd && api.CommDestroy;
-  return api;
-}
 
 double now_s() {
   timespec ts;
@@ -171,7 +132,7 @@ struct liger_ctx {
   int h, a, d, f, V, hl, al, fl, Vl, L, F;
   double cf;
   std::string err;
-  ncclComm_t comm = nullptr;
+  Comm* comm = nullptr;   // NCCL or loopback (comm.cu); nullptr at world == 1
   cudaStream_t s_comp = nullptr, s_comm = nullptr;
   std::vector<LayerW> layers;
   void *e_tok = nullptr, *e_pos = nullptr, *lnf_g = nullptr, *lnf_b = nullptr;
@@ -491,9 +452,8 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       const size_t e0 = E * u0 / F, e1 = E * u1 / F;
       timed_begin(c, st, &ta);
       if (e1 > e0) {
-        ncclResult_t r = nccl().AllReduce((char*)S.part + e0 * 2, (char*)S.part + e0 * 2, e1 - e0, ncclBfloat16,
-                                          ncclSum, c->comm, st);
-        if (r != ncclSuccess) return fail(c, LIGER_ENCCL, std::string("ncclAllReduce: ") + nccl().GetErrorString(r));
+        if (c->comm->allreduce((char*)S.part + e0 * 2, e1 - e0, CD_BF16, CO_SUM, st))
+          return fail(c, LIGER_ENCCL, c->comm->err);
       }
       timed_end(c, st, ta, LIGER_KT_ALLREDUCE, (double)(e1 - e0) * 2, 0);
       c->st.comm_kernels++;
@@ -530,11 +490,9 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
     }
     case OP_TOKG: {
       const int b = bt->b;
-      nccl().GroupStart();
-      nccl().AllGather(S.vals_all + (size_t)c->rank * b, S.vals_all, b, ncclFloat32, c->comm, st);
-      nccl().AllGather(S.idx_all + (size_t)c->rank * b, S.idx_all, b, ncclInt32, c->comm, st);
-      ncclResult_t r = nccl().GroupEnd();
-      if (r != ncclSuccess) return fail(c, LIGER_ENCCL, "ncclAllGather failed");
+      if (c->comm->allgather2(S.vals_all + (size_t)c->rank * b, S.vals_all, b, CD_F32,
+                              S.idx_all + (size_t)c->rank * b, S.idx_all, b, CD_I32, st))
+        return fail(c, LIGER_ENCCL, c->comm->err);
       c->st.comm_kernels++;
       c->st.gpu_launches++;
       break;
@@ -711,6 +669,12 @@ int launch_run(liger_ctx* c, const std::vector<Piece>& pieces, const std::vector
 // ================================================================== C ABI
 extern "C" {
 
+int liger_loopback_unique_id(uint8_t* uid) {
+  if (!uid) return LIGER_EINVAL;
+  make_loopback_uid(uid);
+  return LIGER_OK;
+}
+
 int liger_nccl_unique_id(uint8_t* uid) {
   if (!uid) return LIGER_EINVAL;
   if (!nccl().ok) return fail(nullptr, LIGER_ENCCL, "NCCL library not loadable");
@@ -740,12 +704,10 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (world > 2);
   if (world > 1) {
-    if (!nccl().ok) return fail(nullptr, LIGER_ENCCL, "NCCL library not loadable");
     if (!nccl_uid) return fail(nullptr, LIGER_EINVAL, "liger_init: nccl_uid required for world > 1");
-    ncclUniqueId id;
-    memcpy(&id, nccl_uid, sizeof(id));
-    ncclResult_t r = nccl().CommInitRank(&c->comm, world, id, rank);
-    if (r != ncclSuccess) return fail(nullptr, LIGER_ENCCL, std::string("ncclCommInitRank: ") + nccl().GetErrorString(r));
+    std::string err;
+    c->comm = comm_create(world, rank, nccl_uid, &err);
+    if (!c->comm) return fail(nullptr, LIGER_ENCCL, "liger_init: " + err);
   }
   int lo, hi;
   cudaDeviceGetStreamPriorityRange(&lo, &hi);
@@ -1110,12 +1072,15 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
                        double* detail /* [n_m][4][2] slowdowns (gemm, ar) or NULL */) {
   if (!c || !m_list || n_m <= 0) return LIGER_EINVAL;
   if (!c->processing.empty() || !c->waiting.empty()) return fail(c, LIGER_ESTATE, "liger_calibrate_cf: batches in flight");
-  if (!nccl().ok) return fail(c, LIGER_ENCCL, "NCCL library not loadable");
-  ncclComm_t comm = c->comm, own = nullptr;
-  if (!comm) {
+  Comm* comm = c->comm;
+  Comm* own = nullptr;
+  if (!comm) {   // t = 1: a 1-rank NCCL communicator's all-reduce kernel as the proxy
+    if (!nccl().ok) return fail(c, LIGER_ENCCL, "NCCL library not loadable");
     ncclUniqueId id;
-    if (nccl().GetUniqueId(&id) != ncclSuccess || nccl().CommInitRank(&own, 1, id, 0) != ncclSuccess)
-      return fail(c, LIGER_ENCCL, "liger_calibrate_cf: 1-rank NCCL communicator");
+    if (nccl().GetUniqueId(&id) != ncclSuccess) return fail(c, LIGER_ENCCL, "ncclGetUniqueId failed");
+    std::string err;
+    own = comm_create(1, 0, reinterpret_cast<const uint8_t*>(&id), &err);
+    if (!own) return fail(c, LIGER_ENCCL, "liger_calibrate_cf: " + err);
     comm = own;
   }
   CK(cudaDeviceSynchronize());
@@ -1130,9 +1095,7 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
   fake.n_new = 1;
   fake.b = 1;
   double cf = 1.0;
-  auto ar = [&](size_t elems) {
-    nccl().AllReduce(S.part, S.part, elems, ncclBfloat16, ncclSum, comm, c->s_comm);
-  };
+  auto ar = [&](size_t elems) { comm->allreduce(S.part, elems, CD_BF16, CO_SUM, c->s_comm); };
   for (int mi = 0; mi < n_m; ++mi) {
     const int M = std::min<int>(m_list[mi], Mmax);
     fake.s = M;
@@ -1178,13 +1141,13 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
   }
   c->timing = saved_timing;
   for (auto& e : ev) cudaEventDestroy(e);
-  if (own) nccl().CommDestroy(own);
+  delete own;
   if (c->world > 1) {   // all ranks must use the same cf (identical plans)
     float* dv = nullptr;
     float v = (float)cf;
     CK(cudaMalloc(&dv, 4));
     CK(cudaMemcpy(dv, &v, 4, cudaMemcpyHostToDevice));
-    nccl().AllReduce(dv, dv, 1, ncclFloat32, ncclMax, c->comm, c->s_comp);
+    if (c->comm->allreduce(dv, 1, CD_F32, CO_MAX, c->s_comp)) return fail(c, LIGER_ENCCL, c->comm->err);
     CK(cudaMemcpyAsync(&v, dv, 4, cudaMemcpyDeviceToHost, c->s_comp));
     CK(cudaStreamSynchronize(c->s_comp));
     cudaFree(dv);
@@ -1254,7 +1217,7 @@ int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
       for (int k = 1; k <= op_units(c, OP_AR1); ++k) {
         const int kk = op_units(c, OP_AR1) > 1 ? k : F;
         const double t = time_it([&] {
-          nccl().AllReduce(S.part, S.part, E * k / op_units(c, OP_AR1), ncclBfloat16, ncclSum, c->comm, st);
+          c->comm->allreduce(S.part, E * k / op_units(c, OP_AR1), CD_BF16, CO_SUM, st);
         });
         liger_set_duration(c, OP_AR1, M, kk, t * 1e6);
         liger_set_duration(c, OP_AR2, M, kk, t * 1e6);
@@ -1304,7 +1267,7 @@ int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
     float* dv = nullptr;
     CK(cudaMalloc(&dv, flat.size() * 4));
     CK(cudaMemcpy(dv, flat.data(), flat.size() * 4, cudaMemcpyHostToDevice));
-    nccl().AllReduce(dv, dv, flat.size(), ncclFloat32, ncclMax, c->comm, st);
+    if (c->comm->allreduce(dv, flat.size(), CD_F32, CO_MAX, st)) return fail(c, LIGER_ENCCL, c->comm->err);
     CK(cudaMemcpyAsync(flat.data(), dv, flat.size() * 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     cudaFree(dv);
@@ -1324,7 +1287,7 @@ const char* liger_last_error(const liger_ctx* c) { return c ? c->err.c_str() : g
 int liger_finalize(liger_ctx* c) {
   if (!c) return LIGER_EINVAL;
   cudaDeviceSynchronize();
-  if (c->comm) nccl().CommDestroy(c->comm);
+  delete c->comm;
   for (void* p : c->allocs) cudaFree(p);
   for (auto& S : c->slots) {
     cudaFreeHost(S.h_page_table);

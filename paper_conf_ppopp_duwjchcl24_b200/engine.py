@@ -44,6 +44,13 @@ class LigerEngine:
         L.check(L.lib().liger_nccl_unique_id(buf), None, "liger_nccl_unique_id")
         return buf.raw
 
+    @staticmethod
+    def loopback_id():
+        """Id for ranks running as threads of this process on one GPU (test vehicle)."""
+        buf = C.create_string_buffer(128)
+        L.check(L.lib().liger_loopback_unique_id(buf), None, "liger_loopback_unique_id")
+        return buf.raw
+
     def _chk(self, rc, what):
         return L.check(rc, self.ctx, what)
 

@@ -46,6 +46,7 @@ _P, _I, _I64, _F, _SZ, _U64, _D = C.c_void_p, C.c_int, C.c_int64, C.c_float, C.c
 _SIGS = {
     "liger_init": (_I, [_I, _I, C.POINTER(liger_cfg), _P, C.POINTER(_P)]),
     "liger_nccl_unique_id": (_I, [_P]),
+    "liger_loopback_unique_id": (_I, [_P]),
     "liger_load_layer": (_I, [_P, _I, _U64]),
     "liger_load_embed": (_I, [_P, _U64]),
     "liger_submit": (_I64, [_P, _I, _I, _P, _I, _I, _D]),
