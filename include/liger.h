@@ -138,8 +138,9 @@ int64_t liger_submit(liger_ctx* ctx, int batch, int seq_len, const int32_t* toke
 /* One scheduling round (one iteration of Algorithm 1): update the
  * processing list, wait for the running round's E1 event (hybrid sync,
  * P:236), plan SubSet0/SubSet1 and launch them (communication first) gated
- * on the running round's E2 event.  Returns the number of kernel pieces
- * launched (>= 0), LIGER_IDLE when no batch is pending, or an error.
+ * on the running round's E2 event.  Returns LIGER_OK after a round (or while
+ * waiting batches cannot be admitted yet), LIGER_IDLE when no batch is
+ * pending, or an error; launched pieces are counted in liger_stats().
  * [collective] */
 int liger_step(liger_ctx* ctx);
 
