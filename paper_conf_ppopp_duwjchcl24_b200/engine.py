@@ -64,6 +64,11 @@ class LigerEngine:
         arr = (C.c_int32 * len(m_list))(*m_list)
         self._chk(L.lib().liger_profile(self.ctx, arr, len(m_list)), "liger_profile")
 
+    def set_duration(self, op, m_tokens, k_of_F, us):
+        """Duration-table entry for kernel class `op` (liger.OPS name)."""
+        self._chk(L.lib().liger_set_duration(self.ctx, L.OPS.index(op), m_tokens, k_of_F, float(us)),
+                  "liger_set_duration")
+
     def calibrate_cf(self, m_list, set_cf=True):
         arr = (C.c_int32 * len(m_list))(*m_list)
         cf = C.c_double()

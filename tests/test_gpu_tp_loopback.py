@@ -28,7 +28,7 @@ def E():
     return LigerEngine
 
 
-def serve_tp(E, cfg, world, trace, **kw):
+def serve_tp(E, cfg, world, trace, durations=None, **kw):
     """Run `trace` on `world` loopback ranks; returns (tokens per batch, stats) of each rank."""
     uid = E.loopback_id()
     out = [None] * world
@@ -38,6 +38,8 @@ def serve_tp(E, cfg, world, trace, **kw):
         try:
             torch.cuda.set_device(0)
             eng = E(cfg, world=world, rank=r, nccl_uid=uid, **kw)
+            for args in durations or ():
+                eng.set_duration(*args)
             ids = [eng.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], t["arrival_s"]) for t in trace]
             eng.drain()
             toks = [eng.poll(i, want_tokens=True)[1] for i in ids]
@@ -95,3 +97,28 @@ def test_interleaved_equals_serial_bit_exact(E, world):
         for i in range(t["batch"]):
             n = int(np.argmin(ok[i])) if not ok[i].all() else t["n_decode"]
             assert np.array_equal(toks[i, :n], ref[i, :n])
+
+
+def test_runtime_decomposition_bit_exact(E):
+    """§3.6: with a duration table where the GEMMs are much longer than the
+    all-reduce windows, Algorithm 1 must split secondary GEMMs into k/F pieces
+    (P:254-262); the result stays bit-identical to serial TP."""
+    cfg = get_config("tiny")
+    F = 8
+    dur = []
+    for m in (1, 4096):
+        for op in ("qkv", "out", "fc1", "fc2"):
+            for k in range(1, F + 1):
+                dur.append((op, m, k, 20.0 + 200.0 * k / F))
+        for op in ("ar1", "ar2"):
+            for k in range(1, F + 1):
+                dur.append((op, m, k, 10.0 + 60.0 * k / F))
+    trace = make_trace(4, float("inf"), seed=12, batch_sizes=(2,), prompt_range=(16, 32), n_decode=4,
+                       vocab=cfg.vocab)
+    base = serve_tp(E, cfg, 2, trace, mode="serial", max_batch=2, max_seq=32, max_new=4, seed=4)
+    inter = serve_tp(E, cfg, 2, trace, durations=dur, mode="interleaved", max_batch=2, max_seq=32, max_new=4,
+                     max_inflight=2, decomp_factor=F, contention_factor=1.0, seed=4)
+    for (tb, _), (ti, st) in zip(base, inter):
+        for a, b in zip(tb, ti):
+            assert np.array_equal(a, b)
+    assert inter[0][1]["split_pieces"] > 0, inter[0][1]
