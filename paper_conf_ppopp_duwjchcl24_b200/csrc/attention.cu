@@ -27,7 +27,7 @@ __device__ __forceinline__ int64_t kv_off(int page, int kv, int heads, int head,
 }
 
 // ================================================================== prefill
-constexpr int PF_BQ = 64, PF_BK = 64;
+constexpr int PF_BQ = 128, PF_BK = 64;
 
 __device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
   asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
@@ -52,32 +52,65 @@ __device__ __forceinline__ uint32_t pack_bf16(float lo, float hi) {
   return *reinterpret_cast<uint32_t*>(&v);
 }
 
+__device__ __forceinline__ void cp_async16(void* smem_dst, const void* gsrc, bool valid) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(smem_dst)), "l"(gsrc),
+               "r"(valid ? 16 : 0)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
+// Prefill causal attention, flash-style: CTA = (128-query tile, head, sequence),
+// 8 warps x 16 query rows; 64-key tiles of K and V double-buffered in shared
+// memory with cp.async (the next tile loads while the current one is
+// computed); S = Q K^T and O += P V on bf16 tensor cores (mma.sync m16n8k16,
+// fp32 accumulate); online softmax in registers.  The CTA whose query range
+// contains a key tile also writes that tile's K/V into the paged cache.
+constexpr int PF_THREADS = 256;
 template <int D>
-__global__ void __launch_bounds__(128) attn_prefill_kernel(const __nv_bfloat16* __restrict__ qkv,
-                                                           __nv_bfloat16* __restrict__ o,
-                                                           __nv_bfloat16* __restrict__ kv_pool,
-                                                           const int32_t* __restrict__ page_table, int max_pages,
-                                                           int s, int heads) {
+__global__ void __launch_bounds__(PF_THREADS) attn_prefill_kernel(const __nv_bfloat16* __restrict__ qkv,
+                                                                  __nv_bfloat16* __restrict__ o,
+                                                                  __nv_bfloat16* __restrict__ kv_pool,
+                                                                  const int32_t* __restrict__ page_table,
+                                                                  int max_pages, int s, int heads) {
   constexpr int LDS = D + 8;   // padded smem row (bank-conflict-free ldmatrix)
   constexpr int NV = D / 8;    // 16-byte vectors per row
   extern __shared__ __align__(16) uint8_t pf_smem[];
-  __nv_bfloat16* sQ = reinterpret_cast<__nv_bfloat16*>(pf_smem);
-  __nv_bfloat16* sK = sQ + PF_BQ * LDS;
-  __nv_bfloat16* sV = sK + PF_BK * LDS;
+  __nv_bfloat16* sQ = reinterpret_cast<__nv_bfloat16*>(pf_smem);       // [PF_BQ][LDS]
+  __nv_bfloat16* sK = sQ + PF_BQ * LDS;                                  // [2][PF_BK][LDS]
+  __nv_bfloat16* sV = sK + 2 * PF_BK * LDS;                              // [2][PF_BK][LDS]
 
-  pdl_enter();
-  const int qt = blockIdx.x, head = blockIdx.y, bi = blockIdx.z;
+  const int nqt = gridDim.x;
+  const int qt = nqt - 1 - blockIdx.x;   // longest (most key tiles) first
+  const int head = blockIdx.y, bi = blockIdx.z;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t ld = (int64_t)3 * heads * D;
   const __nv_bfloat16* base = qkv + (int64_t)bi * s * ld;
   const int q0 = qt * PF_BQ;
+  const int q_hi = min(s, q0 + PF_BQ);            // rows [q0, q_hi)
+  const int nkt = (q_hi - 1) / PF_BK + 1;         // key tiles with k0 <= last row
+  pdl_enter();
 
-  for (int i = tid; i < PF_BQ * NV; i += 128) {
+  auto load_kv = [&](int kt, int buf) {
+    const int k0 = kt * PF_BK;
+    for (int i = tid; i < PF_BK * NV; i += PF_THREADS) {
+      const int r = i / NV, c = (i % NV) * 8;
+      const bool ok = k0 + r < s;
+      const __nv_bfloat16* rowp = base + (int64_t)(ok ? k0 + r : 0) * ld;
+      cp_async16(&sK[(buf * PF_BK + r) * LDS + c], rowp + (int64_t)heads * D + head * D + c, ok);
+      cp_async16(&sV[(buf * PF_BK + r) * LDS + c], rowp + (int64_t)2 * heads * D + head * D + c, ok);
+    }
+  };
+  for (int i = tid; i < PF_BQ * NV; i += PF_THREADS) {
     const int r = i / NV, c = (i % NV) * 8;
-    uint4 v = make_uint4(0, 0, 0, 0);
-    if (q0 + r < s) v = *reinterpret_cast<const uint4*>(base + (int64_t)(q0 + r) * ld + head * D + c);
-    *reinterpret_cast<uint4*>(&sQ[r * LDS + c]) = v;
+    const bool ok = q0 + r < s;
+    cp_async16(&sQ[r * LDS + c], base + (int64_t)(ok ? q0 + r : 0) * ld + head * D + c, ok);
   }
+  load_kv(0, 0);
+  cp_async_commit();
 
   const int g = lane >> 2, tig = lane & 3;
   float m_r[2] = {-INFINITY, -INFINITY}, l_r[2] = {0.f, 0.f};
@@ -85,110 +118,112 @@ __global__ void __launch_bounds__(128) attn_prefill_kernel(const __nv_bfloat16* 
 #pragma unroll
   for (int j = 0; j < D / 8; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
   const float L2E = 1.4426950408889634f;
-  const int row0 = q0 + warp * 16 + g;   // this thread's rows: row0, row0 + 8
+  const int wrow0 = q0 + warp * 16;        // this warp's rows [wrow0, wrow0 + 16)
+  const int row0 = wrow0 + g;              // this thread's rows: row0, row0 + 8
 
-  for (int kt = 0; kt <= qt; ++kt) {
+  for (int kt = 0; kt < nkt; ++kt) {
+    const int buf = kt & 1;
     const int k0 = kt * PF_BK;
+    if (kt + 1 < nkt) load_kv(kt + 1, buf ^ 1);
+    cp_async_commit();
+    cp_async_wait<1>();   // tile kt (and Q) landed
     __syncthreads();
-    for (int i = tid; i < PF_BK * NV; i += 128) {
-      const int r = i / NV, c = (i % NV) * 8;
-      uint4 kv = make_uint4(0, 0, 0, 0), vv = make_uint4(0, 0, 0, 0);
-      if (k0 + r < s) {
-        const __nv_bfloat16* rowp = base + (int64_t)(k0 + r) * ld;
-        kv = *reinterpret_cast<const uint4*>(rowp + (int64_t)heads * D + head * D + c);
-        vv = *reinterpret_cast<const uint4*>(rowp + (int64_t)2 * heads * D + head * D + c);
-        if (kt == qt) {   // diagonal CTA appends this key tile to the paged cache
-          const int p = k0 + r;
+    const __nv_bfloat16* cK = sK + buf * PF_BK * LDS;
+    const __nv_bfloat16* cV = sV + buf * PF_BK * LDS;
+    if (k0 >= q0 && k0 < q0 + PF_BQ) {   // this CTA appends key tile kt to the paged cache
+      for (int i = tid; i < PF_BK * NV; i += PF_THREADS) {
+        const int r = i / NV, c = (i % NV) * 8;
+        const int p = k0 + r;
+        if (p < s) {
           const int page = page_table[(int64_t)bi * max_pages + p / KVB];
-          *reinterpret_cast<uint4*>(kv_pool + kv_off(page, 0, heads, head, p % KVB, D) + c) = kv;
-          *reinterpret_cast<uint4*>(kv_pool + kv_off(page, 1, heads, head, p % KVB, D) + c) = vv;
+          *reinterpret_cast<uint4*>(kv_pool + kv_off(page, 0, heads, head, p % KVB, D) + c) =
+              *reinterpret_cast<const uint4*>(&cK[r * LDS + c]);
+          *reinterpret_cast<uint4*>(kv_pool + kv_off(page, 1, heads, head, p % KVB, D) + c) =
+              *reinterpret_cast<const uint4*>(&cV[r * LDS + c]);
         }
       }
-      *reinterpret_cast<uint4*>(&sK[r * LDS + c]) = kv;
-      *reinterpret_cast<uint4*>(&sV[r * LDS + c]) = vv;
     }
-    __syncthreads();
-
-    // S = Q K^T for this warp's 16 rows x 64 keys
-    float sc[8][4];
+    if (k0 <= wrow0 + 15 && wrow0 < s) {   // warp-uniform: some key of this tile is visible to the warp
+      float sc[8][4];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) sc[j][0] = sc[j][1] = sc[j][2] = sc[j][3] = 0.f;
+      for (int j = 0; j < 8; ++j) sc[j][0] = sc[j][1] = sc[j][2] = sc[j][3] = 0.f;
 #pragma unroll
-    for (int kc = 0; kc < D; kc += 16) {
-      uint32_t a0, a1, a2, a3;
-      const int ar = warp * 16 + (lane % 8) + ((lane / 8) % 2) * 8;
-      const int ac = kc + (lane / 16) * 8;
-      ldsm_x4(smem_u32(&sQ[ar * LDS + ac]), a0, a1, a2, a3);
+      for (int kc = 0; kc < D; kc += 16) {
+        uint32_t a0, a1, a2, a3;
+        const int ar = warp * 16 + (lane % 8) + ((lane / 8) % 2) * 8;
+        const int ac = kc + (lane / 16) * 8;
+        ldsm_x4(smem_u32(&sQ[ar * LDS + ac]), a0, a1, a2, a3);
 #pragma unroll
-      for (int nb = 0; nb < 8; nb += 2) {
-        uint32_t b0, b1, b2, b3;
-        const int br = nb * 8 + (lane % 8) + (lane / 16) * 8;
-        const int bc = kc + ((lane / 8) % 2) * 8;
-        ldsm_x4(smem_u32(&sK[br * LDS + bc]), b0, b1, b2, b3);
-        mma_bf16_16816(sc[nb], a0, a1, a2, a3, b0, b1);
-        mma_bf16_16816(sc[nb + 1], a0, a1, a2, a3, b2, b3);
-      }
-    }
-    // mask (causal on the diagonal tile; key padding beyond s)
-#pragma unroll
-    for (int nb = 0; nb < 8; ++nb) {
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int key = k0 + nb * 8 + tig * 2 + (e & 1);
-        const int row = row0 + (e >> 1) * 8;
-        if (key > row || key >= s) sc[nb][e] = -INFINITY;
-      }
-    }
-    // online softmax
-#pragma unroll
-    for (int h2 = 0; h2 < 2; ++h2) {
-      float mx = -INFINITY;
-#pragma unroll
-      for (int nb = 0; nb < 8; ++nb) mx = fmaxf(mx, fmaxf(sc[nb][2 * h2], sc[nb][2 * h2 + 1]));
-      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
-      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
-      const float m_new = fmaxf(m_r[h2], mx);
-      const float corr = (m_r[h2] == -INFINITY) ? 0.f : exp2f((m_r[h2] - m_new) * L2E);
-      float sum = 0.f;
-#pragma unroll
-      for (int nb = 0; nb < 8; ++nb) {
-#pragma unroll
-        for (int e = 0; e < 2; ++e) {
-          const float v = sc[nb][2 * h2 + e];
-          const float pv = (v == -INFINITY) ? 0.f : exp2f((v - m_new) * L2E);
-          sc[nb][2 * h2 + e] = pv;
-          sum += pv;
+        for (int nb = 0; nb < 8; nb += 2) {
+          uint32_t b0, b1, b2, b3;
+          const int br = nb * 8 + (lane % 8) + (lane / 16) * 8;
+          const int bc = kc + ((lane / 8) % 2) * 8;
+          ldsm_x4(smem_u32(&cK[br * LDS + bc]), b0, b1, b2, b3);
+          mma_bf16_16816(sc[nb], a0, a1, a2, a3, b0, b1);
+          mma_bf16_16816(sc[nb + 1], a0, a1, a2, a3, b2, b3);
         }
       }
-      sum += __shfl_xor_sync(0xffffffffu, sum, 1);
-      sum += __shfl_xor_sync(0xffffffffu, sum, 2);
-      l_r[h2] = l_r[h2] * corr + sum;
-      m_r[h2] = m_new;
+      if (k0 + PF_BK - 1 > wrow0 || k0 + PF_BK > s) {   // diagonal / ragged tile: mask
 #pragma unroll
-      for (int j = 0; j < D / 8; ++j) {
-        acc[j][2 * h2] *= corr;
-        acc[j][2 * h2 + 1] *= corr;
+        for (int nb = 0; nb < 8; ++nb) {
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const int key = k0 + nb * 8 + tig * 2 + (e & 1);
+            const int row = row0 + (e >> 1) * 8;
+            if (key > row || key >= s) sc[nb][e] = -INFINITY;
+          }
+        }
+      }
+#pragma unroll
+      for (int h2 = 0; h2 < 2; ++h2) {
+        float mx = -INFINITY;
+#pragma unroll
+        for (int nb = 0; nb < 8; ++nb) mx = fmaxf(mx, fmaxf(sc[nb][2 * h2], sc[nb][2 * h2 + 1]));
+        mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
+        mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
+        const float m_new = fmaxf(m_r[h2], mx);
+        const float corr = (m_new == -INFINITY) ? 1.f : exp2f((m_r[h2] - m_new) * L2E);
+        float sum = 0.f;
+#pragma unroll
+        for (int nb = 0; nb < 8; ++nb) {
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const float v = sc[nb][2 * h2 + e];
+            const float pv = (v == -INFINITY) ? 0.f : exp2f((v - m_new) * L2E);
+            sc[nb][2 * h2 + e] = pv;
+            sum += pv;
+          }
+        }
+        sum += __shfl_xor_sync(0xffffffffu, sum, 1);
+        sum += __shfl_xor_sync(0xffffffffu, sum, 2);
+        l_r[h2] = l_r[h2] * corr + sum;
+        m_r[h2] = m_new;
+#pragma unroll
+        for (int j = 0; j < D / 8; ++j) {
+          acc[j][2 * h2] *= corr;
+          acc[j][2 * h2 + 1] *= corr;
+        }
+      }
+#pragma unroll
+      for (int kc = 0; kc < 4; ++kc) {   // 16 keys per step
+        const uint32_t a0 = pack_bf16(sc[2 * kc][0], sc[2 * kc][1]);
+        const uint32_t a1 = pack_bf16(sc[2 * kc][2], sc[2 * kc][3]);
+        const uint32_t a2 = pack_bf16(sc[2 * kc + 1][0], sc[2 * kc + 1][1]);
+        const uint32_t a3 = pack_bf16(sc[2 * kc + 1][2], sc[2 * kc + 1][3]);
+#pragma unroll
+        for (int nb = 0; nb < D / 8; nb += 2) {
+          uint32_t b0, b1, b2, b3;
+          const int vr = kc * 16 + (lane % 8) + ((lane / 8) % 2) * 8;
+          const int vc = nb * 8 + (lane / 16) * 8;
+          ldsm_x4_t(smem_u32(&cV[vr * LDS + vc]), b0, b1, b2, b3);
+          mma_bf16_16816(acc[nb], a0, a1, a2, a3, b0, b1);
+          mma_bf16_16816(acc[nb + 1], a0, a1, a2, a3, b2, b3);
+        }
       }
     }
-    // O += P V
-#pragma unroll
-    for (int kc = 0; kc < 4; ++kc) {   // 16 keys per step
-      const uint32_t a0 = pack_bf16(sc[2 * kc][0], sc[2 * kc][1]);
-      const uint32_t a1 = pack_bf16(sc[2 * kc][2], sc[2 * kc][3]);
-      const uint32_t a2 = pack_bf16(sc[2 * kc + 1][0], sc[2 * kc + 1][1]);
-      const uint32_t a3 = pack_bf16(sc[2 * kc + 1][2], sc[2 * kc + 1][3]);
-#pragma unroll
-      for (int nb = 0; nb < D / 8; nb += 2) {
-        uint32_t b0, b1, b2, b3;
-        const int vr = kc * 16 + (lane % 8) + ((lane / 8) % 2) * 8;
-        const int vc = nb * 8 + (lane / 16) * 8;
-        ldsm_x4_t(smem_u32(&sV[vr * LDS + vc]), b0, b1, b2, b3);
-        mma_bf16_16816(acc[nb], a0, a1, a2, a3, b0, b1);
-        mma_bf16_16816(acc[nb + 1], a0, a1, a2, a3, b2, b3);
-      }
-    }
+    __syncthreads();   // buffer `buf` is refilled at iteration kt + 2
   }
-  // normalise and store
+  cp_async_wait<0>();
 #pragma unroll
   for (int h2 = 0; h2 < 2; ++h2) {
     const int row = row0 + h2 * 8;
@@ -209,19 +244,21 @@ int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* 
                         int s, int heads, int d, cudaStream_t stream) {
   if (b <= 0 || s <= 0) return 0;
   dim3 grid((s + PF_BQ - 1) / PF_BQ, heads, b);
-  const size_t smem = (size_t)(PF_BQ + 2 * PF_BK) * (d + 8) * 2;
+  const size_t smem = (size_t)(PF_BQ + 4 * PF_BK) * (d + 8) * 2;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(attn_prefill_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
-    cudaFuncSetAttribute(attn_prefill_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+    cudaFuncSetAttribute(attn_prefill_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (PF_BQ + 4 * PF_BK) * (128 + 8) * 2);
+    cudaFuncSetAttribute(attn_prefill_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (PF_BQ + 4 * PF_BK) * (64 + 8) * 2);
     attr = true;
   }
   int rc;
   if (d == 128)
-    rc = launch_pdl(attn_prefill_kernel<128>, grid, dim3(128), smem, stream, (const __nv_bfloat16*)qkv,
+    rc = launch_pdl(attn_prefill_kernel<128>, grid, dim3(PF_THREADS), smem, stream, (const __nv_bfloat16*)qkv,
                     (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
   else if (d == 64)
-    rc = launch_pdl(attn_prefill_kernel<64>, grid, dim3(128), smem, stream, (const __nv_bfloat16*)qkv,
+    rc = launch_pdl(attn_prefill_kernel<64>, grid, dim3(PF_THREADS), smem, stream, (const __nv_bfloat16*)qkv,
                     (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
   else
     return LIGER_EINVAL;
