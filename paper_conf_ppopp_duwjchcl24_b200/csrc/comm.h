@@ -36,6 +36,8 @@ struct Comm {
   virtual int allgather2(const void* s0, void* r0, size_t n0, CommDType d0, const void* s1, void* r1, size_t n1,
                          CommDType d1, cudaStream_t st) = 0;
   virtual int check_async() = 0;
+  // host-side barrier of the group (loopback: every rank's thread has arrived)
+  virtual void barrier() {}
 };
 
 Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err);

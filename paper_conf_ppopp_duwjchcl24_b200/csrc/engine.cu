@@ -1287,7 +1287,11 @@ const char* liger_last_error(const liger_ctx* c) { return c ? c->err.c_str() : g
 
 int liger_finalize(liger_ctx* c) {
   if (!c) return LIGER_EINVAL;
+  // [collective]: every rank has finished enqueueing before anyone frees memory
+  // or events a peer's pending work may reference
+  if (c->comm) c->comm->barrier();
   cudaDeviceSynchronize();
+  if (c->comm) c->comm->barrier();
   delete c->comm;
   for (void* p : c->allocs) cudaFree(p);
   for (auto& S : c->slots) {
