@@ -368,14 +368,18 @@ __device__ __forceinline__ float cluster_sum(float v, float* slot, float* red) {
     *slot = s;
   }
   asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-  float tot = 0.f;
+  // all LN_FUSE_CLUSTER remote slots requested back to back, then summed in rank order
+  float x[LN_FUSE_CLUSTER];
+#pragma unroll
   for (int r = 0; r < LN_FUSE_CLUSTER; ++r) {
     uint32_t remote;
+    // volatile: stays after the cluster barrier; no use until all are issued
     asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(smem_u32(slot)), "r"(r));
-    float x;
-    asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(x) : "r"(remote) : "memory");
-    tot += x;
+    asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(x[r]) : "r"(remote));
   }
+  float tot = 0.f;
+#pragma unroll
+  for (int r = 0; r < LN_FUSE_CLUSTER; ++r) tot += x[r];
   return tot;
 }
 
@@ -393,7 +397,19 @@ __global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const Gem
   const int tiles = p.n_tiles * p.m_tiles;
   const int64_t zstride = (int64_t)tiles * (BM * p.bn);
   const int mt = m / p.bn, col = m % p.bn;
-  float r[LNF_MAXC];
+  float r[LNF_MAXC], xv[LNF_MAXC], bv[LNF_MAXC], gv[LNF_MAXC], bev[LNF_MAXC];
+#pragma unroll
+  for (int i = 0; i < LNF_MAXC; ++i) {   // operands first: their loads overlap the partial sums
+    const int c = threadIdx.x + i * LNF_THREADS;
+    xv[i] = bv[i] = gv[i] = bev[i] = 0.f;
+    if (c < cw) {
+      const int n = n_begin + c;
+      xv[i] = __bfloat162float(q.x[(int64_t)m * p.N + n]);
+      if (q.add_bias) bv[i] = __bfloat162float(q.add_bias[n]);
+      gv[i] = __bfloat162float(q.g[n]);
+      bev[i] = __bfloat162float(q.b[n]);
+    }
+  }
   float s = 0.f;
 #pragma unroll
   for (int i = 0; i < LNF_MAXC; ++i) {
@@ -404,8 +420,8 @@ __global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const Gem
       const float* src = p.ws + (int64_t)((n / BM) * p.m_tiles + mt) * (BM * p.bn) + (int64_t)col * BM + (n % BM);
       const float acc = sum_partials(src, zstride, p.splits);
       const float part = __bfloat162float(__float2bfloat16_rn(acc));
-      float v = __bfloat162float(q.x[(int64_t)m * p.N + n]) + part;
-      if (q.add_bias) v += __bfloat162float(q.add_bias[n]);
+      float v = xv[i] + part;
+      if (q.add_bias) v += bv[i];
       v = __bfloat162float(__float2bfloat16_rn(v));   // residual stream is bf16
       r[i] = v;
       s += v;
@@ -424,8 +440,7 @@ __global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const Gem
     if (c < cw) {
       const int n = n_begin + c;
       q.x_out[(int64_t)m * p.N + n] = __float2bfloat16_rn(r[i]);
-      q.y[(int64_t)m * p.N + n] =
-          __float2bfloat16_rn((r[i] - mean) * rstd * __bfloat162float(q.g[n]) + __bfloat162float(q.b[n]));
+      q.y[(int64_t)m * p.N + n] = __float2bfloat16_rn((r[i] - mean) * rstd * gv[i] + bev[i]);
     }
   }
   // keep this CTA's shared slots alive until every CTA of the cluster has read them
