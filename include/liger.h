@@ -54,6 +54,9 @@ extern "C" {
 
 #define LIGER_MODE_SERIAL 0      /* Intra-Op baseline: compute then all-reduce, in order */
 #define LIGER_MODE_INTERLEAVED 1 /* Liger: Algorithm 1 + hybrid sync               */
+#define LIGER_MODE_PIPELINE 2    /* Inter-Op baseline: rank r holds an equal stage of unsharded
+                                    layers, activations / tokens travel by send/recv;
+                                    generated tokens are reported by the last stage */
 
 /* ------------------------------------------------------------------ config */
 typedef struct {

@@ -45,6 +45,8 @@ NcclApi& nccl() {
     LIGER_SYM(CommInitRank, "ncclCommInitRank");
     LIGER_SYM(AllReduce, "ncclAllReduce");
     LIGER_SYM(AllGather, "ncclAllGather");
+    LIGER_SYM(Send, "ncclSend");
+    LIGER_SYM(Recv, "ncclRecv");
     LIGER_SYM(GroupStart, "ncclGroupStart");
     LIGER_SYM(GroupEnd, "ncclGroupEnd");
     LIGER_SYM(CommDestroy, "ncclCommDestroy");
@@ -88,6 +90,24 @@ struct NcclComm : Comm {
     }
     return 0;
   }
+  int send(const void* buf, size_t bytes, int peer, cudaStream_t st) override {
+    if (!nccl().Send) return LIGER_ENCCL;
+    ncclResult_t r = nccl().Send(buf, bytes, ncclUint8, peer, comm, st);
+    if (r != ncclSuccess) {
+      err = std::string("ncclSend: ") + nccl().GetErrorString(r);
+      return LIGER_ENCCL;
+    }
+    return 0;
+  }
+  int recv(void* buf, size_t bytes, int peer, cudaStream_t st) override {
+    if (!nccl().Recv) return LIGER_ENCCL;
+    ncclResult_t r = nccl().Recv(buf, bytes, ncclUint8, peer, comm, st);
+    if (r != ncclSuccess) {
+      err = std::string("ncclRecv: ") + nccl().GetErrorString(r);
+      return LIGER_ENCCL;
+    }
+    return 0;
+  }
   int check_async() override {
     if (!nccl().CommGetAsyncError) return 0;
     ncclResult_t a = ncclSuccess;
@@ -101,6 +121,50 @@ struct NcclComm : Comm {
 };
 
 // ------------------------------------------------------------------ loopback (ranks = threads, one GPU)
+// Point-to-point mailbox of one directed pair (src -> dst): a ring of device
+// slots.  send copies into slot k % NSLOT and records a per-slot event; recv
+// waits for it and copies out, recording a per-slot "consumed" event that the
+// sender waits on before reusing the slot.  The host only blocks when a sender
+// is NSLOT messages ahead of its receiver's host (no cyclic wait: the
+// receiver of a full ring is never waiting for that sender).
+constexpr int P2P_SLOTS = 4;
+struct P2PBox {
+  std::mutex mu;
+  std::condition_variable cv;
+  uint64_t sent = 0, recvd = 0;              // messages enqueued by the two hosts
+  void* slot[P2P_SLOTS] = {};
+  size_t cap[P2P_SLOTS] = {};
+  size_t len[P2P_SLOTS] = {};
+  cudaEvent_t full[P2P_SLOTS] = {}, empty[P2P_SLOTS] = {};
+  bool empty_recorded[P2P_SLOTS] = {};
+};
+struct P2PTable {
+  std::mutex mu;
+  std::map<std::pair<int, int>, P2PBox*> boxes;
+  P2PBox* get(int s, int d) {
+    std::lock_guard<std::mutex> l(mu);
+    P2PBox*& b = boxes[{s, d}];
+    if (!b) {
+      b = new P2PBox();
+      for (int i = 0; i < P2P_SLOTS; ++i) {
+        cudaEventCreateWithFlags(&b->full[i], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&b->empty[i], cudaEventDisableTiming);
+      }
+    }
+    return b;
+  }
+  ~P2PTable() {
+    for (auto& kv : boxes) {
+      for (int i = 0; i < P2P_SLOTS; ++i) {
+        if (kv.second->slot[i]) cudaFree(kv.second->slot[i]);
+        cudaEventDestroy(kv.second->full[i]);
+        cudaEventDestroy(kv.second->empty[i]);
+      }
+      delete kv.second;
+    }
+  }
+};
+
 struct LoopGroup {
   int world;
   std::mutex mu;
@@ -113,6 +177,7 @@ struct LoopGroup {
   std::vector<const void*> a[2], b[2];
   std::vector<cudaEvent_t> ev[2];
   int members = 0;
+  P2PTable p2p;
 };
 
 static std::mutex g_groups_mu;
@@ -243,6 +308,44 @@ struct LoopbackComm : Comm {
     cudaEventRecord(ev_done, st);
     rendezvous(nullptr, nullptr, ev_done, &xs, &ys, &es);
     wait_all(es, st);
+    return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  }
+  int send(const void* buf, size_t bytes, int peer, cudaStream_t st) override {
+    P2PBox* b = g->p2p.get(rank, peer);
+    std::unique_lock<std::mutex> l(b->mu);
+    b->cv.wait(l, [&] { return b->sent - b->recvd < (uint64_t)P2P_SLOTS; });   // ring has room (host)
+    const int k = (int)(b->sent % P2P_SLOTS);
+    if (b->cap[k] < bytes) {
+      if (b->slot[k]) {
+        cudaEventSynchronize(b->empty[k]);
+        cudaFree(b->slot[k]);
+      }
+      if (cudaMalloc(&b->slot[k], bytes) != cudaSuccess) return LIGER_ENOMEM;
+      b->cap[k] = bytes;
+    }
+    if (b->empty_recorded[k]) cudaStreamWaitEvent(st, b->empty[k], 0);   // receiver done with the slot
+    cudaMemcpyAsync(b->slot[k], buf, bytes, cudaMemcpyDeviceToDevice, st);
+    cudaEventRecord(b->full[k], st);
+    b->len[k] = bytes;
+    ++b->sent;
+    b->cv.notify_all();
+    return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  }
+  int recv(void* buf, size_t bytes, int peer, cudaStream_t st) override {
+    P2PBox* b = g->p2p.get(peer, rank);
+    std::unique_lock<std::mutex> l(b->mu);
+    b->cv.wait(l, [&] { return b->sent > b->recvd; });   // the matching send was enqueued (host)
+    const int k = (int)(b->recvd % P2P_SLOTS);
+    if (b->len[k] != bytes) {
+      err = "loopback recv: size mismatch";
+      return LIGER_EINVAL;
+    }
+    cudaStreamWaitEvent(st, b->full[k], 0);
+    cudaMemcpyAsync(buf, b->slot[k], bytes, cudaMemcpyDeviceToDevice, st);
+    cudaEventRecord(b->empty[k], st);
+    b->empty_recorded[k] = true;
+    ++b->recvd;
+    b->cv.notify_all();
     return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
   }
   int check_async() override { return 0; }

@@ -16,6 +16,8 @@ struct NcclApi {
   ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
                             cudaStream_t) = nullptr;
   ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
   ncclResult_t (*GroupStart)() = nullptr;
   ncclResult_t (*GroupEnd)() = nullptr;
   ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
@@ -35,6 +37,9 @@ struct Comm {
   // two all-gathers issued as one group: recv[q * n + i] = send_q[i]
   virtual int allgather2(const void* s0, void* r0, size_t n0, CommDType d0, const void* s1, void* r1, size_t n1,
                          CommDType d1, cudaStream_t st) = 0;
+  // point-to-point (inter-operator pipeline baseline): `bytes` from this rank to `peer`
+  virtual int send(const void* buf, size_t bytes, int peer, cudaStream_t st) = 0;
+  virtual int recv(void* buf, size_t bytes, int peer, cudaStream_t st) = 0;
   virtual int check_async() = 0;
   // host-side barrier of the group (loopback: every rank's thread has arrived)
   virtual void barrier() {}

@@ -54,10 +54,13 @@ constexpr uint64_t GID_ETOK = 0xFFFF00, GID_EPOS = 0xFFFF01, GID_LNFG = 0xFFFF02
 
 // ------------------------------------------------------------------ ops of one pass
 enum Op { OP_EMBED, OP_LN1, OP_QKV, OP_ATTN, OP_OUT, OP_AR1, OP_LN2, OP_FC1, OP_FC2, OP_AR2, OP_HEAD, OP_TOKG,
-          OP_PICK, OP_COUNT };
-const char* kOpName[OP_COUNT] = {"embed", "ln1", "qkv", "attn", "out", "ar1", "ln2", "fc1", "fc2", "ar2",
-                                 "head",  "tokg", "pick"};
-inline bool op_is_comm(int op) { return op == OP_AR1 || op == OP_AR2 || op == OP_TOKG; }
+          OP_PICK, OP_RECV_X, OP_SEND_X, OP_RECV_TOK, OP_SEND_TOK, OP_COUNT };
+const char* kOpName[OP_COUNT] = {"embed", "ln1",  "qkv",    "attn",   "out",      "ar1",     "ln2", "fc1", "fc2",
+                                 "ar2",   "head", "tokg",   "pick",   "recv_x",   "send_x",  "recv_tok", "send_tok"};
+inline bool op_is_comm(int op) {
+  return op == OP_AR1 || op == OP_AR2 || op == OP_TOKG || op == OP_RECV_X || op == OP_SEND_X || op == OP_RECV_TOK ||
+         op == OP_SEND_TOK;
+}
 inline bool op_is_gemm(int op) { return op == OP_QKV || op == OP_OUT || op == OP_FC1 || op == OP_FC2; }
 inline bool op_is_ar(int op) { return op == OP_AR1 || op == OP_AR2; }
 
@@ -73,6 +76,8 @@ struct LayerW {
   void *w_qkv, *b_qkv, *w_o, *b_o, *w_1, *b_1, *w_2, *b_2, *g1, *be1, *g2, *be2;
 };
 
+struct Batch;
+
 // Per in-flight batch slot device buffers.
 struct Slot {
   void *x, *y, *qkv, *attn, *part, *hbuf, *yhead;
@@ -84,7 +89,7 @@ struct Slot {
   int32_t* h_prompt;       // pinned
   int32_t* h_tok_out;      // pinned
   cudaEvent_t free_ev;     // completes when the last batch using the slot finished
-  bool busy = false;
+  Batch* owner = nullptr;  // batch currently (or last) assigned to the slot
 };
 
 struct DurTable {
@@ -128,6 +133,10 @@ struct Batch {
 
 struct liger_ctx {
   int world = 1, rank = 0;
+  int tp = 1, tp_rank = 0;   // tensor-parallel degree / index (1 / 0 in pipeline mode)
+  bool pipe = false;         // inter-operator pipeline baseline
+  int l0 = 0, l1 = 0;        // this rank's layers [l0, l1) (all of them in TP modes)
+  int64_t admitted = 0;      // batches admitted so far (round-robin slot assignment)
   liger_cfg cfg;
   int h, a, d, f, V, hl, al, fl, Vl, L, F;
   double cf;
@@ -141,7 +150,6 @@ struct liger_ctx {
   void* kv = nullptr;
   int n_pages = 0, max_pages = 0;
   size_t kv_layer_elems = 0;
-  std::vector<int> free_pages;
   std::vector<Slot> slots;
   std::vector<PassOp> pass_ops;
   // scheduler state
@@ -213,8 +221,8 @@ cudaEvent_t pool_event(liger_ctx* c) {
 // ------------------------------------------------------------------ geometry helpers
 int op_units(liger_ctx* c, int op) {
   // decomposition exists to fill a communication window; at t = 1 there is none
-  if (c->F <= 1 || c->world == 1) return 1;
-  if (op_is_gemm(op) || (op_is_ar(op) && c->world > 1)) return c->F;
+  if (c->F <= 1 || c->tp == 1) return 1;
+  if (op_is_gemm(op) || (op_is_ar(op) && c->tp > 1)) return c->F;
   return 1;
 }
 
@@ -251,8 +259,8 @@ int batch_M(const Batch* bt, int pass) { return pass == 0 ? bt->b * bt->s : bt->
 // fused into that GEMM's split-K fixup?  (t = 1 only: at t > 1 the all-reduce
 // sits between them.  The last layer's FC2 feeds the LM head's own LN.)
 bool ln_fused(liger_ctx* c, const Batch* bt, int pass, int gemm_op, int layer) {
-  if (c->world != 1 || c->no_ln_fuse) return false;
-  if (gemm_op == OP_FC2 && layer == c->L - 1) return false;
+  if (c->tp != 1 || c->no_ln_fuse) return false;
+  if (gemm_op == OP_FC2 && layer == c->l1 - 1) return false;   // next LN is on another stage / the LM head
   return gemm_can_fuse_ln(batch_M(bt, pass), c->h, gemm_K(c, gemm_op));
 }
 
@@ -267,7 +275,7 @@ double model_dur(liger_ctx* c, int op, int M, int k, int ctx_len, int s_len) {
   }
   if (op_is_ar(op)) {
     const double bytes = (double)M * c->h * 2 * frac;
-    return 8e-6 + bytes * 2 * (c->world - 1) / c->world / 600e9;
+    return 8e-6 + bytes * 2 * (c->tp - 1) / c->tp / 600e9;
   }
   switch (op) {
     case OP_EMBED:
@@ -370,13 +378,13 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_LN1: {
-      if (li > 0 && ln_fused(c, bt, pass, OP_FC2, li - 1)) break;   // done in FC2's fixup
+      if (li > c->l0 && ln_fused(c, bt, pass, OP_FC2, li - 1)) break;   // done in FC2's fixup
       timed_begin(c, st, &ta);
-      if (li == 0)
+      if (li == c->l0)   // first layer of the model / of this pipeline stage: x is complete
         rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
       else
         rc = add_layernorm_launch(S.x, S.part, c->layers[li - 1].b_2, S.x, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
-      timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * (li == 0 ? 2 : 4), 0);
+      timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * (li == c->l0 ? 2 : 4), 0);
       c->st.gpu_launches++;
       break;
     }
@@ -430,7 +438,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_ATTN: {
-      void* pool = (char*)c->kv + (size_t)li * c->kv_layer_elems * 2;
+      void* pool = (char*)c->kv + (size_t)(li - c->l0) * c->kv_layer_elems * 2;
       timed_begin(c, st, &ta);
       if (pass == 0) {
         rc = attn_prefill_launch(S.qkv, S.attn, pool, S.page_table, c->max_pages, bt->b, bt->s, c->al, c->d, st);
@@ -469,7 +477,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       if (rc) break;
       GemmArgs g{};
       g.x = S.yhead; g.ldx = h;
-      g.w = (char*)c->e_tok + (size_t)c->rank * c->Vl * h * 2; g.ldw = h;
+      g.w = (char*)c->e_tok + (size_t)c->tp_rank * c->Vl * h * 2; g.ldw = h;
       g.out = S.logits; g.ldo = c->Vl; g.out_f32 = 1;
       g.M = b; g.N = c->Vl; g.K = h; g.n0 = 0; g.n1 = c->Vl; g.scale = 1.0f;
       g.workspace = S.gemm_ws; g.ws_bytes = S.gemm_ws_bytes;
@@ -478,11 +486,11 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       timed_end(c, st, ta, LIGER_KT_LMHEAD, ((double)c->Vl * h + (double)b * h) * 2 + (double)b * c->Vl * 4,
                 2.0 * b * c->Vl * h);
       if (rc) break;
-      rc = argmax_launch(S.logits, c->Vl, b, c->Vl, c->rank * c->Vl, S.vals_all + (size_t)c->rank * b,
-                         S.idx_all + (size_t)c->rank * b, st);
+      rc = argmax_launch(S.logits, c->Vl, b, c->Vl, c->tp_rank * c->Vl, S.vals_all + (size_t)c->tp_rank * b,
+                         S.idx_all + (size_t)c->tp_rank * b, st);
       if (rc) break;
       c->st.gpu_launches += 3;
-      if (c->world == 1) {
+      if (c->tp == 1) {
         rc = argmax_pick_launch(S.vals_all, S.idx_all, 1, b, S.cur_tok, S.tok_out, bt->n_new, pass, st);
         c->st.gpu_launches++;
       }
@@ -498,8 +506,38 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_PICK: {
-      rc = argmax_pick_launch(S.vals_all, S.idx_all, c->world, bt->b, S.cur_tok, S.tok_out, bt->n_new, pass, st);
+      rc = argmax_pick_launch(S.vals_all, S.idx_all, c->tp, bt->b, S.cur_tok, S.tok_out, bt->n_new, pass, st);
       c->st.gpu_launches++;
+      break;
+    }
+    // ---- inter-operator pipeline baseline: stage-to-stage activations and the token
+    case OP_RECV_X: {
+      if (c->comm->recv(S.x, (size_t)M * h * 2, c->rank - 1, st)) return fail(c, LIGER_ENCCL, c->comm->err);
+      c->st.comm_kernels++;
+      break;
+    }
+    case OP_SEND_X: {
+      // complete the residual stream of the stage's last layer (x += FC2 + b_2), then send it on
+      rc = add_layernorm_launch(S.x, S.part, c->layers[c->l1 - 1].b_2, S.x, S.y, c->lnf_g, c->lnf_b, M, h, 1, 0,
+                                eps, st);
+      if (rc) break;
+      c->st.gpu_launches++;
+      if (c->comm->send(S.x, (size_t)M * h * 2, c->rank + 1, st)) return fail(c, LIGER_ENCCL, c->comm->err);
+      c->st.comm_kernels++;
+      break;
+    }
+    case OP_RECV_TOK: {   // stage 0, pass > 0: the token of the previous pass from the last stage
+      if (pass == 0) break;
+      if (c->comm->recv(S.cur_tok, (size_t)bt->b * 4, c->world - 1, st)) return fail(c, LIGER_ENCCL, c->comm->err);
+      c->st.comm_kernels++;
+      rc = argmax_pick_launch(S.vals_all, S.cur_tok, 1, bt->b, S.cur_tok, S.tok_out, bt->n_new, pass - 1, st);
+      c->st.gpu_launches++;
+      break;
+    }
+    case OP_SEND_TOK: {   // last stage: the new token back to stage 0 (not after the final pass)
+      if (pass == bt->n_new - 1) break;
+      if (c->comm->send(S.cur_tok, (size_t)bt->b * 4, 0, st)) return fail(c, LIGER_ENCCL, c->comm->err);
+      c->st.comm_kernels++;
       break;
     }
   }
@@ -547,26 +585,25 @@ struct BatchCursor : Cursor {
 };
 
 // ------------------------------------------------------------------ admission / completion
-int admit(liger_ctx* c, Batch* bt) {
-  int slot = -1;
-  for (size_t i = 0; i < c->slots.size(); ++i)
-    if (!c->slots[i].busy) {
-      slot = (int)i;
-      break;
-    }
-  if (slot < 0) return 1;   // no free slot yet
-  const int ppseq = (bt->s + bt->n_new + LIGER_KV_BLOCK - 1) / LIGER_KV_BLOCK;
-  if ((int)c->free_pages.size() < ppseq * bt->b) return 1;
+void reap(liger_ctx* c);
+
+// Admission is a pure function of the submit order (round-robin slots with a
+// fixed page range each), so every rank admits the same batch at the same
+// liger_step and all ranks issue identical plans / collectives.  Reusing a
+// slot waits (host) for its previous occupant, whose kernels are all enqueued.
+void admit(liger_ctx* c, Batch* bt) {
+  const int slot = (int)(c->admitted++ % (int64_t)c->slots.size());
   Slot& S = c->slots[slot];
-  S.busy = true;
+  if (S.owner && !S.owner->finished) {
+    cudaEventSynchronize(S.owner->final_ev);
+    reap(c);
+  }
+  S.owner = bt;
   bt->slot = slot;
+  const int ppseq = (bt->s + bt->n_new + LIGER_KV_BLOCK - 1) / LIGER_KV_BLOCK;
+  const int base = slot * c->cfg.max_batch * c->max_pages;
   for (int i = 0; i < bt->b; ++i)
-    for (int p = 0; p < ppseq; ++p) {
-      const int pg = c->free_pages.back();
-      c->free_pages.pop_back();
-      bt->pages.push_back(pg);
-      S.h_page_table[i * c->max_pages + p] = pg;
-    }
+    for (int p = 0; p < ppseq; ++p) S.h_page_table[i * c->max_pages + p] = base + i * c->max_pages + p;
   // inputs for the first kernels: wait until the previous user of the slot is done
   cudaStreamWaitEvent(c->s_comp, S.free_ev, 0);
   cudaMemcpyAsync(S.page_table, S.h_page_table, sizeof(int32_t) * bt->b * c->max_pages, cudaMemcpyHostToDevice,
@@ -579,7 +616,6 @@ int admit(liger_ctx* c, Batch* bt) {
   bt->last_ev = pool_event(c);
   cudaEventRecord(bt->last_ev, c->s_comp);
   bt->has_last_ev = true;
-  return 0;
 }
 
 void CUDART_CB host_finish(void* p) {
@@ -608,9 +644,6 @@ void reap(liger_ctx* c) {
       bt->tokens.assign(S.h_tok_out, S.h_tok_out + bt->b * bt->n_new);
       bt->results_copied = true;
     }
-    for (int pg : bt->pages) c->free_pages.push_back(pg);
-    bt->pages.clear();
-    S.busy = false;
     if (bt->finish_s.load() == 0) bt->finish_s.store(now_s());
   }
 }
@@ -625,10 +658,7 @@ void update_list(liger_ctx* c) {
   reap(c);
   while ((int)c->processing.size() < cap && !c->waiting.empty()) {
     Batch* bt = c->waiting.front().get();
-    if (admit(c, bt)) {
-      reap(c);
-      if (admit(c, bt)) break;
-    }
+    admit(c, bt);
     c->processing.push_back(bt);
     c->all_batches[bt->id] = std::move(c->waiting.front());
     c->waiting.pop_front();
@@ -693,16 +723,30 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   c->rank = rank;
   c->cfg = *cfg;
   c->h = cfg->hidden; c->a = cfg->n_heads; c->f = cfg->ffn; c->V = cfg->vocab; c->L = cfg->n_layers;
-  if (c->a <= 0 || c->h % c->a || c->a % world || c->f % world || c->V % world || c->h % 64)
+  c->pipe = cfg->mode == LIGER_MODE_PIPELINE;
+  c->tp = c->pipe ? 1 : world;
+  c->tp_rank = c->pipe ? 0 : rank;
+  const int tp = c->tp;
+  if (c->a <= 0 || c->h % c->a || c->a % tp || c->f % tp || c->V % tp || c->h % 64)
     return fail(nullptr, LIGER_EINVAL, "liger_init: shapes not divisible by the TP degree");
+  if (c->pipe && c->L < world) return fail(nullptr, LIGER_EINVAL, "liger_init: fewer layers than pipeline stages");
   c->d = c->h / c->a;
   if (c->d != 64 && c->d != 128) return fail(nullptr, LIGER_EINVAL, "liger_init: head_dim must be 64 or 128");
-  c->hl = c->h / world; c->al = c->a / world; c->fl = c->f / world; c->Vl = c->V / world;
+  c->hl = c->h / tp; c->al = c->a / tp; c->fl = c->f / tp; c->Vl = c->V / tp;
+  // layers of this rank: all (TP) or an equal pipeline stage, the first L % world stages one more (AMB-29)
+  if (c->pipe) {
+    const int base = c->L / world, extra = c->L % world;
+    c->l0 = rank * base + std::min(rank, extra);
+    c->l1 = c->l0 + base + (rank < extra ? 1 : 0);
+  } else {
+    c->l0 = 0;
+    c->l1 = c->L;
+  }
   c->F = std::max(1, cfg->decomp_factor);
   c->cf = cfg->contention_factor > 0 ? cfg->contention_factor : 1.0;
   c->no_ln_fuse = getenv("LIGER_NO_LN_FUSE") != nullptr;
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
-  c->ar_atomic_chunks = env ? atoi(env) != 0 : (world > 2);
+  c->ar_atomic_chunks = env ? atoi(env) != 0 : (tp > 2);
   if (world > 1) {
     if (!nccl_uid) return fail(nullptr, LIGER_EINVAL, "liger_init: nccl_uid required for world > 1");
     std::string err;
@@ -719,7 +763,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   // weights (this rank's shards, K-major [N_local, K])
   c->layers.resize(c->L);
   const size_t h = c->h;
-  for (int l = 0; l < c->L; ++l) {
+  for (int l = c->l0; l < c->l1; ++l) {
     LayerW& W = c->layers[l];
     W.w_qkv = dalloc(c, (size_t)pad128(3 * c->hl) * h * 2);
     W.b_qkv = dalloc(c, 3 * c->hl * 2);
@@ -746,9 +790,8 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   c->max_pages = (Smax + cfg->max_new + LIGER_KV_BLOCK - 1) / LIGER_KV_BLOCK;
   c->n_pages = nslots * B * c->max_pages;
   c->kv_layer_elems = (size_t)c->n_pages * 2 * c->al * LIGER_KV_BLOCK * c->d;
-  c->kv = dalloc(c, c->kv_layer_elems * 2 * c->L);
+  c->kv = dalloc(c, c->kv_layer_elems * 2 * (c->l1 - c->l0));
   if (!c->kv) return fail(nullptr, LIGER_ENOMEM, "liger_init: KV pool");
-  for (int p = c->n_pages - 1; p >= 0; --p) c->free_pages.push_back(p);
   // split-K workspace: the maximum over every token count a pass can have
   size_t ws = 0;
   for (int M = 1; M <= Mmax; ++M) {
@@ -768,8 +811,8 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     S.hbuf = dalloc(c, (size_t)Mmax * c->fl * 2);
     S.yhead = dalloc(c, (size_t)B * h * 2);
     S.logits = (float*)dalloc(c, (size_t)B * c->Vl * 4);
-    S.vals_all = (float*)dalloc(c, (size_t)world * B * 4);
-    S.idx_all = (int32_t*)dalloc(c, (size_t)world * B * 4);
+    S.vals_all = (float*)dalloc(c, (size_t)tp * B * 4);
+    S.idx_all = (int32_t*)dalloc(c, (size_t)tp * B * 4);
     S.cur_tok = (int32_t*)dalloc(c, (size_t)B * 4);
     S.tok_out = (int32_t*)dalloc(c, (size_t)B * cfg->max_new * 4);
     S.prompt = (int32_t*)dalloc(c, (size_t)Mmax * 4);
@@ -788,23 +831,34 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     CK(cudaEventCreateWithFlags(&S.free_ev, cudaEventDisableTiming));
     CK(cudaEventRecord(S.free_ev, c->s_comp));
   }
-  // function assembly template of one pass (§3.2)
-  c->pass_ops.push_back({OP_EMBED, -1});
-  for (int l = 0; l < c->L; ++l) {
+  // function assembly template of one pass (§3.2) on this rank
+  const bool first = c->l0 == 0, last = c->l1 == c->L;
+  if (first) {
+    if (c->pipe && world > 1) c->pass_ops.push_back({OP_RECV_TOK, -1});
+    c->pass_ops.push_back({OP_EMBED, -1});
+  } else {
+    c->pass_ops.push_back({OP_RECV_X, -1});
+  }
+  for (int l = c->l0; l < c->l1; ++l) {
     c->pass_ops.push_back({OP_LN1, l});
     c->pass_ops.push_back({OP_QKV, l});
     c->pass_ops.push_back({OP_ATTN, l});
     c->pass_ops.push_back({OP_OUT, l});
-    if (world > 1) c->pass_ops.push_back({OP_AR1, l});
+    if (tp > 1) c->pass_ops.push_back({OP_AR1, l});
     c->pass_ops.push_back({OP_LN2, l});
     c->pass_ops.push_back({OP_FC1, l});
     c->pass_ops.push_back({OP_FC2, l});
-    if (world > 1) c->pass_ops.push_back({OP_AR2, l});
+    if (tp > 1) c->pass_ops.push_back({OP_AR2, l});
   }
-  c->pass_ops.push_back({OP_HEAD, -1});
-  if (world > 1) {
-    c->pass_ops.push_back({OP_TOKG, -1});
-    c->pass_ops.push_back({OP_PICK, -1});
+  if (!last) {
+    c->pass_ops.push_back({OP_SEND_X, -1});
+  } else {
+    c->pass_ops.push_back({OP_HEAD, -1});
+    if (tp > 1) {
+      c->pass_ops.push_back({OP_TOKG, -1});
+      c->pass_ops.push_back({OP_PICK, -1});
+    }
+    if (c->pipe && world > 1) c->pass_ops.push_back({OP_SEND_TOK, -1});
   }
   CK(cudaDeviceSynchronize());
   *out = cp.release();
@@ -813,7 +867,8 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
 
 int liger_load_layer(liger_ctx* c, int l, uint64_t seed) {
   if (!c || l < 0 || l >= c->L) return LIGER_EINVAL;
-  const int r = c->rank, t = c->world;
+  if (l < c->l0 || l >= c->l1) return LIGER_OK;   // another pipeline stage's layer
+  const int r = c->tp_rank, t = c->tp;
   const int64_t h = c->h, hl = c->hl, fl = c->fl, f = c->f;
   LayerW& W = c->layers[l];
   cudaStream_t st = c->s_comp;
@@ -904,7 +959,23 @@ int liger_step(liger_ctx* c) {
   }
   std::vector<Piece> pieces;
   int n = 0;
-  if (c->cfg.mode == LIGER_MODE_SERIAL) {
+  if (c->pipe) {
+    // Inter-operator pipeline: one pass of every in-flight batch, in arrival
+    // order, on one stream; stages are decoupled by the send/recv of activations
+    // and tokens, so consecutive batches occupy different stages concurrently.
+    for (Batch* bt : c->processing) {
+      if (bt->all_launched) continue;
+      BatchCursor cur(c, bt, &pieces);
+      const int pass = bt->pass;
+      while (!cur.empty() && bt->pass == pass) cur.take(cur.head_left());
+    }
+    std::vector<int> all(pieces.size());
+    for (size_t i = 0; i < pieces.size(); ++i) all[i] = (int)i;
+    CKR(launch_run(c, pieces, all, 0));
+    c->st.rounds++;
+    c->have_round = false;
+    n = (int)pieces.size();
+  } else if (c->cfg.mode == LIGER_MODE_SERIAL) {
     // Intra-Op baseline: the single batch's whole remaining list, in order,
     // on one stream (computation then all-reduce, serially).
     Batch* bt = c->processing[0];
@@ -1207,13 +1278,13 @@ int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
     }
     // memory-bound ops
     const double tln = time_it([&] {
-      add_layernorm_launch(S.x, S.part, c->layers[0].b_o, S.x, S.y, c->layers[0].g2, c->layers[0].be2, M, c->h, 1,
-                           0, c->cfg.ln_eps, st);
+      add_layernorm_launch(S.x, S.part, c->layers[c->l0].b_o, S.x, S.y, c->layers[c->l0].g2, c->layers[c->l0].be2, M,
+                           c->h, 1, 0, c->cfg.ln_eps, st);
     });
     liger_set_duration(c, OP_LN1, M, F, tln * 1e6);
     liger_set_duration(c, OP_LN2, M, F, tln * 1e6);
     liger_set_duration(c, OP_EMBED, M, F, tln * 1e6);
-    if (c->world > 1) {
+    if (c->tp > 1) {
       const size_t E = (size_t)M * c->h;
       for (int k = 1; k <= op_units(c, OP_AR1); ++k) {
         const int kk = op_units(c, OP_AR1) > 1 ? k : F;
@@ -1225,8 +1296,8 @@ int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
       }
     }
   }
-  // LM head at batch sizes
-  {
+  // LM head at batch sizes (last stage only)
+  if (c->l1 == c->L) {
     int pidx = 0;
     while (c->pass_ops[pidx].op != OP_HEAD) ++pidx;
     for (int bb : {1, c->cfg.max_batch}) {

@@ -122,3 +122,26 @@ def test_runtime_decomposition_bit_exact(E):
         for a, b in zip(tb, ti):
             assert np.array_equal(a, b)
     assert inter[0][1]["split_pieces"] > 0, inter[0][1]
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_pipeline_baseline_equals_single_gpu(E, world):
+    """Inter-operator pipeline baseline: `world` stages of unsharded layers,
+    activations and tokens passed stage to stage; several batches in flight.
+    The last stage's tokens are bit-identical to the single-GPU run (the same
+    unsharded kernels)."""
+    from liger_inputs.configs import ModelConfig
+    cfg = ModelConfig("tiny6", 6, 256, 4, 1024, 512, 64, "gelu_tanh")
+    trace = make_trace(4, float("inf"), seed=13, batch_sizes=(1, 2), prompt_range=(8, 30), n_decode=5,
+                       vocab=cfg.vocab)
+    eng = E(cfg, mode="serial", max_batch=2, max_seq=32, max_new=8, seed=5)
+    ids = [eng.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], 0.0) for t in trace]
+    eng.drain()
+    ref = [eng.poll(i, want_tokens=True)[1] for i in ids]
+    eng.close()
+    pipe = serve_tp(E, cfg, world, trace, mode="pipeline", max_batch=2, max_seq=32, max_new=8, max_inflight=world,
+                    seed=5)
+    toks, st = pipe[world - 1]
+    for a, b in zip(ref, toks):
+        assert np.array_equal(a, b)
+    assert st["comm_kernels"] > 0
