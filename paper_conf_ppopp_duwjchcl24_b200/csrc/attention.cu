@@ -337,7 +337,9 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
     fence_barrier_init();
   }
   __syncthreads();
-  pdl_enter();
+  // The cached positions (< pos) were written by earlier passes, and the page
+  // table at admission: staging them does not depend on the preceding kernel
+  // (QKV), so it is issued before griddepcontrol.wait.
   if (warp == 0) {   // lane g stages page g (page ids loaded in parallel, not a serial chain)
     if (lane == 0) mbar_arrive_expect_tx(&bar, (uint32_t)npg * 2 * KVB * D * 2);
     __syncwarp();
@@ -347,6 +349,7 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
       bulk_load(sV + lane * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &bar);
     }
   }
+  pdl_enter();   // q and the new token's k / v come from the QKV kernel
   float qf[8];
   {
     uint4 qv = *reinterpret_cast<const uint4*>(qp + (lane % LPT) * 8);

@@ -145,10 +145,12 @@ LIGER_DEV void grid_dependency_wait() { asm volatile("griddepcontrol.wait;" ::: 
 // Allow the next PDL kernel in the stream to be scheduled (its CTAs wait in
 // grid_dependency_wait until this grid has completed).
 LIGER_DEV void grid_dependency_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
-// Both, for kernels whose whole body depends on upstream data.
+// For kernels whose whole body depends on upstream data.  The trigger comes
+// AFTER the wait: the next kernel's pre-wait code (weight / KV-cache prefetch)
+// then overlaps only this kernel, never an older one still running.
 LIGER_DEV void pdl_enter() {
-  grid_dependency_trigger();
   grid_dependency_wait();
+  grid_dependency_trigger();
 }
 
 LIGER_DEV float bf16_bits_to_f32(uint16_t b) { return __uint_as_float(((uint32_t)b) << 16); }

@@ -141,7 +141,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     fence_barrier_init();
   }
   if (warp == 0 && lane == 0) {
-    grid_dependency_trigger();
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
   }
@@ -174,6 +173,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         pre = it;
       }
       grid_dependency_wait();
+      grid_dependency_trigger();   // after the wait: dependents overlap only this kernel
       int it = 0;
       for (int u = blockIdx.x; u < p.units; u += G) {
         const Unit w = unit_of(p, u);
@@ -294,8 +294,7 @@ __device__ __forceinline__ float sum_partials(const float* src, int64_t zstride,
 // same bits whatever slice or CTA produced each chunk).  One thread per (m, 4 rows n),
 // reading the column-major per-tile partials coalesced.
 __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) {
-  grid_dependency_trigger();
-  grid_dependency_wait();
+  pdl_enter();
   const int tiles = p.n_tiles * p.m_tiles;
   const int64_t zstride = (int64_t)tiles * (BM * p.bn);
   const int slice_w = p.n1 - p.n0;
@@ -388,8 +387,7 @@ constexpr int LNF_THREADS = 256, LNF_MAXC = 8;
 __global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const GemmParams p, const LnFuseParams q) {
   __shared__ float red[LNF_THREADS / 32];
   __shared__ float slot[2];
-  grid_dependency_trigger();
-  grid_dependency_wait();
+  pdl_enter();
   const int m = blockIdx.y;
   const int rank = blockIdx.x;   // == %cluster_ctarank for cluster dims (LN_FUSE_CLUSTER, 1, 1)
   const int cw = p.N / LN_FUSE_CLUSTER;
