@@ -164,6 +164,7 @@ struct liger_ctx {
   DurTable dur;
   double attn_scale[2] = {1.0, 1.0};   // calibration of the attention duration model (prefill, decode)
   bool no_ln_fuse = false;             // LIGER_NO_LN_FUSE=1 disables the fused fixup + LN
+  uint32_t dbg_skip = 0;               // LIGER_DBG_SKIP=op,op,...: timing experiments only (wrong results)
   bool ar_atomic_chunks = false;
   // stats / timing
   liger_stats_t st{};
@@ -369,6 +370,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
   const LayerW* W = li >= 0 ? &c->layers[li] : nullptr;
   int rc = 0;
   cudaEvent_t ta = nullptr;
+  if (c->dbg_skip & (1u << po.op)) return 0;
   switch (po.op) {
     case OP_EMBED: {
       const int32_t* ids = pass == 0 ? (bt->dev_tokens ? bt->dev_tokens : S.prompt) : S.cur_tok;
@@ -745,6 +747,11 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   c->F = std::max(1, cfg->decomp_factor);
   c->cf = cfg->contention_factor > 0 ? cfg->contention_factor : 1.0;
   c->no_ln_fuse = getenv("LIGER_NO_LN_FUSE") != nullptr;
+  if (const char* sk = getenv("LIGER_DBG_SKIP")) {
+    std::string all = std::string(",") + sk + ",";
+    for (int o = 0; o < OP_COUNT; ++o)
+      if (all.find(std::string(",") + kOpName[o] + ",") != std::string::npos) c->dbg_skip |= 1u << o;
+  }
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (tp > 2);
   if (world > 1) {
