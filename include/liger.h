@@ -173,7 +173,8 @@ int liger_reset_stats(liger_ctx* ctx);
 #define LIGER_KT_ALLREDUCE 3
 #define LIGER_KT_GEMM_PREFILL 4  /* projection GEMMs with M > 64 tokens (tensor-bound) */
 #define LIGER_KT_LMHEAD 5
-#define LIGER_KT_CLASSES 6
+#define LIGER_KT_FIXUP 6         /* split-K fixup kernels (+ fused residual add + LN at t = 1) */
+#define LIGER_KT_CLASSES 7
 int liger_set_kernel_timing(liger_ctx* ctx, int on);
 int liger_kernel_timing(liger_ctx* ctx, int64_t* count, double* ms, double* bytes, double* flops);
 

@@ -328,7 +328,7 @@ double op_dur(liger_ctx* c, const Batch* bt, int pass, int op, int k) {
 // ------------------------------------------------------------------ timing instrumentation
 void timed_begin(liger_ctx* c, cudaStream_t s, cudaEvent_t* a) {
   if (!c->timing) return;
-  if (c->timing_next + 2 > c->timing_pool.size()) {
+  if (c->timing_next + 3 > c->timing_pool.size()) {
     for (int i = 0; i < 256; ++i) {
       cudaEvent_t e;
       cudaEventCreate(&e);
@@ -337,6 +337,11 @@ void timed_begin(liger_ctx* c, cudaStream_t s, cudaEvent_t* a) {
   }
   *a = c->timing_pool[c->timing_next++];
   cudaEventRecord(*a, s);
+}
+// a spare timing event (recorded by gemm_launch between the GEMM kernel and its fixup)
+cudaEvent_t timed_mid(liger_ctx* c) {
+  if (!c->timing) return nullptr;
+  return c->timing_pool[c->timing_next++];
 }
 void timed_end(liger_ctx* c, cudaStream_t s, cudaEvent_t a, int cls, double bytes, double flops) {
   if (!c->timing) return;
@@ -432,10 +437,22 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
         }
       }
       timed_begin(c, st, &ta);
+      cudaEvent_t tmid = timed_mid(c);
+      bool fix = false;
+      g.ev_mid = tmid;
+      g.had_fixup = &fix;
       rc = gemm_launch(g, st);
       const double n = g.n1 - g.n0;
-      timed_end(c, st, ta, M <= 64 ? LIGER_KT_GEMM_DECODE : LIGER_KT_GEMM_PREFILL,
-                (n * K + (double)M * K + (double)M * n) * 2, 2.0 * M * n * K);
+      if (c->timing) {
+        // GEMM kernel: algorithmic bytes / flops; fixup: fp32 partials read + output (and LN operands) written
+        c->timed.push_back({M <= 64 ? LIGER_KT_GEMM_DECODE : LIGER_KT_GEMM_PREFILL, ta, tmid,
+                            (n * K + (double)M * K + (double)M * n) * 2, 2.0 * M * n * K});
+        if (fix) {
+          const GemmPlan pl = gemm_plan(M, N, K);
+          timed_end(c, st, tmid, LIGER_KT_FIXUP,
+                    (double)pl.splits * M * n * 4 + (double)M * n * (g.ln_y ? 2 * 4 : 2), 0);
+        }
+      }
       c->st.gpu_launches++;
       break;
     }

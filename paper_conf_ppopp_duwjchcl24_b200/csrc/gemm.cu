@@ -634,6 +634,8 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.units = ntiles * pl.m_tiles * pl.splits;
   const int grid = p.units < num_sms() ? p.units : num_sms();
   int rc2 = launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
+  if (a.had_fixup) *a.had_fixup = p.splits > 1;
+  if (a.ev_mid) cudaEventRecord(a.ev_mid, stream);
   if (rc2 || p.splits == 1) return rc2 ? LIGER_ECUDA : 0;
   if (a.ln_y) {
     if (a.n0 != 0 || a.n1 != a.N || !gemm_can_fuse_ln(a.M, a.N, a.K) || !a.ln_x || !a.ln_xout || !a.ln_g || !a.ln_b)

@@ -41,6 +41,10 @@ struct GemmArgs {
   const void* ln_b = nullptr;
   void* ln_y = nullptr;
   float ln_eps = 1e-5f;
+  // optional: recorded on the stream between the GEMM kernel and its split-K fixup
+  // (per-kernel timing; breaks the PDL overlap of the two)
+  cudaEvent_t ev_mid = nullptr;
+  bool* had_fixup = nullptr;
 };
 
 GemmPlan gemm_plan(int M, int N, int K);

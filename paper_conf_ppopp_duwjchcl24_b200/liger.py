@@ -12,7 +12,7 @@ LIGER_OK, LIGER_PENDING, LIGER_IDLE = 0, 1, 2
 ACT = {"none": 0, "relu": 1, "gelu_tanh": 2}
 MODE = {"serial": 0, "interleaved": 1, "pipeline": 2}
 KV_BLOCK = 16
-KT_NAMES = ["gemm_decode", "attn", "ln", "allreduce", "gemm_prefill", "lm_head"]   # LIGER_KT_* order
+KT_NAMES = ["gemm_decode", "attn", "ln", "allreduce", "gemm_prefill", "lm_head", "splitk_fixup"]   # LIGER_KT_*
 OPS = ["embed", "ln1", "qkv", "attn", "out", "ar1", "ln2", "fc1", "fc2", "ar2", "head", "tokg", "pick",
        "recv_x", "send_x", "recv_tok", "send_tok"]
 
