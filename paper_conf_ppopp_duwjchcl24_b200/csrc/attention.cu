@@ -457,18 +457,27 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   }
   __syncthreads();
   if (!last) return;
-  float M = -INFINITY;
-  for (int s2 = 0; s2 < nsp; ++s2) M = fmaxf(M, __ldcg(&ws[(unit * nsp + s2) * (D + 2) + D]));
-  float L = 0.f;
-  for (int s2 = 0; s2 < nsp; ++s2) {
+  // merge in chunk order; every load issued in parallel (one per thread, then smem)
+  __shared__ float mw[64], lw[64];   // nsp <= 64 (ctx <= 2048 with 32-position chunks)
+  for (int s2 = tid; s2 < nsp; s2 += DC_THREADS) {
     const float* w2 = ws + (unit * nsp + s2) * (D + 2);
-    L += __ldcg(&w2[D + 1]) * __expf(__ldcg(&w2[D]) - M);
+    mw[s2] = __ldcg(&w2[D]);
+    lw[s2] = __ldcg(&w2[D + 1]);
   }
+  __syncthreads();
+  float M = -INFINITY;
+  for (int s2 = 0; s2 < nsp; ++s2) M = fmaxf(M, mw[s2]);
+  float L = 0.f;
+  for (int s2 = 0; s2 < nsp; ++s2) L += lw[s2] * __expf(mw[s2] - M);
   for (int e = tid; e < D; e += DC_THREADS) {
     float a = 0.f;
-    for (int s2 = 0; s2 < nsp; ++s2) {
-      const float* w2 = ws + (unit * nsp + s2) * (D + 2);
-      a += __ldcg(&w2[e]) * __expf(__ldcg(&w2[D]) - M);
+    for (int z0 = 0; z0 < nsp; z0 += 8) {
+      float v[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) v[i] = (z0 + i < nsp) ? __ldcg(&ws[(unit * nsp + z0 + i) * (D + 2) + e]) : 0.f;
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        if (z0 + i < nsp) a += v[i] * __expf(mw[z0 + i] - M);
     }
     o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / L);
   }
@@ -496,8 +505,9 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   const int ctx = pos + 1;
   // 32-position chunks when 64-position ones would leave SMs without ~6 resident CTAs
   const bool small = (size_t)b * heads * ((ctx + 63) / 64) < (size_t)148 * 6;
-  const int CH = small ? 32 : 64;
+  const int CH = (small && (ctx + 31) / 32 <= 64) ? 32 : 64;
   const int ns = (ctx + CH - 1) / CH;
+  if (ns > 64) return LIGER_EINVAL;   // context longer than 4096 positions
   if (ns > 1) {
     if (!workspace || ws_bytes < attn_decode_workspace_bytes(b, heads, d, ctx) ||
         (size_t)b * heads * 4 > ATTN_COUNTER_BYTES)
@@ -507,10 +517,10 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   float* ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
   int rc;
   if (d == 128)
-    rc = small ? launch_decode<128, 32>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream)
+    rc = CH == 32 ? launch_decode<128, 32>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream)
                : launch_decode<128, 64>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream);
   else if (d == 64)
-    rc = small ? launch_decode<64, 32>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream)
+    rc = CH == 32 ? launch_decode<64, 32>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream)
                : launch_decode<64, 64>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream);
   else
     return LIGER_EINVAL;
