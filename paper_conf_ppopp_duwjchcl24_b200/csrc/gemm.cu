@@ -382,7 +382,7 @@ __device__ __forceinline__ float cluster_sum(float v, float* slot, float* red) {
   return tot;
 }
 
-constexpr int LNF_THREADS = 256, LNF_MAXC = 8;
+constexpr int LNF_THREADS = 256, LNF_MAXC = 6;   // h / 8 <= 1536 columns per CTA
 
 __global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const GemmParams p, const LnFuseParams q) {
   __shared__ float red[LNF_THREADS / 32];
@@ -408,6 +408,29 @@ __global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const Gem
       bev[i] = __bfloat162float(q.b[n]);
     }
   }
+  // partial sums of all this thread's columns: 8 chunks x all columns per batch of loads
+  const float* srcs[LNF_MAXC];
+  float accs[LNF_MAXC];
+#pragma unroll
+  for (int i = 0; i < LNF_MAXC; ++i) {
+    const int n = n_begin + min(threadIdx.x + i * LNF_THREADS, cw - 1);
+    srcs[i] = p.ws + (int64_t)((n / BM) * p.m_tiles + mt) * (BM * p.bn) + (int64_t)col * BM + (n % BM);
+    accs[i] = 0.f;
+  }
+  const int nvalid = (cw - (int)threadIdx.x + LNF_THREADS - 1) / LNF_THREADS;   // columns of this thread
+  for (int z0 = 0; z0 < p.splits; z0 += 8) {
+    float v[LNF_MAXC][8];
+#pragma unroll
+    for (int i = 0; i < LNF_MAXC; ++i)
+#pragma unroll
+      for (int j = 0; j < 8; ++j)
+        v[i][j] = (i < nvalid && z0 + j < p.splits) ? __ldcg(srcs[i] + (z0 + j) * zstride) : 0.f;
+#pragma unroll
+    for (int i = 0; i < LNF_MAXC; ++i)
+#pragma unroll
+      for (int j = 0; j < 8; ++j)
+        if (z0 + j < p.splits) accs[i] = (z0 + j == 0) ? v[i][j] : accs[i] + v[i][j];   // chunk order
+  }
   float s = 0.f;
 #pragma unroll
   for (int i = 0; i < LNF_MAXC; ++i) {
@@ -415,8 +438,7 @@ __global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const Gem
     r[i] = 0.f;
     if (c < cw) {
       const int n = n_begin + c;
-      const float* src = p.ws + (int64_t)((n / BM) * p.m_tiles + mt) * (BM * p.bn) + (int64_t)col * BM + (n % BM);
-      const float acc = sum_partials(src, zstride, p.splits);
+      const float acc = accs[i];
       const float part = __bfloat162float(__float2bfloat16_rn(acc));
       float v = xv[i] + part;
       if (q.add_bias) v += bv[i];
