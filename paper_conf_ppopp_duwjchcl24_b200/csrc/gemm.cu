@@ -307,9 +307,9 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
     const int mt = m / p.bn, col = m % p.bn;
     const int tile_id = nt * p.m_tiles + mt;
     const float4* src = reinterpret_cast<const float4*>(p.ws + (int64_t)tile_id * (BM * p.bn) + (int64_t)col * BM) + rq;
-    float4 acc = __ldcg(src);
-    // chunk order z = 1..S-1; the loads of a group of 8 are all in flight before the adds
-    for (int z0 = 1; z0 < p.splits; z0 += 8) {
+    // chunk order z = 0..S-1; a group of 8 chunks' loads are all in flight before the adds
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int z0 = 0; z0 < p.splits; z0 += 8) {
       float4 v[8];
 #pragma unroll
       for (int i = 0; i < 8; ++i)
@@ -319,10 +319,14 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
 #pragma unroll
       for (int i = 0; i < 8; ++i)
         if (z0 + i < p.splits) {
-          acc.x += v[i].x;
-          acc.y += v[i].y;
-          acc.z += v[i].z;
-          acc.w += v[i].w;
+          if (z0 + i == 0) {
+            acc = v[0];
+          } else {
+            acc.x += v[i].x;
+            acc.y += v[i].y;
+            acc.z += v[i].z;
+            acc.w += v[i].w;
+          }
         }
     }
     const float a[4] = {acc.x, acc.y, acc.z, acc.w};
