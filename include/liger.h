@@ -227,18 +227,6 @@ int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* 
 int liger_op_gemm_tiled(const void* x, int64_t ldx, const void* w_tiled, void* out, int64_t ldo, int M, int N,
                         int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
                         void* workspace, size_t ws_bytes, void* stream);
-/* Row-parallel projection fused with the residual add + LayerNorm that follows
- * it (decode, t = 1; PAPER.md P:286 layer, §8(a) a5+a7 / a9+a11):
- *   part = bf16(x @ W^T) (not stored); resid_out = bf16(resid + part + add_bias);
- *   y = LN(resid_out) * gamma + beta
- * Only when liger_gemm_can_fuse_ln(M, N, K) (the plan splits K; the fused
- * split-K fixup runs one 8-CTA cluster per row).  Bit-identical to
- * liger_op_gemm_tiled followed by liger_op_add_layernorm.  resid_out may alias resid. */
-int liger_op_gemm_tiled_add_ln(const void* x, int64_t ldx, const void* w_tiled, int M, int N, int K,
-                               void* workspace, size_t ws_bytes, const void* resid, void* resid_out,
-                               const void* add_bias, const void* gamma, const void* beta, void* y, float eps,
-                               void* stream);
-int liger_gemm_can_fuse_ln(int M, int N, int K);
 /* Convert a row-major bf16 W [N, K] (row stride ld) to the tiled layout
  * (dst holds ceil(N/128)*128*K elements; padding rows are zero). */
 int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K, void* stream);

@@ -69,18 +69,6 @@ int liger_op_gemm_tiled(const void* x, int64_t ldx, const void* w, void* out, in
   return ret(gemm_launch(a, (cudaStream_t)stream), "liger_op_gemm_tiled");
 }
 
-int liger_op_gemm_tiled_add_ln(const void* x, int64_t ldx, const void* w, int M, int N, int K, void* workspace,
-                               size_t ws_bytes, const void* resid, void* resid_out, const void* add_bias,
-                               const void* gamma, const void* beta, void* y, float eps, void* stream) {
-  if (int rc = check_device()) return rc;
-  GemmArgs a{x, ldx, w, 64, nullptr, N, M, N, K, 0, N, nullptr, 0, 0, 1.0f, 0, workspace, ws_bytes, 1};
-  a.ln_x = resid; a.ln_xout = resid_out; a.ln_add_bias = add_bias; a.ln_g = gamma; a.ln_b = beta; a.ln_y = y;
-  a.ln_eps = eps;
-  return ret(gemm_launch(a, (cudaStream_t)stream), "liger_op_gemm_tiled_add_ln");
-}
-
-int liger_gemm_can_fuse_ln(int M, int N, int K) { return gemm_can_fuse_ln(M, N, K) ? 1 : 0; }
-
 int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K, void* stream) {
   if (int rc = check_device()) return rc;
   return ret(tile_weight_launch(w, ld, w_tiled, N, K, (cudaStream_t)stream), "liger_op_tile_weight");

@@ -163,7 +163,6 @@ struct liger_ctx {
   size_t ev_next = 0;
   DurTable dur;
   double attn_scale[2] = {1.0, 1.0};   // calibration of the attention duration model (prefill, decode)
-  bool no_ln_fuse = false;             // LIGER_NO_LN_FUSE=1 disables the fused fixup + LN
   uint32_t dbg_skip = 0;               // LIGER_DBG_SKIP=op,op,...: timing experiments only (wrong results)
   bool ar_atomic_chunks = false;
   // stats / timing
@@ -255,15 +254,6 @@ int unit_col(int N, int u, int F) {
 int pad128(int n) { return (n + 127) / 128 * 128; }
 
 int batch_M(const Batch* bt, int pass) { return pass == 0 ? bt->b * bt->s : bt->b; }
-
-// Is the residual add + LayerNorm after row-parallel GEMM `gemm_op` of `layer`
-// fused into that GEMM's split-K fixup?  (t = 1 only: at t > 1 the all-reduce
-// sits between them.  The last layer's FC2 feeds the LM head's own LN.)
-bool ln_fused(liger_ctx* c, const Batch* bt, int pass, int gemm_op, int layer) {
-  if (c->tp != 1 || c->no_ln_fuse) return false;
-  if (gemm_op == OP_FC2 && layer == c->l1 - 1) return false;   // next LN is on another stage / the LM head
-  return gemm_can_fuse_ln(batch_M(bt, pass), c->h, gemm_K(c, gemm_op));
-}
 
 // ------------------------------------------------------------------ durations
 double model_dur(liger_ctx* c, int op, int M, int k, int ctx_len, int s_len) {
@@ -385,7 +375,6 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_LN1: {
-      if (li > c->l0 && ln_fused(c, bt, pass, OP_FC2, li - 1)) break;   // done in FC2's fixup
       timed_begin(c, st, &ta);
       if (li == c->l0)   // first layer of the model / of this pipeline stage: x is complete
         rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
@@ -396,7 +385,6 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_LN2: {
-      if (ln_fused(c, bt, pass, OP_OUT, li)) break;                 // done in out-proj's fixup
       timed_begin(c, st, &ta);
       rc = add_layernorm_launch(S.x, S.part, W->b_o, S.x, S.y, W->g2, W->be2, M, h, 1, 0, eps, st);
       timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * 4, 0);
@@ -421,20 +409,11 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
         g.scale_cols = c->hl; g.scale = 1.0f / sqrtf((float)c->d);
       } else if (po.op == OP_OUT) {
         g.x = S.attn; g.ldx = c->hl; g.w = W->w_o; g.ldw = K; g.out = S.part; g.ldo = h;
-        if (ln_fused(c, bt, pass, OP_OUT, li) && g.n0 == 0 && g.n1 == N) {
-          g.ln_x = S.x; g.ln_xout = S.x; g.ln_add_bias = W->b_o; g.ln_g = W->g2; g.ln_b = W->be2; g.ln_y = S.y;
-          g.ln_eps = eps;
-        }
       } else if (po.op == OP_FC1) {
         g.x = S.y; g.ldx = h; g.w = W->w_1; g.ldw = K; g.out = S.hbuf; g.ldo = N; g.bias = W->b_1;
         g.act = c->cfg.act;
       } else {
         g.x = S.hbuf; g.ldx = c->fl; g.w = W->w_2; g.ldw = K; g.out = S.part; g.ldo = h;
-        if (ln_fused(c, bt, pass, OP_FC2, li) && g.n0 == 0 && g.n1 == N) {
-          const LayerW& Wn = c->layers[li + 1];
-          g.ln_x = S.x; g.ln_xout = S.x; g.ln_add_bias = W->b_2; g.ln_g = Wn.g1; g.ln_b = Wn.be1; g.ln_y = S.y;
-          g.ln_eps = eps;
-        }
       }
       timed_begin(c, st, &ta);
       cudaEvent_t tmid = timed_mid(c);
@@ -444,13 +423,13 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       rc = gemm_launch(g, st);
       const double n = g.n1 - g.n0;
       if (c->timing) {
-        // GEMM kernel: algorithmic bytes / flops; fixup: fp32 partials read + output (and LN operands) written
+        // GEMM kernel: algorithmic bytes / flops; fixup: fp32 partials read + output written
         c->timed.push_back({M <= 64 ? LIGER_KT_GEMM_DECODE : LIGER_KT_GEMM_PREFILL, ta, tmid,
                             (n * K + (double)M * K + (double)M * n) * 2, 2.0 * M * n * K});
         if (fix) {
           const GemmPlan pl = gemm_plan(M, N, K);
           timed_end(c, st, tmid, LIGER_KT_FIXUP,
-                    (double)pl.splits * M * n * 4 + (double)M * n * (g.ln_y ? 2 * 4 : 2), 0);
+                    (double)pl.splits * M * n * 4 + (double)M * n * 2, 0);
         }
       }
       c->st.gpu_launches++;
@@ -763,7 +742,6 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   }
   c->F = std::max(1, cfg->decomp_factor);
   c->cf = cfg->contention_factor > 0 ? cfg->contention_factor : 1.0;
-  c->no_ln_fuse = getenv("LIGER_NO_LN_FUSE") != nullptr;
   if (const char* sk = getenv("LIGER_DBG_SKIP")) {
     std::string all = std::string(",") + sk + ",";
     for (int o = 0; o < OP_COUNT; ++o)

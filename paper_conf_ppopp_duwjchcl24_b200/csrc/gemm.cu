@@ -342,135 +342,6 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
   }
 }
 
-// Split-K fixup fused with the residual add and LayerNorm that follow the
-// row-parallel projections (decode, t = 1):
-//   part = bf16(sum_z partial[z]);  r = bf16(x + part + add_bias);  y = LN(r)
-// A cluster of LN_FUSE_CLUSTER CTAs owns one row m; each CTA sums its column
-// block, and the row statistics are reduced over the cluster through DSMEM in
-// rank order (deterministic).  Same bits as the unfused GEMM -> add_ln path.
-struct LnFuseParams {
-  const __nv_bfloat16* x;
-  __nv_bfloat16* x_out;
-  const __nv_bfloat16* add_bias;
-  const __nv_bfloat16* g;
-  const __nv_bfloat16* b;
-  __nv_bfloat16* y;
-  float eps;
-};
-
-__device__ __forceinline__ float cluster_sum(float v, float* slot, float* red) {
-  // CTA-level sum (warp shuffles + smem), then over the cluster's CTAs in rank order
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
-  if (l == 0) red[w] = v;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    float s = 0.f;
-    for (int i = 0; i < (int)(blockDim.x >> 5); ++i) s += red[i];
-    *slot = s;
-  }
-  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-  // all LN_FUSE_CLUSTER remote slots requested back to back, then summed in rank order
-  float x[LN_FUSE_CLUSTER];
-#pragma unroll
-  for (int r = 0; r < LN_FUSE_CLUSTER; ++r) {
-    uint32_t remote;
-    // volatile: stays after the cluster barrier; no use until all are issued
-    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(smem_u32(slot)), "r"(r));
-    asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(x[r]) : "r"(remote));
-  }
-  float tot = 0.f;
-#pragma unroll
-  for (int r = 0; r < LN_FUSE_CLUSTER; ++r) tot += x[r];
-  return tot;
-}
-
-constexpr int LNF_THREADS = 256, LNF_MAXC = 6;   // h / 8 <= 1536 columns per CTA
-
-__global__ void __launch_bounds__(LNF_THREADS) splitk_reduce_ln_kernel(const GemmParams p, const LnFuseParams q) {
-  __shared__ float red[LNF_THREADS / 32];
-  __shared__ float slot[2];
-  pdl_enter();
-  const int m = blockIdx.y;
-  const int rank = blockIdx.x;   // == %cluster_ctarank for cluster dims (LN_FUSE_CLUSTER, 1, 1)
-  const int cw = p.N / LN_FUSE_CLUSTER;
-  const int n_begin = rank * cw;
-  const int tiles = p.n_tiles * p.m_tiles;
-  const int64_t zstride = (int64_t)tiles * (BM * p.bn);
-  const int mt = m / p.bn, col = m % p.bn;
-  float r[LNF_MAXC], xv[LNF_MAXC], bv[LNF_MAXC], gv[LNF_MAXC], bev[LNF_MAXC];
-#pragma unroll
-  for (int i = 0; i < LNF_MAXC; ++i) {   // operands first: their loads overlap the partial sums
-    const int c = threadIdx.x + i * LNF_THREADS;
-    xv[i] = bv[i] = gv[i] = bev[i] = 0.f;
-    if (c < cw) {
-      const int n = n_begin + c;
-      xv[i] = __bfloat162float(q.x[(int64_t)m * p.N + n]);
-      if (q.add_bias) bv[i] = __bfloat162float(q.add_bias[n]);
-      gv[i] = __bfloat162float(q.g[n]);
-      bev[i] = __bfloat162float(q.b[n]);
-    }
-  }
-  // partial sums of all this thread's columns: 8 chunks x all columns per batch of loads
-  const float* srcs[LNF_MAXC];
-  float accs[LNF_MAXC];
-#pragma unroll
-  for (int i = 0; i < LNF_MAXC; ++i) {
-    const int n = n_begin + min(threadIdx.x + i * LNF_THREADS, cw - 1);
-    srcs[i] = p.ws + (int64_t)((n / BM) * p.m_tiles + mt) * (BM * p.bn) + (int64_t)col * BM + (n % BM);
-    accs[i] = 0.f;
-  }
-  const int nvalid = (cw - (int)threadIdx.x + LNF_THREADS - 1) / LNF_THREADS;   // columns of this thread
-  for (int z0 = 0; z0 < p.splits; z0 += 8) {
-    float v[LNF_MAXC][8];
-#pragma unroll
-    for (int i = 0; i < LNF_MAXC; ++i)
-#pragma unroll
-      for (int j = 0; j < 8; ++j)
-        v[i][j] = (i < nvalid && z0 + j < p.splits) ? __ldcg(srcs[i] + (z0 + j) * zstride) : 0.f;
-#pragma unroll
-    for (int i = 0; i < LNF_MAXC; ++i)
-#pragma unroll
-      for (int j = 0; j < 8; ++j)
-        if (z0 + j < p.splits) accs[i] = (z0 + j == 0) ? v[i][j] : accs[i] + v[i][j];   // chunk order
-  }
-  float s = 0.f;
-#pragma unroll
-  for (int i = 0; i < LNF_MAXC; ++i) {
-    const int c = threadIdx.x + i * LNF_THREADS;
-    r[i] = 0.f;
-    if (c < cw) {
-      const int n = n_begin + c;
-      const float acc = accs[i];
-      const float part = __bfloat162float(__float2bfloat16_rn(acc));
-      float v = xv[i] + part;
-      if (q.add_bias) v += bv[i];
-      v = __bfloat162float(__float2bfloat16_rn(v));   // residual stream is bf16
-      r[i] = v;
-      s += v;
-    }
-  }
-  const float mean = cluster_sum(s, &slot[0], red) / (float)p.N;
-  float sq = 0.f;
-#pragma unroll
-  for (int i = 0; i < LNF_MAXC; ++i)
-    if (threadIdx.x + i * LNF_THREADS < cw) sq += (r[i] - mean) * (r[i] - mean);
-  const float var = cluster_sum(sq, &slot[1], red) / (float)p.N;
-  const float rstd = 1.0f / sqrtf(var + q.eps);
-#pragma unroll
-  for (int i = 0; i < LNF_MAXC; ++i) {
-    const int c = threadIdx.x + i * LNF_THREADS;
-    if (c < cw) {
-      const int n = n_begin + c;
-      q.x_out[(int64_t)m * p.N + n] = __float2bfloat16_rn(r[i]);
-      q.y[(int64_t)m * p.N + n] = __float2bfloat16_rn((r[i] - mean) * rstd * gv[i] + bev[i]);
-    }
-  }
-  // keep this CTA's shared slots alive until every CTA of the cluster has read them
-  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-
 // ------------------------------------------------------------------ host side
 typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                     const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
@@ -606,10 +477,6 @@ GemmPlan gemm_plan(int M, int N, int K) {
   return pl;
 }
 
-bool gemm_can_fuse_ln(int M, int N, int K) {
-  return gemm_plan(M, N, K).splits > 1 && N % LN_FUSE_CLUSTER == 0 && N / LN_FUSE_CLUSTER <= LNF_THREADS * LNF_MAXC;
-}
-
 size_t gemm_workspace_bytes(int M, int N, int K) {
   GemmPlan pl = gemm_plan(M, N, K);
   if (pl.splits <= 1) return GEMM_COUNTER_BYTES;
@@ -663,26 +530,6 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (a.had_fixup) *a.had_fixup = p.splits > 1;
   if (a.ev_mid) cudaEventRecord(a.ev_mid, stream);
   if (rc2 || p.splits == 1) return rc2 ? LIGER_ECUDA : 0;
-  if (a.ln_y) {
-    if (a.n0 != 0 || a.n1 != a.N || !gemm_can_fuse_ln(a.M, a.N, a.K) || !a.ln_x || !a.ln_xout || !a.ln_g || !a.ln_b)
-      return LIGER_EINVAL;
-    LnFuseParams q{(const __nv_bfloat16*)a.ln_x, (__nv_bfloat16*)a.ln_xout, (const __nv_bfloat16*)a.ln_add_bias,
-                   (const __nv_bfloat16*)a.ln_g, (const __nv_bfloat16*)a.ln_b, (__nv_bfloat16*)a.ln_y, a.ln_eps};
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(LN_FUSE_CLUSTER, a.M);
-    cfg.blockDim = dim3(LNF_THREADS);
-    cfg.stream = stream;
-    cudaLaunchAttribute attr[2];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = LN_FUSE_CLUSTER;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[1].val.programmaticStreamSerializationAllowed = getenv("LIGER_NO_PDL") ? 0 : 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 2;
-    return cudaLaunchKernelEx(&cfg, splitk_reduce_ln_kernel, p, q) == cudaSuccess ? 0 : LIGER_ECUDA;
-  }
   const int64_t work = (int64_t)p.M * (BM / 4) * p.n_tiles;
   int rblocks = (int)((work + 255) / 256);
   if (rblocks > num_sms() * 8) rblocks = num_sms() * 8;

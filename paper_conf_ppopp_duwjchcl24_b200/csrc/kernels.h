@@ -34,13 +34,6 @@ struct GemmArgs {
   // Optional fused residual add + LayerNorm on the split-K fixup (full rows only,
   // n0 == 0 && n1 == N, splits > 1): x_out = bf16(x + bf16(out) + add_bias),
   // y = LN(x_out) * g + b; `out` itself is then not written.
-  const void* ln_x = nullptr;
-  void* ln_xout = nullptr;
-  const void* ln_add_bias = nullptr;
-  const void* ln_g = nullptr;
-  const void* ln_b = nullptr;
-  void* ln_y = nullptr;
-  float ln_eps = 1e-5f;
   // optional: recorded on the stream between the GEMM kernel and its split-K fixup
   // (per-kernel timing; breaks the PDL overlap of the two)
   cudaEvent_t ev_mid = nullptr;
@@ -48,7 +41,6 @@ struct GemmArgs {
 };
 
 GemmPlan gemm_plan(int M, int N, int K);
-constexpr int LN_FUSE_CLUSTER = 8;   // CTAs per row in the fused fixup + LayerNorm
 // true when gemm_launch can fuse add + LN for this full GEMM
 bool gemm_can_fuse_ln(int M, int N, int K);
 size_t gemm_workspace_bytes(int M, int N, int K);
