@@ -173,10 +173,26 @@ int liger_reset_stats(liger_ctx* ctx);
 #define LIGER_KT_ALLREDUCE 3
 #define LIGER_KT_GEMM_PREFILL 4  /* projection GEMMs with M > 64 tokens (tensor-bound) */
 #define LIGER_KT_LMHEAD 5
-#define LIGER_KT_FIXUP 6         /* split-K fixup kernels (+ fused residual add + LN at t = 1) */
-#define LIGER_KT_CLASSES 7
+#define LIGER_KT_FIXUP 6         /* split-K fixup kernels */
+#define LIGER_KT_DECODE_FUSED 7  /* fused decode pass (all layers of a decode step at t = 1, HBM-bound) */
+#define LIGER_KT_CLASSES 8
 int liger_set_kernel_timing(liger_ctx* ctx, int on);
 int liger_kernel_timing(liger_ctx* ctx, int64_t* count, double* ms, double* bytes, double* flops);
+
+/* Timeline trace (diagnostics, not part of the serving path).  liger_trace_start
+ * installs a device buffer of `capacity` records; from then on thread 0 of every
+ * CTA of the GEMM, split-K fixup, add+LN and attention kernels appends one
+ * LIGER_TRACE_REC_BYTES-byte record {uint32 kernel id, CTA index, SM id, pad;
+ * uint64 %globaltimer ns at entry, after the PDL wait, at exit}.  Kernel ids:
+ * 1 GEMM, 2 fixup, 3 decode attention (0x103 = its merging CTA), 5 add+LN.
+ * liger_trace_stop synchronises the device, copies min(n, capacity) records to
+ * host_records (caller-owned), stores the number recorded in *n_out and frees the
+ * buffer.  Records beyond the capacity are dropped.  Process-global; not
+ * thread-safe.  Errors: LIGER_EINVAL (capacity 0), LIGER_ESTATE (not started),
+ * LIGER_ECUDA. */
+#define LIGER_TRACE_REC_BYTES 40
+int liger_trace_start(unsigned int capacity);
+int liger_trace_stop(void* host_records, unsigned int capacity, unsigned int* n_out);
 
 /* Set the per-kernel duration table used by Algorithm 1:
  * durations in microseconds for a kernel class at a token count, piecewise
@@ -269,6 +285,42 @@ int liger_op_attn_prefill(const void* qkv, void* o, void* kv_pool, const int32_t
 int liger_op_attn_decode(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
                          int pos, int heads, int d, void* workspace, size_t ws_bytes, void* stream);
 size_t liger_attn_decode_workspace_bytes(int b, int heads, int d, int ctx);
+
+/* Fused decode pass (§8(a) a2-a11 for one decode step, t = 1): for each layer
+ * l = 0..L-1 of `layers` (device pointers; weights in the tiled layout of
+ * liger_op_gemm_tiled), with M = b <= 32 tokens, in ONE persistent kernel:
+ *   x += part + b_2(l-1) (skipped at l = 0 when first_no_add); y = LN1(x)
+ *   qkv = y W_qkv^T + b_qkv (q columns * qscale); attn = decode attention at `pos`
+ *   over the paged cache of layer l (kv + l * kv_layer_elems elements; appends k, v)
+ *   part = attn W_o^T; x += part + b_o; y = LN2(x); hbuf = act(y W_1^T + b_1);
+ *   part = hbuf W_2^T   (the last layer's b_2 / residual are left to the caller).
+ * Buffers: x, y, part bf16 [M, h]; qkv [M, 3*heads*d]; attn [M, heads*d];
+ * hbuf [M, ffn].  gemm_ws: >= liger_gemm_workspace_bytes of each of the four
+ * GEMMs at M, first 16 KiB zero before first use (left zero); attn_ws as for
+ * liger_op_attn_decode.  The results are bit-identical to the same layers run
+ * op by op (liger_op_add_layernorm, liger_op_gemm_tiled, liger_op_attn_decode).
+ * Shape limits: d in {64, 128}; h, ffn, 3*heads*d multiples of 128; else
+ * LIGER_EINVAL.  The layer table is copied; the library keeps device copies of
+ * its TMA descriptors until the weight pointers change.  Not thread-safe. */
+typedef struct {
+  const void *b_qkv, *b_o, *b_1, *b_2, *g1, *be1, *g2, *be2;
+  const void *w_qkv, *w_o, *w_1, *w_2;
+} liger_fused_layer;
+typedef struct {
+  int32_t L, M, h, heads, d, ffn, act, pos;
+  float eps, qscale;
+  int32_t first_no_add;
+  const liger_fused_layer* layers;   /* host array [L] */
+  void *x, *y, *qkv, *attn, *part, *hbuf, *kv;
+  int64_t kv_layer_elems;
+  const int32_t* page_table;
+  int32_t max_pages;
+  void* gemm_ws;
+  size_t gemm_ws_bytes;
+  void* attn_ws;
+  size_t attn_ws_bytes;
+} liger_fused_decode_args;
+int liger_op_decode_fused(const liger_fused_decode_args* args, void* stream);
 
 /* Row-wise argmax over fp32 logits [rows, n] (row stride ld): writes the
  * maximum value and its index + idx_offset (lowest index on ties, C7). */

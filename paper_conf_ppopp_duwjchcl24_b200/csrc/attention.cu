@@ -15,16 +15,11 @@
 #include <cuda_bf16.h>
 #include <stdint.h>
 
+#include "attn_decode.cuh"
 #include "common.cuh"
 #include "kernels.h"
 
 namespace liger {
-
-constexpr int KVB = LIGER_KV_BLOCK;
-
-__device__ __forceinline__ int64_t kv_off(int page, int kv, int heads, int head, int tok, int D) {
-  return ((((int64_t)page * 2 + kv) * heads + head) * KVB + tok) * D;
-}
 
 // ================================================================== prefill
 constexpr int PF_BQ = 128, PF_BK = 64;
@@ -276,63 +271,39 @@ int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* 
 // products); two-pass softmax over the chunk; phase 2: thread (slot, vec)
 // accumulates p_t V[t] over positions t = slot (mod SLOTS).  Chunks of one
 // (sequence, head) are merged in chunk order by the last CTA (deterministic).
-constexpr int DC_CHUNK_MIN = 32;   // positions per CTA: 32 or 64 (template), chosen per launch
-constexpr int DC_THREADS = 128;
-
 size_t attn_decode_workspace_bytes(int b, int heads, int d, int ctx) {
   const int ns = (ctx + DC_CHUNK_MIN - 1) / DC_CHUNK_MIN;   // worst case (32-position chunks)
   return ATTN_COUNTER_BYTES + (size_t)b * heads * ns * (d + 2) * sizeof(float);
 }
 
-__device__ __forceinline__ void bf16x8_to_f32(const uint4& v, float* f) {
-  const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&v);
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    float2 t = __bfloat1622float2(h[i]);
-    f[2 * i] = t.x;
-    f[2 * i + 1] = t.y;
-  }
-}
+struct CtaSync {
+  __device__ __forceinline__ void operator()() const { __syncthreads(); }
+};
 
+// One CTA per work item (head, sequence, chunk); see attn_decode.cuh.
 template <int D, int DC_CHUNK>
-__global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bfloat16* __restrict__ qkv,
-                                                                 __nv_bfloat16* __restrict__ o,
-                                                                 __nv_bfloat16* __restrict__ kv_pool,
-                                                                 const int32_t* __restrict__ page_table,
-                                                                 int max_pages, int pos, int heads, float* ws,
-                                                                 int* counters) {
-  constexpr int LPT = D / 8;            // lanes per token
-  constexpr int TPW = 32 / LPT;         // tokens per warp step
-  constexpr int WPOS = DC_CHUNK / 4;    // positions per warp in phase 1
-  constexpr int STEPS = WPOS / TPW;     // steps for the warp's positions
-  constexpr int NVEC = D / 8;
-  constexpr int SLOTS = DC_THREADS / NVEC;
-  constexpr int PER = DC_CHUNK / SLOTS; // positions per thread in phase 2
-  constexpr int NPG = DC_CHUNK / KVB;   // pages per chunk
+__global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const DecAttnArgs a) {
+  constexpr int SLOTS = DecAttnSmem<D, DC_CHUNK>::SLOTS;
+  const uint64_t tr0 = trace_now();
   extern __shared__ __align__(128) uint8_t dsm[];
-  __nv_bfloat16* sK = reinterpret_cast<__nv_bfloat16*>(dsm);
-  __nv_bfloat16* sV = sK + DC_CHUNK * D;
   __shared__ float sc[DC_CHUNK];
   __shared__ float red[DC_THREADS / 32];
-  __shared__ float part[SLOTS][D];
+  __shared__ float part[SLOTS * D];
+  __shared__ float mw[DC_MAX_SPLITS], lw[DC_MAX_SPLITS];
   __shared__ __align__(8) uint64_t bar;
   __shared__ int last;
-
+  DecAttnSmem<D, DC_CHUNK> sm;
+  sm.sK = reinterpret_cast<__nv_bfloat16*>(dsm);
+  sm.sV = sm.sK + DC_CHUNK * D;
+  sm.bar = &bar;
+  sm.sc = sc;
+  sm.red = red;
+  sm.part = part;
+  sm.mw = mw;
+  sm.lw = lw;
+  sm.last = &last;
   const int head = blockIdx.x, bi = blockIdx.y, sp = blockIdx.z, nsp = gridDim.z;
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int ctx = pos + 1;
-  const int t0 = sp * DC_CHUNK, t1 = min(ctx, t0 + DC_CHUNK);
-  const int64_t ld = (int64_t)3 * heads * D;
-  const __nv_bfloat16* row = qkv + (int64_t)bi * ld;
-  const __nv_bfloat16* qp = row + head * D;
-  const __nv_bfloat16* knew = row + (int64_t)heads * D + head * D;
-  const __nv_bfloat16* vnew = row + (int64_t)2 * heads * D + head * D;
-  const int32_t* pt = page_table + (int64_t)bi * max_pages;
-  // cached positions of this chunk: [t0, min(t1, pos)) -- pages touching them
-  const int tc1 = min(t1, pos);
-  const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
-
-  if (tid == 0) {
+  if (threadIdx.x == 0) {
     mbar_init(&bar, 1);
     fence_barrier_init();
   }
@@ -340,191 +311,74 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const __nv_bflo
   // The cached positions (< pos) were written by earlier passes, and the page
   // table at admission: staging them does not depend on the preceding kernel
   // (QKV), so it is issued before griddepcontrol.wait.
-  if (warp == 0) {   // lane g stages page g (page ids loaded in parallel, not a serial chain)
-    if (lane == 0) mbar_arrive_expect_tx(&bar, (uint32_t)npg * 2 * KVB * D * 2);
-    __syncwarp();
-    if (lane < npg) {
-      const int page = pt[(t0 >> 4) + lane];
-      bulk_load(sK + lane * KVB * D, kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &bar);
-      bulk_load(sV + lane * KVB * D, kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &bar);
-    }
-  }
+  if (threadIdx.x < 32) dec_attn_issue<D, DC_CHUNK>(a, head, bi, sp, sm.sK, sm.sV, &bar, threadIdx.x);
   pdl_enter();   // q and the new token's k / v come from the QKV kernel
-  float qf[8];
-  {
-    uint4 qv = *reinterpret_cast<const uint4*>(qp + (lane % LPT) * 8);
-    bf16x8_to_f32(qv, qf);
-  }
-  const bool has_new = (t0 <= pos && pos < t1);
-  if (has_new && tid < 2 * NVEC) {   // append the new token's K/V (position pos) to its page
-    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
-    const int page = pt[pos / KVB];
-    *reinterpret_cast<uint4*>(kv_pool + kv_off(page, kv, heads, head, pos % KVB, D) + c) =
-        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
-  }
-  mbar_wait(&bar, 0);
-  if (has_new && tid < 2 * NVEC) {   // ... and into the staged chunk (the bulk copy may predate it)
-    const int kv = tid / NVEC, c = (tid % NVEC) * 8;
-    *reinterpret_cast<uint4*>((kv ? sV : sK) + (pos - t0) * D + c) =
-        *reinterpret_cast<const uint4*>((kv ? vnew : knew) + c);
-  }
-  __syncthreads();
-
-  // ---- phase 1: scores for positions [t0 + warp*WPOS, +WPOS)
-  {
-    const int c = (lane % LPT) * 8;
-#pragma unroll
-    for (int st = 0; st < STEPS; ++st) {
-      const int lt = warp * WPOS + st * TPW + lane / LPT;   // local position
-      float dot = 0.f;
-      if (t0 + lt < t1) {
-        float f[8];
-        bf16x8_to_f32(*reinterpret_cast<const uint4*>(sK + lt * D + c), f);
-#pragma unroll
-        for (int i = 0; i < 8; ++i) dot += qf[i] * f[i];
-      }
-#pragma unroll
-      for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
-      if (t0 + lt < t1 && (lane % LPT) == 0) sc[lt] = dot;
+  const uint64_t tr1 = trace_now();
+  dec_attn_partial<D, DC_CHUNK>(a, head, bi, sp, nsp, sm, 0, threadIdx.x, CtaSync{});
+  bool merged = false;
+  if (nsp > 1) {   // the last chunk of (sequence, head) to finish merges (acq_rel counter)
+    const int64_t unit = (int64_t)bi * a.heads + head;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int prev;
+      asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&a.counters[unit]) : "memory");
+      last = (prev == nsp - 1);
+    }
+    __syncthreads();
+    if (last) {
+      dec_attn_merge<D, DC_CHUNK>(a, head, bi, nsp, sm, threadIdx.x, CtaSync{});
+      if (threadIdx.x == 0) a.counters[unit] = 0;
+      merged = true;
     }
   }
-  __syncthreads();
-  const int n = t1 - t0;
-  float mx = (tid < n) ? sc[tid] : -INFINITY;   // n <= DC_CHUNK <= DC_THREADS
-#pragma unroll
-  for (int off = 16; off > 0; off >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
-  if (lane == 0) red[warp] = mx;
-  __syncthreads();
-  mx = fmaxf(fmaxf(red[0], red[1]), fmaxf(red[2], red[3]));
-  __syncthreads();
-  float p_t = 0.f;
-  if (tid < n) {
-    p_t = __expf(sc[tid] - mx);
-    sc[tid] = p_t;
-  }
-  float sum = p_t;
-#pragma unroll
-  for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
-  if (lane == 0) red[warp] = sum;
-  __syncthreads();
-  const float l = red[0] + red[1] + red[2] + red[3];
-
-  // ---- phase 2: o = sum_t p_t v_t
-  const int vec = tid % NVEC, slot = tid / NVEC;
-  float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-#pragma unroll 4
-  for (int i = 0; i < PER; ++i) {
-    const int lt = slot + i * SLOTS;
-    if (t0 + lt < t1) {
-      const float pw = sc[lt];
-      float f[8];
-      bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + vec * 8), f);
-#pragma unroll
-      for (int e = 0; e < 8; ++e) acc[e] += pw * f[e];
-    }
-  }
-#pragma unroll
-  for (int i = 0; i < 8; ++i) part[slot][vec * 8 + i] = acc[i];
-  __syncthreads();
-
-  if (nsp == 1) {
-    for (int e = tid; e < D; e += DC_THREADS) {
-      float a = 0.f;
-#pragma unroll
-      for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
-      o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / l);
-    }
-    return;
-  }
-  // split: write partial (m, l, acc[D]); the last CTA merges in chunk order
-  const int64_t unit = (int64_t)bi * heads + head;
-  float* wp = ws + (unit * nsp + sp) * (D + 2);
-  for (int e = tid; e < D; e += DC_THREADS) {
-    float a = 0.f;
-#pragma unroll
-    for (int s2 = 0; s2 < SLOTS; ++s2) a += part[s2][e];
-    wp[e] = a;
-  }
-  if (tid == 0) {
-    wp[D] = mx;
-    wp[D + 1] = l;
-  }
-  __syncthreads();
-  if (tid == 0) {
-    int prev;
-    asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&counters[unit]) : "memory");
-    last = (prev == nsp - 1);
-  }
-  __syncthreads();
-  if (!last) return;
-  // merge in chunk order; every load issued in parallel (one per thread, then smem)
-  __shared__ float mw[64], lw[64];   // nsp <= 64 (ctx <= 2048 with 32-position chunks)
-  for (int s2 = tid; s2 < nsp; s2 += DC_THREADS) {
-    const float* w2 = ws + (unit * nsp + s2) * (D + 2);
-    mw[s2] = __ldcg(&w2[D]);
-    lw[s2] = __ldcg(&w2[D + 1]);
-  }
-  __syncthreads();
-  float M = -INFINITY;
-  for (int s2 = 0; s2 < nsp; ++s2) M = fmaxf(M, mw[s2]);
-  float L = 0.f;
-  for (int s2 = 0; s2 < nsp; ++s2) L += lw[s2] * __expf(mw[s2] - M);
-  for (int e = tid; e < D; e += DC_THREADS) {
-    float a = 0.f;
-    for (int z0 = 0; z0 < nsp; z0 += 8) {
-      float v[8];
-#pragma unroll
-      for (int i = 0; i < 8; ++i) v[i] = (z0 + i < nsp) ? __ldcg(&ws[(unit * nsp + z0 + i) * (D + 2) + e]) : 0.f;
-#pragma unroll
-      for (int i = 0; i < 8; ++i)
-        if (z0 + i < nsp) a += v[i] * __expf(mw[z0 + i] - M);
-    }
-    o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(a / L);
-  }
-  if (tid == 0) counters[unit] = 0;
+  if (threadIdx.x == 0) trace_write(merged ? (TK_ATTN_DEC | 0x100) : TK_ATTN_DEC, tr0, tr1);
 }
 
 template <int D, int CH>
-static int launch_decode(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
-                         int pos, int heads, float* ws, int* counters, cudaStream_t stream) {
-  const int ns = (pos + 1 + CH - 1) / CH;
+static int launch_decode(const DecAttnArgs& a, int b, cudaStream_t stream) {
+  const int ns = (a.pos + 1 + CH - 1) / CH;
   const size_t dsmem = (size_t)2 * CH * D * 2;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(attn_decode_kernel<D, CH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
     attr = true;
   }
-  return launch_pdl(attn_decode_kernel<D, CH>, dim3(heads, b, ns), dim3(DC_THREADS), dsmem, stream,
-                    (const __nv_bfloat16*)qkv, (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages,
-                    pos, heads, ws, counters);
+  return launch_pdl(attn_decode_kernel<D, CH>, dim3(a.heads, b, ns), dim3(DC_THREADS), dsmem, stream, a);
 }
 
 int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
                        int pos, int heads, int d, void* workspace, size_t ws_bytes, cudaStream_t stream) {
   if (b <= 0) return 0;
   const int ctx = pos + 1;
-  // 32-position chunks when 64-position ones would leave SMs without ~6 resident CTAs
-  const bool small = (size_t)b * heads * ((ctx + 63) / 64) < (size_t)148 * 6;
-  const int CH = (small && (ctx + 31) / 32 <= 64) ? 32 : 64;
+  const int CH = dec_attn_chunk(b, heads, ctx);
   const int ns = (ctx + CH - 1) / CH;
-  if (ns > 64) return LIGER_EINVAL;   // context longer than 4096 positions
+  if (ns > DC_MAX_SPLITS) return LIGER_EINVAL;   // context longer than 4096 positions
   if (ns > 1) {
     if (!workspace || ws_bytes < attn_decode_workspace_bytes(b, heads, d, ctx) ||
         (size_t)b * heads * 4 > ATTN_COUNTER_BYTES)
       return LIGER_EINVAL;
   }
-  int* counters = (int*)workspace;
-  float* ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
+  DecAttnArgs a;
+  a.qkv = (const __nv_bfloat16*)qkv;
+  a.o = (__nv_bfloat16*)o;
+  a.kv_pool = (__nv_bfloat16*)kv_pool;
+  a.page_table = page_table;
+  a.max_pages = max_pages;
+  a.pos = pos;
+  a.heads = heads;
+  a.counters = (int*)workspace;
+  a.ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
   int rc;
   if (d == 128)
-    rc = CH == 32 ? launch_decode<128, 32>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream)
-               : launch_decode<128, 64>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream);
+    rc = CH == 32 ? launch_decode<128, 32>(a, b, stream) : launch_decode<128, 64>(a, b, stream);
   else if (d == 64)
-    rc = CH == 32 ? launch_decode<64, 32>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream)
-               : launch_decode<64, 64>(qkv, o, kv_pool, page_table, max_pages, b, pos, heads, ws, counters, stream);
+    rc = CH == 32 ? launch_decode<64, 32>(a, b, stream) : launch_decode<64, 64>(a, b, stream);
   else
     return LIGER_EINVAL;
   return rc ? LIGER_ECUDA : 0;
 }
+
+LIGER_TRACE_SETTER(attention)
 
 }  // namespace liger

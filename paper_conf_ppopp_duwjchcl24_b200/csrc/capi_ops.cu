@@ -135,3 +135,64 @@ int liger_op_c0_fill(void* dst, int rows, int cols, int64_t ld, uint64_t seed, u
 }
 
 }  // extern "C"
+
+extern "C" int liger_op_decode_fused(const liger_fused_decode_args* in, void* stream) {
+  if (int rc = check_device()) return rc;
+  if (!in || !in->layers || in->L <= 0) return LIGER_EINVAL;
+  static FusedDecodeState* state = nullptr;   // descriptor tables of the last call's weights
+  static_assert(sizeof(liger_fused_layer) == sizeof(FusedLayerPtrs), "layer table layout");
+  FusedDecodeArgs a{};
+  a.L = in->L; a.M = in->M; a.h = in->h; a.heads = in->heads; a.d = in->d; a.ffn = in->ffn; a.act = in->act;
+  a.pos = in->pos; a.eps = in->eps; a.qscale = in->qscale; a.first_no_add = in->first_no_add;
+  a.layers = reinterpret_cast<const FusedLayerPtrs*>(in->layers);
+  a.x = in->x; a.y = in->y; a.qkv = in->qkv; a.attn = in->attn; a.part = in->part; a.hbuf = in->hbuf;
+  a.kv = in->kv; a.kv_layer_elems = in->kv_layer_elems; a.page_table = in->page_table; a.max_pages = in->max_pages;
+  a.gemm_ws = in->gemm_ws; a.gemm_ws_bytes = in->gemm_ws_bytes; a.attn_ws = in->attn_ws;
+  a.attn_ws_bytes = in->attn_ws_bytes;
+  return ret(fused_decode_launch(&state, a, (cudaStream_t)stream), "liger_op_decode_fused");
+}
+
+// ------------------------------------------------------------------ timeline trace (diagnostics)
+static void* g_trace_rec = nullptr;
+static unsigned int* g_trace_n = nullptr;
+static unsigned int g_trace_cap = 0;
+
+extern "C" int liger_trace_start(unsigned int capacity) {
+  if (capacity == 0) return LIGER_EINVAL;
+  if (g_trace_rec) cudaFree(g_trace_rec);
+  if (g_trace_n) cudaFree(g_trace_n);
+  g_trace_rec = nullptr;
+  g_trace_n = nullptr;
+  if (cudaMalloc(&g_trace_rec, (size_t)capacity * LIGER_TRACE_REC_BYTES) != cudaSuccess ||
+      cudaMalloc((void**)&g_trace_n, sizeof(unsigned int)) != cudaSuccess ||
+      cudaMemset(g_trace_n, 0, sizeof(unsigned int)) != cudaSuccess)
+    return LIGER_ECUDA;
+  g_trace_cap = capacity;
+  TraceRec* r = (TraceRec*)g_trace_rec;
+  trace_set_gemm(r, g_trace_n, capacity);
+  trace_set_norm(r, g_trace_n, capacity);
+  trace_set_attention(r, g_trace_n, capacity);
+  trace_set_fused(r, g_trace_n, capacity);
+  return cudaDeviceSynchronize() == cudaSuccess ? LIGER_OK : LIGER_ECUDA;
+}
+
+extern "C" int liger_trace_stop(void* host_records, unsigned int capacity, unsigned int* n_out) {
+  if (!g_trace_rec) return LIGER_ESTATE;
+  if (cudaDeviceSynchronize() != cudaSuccess) return LIGER_ECUDA;
+  trace_set_gemm(nullptr, nullptr, 0);
+  trace_set_norm(nullptr, nullptr, 0);
+  trace_set_attention(nullptr, nullptr, 0);
+  trace_set_fused(nullptr, nullptr, 0);
+  unsigned int n = 0;
+  cudaMemcpy(&n, g_trace_n, sizeof(n), cudaMemcpyDeviceToHost);
+  if (n > g_trace_cap) n = g_trace_cap;
+  if (n_out) *n_out = n;
+  if (host_records && capacity)
+    cudaMemcpy(host_records, g_trace_rec, (size_t)(n < capacity ? n : capacity) * LIGER_TRACE_REC_BYTES,
+               cudaMemcpyDeviceToHost);
+  cudaFree(g_trace_rec);
+  cudaFree(g_trace_n);
+  g_trace_rec = nullptr;
+  g_trace_n = nullptr;
+  return cudaGetLastError() == cudaSuccess ? LIGER_OK : LIGER_ECUDA;
+}

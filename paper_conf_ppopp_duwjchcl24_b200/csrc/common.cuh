@@ -71,6 +71,10 @@ LIGER_DEV void bulk_load(void* smem_dst, const void* gsrc, uint32_t bytes, uint6
       "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+// Fire-and-forget L2 prefetch of [gsrc, gsrc + bytes) (TMA bulk engine; 16-B aligned, bytes % 16 == 0).
+LIGER_DEV void bulk_prefetch_l2(const void* gsrc, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(gsrc), "r"(bytes) : "memory");
+}
 LIGER_DEV uint64_t policy_evict_first() {
   uint64_t p;
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
@@ -152,6 +156,50 @@ LIGER_DEV void pdl_enter() {
   grid_dependency_wait();
   grid_dependency_trigger();
 }
+
+// ---------------------------------------------------------------- timeline trace
+// Development diagnostics (liger_trace_start / liger_trace_stop): thread 0 of every
+// CTA of a traced kernel appends {kernel id, CTA, SM, entry, after-PDL-wait, exit}
+// %globaltimer stamps.  Off (one predicated load) unless a buffer is installed.
+// Each translation unit holds its own copy of the buffer descriptor.
+struct TraceRec {
+  uint32_t kid, cta, smid, pad;
+  uint64_t t0, t1, t2;
+};
+struct TraceBuf {
+  TraceRec* rec;
+  unsigned int* n;
+  unsigned int cap;
+};
+static __device__ TraceBuf g_trace = {nullptr, nullptr, 0};
+LIGER_DEV uint64_t trace_now() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+LIGER_DEV void trace_write(uint32_t kid, uint64_t t0, uint64_t t1) {
+  if (g_trace.rec == nullptr) return;
+  const uint64_t t2 = trace_now();
+  const unsigned int i = atomicAdd(g_trace.n, 1u);
+  if (i >= g_trace.cap) return;
+  uint32_t sm;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+  TraceRec r;
+  r.kid = kid;
+  r.cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+  r.smid = sm;
+  r.pad = 0;
+  r.t0 = t0;
+  r.t1 = t1;
+  r.t2 = t2;
+  g_trace.rec[i] = r;
+}
+#define LIGER_TRACE_SETTER(name) \
+  void trace_set_##name(TraceRec* rec, unsigned int* n, unsigned int cap) { \
+    TraceBuf b{rec, n, cap};                                                \
+    cudaMemcpyToSymbol(g_trace, &b, sizeof(b));                             \
+  }
+enum TraceKid : uint32_t { TK_GEMM = 1, TK_FIXUP, TK_ATTN_DEC, TK_ATTN_PRE, TK_ADDLN, TK_EMBED, TK_ARGMAX, TK_PICK, TK_FUSED };
 
 LIGER_DEV float bf16_bits_to_f32(uint16_t b) { return __uint_as_float(((uint32_t)b) << 16); }
 

@@ -89,6 +89,7 @@ struct Slot {
   int32_t* h_prompt;       // pinned
   int32_t* h_tok_out;      // pinned
   cudaEvent_t free_ev;     // completes when the last batch using the slot finished
+  FusedDecodeState* fused = nullptr;   // fused decode pass tables of this slot
   Batch* owner = nullptr;  // batch currently (or last) assigned to the slot
 };
 
@@ -165,6 +166,9 @@ struct liger_ctx {
   double attn_scale[2] = {1.0, 1.0};   // calibration of the attention duration model (prefill, decode)
   uint32_t dbg_skip = 0;               // LIGER_DBG_SKIP=op,op,...: timing experiments only (wrong results)
   bool ar_atomic_chunks = false;
+  // decode passes at t = 1 as one fused kernel (LIGER_FUSED_DECODE=1).  Off by default:
+  // measured 17-33 % slower than the per-kernel PDL chain.
+  bool fused_decode = false;
   // stats / timing
   liger_stats_t st{};
   bool timing = false;
@@ -355,6 +359,12 @@ void timing_flush(liger_ctx* c) {
 }
 
 // ------------------------------------------------------------------ launching one piece
+// Decode passes at t = 1 (no all-reduce between the layers' compute runs) go through
+// the fused decode-pass kernel (decode_fused.cu) when its shape limits allow.
+bool fused_pass(liger_ctx* c, int M) {
+  return c->fused_decode && c->tp == 1 && fused_decode_supported(M, c->h, c->al, c->d, c->fl);
+}
+
 int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cudaStream_t st) {
   const PassOp po = c->pass_ops[pidx];
   Slot& S = c->slots[bt->slot];
@@ -366,6 +376,41 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
   int rc = 0;
   cudaEvent_t ta = nullptr;
   if (c->dbg_skip & (1u << po.op)) return 0;
+  if (pass > 0 && li >= 0 && fused_pass(c, M)) {
+    // decode step at t = 1: the whole layer range is one fused kernel, launched at
+    // the range's first op; the per-layer ops it covers launch nothing
+    if (po.op != OP_LN1 || li != c->l0) return 0;
+    FusedDecodeArgs fa{};
+    std::vector<FusedLayerPtrs> lp(c->l1 - c->l0);
+    for (int l = c->l0; l < c->l1; ++l) {
+      const LayerW& w = c->layers[l];
+      lp[l - c->l0] = FusedLayerPtrs{w.b_qkv, w.b_o, w.b_1, w.b_2, w.g1, w.be1, w.g2, w.be2,
+                                     w.w_qkv, w.w_o, w.w_1, w.w_2};
+    }
+    fa.L = c->l1 - c->l0; fa.M = M; fa.h = h; fa.heads = c->al; fa.d = c->d; fa.ffn = c->fl;
+    fa.act = c->cfg.act; fa.pos = bt->s + pass - 1; fa.eps = eps; fa.qscale = 1.0f / sqrtf((float)c->d);
+    fa.first_no_add = 1; fa.layers = lp.data();
+    fa.x = S.x; fa.y = S.y; fa.qkv = S.qkv; fa.attn = S.attn; fa.part = S.part; fa.hbuf = S.hbuf;
+    fa.kv = c->kv; fa.kv_layer_elems = (int64_t)c->kv_layer_elems; fa.page_table = S.page_table;
+    fa.max_pages = c->max_pages;
+    fa.gemm_ws = S.gemm_ws; fa.gemm_ws_bytes = S.gemm_ws_bytes;
+    fa.attn_ws = S.attn_ws; fa.attn_ws_bytes = S.attn_ws_bytes;
+    timed_begin(c, st, &ta);
+    rc = fused_decode_launch(&S.fused, fa, st);
+    if (c->timing) {
+      const double ctx = fa.pos + 1, L = fa.L, hl = c->hl;
+      const double gemm_bytes = ((3 * hl * h + (double)M * h + M * 3 * hl) + (h * hl + M * hl + (double)M * h) +
+                                 ((double)c->fl * h + (double)M * h + (double)M * c->fl) +
+                                 ((double)h * c->fl + (double)M * c->fl + (double)M * h)) * 2;
+      const double attn_bytes = (double)M * hl * 2 * 2 * ctx;
+      const double ln_bytes = 2.0 * M * h * 2 * 4;
+      const double flops = 2.0 * M * (3 * hl * h + h * hl + 2.0 * c->fl * h) + 4.0 * M * hl * ctx;
+      timed_end(c, st, ta, LIGER_KT_DECODE_FUSED, L * (gemm_bytes + attn_bytes + ln_bytes), L * flops);
+    }
+    c->st.gpu_launches++;
+    if (rc < 0) return fail(c, rc, "launch of the fused decode pass failed");
+    return 0;
+  }
   switch (po.op) {
     case OP_EMBED: {
       const int32_t* ids = pass == 0 ? (bt->dev_tokens ? bt->dev_tokens : S.prompt) : S.cur_tok;
@@ -747,6 +792,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     for (int o = 0; o < OP_COUNT; ++o)
       if (all.find(std::string(",") + kOpName[o] + ",") != std::string::npos) c->dbg_skip |= 1u << o;
   }
+  if (const char* fd = getenv("LIGER_FUSED_DECODE")) c->fused_decode = atoi(fd) != 0;
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (tp > 2);
   if (world > 1) {
@@ -1372,6 +1418,7 @@ int liger_finalize(liger_ctx* c) {
     cudaFreeHost(S.h_prompt);
     cudaFreeHost(S.h_tok_out);
     cudaEventDestroy(S.free_ev);
+    fused_decode_free(S.fused);
   }
   for (auto e : c->ev_pool) cudaEventDestroy(e);
   for (auto e : c->timing_pool) cudaEventDestroy(e);

@@ -72,6 +72,8 @@ struct GemmParams {
   int out_f32;
   float* ws;
   int* counters;
+  const void* w_base;   // tiled weights (for the L2 prefetch)
+  int pf_blocks;        // weight blocks (beyond the smem stages) prefetched into L2 before the PDL wait
 };
 
 __device__ __forceinline__ float epi_apply(const GemmParams& p, float v, int n, float bias_v) {
@@ -108,6 +110,8 @@ __device__ __forceinline__ Unit unit_of(const GemmParams& p, int u) {
 __global__ void __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmParams p) {
+  const uint64_t tr0 = trace_now();
+  uint64_t tr1 = tr0;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int S = p.stages;
@@ -171,9 +175,30 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
           }
         }
         pre = it;
+        // While the preceding kernels (fixup, attention, add + LN) finish -- they
+        // leave HBM mostly idle -- pull the next weight blocks of this CTA's own
+        // stream into L2 (a hint; the TMA loads below read them from there).
+        int left = p.pf_blocks, skip = pre;
+        for (int u = blockIdx.x; u < p.units && left > 0; u += G) {
+          const Unit w = unit_of(p, u);
+          if (w.mt) continue;
+          const int k0b = w.z * (p.kc / BK);
+          const int nkb = (min(p.K, w.z * p.kc + p.kc) - w.z * p.kc + BK - 1) / BK;
+          int b0 = skip < nkb ? skip : nkb;
+          skip -= b0;
+          int nb = nkb - b0;
+          if (nb > left) nb = left;
+          if (nb <= 0) continue;
+          const int nt = (p.n0 / BM) + w.nt;
+          bulk_prefetch_l2(reinterpret_cast<const uint8_t*>(p.w_base) +
+                               ((size_t)nt * p.nkb_total + k0b + b0) * A_BYTES,
+                           (uint32_t)nb * A_BYTES);
+          left -= nb;
+        }
       }
       grid_dependency_wait();
       grid_dependency_trigger();   // after the wait: dependents overlap only this kernel
+      tr1 = trace_now();
       int it = 0;
       for (int u = blockIdx.x; u < p.units; u += G) {
         const Unit w = unit_of(p, u);
@@ -274,6 +299,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     tc_fence_after();
     tmem_dealloc(tmem_base, tmem_cols);
   }
+  if (threadIdx.x == 0) trace_write(TK_GEMM, tr0, tr1);
 }
 
 // sum_{z=0..S-1} src[z * zstride] in chunk order, 8 loads in flight
@@ -294,7 +320,9 @@ __device__ __forceinline__ float sum_partials(const float* src, int64_t zstride,
 // same bits whatever slice or CTA produced each chunk).  One thread per (m, 4 rows n),
 // reading the column-major per-tile partials coalesced.
 __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) {
+  const uint64_t tr0 = trace_now();
   pdl_enter();
+  const uint64_t tr1 = trace_now();
   const int tiles = p.n_tiles * p.m_tiles;
   const int64_t zstride = (int64_t)tiles * (BM * p.bn);
   const int slice_w = p.n1 - p.n0;
@@ -340,6 +368,7 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
       }
     }
   }
+  if (threadIdx.x == 0) trace_write(TK_FIXUP, tr0, tr1);
 }
 
 // ------------------------------------------------------------------ host side
@@ -406,6 +435,17 @@ static int make_map(CUtensorMap* out, const void* ptr, int64_t rows, int64_t col
   return 0;
 }
 
+int gemm_weight_map(void* out_, const void* w_tiled, int N, int K) {
+  CUtensorMap* out = static_cast<CUtensorMap*>(out_);
+  if (K % BK) return LIGER_EINVAL;
+  const int64_t rows = (int64_t)((N + BM - 1) / BM) * (K / BK) * BM;
+  return make_map(out, w_tiled, rows, BK, BK, BM);
+}
+int gemm_act_map(void* out_, const void* x, int M, int K, int64_t ldx, int bn) {
+  CUtensorMap* out = static_cast<CUtensorMap*>(out_);
+  return make_map(out, x, M, K, ldx, bn);
+}
+
 void gemm_forget_pointer_range(const void* base, size_t bytes) {
   std::lock_guard<std::mutex> g(g_map_mu);
   for (auto it = g_maps.begin(); it != g_maps.end();) {
@@ -467,7 +507,8 @@ GemmPlan gemm_plan(int M, int N, int K) {
   const int stage_bytes = A_BYTES + pl.bn * BK * 2;
   int st = (MAX_SMEM - 1024 - 512) / stage_bytes;
   if (st > 12) st = 12;
-  if (pl.bn <= 32 && st > 6) st = 6;   // decode: 96 KiB of weights in flight suffices (measured)
+  static const int dec_cap = getenv("LIGER_GEMM_DECODE_STAGES") ? atoi(getenv("LIGER_GEMM_DECODE_STAGES")) : 6;
+  if (pl.bn <= 32 && st > dec_cap) st = dec_cap;   // decode: 96 KiB of weights in flight suffices (measured)
   if (const char* e = getenv("LIGER_GEMM_STAGES")) {   // experiments only
     const int f = atoi(e);
     if (f >= 2 && f < st) st = f;
@@ -520,6 +561,9 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.counters = reinterpret_cast<int*>(a.workspace);
   p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
   p.w_tiled = a.w_tiled;
+  p.w_base = a.w;
+  static const int pf_env = getenv("LIGER_PF_BLOCKS") ? atoi(getenv("LIGER_PF_BLOCKS")) : 0;
+  p.pf_blocks = (a.w_tiled && pl.bn <= 64) ? pf_env : 0;
 
   p.nkb_total = (a.K + BK - 1) / BK;
   p.n_tiles = ntiles;
@@ -535,5 +579,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (rblocks > num_sms() * 8) rblocks = num_sms() * 8;
   return launch_pdl(splitk_reduce_kernel, dim3(rblocks), dim3(256), 0, stream, p) ? LIGER_ECUDA : 0;
 }
+
+LIGER_TRACE_SETTER(gemm)
 
 }  // namespace liger

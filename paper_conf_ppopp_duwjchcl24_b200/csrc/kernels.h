@@ -31,9 +31,6 @@ struct GemmArgs {
   void* workspace;
   size_t ws_bytes;
   int w_tiled;   // 0: W row-major [N, K] (row stride ldw); 1: tiled [ceil(N/128)][K/64][128][64]
-  // Optional fused residual add + LayerNorm on the split-K fixup (full rows only,
-  // n0 == 0 && n1 == N, splits > 1): x_out = bf16(x + bf16(out) + add_bias),
-  // y = LN(x_out) * g + b; `out` itself is then not written.
   // optional: recorded on the stream between the GEMM kernel and its split-K fixup
   // (per-kernel timing; breaks the PDL overlap of the two)
   cudaEvent_t ev_mid = nullptr;
@@ -41,11 +38,40 @@ struct GemmArgs {
 };
 
 GemmPlan gemm_plan(int M, int N, int K);
-// true when gemm_launch can fuse add + LN for this full GEMM
-bool gemm_can_fuse_ln(int M, int N, int K);
 size_t gemm_workspace_bytes(int M, int N, int K);
 int gemm_launch(const GemmArgs& a, cudaStream_t stream);
 void gemm_forget_pointer_range(const void* base, size_t bytes);
+// TMA descriptors as gemm_launch builds them (CUtensorMap, 128 B): a tiled weight
+// matrix (box 64 x 128, SWIZZLE_128B) and a row-major activation [M, K] (box 64 x bn).
+int gemm_weight_map(void* out_map, const void* w_tiled, int N, int K);
+int gemm_act_map(void* out_map, const void* x, int M, int K, int64_t ldx, int bn);
+
+// Fused decode pass (decode_fused.cu): every layer of [l0, l1) of one decode step
+// of one batch (M = b <= 32 tokens, t = 1) in one persistent kernel.
+struct FusedLayerPtrs {
+  const void *b_qkv, *b_o, *b_1, *b_2, *g1, *be1, *g2, *be2;
+  const void *w_qkv, *w_o, *w_1, *w_2;   // tiled weights
+};
+struct FusedDecodeArgs {
+  int L, M, h, heads, d, ffn, act;
+  int pos;             // position of the new token (context = pos + 1)
+  float eps, qscale;
+  int first_no_add;    // layer 0 of the range: x is complete (embedding / received), LN1 adds nothing
+  const FusedLayerPtrs* layers;   // host array [L]
+  void *x, *y, *qkv, *attn, *part, *hbuf;
+  void* kv;            // KV pool of the range's first layer; layer i at kv + i * kv_layer_elems
+  int64_t kv_layer_elems;
+  const int32_t* page_table;
+  int max_pages;
+  void* gemm_ws;       // split-K workspace (GEMM_COUNTER_BYTES of counters + partials)
+  size_t gemm_ws_bytes;
+  void* attn_ws;       // decode-attention workspace
+  size_t attn_ws_bytes;
+};
+struct FusedDecodeState;   // per-slot device tables (weight descriptors, sync counter base)
+bool fused_decode_supported(int M, int h, int heads, int d, int ffn);
+int fused_decode_launch(FusedDecodeState** state, const FusedDecodeArgs& a, cudaStream_t stream);
+void fused_decode_free(FusedDecodeState* state);
 
 int add_layernorm_launch(const void* x, const void* add, const void* add_bias, void* x_out, void* y,
                          const void* gamma, const void* beta, int rows, int h, int in_row_step, int in_row_off,
@@ -70,5 +96,12 @@ int tile_weight_launch(const void* src, int64_t ld, void* dst, int N, int K, cud
 inline __host__ __device__ int64_t tiled_offset(int n, int k, int K) {
   return (((int64_t)(n >> 7) * (K >> 6) + (k >> 6)) << 13) + ((n & 127) << 6) + (k & 63);
 }
+
+// timeline trace (common.cuh TraceRec): per translation unit buffer installers
+struct TraceRec;
+void trace_set_gemm(TraceRec* rec, unsigned int* n, unsigned int cap);
+void trace_set_norm(TraceRec* rec, unsigned int* n, unsigned int cap);
+void trace_set_attention(TraceRec* rec, unsigned int* n, unsigned int cap);
+void trace_set_fused(TraceRec* rec, unsigned int* n, unsigned int cap);
 
 }  // namespace liger

@@ -53,7 +53,9 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
                                                     const bf16x8* __restrict__ beta, int h, int in_row_step,
                                                     int in_row_off, float eps) {
   __shared__ float red[NT / 32];
+  const uint64_t tr0 = trace_now();
   pdl_enter();
+  const uint64_t tr1 = trace_now();
   const int nv = h >> 3;
   const int64_t in_row = (int64_t)blockIdx.x * in_row_step + in_row_off;
   const bf16x8* xr = x + in_row * nv;
@@ -122,6 +124,7 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
       y[(int64_t)blockIdx.x * nv + v] = pack8(o);
     }
   }
+  if (threadIdx.x == 0) trace_write(TK_ADDLN, tr0, tr1);
 }
 
 int add_layernorm_launch(const void* x, const void* add, const void* add_bias, void* x_out, void* y,
@@ -314,5 +317,7 @@ int copy_tokens_launch(const int32_t* src, int32_t* dst, int n, cudaStream_t str
   copy_i32_kernel<<<(n + 255) / 256, 256, 0, stream>>>(src, dst, n);
   return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
 }
+
+LIGER_TRACE_SETTER(norm)
 
 }  // namespace liger

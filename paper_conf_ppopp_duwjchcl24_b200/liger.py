@@ -12,7 +12,8 @@ LIGER_OK, LIGER_PENDING, LIGER_IDLE = 0, 1, 2
 ACT = {"none": 0, "relu": 1, "gelu_tanh": 2}
 MODE = {"serial": 0, "interleaved": 1, "pipeline": 2}
 KV_BLOCK = 16
-KT_NAMES = ["gemm_decode", "attn", "ln", "allreduce", "gemm_prefill", "lm_head", "splitk_fixup"]   # LIGER_KT_*
+KT_NAMES = ["gemm_decode", "attn", "ln", "allreduce", "gemm_prefill", "lm_head", "splitk_fixup",
+            "decode_fused"]   # LIGER_KT_*
 OPS = ["embed", "ln1", "qkv", "attn", "out", "ar1", "ln2", "fc1", "fc2", "ar2", "head", "tokg", "pick",
        "recv_x", "send_x", "recv_tok", "send_tok"]
 
@@ -33,6 +34,21 @@ class liger_result(C.Structure):
     _fields_ = [("id", C.c_int64), ("batch", C.c_int32), ("seq_len", C.c_int32), ("n_new", C.c_int32),
                 ("done", C.c_int32), ("arrival_s", C.c_double), ("submit_s", C.c_double),
                 ("start_s", C.c_double), ("finish_s", C.c_double)]
+
+
+class liger_fused_layer(C.Structure):
+    _fields_ = [(n, C.c_void_p) for n in ("b_qkv", "b_o", "b_1", "b_2", "g1", "be1", "g2", "be2",
+                                          "w_qkv", "w_o", "w_1", "w_2")]
+
+
+class liger_fused_decode_args(C.Structure):
+    _fields_ = [("L", C.c_int32), ("M", C.c_int32), ("h", C.c_int32), ("heads", C.c_int32), ("d", C.c_int32),
+                ("ffn", C.c_int32), ("act", C.c_int32), ("pos", C.c_int32), ("eps", C.c_float),
+                ("qscale", C.c_float), ("first_no_add", C.c_int32), ("layers", C.POINTER(liger_fused_layer)),
+                ("x", C.c_void_p), ("y", C.c_void_p), ("qkv", C.c_void_p), ("attn", C.c_void_p),
+                ("part", C.c_void_p), ("hbuf", C.c_void_p), ("kv", C.c_void_p), ("kv_layer_elems", C.c_int64),
+                ("page_table", C.c_void_p), ("max_pages", C.c_int32), ("gemm_ws", C.c_void_p),
+                ("gemm_ws_bytes", C.c_size_t), ("attn_ws", C.c_void_p), ("attn_ws_bytes", C.c_size_t)]
 
 
 class liger_stats_t(C.Structure):
@@ -80,6 +96,9 @@ _SIGS = {
     "liger_planner_submit": (_I, [_P, _I64, _I, _P, _P, _P]),
     "liger_plan_round": (_I, [_P, _P, _I, _P, _P, _P]),
     "liger_planner_destroy": (_I, [_P]),
+    "liger_op_decode_fused": (_I, [C.POINTER(liger_fused_decode_args), _P]),
+    "liger_trace_start": (_I, [C.c_uint]),
+    "liger_trace_stop": (_I, [_P, C.c_uint, _P]),
 }
 
 
@@ -207,3 +226,40 @@ def c0_fill(dst, *, seed, tensor_id, row_off=0, col_off=0, idx_row_stride, idx_c
     rows, cols = dst.shape
     check(lib().liger_op_c0_fill(_p(dst), rows, cols, dst.stride(0), seed, tensor_id, row_off, col_off,
                                  idx_row_stride, idx_col_stride, exp, kind, _s(stream)), what="liger_op_c0_fill")
+
+
+def decode_fused(layers, *, M, h, heads, d, ffn, act, pos, x, y, qkv, attn, part, hbuf, kv, kv_layer_elems,
+                 page_table, max_pages, gemm_ws, attn_ws, eps=1e-5, qscale=None, first_no_add=True, stream=None):
+    """liger_op_decode_fused: `layers` = list of dicts of torch tensors (tiled weights)."""
+    arr = (liger_fused_layer * len(layers))()
+    for i, w in enumerate(layers):
+        for n, _ in liger_fused_layer._fields_:
+            setattr(arr[i], n, w[n].data_ptr())
+    a = liger_fused_decode_args(len(layers), M, h, heads, d, ffn, ACT[act], pos, eps,
+                                qscale if qscale is not None else d ** -0.5, int(first_no_add), arr,
+                                x.data_ptr(), y.data_ptr(), qkv.data_ptr(), attn.data_ptr(), part.data_ptr(),
+                                hbuf.data_ptr(), kv.data_ptr(), kv_layer_elems, page_table.data_ptr(), max_pages,
+                                gemm_ws.data_ptr(), gemm_ws.numel() * gemm_ws.element_size(),
+                                attn_ws.data_ptr(), attn_ws.numel() * attn_ws.element_size())
+    check(lib().liger_op_decode_fused(C.byref(a), _s(stream)), None, "liger_op_decode_fused")
+
+
+TRACE_KIDS = {1: "gemm", 2: "fixup", 3: "attn_dec", 0x103: "attn_merge", 4: "attn_pre", 5: "add_ln", 9: "fused"}
+
+
+def trace_start(capacity=1 << 20):
+    """Diagnostics: start the per-CTA kernel timeline trace (liger_trace_start)."""
+    check(lib().liger_trace_start(capacity), None, "liger_trace_start")
+    return capacity
+
+
+def trace_stop(capacity=1 << 20):
+    """Stop the trace; returns a numpy structured array (kid, cta, smid, t0, t1, t2 in ns)."""
+    import numpy as np
+    dt = np.dtype([("kid", "<u4"), ("cta", "<u4"), ("smid", "<u4"), ("pad", "<u4"),
+                   ("t0", "<u8"), ("t1", "<u8"), ("t2", "<u8")])
+    assert dt.itemsize == 40
+    buf = np.zeros(capacity, dtype=dt)
+    n = C.c_uint(0)
+    check(lib().liger_trace_stop(buf.ctypes.data, capacity, C.byref(n)), None, "liger_trace_stop")
+    return buf[:min(n.value, capacity)]
