@@ -64,13 +64,74 @@ static ncclDataType_t nccl_dt(CommDType d) {
 }
 static size_t dt_size(CommDType d) { return d == CD_BF16 ? 2 : 4; }
 
+// One-shot peer all-reduce for decode-size bf16 sums (LIGER_ONESHOT_AR=0/1 overrides
+// the backend default; LIGER_ONESHOT_MAX_KB the largest message, default 1024).
+static bool oneshot_enabled(bool dflt) {
+  const char* e = getenv("LIGER_ONESHOT_AR");
+  return e ? atoi(e) != 0 : dflt;
+}
+static size_t oneshot_cap() {
+  const char* e = getenv("LIGER_ONESHOT_MAX_KB");
+  const size_t kb = e ? (size_t)atoll(e) : 1024;
+  return (kb * 1024 + 255) / 256 * 256;
+}
+static bool oneshot_eligible(size_t count, CommDType dt, CommOp op, const void* buf) {
+  return dt == CD_BF16 && op == CO_SUM && count * 2 <= oneshot_cap() && (count * 2) % 16 == 0 &&
+         reinterpret_cast<uintptr_t>(buf) % 16 == 0;
+}
+
 struct NcclComm : Comm {
   ncclComm_t comm = nullptr;
+  int world = 1, rank = 0;
+  bool oneshot = false;
+  PeerAR* par = nullptr;
+  void* region = nullptr;
+  void* mapped[8] = {};
   ~NcclComm() override {
+    cudaDeviceSynchronize();
+    delete par;
+    for (int q = 0; q < world && q < 8; ++q)
+      if (mapped[q] && q != rank) cudaIpcCloseMemHandle(mapped[q]);
+    if (region) cudaFree(region);
     if (comm) nccl().CommDestroy(comm);
+  }
+  // [collective] map every rank's staging region: CUDA IPC handles exchanged with an
+  // NCCL all-gather (same-node NVLink / NVSwitch peers)
+  int setup_oneshot(cudaStream_t st) {
+    const size_t cap = oneshot_cap(), rb = peer_ar_region_bytes(cap);
+    if (world > 8 || cudaMalloc(&region, rb) != cudaSuccess || cudaMemset(region, 0, rb) != cudaSuccess)
+      return LIGER_ENOMEM;
+    cudaIpcMemHandle_t h;
+    if (cudaIpcGetMemHandle(&h, region) != cudaSuccess) return LIGER_ECUDA;
+    char* d = nullptr;
+    if (cudaMalloc(&d, (size_t)64 * (world + 1)) != cudaSuccess) return LIGER_ENOMEM;
+    cudaMemcpy(d + (size_t)64 * world, &h, 64, cudaMemcpyHostToDevice);
+    ncclResult_t r = nccl().AllGather(d + (size_t)64 * world, d, 64, ncclUint8, comm, st);
+    std::vector<cudaIpcMemHandle_t> all(world);
+    if (r == ncclSuccess && cudaStreamSynchronize(st) == cudaSuccess)
+      cudaMemcpy(all.data(), d, (size_t)64 * world, cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    if (r != ncclSuccess) return LIGER_ENCCL;
+    for (int q = 0; q < world; ++q) {
+      if (q == rank) {
+        mapped[q] = region;
+        continue;
+      }
+      if (cudaIpcOpenMemHandle(&mapped[q], all[q], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        err = "cudaIpcOpenMemHandle failed (peers not P2P-capable?)";
+        return LIGER_ECUDA;
+      }
+    }
+    par = new PeerAR();
+    return par->init(world, rank, cap, region, mapped);
   }
   int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
     if (!count) return 0;
+    if (oneshot && oneshot_eligible(count, dt, op, buf)) {
+      if (!par)
+        if (int rc = setup_oneshot(st)) return rc;
+      return par->allreduce_bf16(buf, count, st);
+    }
     ncclResult_t r = nccl().AllReduce(buf, buf, count, nccl_dt(dt), op == CO_SUM ? ncclSum : ncclMax, comm, st);
     if (r != ncclSuccess) {
       err = std::string("ncclAllReduce: ") + nccl().GetErrorString(r);
@@ -217,8 +278,13 @@ struct LoopbackComm : Comm {
   cudaEvent_t ev_ready = nullptr, ev_done = nullptr;
   void* scratch = nullptr;
   size_t scratch_bytes = 0;
+  bool oneshot = true;
+  PeerAR* par = nullptr;
+  void* region = nullptr;
   ~LoopbackComm() override {
     cudaDeviceSynchronize();
+    delete par;
+    if (region) cudaFree(region);
     if (ev_ready) cudaEventDestroy(ev_ready);
     if (ev_done) cudaEventDestroy(ev_done);
     if (scratch) cudaFree(scratch);
@@ -259,8 +325,26 @@ struct LoopbackComm : Comm {
     scratch_bytes = bytes;
     return 0;
   }
+  // [collective] the ranks' staging regions are plain device pointers of one process
+  int setup_oneshot() {
+    const size_t cap = oneshot_cap(), rb = peer_ar_region_bytes(cap);
+    if (cudaMalloc(&region, rb) != cudaSuccess || cudaMemset(region, 0, rb) != cudaSuccess) return LIGER_ENOMEM;
+    cudaDeviceSynchronize();
+    std::vector<const void*> xs, ys;
+    std::vector<cudaEvent_t> es;
+    rendezvous(region, nullptr, nullptr, &xs, &ys, &es);
+    void* peers[8] = {};
+    for (int q = 0; q < world; ++q) peers[q] = const_cast<void*>(xs[q]);
+    par = new PeerAR();
+    return par->init(world, rank, cap, region, peers);
+  }
   int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
     if (!count) return 0;
+    if (oneshot && oneshot_eligible(count, dt, op, buf)) {
+      if (!par)
+        if (int rc = setup_oneshot()) return rc;
+      return par->allreduce_bf16(buf, count, st);
+    }
     const size_t bytes = count * dt_size(dt);
     if (int rc = ensure_scratch(bytes)) return rc;
     std::vector<const void*> xs, ys;
@@ -372,6 +456,7 @@ Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err) {
     auto* c = new LoopbackComm();
     c->world = world;
     c->rank = rank;
+    c->oneshot = oneshot_enabled(true);
     c->key.assign((const char*)uid, 48);
     {
       std::lock_guard<std::mutex> l(g_groups_mu);
@@ -413,6 +498,9 @@ Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err) {
   ncclUniqueId id;
   memcpy(&id, uid, sizeof(id));
   auto* c = new NcclComm();
+  c->world = world;
+  c->rank = rank;
+  c->oneshot = oneshot_enabled(false);   // IPC path: opt-in until measured on NVLink
   ncclResult_t r = nccl().CommInitRank(&c->comm, world, id, rank);
   if (r != ncclSuccess) {
     *err = std::string("ncclCommInitRank: ") + nccl().GetErrorString(r);

@@ -26,6 +26,22 @@ struct NcclApi {
 };
 NcclApi& nccl();
 
+// One-shot all-reduce over peer memory (peer_ar.cu): every rank's staging region
+// (peer_ar_region_bytes(cap) bytes, zeroed; [2 buffers][cap] + epoch flag) is
+// mapped by every rank; calls must be issued in the same order on all ranks.
+struct PeerAR {
+  int world = 1, rank = 0;
+  size_t cap = 0;
+  void* local = nullptr;      // this rank's region (owned by the backend)
+  void* peer[8] = {};         // every rank's region as seen from this rank (peer[rank] = local)
+  unsigned int* counter = nullptr;
+  uint64_t epoch = 0;
+  int init(int world, int rank, size_t cap, void* local_region, void* const* peer_regions);
+  int allreduce_bf16(void* buf, size_t count, cudaStream_t st);   // in place, sum in rank order
+  ~PeerAR();
+};
+size_t peer_ar_region_bytes(size_t cap);
+
 enum CommDType { CD_BF16, CD_F32, CD_I32 };
 enum CommOp { CO_SUM, CO_MAX };
 

@@ -145,3 +145,30 @@ def test_pipeline_baseline_equals_single_gpu(E, world):
     for a, b in zip(ref, toks):
         assert np.array_equal(a, b)
     assert st["comm_kernels"] > 0
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_oneshot_peer_allreduce_equals_rendezvous_reduction(E, world):
+    """The one-shot peer-memory all-reduce (csrc/peer_ar.cu: epoch flags, rank-ordered
+    fp32 sum) against the loopback backend's rendezvous reduction (same sum order):
+    identical tokens, with prefill all-reduces above the one-shot cap (NCCL-style
+    path) and decode ones below it, interleaved with decomposition."""
+    import os
+    cfg = get_config("tiny")
+    trace = make_trace(4, float("inf"), seed=5, batch_sizes=(1, 2, 3), prompt_range=(8, 40), n_decode=5,
+                       vocab=cfg.vocab)
+    res = {}
+    for flag in ("0", "1"):
+        os.environ["LIGER_ONESHOT_AR"] = flag
+        os.environ["LIGER_ONESHOT_MAX_KB"] = "16"   # tiny: decode messages one-shot, most prefill ones not
+        try:
+            res[flag] = serve_tp(E, cfg, world, trace, mode="interleaved", max_batch=4, max_seq=48, max_new=8,
+                                 max_inflight=3, decomp_factor=8, seed=2)
+        finally:
+            os.environ.pop("LIGER_ONESHOT_AR", None)
+            os.environ.pop("LIGER_ONESHOT_MAX_KB", None)
+    for r in range(world):
+        for a, b in zip(res["0"][r][0], res["1"][r][0]):
+            assert np.array_equal(a, b)
+        for a, b in zip(res["1"][0][0], res["1"][r][0]):   # every rank holds the same tokens
+            assert np.array_equal(a, b)
