@@ -184,7 +184,14 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-latency", action="store_true")
     ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--workload", default="mixed", choices=["mixed", "generative"],
+                    help="mixed: batches of 2/4/8 x prompt U[128,512] + n_new generated tokens (BASELINE.json "
+                         "configs[1]); generative: the paper's sampling-phase task (P:316, Fig. 11) -- batches of "
+                         "32 sequences at start length 16, one sampling iteration each (the 16-token conditioning "
+                         "pass that fills the KV cache is included in the step)")
     args = ap.parse_args()
+    if args.workload == "generative":
+        args.n_new = 2
     _redirect_stdout()
     if args.impl == "reference":
         return run_reference(args)
@@ -205,8 +212,10 @@ def main():
         obj = [LigerEngine.unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0, group=gloo)
         uid = obj[0]
-    eng = LigerEngine(cfg, world=world, rank=rank, nccl_uid=uid, mode=args.mode, max_batch=8, max_seq=512,
-                      max_new=args.n_new, max_inflight=args.inflight, decomp_factor=args.F,
+    gen = args.workload == "generative"
+    trace_kw = (dict(batch_sizes=(32,), prompt_range=(16, 16)) if gen else {})
+    eng = LigerEngine(cfg, world=world, rank=rank, nccl_uid=uid, mode=args.mode, max_batch=32 if gen else 8,
+                      max_seq=16 if gen else 512, max_new=args.n_new, max_inflight=args.inflight, decomp_factor=args.F,
                       contention_factor=args.cf, seed=args.seed)
     eng.profile([8, 64, 256, 512, 1024, 2048, 4096])
     # contention factor: measured GEMM || all-reduce slowdown (1-rank proxy at N=1)
@@ -225,7 +234,7 @@ def main():
         return float(t.item())
 
     trace = make_trace(args.warmup + args.steps, float("inf"), seed=args.seed, vocab=cfg.vocab,
-                       n_decode=args.n_new)
+                       n_decode=args.n_new, **trace_kw)
     warm, timed = trace[:args.warmup], trace[args.warmup:]
     seqs = sum(r["batch"] for r in timed)
     dev_tokens = [torch.from_numpy(r["tokens"]).cuda() for r in timed]
@@ -315,7 +324,7 @@ def main():
     if not args.no_latency:
         cap_batches = len(timed) / dev_s
         rate = 0.5 * cap_batches
-        tr = make_trace(len(timed), rate, seed=args.seed + 1, vocab=cfg.vocab, n_decode=args.n_new)
+        tr = make_trace(len(timed), rate, seed=args.seed + 1, vocab=cfg.vocab, n_decode=args.n_new, **trace_kw)
         barrier()
         t0 = time.monotonic()
         ids, arr = [], []
@@ -354,9 +363,12 @@ def main():
             "metric": METRIC, "value": round(value, 3), "unit": "req/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(1e3 * dev_s / len(timed), 3), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-            "config": {"workload": f"{cfg.name} random-init bf16, TP={world}, batches of 2/4/8 x prompt "
-                                   f"U[128,512], {args.n_new} generated tokens, all {len(timed)} batches offered "
-                                   f"at once (capacity)", "model": cfg.name, "tp": world,
+            "config": {"workload": (f"{cfg.name} random-init bf16, TP={world}, " +
+                                    (f"generative (P:316): batches of 32 x start length 16, one sampling "
+                                     f"iteration (+ the conditioning pass)" if gen else
+                                     f"batches of 2/4/8 x prompt U[128,512], {args.n_new} generated tokens") +
+                                    f", all {len(timed)} batches offered at once (capacity)"),
+                       "model": cfg.name, "tp": world,
                        "mode": args.mode, "max_inflight": args.inflight, "decomp_factor": args.F,
                        "contention_factor": args.cf if args.cf > 0 else cf_cal,
                        "contention_factor_calibrated": round(cf_cal, 4),
