@@ -184,6 +184,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-latency", action="store_true")
     ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--sync", default="hybrid", choices=["hybrid", "cpu_gpu", "inter_stream"],
+                    help="Algorithm 1 round synchronisation (§3.4 Fig. 8; ablation §4.5)")
     ap.add_argument("--workload", default="mixed", choices=["mixed", "generative"],
                     help="mixed: batches of 2/4/8 x prompt U[128,512] + n_new generated tokens (BASELINE.json "
                          "configs[1]); generative: the paper's sampling-phase task (P:316, Fig. 11) -- batches of "
@@ -216,7 +218,7 @@ def main():
     trace_kw = (dict(batch_sizes=(32,), prompt_range=(16, 16)) if gen else {})
     eng = LigerEngine(cfg, world=world, rank=rank, nccl_uid=uid, mode=args.mode, max_batch=32 if gen else 8,
                       max_seq=16 if gen else 512, max_new=args.n_new, max_inflight=args.inflight, decomp_factor=args.F,
-                      contention_factor=args.cf, seed=args.seed)
+                      contention_factor=args.cf, seed=args.seed, sync=args.sync)
     eng.profile([8, 64, 256, 512, 1024, 2048, 4096])
     # contention factor: measured GEMM || all-reduce slowdown (1-rank proxy at N=1)
     cf_cal, _ = eng.calibrate_cf([8, 256, 1024], set_cf=args.cf <= 0)
@@ -369,7 +371,7 @@ def main():
                                      f"batches of 2/4/8 x prompt U[128,512], {args.n_new} generated tokens") +
                                     f", all {len(timed)} batches offered at once (capacity)"),
                        "model": cfg.name, "tp": world,
-                       "mode": args.mode, "max_inflight": args.inflight, "decomp_factor": args.F,
+                       "mode": args.mode, "sync": args.sync, "max_inflight": args.inflight, "decomp_factor": args.F,
                        "contention_factor": args.cf if args.cf > 0 else cf_cal,
                        "contention_factor_calibrated": round(cf_cal, 4),
                        "sequences": seqs, "batches": len(timed),

@@ -54,6 +54,17 @@ extern "C" {
 
 #define LIGER_MODE_SERIAL 0      /* Intra-Op baseline: compute then all-reduce, in order */
 #define LIGER_MODE_INTERLEAVED 1 /* Liger: Algorithm 1 + hybrid sync               */
+/* Synchronisation of Algorithm 1 rounds (§3.4, Fig. 8; ablation §4.5):
+ * HYBRID      the host waits for E1 (recorded before the running round's last
+ *             primary kernel), then launches the next round's subsets -- comm
+ *             first -- gated on E2 (after that kernel) by inter-stream waits;
+ * CPU_GPU     the host waits until every kernel of the running round has
+ *             finished, then launches (launch latency exposed);
+ * INTER_STREAM no host wait: every round is launched ahead and ordered only by
+ *             the E2 inter-stream waits (the paper's "lag" variant). */
+#define LIGER_SYNC_HYBRID 0
+#define LIGER_SYNC_CPU_GPU 1
+#define LIGER_SYNC_INTER_STREAM 2
 #define LIGER_MODE_PIPELINE 2    /* Inter-Op baseline: rank r holds an equal stage of unsharded
                                     layers, activations / tokens travel by send/recv;
                                     generated tokens are reported by the last stage */
@@ -71,6 +82,7 @@ typedef struct {
   int32_t decomp_factor;    /* F (P:254, 8 in the paper); 1 => no decomposition               */
   float contention_factor;  /* cf scaling secondary durations; <= 0 => 1.0            */
   uint64_t seed;            /* seed of the counter-based weight generator (C0)       */
+  int32_t sync_mode;        /* LIGER_SYNC_* (interleaved mode; §3.4 Fig. 8, §4.5)    */
 } liger_cfg;
 
 typedef struct liger_ctx liger_ctx;
@@ -249,7 +261,11 @@ int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K,
 size_t liger_gemm_workspace_bytes(int M, int N, int K);
 /* The tiling plan liger_op_gemm uses for a GEMM of full size (M, N, K) (host
  * only; a function of (M, N, K), identical for every column slice):
- * out[5] = {token tile bn, m tiles, split-K chunk kc, splits, pipeline stages}. */
+ * out[7] = {token tile bn, m tiles, split-K chunk kc, splits, pipeline stages,
+ *           cluster, co-resident clusters} -- cluster > 1: the splits are reduced in-kernel across a
+ *           thread-block cluster of that many CTAs (DSMEM, decode M <= 64; needs
+ *           the device to size it, so a host without one reports 1); else a
+ *           split-K fixup kernel follows.  Both sum chunks in the same order. */
 int liger_gemm_plan(int M, int N, int K, int32_t* out);
 
 /* Fused residual add + LayerNorm (§8(a) a2/a7/a11; C2):

@@ -80,6 +80,7 @@ int liger_gemm_plan(int M, int N, int K, int32_t* out) {
   if (!out || M <= 0 || N <= 0 || K <= 0) return LIGER_EINVAL;
   GemmPlan pl = gemm_plan(M, N, K);
   out[0] = pl.bn; out[1] = pl.m_tiles; out[2] = pl.kc; out[3] = pl.splits; out[4] = pl.stages;
+  out[5] = pl.cluster; out[6] = pl.clusters;
   return LIGER_OK;
 }
 

@@ -159,6 +159,7 @@ struct liger_ctx {
   std::vector<std::unique_ptr<Batch>> all_batches;   // id -> batch
   int64_t next_id = 0;
   cudaEvent_t e1 = nullptr, e2 = nullptr;
+  cudaEvent_t e_end[2] = {nullptr, nullptr};   // CPU_GPU sync: end of the round on each stream
   bool have_round = false;
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_next = 0;
@@ -785,6 +786,8 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     c->l0 = 0;
     c->l1 = c->L;
   }
+  if (cfg->sync_mode < LIGER_SYNC_HYBRID || cfg->sync_mode > LIGER_SYNC_INTER_STREAM)
+    return fail(nullptr, LIGER_EINVAL, "liger_init: unknown sync_mode");
   c->F = std::max(1, cfg->decomp_factor);
   c->cf = cfg->contention_factor > 0 ? cfg->contention_factor : 1.0;
   if (const char* sk = getenv("LIGER_DBG_SKIP")) {
@@ -807,6 +810,8 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   CK(cudaStreamCreateWithPriority(&c->s_comm, cudaStreamNonBlocking, hi));
   CK(cudaEventCreateWithFlags(&c->e1, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&c->e2, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&c->e_end[0], cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&c->e_end[1], cudaEventDisableTiming));
 
   // weights (this rank's shards, K-major [N_local, K])
   c->layers.resize(c->L);
@@ -993,10 +998,17 @@ int64_t liger_submit(liger_ctx* c, int batch, int seq_len, const int32_t* tokens
 int liger_step(liger_ctx* c) {
   if (!c) return LIGER_EINVAL;
   const double t0 = now_s();
-  // hybrid synchronization: wait for E1 of the running round (CPU-GPU sync)
-  if (c->have_round) {
+  // hybrid synchronization: wait for E1 of the running round (CPU-GPU sync);
+  // the CPU_GPU ablation waits for the whole round, INTER_STREAM does not wait.
+  if (c->have_round && c->cfg.sync_mode != LIGER_SYNC_INTER_STREAM) {
     const double w0 = now_s();
-    while (cudaEventQuery(c->e1) == cudaErrorNotReady) {
+    if (c->cfg.sync_mode == LIGER_SYNC_CPU_GPU) {
+      for (int i = 0; i < 2; ++i)
+        while (cudaEventQuery(c->e_end[i]) == cudaErrorNotReady) {
+        }
+    } else {
+      while (cudaEventQuery(c->e1) == cudaErrorNotReady) {
+      }
     }
     c->st.wait_us += (now_s() - w0) * 1e6;
   }
@@ -1074,6 +1086,10 @@ int liger_step(liger_ctx* c) {
       CKR(launch_run(c, pieces, w1, s1));
     }
     c->have_round = !w0.empty();
+    if (c->cfg.sync_mode == LIGER_SYNC_CPU_GPU) {
+      cudaEventRecord(c->e_end[0], c->s_comp);
+      cudaEventRecord(c->e_end[1], c->s_comm);
+    }
     c->st.rounds++;
     if (!w1.empty()) c->st.overlapped_rounds++;
     n = (int)pieces.size();
@@ -1427,6 +1443,8 @@ int liger_finalize(liger_ctx* c) {
   for (auto& b : c->waiting) cudaEventDestroy(b->final_ev);
   cudaEventDestroy(c->e1);
   cudaEventDestroy(c->e2);
+  cudaEventDestroy(c->e_end[0]);
+  cudaEventDestroy(c->e_end[1]);
   cudaStreamDestroy(c->s_comp);
   cudaStreamDestroy(c->s_comm);
   gemm_forget_pointer_range(nullptr, ~size_t(0));

@@ -26,6 +26,7 @@
 #include <stdint.h>
 #include <stdio.h>
 #include <stdlib.h>
+#include <algorithm>
 #include <mutex>
 #include <unordered_map>
 #include <vector>
@@ -74,6 +75,7 @@ struct GemmParams {
   int* counters;
   const void* w_base;   // tiled weights (for the L2 prefetch)
   int pf_blocks;        // weight blocks (beyond the smem stages) prefetched into L2 before the PDL wait
+  int cluster;          // > 1: split-K reduced in-kernel across a (splits x 1 x 1) thread-block cluster
 };
 
 __device__ __forceinline__ float epi_apply(const GemmParams& p, float v, int n, float bias_v) {
@@ -124,6 +126,10 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   uint64_t* tmem_full = bars + 2 * S;       // [TS]
   uint64_t* tmem_empty = bars + 2 * S + 4;  // [TS]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 8);
+  uint64_t* red_full = bars + 2 * S + 9;    // [2] cluster split-K: all chunks' partials staged
+  uint64_t* red_empty = bars + 2 * S + 11;  // [2] cluster split-K: all CTAs done reading a stage
+  float* red0 = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 512);   // [2][bn][128] fp32
+  const bool cl = p.cluster > 1;
 
 
   const int warp = threadIdx.x >> 5;
@@ -142,6 +148,11 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       mbar_init(&tmem_full[i], 1);
       mbar_init(&tmem_empty[i], 4);   // one arrive per epilogue warp
     }
+    if (cl)
+      for (int i = 0; i < 2; ++i) {
+        mbar_init(&red_full[i], 4 * p.cluster);    // every epilogue warp of every CTA of the cluster
+        mbar_init(&red_empty[i], 4 * p.cluster);
+      }
     fence_barrier_init();
   }
   if (warp == 0 && lane == 0) {
@@ -152,6 +163,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
+  if (cl) cluster_sync_all();   // peers' barriers are initialised before any remote arrive
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp == 0) {
@@ -253,7 +265,9 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     // ---------------- epilogue: warps 2..5 own TMEM lane quarters (warp % 4)
     const int q = warp & 3;
     const int row = q * 32 + lane;
+    const int etid = threadIdx.x - 64;
     const int tiles = p.n_tiles * p.m_tiles;
+    const uint32_t crank = cl ? cluster_ctarank() : 0;   // == the unit's K chunk z
     int lu = 0;
     for (int u = blockIdx.x; u < p.units; u += G, ++lu) {
       const Unit w = unit_of(p, u);
@@ -266,7 +280,9 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       const int mcount = min(p.bn, p.M - m_base);
       const int tile_id = w.nt * p.m_tiles + w.mt;
       // fp32 partial of (chunk z, tile): [bn cols][128 rows] (a warp writes 128 B per column)
-      float* my_ws = p.splits > 1 ? p.ws + ((int64_t)w.z * tiles + tile_id) * (BM * p.bn) + row : nullptr;
+      float* my_ws = (p.splits > 1 && !cl) ? p.ws + ((int64_t)w.z * tiles + tile_id) * (BM * p.bn) + row : nullptr;
+      float* red = red0 + (lu & 1) * (BM * p.bn);
+      if (cl && lu >= 2) mbar_wait_cluster(&red_empty[lu & 1], ((lu >> 1) - 1) & 1);
       mbar_wait(&tmem_full[acc], acc_ph);
       tc_fence_after();
       const uint32_t tacc = tmem_base + (uint32_t)acc * acc_cols + ((uint32_t)(q * 32) << 16);
@@ -281,6 +297,10 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
             for (int j = 0; j < 16; ++j)
               if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, __uint_as_float(r[j]), n, bias_v));
           }
+        } else if (cl) {
+#pragma unroll
+          for (int j = 0; j < 16; ++j)
+            if (c0 + j < mcount) red[(c0 + j) * BM + row] = __uint_as_float(r[j]);
         } else {
 #pragma unroll
           for (int j = 0; j < 16; ++j)
@@ -291,6 +311,54 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tmem_empty[acc]);
+      if (cl) {
+        // In-cluster split-K reduction (replaces the fixup kernel): the S CTAs of the
+        // cluster hold chunks z = 0..S-1 of this tile in shared memory; CTA z sums
+        // slice z of the tile's elements over the S chunks in z order (the fixup's
+        // order: the same bits) through DSMEM and applies the epilogue.
+        if (lane == 0)
+          for (int r = 0; r < p.cluster; ++r) mbar_arrive_remote(&red_full[lu & 1], (uint32_t)r);
+        mbar_wait_cluster(&red_full[lu & 1], (lu >> 1) & 1);
+        const int E4 = mcount * (BM / 4);
+        const int lo = (int)((int64_t)E4 * crank / p.cluster), hi = (int)((int64_t)E4 * (crank + 1) / p.cluster);
+        const uint32_t red_local = smem_u32(red);
+        for (int e = lo + etid; e < hi; e += 128) {
+          const uint32_t off = red_local + (uint32_t)e * 16u;
+          float4 v[8];
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            if (i < p.cluster) v[i] = ld_dsmem_f4(dsmem_map(off, (uint32_t)i));
+          float4 a = v[0];
+#pragma unroll
+          for (int i = 1; i < 8; ++i)
+            if (i < p.cluster) {
+              a.x += v[i].x;
+              a.y += v[i].y;
+              a.z += v[i].z;
+              a.w += v[i].w;
+            }
+          const int col = e >> 5, rq = e & 31;
+          const float av[4] = {a.x, a.y, a.z, a.w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const int nn = n_base + rq * 4 + i;
+            if (nn < p.n1 && nn < p.N) {
+              const float bv = p.bias ? __bfloat162float(p.bias[nn]) : 0.0f;
+              epi_store(p, m_base + col, nn, epi_apply(p, av[i], nn, bv));
+            }
+          }
+        }
+        __syncwarp();
+        if (lane == 0)
+          for (int r = 0; r < p.cluster; ++r) mbar_arrive_remote(&red_empty[lu & 1], (uint32_t)r);
+      }
+    }
+    if (cl) {
+      // peers read this CTA's shared memory: stay resident until they are done
+      for (int buf = 0; buf < 2; ++buf) {
+        const int j = (((lu - 1) & 1) == buf) ? lu - 1 : lu - 2;   // last unit staged in buf
+        if (j >= 0) mbar_wait_cluster(&red_empty[buf], (j >> 1) & 1);
+      }
     }
   }
   tc_fence_before();
@@ -464,6 +532,72 @@ void gemm_forget_pointer_range(const void* base, size_t bytes) {
 // split reduction -- is a function of (M, N, K) and identical for the full GEMM
 // and all of its slices: slices are bit-exact.  The split count is chosen by a
 // small cost model that balances units over the SMs.
+// Pipeline stages for a token tile bn within a per-CTA shared-memory budget.
+static int stages_for(int bn, int extra_smem, int budget) {
+  const int stage_bytes = A_BYTES + bn * BK * 2;
+  int st = (budget - 1024 - 512 - extra_smem) / stage_bytes;
+  if (st > 12) st = 12;
+  static const int dec_cap = getenv("LIGER_GEMM_DECODE_STAGES") ? atoi(getenv("LIGER_GEMM_DECODE_STAGES")) : 6;
+  if (bn <= 32 && st > dec_cap) st = dec_cap;   // decode: 96 KiB of weights in flight suffices (measured)
+  if (const char* e = getenv("LIGER_GEMM_STAGES")) {   // experiments only
+    const int f = atoi(e);
+    if (f >= 2 && f < st) st = f;
+  }
+  return st;
+}
+
+static int cluster_red_bytes(int bn) { return 2 * BM * bn * (int)sizeof(float); }
+// Cluster (decode) mode runs two CTAs per SM: a CTA gets half of the SM's 228 KiB
+// minus the 1 KiB the hardware reserves per CTA.
+constexpr int CLUSTER_CTA_SMEM = 233472 / 2 - 1024;
+static int cluster_smem(int bn) {
+  const int red = cluster_red_bytes(bn);
+  return 1024 + stages_for(bn, red, CLUSTER_CTA_SMEM) * (A_BYTES + bn * BK * 2) + 512 + red;
+}
+
+// Co-resident (S x 1 x 1) clusters of gemm_tc_kernel in cluster (decode) mode
+// (clusters must fit inside a GPC; up to two CTAs per SM).
+static int max_clusters(int S, int bn) {
+  static std::mutex mu;
+  static std::unordered_map<int, int> cache;
+  const int key = S * 1024 + bn;
+  std::lock_guard<std::mutex> g(mu);
+  auto it = cache.find(key);
+  if (it != cache.end()) return it->second;
+  cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
+  cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(S * 128);
+  cfg.blockDim = dim3(GEMM_THREADS);
+  cfg.dynamicSmemBytes = cluster_smem(bn);
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = S;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, gemm_tc_kernel, &cfg) != cudaSuccess || n <= 0) {
+    cudaGetLastError();
+    n = 0;   // cluster mode unavailable for this S
+  }
+  cache[key] = n;
+  return n;
+}
+
+// Tiling policy.  A decomposition piece of a GEMM (a column slice [n0, n1)) keeps
+// the full GEMM's (M, N, K), so every per-element quantity -- the token tiling
+// bn, the split-K chunk kc, the K order inside a chunk and the z-order of the
+// split reduction -- is a function of (M, N, K) and identical for the full GEMM
+// and all of its slices: slices are bit-exact.  The split count is chosen by a
+// small cost model that balances the weight stream over the SMs.  Split chunks
+// are summed by the PDL-chained fixup kernel.  Opt-in (LIGER_GEMM_CLUSTER=1):
+// decode GEMMs (M <= 64) reduce their K chunks inside a thread-block cluster
+// (S <= 8 CTAs, DSMEM) instead -- the same z order, so the same bits.  Measured
+// slower (OPT-13B decode chain 130 vs 117 us/layer, pass 5.7-5.9 vs 5.4 ms):
+// with N/128 = 40 tiles a cluster of S CTAs per tile keeps only 40 S <= 148 SMs
+// streaming, and larger S leaves clusters waiting for whole free GPC slots.
 GemmPlan gemm_plan(int M, int N, int K) {
   GemmPlan pl{};
   const int G = num_sms();
@@ -474,53 +608,74 @@ GemmPlan gemm_plan(int M, int N, int K) {
   bn = (bn + 15) / 16 * 16;
   if (bn < 16) bn = 16;
   const int tiles = n_tiles * mt;
+  static const bool cluster_on = getenv("LIGER_GEMM_CLUSTER") && atoi(getenv("LIGER_GEMM_CLUSTER")) != 0;
+  const bool use_cluster = cluster_on && M <= 64;
   // Cost model in SM cycles: a k-block costs max(MMA = 8 bn, weight stream at
-  // ~23 B/clk/SM + activation tile from L2 at ~64 B/clk); a unit adds 300; a
-  // split adds the fixup kernel (launch + S*M*N*4 B of partial traffic x 2).
+  // ~23 B/clk/SM + activation tile from L2 at ~64 B/clk); a unit adds 300.
+  // Non-cluster: units spread over G persistent CTAs; a split adds the fixup
+  // kernel (launch + S*M*N*4 B of partial traffic x 2).  Cluster: waves of
+  // co-resident clusters, an SM holding two CTAs streams for both; each wave
+  // adds the DSMEM exchange.
   const double kb_time = fmax(8.0 * bn, A_BYTES / 23.0 + 128.0 * bn / 64.0);
-  int best_s = 1;
+  int best_s = 1, best_nc = 0;
   double best = 1e300;
   // Prefill GEMMs that already fill the SMs are not split (their fp32 partials
   // would exceed L2); decode GEMMs always consider it.
-  const int smax = (M > 64 && tiles >= G) ? 1 : (nkb >= 8 ? nkb / 4 : 1);
+  int smax = (M > 64 && tiles >= G) ? 1 : (nkb >= 8 ? nkb / 4 : 1);
+  if (use_cluster && smax > 8) smax = 8;
   for (int sp = 1; sp <= smax; ++sp) {
     const int kcb = (nkb + sp - 1) / sp;
     const int S = (nkb + kcb - 1) / kcb;
     if (S != sp) continue;
-    const double units = (double)tiles * S;
-    double cost = ceil(units / G) * (kcb * kb_time + 300.0);
-    if (S > 1) cost += 6000.0 + (double)S * M * N * 8.0 / 2600.0;   // fixup launch + partial traffic
+    double cost;
+    int nc = 0;
+    if (use_cluster && S > 1) {
+      nc = max_clusters(S, bn);
+      if (nc <= 0) continue;
+      if (nc > tiles) nc = tiles;
+      cost = 0.0;
+      for (int left = tiles; left > 0; left -= nc) {
+        const int ctas = std::min(left, nc) * S;
+        cost += (double)((ctas + G - 1) / G) * (kcb * kb_time + 300.0) + 1200.0;
+      }
+    } else {
+      const double units = (double)tiles * S;
+      cost = ceil(units / G) * (kcb * kb_time + 300.0);
+      if (S > 1) cost += 6000.0 + (double)S * M * N * 8.0 / 2600.0;   // fixup launch + partial traffic
+    }
     if (cost < best - 1e-9) {
       best = cost;
       best_s = S;
+      best_nc = nc;
     }
   }
   if (const char* e = getenv("LIGER_GEMM_FORCE_SPLITS")) {   // experiments only
     const int f = atoi(e);
-    if (f >= 1 && f <= nkb) best_s = f;
+    if (f >= 1 && f <= nkb && (!use_cluster || f <= 8)) {
+      best_s = f;
+      best_nc = (use_cluster && f > 1) ? std::min(max_clusters(f, bn), tiles) : 0;
+    }
   }
   const int kcb = (nkb + best_s - 1) / best_s;
   pl.bn = bn;
   pl.m_tiles = mt;
   pl.kc = kcb * BK;
   pl.splits = (nkb + kcb - 1) / kcb;
-  const int stage_bytes = A_BYTES + pl.bn * BK * 2;
-  int st = (MAX_SMEM - 1024 - 512) / stage_bytes;
-  if (st > 12) st = 12;
-  static const int dec_cap = getenv("LIGER_GEMM_DECODE_STAGES") ? atoi(getenv("LIGER_GEMM_DECODE_STAGES")) : 6;
-  if (pl.bn <= 32 && st > dec_cap) st = dec_cap;   // decode: 96 KiB of weights in flight suffices (measured)
-  if (const char* e = getenv("LIGER_GEMM_STAGES")) {   // experiments only
-    const int f = atoi(e);
-    if (f >= 2 && f < st) st = f;
+  pl.cluster = (use_cluster && pl.splits > 1 && best_nc > 0) ? pl.splits : 1;
+  pl.clusters = pl.cluster > 1 ? best_nc : 0;
+  if (pl.cluster > 1) {
+    pl.stages = stages_for(bn, cluster_red_bytes(bn), CLUSTER_CTA_SMEM);
+    pl.smem = cluster_smem(bn);
+  } else {
+    pl.stages = stages_for(bn, 0, MAX_SMEM);
+    pl.smem = 1024 + pl.stages * (A_BYTES + pl.bn * BK * 2) + 512;
   }
-  pl.stages = st;
-  pl.smem = 1024 + st * stage_bytes + 512;
   return pl;
 }
 
 size_t gemm_workspace_bytes(int M, int N, int K) {
   GemmPlan pl = gemm_plan(M, N, K);
-  if (pl.splits <= 1) return GEMM_COUNTER_BYTES;
+  if (pl.splits <= 1 || pl.cluster > 1) return GEMM_COUNTER_BYTES;
   const size_t tiles = (size_t)((N + BM - 1) / BM + 1) * pl.m_tiles;   // +1: unaligned slices
   return GEMM_COUNTER_BYTES + (size_t)pl.splits * tiles * BM * pl.bn * sizeof(float);
 }
@@ -530,7 +685,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (a.K <= 0 || a.K % 8 || a.ldx % 8 || (!a.w_tiled && a.ldw % 8) || a.n0 < 0 || a.n1 > a.N) return LIGER_EINVAL;
   GemmPlan pl = gemm_plan(a.M, a.N, a.K);
   const int ntiles = (a.n1 - a.n0 + BM - 1) / BM;
-  if (pl.splits > 1) {
+  if (pl.splits > 1 && pl.cluster <= 1) {
     if (!a.workspace) return LIGER_EINVAL;
     const size_t need = GEMM_COUNTER_BYTES + (size_t)pl.splits * ntiles * pl.m_tiles * BM * pl.bn * sizeof(float);
     if (a.ws_bytes < need) return LIGER_EINVAL;
@@ -550,6 +705,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   static bool attr_set = false;
   if (!attr_set) {
     cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
+    cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     attr_set = true;
   }
   GemmParams p;
@@ -569,11 +725,22 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.n_tiles = ntiles;
   p.m_tiles = pl.m_tiles;
   p.units = ntiles * pl.m_tiles * pl.splits;
-  const int grid = p.units < num_sms() ? p.units : num_sms();
-  int rc2 = launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
-  if (a.had_fixup) *a.had_fixup = p.splits > 1;
+  p.cluster = pl.cluster;
+  int rc2;
+  if (pl.cluster > 1) {
+    // one cluster of `splits` CTAs per tile in flight; CTA z of a cluster takes chunk z
+    // (grid = clusters x S, so unit u = blockIdx.x + j * grid keeps z = blockIdx.x % S)
+    const int nc = std::min(pl.clusters, ntiles * pl.m_tiles);
+    rc2 = launch_pdl_cluster(gemm_tc_kernel, dim3(nc * pl.cluster), dim3(GEMM_THREADS), pl.cluster, pl.smem, stream,
+                             tA, tB, p);
+  } else {
+    const int grid = p.units < num_sms() ? p.units : num_sms();
+    rc2 = launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
+  }
+  const bool fixup = p.splits > 1 && pl.cluster <= 1;
+  if (a.had_fixup) *a.had_fixup = fixup;
   if (a.ev_mid) cudaEventRecord(a.ev_mid, stream);
-  if (rc2 || p.splits == 1) return rc2 ? LIGER_ECUDA : 0;
+  if (rc2 || !fixup) return rc2 ? LIGER_ECUDA : 0;
   const int64_t work = (int64_t)p.M * (BM / 4) * p.n_tiles;
   int rblocks = (int)((work + 255) / 256);
   if (rblocks > num_sms() * 8) rblocks = num_sms() * 8;

@@ -13,6 +13,8 @@ constexpr size_t ATTN_COUNTER_BYTES = 16384;
 
 struct GemmPlan {
   int bn, m_tiles, kc, splits, stages, smem;
+  int cluster;    // > 1: splits reduced in-kernel over a (splits x 1 x 1) cluster (no fixup kernel)
+  int clusters;   // cluster mode: co-resident clusters the persistent grid uses
 };
 
 struct GemmArgs {

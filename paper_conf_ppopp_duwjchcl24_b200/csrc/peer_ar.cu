@@ -55,7 +55,11 @@ __global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf
                                                                       unsigned int* counter, PeerPtrs peers,
                                                                       int world, unsigned long long epoch) {
   const size_t stride = (size_t)gridDim.x * blockDim.x;
-  pdl_enter();   // the partials come from the preceding GEMM
+  // The partials come from the preceding GEMM.  Dependents are released only after
+  // every peer has arrived (below): a kernel parked at its griddepcontrol.wait
+  // must not hold SM resources while this one spins on other ranks -- on the
+  // loopback backend those ranks share this GPU and would need them to progress.
+  grid_dependency_wait();
   for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += stride) my_stage[i] = buf[i];
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -70,10 +74,11 @@ __global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf
     for (int q = 0; q < world; ++q)
       while (ld_acquire_sys(peers.flag[q]) < epoch) {
         __nanosleep(64);
-        if (trace_now() - t0 > 4000000000ull) __trap();   // a peer never arrived: fail, do not hang
+        if (trace_now() - t0 > 10000000000ull) __trap();   // a peer never arrived: fail, do not hang
       }
   }
   __syncthreads();
+  grid_dependency_trigger();
   for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += stride) {
     uint4 v[PAR_MAX_WORLD];
 #pragma unroll

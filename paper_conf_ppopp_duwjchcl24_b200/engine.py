@@ -14,7 +14,7 @@ from . import liger as L
 class LigerEngine:
     def __init__(self, model_cfg, *, world=1, rank=0, nccl_uid=None, mode="interleaved", max_batch=8,
                  max_seq=512, max_new=32, max_inflight=2, decomp_factor=8, contention_factor=1.0, seed=0,
-                 load=True):
+                 load=True, sync="hybrid"):
         lib = L.lib()
         cfg = L.liger_cfg()
         cfg.n_layers, cfg.hidden, cfg.n_heads = model_cfg.n_layers, model_cfg.hidden, model_cfg.n_heads
@@ -27,6 +27,7 @@ class LigerEngine:
         cfg.decomp_factor = decomp_factor
         cfg.contention_factor = contention_factor
         cfg.seed = seed
+        cfg.sync_mode = L.SYNC[sync]
         self.cfg = cfg
         self.model = model_cfg
         self.world, self.rank = world, rank

@@ -10,6 +10,7 @@ LIB_PATH = os.path.join(HERE, "libliger.so")
 
 LIGER_OK, LIGER_PENDING, LIGER_IDLE = 0, 1, 2
 ACT = {"none": 0, "relu": 1, "gelu_tanh": 2}
+SYNC = {"hybrid": 0, "cpu_gpu": 1, "inter_stream": 2}
 MODE = {"serial": 0, "interleaved": 1, "pipeline": 2}
 KV_BLOCK = 16
 KT_NAMES = ["gemm_decode", "attn", "ln", "allreduce", "gemm_prefill", "lm_head", "splitk_fixup",
@@ -27,7 +28,7 @@ class liger_cfg(C.Structure):
                 ("vocab", C.c_int32), ("max_pos", C.c_int32), ("act", C.c_int32), ("ln_eps", C.c_float),
                 ("max_batch", C.c_int32), ("max_seq", C.c_int32), ("max_new", C.c_int32), ("mode", C.c_int32),
                 ("max_inflight", C.c_int32), ("decomp_factor", C.c_int32), ("contention_factor", C.c_float),
-                ("seed", C.c_uint64)]
+                ("seed", C.c_uint64), ("sync_mode", C.c_int32)]
 
 
 class liger_result(C.Structure):
@@ -182,9 +183,9 @@ def gemm_workspace_bytes(M, N, K):
 
 
 def gemm_plan(M, N, K):
-    out = (C.c_int32 * 5)()
+    out = (C.c_int32 * 7)()
     check(lib().liger_gemm_plan(M, N, K, out), what="liger_gemm_plan")
-    return dict(zip(("bn", "m_tiles", "kc", "splits", "stages"), list(out)))
+    return dict(zip(("bn", "m_tiles", "kc", "splits", "stages", "cluster", "clusters"), list(out)))
 
 
 def add_layernorm(x, gamma, beta, y, *, add=None, add_bias=None, x_out=None, rows=None, in_row_step=1,

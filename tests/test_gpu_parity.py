@@ -305,3 +305,51 @@ def test_tp_layer_vs_oracle(L, name, t, b, s):
     for got, ref in ((out_pf, ref_pf.reshape(M, -1)), (out_dc, ref_dc.reshape(b, -1))):
         rel, mae = errs(to_np64(got), ref)
         assert rel <= REL and mae <= MAE, (rel, mae)
+
+
+_CLUSTER_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r})
+from liger_inputs import c0_values
+from paper_conf_ppopp_duwjchcl24_b200 import liger as L
+out = []
+for (M, N, K) in {shapes!r}:
+    x = torch.from_numpy(c0_values(4, 1, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K).astype(np.float32)).cuda().bfloat16()
+    w = torch.from_numpy(c0_values(4, 2, np.arange(N * K, dtype=np.uint64), -6).reshape(N, K).astype(np.float32)).cuda().bfloat16()
+    b = torch.from_numpy(c0_values(4, 3, np.arange(N, dtype=np.uint64), -4).astype(np.float32)).cuda().bfloat16()
+    ws = torch.zeros(max(L.gemm_workspace_bytes(M, N, K), 16384) // 4 + 16, dtype=torch.int32, device="cuda")
+    o = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
+    L.gemm(x, w, o, bias=b, act="relu", workspace=ws)
+    torch.cuda.synchronize()
+    out.append((L.gemm_plan(M, N, K), o.view(torch.int16).cpu().numpy().tobytes().hex()))
+print(repr(out))
+"""
+
+
+def test_gemm_cluster_splitk_equals_fixup_kernel(L):
+    """Opt-in (LIGER_GEMM_CLUSTER=1): decode GEMMs reduce their split-K chunks inside
+    a thread-block cluster over DSMEM; the default fixup-kernel path sums the same
+    chunks in the same order, so the two must agree bit for bit (and both meet the oracle,
+    test_gemm_vs_oracle).  Shapes: OPT-13B decode projections at b = 8 and ragged M."""
+    import ast
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    shapes = [(8, 5120, 5120), (8, 5120, 20480), (8, 20480, 5120), (3, 1000, 2560), (33, 640, 4096)]
+    code = _CLUSTER_CHILD.format(root=root, shapes=shapes)
+    res = {}
+    runs = (("default", {"LIGER_GEMM_CLUSTER": "1"}),
+            ("cluster4", {"LIGER_GEMM_FORCE_SPLITS": "4", "LIGER_GEMM_CLUSTER": "1"}),
+            ("fixup4", {"LIGER_GEMM_FORCE_SPLITS": "4", "LIGER_GEMM_CLUSTER": "0"}))
+    for tag, env in runs:
+        p = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env}, capture_output=True, text=True,
+                           timeout=300)
+        assert p.returncode == 0, p.stderr[-2000:]
+        res[tag] = ast.literal_eval(p.stdout.strip().splitlines()[-1])
+    assert any(pl["cluster"] > 1 for pl, _ in res["default"]), res["default"]
+    assert all(pl["cluster"] == 4 for pl, _ in res["cluster4"]), res["cluster4"]
+    assert all(pl["cluster"] == 1 and pl["splits"] == 4 for pl, _ in res["fixup4"])
+    for (pc, hc), (pf, hf), s in zip(res["cluster4"], res["fixup4"], shapes):
+        assert pc["kc"] == pf["kc"]
+        assert hc == hf, (s, pc, pf)

@@ -172,3 +172,22 @@ def test_oneshot_peer_allreduce_equals_rendezvous_reduction(E, world):
             assert np.array_equal(a, b)
         for a, b in zip(res["1"][0][0], res["1"][r][0]):   # every rank holds the same tokens
             assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("sync", ["cpu_gpu", "inter_stream"])
+def test_sync_ablation_modes_bit_exact(E, sync):
+    """§3.4 Fig. 8 / §4.5 ablation: the CPU-GPU-only and inter-stream-only
+    synchronisation variants change when rounds are launched, never what they
+    compute -- tokens bit-identical to the hybrid (default) schedule at TP = 2."""
+    cfg = get_config("tiny")
+    trace = make_trace(4, float("inf"), seed=21, batch_sizes=(1, 2, 3), prompt_range=(8, 40), n_decode=5,
+                       vocab=cfg.vocab)
+    kw = dict(mode="interleaved", max_batch=4, max_seq=48, max_new=8, max_inflight=3, decomp_factor=8, seed=6)
+    hyb = serve_tp(E, cfg, 2, trace, **kw)
+    alt = serve_tp(E, cfg, 2, trace, sync=sync, **kw)
+    for (th, _), (ta, st) in zip(hyb, alt):
+        for a, b in zip(th, ta):
+            assert np.array_equal(a, b)
+    assert alt[0][1]["overlapped_rounds"] > 0
+    if sync == "inter_stream":
+        assert alt[0][1]["wait_us"] == 0.0
