@@ -255,6 +255,20 @@ int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* 
 int liger_op_gemm_tiled(const void* x, int64_t ldx, const void* w_tiled, void* out, int64_t ldo, int M, int N,
                         int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
                         void* workspace, size_t ws_bytes, void* stream);
+/* Row-parallel projection fused with the following residual add + LayerNorm at
+ * t = 1 (§8(a) a5 -> a7 and a9 -> a11 when no all-reduce separates them):
+ *   P = x[M,K] . W[N,K]^T (split-K plan of (M, N, K), which must split),
+ *   x_res = bf16(x_res + bf16(P) + add_bias),  y = LN(x_res; gamma, beta, eps).
+ * The GEMM leaves its fp32 split-K partials in `workspace` and the add + LN kernel
+ * sums them itself, in the fixup kernel's order: bit-identical to
+ * liger_op_gemm_tiled (P into a bf16 buffer) followed by liger_op_add_layernorm,
+ * with one kernel and one hand-off fewer.  N = hidden (multiple of 128), W tiled as
+ * for liger_op_gemm_tiled; x_res/y [M, N] bf16, x_res updated in place; workspace
+ * of liger_gemm_workspace_bytes(M, N, K) bytes.  LIGER_EINVAL if the plan has no
+ * split (use the two calls). */
+int liger_op_gemm_tiled_add_layernorm(const void* x, const void* w_tiled, int M, int N, int K, void* x_res,
+                                      const void* add_bias, void* y, const void* gamma, const void* beta,
+                                      float eps, void* workspace, size_t ws_bytes, void* stream);
 /* Convert a row-major bf16 W [N, K] (row stride ld) to the tiled layout
  * (dst holds ceil(N/128)*128*K elements; padding rows are zero). */
 int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K, void* stream);

@@ -69,6 +69,26 @@ int liger_op_gemm_tiled(const void* x, int64_t ldx, const void* w, void* out, in
   return ret(gemm_launch(a, (cudaStream_t)stream), "liger_op_gemm_tiled");
 }
 
+int liger_op_gemm_tiled_add_layernorm(const void* x, const void* w_tiled, int M, int N, int K, void* x_res,
+                                      const void* add_bias, void* y, const void* gamma, const void* beta,
+                                      float eps, void* workspace, size_t ws_bytes, void* stream) {
+  if (int rc = check_device()) return rc;
+  if (!x_res || !y || !gamma || !beta || M <= 0) return ret(LIGER_EINVAL, "liger_op_gemm_tiled_add_layernorm");
+  const GemmPlan pl = gemm_plan(M, N, K);
+  if (pl.splits <= 1 || pl.cluster > 1) {   // no split-K: plain GEMM into a scratch-free path is not offered
+    set_global_error("liger_op_gemm_tiled_add_layernorm: (M, N, K) has no split-K plan");
+    return LIGER_EINVAL;
+  }
+  GemmArgs a{x, K, w_tiled, 64, nullptr, N, M, N, K, 0, N, nullptr, LIGER_ACT_NONE, 0, 1.0f, 0, workspace, ws_bytes, 1};
+  a.defer_fixup = true;
+  if (int rc = gemm_launch(a, (cudaStream_t)stream)) return ret(rc, "liger_op_gemm_tiled_add_layernorm");
+  const int64_t zstride = (int64_t)((N + 127) / 128) * pl.m_tiles * 128 * pl.bn;
+  return ret(splitk_add_layernorm_launch(reinterpret_cast<const float*>((char*)workspace + GEMM_COUNTER_BYTES),
+                                         zstride, pl.splits, pl.m_tiles, pl.bn, x_res, add_bias, x_res, y, gamma,
+                                         beta, M, N, eps, (cudaStream_t)stream),
+             "liger_op_gemm_tiled_add_layernorm");
+}
+
 int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K, void* stream) {
   if (int rc = check_device()) return rc;
   return ret(tile_weight_launch(w, ld, w_tiled, N, K, (cudaStream_t)stream), "liger_op_tile_weight");

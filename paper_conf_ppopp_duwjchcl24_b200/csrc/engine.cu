@@ -91,6 +91,10 @@ struct Slot {
   cudaEvent_t free_ev;     // completes when the last batch using the slot finished
   FusedDecodeState* fused = nullptr;   // fused decode pass tables of this slot
   Batch* owner = nullptr;  // batch currently (or last) assigned to the slot
+  // split-K partials of the last row-parallel GEMM left in gemm_ws for the next add + LN
+  bool split_pending = false;
+  GemmPlan split_plan{};
+  int split_N = 0;
 };
 
 struct DurTable {
@@ -170,6 +174,11 @@ struct liger_ctx {
   // decode passes at t = 1 as one fused kernel (LIGER_FUSED_DECODE=1).  Off by default:
   // measured 17-33 % slower than the per-kernel PDL chain.
   bool fused_decode = false;
+  // t = 1: split-K sum of out-proj / FC2 folded into the next add + LN (opt-in
+  // LIGER_FUSE_SPLITK_LN=1; bit-identical; measured neutral: OPT-13B decode pass
+  // 5527 vs 5433 us at b = 2, 5688 vs 5747 us at b = 8 -- one CTA per row reading
+  // S x h fp32 partials costs what the fixup kernel and its hand-off did)
+  bool fuse_split_ln = false;
   // stats / timing
   liger_stats_t st{};
   bool timing = false;
@@ -366,6 +375,18 @@ bool fused_pass(liger_ctx* c, int M) {
   return c->fused_decode && c->tp == 1 && fused_decode_supported(M, c->h, c->al, c->d, c->fl);
 }
 
+// add + LN over the split-K partials a deferred row-parallel GEMM left in gemm_ws
+static int split_add_ln(liger_ctx* c, Slot& S, const void* bias, const void* gamma, const void* beta, int M,
+                        cudaStream_t st) {
+  const GemmPlan& pl = S.split_plan;
+  const int n_tiles = (S.split_N + 127) / 128;
+  const int64_t zstride = (int64_t)n_tiles * pl.m_tiles * 128 * pl.bn;
+  S.split_pending = false;
+  return splitk_add_layernorm_launch(reinterpret_cast<const float*>((char*)S.gemm_ws + GEMM_COUNTER_BYTES), zstride,
+                                     pl.splits, pl.m_tiles, pl.bn, S.x, bias, S.x, S.y, gamma, beta, M, c->h,
+                                     c->cfg.ln_eps, st);
+}
+
 int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cudaStream_t st) {
   const PassOp po = c->pass_ops[pidx];
   Slot& S = c->slots[bt->slot];
@@ -424,6 +445,8 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       timed_begin(c, st, &ta);
       if (li == c->l0)   // first layer of the model / of this pipeline stage: x is complete
         rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
+      else if (S.split_pending)
+        rc = split_add_ln(c, S, c->layers[li - 1].b_2, W->g1, W->be1, M, st);
       else
         rc = add_layernorm_launch(S.x, S.part, c->layers[li - 1].b_2, S.x, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
       timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * (li == c->l0 ? 2 : 4), 0);
@@ -432,7 +455,10 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
     }
     case OP_LN2: {
       timed_begin(c, st, &ta);
-      rc = add_layernorm_launch(S.x, S.part, W->b_o, S.x, S.y, W->g2, W->be2, M, h, 1, 0, eps, st);
+      if (S.split_pending)
+        rc = split_add_ln(c, S, W->b_o, W->g2, W->be2, M, st);
+      else
+        rc = add_layernorm_launch(S.x, S.part, W->b_o, S.x, S.y, W->g2, W->be2, M, h, 1, 0, eps, st);
       timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * 4, 0);
       c->st.gpu_launches++;
       break;
@@ -460,6 +486,19 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
         g.act = c->cfg.act;
       } else {
         g.x = S.hbuf; g.ldx = c->fl; g.w = W->w_2; g.ldw = K; g.out = S.part; g.ldo = h;
+      }
+      // t = 1 (no all-reduce follows): leave the split-K partials of out-proj and of
+      // FC2 (not the last layer's, which feeds the LM head / the next stage) to the
+      // next add + LN, which sums them itself (bit-identical, one kernel fewer)
+      if (c->tp == 1 && c->fuse_split_ln && u0 == 0 && u1 == F &&
+          (po.op == OP_OUT || (po.op == OP_FC2 && li + 1 < c->l1))) {
+        const GemmPlan pl = gemm_plan(M, N, K);
+        if (pl.splits > 1 && pl.cluster <= 1) {
+          g.defer_fixup = true;
+          S.split_pending = true;
+          S.split_plan = pl;
+          S.split_N = N;
+        }
       }
       timed_begin(c, st, &ta);
       cudaEvent_t tmid = timed_mid(c);
@@ -796,6 +835,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
       if (all.find(std::string(",") + kOpName[o] + ",") != std::string::npos) c->dbg_skip |= 1u << o;
   }
   if (const char* fd = getenv("LIGER_FUSED_DECODE")) c->fused_decode = atoi(fd) != 0;
+  if (const char* fs = getenv("LIGER_FUSE_SPLITK_LN")) c->fuse_split_ln = atoi(fs) != 0;
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (tp > 2);
   if (world > 1) {

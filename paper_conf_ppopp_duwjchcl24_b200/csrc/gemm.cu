@@ -737,7 +737,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
     const int grid = p.units < num_sms() ? p.units : num_sms();
     rc2 = launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
   }
-  const bool fixup = p.splits > 1 && pl.cluster <= 1;
+  const bool fixup = p.splits > 1 && pl.cluster <= 1 && !a.defer_fixup;
   if (a.had_fixup) *a.had_fixup = fixup;
   if (a.ev_mid) cudaEventRecord(a.ev_mid, stream);
   if (rc2 || !fixup) return rc2 ? LIGER_ECUDA : 0;

@@ -37,6 +37,9 @@ struct GemmArgs {
   // (per-kernel timing; breaks the PDL overlap of the two)
   cudaEvent_t ev_mid = nullptr;
   bool* had_fixup = nullptr;
+  // split-K partials are left in the workspace for a following
+  // splitk_add_layernorm_launch instead of being summed by the fixup kernel
+  bool defer_fixup = false;
 };
 
 GemmPlan gemm_plan(int M, int N, int K);
@@ -78,6 +81,11 @@ void fused_decode_free(FusedDecodeState* state);
 int add_layernorm_launch(const void* x, const void* add, const void* add_bias, void* x_out, void* y,
                          const void* gamma, const void* beta, int rows, int h, int in_row_step, int in_row_off,
                          float eps, cudaStream_t stream);
+// add + LN whose added operand is the split-K sum of the preceding row-parallel GEMM
+// (launched with defer_fixup); bit-identical to splitk fixup -> add_layernorm_launch.
+int splitk_add_layernorm_launch(const float* ws, int64_t zstride, int splits, int m_tiles, int bn, const void* x,
+                                const void* add_bias, void* x_out, void* y, const void* gamma, const void* beta,
+                                int rows, int h, float eps, cudaStream_t stream);
 int embed_launch(const int32_t* ids, const void* e_tok, const void* e_pos, void* out, int rows, int h, int seq_len,
                  int start_pos, cudaStream_t stream);
 int argmax_launch(const float* logits, int64_t ld, int rows, int n, int idx_offset, float* max_out,

@@ -84,6 +84,7 @@ _SIGS = {
     "liger_op_gemm": (_I, [_P, _I64, _P, _I64, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),
     "liger_op_gemm_tiled": (_I, [_P, _I64, _P, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),
     "liger_op_tile_weight": (_I, [_P, _I64, _P, _I, _I, _P]),
+    "liger_op_gemm_tiled_add_layernorm": (_I, [_P, _P, _I, _I, _I, _P, _P, _P, _P, _P, _F, _P, _SZ, _P]),
     "liger_gemm_workspace_bytes": (_SZ, [_I, _I, _I]),
     "liger_gemm_plan": (_I, [_I, _I, _I, _P]),
     "liger_op_add_layernorm": (_I, [_P, _P, _P, _P, _P, _P, _P, _I, _I, _I, _I, _F, _P]),
@@ -167,6 +168,16 @@ def gemm_tiled(x, w_tiled, out, *, N, n0=0, n1=None, bias=None, act="none", scal
     check(lib().liger_op_gemm_tiled(_p(x), x.stride(0), _p(w_tiled), _p(out), out.stride(0), M, N, K, n0, n1,
                                     _p(bias), ACT[act], scale_cols, scale, out_f32, _p(workspace), ws_b,
                                     _s(stream)), what="liger_op_gemm_tiled")
+
+
+def gemm_tiled_add_layernorm(x, w_tiled, x_res, y, gamma, beta, *, N, add_bias=None, eps=1e-5, workspace=None,
+                             stream=None):
+    """Row-parallel projection + residual add + LayerNorm in two kernels (t = 1)."""
+    M, K = x.shape
+    ws_b = workspace.numel() * workspace.element_size() if workspace is not None else 0
+    check(lib().liger_op_gemm_tiled_add_layernorm(_p(x), _p(w_tiled), M, N, K, _p(x_res), _p(add_bias), _p(y),
+                                                  _p(gamma), _p(beta), eps, _p(workspace), ws_b, _s(stream)),
+          what="liger_op_gemm_tiled_add_layernorm")
 
 
 def tile_weight(w, w_tiled, stream=None):

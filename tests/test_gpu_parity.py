@@ -353,3 +353,92 @@ def test_gemm_cluster_splitk_equals_fixup_kernel(L):
     for (pc, hc), (pf, hf), s in zip(res["cluster4"], res["fixup4"], shapes):
         assert pc["kc"] == pf["kc"]
         assert hc == hf, (s, pc, pf)
+
+
+@pytest.mark.parametrize("M,N,K", [(2, 5120, 5120), (8, 5120, 20480), (5, 1024, 4096), (33, 9216, 1152)])
+def test_gemm_add_layernorm_fused_bit_exact(L, M, N, K):
+    """t = 1: the row-parallel projection's split-K partials summed inside the add + LN
+    kernel (liger_op_gemm_tiled_add_layernorm) equal the GEMM -> fixup -> add + LN
+    sequence bit for bit, and the oracle (P = x W^T, x1 = x_res + P + b, LN) within
+    the BASELINE.json tolerance.  Shapes: OPT-13B out-proj / FC2 at b = 2 / 8, a
+    small ragged case, OPT-66B TP = 8 out-proj shape at M = 33."""
+    if L.gemm_plan(M, N, K)["splits"] < 2:
+        pytest.skip("no split-K plan at this shape")
+    x = c0_values(6, 1, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K)
+    w = c0_values(6, 2, np.arange(N * K, dtype=np.uint64), -6).reshape(N, K)
+    xr = c0_values(6, 3, np.arange(M * N, dtype=np.uint64), -2).reshape(M, N)
+    b = c0_values(6, 4, np.arange(N, dtype=np.uint64), -5)
+    g = 1 + c0_values(6, 5, np.arange(N, dtype=np.uint64), -4)
+    be = c0_values(6, 6, np.arange(N, dtype=np.uint64), -4)
+    wt = torch.empty(L.tiled_numel(N, K), dtype=torch.bfloat16, device="cuda")
+    L.tile_weight(bf16_dev(w), wt)
+    xd, bd, gd, bed = bf16_dev(x), bf16_dev(b), bf16_dev(g), bf16_dev(be)
+    ws = workspace(L.gemm_workspace_bytes(M, N, K))
+    # unfused: GEMM (with its fixup) into P, then add + LN
+    p = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
+    L.gemm_tiled(xd, wt, p, N=N, workspace=ws)
+    x1 = bf16_dev(xr)
+    y1 = torch.empty_like(x1)
+    L.add_layernorm(x1, gd, bed, y1, add=p, add_bias=bd, x_out=x1)
+    # fused
+    x2 = bf16_dev(xr)
+    y2 = torch.empty_like(x2)
+    L.gemm_tiled_add_layernorm(xd, wt, x2, y2, gd, bed, N=N, add_bias=bd, workspace=ws)
+    torch.cuda.synchronize()
+    assert torch.equal(x1.view(torch.int16), x2.view(torch.int16))
+    assert torch.equal(y1.view(torch.int16), y2.view(torch.int16))
+    ref_x = xr.astype(np.float64) + x.astype(np.float64) @ w.astype(np.float64).T + b
+    assert errs(to_np64(x2), ref_x)[0] <= REL
+    ref_y = om.layer_norm(to_np64(x2), g.astype(np.float64), be, 1e-5)
+    rel, mae = errs(to_np64(y2), ref_y)
+    assert rel <= REL and mae <= 1e-2
+
+
+_FUSE_CHILD = r"""
+import sys, numpy as np
+sys.path.insert(0, {root!r})
+from liger_inputs import make_trace
+from liger_inputs.configs import ModelConfig
+from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
+cfg = ModelConfig("mid3", 3, 1024, 8, 4096, 1024, 96, "relu")
+trace = make_trace(3, float("inf"), seed=4, batch_sizes=(2, 5), prompt_range=(20, 60), n_decode=6, vocab=cfg.vocab)
+eng = LigerEngine(cfg, mode="interleaved", max_batch=8, max_seq=64, max_new=8, seed=7)
+ids = [eng.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], 0.0) for t in trace]
+eng.drain()
+print(repr([eng.poll(i, want_tokens=True)[1].tolist() for i in ids]))
+eng.close()
+"""
+
+
+def test_engine_split_ln_fusion_bit_exact_and_oracle(L):
+    """Engine at t = 1 on a config whose decode projections split K (h = 1024,
+    ffn 4096, d = 128): LIGER_FUSE_SPLITK_LN=1 (out-proj / FC2 partials summed inside
+    the next add + LN) and the default fixup-kernel path give identical tokens,
+    equal to the fp64 oracle's greedy tokens where its top-2 margin is clear."""
+    import ast
+    import os
+    import subprocess
+    import sys
+    from liger_inputs.configs import ModelConfig
+    from liger_inputs import make_trace
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    assert L.gemm_plan(2, 1024, 4096)["splits"] > 1 and L.gemm_plan(5, 1024, 1024)["splits"] > 1
+    res = {}
+    for flag in ("1", "0"):
+        p = subprocess.run([sys.executable, "-c", _FUSE_CHILD.format(root=root)],
+                           env={**os.environ, "LIGER_FUSE_SPLITK_LN": flag}, capture_output=True, text=True,
+                           timeout=600)
+        assert p.returncode == 0, p.stderr[-2000:]
+        res[flag] = ast.literal_eval(p.stdout.strip().splitlines()[-1])
+    assert res["1"] == res["0"]
+    cfg = ModelConfig("mid3", 3, 1024, 8, 4096, 1024, 96, "relu")
+    trace = make_trace(3, float("inf"), seed=4, batch_sizes=(2, 5), prompt_range=(20, 60), n_decode=6,
+                       vocab=cfg.vocab)
+    t = trace[0]
+    pr = t["tokens"].reshape(t["batch"], t["seq_len"])
+    ref, logits = om.greedy_generate(cfg, 7, pr, t["n_decode"], return_logits=True)
+    ok = om.top2_margin(logits) > 0.02 * np.sqrt((logits ** 2).mean())
+    got = np.array(res["1"][0])
+    for i in range(t["batch"]):
+        n = int(np.argmin(ok[i])) if not ok[i].all() else t["n_decode"]
+        assert np.array_equal(got[i, :n], ref[i, :n])
