@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "attn_decode.cuh"
 #include "common.cuh"
@@ -351,7 +352,9 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
                        int pos, int heads, int d, void* workspace, size_t ws_bytes, cudaStream_t stream) {
   if (b <= 0) return 0;
   const int ctx = pos + 1;
-  const int CH = dec_attn_chunk(b, heads, ctx);
+  int CH = dec_attn_chunk(b, heads, ctx);
+  static const int ch_env = getenv("LIGER_ATTN_CHUNK") ? atoi(getenv("LIGER_ATTN_CHUNK")) : 0;   // experiments
+  if ((ch_env == 32 || ch_env == 64 || ch_env == 128) && (ctx + ch_env - 1) / ch_env <= DC_MAX_SPLITS) CH = ch_env;
   const int ns = (ctx + CH - 1) / CH;
   if (ns > DC_MAX_SPLITS) return LIGER_EINVAL;   // context longer than 4096 positions
   if (ns > 1) {
@@ -371,9 +374,11 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   a.ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
   int rc;
   if (d == 128)
-    rc = CH == 32 ? launch_decode<128, 32>(a, b, stream) : launch_decode<128, 64>(a, b, stream);
+    rc = CH == 32 ? launch_decode<128, 32>(a, b, stream)
+                  : CH == 64 ? launch_decode<128, 64>(a, b, stream) : launch_decode<128, 128>(a, b, stream);
   else if (d == 64)
-    rc = CH == 32 ? launch_decode<64, 32>(a, b, stream) : launch_decode<64, 64>(a, b, stream);
+    rc = CH == 32 ? launch_decode<64, 32>(a, b, stream)
+                  : CH == 64 ? launch_decode<64, 64>(a, b, stream) : launch_decode<64, 128>(a, b, stream);
   else
     return LIGER_EINVAL;
   return rc ? LIGER_ECUDA : 0;

@@ -35,9 +35,11 @@ __host__ __device__ __forceinline__ int64_t kv_off(int page, int kv, int heads, 
 }
 
 // Chunk length for a decode step of b sequences x heads at context ctx: 32-position
-// chunks when 64-position ones would leave the SMs without ~6 items each.
+// chunks only when 64-position ones would leave the SMs with fewer than ~2.5 items
+// each (tools/kbench_attn.py, profiles/r01/attn_chunk_sweep.txt: 64 wins at b = 4,
+// ctx 300 (9.8 vs 13.5 us) and b = 2, ctx 300 (7.8 vs 8.8); 32 at b = 2, ctx 160).
 inline int dec_attn_chunk(int b, int heads, int ctx) {
-  const bool small = (size_t)b * heads * ((ctx + 63) / 64) < (size_t)148 * 6;
+  const bool small = (size_t)b * heads * ((ctx + 63) / 64) * 2 < (size_t)148 * 5;
   return (small && (ctx + 31) / 32 <= DC_MAX_SPLITS) ? 32 : 64;
 }
 

@@ -171,6 +171,7 @@ struct liger_ctx {
   double attn_scale[2] = {1.0, 1.0};   // calibration of the attention duration model (prefill, decode)
   uint32_t dbg_skip = 0;               // LIGER_DBG_SKIP=op,op,...: timing experiments only (wrong results)
   bool ar_atomic_chunks = false;
+  size_t ar_decomp_min_bytes = 1 << 20;   // all-reduces below this are not decomposed
   // decode passes at t = 1 as one fused kernel (LIGER_FUSED_DECODE=1).  Off by default:
   // measured 17-33 % slower than the per-kernel PDL chain.
   bool fused_decode = false;
@@ -233,11 +234,34 @@ cudaEvent_t pool_event(liger_ctx* c) {
 }
 
 // ------------------------------------------------------------------ geometry helpers
-int op_units(liger_ctx* c, int op) {
-  // decomposition exists to fill a communication window; at t = 1 there is none
+// Units (1/F pieces) an op of a pass with M tokens splits into.  Decomposition
+// exists to fill a communication window; at t = 1 there is none.  An
+// all-reduce is a "giant kernel" worth splitting only when its message is
+// large: decode-size messages (< ar_decomp_min_bytes) are latency-bound and stay
+// whole -- a function of M only, identical on every rank and in every mode.
+int op_units(liger_ctx* c, int op, int M) {
   if (c->F <= 1 || c->tp == 1) return 1;
-  if (op_is_gemm(op) || (op_is_ar(op) && c->tp > 1)) return c->F;
+  if (op_is_gemm(op)) return c->F;
+  if (op_is_ar(op)) return (M >= 0 && (size_t)M * c->h * 2 < c->ar_decomp_min_bytes) ? 1 : c->F;
   return 1;
+}
+
+// All-reduce of units [u0, u1) of F of the bf16 buffer buf[E].  With atomic chunks
+// (t > 2 over NCCL, whose reduction order depends on the message), every unit is
+// its own collective, so a piece of k units and the whole all-reduce produce the
+// same bits (R9).
+int issue_ar(liger_ctx* c, void* buf, size_t E, int u0, int u1, int F, cudaStream_t st) {
+  if (c->ar_atomic_chunks && F > 1) {
+    for (int u = u0; u < u1; ++u) {
+      const size_t e0 = E * u / F, e1 = E * (u + 1) / F;
+      if (e1 > e0)
+        if (c->comm->allreduce((char*)buf + e0 * 2, e1 - e0, CD_BF16, CO_SUM, st)) return LIGER_ENCCL;
+    }
+    return 0;
+  }
+  const size_t e0 = E * u0 / F, e1 = E * u1 / F;
+  if (e1 > e0 && c->comm->allreduce((char*)buf + e0 * 2, e1 - e0, CD_BF16, CO_SUM, st)) return LIGER_ENCCL;
+  return 0;
 }
 
 int gemm_N(liger_ctx* c, int op) {
@@ -272,7 +296,7 @@ int batch_M(const Batch* bt, int pass) { return pass == 0 ? bt->b * bt->s : bt->
 // ------------------------------------------------------------------ durations
 double model_dur(liger_ctx* c, int op, int M, int k, int ctx_len, int s_len) {
   const double F = c->F > 1 ? c->F : 1;
-  const double frac = (op_units(c, op) > 1) ? k / F : 1.0;
+  const double frac = (op_units(c, op, M) > 1) ? k / F : 1.0;
   const double bw = 5.0e12, tc = 1.0e15;
   if (op_is_gemm(op)) {
     const double N = gemm_N(c, op) * frac, K = gemm_K(c, op);
@@ -324,7 +348,7 @@ double op_dur(liger_ctx* c, const Batch* bt, int pass, int op, int k) {
     const double m = model_dur(c, op, M, k, ctx_len, s_len);
     return m * (s_len > 0 ? c->attn_scale[0] : c->attn_scale[1]);
   }
-  const int kk = op_units(c, op) > 1 ? k : std::max(1, c->F);
+  const int kk = op_units(c, op, M) > 1 ? k : std::max(1, c->F);
   const double t = table_dur(c, op, M, kk);
   return t > 0 ? t : model_dur(c, op, M, k, ctx_len, s_len);
 }
@@ -468,7 +492,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
     case OP_FC1:
     case OP_FC2: {
       const int N = gemm_N(c, po.op), K = gemm_K(c, po.op);
-      const int F = op_units(c, po.op);
+      const int F = op_units(c, po.op, M);
       GemmArgs g{};
       g.M = M; g.N = N; g.K = K;
       g.n0 = unit_col(N, u0, F);
@@ -538,15 +562,11 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
     }
     case OP_AR1:
     case OP_AR2: {
-      const int F = op_units(c, po.op);
+      const int F = op_units(c, po.op, M);
       const size_t E = (size_t)M * h;
-      const size_t e0 = E * u0 / F, e1 = E * u1 / F;
       timed_begin(c, st, &ta);
-      if (e1 > e0) {
-        if (c->comm->allreduce((char*)S.part + e0 * 2, e1 - e0, CD_BF16, CO_SUM, st))
-          return fail(c, LIGER_ENCCL, c->comm->err);
-      }
-      timed_end(c, st, ta, LIGER_KT_ALLREDUCE, (double)(e1 - e0) * 2, 0);
+      if (issue_ar(c, S.part, E, u0, u1, F, st)) return fail(c, LIGER_ENCCL, c->comm->err);
+      timed_end(c, st, ta, LIGER_KT_ALLREDUCE, (double)(E * u1 / F - E * u0 / F) * 2, 0);
       c->st.comm_kernels++;
       c->st.gpu_launches++;
       break;
@@ -637,8 +657,9 @@ struct BatchCursor : Cursor {
   bool empty() const override { return bt->all_launched; }
   int cur_op() const { return c->pass_ops[bt->idx].op; }
   int head_type() const override { return op_is_comm(cur_op()) ? KT_COMM : KT_COMPUTE; }
-  int head_left() const override { return op_units(c, cur_op()) - bt->done; }
-  bool head_decomposable() const override { return op_units(c, cur_op()) > 1; }
+  int units() const { return op_units(c, cur_op(), batch_M(bt, bt->pass)); }
+  int head_left() const override { return units() - bt->done; }
+  bool head_decomposable() const override { return units() > 1; }
   double head_dur(int k) const override {
     // duration of units [done, done + k): profiled piece of k units
     return op_dur(c, bt, bt->pass, cur_op(), k);
@@ -656,7 +677,7 @@ struct BatchCursor : Cursor {
     Piece p{bt, bt->pass, bt->idx, bt->done, bt->done + k};
     out->push_back(p);
     bt->done += k;
-    if (bt->done >= op_units(c, cur_op())) {
+    if (bt->done >= units()) {
       bt->done = 0;
       if (++bt->idx >= (int)c->pass_ops.size()) {
         bt->idx = 0;
@@ -762,7 +783,7 @@ int launch_run(liger_ctx* c, const std::vector<Piece>& pieces, const std::vector
     int rc = launch_piece(c, bt, p.pass, p.idx, p.u0, p.u1, st);
     if (rc < 0) return rc;
     c->st.kernels++;
-    const int units = op_units(c, c->pass_ops[p.idx].op);
+    const int units = op_units(c, c->pass_ops[p.idx].op, batch_M(bt, p.pass));
     if (p.u1 - p.u0 < units) c->st.split_pieces++;
     const bool batch_changes = (j + 1 == which.size()) || pieces[which[j + 1]].bt != bt;
     if (batch_changes) {
@@ -838,6 +859,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   if (const char* fs = getenv("LIGER_FUSE_SPLITK_LN")) c->fuse_split_ln = atoi(fs) != 0;
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (tp > 2);
+  if (const char* e = getenv("LIGER_AR_DECOMP_MIN_KB")) c->ar_decomp_min_bytes = (size_t)atoll(e) * 1024;
   if (world > 1) {
     if (!nccl_uid) return fail(nullptr, LIGER_EINVAL, "liger_init: nccl_uid required for world > 1");
     std::string err;
@@ -1280,7 +1302,7 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
       int pidx = 0;
       while (c->pass_ops[pidx].op != op) ++pidx;
       const size_t elems = (size_t)M * c->h;
-      auto gemm = [&] { launch_piece(c, &fake, 0, pidx, 0, op_units(c, op), c->s_comp); };
+      auto gemm = [&] { launch_piece(c, &fake, 0, pidx, 0, op_units(c, op, M), c->s_comp); };
       float tg = 1e30f, ta = 1e30f, tgc = 1e30f, tac = 1e30f;
       for (int rep = 0; rep < 4; ++rep) {
         float x;
@@ -1373,7 +1395,7 @@ int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
     for (int op : {OP_QKV, OP_OUT, OP_FC1, OP_FC2}) {
       int pidx = 0;
       while (c->pass_ops[pidx].op != op) ++pidx;
-      const int units = op_units(c, op);
+      const int units = op_units(c, op, M);
       for (int k = 1; k <= units; ++k) {
         const int kk = units > 1 ? k : F;
         const double t = time_it([&] { launch_piece(c, &fake, 0, pidx, 0, k, st); });
@@ -1390,11 +1412,10 @@ int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
     liger_set_duration(c, OP_EMBED, M, F, tln * 1e6);
     if (c->tp > 1) {
       const size_t E = (size_t)M * c->h;
-      for (int k = 1; k <= op_units(c, OP_AR1); ++k) {
-        const int kk = op_units(c, OP_AR1) > 1 ? k : F;
-        const double t = time_it([&] {
-          c->comm->allreduce(S.part, E * k / op_units(c, OP_AR1), CD_BF16, CO_SUM, st);
-        });
+      const int ua = op_units(c, OP_AR1, M);
+      for (int k = 1; k <= ua; ++k) {
+        const int kk = ua > 1 ? k : F;
+        const double t = time_it([&] { issue_ar(c, S.part, E, 0, k, ua, st); });
         liger_set_duration(c, OP_AR1, M, kk, t * 1e6);
         liger_set_duration(c, OP_AR2, M, kk, t * 1e6);
       }

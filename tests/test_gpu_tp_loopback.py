@@ -76,12 +76,19 @@ def test_interleaved_equals_serial_bit_exact(E, world):
     """Several batches in flight: Algorithm 1 interleaves one batch's all-reduces
     with another's GEMMs (secondary subsets, decomposition pieces); the tokens
     must be bit-identical to serial intra-op TP and to every rank's."""
+    import os
     cfg = get_config("tiny")
     trace = make_trace(5, float("inf"), seed=11, batch_sizes=(1, 2, 3), prompt_range=(8, 40), n_decode=6,
                        vocab=cfg.vocab)
-    base = serve_tp(E, cfg, world, trace, mode="serial", max_batch=4, max_seq=64, max_new=8, seed=3)
-    inter = serve_tp(E, cfg, world, trace, mode="interleaved", max_batch=4, max_seq=64, max_new=8, max_inflight=3,
-                     decomp_factor=8, contention_factor=1.0, seed=3)
+    # tiny messages: let every all-reduce be decomposable (and, at t > 2, issued as
+    # atomic 1/F chunks) so the pieces path is exercised
+    os.environ["LIGER_AR_DECOMP_MIN_KB"] = "0"
+    try:
+        base = serve_tp(E, cfg, world, trace, mode="serial", max_batch=4, max_seq=64, max_new=8, seed=3)
+        inter = serve_tp(E, cfg, world, trace, mode="interleaved", max_batch=4, max_seq=64, max_new=8,
+                         max_inflight=3, decomp_factor=8, contention_factor=1.0, seed=3)
+    finally:
+        os.environ.pop("LIGER_AR_DECOMP_MIN_KB", None)
     ref_toks = base[0][0]
     for toks, st in base + inter:
         for a, b in zip(ref_toks, toks):
@@ -115,9 +122,14 @@ def test_runtime_decomposition_bit_exact(E):
                 dur.append((op, m, k, 10.0 + 60.0 * k / F))
     trace = make_trace(4, float("inf"), seed=12, batch_sizes=(2,), prompt_range=(16, 32), n_decode=4,
                        vocab=cfg.vocab)
-    base = serve_tp(E, cfg, 2, trace, mode="serial", max_batch=2, max_seq=32, max_new=4, seed=4)
-    inter = serve_tp(E, cfg, 2, trace, durations=dur, mode="interleaved", max_batch=2, max_seq=32, max_new=4,
-                     max_inflight=2, decomp_factor=F, contention_factor=1.0, seed=4)
+    import os
+    os.environ["LIGER_AR_DECOMP_MIN_KB"] = "0"   # tiny messages: all-reduces decomposable too
+    try:
+        base = serve_tp(E, cfg, 2, trace, mode="serial", max_batch=2, max_seq=32, max_new=4, seed=4)
+        inter = serve_tp(E, cfg, 2, trace, durations=dur, mode="interleaved", max_batch=2, max_seq=32, max_new=4,
+                         max_inflight=2, decomp_factor=F, contention_factor=1.0, seed=4)
+    finally:
+        os.environ.pop("LIGER_AR_DECOMP_MIN_KB", None)
     for (tb, _), (ti, st) in zip(base, inter):
         for a, b in zip(tb, ti):
             assert np.array_equal(a, b)
