@@ -335,7 +335,7 @@ def main():
             now = time.monotonic() - t0
             # all ranks must submit identically: rank 0 decides how many arrivals are due
             due = sum(1 for r in tr[i:] if r["arrival_s"] <= now)
-            if world > 1:
+            if world > 1 and i < len(tr):   # i advances identically on every rank; afterwards no collective
                 obj = [due]
                 dist.broadcast_object_list(obj, src=0, group=gloo)
                 due = obj[0]

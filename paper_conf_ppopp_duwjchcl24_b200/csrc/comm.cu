@@ -125,6 +125,11 @@ struct NcclComm : Comm {
     par = new PeerAR();
     return par->init(world, rank, cap, region, mapped);
   }
+  PeerAR* peer_ar(cudaStream_t st) override {
+    if (!oneshot) return nullptr;
+    if (!par && setup_oneshot(st)) return nullptr;
+    return par;
+  }
   int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
     if (!count) return 0;
     if (oneshot && oneshot_eligible(count, dt, op, buf)) {
@@ -337,6 +342,11 @@ struct LoopbackComm : Comm {
     for (int q = 0; q < world; ++q) peers[q] = const_cast<void*>(xs[q]);
     par = new PeerAR();
     return par->init(world, rank, cap, region, peers);
+  }
+  PeerAR* peer_ar(cudaStream_t) override {
+    if (!oneshot) return nullptr;
+    if (!par && setup_oneshot()) return nullptr;
+    return par;
   }
   int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
     if (!count) return 0;

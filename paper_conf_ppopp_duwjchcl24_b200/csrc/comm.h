@@ -7,6 +7,8 @@
 
 #include <string>
 
+#include "kernels.h"
+
 namespace liger {
 
 struct NcclApi {
@@ -26,6 +28,7 @@ struct NcclApi {
 };
 NcclApi& nccl();
 
+
 // One-shot all-reduce over peer memory (peer_ar.cu): every rank's staging region
 // (peer_ar_region_bytes(cap) bytes, zeroed; [2 buffers][cap] + epoch flag) is
 // mapped by every rank; calls must be issued in the same order on all ranks.
@@ -38,6 +41,9 @@ struct PeerAR {
   uint64_t epoch = 0;
   int init(int world, int rank, size_t cap, void* local_region, void* const* peer_regions);
   int allreduce_bf16(void* buf, size_t count, cudaStream_t st);   // in place, sum in rank order
+  unsigned int* fused_counter = nullptr;
+  // take the next epoch for a fused producer/consumer pair (same order on all ranks)
+  int fused_begin(size_t bytes, FusedARDesc* out);
   ~PeerAR();
 };
 size_t peer_ar_region_bytes(size_t cap);
@@ -59,6 +65,9 @@ struct Comm {
   virtual int check_async() = 0;
   // host-side barrier of the group (loopback: every rank's thread has arrived)
   virtual void barrier() {}
+  // the one-shot peer all-reduce state (set up on first use; [collective]), or
+  // nullptr when this backend does not use it
+  virtual PeerAR* peer_ar(cudaStream_t) { return nullptr; }
 };
 
 Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err);

@@ -95,6 +95,10 @@ struct Slot {
   bool split_pending = false;
   GemmPlan split_plan{};
   int split_N = 0;
+  // fused all-reduce (t > 1, serial mode): the last row-parallel GEMM's fixup staged
+  // its partial for epoch far.epoch; the next add + LN reduces it over the peers
+  bool far_pending = false;
+  FusedARDesc far{};
 };
 
 struct DurTable {
@@ -180,6 +184,10 @@ struct liger_ctx {
   // 5527 vs 5433 us at b = 2, 5688 vs 5747 us at b = 8 -- one CTA per row reading
   // S x h fp32 partials costs what the fixup kernel and its hand-off did)
   bool fuse_split_ln = false;
+  // t > 1, serial mode (LIGER_FUSED_AR=1, needs the one-shot peer backend): the
+  // all-reduce of out-proj / FC2 is fused into the GEMM's fixup (stage + publish)
+  // and the following add + LN (wait + rank-ordered sum): no all-reduce kernel
+  bool fused_ar = false;
   // stats / timing
   liger_stats_t st{};
   bool timing = false;
@@ -411,6 +419,13 @@ static int split_add_ln(liger_ctx* c, Slot& S, const void* bias, const void* gam
                                      c->cfg.ln_eps, st);
 }
 
+// add + LN over the peers' staged partials of a fused all-reduce epoch
+static int peer_add_ln(liger_ctx* c, Slot& S, const void* bias, const void* gamma, const void* beta, int M,
+                       cudaStream_t st) {
+  S.far_pending = false;
+  return peer_add_layernorm_launch(S.far, S.x, bias, S.x, S.y, gamma, beta, M, c->h, c->cfg.ln_eps, st);
+}
+
 int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cudaStream_t st) {
   const PassOp po = c->pass_ops[pidx];
   Slot& S = c->slots[bt->slot];
@@ -469,6 +484,8 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       timed_begin(c, st, &ta);
       if (li == c->l0)   // first layer of the model / of this pipeline stage: x is complete
         rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
+      else if (S.far_pending)
+        rc = peer_add_ln(c, S, c->layers[li - 1].b_2, W->g1, W->be1, M, st);
       else if (S.split_pending)
         rc = split_add_ln(c, S, c->layers[li - 1].b_2, W->g1, W->be1, M, st);
       else
@@ -479,7 +496,9 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
     }
     case OP_LN2: {
       timed_begin(c, st, &ta);
-      if (S.split_pending)
+      if (S.far_pending)
+        rc = peer_add_ln(c, S, W->b_o, W->g2, W->be2, M, st);
+      else if (S.split_pending)
         rc = split_add_ln(c, S, W->b_o, W->g2, W->be2, M, st);
       else
         rc = add_layernorm_launch(S.x, S.part, W->b_o, S.x, S.y, W->g2, W->be2, M, h, 1, 0, eps, st);
@@ -524,6 +543,16 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
           S.split_N = N;
         }
       }
+      if (c->tp > 1 && c->fused_ar && c->cfg.mode == LIGER_MODE_SERIAL && u0 == 0 && u1 == F &&
+          (po.op == OP_OUT || (po.op == OP_FC2 && li + 1 < c->l1))) {
+        const GemmPlan pl = gemm_plan(M, N, K);
+        PeerAR* par = c->comm ? c->comm->peer_ar(st) : nullptr;
+        if (pl.splits > 1 && pl.cluster <= 1 && par && (size_t)M * N * 2 <= par->cap) {
+          if (par->fused_begin((size_t)M * N * 2, &S.far)) return fail(c, LIGER_ECUDA, "fused all-reduce setup");
+          g.far = &S.far;
+          S.far_pending = true;
+        }
+      }
       timed_begin(c, st, &ta);
       cudaEvent_t tmid = timed_mid(c);
       bool fix = false;
@@ -562,6 +591,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
     }
     case OP_AR1:
     case OP_AR2: {
+      if (S.far_pending) break;   // fused into the preceding GEMM and the next add + LN
       const int F = op_units(c, po.op, M);
       const size_t E = (size_t)M * h;
       timed_begin(c, st, &ta);
@@ -857,6 +887,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   }
   if (const char* fd = getenv("LIGER_FUSED_DECODE")) c->fused_decode = atoi(fd) != 0;
   if (const char* fs = getenv("LIGER_FUSE_SPLITK_LN")) c->fuse_split_ln = atoi(fs) != 0;
+  if (const char* fa = getenv("LIGER_FUSED_AR")) c->fused_ar = atoi(fa) != 0;
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (tp > 2);
   if (const char* e = getenv("LIGER_AR_DECOMP_MIN_KB")) c->ar_decomp_min_bytes = (size_t)atoll(e) * 1024;

@@ -76,6 +76,11 @@ struct GemmParams {
   const void* w_base;   // tiled weights (for the L2 prefetch)
   int pf_blocks;        // weight blocks (beyond the smem stages) prefetched into L2 before the PDL wait
   int cluster;          // > 1: split-K reduced in-kernel across a (splits x 1 x 1) thread-block cluster
+  // fused all-reduce producer (fixup kernel): publish pub_epoch on pub_flag (system
+  // scope) once every CTA's output stores are visible
+  unsigned long long* pub_flag;
+  unsigned int* pub_counter;
+  unsigned long long pub_epoch;
 };
 
 __device__ __forceinline__ float epi_apply(const GemmParams& p, float v, int n, float bias_v) {
@@ -436,6 +441,18 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
       }
     }
   }
+  if (p.pub_flag) {   // fused all-reduce: the staged partial is complete once every CTA got here
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      const unsigned int prev = atomicAdd(p.pub_counter, 1u);
+      if (prev == gridDim.x - 1) {
+        *p.pub_counter = 0;
+        __threadfence_system();
+        asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p.pub_flag), "l"(p.pub_epoch) : "memory");
+      }
+    }
+  }
   if (threadIdx.x == 0) trace_write(TK_FIXUP, tr0, tr1);
 }
 
@@ -714,6 +731,16 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.bias = reinterpret_cast<const __nv_bfloat16*>(a.bias);
   p.act = a.act; p.scale_cols = a.scale_cols; p.scale = a.scale;
   p.out = a.out; p.ldo = a.ldo; p.out_f32 = a.out_f32;
+  p.pub_flag = nullptr; p.pub_counter = nullptr; p.pub_epoch = 0;
+  if (a.far) {   // fused all-reduce producer: needs the fixup kernel and the whole GEMM
+    if (pl.splits <= 1 || pl.cluster > 1 || a.defer_fixup || a.out_f32 || a.n0 != 0 || a.n1 != a.N)
+      return LIGER_EINVAL;
+    p.out = a.far->stage;
+    p.ldo = a.N;
+    p.pub_flag = a.far->flag;
+    p.pub_counter = a.far->counter;
+    p.pub_epoch = a.far->epoch;
+  }
   p.counters = reinterpret_cast<int*>(a.workspace);
   p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
   p.w_tiled = a.w_tiled;

@@ -17,6 +17,21 @@ struct GemmPlan {
   int clusters;   // cluster mode: co-resident clusters the persistent grid uses
 };
 
+// Descriptor of one fused all-reduce (epoch) for kernels that do the one-shot
+// all-reduce's two phases themselves: the producer (row-parallel GEMM fixup) writes
+// its bf16 partial into `stage` and publishes `epoch` on `flag` when its grid is
+// done; the consumer (add + LN) waits for every peer's flag and sums the peers'
+// staged rows in rank order -- the one-shot kernel's arithmetic.
+struct FusedARDesc {
+  void* stage;                        // this rank's staging buffer (epoch parity)
+  unsigned long long* flag;           // this rank's epoch flag
+  unsigned int* counter;              // producer-grid completion counter (zero between uses)
+  const void* peer_stage[8];          // every rank's staging buffer of this epoch
+  const unsigned long long* peer_flag[8];
+  int world;
+  unsigned long long epoch;
+};
+
 struct GemmArgs {
   const void* x;
   int64_t ldx;
@@ -40,6 +55,9 @@ struct GemmArgs {
   // split-K partials are left in the workspace for a following
   // splitk_add_layernorm_launch instead of being summed by the fixup kernel
   bool defer_fixup = false;
+  // t > 1 fused all-reduce: the fixup kernel writes the bf16 result into far->stage
+  // (row-major [M, N], replacing `out`) and publishes far->epoch when the grid is done
+  const FusedARDesc* far = nullptr;
 };
 
 GemmPlan gemm_plan(int M, int N, int K);
@@ -86,6 +104,10 @@ int add_layernorm_launch(const void* x, const void* add, const void* add_bias, v
 int splitk_add_layernorm_launch(const float* ws, int64_t zstride, int splits, int m_tiles, int bn, const void* x,
                                 const void* add_bias, void* x_out, void* y, const void* gamma, const void* beta,
                                 int rows, int h, float eps, cudaStream_t stream);
+// add + LN whose added operand is the all-reduce (rank-ordered fp32 sum, RNE to bf16)
+// of the peers' staged partials of epoch far.epoch; waits for every peer's flag.
+int peer_add_layernorm_launch(const FusedARDesc& far, const void* x, const void* add_bias, void* x_out, void* y,
+                              const void* gamma, const void* beta, int rows, int h, float eps, cudaStream_t stream);
 int embed_launch(const int32_t* ids, const void* e_tok, const void* e_pos, void* out, int rows, int h, int seq_len,
                  int start_pos, cudaStream_t stream);
 int argmax_launch(const float* logits, int64_t ld, int rows, int n, int idx_offset, float* max_out,

@@ -59,12 +59,18 @@ struct SplitSrc {
 // preceding GEMM, formed here exactly as the fixup kernel would have formed it
 // (chunks summed in z order from chunk 0, + 0 bias, RNE to bf16), so the result
 // is bit-identical to fixup -> add + LN with one kernel and one hand-off fewer.
-template <int NT, int MAXV, bool SPLIT>
+// PEER: the added operand is the fused all-reduce of the row-parallel partials the
+// peers staged for epoch far.epoch (peer_ar.cu protocol): wait for every peer's
+// flag, then sum the staged rows over ranks 0..t-1 in fp32 in that order and round
+// to bf16 -- the one-shot all-reduce's bits, without its kernel.
+template <int NT, int MAXV, int MODE>
 __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x, const bf16x8* __restrict__ add,
                                                     const bf16x8* __restrict__ add_bias, bf16x8* x_out,
                                                     bf16x8* __restrict__ y, const bf16x8* __restrict__ gamma,
                                                     const bf16x8* __restrict__ beta, int h, int in_row_step,
-                                                    int in_row_off, float eps, const SplitSrc sp) {
+                                                    int in_row_off, float eps, const SplitSrc sp,
+                                                    const FusedARDesc far) {
+  constexpr bool SPLIT = MODE == 1, PEER = MODE == 2;
   __shared__ float red[NT / 32];
   const uint64_t tr0 = trace_now();
   const int nv = h >> 3;
@@ -78,7 +84,7 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
   // (by the previous add + LN; the partial `add` comes from the preceding kernel):
   // their loads are issued before the wait.  Without `add`, x may come from the
   // preceding kernel (the embedding) and is loaded after it.
-  const bool x_early = SPLIT || add != nullptr;
+  const bool x_early = SPLIT || PEER || add != nullptr;
 #pragma unroll
   for (int j = 0; j < MAXV; ++j) {
     const int v = threadIdx.x + j * NT;
@@ -89,14 +95,62 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
       vbe[j] = beta[v];
     }
   }
-  pdl_enter();
+  if (PEER) {
+    // dependents are released only after every peer has arrived (a kernel parked at
+    // its griddepcontrol.wait must not hold SMs peers sharing this GPU may need)
+    grid_dependency_wait();
+    if (threadIdx.x == 0) {
+      const uint64_t t0 = trace_now();
+      for (int q = 0; q < far.world; ++q) {
+        unsigned long long f;
+        for (;;) {
+          asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(f) : "l"(far.peer_flag[q]) : "memory");
+          if (f >= far.epoch) break;
+          __nanosleep(64);
+          if (trace_now() - t0 > 10000000000ull) __trap();   // a peer never arrived: fail, do not hang
+        }
+      }
+    }
+    __syncthreads();
+    grid_dependency_trigger();
+  } else {
+    pdl_enter();
+  }
   const uint64_t tr1 = trace_now();
 #pragma unroll
   for (int j = 0; j < MAXV; ++j) {
     const int v = threadIdx.x + j * NT;
     if (v < nv) {
       if (!x_early) vx[j] = xr[v];
-      if (!SPLIT && add) va[j] = add[in_row * nv + v];
+      if (!SPLIT && !PEER && add) va[j] = add[in_row * nv + v];
+    }
+  }
+  if (PEER) {
+    uint4 pv[MAXV][8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q)
+#pragma unroll
+      for (int j = 0; j < MAXV; ++j) {
+        const int v = threadIdx.x + j * NT;
+        if (q < far.world && v < nv)
+          pv[j][q] = __ldcv(reinterpret_cast<const uint4*>(far.peer_stage[q]) + in_row * nv + v);
+      }
+#pragma unroll
+    for (int j = 0; j < MAXV; ++j) {
+      const int v = threadIdx.x + j * NT;
+      if (v < nv) {
+        float acc[8];
+        unpack8(*reinterpret_cast<const bf16x8*>(&pv[j][0]), acc);
+#pragma unroll
+        for (int q = 1; q < 8; ++q)
+          if (q < far.world) {
+            float f[8];
+            unpack8(*reinterpret_cast<const bf16x8*>(&pv[j][q]), f);
+#pragma unroll
+            for (int e = 0; e < 8; ++e) acc[e] += f[e];
+          }
+        va[j] = pack8(acc);
+      }
     }
   }
   if (SPLIT) {
@@ -147,7 +201,7 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
     const int v = threadIdx.x + j * NT;
     if (v < nv) {
       unpack8(vx[j], r[j]);
-      if (SPLIT || add) {
+      if (SPLIT || PEER || add) {
         float a[8];
         unpack8(va[j], a);
 #pragma unroll
@@ -206,9 +260,11 @@ int add_layernorm_launch(const void* x, const void* add, const void* add_bias, v
   const bf16x8* AB = (const bf16x8*)add_bias;
   const int nv = h / 8;
   const SplitSrc none{};
+  const FusedARDesc nofar{};
 #define LIGER_LN(NT, MV)                                                                                  \
-  launch_pdl(add_ln_kernel<NT, MV, false>, dim3(rows), dim3(NT), 0, stream, X, A, AB, (bf16x8*)x_out,     \
-             (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, in_row_step, in_row_off, eps, none)
+  launch_pdl(add_ln_kernel<NT, MV, 0>, dim3(rows), dim3(NT), 0, stream, X, A, AB, (bf16x8*)x_out,         \
+             (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, in_row_step, in_row_off, eps, none,  \
+             nofar)
   int rc;
   if (nv <= 128) rc = LIGER_LN(128, 1);
   else if (nv <= 512) rc = LIGER_LN(128, 4);
@@ -224,12 +280,33 @@ int splitk_add_layernorm_launch(const float* ws, int64_t zstride, int splits, in
   if (rows <= 0) return 0;
   if (h % 128 || h > 16384 || !ws || splits < 1 || !x || !y || !gamma || !beta) return LIGER_EINVAL;
   const SplitSrc sp{ws, zstride, splits, m_tiles, bn};
+  const FusedARDesc nofar{};
   const bf16x8* X = (const bf16x8*)x;
   const bf16x8* AB = (const bf16x8*)add_bias;
   const int nv = h / 8;
 #define LIGER_LN(NT, MV)                                                                                      \
-  launch_pdl(add_ln_kernel<NT, MV, true>, dim3(rows), dim3(NT), 0, stream, X, (const bf16x8*)nullptr, AB,     \
-             (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, 1, 0, eps, sp)
+  launch_pdl(add_ln_kernel<NT, MV, 1>, dim3(rows), dim3(NT), 0, stream, X, (const bf16x8*)nullptr, AB,        \
+             (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, 1, 0, eps, sp, nofar)
+  int rc;
+  if (nv <= 128) rc = LIGER_LN(128, 1);
+  else if (nv <= 512) rc = LIGER_LN(128, 4);
+  else if (nv <= 1024) rc = LIGER_LN(256, 4);
+  else rc = LIGER_LN(512, 4);
+#undef LIGER_LN
+  return rc ? LIGER_ECUDA : 0;
+}
+
+int peer_add_layernorm_launch(const FusedARDesc& far, const void* x, const void* add_bias, void* x_out, void* y,
+                              const void* gamma, const void* beta, int rows, int h, float eps, cudaStream_t stream) {
+  if (rows <= 0) return 0;
+  if (h % 8 || h > 16384 || far.world < 1 || far.world > 8 || !x || !y || !gamma || !beta) return LIGER_EINVAL;
+  const SplitSrc none{};
+  const bf16x8* X = (const bf16x8*)x;
+  const bf16x8* AB = (const bf16x8*)add_bias;
+  const int nv = h / 8;
+#define LIGER_LN(NT, MV)                                                                                      \
+  launch_pdl(add_ln_kernel<NT, MV, 2>, dim3(rows), dim3(NT), 0, stream, X, (const bf16x8*)nullptr, AB,        \
+             (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, 1, 0, eps, none, far)
   int rc;
   if (nv <= 128) rc = LIGER_LN(128, 1);
   else if (nv <= 512) rc = LIGER_LN(128, 4);

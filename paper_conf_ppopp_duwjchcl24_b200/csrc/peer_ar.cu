@@ -61,6 +61,7 @@ __global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf
   // loopback backend those ranks share this GPU and would need them to progress.
   grid_dependency_wait();
   for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += stride) my_stage[i] = buf[i];
+  __threadfence_system();   // every thread's staging stores before the block's publish
   __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence_system();
@@ -132,6 +133,29 @@ int PeerAR::init(int world_, int rank_, size_t cap_, void* local_region, void* c
 
 PeerAR::~PeerAR() {
   if (counter) cudaFree(counter);
+  if (fused_counter) cudaFree(fused_counter);
+}
+
+int PeerAR::fused_begin(size_t bytes, FusedARDesc* out) {
+  if (bytes > cap || bytes % 16) return LIGER_EINVAL;
+  if (!fused_counter) {
+    if (cudaMalloc(&fused_counter, sizeof(unsigned int)) != cudaSuccess) return LIGER_ENOMEM;
+    if (cudaMemset(fused_counter, 0, sizeof(unsigned int)) != cudaSuccess) return LIGER_ECUDA;
+  }
+  ++epoch;
+  const int b = (int)(epoch & 1);
+  FusedARDesc d{};
+  d.stage = static_cast<char*>(local) + (size_t)b * cap;
+  d.flag = reinterpret_cast<unsigned long long*>(static_cast<char*>(local) + 2 * cap);
+  d.counter = fused_counter;
+  for (int q = 0; q < world; ++q) {
+    d.peer_stage[q] = static_cast<const char*>(peer[q]) + (size_t)b * cap;
+    d.peer_flag[q] = reinterpret_cast<const unsigned long long*>(static_cast<const char*>(peer[q]) + 2 * cap);
+  }
+  d.world = world;
+  d.epoch = epoch;
+  *out = d;
+  return 0;
 }
 
 int PeerAR::allreduce_bf16(void* buf, size_t count, cudaStream_t st) {

@@ -203,3 +203,34 @@ def test_sync_ablation_modes_bit_exact(E, sync):
     assert alt[0][1]["overlapped_rounds"] > 0
     if sync == "inter_stream":
         assert alt[0][1]["wait_us"] == 0.0
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_fused_gemm_allreduce_bit_exact(E, world):
+    """§8(f) next row 4: the row-parallel GEMM's all-reduce fused into its split-K
+    fixup (bf16 partial staged in peer-visible memory, epoch published with a
+    system-scope release) and the following add + LN (waits for every peer, sums the
+    staged rows in rank order) -- no all-reduce kernel.  Serial TP with the fusion
+    must give the tokens of serial TP with the one-shot all-reduce kernel, bit for
+    bit, on every rank; the config makes the decode projections split K (h = 1024)."""
+    import os
+    from liger_inputs.configs import ModelConfig
+    from paper_conf_ppopp_duwjchcl24_b200 import liger as L
+    cfg = ModelConfig("mid2", 2, 1024, 8, 4096, 1024, 96, "relu")
+    hl, fl = cfg.hidden // world, cfg.ffn // world
+    assert L.gemm_plan(3, cfg.hidden, fl)["splits"] > 1
+    trace = make_trace(3, float("inf"), seed=8, batch_sizes=(1, 3), prompt_range=(10, 40), n_decode=5,
+                       vocab=cfg.vocab)
+    kw = dict(mode="serial", max_batch=4, max_seq=48, max_new=8, seed=9)
+    res = {}
+    for flag in ("0", "1"):
+        os.environ["LIGER_FUSED_AR"] = flag
+        try:
+            res[flag] = serve_tp(E, cfg, world, trace, **kw)
+        finally:
+            os.environ.pop("LIGER_FUSED_AR", None)
+    for r in range(world):
+        for a, b in zip(res["0"][0][0], res["1"][r][0]):
+            assert np.array_equal(a, b)
+    # the fused run issued fewer all-reduce kernels (only those that could not fuse)
+    assert res["1"][0][1]["comm_kernels"] < res["0"][0][1]["comm_kernels"]
