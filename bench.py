@@ -184,6 +184,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-latency", action="store_true")
     ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--fused-ar", action="store_true",
+                    help="serial TP competitor: row-parallel GEMM + all-reduce fused over peer memory "
+                         "(LIGER_FUSED_AR=1 with the one-shot peer backend; use with --mode serial)")
     ap.add_argument("--sync", default="hybrid", choices=["hybrid", "cpu_gpu", "inter_stream"],
                     help="Algorithm 1 round synchronisation (§3.4 Fig. 8; ablation §4.5)")
     ap.add_argument("--workload", default="mixed", choices=["mixed", "generative"],
@@ -194,6 +197,9 @@ def main():
     args = ap.parse_args()
     if args.workload == "generative":
         args.n_new = 2
+    if args.fused_ar:
+        os.environ["LIGER_FUSED_AR"] = "1"
+        os.environ["LIGER_ONESHOT_AR"] = "1"
     _redirect_stdout()
     if args.impl == "reference":
         return run_reference(args)
@@ -222,6 +228,14 @@ def main():
     eng.profile([8, 64, 256, 512, 1024, 2048, 4096])
     # contention factor: measured GEMM || all-reduce slowdown (1-rank proxy at N=1)
     cf_cal, _ = eng.calibrate_cf([8, 256, 1024], set_cf=args.cf <= 0)
+    # contention control: the same calibration with the GEMM grid
+    # leaving SMs to the communication kernel
+    cf_reserve = {}
+    for rsv in (8, 16, 32):
+        eng.set_gemm_sm_reserve(rsv)
+        cf_reserve[rsv] = round(eng.calibrate_cf([8, 256, 1024], set_cf=False)[0], 4)
+    eng.set_gemm_sm_reserve(int(os.environ.get("LIGER_GEMM_SM_RESERVE", "0")))
+    cf_reserve[0] = round(cf_cal, 4)
 
     def barrier():
         if world > 1:
@@ -371,9 +385,10 @@ def main():
                                      f"batches of 2/4/8 x prompt U[128,512], {args.n_new} generated tokens") +
                                     f", all {len(timed)} batches offered at once (capacity)"),
                        "model": cfg.name, "tp": world,
-                       "mode": args.mode, "sync": args.sync, "max_inflight": args.inflight, "decomp_factor": args.F,
+                       "mode": args.mode, "sync": args.sync, "fused_ar": args.fused_ar, "max_inflight": args.inflight, "decomp_factor": args.F,
                        "contention_factor": args.cf if args.cf > 0 else cf_cal,
                        "contention_factor_calibrated": round(cf_cal, 4),
+                       "contention_factor_vs_gemm_sm_reserve": {str(k): v for k, v in sorted(cf_reserve.items())},
                        "sequences": seqs, "batches": len(timed),
                        "l2": "inputs larger than L2 (weights 26 GB per TP=1 rank)"},
             "latency": lat,

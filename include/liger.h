@@ -174,6 +174,14 @@ int liger_result_tokens_device(liger_ctx* ctx, int64_t id, const int32_t** dev_t
 int liger_stats(liger_ctx* ctx, liger_stats_t* out);
 int liger_reset_stats(liger_ctx* ctx);
 
+/* Contention control (§3.5): at t > 1
+ * (and inside liger_calibrate_cf) every projection GEMM's persistent grid leaves
+ * `reserve` SMs free for a concurrently running all-reduce kernel.  The grid size
+ * never changes a GEMM's bits.  0 <= reserve < #SMs, else LIGER_EINVAL.  Default 0
+ * (or LIGER_GEMM_SM_RESERVE).  Local (not collective), but every rank should use
+ * the same value, since it changes the profiled durations the plans are made from. */
+int liger_set_gemm_sm_reserve(liger_ctx* ctx, int reserve);
+
 /* Enable (1) / disable (0) CUDA-event timing of every GEMM, attention,
  * layernorm and all-reduce launch on the stream it runs on;
  * liger_kernel_timing returns, per kernel class (LIGER_KT_*), the launch

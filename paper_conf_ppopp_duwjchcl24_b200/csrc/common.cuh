@@ -6,6 +6,8 @@
 
 #include <stdlib.h>
 
+#include <mutex>
+#include <unordered_set>
 #include <utility>
 
 #define LIGER_DEV __device__ __forceinline__
@@ -252,12 +254,27 @@ LIGER_DEV float gelu_tanh_f(float x) {
   return 0.5f * x * (1.0f + tanhf(k0 * (x + k1 * x * x * x)));
 }
 
+// Every kernel of the library prefers the maximal shared-memory carveout.  An SM's
+// L1/shared split can only change while it is idle, so a kernel that stays resident
+// (the all-reduce kernels spinning on peers' flags) would otherwise pin a small-smem
+// configuration and keep a persistent GEMM CTA (up to 217 KB) off that SM -- with
+// static unit assignment that GEMM then never completes (a TP = 4 loopback hang).
+inline void prefer_max_smem(const void* fn) {
+  static std::mutex mu;
+  static std::unordered_set<const void*> done;
+  static const bool off = getenv("LIGER_NO_CARVEOUT") != nullptr;   // experiments only
+  if (off) return;
+  std::lock_guard<std::mutex> g(mu);
+  if (done.insert(fn).second) cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+}
+
 // Launch with programmatic stream serialization so the kernel's prologue overlaps
 // the tail of the previous kernel on the stream (the kernel calls
 // grid_dependency_wait() before touching data produced or consumed upstream).
 template <typename... KArgs, typename... Args>
 inline int launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
                       Args&&... args) {
+  prefer_max_smem(reinterpret_cast<const void*>(kernel));
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = grid;
   cfg.blockDim = block;
@@ -276,6 +293,7 @@ inline int launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t sm
 template <typename... KArgs, typename... Args>
 inline int launch_pdl_cluster(void (*kernel)(KArgs...), dim3 grid, dim3 block, int cluster_x, size_t smem,
                               cudaStream_t stream, Args&&... args) {
+  prefer_max_smem(reinterpret_cast<const void*>(kernel));
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = grid;
   cfg.blockDim = block;

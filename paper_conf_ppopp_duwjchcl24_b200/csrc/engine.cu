@@ -188,6 +188,11 @@ struct liger_ctx {
   // all-reduce of out-proj / FC2 is fused into the GEMM's fixup (stage + publish)
   // and the following add + LN (wait + rank-ordered sum): no all-reduce kernel
   bool fused_ar = false;
+  // SMs a t > 1 GEMM leaves free for a concurrent all-reduce (LIGER_GEMM_SM_RESERVE,
+  // liger_set_gemm_sm_reserve); the grid size never changes a GEMM's bits
+  int gemm_sm_reserve = 0;
+  bool calibrating = false;   // liger_calibrate_cf at t = 1 (proxy communicator)
+  int n_sms = 148;
   // stats / timing
   liger_stats_t st{};
   bool timing = false;
@@ -206,8 +211,13 @@ struct liger_ctx {
 namespace {
 
 int fail(liger_ctx* c, int rc, const std::string& msg) {
-  if (c) c->err = msg;
-  set_global_error(msg);
+  std::string m = msg;
+  if (rc == LIGER_ECUDA || rc == -1000) {   // say which CUDA error (sticky errors surface at a later launch)
+    const cudaError_t e = cudaPeekAtLastError();
+    if (e != cudaSuccess) m += std::string(" [") + cudaGetErrorString(e) + "]";
+  }
+  if (c) c->err = m;
+  set_global_error(m);
   return rc;
 }
 
@@ -519,6 +529,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       g.workspace = S.gemm_ws; g.ws_bytes = S.gemm_ws_bytes;
       g.scale = 1.0f;
       g.w_tiled = 1;
+      if (c->gemm_sm_reserve > 0 && (c->comm || c->calibrating)) g.sm_budget = std::max(1, c->n_sms - c->gemm_sm_reserve);
       if (po.op == OP_QKV) {
         g.x = S.y; g.ldx = h; g.w = W->w_qkv; g.ldw = K; g.out = S.qkv; g.ldo = N; g.bias = W->b_qkv;
         g.scale_cols = c->hl; g.scale = 1.0f / sqrtf((float)c->d);
@@ -888,6 +899,12 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   if (const char* fd = getenv("LIGER_FUSED_DECODE")) c->fused_decode = atoi(fd) != 0;
   if (const char* fs = getenv("LIGER_FUSE_SPLITK_LN")) c->fuse_split_ln = atoi(fs) != 0;
   if (const char* fa = getenv("LIGER_FUSED_AR")) c->fused_ar = atoi(fa) != 0;
+  if (const char* sr = getenv("LIGER_GEMM_SM_RESERVE")) c->gemm_sm_reserve = atoi(sr);
+  {
+    int dev = 0, n = 0;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && n > 0) c->n_sms = n;
+  }
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (tp > 2);
   if (const char* e = getenv("LIGER_AR_DECOMP_MIN_KB")) c->ar_decomp_min_bytes = (size_t)atoll(e) * 1024;
@@ -1253,6 +1270,12 @@ int liger_reset_stats(liger_ctx* c) {
   return LIGER_OK;
 }
 
+int liger_set_gemm_sm_reserve(liger_ctx* c, int reserve) {
+  if (!c || reserve < 0 || reserve >= c->n_sms) return LIGER_EINVAL;
+  c->gemm_sm_reserve = reserve;
+  return LIGER_OK;
+}
+
 int liger_set_kernel_timing(liger_ctx* c, int on) {
   if (!c) return LIGER_EINVAL;
   timing_flush(c);
@@ -1319,6 +1342,7 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
   for (auto& e : ev) CK(cudaEventCreate(&e));
   const bool saved_timing = c->timing;
   c->timing = false;
+  c->calibrating = true;
   Batch fake;
   fake.slot = 0;
   fake.n_new = 1;
@@ -1369,6 +1393,7 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
     }
   }
   c->timing = saved_timing;
+  c->calibrating = false;
   for (auto& e : ev) cudaEventDestroy(e);
   delete own;
   if (c->world > 1) {   // all ranks must use the same cf (identical plans)

@@ -761,7 +761,9 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
     rc2 = launch_pdl_cluster(gemm_tc_kernel, dim3(nc * pl.cluster), dim3(GEMM_THREADS), pl.cluster, pl.smem, stream,
                              tA, tB, p);
   } else {
-    const int grid = p.units < num_sms() ? p.units : num_sms();
+    // unit u runs on CTA u % grid: the grid size never changes what a unit computes
+    const int sms = (a.sm_budget > 0 && a.sm_budget < num_sms()) ? a.sm_budget : num_sms();
+    const int grid = p.units < sms ? p.units : sms;
     rc2 = launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
   }
   const bool fixup = p.splits > 1 && pl.cluster <= 1 && !a.defer_fixup;

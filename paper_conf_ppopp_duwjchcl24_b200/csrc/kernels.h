@@ -58,6 +58,9 @@ struct GemmArgs {
   // t > 1 fused all-reduce: the fixup kernel writes the bf16 result into far->stage
   // (row-major [M, N], replacing `out`) and publishes far->epoch when the grid is done
   const FusedARDesc* far = nullptr;
+  // SM budget of the persistent GEMM grid (0 = every SM): leaves SMs to a
+  // communication kernel running concurrently (contention control)
+  int sm_budget = 0;
 };
 
 GemmPlan gemm_plan(int M, int N, int K);

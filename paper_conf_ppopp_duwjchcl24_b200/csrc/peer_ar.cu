@@ -23,6 +23,7 @@
 #include <cuda_bf16.h>
 #include <stdint.h>
 #include <string.h>
+#include <stdio.h>
 
 #include "comm.h"
 #include "common.cuh"
@@ -75,7 +76,11 @@ __global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf
     for (int q = 0; q < world; ++q)
       while (ld_acquire_sys(peers.flag[q]) < epoch) {
         __nanosleep(64);
-        if (trace_now() - t0 > 10000000000ull) __trap();   // a peer never arrived: fail, do not hang
+        if (trace_now() - t0 > 10000000000ull) {   // a peer never arrived: fail, do not hang
+          printf("liger one-shot all-reduce: epoch %llu, waited 10 s for peer %d (flag %llu), block %d of %d\n",
+                 epoch, q, ld_acquire_sys(peers.flag[q]), blockIdx.x, gridDim.x);
+          __trap();
+        }
       }
   }
   __syncthreads();
@@ -117,7 +122,12 @@ __global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf
 
 }  // namespace
 
-size_t peer_ar_region_bytes(size_t cap) { return 2 * cap + 256; }
+// [2 buffers][cap] | epoch flag (+0) | one-shot block counter (+128) | fused-producer
+// counter (+256): the counters live in the zeroed region so that nothing is
+// allocated after the ranks' setup rendezvous -- on the loopback backend a
+// cudaMalloc / cudaMemset there can wait for a peer's kernel that is spinning on
+// this rank's flag (seen as a TP = 4 hang).
+size_t peer_ar_region_bytes(size_t cap) { return 2 * cap + 512; }
 
 int PeerAR::init(int world_, int rank_, size_t cap_, void* local_region, void* const* peer_regions) {
   if (world_ < 1 || world_ > PAR_MAX_WORLD || cap_ % 256) return LIGER_EINVAL;
@@ -126,22 +136,15 @@ int PeerAR::init(int world_, int rank_, size_t cap_, void* local_region, void* c
   cap = cap_;
   local = local_region;
   for (int q = 0; q < world; ++q) peer[q] = peer_regions[q];
-  if (cudaMalloc(&counter, sizeof(unsigned int)) != cudaSuccess) return LIGER_ENOMEM;
-  cudaMemset(counter, 0, sizeof(unsigned int));
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
+  counter = reinterpret_cast<unsigned int*>(static_cast<char*>(local) + 2 * cap + 128);
+  fused_counter = reinterpret_cast<unsigned int*>(static_cast<char*>(local) + 2 * cap + 256);
+  return 0;
 }
 
-PeerAR::~PeerAR() {
-  if (counter) cudaFree(counter);
-  if (fused_counter) cudaFree(fused_counter);
-}
+PeerAR::~PeerAR() {}
 
 int PeerAR::fused_begin(size_t bytes, FusedARDesc* out) {
   if (bytes > cap || bytes % 16) return LIGER_EINVAL;
-  if (!fused_counter) {
-    if (cudaMalloc(&fused_counter, sizeof(unsigned int)) != cudaSuccess) return LIGER_ENOMEM;
-    if (cudaMemset(fused_counter, 0, sizeof(unsigned int)) != cudaSuccess) return LIGER_ECUDA;
-  }
   ++epoch;
   const int b = (int)(epoch & 1);
   FusedARDesc d{};

@@ -122,6 +122,9 @@ class LigerEngine:
     def reset_stats(self):
         self._chk(L.lib().liger_reset_stats(self.ctx), "liger_reset_stats")
 
+    def set_gemm_sm_reserve(self, reserve):
+        self._chk(L.lib().liger_set_gemm_sm_reserve(self.ctx, int(reserve)), "liger_set_gemm_sm_reserve")
+
     def set_kernel_timing(self, on):
         self._chk(L.lib().liger_set_kernel_timing(self.ctx, int(on)), "liger_set_kernel_timing")
 

@@ -74,6 +74,7 @@ _SIGS = {
     "liger_result_tokens_device": (_I, [_P, _I64, C.POINTER(_P)]),
     "liger_stats": (_I, [_P, C.POINTER(liger_stats_t)]),
     "liger_reset_stats": (_I, [_P]),
+    "liger_set_gemm_sm_reserve": (_I, [_P, _I]),
     "liger_set_kernel_timing": (_I, [_P, _I]),
     "liger_kernel_timing": (_I, [_P, _P, _P, _P, _P]),
     "liger_set_duration": (_I, [_P, _I, _I, _I, _D]),

@@ -234,3 +234,22 @@ def test_fused_gemm_allreduce_bit_exact(E, world):
             assert np.array_equal(a, b)
     # the fused run issued fewer all-reduce kernels (only those that could not fuse)
     assert res["1"][0][1]["comm_kernels"] < res["0"][0][1]["comm_kernels"]
+
+
+def test_gemm_sm_reserve_bit_exact(E):
+    """Contention control (§3.5): GEMM grids that leave SMs free for a
+    concurrent all-reduce compute the same units, so tokens are bit-identical."""
+    import os
+    cfg = get_config("tiny")
+    trace = make_trace(3, float("inf"), seed=31, batch_sizes=(1, 2), prompt_range=(8, 40), n_decode=5,
+                       vocab=cfg.vocab)
+    kw = dict(mode="interleaved", max_batch=4, max_seq=48, max_new=8, max_inflight=2, seed=10)
+    ref = serve_tp(E, cfg, 2, trace, **kw)
+    os.environ["LIGER_GEMM_SM_RESERVE"] = "145"   # 3-CTA grids: units wrap around
+    try:
+        alt = serve_tp(E, cfg, 2, trace, **kw)
+    finally:
+        os.environ.pop("LIGER_GEMM_SM_RESERVE", None)
+    for (tr, _), (ta, _) in zip(ref, alt):
+        for a, b in zip(tr, ta):
+            assert np.array_equal(a, b)
