@@ -96,31 +96,52 @@ struct NcclComm : Comm {
     if (comm) nccl().CommDestroy(comm);
   }
   // [collective] map every rank's staging region: CUDA IPC handles exchanged with an
-  // NCCL all-gather (same-node NVLink / NVSwitch peers)
+  // NCCL all-gather (same-node NVLink / NVSwitch peers).  The ranks then agree (NCCL
+  // min) on whether every rank mapped every peer; if any could not (e.g. peers not
+  // P2P-reachable from this process), all of them fall back to NCCL all-reduces.
   int setup_oneshot(cudaStream_t st) {
     const size_t cap = oneshot_cap(), rb = peer_ar_region_bytes(cap);
     if (world > 8 || cudaMalloc(&region, rb) != cudaSuccess || cudaMemset(region, 0, rb) != cudaSuccess)
       return LIGER_ENOMEM;
     cudaIpcMemHandle_t h;
-    if (cudaIpcGetMemHandle(&h, region) != cudaSuccess) return LIGER_ECUDA;
+    int ok = cudaIpcGetMemHandle(&h, region) == cudaSuccess ? 1 : 0;
     char* d = nullptr;
-    if (cudaMalloc(&d, (size_t)64 * (world + 1)) != cudaSuccess) return LIGER_ENOMEM;
+    if (cudaMalloc(&d, (size_t)64 * (world + 1) + 16) != cudaSuccess) return LIGER_ENOMEM;
     cudaMemcpy(d + (size_t)64 * world, &h, 64, cudaMemcpyHostToDevice);
     ncclResult_t r = nccl().AllGather(d + (size_t)64 * world, d, 64, ncclUint8, comm, st);
     std::vector<cudaIpcMemHandle_t> all(world);
     if (r == ncclSuccess && cudaStreamSynchronize(st) == cudaSuccess)
       cudaMemcpy(all.data(), d, (size_t)64 * world, cudaMemcpyDeviceToHost);
-    cudaFree(d);
-    if (r != ncclSuccess) return LIGER_ENCCL;
-    for (int q = 0; q < world; ++q) {
+    if (r != ncclSuccess) {
+      cudaFree(d);
+      return LIGER_ENCCL;
+    }
+    for (int q = 0; q < world && ok; ++q) {
       if (q == rank) {
         mapped[q] = region;
         continue;
       }
       if (cudaIpcOpenMemHandle(&mapped[q], all[q], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
-        err = "cudaIpcOpenMemHandle failed (peers not P2P-capable?)";
-        return LIGER_ECUDA;
+        cudaGetLastError();
+        mapped[q] = nullptr;
+        ok = 0;
       }
+    }
+    int32_t* flag = reinterpret_cast<int32_t*>(d + (size_t)64 * (world + 1));
+    cudaMemcpy(flag, &ok, sizeof(int32_t), cudaMemcpyHostToDevice);
+    r = nccl().AllReduce(flag, flag, 1, ncclInt32, ncclMin, comm, st);
+    int all_ok = 0;
+    if (r == ncclSuccess && cudaStreamSynchronize(st) == cudaSuccess)
+      cudaMemcpy(&all_ok, flag, sizeof(int32_t), cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    if (r != ncclSuccess) return LIGER_ENCCL;
+    if (!all_ok) {   // agreed fallback: NCCL for every all-reduce from now on
+      for (int q = 0; q < world; ++q)
+        if (mapped[q] && q != rank) cudaIpcCloseMemHandle(mapped[q]);
+      for (int q = 0; q < world; ++q) mapped[q] = nullptr;
+      oneshot = false;
+      err = "one-shot all-reduce disabled: a rank could not map its peers' staging buffers";
+      return 0;
     }
     par = new PeerAR();
     return par->init(world, rank, cap, region, mapped);
@@ -128,14 +149,14 @@ struct NcclComm : Comm {
   PeerAR* peer_ar(cudaStream_t st) override {
     if (!oneshot) return nullptr;
     if (!par && setup_oneshot(st)) return nullptr;
-    return par;
+    return par;   // nullptr after an agreed fallback
   }
   int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
     if (!count) return 0;
     if (oneshot && oneshot_eligible(count, dt, op, buf)) {
       if (!par)
         if (int rc = setup_oneshot(st)) return rc;
-      return par->allreduce_bf16(buf, count, st);
+      if (par) return par->allreduce_bf16(buf, count, st);
     }
     ncclResult_t r = nccl().AllReduce(buf, buf, count, nccl_dt(dt), op == CO_SUM ? ncclSum : ncclMax, comm, st);
     if (r != ncclSuccess) {
@@ -510,7 +531,7 @@ Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err) {
   auto* c = new NcclComm();
   c->world = world;
   c->rank = rank;
-  c->oneshot = oneshot_enabled(false);   // IPC path: opt-in until measured on NVLink
+  c->oneshot = oneshot_enabled(false);   // IPC path: opt-in (LIGER_ONESHOT_AR=1) until measured on NVLink
   ncclResult_t r = nccl().CommInitRank(&c->comm, world, id, rank);
   if (r != ncclSuccess) {
     *err = std::string("ncclCommInitRank: ") + nccl().GetErrorString(r);
