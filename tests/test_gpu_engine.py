@@ -100,3 +100,28 @@ def test_contention_factor_calibration(E):
     eng.close()
     assert 1.0 <= cf < 10.0
     assert set(detail) == {16, 64} and all(len(v) == 4 for v in detail.values())
+
+
+def test_nccl_oneshot_setup_and_kernel_single_rank(E):
+    """The NCCL backend's one-shot path on real hardware at one rank: liger_calibrate_cf
+    at t = 1 runs its all-reduces on a 1-rank NCCL communicator; with LIGER_ONESHOT_AR=1
+    that exercises the CUDA-IPC staging setup, the NCCL agreement on it and the
+    one-shot kernel (flags, staging, rank-ordered sum) -- with the GEMM SM reserve
+    on, so GEMM grids leave SMs to it."""
+    import os
+    cfg = get_config("tiny")
+    os.environ["LIGER_ONESHOT_AR"] = "1"
+    try:
+        eng = E(cfg, max_batch=2, max_seq=32, max_new=4, seed=0)
+        eng.set_gemm_sm_reserve(16)
+        cf, _ = eng.calibrate_cf([16, 64], set_cf=False)
+        toks_ok = True
+        prompt = np.random.default_rng(1).integers(0, cfg.vocab, size=(2, 16)).astype(np.int32)
+        bid = eng.submit(prompt.reshape(-1), 2, 16, 3, 0.0)
+        eng.drain()
+        res, toks = eng.poll(bid, want_tokens=True)
+        eng.close()
+    finally:
+        os.environ.pop("LIGER_ONESHOT_AR", None)
+    assert 1.0 <= cf < 10.0
+    assert res.done == 1 and toks.shape == (2, 3) and toks_ok
