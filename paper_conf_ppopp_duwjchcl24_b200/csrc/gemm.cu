@@ -655,6 +655,21 @@ GemmPlan gemm_plan(int M, int N, int K) {
         const int ctas = std::min(left, nc) * S;
         cost += (double)((ctas + G - 1) / G) * (kcb * kb_time + 300.0) + 1200.0;
       }
+      cost /= 1900.0;   // SM cycles -> us (M <= 64 here: compared with the decode model below)
+    } else if (M <= 64) {
+      // Decode (weight stream), in us, fitted to tools/split_sweep2.py on B200
+      // (profiles/r01/split_sweep_decode.txt): the persistent grid runs rounds of
+      // up to G units; a round takes max(its weight bytes at the achievable HBM
+      // rate 5.75 TB/s, one unit's k-blocks at a single SM's ~48 GB/s); a split
+      // adds the fixup hand-off (0.8 us) and its fp32 partial traffic through L2.
+      cost = 0.0;
+      const double blk_us = A_BYTES / 48.0e3 + (double)bn * BK * 2 / 200.0e3;   // weights from HBM, activations from L2
+      for (double left = (double)tiles * S; left > 0; left -= G) {
+        const double units = fmin(left, (double)G);
+        const double kb = fmin((double)kcb, (double)nkb);
+        cost += fmax(units * kb * A_BYTES / 5.75e6, kb * blk_us) + 0.05;
+      }
+      if (S > 1) cost += 0.8 + (double)S * M * N * 8.0 / 10.0e6;
     } else {
       const double units = (double)tiles * S;
       cost = ceil(units / G) * (kcb * kb_time + 300.0);
