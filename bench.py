@@ -175,7 +175,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="opt-13b")
     ap.add_argument("--layers", type=int, default=None, help="debug only: fewer layers (invalid for reporting)")
-    ap.add_argument("--mode", default="interleaved", choices=["interleaved", "serial", "pipeline"],
+    ap.add_argument("--mode", default="interleaved", choices=["interleaved", "serial", "pipeline", "pipeline_th"],
                     help="Liger (interleaved), Intra-Op (serial TP) or Inter-Op (pipeline) baseline")
     ap.add_argument("--inflight", type=int, default=2)
     ap.add_argument("--F", type=int, default=8)

@@ -68,6 +68,10 @@ extern "C" {
 #define LIGER_MODE_PIPELINE 2    /* Inter-Op baseline: rank r holds an equal stage of unsharded
                                     layers, activations / tokens travel by send/recv;
                                     generated tokens are reported by the last stage */
+#define LIGER_MODE_PIPELINE_TH 3 /* Inter-Th baseline: the Inter-Op pipeline whose every
+                                    projection GEMM runs as `world` partitioned kernels (1/world
+                                    of the output columns each, as intra-op partitions them);
+                                    bit-identical to LIGER_MODE_PIPELINE */
 
 /* ------------------------------------------------------------------ config */
 typedef struct {

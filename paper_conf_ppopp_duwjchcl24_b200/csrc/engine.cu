@@ -191,6 +191,7 @@ struct liger_ctx {
   // SMs a t > 1 GEMM leaves free for a concurrent all-reduce (LIGER_GEMM_SM_RESERVE,
   // liger_set_gemm_sm_reserve); the grid size never changes a GEMM's bits
   int gemm_sm_reserve = 0;
+  int th_parts = 1;   // Inter-Th: projection GEMMs issued as this many partitioned kernels
   bool calibrating = false;   // liger_calibrate_cf at t = 1 (proxy communicator)
   int n_sms = 148;
   // stats / timing
@@ -569,7 +570,19 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       bool fix = false;
       g.ev_mid = tmid;
       g.had_fixup = &fix;
-      rc = gemm_launch(g, st);
+      if (c->th_parts > 1) {
+        // Inter-Th: the GEMM as th_parts partitioned kernels over its output columns
+        // (each a full-plan slice: the bits of the whole GEMM)
+        const int P = c->th_parts, a0 = g.n0, a1 = g.n1;
+        for (int r = 0; r < P && !rc; ++r) {
+          g.n0 = std::max(a0, unit_col(N, r, P));
+          g.n1 = std::min(a1, r + 1 == P ? N : unit_col(N, r + 1, P));
+          if (g.n1 > g.n0) rc = gemm_launch(g, st);
+        }
+        c->st.gpu_launches += P - 1;
+      } else {
+        rc = gemm_launch(g, st);
+      }
       const double n = g.n1 - g.n0;
       if (c->timing) {
         // GEMM kernel: algorithmic bytes / flops; fixup: fp32 partials read + output written
@@ -868,7 +881,8 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   c->rank = rank;
   c->cfg = *cfg;
   c->h = cfg->hidden; c->a = cfg->n_heads; c->f = cfg->ffn; c->V = cfg->vocab; c->L = cfg->n_layers;
-  c->pipe = cfg->mode == LIGER_MODE_PIPELINE;
+  c->pipe = cfg->mode == LIGER_MODE_PIPELINE || cfg->mode == LIGER_MODE_PIPELINE_TH;
+  c->th_parts = cfg->mode == LIGER_MODE_PIPELINE_TH ? world : 1;
   c->tp = c->pipe ? 1 : world;
   c->tp_rank = c->pipe ? 0 : rank;
   const int tp = c->tp;
@@ -887,6 +901,8 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     c->l0 = 0;
     c->l1 = c->L;
   }
+  if (cfg->mode < LIGER_MODE_SERIAL || cfg->mode > LIGER_MODE_PIPELINE_TH)
+    return fail(nullptr, LIGER_EINVAL, "liger_init: unknown mode");
   if (cfg->sync_mode < LIGER_SYNC_HYBRID || cfg->sync_mode > LIGER_SYNC_INTER_STREAM)
     return fail(nullptr, LIGER_EINVAL, "liger_init: unknown sync_mode");
   c->F = std::max(1, cfg->decomp_factor);

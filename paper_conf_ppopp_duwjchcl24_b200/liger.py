@@ -11,7 +11,7 @@ LIB_PATH = os.path.join(HERE, "libliger.so")
 LIGER_OK, LIGER_PENDING, LIGER_IDLE = 0, 1, 2
 ACT = {"none": 0, "relu": 1, "gelu_tanh": 2}
 SYNC = {"hybrid": 0, "cpu_gpu": 1, "inter_stream": 2}
-MODE = {"serial": 0, "interleaved": 1, "pipeline": 2}
+MODE = {"serial": 0, "interleaved": 1, "pipeline": 2, "pipeline_th": 3}
 KV_BLOCK = 16
 KT_NAMES = ["gemm_decode", "attn", "ln", "allreduce", "gemm_prefill", "lm_head", "splitk_fixup",
             "decode_fused"]   # LIGER_KT_*

@@ -136,12 +136,13 @@ def test_runtime_decomposition_bit_exact(E):
     assert inter[0][1]["split_pieces"] > 0, inter[0][1]
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_pipeline_baseline_equals_single_gpu(E, world):
+@pytest.mark.parametrize("world,mode", [(2, "pipeline"), (3, "pipeline"), (2, "pipeline_th"), (3, "pipeline_th")])
+def test_pipeline_baseline_equals_single_gpu(E, world, mode):
     """Inter-operator pipeline baseline: `world` stages of unsharded layers,
     activations and tokens passed stage to stage; several batches in flight.
     The last stage's tokens are bit-identical to the single-GPU run (the same
-    unsharded kernels)."""
+    unsharded kernels).  Inter-Th issues every projection GEMM as `world`
+    partitioned kernels (output-column slices of the full plan): the same bits."""
     from liger_inputs.configs import ModelConfig
     cfg = ModelConfig("tiny6", 6, 256, 4, 1024, 512, 64, "gelu_tanh")
     trace = make_trace(4, float("inf"), seed=13, batch_sizes=(1, 2), prompt_range=(8, 30), n_decode=5,
@@ -151,7 +152,7 @@ def test_pipeline_baseline_equals_single_gpu(E, world):
     eng.drain()
     ref = [eng.poll(i, want_tokens=True)[1] for i in ids]
     eng.close()
-    pipe = serve_tp(E, cfg, world, trace, mode="pipeline", max_batch=2, max_seq=32, max_new=8, max_inflight=world,
+    pipe = serve_tp(E, cfg, world, trace, mode=mode, max_batch=2, max_seq=32, max_new=8, max_inflight=world,
                     seed=5)
     toks, st = pipe[world - 1]
     for a, b in zip(ref, toks):
