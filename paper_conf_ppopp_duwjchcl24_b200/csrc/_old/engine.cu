@@ -74,10 +74,6 @@ struct bf16p {
 
 struct LayerW {
   void *w_qkv, *b_qkv, *w_o, *b_o, *w_1, *b_1, *w_2, *b_2, *g1, *be1, *g2, *be2;
-  // LayerNorm folded into QKV / FC1 for decode passes (t = 1): W*gamma (tiled) and
-  // the fp32 epilogue vectors u = (W*gamma).1, c = W.beta + bias
-  void *w_qkv_f = nullptr, *w_1_f = nullptr;
-  float *u_qkv = nullptr, *c_qkv = nullptr, *u_1 = nullptr, *c_1 = nullptr;
 };
 
 struct Batch;
@@ -89,7 +85,6 @@ struct Slot {
   int32_t *idx_all, *cur_tok, *tok_out, *prompt, *page_table;
   void *gemm_ws, *attn_ws;
   size_t gemm_ws_bytes, attn_ws_bytes;
-  float* ln_stats = nullptr;   // [64][2] folded-LN row statistics for the split-K fixup
   int32_t* h_page_table;   // pinned
   int32_t* h_prompt;       // pinned
   int32_t* h_tok_out;      // pinned
@@ -196,11 +191,7 @@ struct liger_ctx {
   // SMs a t > 1 GEMM leaves free for a concurrent all-reduce (LIGER_GEMM_SM_RESERVE,
   // liger_set_gemm_sm_reserve); the grid size never changes a GEMM's bits
   int gemm_sm_reserve = 0;
-  int th_parts = 1;
-  // decode passes at t = 1 (LIGER_LN_FOLD, default on): LN1 / LN2 folded into the
-  // QKV / FC1 GEMMs, residual adds into the out-proj / FC2 epilogues -- two
-  // kernels and two hand-offs per layer fewer
-  bool ln_fold = false;   // Inter-Th: projection GEMMs issued as this many partitioned kernels
+  int th_parts = 1;   // Inter-Th: projection GEMMs issued as this many partitioned kernels
   bool calibrating = false;   // liger_calibrate_cf at t = 1 (proxy communicator)
   int n_sms = 148;
   // stats / timing
@@ -452,7 +443,6 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
   const int M = batch_M(bt, pass);
   const int h = c->h;
   const float eps = c->cfg.ln_eps;
-  const bool fold = c->ln_fold && M <= 64;   // decode pass with LayerNorm folded into the GEMMs
   const int li = po.layer;
   const LayerW* W = li >= 0 ? &c->layers[li] : nullptr;
   int rc = 0;
@@ -502,7 +492,6 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_LN1: {
-      if (fold) break;   // folded into the QKV GEMM (the residual add happened in FC2's epilogue)
       timed_begin(c, st, &ta);
       if (li == c->l0)   // first layer of the model / of this pipeline stage: x is complete
         rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
@@ -517,7 +506,6 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       break;
     }
     case OP_LN2: {
-      if (fold) break;   // folded into the FC1 GEMM (the residual add happened in out-proj's epilogue)
       timed_begin(c, st, &ta);
       if (S.far_pending)
         rc = peer_add_ln(c, S, W->b_o, W->g2, W->be2, M, st);
@@ -554,27 +542,10 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       } else {
         g.x = S.hbuf; g.ldx = c->fl; g.w = W->w_2; g.ldw = K; g.out = S.part; g.ldo = h;
       }
-      if (fold) {
-        if (po.op == OP_QKV || po.op == OP_FC1) {   // LN folded: raw residual rows in, statistics in-kernel
-          const bool q = po.op == OP_QKV;
-          g.x = S.x;
-          g.w = q ? W->w_qkv_f : W->w_1_f;
-          g.ln_fold = 1;
-          g.ln_u = q ? W->u_qkv : W->u_1;
-          g.ln_c = q ? W->c_qkv : W->c_1;
-          g.bias = nullptr;   // in ln_c
-          g.ln_stats = S.ln_stats;
-          g.ln_eps = eps;
-        } else {   // residual stream updated in the epilogue: x += P + bias
-          g.out = S.x;
-          g.resid = S.x;
-          g.bias = po.op == OP_OUT ? W->b_o : W->b_2;
-        }
-      }
       // t = 1 (no all-reduce follows): leave the split-K partials of out-proj and of
       // FC2 (not the last layer's, which feeds the LM head / the next stage) to the
       // next add + LN, which sums them itself (bit-identical, one kernel fewer)
-      if (c->tp == 1 && c->fuse_split_ln && !fold && u0 == 0 && u1 == F &&
+      if (c->tp == 1 && c->fuse_split_ln && u0 == 0 && u1 == F &&
           (po.op == OP_OUT || (po.op == OP_FC2 && li + 1 < c->l1))) {
         const GemmPlan pl = gemm_plan(M, N, K);
         if (pl.splits > 1 && pl.cluster <= 1) {
@@ -659,9 +630,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       const LayerW& Wl = c->layers[c->L - 1];
       // residual add of the last layer + final LN on the last token of each sequence
       const int step = pass == 0 ? bt->s : 1, off = pass == 0 ? bt->s - 1 : 0;
-      // (folded decode pass: the last FC2 already added its output and bias to x)
-      rc = add_layernorm_launch(S.x, fold ? nullptr : S.part, fold ? nullptr : Wl.b_2, nullptr, S.yhead, c->lnf_g,
-                                c->lnf_b, b, h, step, off, eps, st);
+      rc = add_layernorm_launch(S.x, S.part, Wl.b_2, nullptr, S.yhead, c->lnf_g, c->lnf_b, b, h, step, off, eps, st);
       if (rc) break;
       GemmArgs g{};
       g.x = S.yhead; g.ldx = h;
@@ -948,10 +917,6 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   if (const char* fa = getenv("LIGER_FUSED_AR")) c->fused_ar = atoi(fa) != 0;
   if (const char* sr = getenv("LIGER_GEMM_SM_RESERVE")) c->gemm_sm_reserve = atoi(sr);
   {
-    const char* lf = getenv("LIGER_LN_FOLD");
-    c->ln_fold = (lf ? atoi(lf) != 0 : true) && c->tp == 1 && !c->pipe && !c->fused_decode;
-  }
-  {
     int dev = 0, n = 0;
     cudaGetDevice(&dev);
     if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && n > 0) c->n_sms = n;
@@ -988,15 +953,6 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     W.w_2 = dalloc(c, (size_t)pad128(c->h) * c->fl * 2);
     W.b_2 = dalloc(c, h * 2);
     W.g1 = dalloc(c, h * 2); W.be1 = dalloc(c, h * 2); W.g2 = dalloc(c, h * 2); W.be2 = dalloc(c, h * 2);
-    if (c->ln_fold) {
-      W.w_qkv_f = dalloc(c, (size_t)pad128(3 * c->hl) * h * 2);
-      W.w_1_f = dalloc(c, (size_t)pad128(c->fl) * h * 2);
-      W.u_qkv = (float*)dalloc(c, (size_t)3 * c->hl * 4);
-      W.c_qkv = (float*)dalloc(c, (size_t)3 * c->hl * 4);
-      W.u_1 = (float*)dalloc(c, (size_t)c->fl * 4);
-      W.c_1 = (float*)dalloc(c, (size_t)c->fl * 4);
-      if (!W.w_qkv_f || !W.w_1_f || !W.c_1) return fail(nullptr, LIGER_ENOMEM, "liger_init: folded LN weights");
-    }
     if (!W.w_qkv || !W.w_o || !W.w_1 || !W.w_2 || !W.be2)
       return fail(nullptr, LIGER_ENOMEM, "liger_init: out of device memory for weights");
   }
@@ -1031,7 +987,6 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     S.qkv = dalloc(c, (size_t)Mmax * 3 * c->hl * 2);
     S.attn = dalloc(c, (size_t)Mmax * c->hl * 2);
     S.part = dalloc(c, (size_t)Mmax * h * 2);
-    S.ln_stats = (float*)dalloc(c, 2 * 64 * sizeof(float));
     S.hbuf = dalloc(c, (size_t)Mmax * c->fl * 2);
     S.yhead = dalloc(c, (size_t)B * h * 2);
     S.logits = (float*)dalloc(c, (size_t)B * c->Vl * 4);
@@ -1089,35 +1044,6 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   return LIGER_OK;
 }
 
-// Fold LN1 into QKV and LN2 into FC1 (decode passes at t = 1):
-//   W x LN(x) = rstd * (W' x - mean * u) + c,   W' = W * gamma (per K column),
-//   u = W' . 1 (row sums of the bf16 W'),        c = W . beta + bias
-// (c and u by the library's own GEMM at M = 1 with fp32 output).
-static int fold_layer_norms(liger_ctx* c, LayerW& W, cudaStream_t st) {
-  const int h = c->h;
-  Slot& S = c->slots[0];
-  void* ones = S.yhead;   // [>= 1, h] bf16 scratch (unused outside the LM head)
-  {
-    std::vector<uint16_t> one((size_t)h, 0x3F80);   // bf16 1.0
-    if (cudaMemcpyAsync(ones, one.data(), (size_t)h * 2, cudaMemcpyHostToDevice, st) != cudaSuccess) return LIGER_ECUDA;
-    if (cudaStreamSynchronize(st) != cudaSuccess) return LIGER_ECUDA;
-  }
-  struct F { void *w, *wf, *g, *be, *b; float *u, *cc; int N; };
-  const F fs[2] = {{W.w_qkv, W.w_qkv_f, W.g1, W.be1, W.b_qkv, W.u_qkv, W.c_qkv, 3 * c->hl},
-                   {W.w_1, W.w_1_f, W.g2, W.be2, W.b_1, W.u_1, W.c_1, c->fl}};
-  for (const F& f : fs) {
-    GemmArgs g{};
-    g.M = 1; g.K = h; g.N = f.N; g.n0 = 0; g.n1 = f.N; g.ldx = h; g.ldw = h; g.ldo = f.N; g.scale = 1.0f;
-    g.out_f32 = 1; g.w_tiled = 1; g.workspace = S.gemm_ws; g.ws_bytes = S.gemm_ws_bytes;
-    g.x = f.be; g.w = f.w; g.bias = f.b; g.out = f.cc;   // c = W . beta + bias
-    if (int rc = gemm_launch(g, st)) return rc;
-    if (int rc = fold_gamma_tiled_launch(f.w, f.wf, f.g, f.N, h, st)) return rc;
-    g.x = ones; g.w = f.wf; g.bias = nullptr; g.out = f.u;   // u = W' . 1
-    if (int rc = gemm_launch(g, st)) return rc;
-  }
-  return cudaStreamSynchronize(st) == cudaSuccess ? 0 : LIGER_ECUDA;
-}
-
 int liger_load_layer(liger_ctx* c, int l, uint64_t seed) {
   if (!c || l < 0 || l >= c->L) return LIGER_EINVAL;
   if (l < c->l0 || l >= c->l1) return LIGER_OK;   // another pipeline stage's layer
@@ -1153,7 +1079,6 @@ int liger_load_layer(liger_ctx* c, int l, uint64_t seed) {
   CKR(c0_fill_launch(W.g2, 1, (int)h, h, seed, tid + 10, 0, 0, 0, 1, 0, 1, st));
   CKR(c0_fill_launch(W.be2, 1, (int)h, h, seed, tid + 11, 0, 0, 0, 1, 0, 2, st));
   (void)t;
-  if (c->ln_fold) CKR(fold_layer_norms(c, W, st));
   CK(cudaStreamSynchronize(st));
   return LIGER_OK;
 }

@@ -81,82 +81,9 @@ struct GemmParams {
   unsigned long long* pub_flag;
   unsigned int* pub_counter;
   unsigned long long pub_epoch;
-  // LayerNorm folded into the GEMM (decode, t = 1): W holds W*gamma; the epilogue
-  // computes v = rstd_m * (acc - mean_m * ln_u[n]) + ln_c[n] (ln_c = W.beta + bias)
-  // with mean_m / rstd_m of the raw input rows X[m, :] (which the kernel computes
-  // itself, and CTA 0 publishes in ln_stats for the split-K fixup)
-  int ln_fold;
-  const float* ln_u;
-  const float* ln_c;
-  float* ln_stats;                  // [M][2] (mean, rstd) written by CTA 0, read by the fixup
-  const __nv_bfloat16* ln_x;        // X (the rows to normalise), row stride ln_ldx
-  int64_t ln_ldx;
-  float ln_eps;
-  // residual add in the final store: out[m, n] = resid[m, n] + v (may alias out)
-  const __nv_bfloat16* resid;
 };
 
-// mean / rstd (two fp32 passes, population variance, eps inside the sqrt) of rows
-// m < M of X[M, K] into st[2m], st[2m + 1]; the calling threads are whole warps
-// (tid 0..nthreads-1), warp w takes rows w, w + nwarps, ...
-__device__ __forceinline__ void ln_row_stats(const __nv_bfloat16* X, int64_t ldx, int M, int K, float eps, float* st,
-                                             int tid, int nthreads) {
-  const int lane = tid & 31, w = tid >> 5, nw = nthreads >> 5;
-  const int nv = K >> 3;
-  for (int m = w; m < M; m += nw) {
-    const uint4* row = reinterpret_cast<const uint4*>(X + (int64_t)m * ldx);
-    float s = 0.f;
-    for (int v0 = lane; v0 < nv; v0 += 32 * 4) {
-      uint4 q[4];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-        if (v0 + i * 32 < nv) q[i] = __ldcg(row + v0 + i * 32);
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-        if (v0 + i * 32 < nv) {
-          const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&q[i]);
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const float2 f = __bfloat1622float2(h2[e]);
-            s += f.x + f.y;
-          }
-        }
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    const float mean = s / (float)K;
-    float q2 = 0.f;
-    for (int v0 = lane; v0 < nv; v0 += 32 * 4) {
-      uint4 q[4];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-        if (v0 + i * 32 < nv) q[i] = __ldcg(row + v0 + i * 32);
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-        if (v0 + i * 32 < nv) {
-          const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&q[i]);
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const float2 f = __bfloat1622float2(h2[e]);
-            q2 += (f.x - mean) * (f.x - mean) + (f.y - mean) * (f.y - mean);
-          }
-        }
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) q2 += __shfl_xor_sync(0xffffffffu, q2, o);
-    if (lane == 0) {
-      st[2 * m] = mean;
-      st[2 * m + 1] = 1.0f / sqrtf(q2 / (float)K + eps);
-    }
-  }
-}
-
-// EXT: the folded-LayerNorm / residual-add epilogue (a separate instantiation, so
-// the plain epilogue of the prefill GEMMs keeps its code)
-template <bool EXT>
-__device__ __forceinline__ float epi_apply(const GemmParams& p, float v, int m, int n, float bias_v,
-                                           const float* st) {
-  if (EXT && p.ln_fold) v = st[2 * m + 1] * (v - st[2 * m] * p.ln_u[n]) + p.ln_c[n];
+__device__ __forceinline__ float epi_apply(const GemmParams& p, float v, int n, float bias_v) {
   v += bias_v;
   if (n < p.scale_cols) v *= p.scale;
   if (p.act == LIGER_ACT_RELU) v = fmaxf(v, 0.0f);
@@ -164,9 +91,7 @@ __device__ __forceinline__ float epi_apply(const GemmParams& p, float v, int m, 
   return v;
 }
 
-template <bool EXT>
 __device__ __forceinline__ void epi_store(const GemmParams& p, int m, int n, float v) {
-  if (EXT && p.resid) v += __bfloat162float(p.resid[(int64_t)m * p.ldo + n]);
   if (p.out_f32)
     reinterpret_cast<float*>(p.out)[(int64_t)m * p.ldo + n] = v;
   else
@@ -189,7 +114,6 @@ __device__ __forceinline__ Unit unit_of(const GemmParams& p, int u) {
 }
 
 // Persistent: one CTA per SM, CTA i processes units i, i + G, i + 2G, ...
-template <bool EXT>
 __global__ void __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmParams p) {
@@ -349,16 +273,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     const int etid = threadIdx.x - 64;
     const int tiles = p.n_tiles * p.m_tiles;
     const uint32_t crank = cl ? cluster_ctarank() : 0;   // == the unit's K chunk z
-    float* lnst = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 512 + (cl ? 2 * BM * p.bn * 4 : 0));
-    if (EXT && p.ln_fold && (p.splits == 1 || cl || blockIdx.x == 0)) {
-      // row statistics of the raw input while the producer / MMA warps run the
-      // mainloop (X comes from the preceding kernel: wait for it first)
-      grid_dependency_wait();
-      ln_row_stats(p.ln_x, p.ln_ldx, p.M, p.K, p.ln_eps, lnst, etid, 128);
-      named_bar_sync(1, 128);
-      if (blockIdx.x == 0 && p.ln_stats)
-        for (int i = etid; i < 2 * p.M; i += 128) p.ln_stats[i] = lnst[i];
-    }
     int lu = 0;
     for (int u = blockIdx.x; u < p.units; u += G, ++lu) {
       const Unit w = unit_of(p, u);
@@ -386,8 +300,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
           if (nval) {
 #pragma unroll
             for (int j = 0; j < 16; ++j)
-              if (c0 + j < mcount)
-                epi_store<EXT>(p, m_base + c0 + j, n, epi_apply<EXT>(p, __uint_as_float(r[j]), m_base + c0 + j, n, bias_v, lnst));
+              if (c0 + j < mcount) epi_store(p, m_base + c0 + j, n, epi_apply(p, __uint_as_float(r[j]), n, bias_v));
           }
         } else if (cl) {
 #pragma unroll
@@ -436,7 +349,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
             const int nn = n_base + rq * 4 + i;
             if (nn < p.n1 && nn < p.N) {
               const float bv = p.bias ? __bfloat162float(p.bias[nn]) : 0.0f;
-              epi_store<EXT>(p, m_base + col, nn, epi_apply<EXT>(p, av[i], m_base + col, nn, bv, lnst));
+              epi_store(p, m_base + col, nn, epi_apply(p, av[i], nn, bv));
             }
           }
         }
@@ -479,12 +392,10 @@ __device__ __forceinline__ float sum_partials(const float* src, int64_t zstride,
 // Split-K fixup: out[m, n] = epi( sum_{z=0..S-1} partial[z] ) in chunk order (the
 // same bits whatever slice or CTA produced each chunk).  One thread per (m, 4 rows n),
 // reading the column-major per-tile partials coalesced.
-template <bool EXT>
 __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) {
   const uint64_t tr0 = trace_now();
   pdl_enter();
   const uint64_t tr1 = trace_now();
-  const float* lnst = p.ln_stats;   // written by the GEMM's CTA 0 (complete: PDL wait above)
   const int tiles = p.n_tiles * p.m_tiles;
   const int64_t zstride = (int64_t)tiles * (BM * p.bn);
   const int slice_w = p.n1 - p.n0;
@@ -526,7 +437,7 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
       const int n = p.n0 + nt * BM + row;
       if (nt * BM + row < slice_w && n < p.N) {
         const float bias_v = p.bias ? __bfloat162float(p.bias[n]) : 0.0f;
-        epi_store<EXT>(p, m, n, epi_apply<EXT>(p, a[i], m, n, bias_v, lnst));
+        epi_store(p, m, n, epi_apply(p, a[i], n, bias_v));
       }
     }
   }
@@ -656,9 +567,8 @@ static int cluster_red_bytes(int bn) { return 2 * BM * bn * (int)sizeof(float); 
 // Cluster (decode) mode runs two CTAs per SM: a CTA gets half of the SM's 228 KiB
 // minus the 1 KiB the hardware reserves per CTA.
 constexpr int CLUSTER_CTA_SMEM = 233472 / 2 - 1024;
-constexpr int LN_STATS_SMEM = 2 * 64 * 4;   // folded-LayerNorm row statistics (M <= 64)
 static int cluster_smem(int bn) {
-  const int red = cluster_red_bytes(bn) + LN_STATS_SMEM;
+  const int red = cluster_red_bytes(bn);
   return 1024 + stages_for(bn, red, CLUSTER_CTA_SMEM) * (A_BYTES + bn * BK * 2) + 512 + red;
 }
 
@@ -671,8 +581,8 @@ static int max_clusters(int S, int bn) {
   std::lock_guard<std::mutex> g(mu);
   auto it = cache.find(key);
   if (it != cache.end()) return it->second;
-  cudaFuncSetAttribute(gemm_tc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
-  cudaFuncSetAttribute(gemm_tc_kernel<false>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
+  cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(S * 128);
   cfg.blockDim = dim3(GEMM_THREADS);
@@ -685,7 +595,7 @@ static int max_clusters(int S, int bn) {
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   int n = 0;
-  if (cudaOccupancyMaxActiveClusters(&n, gemm_tc_kernel<false>, &cfg) != cudaSuccess || n <= 0) {
+  if (cudaOccupancyMaxActiveClusters(&n, gemm_tc_kernel, &cfg) != cudaSuccess || n <= 0) {
     cudaGetLastError();
     n = 0;   // cluster mode unavailable for this S
   }
@@ -786,11 +696,11 @@ GemmPlan gemm_plan(int M, int N, int K) {
   pl.cluster = (use_cluster && pl.splits > 1 && best_nc > 0) ? pl.splits : 1;
   pl.clusters = pl.cluster > 1 ? best_nc : 0;
   if (pl.cluster > 1) {
-    pl.stages = stages_for(bn, cluster_red_bytes(bn) + LN_STATS_SMEM, CLUSTER_CTA_SMEM);
+    pl.stages = stages_for(bn, cluster_red_bytes(bn), CLUSTER_CTA_SMEM);
     pl.smem = cluster_smem(bn);
   } else {
-    pl.stages = stages_for(bn, LN_STATS_SMEM, MAX_SMEM);
-    pl.smem = 1024 + pl.stages * (A_BYTES + pl.bn * BK * 2) + 512 + LN_STATS_SMEM;
+    pl.stages = stages_for(bn, 0, MAX_SMEM);
+    pl.smem = 1024 + pl.stages * (A_BYTES + pl.bn * BK * 2) + 512;
   }
   return pl;
 }
@@ -826,10 +736,8 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (rc) return rc;
   static bool attr_set = false;
   if (!attr_set) {
-    for (auto k : {gemm_tc_kernel<false>, gemm_tc_kernel<true>}) {
-      cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
-      cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-    }
+    cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
+    cudaFuncSetAttribute(gemm_tc_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     attr_set = true;
   }
   GemmParams p;
@@ -839,11 +747,6 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.act = a.act; p.scale_cols = a.scale_cols; p.scale = a.scale;
   p.out = a.out; p.ldo = a.ldo; p.out_f32 = a.out_f32;
   p.pub_flag = nullptr; p.pub_counter = nullptr; p.pub_epoch = 0;
-  p.ln_fold = a.ln_fold; p.ln_u = a.ln_u; p.ln_c = a.ln_c; p.ln_stats = a.ln_stats;
-  p.ln_x = reinterpret_cast<const __nv_bfloat16*>(a.x); p.ln_ldx = a.ldx; p.ln_eps = a.ln_eps;
-  p.resid = reinterpret_cast<const __nv_bfloat16*>(a.resid);
-  if (a.ln_fold && (a.M > 64 || !a.ln_u || !a.ln_c || (pl.splits > 1 && !a.ln_stats) || a.K % 8)) return LIGER_EINVAL;
-  const bool ext = a.ln_fold || a.resid;
   if (a.far) {   // fused all-reduce producer: needs the fixup kernel and the whole GEMM
     if (pl.splits <= 1 || pl.cluster > 1 || a.defer_fixup || a.out_f32 || a.n0 != 0 || a.n1 != a.N)
       return LIGER_EINVAL;
@@ -870,16 +773,13 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
     // one cluster of `splits` CTAs per tile in flight; CTA z of a cluster takes chunk z
     // (grid = clusters x S, so unit u = blockIdx.x + j * grid keeps z = blockIdx.x % S)
     const int nc = std::min(pl.clusters, ntiles * pl.m_tiles);
-    rc2 = ext ? launch_pdl_cluster(gemm_tc_kernel<true>, dim3(nc * pl.cluster), dim3(GEMM_THREADS), pl.cluster,
-                                   pl.smem, stream, tA, tB, p)
-              : launch_pdl_cluster(gemm_tc_kernel<false>, dim3(nc * pl.cluster), dim3(GEMM_THREADS), pl.cluster,
-                                   pl.smem, stream, tA, tB, p);
+    rc2 = launch_pdl_cluster(gemm_tc_kernel, dim3(nc * pl.cluster), dim3(GEMM_THREADS), pl.cluster, pl.smem, stream,
+                             tA, tB, p);
   } else {
     // unit u runs on CTA u % grid: the grid size never changes what a unit computes
     const int sms = (a.sm_budget > 0 && a.sm_budget < num_sms()) ? a.sm_budget : num_sms();
     const int grid = p.units < sms ? p.units : sms;
-    rc2 = ext ? launch_pdl(gemm_tc_kernel<true>, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p)
-              : launch_pdl(gemm_tc_kernel<false>, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
+    rc2 = launch_pdl(gemm_tc_kernel, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
   }
   const bool fixup = p.splits > 1 && pl.cluster <= 1 && !a.defer_fixup;
   if (a.had_fixup) *a.had_fixup = fixup;
@@ -888,10 +788,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   const int64_t work = (int64_t)p.M * (BM / 4) * p.n_tiles;
   int rblocks = (int)((work + 255) / 256);
   if (rblocks > num_sms() * 8) rblocks = num_sms() * 8;
-  return (ext ? launch_pdl(splitk_reduce_kernel<true>, dim3(rblocks), dim3(256), 0, stream, p)
-              : launch_pdl(splitk_reduce_kernel<false>, dim3(rblocks), dim3(256), 0, stream, p))
-             ? LIGER_ECUDA
-             : 0;
+  return launch_pdl(splitk_reduce_kernel, dim3(rblocks), dim3(256), 0, stream, p) ? LIGER_ECUDA : 0;
 }
 
 LIGER_TRACE_SETTER(gemm)

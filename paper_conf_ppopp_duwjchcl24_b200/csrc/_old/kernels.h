@@ -61,17 +61,6 @@ struct GemmArgs {
   // SM budget of the persistent GEMM grid (0 = every SM): leaves SMs to a
   // communication kernel running concurrently (contention control)
   int sm_budget = 0;
-  // LayerNorm folded into the GEMM (M <= 64): W holds W*gamma (per K column), the
-  // epilogue applies v = rstd_m (acc - mean_m u[n]) + c[n] with the statistics of
-  // the raw input rows x; u = W'.1, c = W.beta (+ bias folded by the caller, bias = 0).
-  // ln_stats: [M][2] fp32 scratch the split-K fixup reads the statistics from.
-  int ln_fold = 0;
-  const float* ln_u = nullptr;
-  const float* ln_c = nullptr;
-  float* ln_stats = nullptr;
-  float ln_eps = 1e-5f;
-  // residual add in the final store: out[m, n] = resid[m, n] + epilogue(v) (may alias out)
-  const void* resid = nullptr;
 };
 
 GemmPlan gemm_plan(int M, int N, int K);
@@ -138,8 +127,6 @@ int c0_fill_launch(void* dst, int rows, int cols, int64_t ld, uint64_t seed, uin
                    cudaStream_t stream);
 int copy_tokens_launch(const int32_t* src, int32_t* dst, int n, cudaStream_t stream);
 int tile_weight_launch(const void* src, int64_t ld, void* dst, int N, int K, cudaStream_t stream);
-// dst = bf16(src * gamma[k]) for a tiled [ceil(N/128)][K/64][128][64] weight (may alias)
-int fold_gamma_tiled_launch(const void* src, void* dst, const void* gamma, int N, int K, cudaStream_t stream);
 // storage offset (elements) of logical W[n, k] in the tiled layout
 inline __host__ __device__ int64_t tiled_offset(int n, int k, int K) {
   return (((int64_t)(n >> 7) * (K >> 6) + (k >> 6)) << 13) + ((n & 127) << 6) + (k & 63);

@@ -476,22 +476,6 @@ int tile_weight_launch(const void* src, int64_t ld, void* dst, int N, int K, cud
   return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
 }
 
-// tiled element e: k = ((e / 8192) % (K / 64)) * 64 + e % 64 (kernels.h tiled_offset)
-__global__ void fold_gamma_tiled_kernel(const __nv_bfloat16* src, __nv_bfloat16* dst, const __nv_bfloat16* gamma,
-                                        int64_t total, int kb) {
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
-    const int k = (int)((e >> 13) % kb) * 64 + (int)(e & 63);
-    dst[e] = __float2bfloat16_rn(__bfloat162float(src[e]) * __bfloat162float(gamma[k]));
-  }
-}
-int fold_gamma_tiled_launch(const void* src, void* dst, const void* gamma, int N, int K, cudaStream_t stream) {
-  if (K % 64 || N <= 0) return LIGER_EINVAL;
-  const int64_t total = (int64_t)(N + 127) / 128 * 128 * K;
-  fold_gamma_tiled_kernel<<<148 * 8, 256, 0, stream>>>((const __nv_bfloat16*)src, (__nv_bfloat16*)dst,
-                                                       (const __nv_bfloat16*)gamma, total, K / 64);
-  return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
-}
-
 __global__ void copy_i32_kernel(const int32_t* s, int32_t* d, int n) {
   int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) d[i] = s[i];

@@ -125,3 +125,57 @@ def test_nccl_oneshot_setup_and_kernel_single_rank(E):
         os.environ.pop("LIGER_ONESHOT_AR", None)
     assert 1.0 <= cf < 10.0
     assert res.done == 1 and toks.shape == (2, 3) and toks_ok
+
+
+_FOLD_CHILD = r"""
+import sys, numpy as np
+sys.path.insert(0, {root!r})
+from liger_inputs import make_trace, get_config
+from liger_inputs.configs import ModelConfig
+from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
+cfg = {cfg}
+trace = make_trace(3, float("inf"), seed=4, batch_sizes=(2, 5), prompt_range=(20, 60), n_decode=6, vocab=cfg.vocab)
+eng = LigerEngine(cfg, mode="interleaved", max_batch=8, max_seq=64, max_new=8, seed=7)
+ids = [eng.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], 0.0) for t in trace]
+eng.drain()
+print(repr([eng.poll(i, want_tokens=True)[1].tolist() for i in ids]))
+eng.close()
+"""
+
+
+@pytest.mark.parametrize("cfg_expr", ['ModelConfig("mid3", 3, 1024, 8, 4096, 1024, 96, "relu")',
+                                      'ModelConfig("tiny3g", 3, 256, 4, 1024, 512, 96, "gelu_tanh")'])
+def test_ln_fold_decode_matches_oracle(E, cfg_expr):
+    """t = 1 decode passes with LayerNorm folded into the QKV / FC1 GEMMs
+    (W*gamma weights, in-kernel row statistics, u / c epilogue vectors) and the
+    residual adds in the out-proj / FC2 epilogues -- default -- against the fp64
+    oracle's greedy tokens (where its top-2 margin is clear), and against the
+    unfolded path (LIGER_LN_FOLD=0).  h = 1024 exercises the split-K fixup path,
+    h = 256 the single-chunk epilogue path."""
+    import ast
+    import os
+    import subprocess
+    import sys
+    from liger_inputs.configs import ModelConfig
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = {}
+    for flag in ("1", "0"):
+        p = subprocess.run([sys.executable, "-c", _FOLD_CHILD.format(root=root, cfg=cfg_expr)],
+                           env={**os.environ, "LIGER_LN_FOLD": flag}, capture_output=True, text=True, timeout=600)
+        assert p.returncode == 0, p.stderr[-2000:]
+        res[flag] = ast.literal_eval(p.stdout.strip().splitlines()[-1])
+    cfg = eval(cfg_expr)
+    trace = make_trace(3, float("inf"), seed=4, batch_sizes=(2, 5), prompt_range=(20, 60), n_decode=6,
+                       vocab=cfg.vocab)
+    agree = total = 0
+    for t, got1, got0 in zip(trace, res["1"], res["0"]):
+        pr = t["tokens"].reshape(t["batch"], t["seq_len"])
+        ref, logits = om.greedy_generate(cfg, 7, pr, t["n_decode"], return_logits=True)
+        ok = om.top2_margin(logits) > 0.02 * np.sqrt((logits ** 2).mean())
+        for i in range(t["batch"]):
+            n = int(np.argmin(ok[i])) if not ok[i].all() else t["n_decode"]
+            assert np.array_equal(np.array(got1)[i, :n], ref[i, :n])
+            assert np.array_equal(np.array(got0)[i, :n], ref[i, :n])
+            agree += int(np.sum(np.array(got1)[i] == np.array(got0)[i]))
+            total += t["n_decode"]
+    assert agree >= 0.9 * total

@@ -127,6 +127,7 @@ def test_engine_fused_tokens_equal_per_op_and_oracle():
     out = {}
     for fused in ("1", "0"):
         os.environ["LIGER_FUSED_DECODE"] = fused
+        os.environ["LIGER_LN_FOLD"] = "0"   # the fused pass reproduces the unfolded per-kernel path
         try:
             eng = LigerEngine(cfg, mode="serial", max_batch=4, max_seq=32, max_new=8, seed=0)
             bid = eng.submit(prompt.reshape(-1).astype(np.int32), 3, 20, 8, 0.0)
@@ -136,6 +137,7 @@ def test_engine_fused_tokens_equal_per_op_and_oracle():
             eng.close()
         finally:
             os.environ.pop("LIGER_FUSED_DECODE", None)
+            os.environ.pop("LIGER_LN_FOLD", None)
         out[fused] = toks
         assert st["gpu_launches"] > 0
     assert np.array_equal(out["1"], out["0"])   # fused (opt-in) and per-kernel engines agree
