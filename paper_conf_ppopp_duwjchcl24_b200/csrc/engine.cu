@@ -706,10 +706,13 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
     }
     case OP_SEND_X: {
       // complete the residual stream of the stage's last layer (x += FC2 + b_2), then send it on
-      rc = add_layernorm_launch(S.x, S.part, c->layers[c->l1 - 1].b_2, S.x, S.y, c->lnf_g, c->lnf_b, M, h, 1, 0,
-                                eps, st);
-      if (rc) break;
-      c->st.gpu_launches++;
+      // (a folded decode pass did that in FC2's epilogue)
+      if (!fold) {
+        rc = add_layernorm_launch(S.x, S.part, c->layers[c->l1 - 1].b_2, S.x, S.y, c->lnf_g, c->lnf_b, M, h, 1, 0,
+                                  eps, st);
+        if (rc) break;
+        c->st.gpu_launches++;
+      }
       if (c->comm->send(S.x, (size_t)M * h * 2, c->rank + 1, st)) return fail(c, LIGER_ENCCL, c->comm->err);
       c->st.comm_kernels++;
       break;
@@ -949,7 +952,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   if (const char* sr = getenv("LIGER_GEMM_SM_RESERVE")) c->gemm_sm_reserve = atoi(sr);
   {
     const char* lf = getenv("LIGER_LN_FOLD");
-    c->ln_fold = (lf ? atoi(lf) != 0 : true) && c->tp == 1 && !c->pipe && !c->fused_decode;
+    c->ln_fold = (lf ? atoi(lf) != 0 : true) && c->tp == 1 && !c->fused_decode;
   }
   {
     int dev = 0, n = 0;
