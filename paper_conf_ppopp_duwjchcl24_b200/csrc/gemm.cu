@@ -96,57 +96,47 @@ struct GemmParams {
   const __nv_bfloat16* resid;
 };
 
-// mean / rstd (two fp32 passes, population variance, eps inside the sqrt) of rows
-// m < M of X[M, K] into st[2m], st[2m + 1]; the calling threads are whole warps
-// (tid 0..nthreads-1), warp w takes rows w, w + nwarps, ...
+// mean / rstd (population variance, eps inside the sqrt) of rows m < M of X[M, K]
+// into st[2m], st[2m + 1]: one fp32 pass over the row, shifted by its first element
+// (s1 = sum(x - x0), s2 = sum((x - x0)^2); mean = x0 + s1/K, var = s2/K - (s1/K)^2),
+// which keeps the cancellation of the one-pass form small.  The calling threads are
+// whole warps (tid 0..nthreads-1); warp w takes rows w, w + nwarps, ...
 __device__ __forceinline__ void ln_row_stats(const __nv_bfloat16* X, int64_t ldx, int M, int K, float eps, float* st,
                                              int tid, int nthreads) {
   const int lane = tid & 31, w = tid >> 5, nw = nthreads >> 5;
   const int nv = K >> 3;
   for (int m = w; m < M; m += nw) {
-    const uint4* row = reinterpret_cast<const uint4*>(X + (int64_t)m * ldx);
-    float s = 0.f;
-    for (int v0 = lane; v0 < nv; v0 += 32 * 4) {
-      uint4 q[4];
+    const __nv_bfloat16* rowp = X + (int64_t)m * ldx;
+    const uint4* row = reinterpret_cast<const uint4*>(rowp);
+    const float x0 = __bfloat162float(rowp[0]);
+    float s1 = 0.f, s2 = 0.f;
+    for (int v0 = lane; v0 < nv; v0 += 32 * 8) {
+      uint4 q[8];
 #pragma unroll
-      for (int i = 0; i < 4; ++i)
+      for (int i = 0; i < 8; ++i)
         if (v0 + i * 32 < nv) q[i] = __ldcg(row + v0 + i * 32);
 #pragma unroll
-      for (int i = 0; i < 4; ++i)
+      for (int i = 0; i < 8; ++i)
         if (v0 + i * 32 < nv) {
           const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&q[i]);
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
             const float2 f = __bfloat1622float2(h2[e]);
-            s += f.x + f.y;
+            const float a = f.x - x0, b = f.y - x0;
+            s1 += a + b;
+            s2 += a * a + b * b;
           }
         }
     }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    const float mean = s / (float)K;
-    float q2 = 0.f;
-    for (int v0 = lane; v0 < nv; v0 += 32 * 4) {
-      uint4 q[4];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-        if (v0 + i * 32 < nv) q[i] = __ldcg(row + v0 + i * 32);
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-        if (v0 + i * 32 < nv) {
-          const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&q[i]);
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const float2 f = __bfloat1622float2(h2[e]);
-            q2 += (f.x - mean) * (f.x - mean) + (f.y - mean) * (f.y - mean);
-          }
-        }
+    for (int o = 16; o > 0; o >>= 1) {
+      s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+      s2 += __shfl_xor_sync(0xffffffffu, s2, o);
     }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) q2 += __shfl_xor_sync(0xffffffffu, q2, o);
     if (lane == 0) {
-      st[2 * m] = mean;
-      st[2 * m + 1] = 1.0f / sqrtf(q2 / (float)K + eps);
+      const float d = s1 / (float)K;
+      st[2 * m] = x0 + d;
+      st[2 * m + 1] = 1.0f / sqrtf(fmaxf(s2 / (float)K - d * d, 0.0f) + eps);
     }
   }
 }
@@ -350,14 +340,18 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     const int tiles = p.n_tiles * p.m_tiles;
     const uint32_t crank = cl ? cluster_ctarank() : 0;   // == the unit's K chunk z
     float* lnst = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 512 + (cl ? 2 * BM * p.bn * 4 : 0));
-    if (EXT && p.ln_fold && (p.splits == 1 || cl || blockIdx.x == 0)) {
+    if (EXT && p.ln_fold) {
       // row statistics of the raw input while the producer / MMA warps run the
       // mainloop (X comes from the preceding kernel: wait for it first)
       grid_dependency_wait();
-      ln_row_stats(p.ln_x, p.ln_ldx, p.M, p.K, p.ln_eps, lnst, etid, 128);
-      named_bar_sync(1, 128);
-      if (blockIdx.x == 0 && p.ln_stats)
-        for (int i = etid; i < 2 * p.M; i += 128) p.ln_stats[i] = lnst[i];
+      if (p.splits == 1 || cl) {   // this CTA's epilogue applies the fold: every row here
+        ln_row_stats(p.ln_x, p.ln_ldx, p.M, p.K, p.ln_eps, lnst, etid, 128);
+        named_bar_sync(1, 128);
+      } else {
+        // the fixup applies it: CTA b publishes rows b, b + G, ... (one warp per row)
+        for (int m = blockIdx.x + (etid >> 5) * G; m < p.M; m += 4 * G)
+          ln_row_stats(p.ln_x + (int64_t)m * p.ln_ldx, p.ln_ldx, 1, p.K, p.ln_eps, p.ln_stats + 2 * m, lane, 32);
+      }
     }
     int lu = 0;
     for (int u = blockIdx.x; u < p.units; u += G, ++lu) {
