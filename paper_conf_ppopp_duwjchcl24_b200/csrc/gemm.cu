@@ -41,6 +41,9 @@ constexpr int BK = 64;            // K per stage (one 128-byte swizzle atom)
 constexpr int A_BYTES = BM * BK * 2;
 constexpr int GEMM_THREADS = 192;
 constexpr int MAX_SMEM = 227 * 1024;
+constexpr int GEMM_MAX_READY_TILES = 2048;
+constexpr int GEMM_STATS_CNT = 2048;
+constexpr int GEMM_DONE_CNT = 2049;
 
 static int num_sms() {
   static int n = 0;
@@ -73,6 +76,10 @@ struct GemmParams {
   int out_f32;
   float* ws;
   int* counters;
+  // split-K readiness (workspace counter region, zero between uses): tile_ready[t]
+  // counts the chunks of tile t written, [GEMM_STATS_CNT] the folded-LN rows whose
+  // statistics are out, [GEMM_DONE_CNT] the fixup CTAs done (the last one re-zeroes)
+  unsigned int* tile_ready;
   const void* w_base;   // tiled weights (for the L2 prefetch)
   int pf_blocks;        // weight blocks (beyond the smem stages) prefetched into L2 before the PDL wait
   int cluster;          // > 1: split-K reduced in-kernel across a (splits x 1 x 1) thread-block cluster
@@ -139,6 +146,12 @@ __device__ __forceinline__ void ln_row_stats(const __nv_bfloat16* X, int64_t ldx
       st[2 * m + 1] = 1.0f / sqrtf(fmaxf(s2 / (float)K - d * d, 0.0f) + eps);
     }
   }
+}
+
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
 }
 
 // EXT: the folded-LayerNorm / residual-add epilogue (a separate instantiation, so
@@ -349,8 +362,14 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         named_bar_sync(1, 128);
       } else {
         // the fixup applies it: CTA b publishes rows b, b + G, ... (one warp per row)
-        for (int m = blockIdx.x + (etid >> 5) * G; m < p.M; m += 4 * G)
+        for (int m = blockIdx.x + (etid >> 5) * G; m < p.M; m += 4 * G) {
           ln_row_stats(p.ln_x + (int64_t)m * p.ln_ldx, p.ln_ldx, 1, p.K, p.ln_eps, p.ln_stats + 2 * m, lane, 32);
+          __syncwarp();
+          if (lane == 0 && p.tile_ready) {   // row m's statistics are out (the fixup waits for all M)
+            __threadfence();
+            atomicAdd(p.tile_ready + GEMM_STATS_CNT, 1u);
+          }
+        }
       }
     }
     int lu = 0;
@@ -397,6 +416,15 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tmem_empty[acc]);
+      if (p.splits > 1 && !cl && p.tile_ready) {
+        // chunk w.z of this tile is in the workspace: count it (the fixup reduces a
+        // tile as soon as all its chunks have arrived, during this grid's tail)
+        named_bar_sync(2, 128);
+        if (etid == 0) {
+          __threadfence();
+          atomicAdd(&p.tile_ready[tile_id], 1u);
+        }
+      }
       if (cl) {
         // In-cluster split-K reduction (replaces the fixup kernel): the S CTAs of the
         // cluster hold chunks z = 0..S-1 of this tile in shared memory; CTA z sums
@@ -476,9 +504,19 @@ __device__ __forceinline__ float sum_partials(const float* src, int64_t zstride,
 template <bool EXT>
 __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) {
   const uint64_t tr0 = trace_now();
-  pdl_enter();
+  // With tile_ready, a tile is reduced as soon as all its chunks are in (acquire on
+  // its counter), overlapping the GEMM grid's tail; the wait for the GEMM grid to
+  // complete comes at the end, so this kernel's completion still implies the
+  // GEMM's.  Without it (tile count beyond the counter region): wait up front.
+  const bool early = p.tile_ready != nullptr;
+  if (!early) pdl_enter();
+  else grid_dependency_trigger();   // the next GEMM's weight prefetch overlaps this kernel, as before
   const uint64_t tr1 = trace_now();
-  const float* lnst = p.ln_stats;   // written by the GEMM's CTA 0 (complete: PDL wait above)
+  const float* lnst = p.ln_stats;
+  if (EXT && early && p.ln_fold && (threadIdx.x & 31) == 0) {   // every row's statistics are out
+    while (ld_acquire_u32(p.tile_ready + GEMM_STATS_CNT) < (unsigned)p.M) __nanosleep(200);
+  }
+  __syncwarp();
   const int tiles = p.n_tiles * p.m_tiles;
   const int64_t zstride = (int64_t)tiles * (BM * p.bn);
   const int slice_w = p.n1 - p.n0;
@@ -490,6 +528,11 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
     const int m = (int)(t2 / p.n_tiles);
     const int mt = m / p.bn, col = m % p.bn;
     const int tile_id = nt * p.m_tiles + mt;
+    if (early) {   // warp-uniform: a warp covers the 32 row groups of one (m, tile)
+      if ((threadIdx.x & 31) == 0)
+        while (ld_acquire_u32(p.tile_ready + tile_id) < (unsigned)p.splits) __nanosleep(200);
+      __syncwarp();
+    }
     const float4* src = reinterpret_cast<const float4*>(p.ws + (int64_t)tile_id * (BM * p.bn) + (int64_t)col * BM) + rq;
     // chunk order z = 0..S-1; a group of 8 chunks' loads are all in flight before the adds
     float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -521,6 +564,20 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
       if (nt * BM + row < slice_w && n < p.N) {
         const float bias_v = p.bias ? __bfloat162float(p.bias[n]) : 0.0f;
         epi_store<EXT>(p, m, n, epi_apply<EXT>(p, a[i], m, n, bias_v, lnst));
+      }
+    }
+  }
+  if (early) {
+    grid_dependency_wait();   // the GEMM grid has completed (its dependents may rely on that)
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      if (atomicAdd(p.tile_ready + GEMM_DONE_CNT, 1u) == gridDim.x - 1) {   // last CTA: re-zero the counters
+        const int tiles_all = p.n_tiles * p.m_tiles;
+        for (int t = 0; t < tiles_all; ++t) p.tile_ready[t] = 0;
+        p.tile_ready[GEMM_STATS_CNT] = 0;
+        p.tile_ready[GEMM_DONE_CNT] = 0;
+        __threadfence();
       }
     }
   }
@@ -848,6 +905,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
     p.pub_epoch = a.far->epoch;
   }
   p.counters = reinterpret_cast<int*>(a.workspace);
+  p.tile_ready = nullptr;
   p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
   p.w_tiled = a.w_tiled;
   p.w_base = a.w;
@@ -858,6 +916,17 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   p.n_tiles = ntiles;
   p.m_tiles = pl.m_tiles;
   p.units = ntiles * pl.m_tiles * pl.splits;
+  {
+    // early fixup (opt-in LIGER_EARLY_FIXUP=1; tile readiness counters in the
+    // workspace's counter region): the fixup reduces each tile as soon as its chunks
+    // are in, during the GEMM grid's tail.  Bit-identical, but measured slower
+    // (OPT-13B decode pass 5635 vs 5181 us at b = 2, 6132 vs 5634 at b = 8): the
+    // fixup CTAs launched next to the persistent GEMM poll and occupy SM slots.
+    static const bool early_env = getenv("LIGER_EARLY_FIXUP") ? atoi(getenv("LIGER_EARLY_FIXUP")) != 0 : false;
+    const bool will_fixup = pl.splits > 1 && pl.cluster <= 1 && !a.defer_fixup;
+    if (will_fixup && early_env && a.workspace && ntiles * pl.m_tiles <= GEMM_MAX_READY_TILES)
+      p.tile_ready = reinterpret_cast<unsigned int*>(a.workspace);
+  }
   p.cluster = pl.cluster;
   int rc2;
   if (pl.cluster > 1) {
