@@ -442,3 +442,25 @@ def test_engine_split_ln_fusion_bit_exact_and_oracle(L):
     for i in range(t["batch"]):
         n = int(np.argmin(ok[i])) if not ok[i].all() else t["n_decode"]
         assert np.array_equal(got[i, :n], ref[i, :n])
+
+
+def test_gemm_early_fixup_bit_exact(L):
+    """Opt-in LIGER_EARLY_FIXUP=1: the split-K fixup reduces each tile as soon as its
+    chunks are counted in (per-tile readiness counters) instead of after the whole
+    GEMM grid -- same chunk order, so the same bits as the default fixup."""
+    import ast
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    shapes = [(8, 5120, 5120), (8, 5120, 20480), (8, 20480, 5120), (3, 1000, 2560), (33, 640, 4096)]
+    code = _CLUSTER_CHILD.format(root=root, shapes=shapes)
+    res = {}
+    for flag in ("1", "0"):
+        p = subprocess.run([sys.executable, "-c", code], env={**os.environ, "LIGER_EARLY_FIXUP": flag},
+                           capture_output=True, text=True, timeout=300)
+        assert p.returncode == 0, p.stderr[-2000:]
+        res[flag] = ast.literal_eval(p.stdout.strip().splitlines()[-1])
+    assert any(pl["splits"] > 1 for pl, _ in res["1"])
+    for (p1, h1), (p0, h0), s in zip(res["1"], res["0"], shapes):
+        assert p1 == p0 and h1 == h0, s
