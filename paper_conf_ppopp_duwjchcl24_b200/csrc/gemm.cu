@@ -509,6 +509,35 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
   // complete comes at the end, so this kernel's completion still implies the
   // GEMM's.  Without it (tile count beyond the counter region): wait up front.
   const bool early = p.tile_ready != nullptr;
+  const int tiles = p.n_tiles * p.m_tiles;
+  const int64_t zstride = (int64_t)tiles * (BM * p.bn);
+  const int slice_w = p.n1 - p.n0;
+  const int64_t total = (int64_t)p.M * (BM / 4) * p.n_tiles;   // (m, tile row group of 4)
+  const int64_t t_first = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  // The epilogue operands of this thread's first item (usually its only one) do not
+  // depend on the GEMM -- bias, the folded-LN vectors, and the residual rows, written
+  // by a fixup at least three kernels back -- so they are loaded before the PDL wait.
+  float pb[4] = {0.f, 0.f, 0.f, 0.f}, pu[4] = {0.f, 0.f, 0.f, 0.f}, pc[4] = {0.f, 0.f, 0.f, 0.f},
+        pr[4] = {0.f, 0.f, 0.f, 0.f};
+  if (!early && t_first < total) {
+    const int rq = (int)(t_first % (BM / 4));
+    const int64_t t2 = t_first / (BM / 4);
+    const int nt = (int)(t2 % p.n_tiles);
+    const int m = (int)(t2 / p.n_tiles);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int row = rq * 4 + i;
+      const int n = p.n0 + nt * BM + row;
+      if (nt * BM + row < slice_w && n < p.N) {
+        if (p.bias) pb[i] = __bfloat162float(p.bias[n]);
+        if (EXT && p.ln_fold) {
+          pu[i] = p.ln_u[n];
+          pc[i] = p.ln_c[n];
+        }
+        if (EXT && p.resid) pr[i] = __bfloat162float(p.resid[(int64_t)m * p.ldo + n]);
+      }
+    }
+  }
   if (!early) pdl_enter();
   else grid_dependency_trigger();   // the next GEMM's weight prefetch overlaps this kernel, as before
   const uint64_t tr1 = trace_now();
@@ -517,11 +546,7 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
     while (ld_acquire_u32(p.tile_ready + GEMM_STATS_CNT) < (unsigned)p.M) __nanosleep(200);
   }
   __syncwarp();
-  const int tiles = p.n_tiles * p.m_tiles;
-  const int64_t zstride = (int64_t)tiles * (BM * p.bn);
-  const int slice_w = p.n1 - p.n0;
-  const int64_t total = (int64_t)p.M * (BM / 4) * p.n_tiles;   // (m, tile row group of 4)
-  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+  for (int64_t t = t_first; t < total; t += (int64_t)gridDim.x * blockDim.x) {
     const int rq = (int)(t % (BM / 4));
     const int64_t t2 = t / (BM / 4);
     const int nt = (int)(t2 % p.n_tiles);
@@ -557,13 +582,28 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
         }
     }
     const float a[4] = {acc.x, acc.y, acc.z, acc.w};
+    const bool pre = !early && t == t_first;
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
       const int row = rq * 4 + i;
       const int n = p.n0 + nt * BM + row;
       if (nt * BM + row < slice_w && n < p.N) {
-        const float bias_v = p.bias ? __bfloat162float(p.bias[n]) : 0.0f;
-        epi_store<EXT>(p, m, n, epi_apply<EXT>(p, a[i], m, n, bias_v, lnst));
+        if (pre) {   // epi_apply / epi_store with the prefetched operands (same arithmetic)
+          float v = a[i];
+          if (EXT && p.ln_fold) v = lnst[2 * m + 1] * (v - lnst[2 * m] * pu[i]) + pc[i];
+          v += pb[i];
+          if (n < p.scale_cols) v *= p.scale;
+          if (p.act == LIGER_ACT_RELU) v = fmaxf(v, 0.0f);
+          else if (p.act == LIGER_ACT_GELU_TANH) v = gelu_tanh_f(v);
+          if (EXT && p.resid) v += pr[i];
+          if (p.out_f32)
+            reinterpret_cast<float*>(p.out)[(int64_t)m * p.ldo + n] = v;
+          else
+            reinterpret_cast<__nv_bfloat16*>(p.out)[(int64_t)m * p.ldo + n] = __float2bfloat16_rn(v);
+        } else {
+          const float bias_v = p.bias ? __bfloat162float(p.bias[n]) : 0.0f;
+          epi_store<EXT>(p, m, n, epi_apply<EXT>(p, a[i], m, n, bias_v, lnst));
+        }
       }
     }
   }
