@@ -335,6 +335,40 @@ def main():
                 "traffic_source": traffic.get(dom, {}).get("source"), "peak_source": peak_src,
                 "share_of_kernel_time": round(c["share"], 4)}
 
+    # ---- in-situ decode pass (no per-launch events): device time of a pass of the whole
+    # decode path, from a batch with n_new generated tokens minus one with a single one,
+    # against the bytes a pass must stream (this rank's weights + the KV cache it reads)
+    decode_pass = None
+    if not gen:
+        bsz, slen = 8, 256
+        ids_d = torch.from_numpy(np.random.default_rng(3).integers(0, cfg.vocab, size=bsz * slen)
+                                 .astype(np.int32)).cuda()
+
+        def batch_ms(n_new):
+            best = 1e30
+            for _ in range(2):
+                barrier()
+                a, z = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record()
+                eng.submit(None, bsz, slen, n_new, 0.0, device_tokens=ids_d)
+                eng.drain()
+                z.record()
+                z.synchronize()
+                best = min(best, max_over_ranks(a.elapsed_time(z)))
+            return best
+        t1, tn = batch_ms(1), batch_ms(args.n_new)
+        pass_us = (tn - t1) / (args.n_new - 1) * 1e3
+        h, f, t = cfg.hidden, cfg.ffn, world
+        w_bytes = cfg.n_layers * (4 * h * h + 2 * h * f) / t * 2 + cfg.vocab / t * h * 2
+        ctx_avg = slen + args.n_new / 2
+        kv_bytes = cfg.n_layers * bsz * ctx_avg * 2 * (h / t) * 2
+        gbs = (w_bytes + kv_bytes) / (pass_us * 1e-6) / 1e9
+        decode_pass = {"batch": bsz, "prompt": slen, "us": round(pass_us, 1),
+                       "bytes": round(w_bytes + kv_bytes), "achieved": round(gbs, 1), "peak": hbm,
+                       "unit": "GB/s", "frac": round(gbs / hbm, 4),
+                       "note": "whole decode pass (all kernels, PDL chain intact), CUDA events around "
+                               "batches with n_new and 1 generated tokens; bytes = weights + KV read"}
+
     # ---- latency at a fixed request rate (Poisson, 0.5 x capacity)
     lat = None
     if not args.no_latency:
@@ -395,6 +429,7 @@ def main():
             "e2e": {"value": round(seqs / e2e_s, 3), "unit": "req/s", "h2d_bytes_per_step": int(h2d),
                     "d2h_bytes_per_step": int(d2h)},
             "roofline": roof,
+            "decode_pass_in_situ": decode_pass,
             "kernel_classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv) for kk, vv in v.items()}
                                for k, v in classes.items()},
             "cpu_baseline": cpu,
