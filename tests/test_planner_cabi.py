@@ -189,3 +189,29 @@ def test_plan_agreement_two_ranks_gloo():
         p.join(timeout=60)
         assert p.exitcode == 0
     assert res[0][0] == res[0][1]
+
+
+def test_gemm_plan_host_logic(L):
+    """liger_gemm_plan is host-only (the tiling / split-K policy): a function of
+    (M, N, K) only, every split chunk covers whole 64-wide K blocks and the chunks
+    tile K exactly; prefill GEMMs that fill the SMs are never split; the decode cost
+    model picks the measured-best splits at the OPT-13B t = 1 shapes
+    (profiles/r01/split_sweep_decode.txt)."""
+    for M in (1, 2, 8, 16, 33, 64, 65, 256, 512, 4096):
+        for N, K in ((15360, 5120), (5120, 5120), (20480, 5120), (5120, 20480), (3456, 9216), (384, 256)):
+            pl = L.gemm_plan(M, N, K)
+            assert pl == L.gemm_plan(M, N, K)
+            nkb = K // 64
+            assert pl["kc"] % 64 == 0 and pl["splits"] == -(-nkb // (pl["kc"] // 64))
+            assert (pl["splits"] - 1) * pl["kc"] < K <= pl["splits"] * pl["kc"]
+            assert pl["bn"] % 16 == 0 and pl["bn"] * pl["m_tiles"] >= M and pl["bn"] <= 256
+            tiles = -(-N // 128) * pl["m_tiles"]
+            if M > 64 and tiles >= 148:
+                assert pl["splits"] == 1
+            assert pl["cluster"] == 1   # in-cluster split-K is opt-in (LIGER_GEMM_CLUSTER=1)
+    # decode shapes (profiles/r01/split_sweep_decode.txt): QKV one chunk, out-proj 3,
+    # FC1 8-10, FC2 3-7 -- within 3 % of the best measured at every shape
+    assert L.gemm_plan(8, 15360, 5120)["splits"] == 1
+    assert L.gemm_plan(8, 5120, 5120)["splits"] == 3
+    assert 8 <= L.gemm_plan(8, 20480, 5120)["splits"] <= 10
+    assert 3 <= L.gemm_plan(8, 5120, 20480)["splits"] <= 7
