@@ -192,7 +192,10 @@ __device__ __forceinline__ Unit unit_of(const GemmParams& p, int u) {
 }
 
 // Persistent: one CTA per SM, CTA i processes units i, i + G, i + 2G, ...
-template <bool EXT>
+// OPT: the opt-in experiments (in-cluster split-K, early-fixup readiness counters) --
+// compiled out of the default instantiations (the decode weight stream is sensitive
+// to extra control flow in this kernel: a measured 10 % for a few branches)
+template <bool EXT, bool OPT>
 __global__ void __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmParams p) {
@@ -213,7 +216,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   uint64_t* red_full = bars + 2 * S + 9;    // [2] cluster split-K: all chunks' partials staged
   uint64_t* red_empty = bars + 2 * S + 11;  // [2] cluster split-K: all CTAs done reading a stage
   float* red0 = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 512);   // [2][bn][128] fp32
-  const bool cl = p.cluster > 1;
+  const bool cl = OPT && p.cluster > 1;
 
 
   const int warp = threadIdx.x >> 5;
@@ -365,7 +368,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         for (int m = blockIdx.x + (etid >> 5) * G; m < p.M; m += 4 * G) {
           ln_row_stats(p.ln_x + (int64_t)m * p.ln_ldx, p.ln_ldx, 1, p.K, p.ln_eps, p.ln_stats + 2 * m, lane, 32);
           __syncwarp();
-          if (lane == 0 && p.tile_ready) {   // row m's statistics are out (the fixup waits for all M)
+          if (OPT && lane == 0 && p.tile_ready) {   // row m's statistics are out (the fixup waits for all M)
             __threadfence();
             atomicAdd(p.tile_ready + GEMM_STATS_CNT, 1u);
           }
@@ -416,7 +419,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tmem_empty[acc]);
-      if (p.splits > 1 && !cl && p.tile_ready) {
+      if (OPT && p.splits > 1 && !cl && p.tile_ready) {
         // chunk w.z of this tile is in the workspace: count it (the fixup reduces a
         // tile as soon as all its chunks have arrived, during this grid's tail)
         named_bar_sync(2, 128);
@@ -762,8 +765,8 @@ static int max_clusters(int S, int bn) {
   std::lock_guard<std::mutex> g(mu);
   auto it = cache.find(key);
   if (it != cache.end()) return it->second;
-  cudaFuncSetAttribute(gemm_tc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
-  cudaFuncSetAttribute(gemm_tc_kernel<false>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  cudaFuncSetAttribute(gemm_tc_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
+  cudaFuncSetAttribute(gemm_tc_kernel<false, true>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(S * 128);
   cfg.blockDim = dim3(GEMM_THREADS);
@@ -776,7 +779,7 @@ static int max_clusters(int S, int bn) {
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   int n = 0;
-  if (cudaOccupancyMaxActiveClusters(&n, gemm_tc_kernel<false>, &cfg) != cudaSuccess || n <= 0) {
+  if (cudaOccupancyMaxActiveClusters(&n, gemm_tc_kernel<false, true>, &cfg) != cudaSuccess || n <= 0) {
     cudaGetLastError();
     n = 0;   // cluster mode unavailable for this S
   }
@@ -917,7 +920,8 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (rc) return rc;
   static bool attr_set = false;
   if (!attr_set) {
-    for (auto k : {gemm_tc_kernel<false>, gemm_tc_kernel<true>}) {
+    for (auto k : {gemm_tc_kernel<false, false>, gemm_tc_kernel<true, false>, gemm_tc_kernel<false, true>,
+                   gemm_tc_kernel<true, true>}) {
       cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
       cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     }
@@ -973,16 +977,17 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
     // one cluster of `splits` CTAs per tile in flight; CTA z of a cluster takes chunk z
     // (grid = clusters x S, so unit u = blockIdx.x + j * grid keeps z = blockIdx.x % S)
     const int nc = std::min(pl.clusters, ntiles * pl.m_tiles);
-    rc2 = ext ? launch_pdl_cluster(gemm_tc_kernel<true>, dim3(nc * pl.cluster), dim3(GEMM_THREADS), pl.cluster,
-                                   pl.smem, stream, tA, tB, p)
-              : launch_pdl_cluster(gemm_tc_kernel<false>, dim3(nc * pl.cluster), dim3(GEMM_THREADS), pl.cluster,
-                                   pl.smem, stream, tA, tB, p);
+    rc2 = ext ? launch_pdl_cluster(gemm_tc_kernel<true, true>, dim3(nc * pl.cluster), dim3(GEMM_THREADS),
+                                   pl.cluster, pl.smem, stream, tA, tB, p)
+              : launch_pdl_cluster(gemm_tc_kernel<false, true>, dim3(nc * pl.cluster), dim3(GEMM_THREADS),
+                                   pl.cluster, pl.smem, stream, tA, tB, p);
   } else {
     // unit u runs on CTA u % grid: the grid size never changes what a unit computes
     const int sms = (a.sm_budget > 0 && a.sm_budget < num_sms()) ? a.sm_budget : num_sms();
     const int grid = p.units < sms ? p.units : sms;
-    rc2 = ext ? launch_pdl(gemm_tc_kernel<true>, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p)
-              : launch_pdl(gemm_tc_kernel<false>, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
+    auto kern = p.tile_ready ? (ext ? gemm_tc_kernel<true, true> : gemm_tc_kernel<false, true>)
+                             : (ext ? gemm_tc_kernel<true, false> : gemm_tc_kernel<false, false>);
+    rc2 = launch_pdl(kern, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
   }
   const bool fixup = p.splits > 1 && pl.cluster <= 1 && !a.defer_fixup;
   if (a.had_fixup) *a.had_fixup = fixup;
