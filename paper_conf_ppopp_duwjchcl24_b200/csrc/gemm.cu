@@ -298,15 +298,14 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       grid_dependency_wait();
       grid_dependency_trigger();   // after the wait: dependents overlap only this kernel
       tr1 = trace_now();
-      int it = 0;
+      int it = 0, s = 0;   // ring slot / parity advanced incrementally (no divisions in the loop)
+      uint32_t ph = 0;
       for (int u = blockIdx.x; u < p.units; u += G) {
         const Unit w = unit_of(p, u);
         const int k0 = w.z * p.kc;
         const int nkb = (min(p.K, k0 + p.kc) - k0 + BK - 1) / BK;
         const int n_base = p.n0 + w.nt * BM, m_base = w.mt * p.bn;
-        for (int kb = 0; kb < nkb; ++kb, ++it) {
-          const int s = it % S;
-          const uint32_t ph = (it / S) & 1;
+        for (int kb = 0; kb < nkb; ++kb, ++it, (++s == S) ? (s = 0, ph ^= 1u) : 0u) {
           const int kk = k0 + kb * BK;
           if (it >= pre) {
             mbar_wait(&empty[s], ph ^ 1);
@@ -323,19 +322,16 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       // kind::f16 instruction descriptor: D=f32, A=B=bf16, both K-major, N=bn, M=128.
       const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(p.bn >> 3) << 17) |
                              ((uint32_t)(BM >> 4) << 24);
-      int it = 0, lu = 0;
-      for (int u = blockIdx.x; u < p.units; u += G, ++lu) {
+      int s = 0, acc = 0;
+      uint32_t ph = 0, acc_ph = 0;
+      for (int u = blockIdx.x; u < p.units; u += G, (++acc == TS) ? (acc = 0, acc_ph ^= 1u) : 0u) {
         const Unit w = unit_of(p, u);
         const int k0 = w.z * p.kc;
         const int nkb = (min(p.K, k0 + p.kc) - k0 + BK - 1) / BK;
-        const int acc = lu % TS;
-        const uint32_t acc_ph = (lu / TS) & 1;
         mbar_wait(&tmem_empty[acc], acc_ph ^ 1);
         tc_fence_after();
         const uint32_t tacc = tmem_base + (uint32_t)acc * acc_cols;
-        for (int kb = 0; kb < nkb; ++kb, ++it) {
-          const int s = it % S;
-          const uint32_t ph = (it / S) & 1;
+        for (int kb = 0; kb < nkb; ++kb, (++s == S) ? (s = 0, ph ^= 1u) : 0u) {
           mbar_wait(&full[s], ph);
           tc_fence_after();
           const uint64_t adesc = umma_desc_sw128(smem_u32(smA + (size_t)s * A_BYTES));
