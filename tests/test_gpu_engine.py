@@ -179,3 +179,27 @@ def test_ln_fold_decode_matches_oracle(E, cfg_expr):
             agree += int(np.sum(np.array(got1)[i] == np.array(got0)[i]))
             total += t["n_decode"]
     assert agree >= 0.9 * total
+
+
+def test_ln_fold_full_size_opt13b_layer_tokens(E):
+    """The bench's launch configuration at full size: an OPT-13B-shaped model cut to one
+    decoder layer (h = 5120, ffn 20480, vocab 50272, ReLU) served at t = 1 -- decode
+    passes with the LayerNorms folded into the split-K QKV / FC1 GEMMs and the
+    residual adds in the out-proj / FC2 fixups (plans 1 / 3 / 10 / 7 chunks) -- gives
+    the fp64 oracle's greedy tokens wherever the oracle's top-2 margin is clear."""
+    from liger_inputs.configs import ModelConfig
+    cfg = ModelConfig("opt13b-L1", 1, 5120, 40, 20480, 50272, 64, "relu")
+    prompt = np.random.default_rng(9).integers(0, cfg.vocab, size=(2, 24))
+    eng = E(cfg, mode="interleaved", max_batch=2, max_seq=24, max_new=6, seed=1)
+    bid = eng.submit(prompt.reshape(-1).astype(np.int32), 2, 24, 6, 0.0)
+    eng.drain()
+    _, toks = eng.poll(bid, want_tokens=True)
+    eng.close()
+    ref, logits = om.greedy_generate(cfg, 1, prompt, 6, return_logits=True)
+    ok = om.top2_margin(logits) > 0.02 * np.sqrt((logits ** 2).mean())
+    checked = 0
+    for i in range(2):
+        n = int(np.argmin(ok[i])) if not ok[i].all() else 6
+        assert np.array_equal(toks[i, :n], ref[i, :n]), (toks, ref)
+        checked += n
+    assert checked >= 4
