@@ -808,7 +808,7 @@ void admit(liger_ctx* c, Batch* bt) {
   for (int i = 0; i < bt->b; ++i)
     for (int p = 0; p < ppseq; ++p) S.h_page_table[i * c->max_pages + p] = base + i * c->max_pages + p;
   // inputs for the first kernels: wait until the previous user of the slot is done
-  const int si = c->t1_streams ? (slot & 1) : 0;
+  const int si = (c->t1_streams && !c->timing) ? (slot & 1) : 0;
   cudaStream_t st = si ? c->s_comm : c->s_comp;
   cudaStreamWaitEvent(st, S.free_ev, 0);
   cudaMemcpyAsync(S.page_table, S.h_page_table, sizeof(int32_t) * bt->b * c->max_pages, cudaMemcpyHostToDevice, st);
@@ -1257,8 +1257,9 @@ int liger_step(liger_ctx* c) {
     c->st.rounds++;
     c->have_round = false;
     n = (int)pieces.size();
-  } else if (c->t1_streams) {
+  } else if (c->t1_streams && !c->timing) {
     // t = 1: every in-flight batch's whole list, in order, on the stream of its slot
+    // (per-launch kernel timing runs the batches one at a time instead)
     for (Batch* bt : c->processing) {
       if (bt->all_launched) continue;
       const size_t p0 = pieces.size();
