@@ -267,6 +267,8 @@ def main():
         e0.record()
         t_host0 = time.perf_counter()
         ids = []
+        # NVTX range around the timed region (ncu --nvtx --nvtx-include "timed/" captures just it)
+        torch.cuda.nvtx.range_push("timed" if not host_io else "timed_e2e")
         for r, dt in zip(timed, dev_tokens):
             if host_io:
                 ids.append(eng.submit(r["tokens"], r["batch"], r["seq_len"], r["n_decode"], 0.0))
@@ -277,6 +279,7 @@ def main():
         if host_io:
             for bid in ids:
                 toks.append(eng.poll(bid, want_tokens=True)[1])
+        torch.cuda.nvtx.range_pop()
         torch.cuda.synchronize()
         e1.record()
         e1.synchronize()
