@@ -53,7 +53,13 @@ extern "C" {
 #define LIGER_ACT_GELU_TANH 2 /* tiny and GLM-shaped configs                */
 
 #define LIGER_MODE_SERIAL 0      /* Intra-Op baseline: compute then all-reduce, in order */
-#define LIGER_MODE_INTERLEAVED 1 /* Liger: Algorithm 1 + hybrid sync               */
+#define LIGER_MODE_INTERLEAVED 1 /* Liger: Algorithm 1 + hybrid sync; at t = 1
+                                    (nothing to interleave) the in-flight batches run
+                                    concurrently on the two streams (LIGER_T1_STREAMS=0: one) */
+/* Numerics note (t = 1): decode passes of <= 16 tokens fold LayerNorm into the QKV / FC1
+ * GEMMs and the residual adds into the out-proj / FC2 epilogues (LIGER_LN_FOLD=0
+ * restores the add + LN kernels).  Every mode and schedule of a context computes the
+ * same bits; the two settings differ by rounding only (both meet the oracle). */
 /* Synchronisation of Algorithm 1 rounds (§3.4, Fig. 8; ablation §4.5):
  * HYBRID      the host waits for E1 (recorded before the running round's last
  *             primary kernel), then launches the next round's subsets -- comm
