@@ -987,8 +987,12 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   }
   int lo, hi;
   cudaDeviceGetStreamPriorityRange(&lo, &hi);
+  // the communication stream gets the high priority (its kernels are short and gate the
+  // other ranks); at t = 1 the two streams carry equal work (two batches): same priority
+  // unless LIGER_T1_PRIO=1 (experiment)
+  const bool t1_prio = getenv("LIGER_T1_PRIO") && atoi(getenv("LIGER_T1_PRIO")) != 0;
   CK(cudaStreamCreateWithPriority(&c->s_comp, cudaStreamNonBlocking, lo));
-  CK(cudaStreamCreateWithPriority(&c->s_comm, cudaStreamNonBlocking, hi));
+  CK(cudaStreamCreateWithPriority(&c->s_comm, cudaStreamNonBlocking, (c->t1_streams && !t1_prio) ? lo : hi));
   CK(cudaEventCreateWithFlags(&c->e1, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&c->e2, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&c->e_end[0], cudaEventDisableTiming));
