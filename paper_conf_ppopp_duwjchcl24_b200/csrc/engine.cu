@@ -462,7 +462,8 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
   // statistics every single-chunk GEMM CTA computes within its mainloop (measured:
   // decode pass -2.5 % at b = 2..8; at b = 32 (generative) the statistics outlast
   // the QKV mainloop: 1492 vs 1506 seq/s folded vs not)
-  const bool fold = c->ln_fold && M <= 16;
+  static const int fold_max = getenv("LIGER_LN_FOLD_MAX") ? atoi(getenv("LIGER_LN_FOLD_MAX")) : 16;
+  const bool fold = c->ln_fold && M <= std::min(fold_max, 64);
   const int li = po.layer;
   const LayerW* W = li >= 0 ? &c->layers[li] : nullptr;
   int rc = 0;
