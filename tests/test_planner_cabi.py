@@ -215,3 +215,14 @@ def test_gemm_plan_host_logic(L):
     assert L.gemm_plan(8, 5120, 5120)["splits"] == 3
     assert 8 <= L.gemm_plan(8, 20480, 5120)["splits"] <= 10
     assert 3 <= L.gemm_plan(8, 5120, 20480)["splits"] <= 7
+
+
+def test_missing_library_fails_loudly(monkeypatch, tmp_path):
+    """No CPU fallback (task ③): without libliger.so every entry point raises."""
+    from paper_conf_ppopp_duwjchcl24_b200 import liger
+    monkeypatch.setattr(liger, "LIB_PATH", str(tmp_path / "libliger.so"))
+    monkeypatch.setattr(liger, "_lib", None)
+    with pytest.raises(liger.LigerError, match="not built"):
+        liger.lib()
+    with pytest.raises(liger.LigerError):
+        liger.gemm_plan(8, 5120, 5120)
