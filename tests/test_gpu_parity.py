@@ -246,6 +246,38 @@ def test_decode_attention_long_context_split(L):
     assert errs(to_np64(outs[0]), ref.transpose(0, 2, 1, 3).reshape(b, hd))[0] <= REL
 
 
+def test_decode_attention_max_context_and_limit(L):
+    """The longest context decode attention takes (64 chunks of 64 = 4096 positions),
+    over scattered pages (a seeded permutation: the page-table indirection), against
+    the oracle; the new token's K/V are appended to its page; one position more is
+    rejected with LIGER_EINVAL (include/liger.h, liger_op_attn_decode)."""
+    b, heads, d, pos = 2, 2, 128, 4095
+    maxp = (pos + 1 + 15) // 16
+    n = b * maxp * 2 * heads * 16 * d
+    pool_np = c0_values(11, 7, np.arange(n, dtype=np.uint64), 0).reshape(b * maxp, 2, heads, 16, d)
+    pool = bf16_dev(pool_np)
+    perm = np.random.default_rng(11).permutation(b * maxp).astype(np.int32).reshape(b, maxp)
+    pt = torch.from_numpy(perm).cuda()
+    q1d = bf16_dev(_qkv(b, 1, heads, d, 12))
+    o1 = torch.empty(b, heads * d, dtype=torch.bfloat16, device="cuda")
+    ws = workspace(L.attn_decode_workspace_bytes(b, heads, d, pos + 1))
+    L.attn_decode(q1d, o1, pool, pt, b=b, pos=pos, heads=heads, d=d, workspace=ws)
+    torch.cuda.synchronize()
+    hd = heads * d
+    q1 = to_np64(q1d)
+    pool64 = to_np64(pool)
+    # cached positions 0..pos-1 of sequence i sit in pages perm[i, t // 16], slot t % 16
+    k = np.stack([pool64[perm[i]][:, 0].transpose(1, 0, 2, 3).reshape(heads, maxp * 16, d) for i in range(b)])
+    v = np.stack([pool64[perm[i]][:, 1].transpose(1, 0, 2, 3).reshape(heads, maxp * 16, d) for i in range(b)])
+    knew, vnew = _split(q1[:, hd:2 * hd], b, 1, heads, d), _split(q1[:, 2 * hd:], b, 1, heads, d)
+    assert np.array_equal(k[:, :, pos:pos + 1], knew) and np.array_equal(v[:, :, pos:pos + 1], vnew)
+    ref = om.causal_attention(_split(q1[:, :hd], b, 1, heads, d), k[:, :, :pos + 1], v[:, :, :pos + 1],
+                              np.array([pos]), np.arange(pos + 1))
+    assert errs(to_np64(o1), ref.transpose(0, 2, 1, 3).reshape(b, hd))[0] <= REL
+    with pytest.raises(L.LigerError):
+        L.attn_decode(q1d, o1, pool, pt, b=b, pos=pos + 1, heads=heads, d=d, workspace=ws)
+
+
 # ---------------------------------------------------------------- argmax
 def test_argmax_lowest_index_on_ties(L):
     logits = np.random.default_rng(0).standard_normal((5, 3000)).astype(np.float32)
