@@ -204,8 +204,7 @@ int liger_set_gemm_sm_reserve(liger_ctx* ctx, int reserve);
 #define LIGER_KT_GEMM_PREFILL 4  /* projection GEMMs with M > 64 tokens (tensor-bound) */
 #define LIGER_KT_LMHEAD 5
 #define LIGER_KT_FIXUP 6         /* split-K fixup kernels */
-#define LIGER_KT_DECODE_FUSED 7  /* fused decode pass (all layers of a decode step at t = 1, HBM-bound) */
-#define LIGER_KT_CLASSES 8
+#define LIGER_KT_CLASSES 7
 int liger_set_kernel_timing(liger_ctx* ctx, int on);
 int liger_kernel_timing(liger_ctx* ctx, int64_t* count, double* ms, double* bytes, double* flops);
 
@@ -273,31 +272,14 @@ int liger_op_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, void* 
 int liger_op_gemm_tiled(const void* x, int64_t ldx, const void* w_tiled, void* out, int64_t ldo, int M, int N,
                         int K, int n0, int n1, const void* bias, int act, int scale_cols, float scale, int out_f32,
                         void* workspace, size_t ws_bytes, void* stream);
-/* Row-parallel projection fused with the following residual add + LayerNorm at
- * t = 1 (§8(a) a5 -> a7 and a9 -> a11 when no all-reduce separates them):
- *   P = x[M,K] . W[N,K]^T (split-K plan of (M, N, K), which must split),
- *   x_res = bf16(x_res + bf16(P) + add_bias),  y = LN(x_res; gamma, beta, eps).
- * The GEMM leaves its fp32 split-K partials in `workspace` and the add + LN kernel
- * sums them itself, in the fixup kernel's order: bit-identical to
- * liger_op_gemm_tiled (P into a bf16 buffer) followed by liger_op_add_layernorm,
- * with one kernel and one hand-off fewer.  N = hidden (multiple of 128), W tiled as
- * for liger_op_gemm_tiled; x_res/y [M, N] bf16, x_res updated in place; workspace
- * of liger_gemm_workspace_bytes(M, N, K) bytes.  LIGER_EINVAL if the plan has no
- * split (use the two calls). */
-int liger_op_gemm_tiled_add_layernorm(const void* x, const void* w_tiled, int M, int N, int K, void* x_res,
-                                      const void* add_bias, void* y, const void* gamma, const void* beta,
-                                      float eps, void* workspace, size_t ws_bytes, void* stream);
 /* Convert a row-major bf16 W [N, K] (row stride ld) to the tiled layout
  * (dst holds ceil(N/128)*128*K elements; padding rows are zero). */
 int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K, void* stream);
 size_t liger_gemm_workspace_bytes(int M, int N, int K);
 /* The tiling plan liger_op_gemm uses for a GEMM of full size (M, N, K) (host
  * only; a function of (M, N, K), identical for every column slice):
- * out[7] = {token tile bn, m tiles, split-K chunk kc, splits, pipeline stages,
- *           cluster, co-resident clusters} -- cluster > 1: the splits are reduced in-kernel across a
- *           thread-block cluster of that many CTAs (DSMEM, decode M <= 64; needs
- *           the device to size it, so a host without one reports 1); else a
- *           split-K fixup kernel follows.  Both sum chunks in the same order. */
+ * out[5] = {token tile bn, m tiles, split-K chunk kc, splits, pipeline stages};
+ * splits > 1: a split-K fixup kernel sums the chunks' fp32 partials in chunk order. */
 int liger_gemm_plan(int M, int N, int K, int32_t* out);
 
 /* Fused residual add + LayerNorm (§8(a) a2/a7/a11; C2):
@@ -333,42 +315,6 @@ int liger_op_attn_prefill(const void* qkv, void* o, void* kv_pool, const int32_t
 int liger_op_attn_decode(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
                          int pos, int heads, int d, void* workspace, size_t ws_bytes, void* stream);
 size_t liger_attn_decode_workspace_bytes(int b, int heads, int d, int ctx);
-
-/* Fused decode pass (§8(a) a2-a11 for one decode step, t = 1): for each layer
- * l = 0..L-1 of `layers` (device pointers; weights in the tiled layout of
- * liger_op_gemm_tiled), with M = b <= 32 tokens, in ONE persistent kernel:
- *   x += part + b_2(l-1) (skipped at l = 0 when first_no_add); y = LN1(x)
- *   qkv = y W_qkv^T + b_qkv (q columns * qscale); attn = decode attention at `pos`
- *   over the paged cache of layer l (kv + l * kv_layer_elems elements; appends k, v)
- *   part = attn W_o^T; x += part + b_o; y = LN2(x); hbuf = act(y W_1^T + b_1);
- *   part = hbuf W_2^T   (the last layer's b_2 / residual are left to the caller).
- * Buffers: x, y, part bf16 [M, h]; qkv [M, 3*heads*d]; attn [M, heads*d];
- * hbuf [M, ffn].  gemm_ws: >= liger_gemm_workspace_bytes of each of the four
- * GEMMs at M, first 16 KiB zero before first use (left zero); attn_ws as for
- * liger_op_attn_decode.  The results are bit-identical to the same layers run
- * op by op (liger_op_add_layernorm, liger_op_gemm_tiled, liger_op_attn_decode).
- * Shape limits: d in {64, 128}; h, ffn, 3*heads*d multiples of 128; else
- * LIGER_EINVAL.  The layer table is copied; the library keeps device copies of
- * its TMA descriptors until the weight pointers change.  Not thread-safe. */
-typedef struct {
-  const void *b_qkv, *b_o, *b_1, *b_2, *g1, *be1, *g2, *be2;
-  const void *w_qkv, *w_o, *w_1, *w_2;
-} liger_fused_layer;
-typedef struct {
-  int32_t L, M, h, heads, d, ffn, act, pos;
-  float eps, qscale;
-  int32_t first_no_add;
-  const liger_fused_layer* layers;   /* host array [L] */
-  void *x, *y, *qkv, *attn, *part, *hbuf, *kv;
-  int64_t kv_layer_elems;
-  const int32_t* page_table;
-  int32_t max_pages;
-  void* gemm_ws;
-  size_t gemm_ws_bytes;
-  void* attn_ws;
-  size_t attn_ws_bytes;
-} liger_fused_decode_args;
-int liger_op_decode_fused(const liger_fused_decode_args* args, void* stream);
 
 /* Row-wise argmax over fp32 logits [rows, n] (row stride ld): writes the
  * maximum value and its index + idx_offset (lowest index on ties, C7). */

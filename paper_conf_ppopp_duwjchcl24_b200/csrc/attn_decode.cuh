@@ -1,9 +1,6 @@
 // Decode attention over the paged KV cache:
 // one query token per sequence, split over the context in chunks of CH
-// positions.  The arithmetic of one work item (head, sequence, chunk) lives here
-// so that the standalone kernel (attention.cu) and the fused decode-pass kernel
-// (decode_fused.cu) run the identical instruction sequence -- the two paths give
-// the same bits.
+// positions.  The arithmetic of one work item (head, sequence, chunk) lives here.
 //
 // A work item is run by a group of DC_THREADS = 128 threads (4 warps):
 //  * issue: warp 0 stages the chunk's cached K and V page blocks (16 tokens x d

@@ -69,26 +69,6 @@ int liger_op_gemm_tiled(const void* x, int64_t ldx, const void* w, void* out, in
   return ret(gemm_launch(a, (cudaStream_t)stream), "liger_op_gemm_tiled");
 }
 
-int liger_op_gemm_tiled_add_layernorm(const void* x, const void* w_tiled, int M, int N, int K, void* x_res,
-                                      const void* add_bias, void* y, const void* gamma, const void* beta,
-                                      float eps, void* workspace, size_t ws_bytes, void* stream) {
-  if (int rc = check_device()) return rc;
-  if (!x_res || !y || !gamma || !beta || M <= 0) return ret(LIGER_EINVAL, "liger_op_gemm_tiled_add_layernorm");
-  const GemmPlan pl = gemm_plan(M, N, K);
-  if (pl.splits <= 1 || pl.cluster > 1) {   // no split-K: plain GEMM into a scratch-free path is not offered
-    set_global_error("liger_op_gemm_tiled_add_layernorm: (M, N, K) has no split-K plan");
-    return LIGER_EINVAL;
-  }
-  GemmArgs a{x, K, w_tiled, 64, nullptr, N, M, N, K, 0, N, nullptr, LIGER_ACT_NONE, 0, 1.0f, 0, workspace, ws_bytes, 1};
-  a.defer_fixup = true;
-  if (int rc = gemm_launch(a, (cudaStream_t)stream)) return ret(rc, "liger_op_gemm_tiled_add_layernorm");
-  const int64_t zstride = (int64_t)((N + 127) / 128) * pl.m_tiles * 128 * pl.bn;
-  return ret(splitk_add_layernorm_launch(reinterpret_cast<const float*>((char*)workspace + GEMM_COUNTER_BYTES),
-                                         zstride, pl.splits, pl.m_tiles, pl.bn, x_res, add_bias, x_res, y, gamma,
-                                         beta, M, N, eps, (cudaStream_t)stream),
-             "liger_op_gemm_tiled_add_layernorm");
-}
-
 int liger_op_tile_weight(const void* w, int64_t ld, void* w_tiled, int N, int K, void* stream) {
   if (int rc = check_device()) return rc;
   return ret(tile_weight_launch(w, ld, w_tiled, N, K, (cudaStream_t)stream), "liger_op_tile_weight");
@@ -100,7 +80,6 @@ int liger_gemm_plan(int M, int N, int K, int32_t* out) {
   if (!out || M <= 0 || N <= 0 || K <= 0) return LIGER_EINVAL;
   GemmPlan pl = gemm_plan(M, N, K);
   out[0] = pl.bn; out[1] = pl.m_tiles; out[2] = pl.kc; out[3] = pl.splits; out[4] = pl.stages;
-  out[5] = pl.cluster; out[6] = pl.clusters;
   return LIGER_OK;
 }
 
@@ -157,22 +136,6 @@ int liger_op_c0_fill(void* dst, int rows, int cols, int64_t ld, uint64_t seed, u
 
 }  // extern "C"
 
-extern "C" int liger_op_decode_fused(const liger_fused_decode_args* in, void* stream) {
-  if (int rc = check_device()) return rc;
-  if (!in || !in->layers || in->L <= 0) return LIGER_EINVAL;
-  static FusedDecodeState* state = nullptr;   // descriptor tables of the last call's weights
-  static_assert(sizeof(liger_fused_layer) == sizeof(FusedLayerPtrs), "layer table layout");
-  FusedDecodeArgs a{};
-  a.L = in->L; a.M = in->M; a.h = in->h; a.heads = in->heads; a.d = in->d; a.ffn = in->ffn; a.act = in->act;
-  a.pos = in->pos; a.eps = in->eps; a.qscale = in->qscale; a.first_no_add = in->first_no_add;
-  a.layers = reinterpret_cast<const FusedLayerPtrs*>(in->layers);
-  a.x = in->x; a.y = in->y; a.qkv = in->qkv; a.attn = in->attn; a.part = in->part; a.hbuf = in->hbuf;
-  a.kv = in->kv; a.kv_layer_elems = in->kv_layer_elems; a.page_table = in->page_table; a.max_pages = in->max_pages;
-  a.gemm_ws = in->gemm_ws; a.gemm_ws_bytes = in->gemm_ws_bytes; a.attn_ws = in->attn_ws;
-  a.attn_ws_bytes = in->attn_ws_bytes;
-  return ret(fused_decode_launch(&state, a, (cudaStream_t)stream), "liger_op_decode_fused");
-}
-
 // ------------------------------------------------------------------ timeline trace (diagnostics)
 static void* g_trace_rec = nullptr;
 static unsigned int* g_trace_n = nullptr;
@@ -193,7 +156,6 @@ extern "C" int liger_trace_start(unsigned int capacity) {
   trace_set_gemm(r, g_trace_n, capacity);
   trace_set_norm(r, g_trace_n, capacity);
   trace_set_attention(r, g_trace_n, capacity);
-  trace_set_fused(r, g_trace_n, capacity);
   return cudaDeviceSynchronize() == cudaSuccess ? LIGER_OK : LIGER_ECUDA;
 }
 
@@ -203,7 +165,6 @@ extern "C" int liger_trace_stop(void* host_records, unsigned int capacity, unsig
   trace_set_gemm(nullptr, nullptr, 0);
   trace_set_norm(nullptr, nullptr, 0);
   trace_set_attention(nullptr, nullptr, 0);
-  trace_set_fused(nullptr, nullptr, 0);
   unsigned int n = 0;
   cudaMemcpy(&n, g_trace_n, sizeof(n), cudaMemcpyDeviceToHost);
   if (n > g_trace_cap) n = g_trace_cap;

@@ -94,12 +94,7 @@ struct Slot {
   int32_t* h_prompt;       // pinned
   int32_t* h_tok_out;      // pinned
   cudaEvent_t free_ev;     // completes when the last batch using the slot finished
-  FusedDecodeState* fused = nullptr;   // fused decode pass tables of this slot
   Batch* owner = nullptr;  // batch currently (or last) assigned to the slot
-  // split-K partials of the last row-parallel GEMM left in gemm_ws for the next add + LN
-  bool split_pending = false;
-  GemmPlan split_plan{};
-  int split_N = 0;
   // fused all-reduce (t > 1, serial mode): the last row-parallel GEMM's fixup staged
   // its partial for epoch far.epoch; the next add + LN reduces it over the peers
   bool far_pending = false;
@@ -181,14 +176,6 @@ struct liger_ctx {
   uint32_t dbg_skip = 0;               // LIGER_DBG_SKIP=op,op,...: timing experiments only (wrong results)
   bool ar_atomic_chunks = false;
   size_t ar_decomp_min_bytes = 1 << 20;   // all-reduces below this are not decomposed
-  // decode passes at t = 1 as one fused kernel (LIGER_FUSED_DECODE=1).  Off by default:
-  // measured 17-33 % slower than the per-kernel PDL chain.
-  bool fused_decode = false;
-  // t = 1: split-K sum of out-proj / FC2 folded into the next add + LN (opt-in
-  // LIGER_FUSE_SPLITK_LN=1; bit-identical; measured neutral: OPT-13B decode pass
-  // 5527 vs 5433 us at b = 2, 5688 vs 5747 us at b = 8 -- one CTA per row reading
-  // S x h fp32 partials costs what the fixup kernel and its hand-off did)
-  bool fuse_split_ln = false;
   // t > 1, serial mode (LIGER_FUSED_AR=1, needs the one-shot peer backend): the
   // all-reduce of out-proj / FC2 is fused into the GEMM's fixup (stage + publish)
   // and the following add + LN (wait + rank-ordered sum): no all-reduce kernel
@@ -427,24 +414,6 @@ void timing_flush(liger_ctx* c) {
 }
 
 // ------------------------------------------------------------------ launching one piece
-// Decode passes at t = 1 (no all-reduce between the layers' compute runs) go through
-// the fused decode-pass kernel (decode_fused.cu) when its shape limits allow.
-bool fused_pass(liger_ctx* c, int M) {
-  return c->fused_decode && c->tp == 1 && fused_decode_supported(M, c->h, c->al, c->d, c->fl);
-}
-
-// add + LN over the split-K partials a deferred row-parallel GEMM left in gemm_ws
-static int split_add_ln(liger_ctx* c, Slot& S, const void* bias, const void* gamma, const void* beta, int M,
-                        cudaStream_t st) {
-  const GemmPlan& pl = S.split_plan;
-  const int n_tiles = (S.split_N + 127) / 128;
-  const int64_t zstride = (int64_t)n_tiles * pl.m_tiles * 128 * pl.bn;
-  S.split_pending = false;
-  return splitk_add_layernorm_launch(reinterpret_cast<const float*>((char*)S.gemm_ws + GEMM_COUNTER_BYTES), zstride,
-                                     pl.splits, pl.m_tiles, pl.bn, S.x, bias, S.x, S.y, gamma, beta, M, c->h,
-                                     c->cfg.ln_eps, st);
-}
-
 // add + LN over the peers' staged partials of a fused all-reduce epoch
 static int peer_add_ln(liger_ctx* c, Slot& S, const void* bias, const void* gamma, const void* beta, int M,
                        cudaStream_t st) {
@@ -469,41 +438,6 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
   int rc = 0;
   cudaEvent_t ta = nullptr;
   if (c->dbg_skip & (1u << po.op)) return 0;
-  if (pass > 0 && li >= 0 && fused_pass(c, M)) {
-    // decode step at t = 1: the whole layer range is one fused kernel, launched at
-    // the range's first op; the per-layer ops it covers launch nothing
-    if (po.op != OP_LN1 || li != c->l0) return 0;
-    FusedDecodeArgs fa{};
-    std::vector<FusedLayerPtrs> lp(c->l1 - c->l0);
-    for (int l = c->l0; l < c->l1; ++l) {
-      const LayerW& w = c->layers[l];
-      lp[l - c->l0] = FusedLayerPtrs{w.b_qkv, w.b_o, w.b_1, w.b_2, w.g1, w.be1, w.g2, w.be2,
-                                     w.w_qkv, w.w_o, w.w_1, w.w_2};
-    }
-    fa.L = c->l1 - c->l0; fa.M = M; fa.h = h; fa.heads = c->al; fa.d = c->d; fa.ffn = c->fl;
-    fa.act = c->cfg.act; fa.pos = bt->s + pass - 1; fa.eps = eps; fa.qscale = 1.0f / sqrtf((float)c->d);
-    fa.first_no_add = 1; fa.layers = lp.data();
-    fa.x = S.x; fa.y = S.y; fa.qkv = S.qkv; fa.attn = S.attn; fa.part = S.part; fa.hbuf = S.hbuf;
-    fa.kv = c->kv; fa.kv_layer_elems = (int64_t)c->kv_layer_elems; fa.page_table = S.page_table;
-    fa.max_pages = c->max_pages;
-    fa.gemm_ws = S.gemm_ws; fa.gemm_ws_bytes = S.gemm_ws_bytes;
-    fa.attn_ws = S.attn_ws; fa.attn_ws_bytes = S.attn_ws_bytes;
-    timed_begin(c, st, &ta);
-    rc = fused_decode_launch(&S.fused, fa, st);
-    if (c->timing) {
-      const double ctx = fa.pos + 1, L = fa.L, hl = c->hl;
-      const double gemm_bytes = ((3 * hl * h + (double)M * h + M * 3 * hl) + (h * hl + M * hl + (double)M * h) +
-                                 ((double)c->fl * h + (double)M * h + (double)M * c->fl) +
-                                 ((double)h * c->fl + (double)M * c->fl + (double)M * h)) * 2;
-      const double attn_bytes = (double)M * hl * 2 * 2 * ctx;
-      const double ln_bytes = 2.0 * M * h * 2 * 4;
-      const double flops = 2.0 * M * (3 * hl * h + h * hl + 2.0 * c->fl * h) + 4.0 * M * hl * ctx;
-      timed_end(c, st, ta, LIGER_KT_DECODE_FUSED, L * (gemm_bytes + attn_bytes + ln_bytes), L * flops);
-    }
-    c->st.gpu_launches++;
-    if (rc < 0) return fail(c, rc, "launch of the fused decode pass failed");
-    return 0;
-  }
   switch (po.op) {
     case OP_EMBED: {
       const int32_t* ids = pass == 0 ? (bt->dev_tokens ? bt->dev_tokens : S.prompt) : S.cur_tok;
@@ -519,8 +453,6 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
         rc = add_layernorm_launch(S.x, nullptr, nullptr, nullptr, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
       else if (S.far_pending)
         rc = peer_add_ln(c, S, c->layers[li - 1].b_2, W->g1, W->be1, M, st);
-      else if (S.split_pending)
-        rc = split_add_ln(c, S, c->layers[li - 1].b_2, W->g1, W->be1, M, st);
       else
         rc = add_layernorm_launch(S.x, S.part, c->layers[li - 1].b_2, S.x, S.y, W->g1, W->be1, M, h, 1, 0, eps, st);
       timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * (li == c->l0 ? 2 : 4), 0);
@@ -532,8 +464,6 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       timed_begin(c, st, &ta);
       if (S.far_pending)
         rc = peer_add_ln(c, S, W->b_o, W->g2, W->be2, M, st);
-      else if (S.split_pending)
-        rc = split_add_ln(c, S, W->b_o, W->g2, W->be2, M, st);
       else
         rc = add_layernorm_launch(S.x, S.part, W->b_o, S.x, S.y, W->g2, W->be2, M, h, 1, 0, eps, st);
       timed_end(c, st, ta, LIGER_KT_LN, (double)M * h * 2 * 4, 0);
@@ -583,24 +513,11 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
           g.bias = po.op == OP_OUT ? W->b_o : W->b_2;
         }
       }
-      // t = 1 (no all-reduce follows): leave the split-K partials of out-proj and of
-      // FC2 (not the last layer's, which feeds the LM head / the next stage) to the
-      // next add + LN, which sums them itself (bit-identical, one kernel fewer)
-      if (c->tp == 1 && c->fuse_split_ln && !fold && u0 == 0 && u1 == F &&
-          (po.op == OP_OUT || (po.op == OP_FC2 && li + 1 < c->l1))) {
-        const GemmPlan pl = gemm_plan(M, N, K);
-        if (pl.splits > 1 && pl.cluster <= 1) {
-          g.defer_fixup = true;
-          S.split_pending = true;
-          S.split_plan = pl;
-          S.split_N = N;
-        }
-      }
       if (c->tp > 1 && c->fused_ar && c->cfg.mode == LIGER_MODE_SERIAL && u0 == 0 && u1 == F &&
           (po.op == OP_OUT || (po.op == OP_FC2 && li + 1 < c->l1))) {
         const GemmPlan pl = gemm_plan(M, N, K);
         PeerAR* par = c->comm ? c->comm->peer_ar(st) : nullptr;
-        if (pl.splits > 1 && pl.cluster <= 1 && par && (size_t)M * N * 2 <= par->cap) {
+        if (pl.splits > 1 && par && (size_t)M * N * 2 <= par->cap) {
           if (par->fused_begin((size_t)M * N * 2, &S.far)) return fail(c, LIGER_ECUDA, "fused all-reduce setup");
           g.far = &S.far;
           S.far_pending = true;
@@ -959,18 +876,15 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     for (int o = 0; o < OP_COUNT; ++o)
       if (all.find(std::string(",") + kOpName[o] + ",") != std::string::npos) c->dbg_skip |= 1u << o;
   }
-  if (const char* fd = getenv("LIGER_FUSED_DECODE")) c->fused_decode = atoi(fd) != 0;
-  if (const char* fs = getenv("LIGER_FUSE_SPLITK_LN")) c->fuse_split_ln = atoi(fs) != 0;
   if (const char* fa = getenv("LIGER_FUSED_AR")) c->fused_ar = atoi(fa) != 0;
   if (const char* sr = getenv("LIGER_GEMM_SM_RESERVE")) c->gemm_sm_reserve = atoi(sr);
   {
     const char* ts = getenv("LIGER_T1_STREAMS");
-    c->t1_streams = (ts ? atoi(ts) != 0 : true) && c->tp == 1 && !c->pipe && cfg->mode == LIGER_MODE_INTERLEAVED &&
-                    !c->fused_decode;
+    c->t1_streams = (ts ? atoi(ts) != 0 : true) && c->tp == 1 && !c->pipe && cfg->mode == LIGER_MODE_INTERLEAVED;
   }
   {
     const char* lf = getenv("LIGER_LN_FOLD");
-    c->ln_fold = (lf ? atoi(lf) != 0 : true) && c->tp == 1 && !c->fused_decode;
+    c->ln_fold = (lf ? atoi(lf) != 0 : true) && c->tp == 1;
   }
   {
     int dev = 0, n = 0;
@@ -1683,7 +1597,6 @@ int liger_finalize(liger_ctx* c) {
     cudaFreeHost(S.h_prompt);
     cudaFreeHost(S.h_tok_out);
     cudaEventDestroy(S.free_ev);
-    fused_decode_free(S.fused);
   }
   for (auto e : c->ev_pool) cudaEventDestroy(e);
   for (auto e : c->timing_pool) cudaEventDestroy(e);

@@ -41,9 +41,6 @@ constexpr int BK = 64;            // K per stage (one 128-byte swizzle atom)
 constexpr int A_BYTES = BM * BK * 2;
 constexpr int GEMM_THREADS = 192;
 constexpr int MAX_SMEM = 227 * 1024;
-constexpr int GEMM_MAX_READY_TILES = 2048;
-constexpr int GEMM_STATS_CNT = 2048;
-constexpr int GEMM_DONE_CNT = 2049;
 
 static int num_sms() {
   static int n = 0;
@@ -75,14 +72,6 @@ struct GemmParams {
   int64_t ldo;
   int out_f32;
   float* ws;
-  int* counters;
-  // split-K readiness (workspace counter region, zero between uses): tile_ready[t]
-  // counts the chunks of tile t written, [GEMM_STATS_CNT] the folded-LN rows whose
-  // statistics are out, [GEMM_DONE_CNT] the fixup CTAs done (the last one re-zeroes)
-  unsigned int* tile_ready;
-  const void* w_base;   // tiled weights (for the L2 prefetch)
-  int pf_blocks;        // weight blocks (beyond the smem stages) prefetched into L2 before the PDL wait
-  int cluster;          // > 1: split-K reduced in-kernel across a (splits x 1 x 1) thread-block cluster
   // fused all-reduce producer (fixup kernel): publish pub_epoch on pub_flag (system
   // scope) once every CTA's output stores are visible
   unsigned long long* pub_flag;
@@ -148,12 +137,6 @@ __device__ __forceinline__ void ln_row_stats(const __nv_bfloat16* X, int64_t ldx
   }
 }
 
-__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
-  unsigned v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-
 // EXT: the folded-LayerNorm / residual-add epilogue (a separate instantiation, so
 // the plain epilogue of the prefill GEMMs keeps its code)
 template <bool EXT>
@@ -192,10 +175,7 @@ __device__ __forceinline__ Unit unit_of(const GemmParams& p, int u) {
 }
 
 // Persistent: one CTA per SM, CTA i processes units i, i + G, i + 2G, ...
-// OPT: the opt-in experiments (in-cluster split-K, early-fixup readiness counters) --
-// compiled out of the default instantiations (the decode weight stream is sensitive
-// to extra control flow in this kernel: a measured 10 % for a few branches)
-template <bool EXT, bool OPT>
+template <bool EXT>
 __global__ void __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmParams p) {
@@ -213,11 +193,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   uint64_t* tmem_full = bars + 2 * S;       // [TS]
   uint64_t* tmem_empty = bars + 2 * S + 4;  // [TS]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 8);
-  uint64_t* red_full = bars + 2 * S + 9;    // [2] cluster split-K: all chunks' partials staged
-  uint64_t* red_empty = bars + 2 * S + 11;  // [2] cluster split-K: all CTAs done reading a stage
-  float* red0 = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 512);   // [2][bn][128] fp32
-  const bool cl = OPT && p.cluster > 1;
-
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -235,11 +210,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       mbar_init(&tmem_full[i], 1);
       mbar_init(&tmem_empty[i], 4);   // one arrive per epilogue warp
     }
-    if (cl)
-      for (int i = 0; i < 2; ++i) {
-        mbar_init(&red_full[i], 4 * p.cluster);    // every epilogue warp of every CTA of the cluster
-        mbar_init(&red_empty[i], 4 * p.cluster);
-      }
     fence_barrier_init();
   }
   if (warp == 0 && lane == 0) {
@@ -250,7 +220,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  if (cl) cluster_sync_all();   // peers' barriers are initialised before any remote arrive
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp == 0) {
@@ -274,26 +243,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
           }
         }
         pre = it;
-        // While the preceding kernels (fixup, attention, add + LN) finish -- they
-        // leave HBM mostly idle -- pull the next weight blocks of this CTA's own
-        // stream into L2 (a hint; the TMA loads below read them from there).
-        int left = p.pf_blocks, skip = pre;
-        for (int u = blockIdx.x; u < p.units && left > 0; u += G) {
-          const Unit w = unit_of(p, u);
-          if (w.mt) continue;
-          const int k0b = w.z * (p.kc / BK);
-          const int nkb = (min(p.K, w.z * p.kc + p.kc) - w.z * p.kc + BK - 1) / BK;
-          int b0 = skip < nkb ? skip : nkb;
-          skip -= b0;
-          int nb = nkb - b0;
-          if (nb > left) nb = left;
-          if (nb <= 0) continue;
-          const int nt = (p.n0 / BM) + w.nt;
-          bulk_prefetch_l2(reinterpret_cast<const uint8_t*>(p.w_base) +
-                               ((size_t)nt * p.nkb_total + k0b + b0) * A_BYTES,
-                           (uint32_t)nb * A_BYTES);
-          left -= nb;
-        }
       }
       grid_dependency_wait();
       grid_dependency_trigger();   // after the wait: dependents overlap only this kernel
@@ -350,13 +299,12 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
     const int row = q * 32 + lane;
     const int etid = threadIdx.x - 64;
     const int tiles = p.n_tiles * p.m_tiles;
-    const uint32_t crank = cl ? cluster_ctarank() : 0;   // == the unit's K chunk z
-    float* lnst = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 512 + (cl ? 2 * BM * p.bn * 4 : 0));
+    float* lnst = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 512);
     if (EXT && p.ln_fold) {
       // row statistics of the raw input while the producer / MMA warps run the
       // mainloop (X comes from the preceding kernel: wait for it first)
       grid_dependency_wait();
-      if (p.splits == 1 || cl) {   // this CTA's epilogue applies the fold: every row here
+      if (p.splits == 1) {   // this CTA's epilogue applies the fold: every row here
         ln_row_stats(p.ln_x, p.ln_ldx, p.M, p.K, p.ln_eps, lnst, etid, 128);
         named_bar_sync(1, 128);
       } else {
@@ -364,10 +312,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
         for (int m = blockIdx.x + (etid >> 5) * G; m < p.M; m += 4 * G) {
           ln_row_stats(p.ln_x + (int64_t)m * p.ln_ldx, p.ln_ldx, 1, p.K, p.ln_eps, p.ln_stats + 2 * m, lane, 32);
           __syncwarp();
-          if (OPT && lane == 0 && p.tile_ready) {   // row m's statistics are out (the fixup waits for all M)
-            __threadfence();
-            atomicAdd(p.tile_ready + GEMM_STATS_CNT, 1u);
-          }
         }
       }
     }
@@ -383,9 +327,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       const int mcount = min(p.bn, p.M - m_base);
       const int tile_id = w.nt * p.m_tiles + w.mt;
       // fp32 partial of (chunk z, tile): [bn cols][128 rows] (a warp writes 128 B per column)
-      float* my_ws = (p.splits > 1 && !cl) ? p.ws + ((int64_t)w.z * tiles + tile_id) * (BM * p.bn) + row : nullptr;
-      float* red = red0 + (lu & 1) * (BM * p.bn);
-      if (cl && lu >= 2) mbar_wait_cluster(&red_empty[lu & 1], ((lu >> 1) - 1) & 1);
+      float* my_ws = p.splits > 1 ? p.ws + ((int64_t)w.z * tiles + tile_id) * (BM * p.bn) + row : nullptr;
       mbar_wait(&tmem_full[acc], acc_ph);
       tc_fence_after();
       const uint32_t tacc = tmem_base + (uint32_t)acc * acc_cols + ((uint32_t)(q * 32) << 16);
@@ -401,10 +343,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
               if (c0 + j < mcount)
                 epi_store<EXT>(p, m_base + c0 + j, n, epi_apply<EXT>(p, __uint_as_float(r[j]), m_base + c0 + j, n, bias_v, lnst));
           }
-        } else if (cl) {
-#pragma unroll
-          for (int j = 0; j < 16; ++j)
-            if (c0 + j < mcount) red[(c0 + j) * BM + row] = __uint_as_float(r[j]);
         } else {
 #pragma unroll
           for (int j = 0; j < 16; ++j)
@@ -415,63 +353,6 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tmem_empty[acc]);
-      if (OPT && p.splits > 1 && !cl && p.tile_ready) {
-        // chunk w.z of this tile is in the workspace: count it (the fixup reduces a
-        // tile as soon as all its chunks have arrived, during this grid's tail)
-        named_bar_sync(2, 128);
-        if (etid == 0) {
-          __threadfence();
-          atomicAdd(&p.tile_ready[tile_id], 1u);
-        }
-      }
-      if (cl) {
-        // In-cluster split-K reduction (replaces the fixup kernel): the S CTAs of the
-        // cluster hold chunks z = 0..S-1 of this tile in shared memory; CTA z sums
-        // slice z of the tile's elements over the S chunks in z order (the fixup's
-        // order: the same bits) through DSMEM and applies the epilogue.
-        if (lane == 0)
-          for (int r = 0; r < p.cluster; ++r) mbar_arrive_remote(&red_full[lu & 1], (uint32_t)r);
-        mbar_wait_cluster(&red_full[lu & 1], (lu >> 1) & 1);
-        const int E4 = mcount * (BM / 4);
-        const int lo = (int)((int64_t)E4 * crank / p.cluster), hi = (int)((int64_t)E4 * (crank + 1) / p.cluster);
-        const uint32_t red_local = smem_u32(red);
-        for (int e = lo + etid; e < hi; e += 128) {
-          const uint32_t off = red_local + (uint32_t)e * 16u;
-          float4 v[8];
-#pragma unroll
-          for (int i = 0; i < 8; ++i)
-            if (i < p.cluster) v[i] = ld_dsmem_f4(dsmem_map(off, (uint32_t)i));
-          float4 a = v[0];
-#pragma unroll
-          for (int i = 1; i < 8; ++i)
-            if (i < p.cluster) {
-              a.x += v[i].x;
-              a.y += v[i].y;
-              a.z += v[i].z;
-              a.w += v[i].w;
-            }
-          const int col = e >> 5, rq = e & 31;
-          const float av[4] = {a.x, a.y, a.z, a.w};
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const int nn = n_base + rq * 4 + i;
-            if (nn < p.n1 && nn < p.N) {
-              const float bv = p.bias ? __bfloat162float(p.bias[nn]) : 0.0f;
-              epi_store<EXT>(p, m_base + col, nn, epi_apply<EXT>(p, av[i], m_base + col, nn, bv, lnst));
-            }
-          }
-        }
-        __syncwarp();
-        if (lane == 0)
-          for (int r = 0; r < p.cluster; ++r) mbar_arrive_remote(&red_empty[lu & 1], (uint32_t)r);
-      }
-    }
-    if (cl) {
-      // peers read this CTA's shared memory: stay resident until they are done
-      for (int buf = 0; buf < 2; ++buf) {
-        const int j = (((lu - 1) & 1) == buf) ? lu - 1 : lu - 2;   // last unit staged in buf
-        if (j >= 0) mbar_wait_cluster(&red_empty[buf], (j >> 1) & 1);
-      }
     }
   }
   tc_fence_before();
@@ -483,31 +364,12 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   if (threadIdx.x == 0) trace_write(TK_GEMM, tr0, tr1);
 }
 
-// sum_{z=0..S-1} src[z * zstride] in chunk order, 8 loads in flight
-__device__ __forceinline__ float sum_partials(const float* src, int64_t zstride, int S) {
-  float acc = __ldcg(src);
-  for (int z0 = 1; z0 < S; z0 += 8) {
-    float v[8];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) v[i] = (z0 + i < S) ? __ldcg(src + (z0 + i) * zstride) : 0.f;
-#pragma unroll
-    for (int i = 0; i < 8; ++i)
-      if (z0 + i < S) acc += v[i];
-  }
-  return acc;
-}
-
 // Split-K fixup: out[m, n] = epi( sum_{z=0..S-1} partial[z] ) in chunk order (the
 // same bits whatever slice or CTA produced each chunk).  One thread per (m, 4 rows n),
 // reading the column-major per-tile partials coalesced.
 template <bool EXT>
 __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) {
   const uint64_t tr0 = trace_now();
-  // With tile_ready, a tile is reduced as soon as all its chunks are in (acquire on
-  // its counter), overlapping the GEMM grid's tail; the wait for the GEMM grid to
-  // complete comes at the end, so this kernel's completion still implies the
-  // GEMM's.  Without it (tile count beyond the counter region): wait up front.
-  const bool early = p.tile_ready != nullptr;
   const int tiles = p.n_tiles * p.m_tiles;
   const int64_t zstride = (int64_t)tiles * (BM * p.bn);
   const int slice_w = p.n1 - p.n0;
@@ -518,7 +380,7 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
   // by a fixup at least three kernels back -- so they are loaded before the PDL wait.
   float pb[4] = {0.f, 0.f, 0.f, 0.f}, pu[4] = {0.f, 0.f, 0.f, 0.f}, pc[4] = {0.f, 0.f, 0.f, 0.f},
         pr[4] = {0.f, 0.f, 0.f, 0.f};
-  if (!early && t_first < total) {
+  if (t_first < total) {
     const int rq = (int)(t_first % (BM / 4));
     const int64_t t2 = t_first / (BM / 4);
     const int nt = (int)(t2 % p.n_tiles);
@@ -537,14 +399,9 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
       }
     }
   }
-  if (!early) pdl_enter();
-  else grid_dependency_trigger();   // the next GEMM's weight prefetch overlaps this kernel, as before
+  pdl_enter();
   const uint64_t tr1 = trace_now();
   const float* lnst = p.ln_stats;
-  if (EXT && early && p.ln_fold && (threadIdx.x & 31) == 0) {   // every row's statistics are out
-    while (ld_acquire_u32(p.tile_ready + GEMM_STATS_CNT) < (unsigned)p.M) __nanosleep(200);
-  }
-  __syncwarp();
   for (int64_t t = t_first; t < total; t += (int64_t)gridDim.x * blockDim.x) {
     const int rq = (int)(t % (BM / 4));
     const int64_t t2 = t / (BM / 4);
@@ -552,11 +409,6 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
     const int m = (int)(t2 / p.n_tiles);
     const int mt = m / p.bn, col = m % p.bn;
     const int tile_id = nt * p.m_tiles + mt;
-    if (early) {   // warp-uniform: a warp covers the 32 row groups of one (m, tile)
-      if ((threadIdx.x & 31) == 0)
-        while (ld_acquire_u32(p.tile_ready + tile_id) < (unsigned)p.splits) __nanosleep(200);
-      __syncwarp();
-    }
     const float4* src = reinterpret_cast<const float4*>(p.ws + (int64_t)tile_id * (BM * p.bn) + (int64_t)col * BM) + rq;
     // chunk order z = 0..S-1; a group of 8 chunks' loads are all in flight before the adds
     float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -581,7 +433,7 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
         }
     }
     const float a[4] = {acc.x, acc.y, acc.z, acc.w};
-    const bool pre = !early && t == t_first;
+    const bool pre = t == t_first;
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
       const int row = rq * 4 + i;
@@ -603,20 +455,6 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
           const float bias_v = p.bias ? __bfloat162float(p.bias[n]) : 0.0f;
           epi_store<EXT>(p, m, n, epi_apply<EXT>(p, a[i], m, n, bias_v, lnst));
         }
-      }
-    }
-  }
-  if (early) {
-    grid_dependency_wait();   // the GEMM grid has completed (its dependents may rely on that)
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      if (atomicAdd(p.tile_ready + GEMM_DONE_CNT, 1u) == gridDim.x - 1) {   // last CTA: re-zero the counters
-        const int tiles_all = p.n_tiles * p.m_tiles;
-        for (int t = 0; t < tiles_all; ++t) p.tile_ready[t] = 0;
-        p.tile_ready[GEMM_STATS_CNT] = 0;
-        p.tile_ready[GEMM_DONE_CNT] = 0;
-        __threadfence();
       }
     }
   }
@@ -722,12 +560,6 @@ void gemm_forget_pointer_range(const void* base, size_t bytes) {
 }
 
 
-// Tiling policy.  A decomposition piece of a GEMM (a column slice [n0, n1)) keeps
-// the full GEMM's (M, N, K), so every per-element quantity -- the token tiling
-// bn, the split-K chunk kc, the K order inside a chunk and the z-order of the
-// split reduction -- is a function of (M, N, K) and identical for the full GEMM
-// and all of its slices: slices are bit-exact.  The split count is chosen by a
-// small cost model that balances units over the SMs.
 // Pipeline stages for a token tile bn within a per-CTA shared-memory budget.
 static int stages_for(int bn, int extra_smem, int budget) {
   const int stage_bytes = A_BYTES + bn * BK * 2;
@@ -742,46 +574,7 @@ static int stages_for(int bn, int extra_smem, int budget) {
   return st;
 }
 
-static int cluster_red_bytes(int bn) { return 2 * BM * bn * (int)sizeof(float); }
-// Cluster (decode) mode runs two CTAs per SM: a CTA gets half of the SM's 228 KiB
-// minus the 1 KiB the hardware reserves per CTA.
-constexpr int CLUSTER_CTA_SMEM = 233472 / 2 - 1024;
 constexpr int LN_STATS_SMEM = 2 * 64 * 4;   // folded-LayerNorm row statistics (M <= 64)
-static int cluster_smem(int bn) {
-  const int red = cluster_red_bytes(bn) + LN_STATS_SMEM;
-  return 1024 + stages_for(bn, red, CLUSTER_CTA_SMEM) * (A_BYTES + bn * BK * 2) + 512 + red;
-}
-
-// Co-resident (S x 1 x 1) clusters of gemm_tc_kernel in cluster (decode) mode
-// (clusters must fit inside a GPC; up to two CTAs per SM).
-static int max_clusters(int S, int bn) {
-  static std::mutex mu;
-  static std::unordered_map<int, int> cache;
-  const int key = S * 1024 + bn;
-  std::lock_guard<std::mutex> g(mu);
-  auto it = cache.find(key);
-  if (it != cache.end()) return it->second;
-  cudaFuncSetAttribute(gemm_tc_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
-  cudaFuncSetAttribute(gemm_tc_kernel<false, true>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(S * 128);
-  cfg.blockDim = dim3(GEMM_THREADS);
-  cfg.dynamicSmemBytes = cluster_smem(bn);
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = S;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 1;
-  int n = 0;
-  if (cudaOccupancyMaxActiveClusters(&n, gemm_tc_kernel<false, true>, &cfg) != cudaSuccess || n <= 0) {
-    cudaGetLastError();
-    n = 0;   // cluster mode unavailable for this S
-  }
-  cache[key] = n;
-  return n;
-}
 
 // Tiling policy.  A decomposition piece of a GEMM (a column slice [n0, n1)) keeps
 // the full GEMM's (M, N, K), so every per-element quantity -- the token tiling
@@ -789,12 +582,9 @@ static int max_clusters(int S, int bn) {
 // split reduction -- is a function of (M, N, K) and identical for the full GEMM
 // and all of its slices: slices are bit-exact.  The split count is chosen by a
 // small cost model that balances the weight stream over the SMs.  Split chunks
-// are summed by the PDL-chained fixup kernel.  Opt-in (LIGER_GEMM_CLUSTER=1):
-// decode GEMMs (M <= 64) reduce their K chunks inside a thread-block cluster
-// (S <= 8 CTAs, DSMEM) instead -- the same z order, so the same bits.  Measured
-// slower (OPT-13B decode chain 130 vs 117 us/layer, pass 5.7-5.9 vs 5.4 ms):
-// with N/128 = 40 tiles a cluster of S CTAs per tile keeps only 40 S <= 148 SMs
-// streaming, and larger S leaves clusters waiting for whole free GPC slots.
+// are summed by the PDL-chained fixup kernel.  (An in-cluster DSMEM reduction, a
+// last-CTA reduction and an early fixup were built, measured slower and removed:
+// profiles/r01/cluster_splitk.txt.)
 GemmPlan gemm_plan(int M, int N, int K) {
   GemmPlan pl{};
   const int G = num_sms();
@@ -805,38 +595,22 @@ GemmPlan gemm_plan(int M, int N, int K) {
   bn = (bn + 15) / 16 * 16;
   if (bn < 16) bn = 16;
   const int tiles = n_tiles * mt;
-  static const bool cluster_on = getenv("LIGER_GEMM_CLUSTER") && atoi(getenv("LIGER_GEMM_CLUSTER")) != 0;
-  const bool use_cluster = cluster_on && M <= 64;
-  // Cost model in SM cycles: a k-block costs max(MMA = 8 bn, weight stream at
-  // ~23 B/clk/SM + activation tile from L2 at ~64 B/clk); a unit adds 300.
-  // Non-cluster: units spread over G persistent CTAs; a split adds the fixup
-  // kernel (launch + S*M*N*4 B of partial traffic x 2).  Cluster: waves of
-  // co-resident clusters, an SM holding two CTAs streams for both; each wave
-  // adds the DSMEM exchange.
+  // Cost model in SM cycles (prefill): a k-block costs max(MMA = 8 bn, weight
+  // stream at ~23 B/clk/SM + activation tile from L2 at ~64 B/clk); a unit adds
+  // 300; units spread over G persistent CTAs; a split adds the fixup kernel
+  // (launch + S*M*N*4 B of partial traffic x 2).
   const double kb_time = fmax(8.0 * bn, A_BYTES / 23.0 + 128.0 * bn / 64.0);
-  int best_s = 1, best_nc = 0;
+  int best_s = 1;
   double best = 1e300;
   // Prefill GEMMs that already fill the SMs are not split (their fp32 partials
   // would exceed L2); decode GEMMs always consider it.
-  int smax = (M > 64 && tiles >= G) ? 1 : (nkb >= 8 ? nkb / 4 : 1);
-  if (use_cluster && smax > 8) smax = 8;
+  const int smax = (M > 64 && tiles >= G) ? 1 : (nkb >= 8 ? nkb / 4 : 1);
   for (int sp = 1; sp <= smax; ++sp) {
     const int kcb = (nkb + sp - 1) / sp;
     const int S = (nkb + kcb - 1) / kcb;
     if (S != sp) continue;
     double cost;
-    int nc = 0;
-    if (use_cluster && S > 1) {
-      nc = max_clusters(S, bn);
-      if (nc <= 0) continue;
-      if (nc > tiles) nc = tiles;
-      cost = 0.0;
-      for (int left = tiles; left > 0; left -= nc) {
-        const int ctas = std::min(left, nc) * S;
-        cost += (double)((ctas + G - 1) / G) * (kcb * kb_time + 300.0) + 1200.0;
-      }
-      cost /= 1900.0;   // SM cycles -> us (M <= 64 here: compared with the decode model below)
-    } else if (M <= 64) {
+    if (M <= 64) {
       // Decode (weight stream), in us, fitted to tools/split_sweep2.py on B200
       // (profiles/r01/split_sweep_decode.txt): the persistent grid runs rounds of
       // up to G units; a round takes max(its weight bytes at the achievable HBM
@@ -858,36 +632,25 @@ GemmPlan gemm_plan(int M, int N, int K) {
     if (cost < best - 1e-9) {
       best = cost;
       best_s = S;
-      best_nc = nc;
     }
   }
   if (const char* e = getenv("LIGER_GEMM_FORCE_SPLITS")) {   // experiments only
     const int f = atoi(e);
-    if (f >= 1 && f <= nkb && (!use_cluster || f <= 8)) {
-      best_s = f;
-      best_nc = (use_cluster && f > 1) ? std::min(max_clusters(f, bn), tiles) : 0;
-    }
+    if (f >= 1 && f <= nkb) best_s = f;
   }
   const int kcb = (nkb + best_s - 1) / best_s;
   pl.bn = bn;
   pl.m_tiles = mt;
   pl.kc = kcb * BK;
   pl.splits = (nkb + kcb - 1) / kcb;
-  pl.cluster = (use_cluster && pl.splits > 1 && best_nc > 0) ? pl.splits : 1;
-  pl.clusters = pl.cluster > 1 ? best_nc : 0;
-  if (pl.cluster > 1) {
-    pl.stages = stages_for(bn, cluster_red_bytes(bn) + LN_STATS_SMEM, CLUSTER_CTA_SMEM);
-    pl.smem = cluster_smem(bn);
-  } else {
-    pl.stages = stages_for(bn, LN_STATS_SMEM, MAX_SMEM);
-    pl.smem = 1024 + pl.stages * (A_BYTES + pl.bn * BK * 2) + 512 + LN_STATS_SMEM;
-  }
+  pl.stages = stages_for(bn, LN_STATS_SMEM, MAX_SMEM);
+  pl.smem = 1024 + pl.stages * (A_BYTES + pl.bn * BK * 2) + 512 + LN_STATS_SMEM;
   return pl;
 }
 
 size_t gemm_workspace_bytes(int M, int N, int K) {
   GemmPlan pl = gemm_plan(M, N, K);
-  if (pl.splits <= 1 || pl.cluster > 1) return GEMM_COUNTER_BYTES;
+  if (pl.splits <= 1) return GEMM_COUNTER_BYTES;
   const size_t tiles = (size_t)((N + BM - 1) / BM + 1) * pl.m_tiles;   // +1: unaligned slices
   return GEMM_COUNTER_BYTES + (size_t)pl.splits * tiles * BM * pl.bn * sizeof(float);
 }
@@ -897,7 +660,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (a.K <= 0 || a.K % 8 || a.ldx % 8 || (!a.w_tiled && a.ldw % 8) || a.n0 < 0 || a.n1 > a.N) return LIGER_EINVAL;
   GemmPlan pl = gemm_plan(a.M, a.N, a.K);
   const int ntiles = (a.n1 - a.n0 + BM - 1) / BM;
-  if (pl.splits > 1 && pl.cluster <= 1) {
+  if (pl.splits > 1) {
     if (!a.workspace) return LIGER_EINVAL;
     const size_t need = GEMM_COUNTER_BYTES + (size_t)pl.splits * ntiles * pl.m_tiles * BM * pl.bn * sizeof(float);
     if (a.ws_bytes < need) return LIGER_EINVAL;
@@ -916,8 +679,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (rc) return rc;
   static bool attr_set = false;
   if (!attr_set) {
-    for (auto k : {gemm_tc_kernel<false, false>, gemm_tc_kernel<true, false>, gemm_tc_kernel<false, true>,
-                   gemm_tc_kernel<true, true>}) {
+    for (auto k : {gemm_tc_kernel<false>, gemm_tc_kernel<true>}) {
       cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
       cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     }
@@ -936,56 +698,25 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   if (a.ln_fold && (a.M > 64 || !a.ln_u || !a.ln_c || (pl.splits > 1 && !a.ln_stats) || a.K % 8)) return LIGER_EINVAL;
   const bool ext = a.ln_fold || a.resid;
   if (a.far) {   // fused all-reduce producer: needs the fixup kernel and the whole GEMM
-    if (pl.splits <= 1 || pl.cluster > 1 || a.defer_fixup || a.out_f32 || a.n0 != 0 || a.n1 != a.N)
-      return LIGER_EINVAL;
+    if (pl.splits <= 1 || a.out_f32 || a.n0 != 0 || a.n1 != a.N) return LIGER_EINVAL;
     p.out = a.far->stage;
     p.ldo = a.N;
     p.pub_flag = a.far->flag;
     p.pub_counter = a.far->counter;
     p.pub_epoch = a.far->epoch;
   }
-  p.counters = reinterpret_cast<int*>(a.workspace);
-  p.tile_ready = nullptr;
   p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
   p.w_tiled = a.w_tiled;
-  p.w_base = a.w;
-  static const int pf_env = getenv("LIGER_PF_BLOCKS") ? atoi(getenv("LIGER_PF_BLOCKS")) : 0;
-  p.pf_blocks = (a.w_tiled && pl.bn <= 64) ? pf_env : 0;
-
   p.nkb_total = (a.K + BK - 1) / BK;
   p.n_tiles = ntiles;
   p.m_tiles = pl.m_tiles;
   p.units = ntiles * pl.m_tiles * pl.splits;
-  {
-    // early fixup (opt-in LIGER_EARLY_FIXUP=1; tile readiness counters in the
-    // workspace's counter region): the fixup reduces each tile as soon as its chunks
-    // are in, during the GEMM grid's tail.  Bit-identical, but measured slower
-    // (OPT-13B decode pass 5635 vs 5181 us at b = 2, 6132 vs 5634 at b = 8): the
-    // fixup CTAs launched next to the persistent GEMM poll and occupy SM slots.
-    static const bool early_env = getenv("LIGER_EARLY_FIXUP") ? atoi(getenv("LIGER_EARLY_FIXUP")) != 0 : false;
-    const bool will_fixup = pl.splits > 1 && pl.cluster <= 1 && !a.defer_fixup;
-    if (will_fixup && early_env && a.workspace && ntiles * pl.m_tiles <= GEMM_MAX_READY_TILES)
-      p.tile_ready = reinterpret_cast<unsigned int*>(a.workspace);
-  }
-  p.cluster = pl.cluster;
-  int rc2;
-  if (pl.cluster > 1) {
-    // one cluster of `splits` CTAs per tile in flight; CTA z of a cluster takes chunk z
-    // (grid = clusters x S, so unit u = blockIdx.x + j * grid keeps z = blockIdx.x % S)
-    const int nc = std::min(pl.clusters, ntiles * pl.m_tiles);
-    rc2 = ext ? launch_pdl_cluster(gemm_tc_kernel<true, true>, dim3(nc * pl.cluster), dim3(GEMM_THREADS),
-                                   pl.cluster, pl.smem, stream, tA, tB, p)
-              : launch_pdl_cluster(gemm_tc_kernel<false, true>, dim3(nc * pl.cluster), dim3(GEMM_THREADS),
-                                   pl.cluster, pl.smem, stream, tA, tB, p);
-  } else {
-    // unit u runs on CTA u % grid: the grid size never changes what a unit computes
-    const int sms = (a.sm_budget > 0 && a.sm_budget < num_sms()) ? a.sm_budget : num_sms();
-    const int grid = p.units < sms ? p.units : sms;
-    auto kern = p.tile_ready ? (ext ? gemm_tc_kernel<true, true> : gemm_tc_kernel<false, true>)
-                             : (ext ? gemm_tc_kernel<true, false> : gemm_tc_kernel<false, false>);
-    rc2 = launch_pdl(kern, dim3(grid), dim3(GEMM_THREADS), pl.smem, stream, tA, tB, p);
-  }
-  const bool fixup = p.splits > 1 && pl.cluster <= 1 && !a.defer_fixup;
+  // unit u runs on CTA u % grid: the grid size never changes what a unit computes
+  const int sms = (a.sm_budget > 0 && a.sm_budget < num_sms()) ? a.sm_budget : num_sms();
+  const int grid = p.units < sms ? p.units : sms;
+  const int rc2 = launch_pdl(ext ? gemm_tc_kernel<true> : gemm_tc_kernel<false>, dim3(grid), dim3(GEMM_THREADS),
+                             pl.smem, stream, tA, tB, p);
+  const bool fixup = p.splits > 1;
   if (a.had_fixup) *a.had_fixup = fixup;
   if (a.ev_mid) cudaEventRecord(a.ev_mid, stream);
   if (rc2 || !fixup) return rc2 ? LIGER_ECUDA : 0;

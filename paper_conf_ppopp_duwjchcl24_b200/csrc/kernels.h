@@ -13,8 +13,6 @@ constexpr size_t ATTN_COUNTER_BYTES = 16384;
 
 struct GemmPlan {
   int bn, m_tiles, kc, splits, stages, smem;
-  int cluster;    // > 1: splits reduced in-kernel over a (splits x 1 x 1) cluster (no fixup kernel)
-  int clusters;   // cluster mode: co-resident clusters the persistent grid uses
 };
 
 // Descriptor of one fused all-reduce (epoch) for kernels that do the one-shot
@@ -52,9 +50,6 @@ struct GemmArgs {
   // (per-kernel timing; breaks the PDL overlap of the two)
   cudaEvent_t ev_mid = nullptr;
   bool* had_fixup = nullptr;
-  // split-K partials are left in the workspace for a following
-  // splitk_add_layernorm_launch instead of being summed by the fixup kernel
-  bool defer_fixup = false;
   // t > 1 fused all-reduce: the fixup kernel writes the bf16 result into far->stage
   // (row-major [M, N], replacing `out`) and publishes far->epoch when the grid is done
   const FusedARDesc* far = nullptr;
@@ -83,41 +78,9 @@ void gemm_forget_pointer_range(const void* base, size_t bytes);
 int gemm_weight_map(void* out_map, const void* w_tiled, int N, int K);
 int gemm_act_map(void* out_map, const void* x, int M, int K, int64_t ldx, int bn);
 
-// Fused decode pass (decode_fused.cu): every layer of [l0, l1) of one decode step
-// of one batch (M = b <= 32 tokens, t = 1) in one persistent kernel.
-struct FusedLayerPtrs {
-  const void *b_qkv, *b_o, *b_1, *b_2, *g1, *be1, *g2, *be2;
-  const void *w_qkv, *w_o, *w_1, *w_2;   // tiled weights
-};
-struct FusedDecodeArgs {
-  int L, M, h, heads, d, ffn, act;
-  int pos;             // position of the new token (context = pos + 1)
-  float eps, qscale;
-  int first_no_add;    // layer 0 of the range: x is complete (embedding / received), LN1 adds nothing
-  const FusedLayerPtrs* layers;   // host array [L]
-  void *x, *y, *qkv, *attn, *part, *hbuf;
-  void* kv;            // KV pool of the range's first layer; layer i at kv + i * kv_layer_elems
-  int64_t kv_layer_elems;
-  const int32_t* page_table;
-  int max_pages;
-  void* gemm_ws;       // split-K workspace (GEMM_COUNTER_BYTES of counters + partials)
-  size_t gemm_ws_bytes;
-  void* attn_ws;       // decode-attention workspace
-  size_t attn_ws_bytes;
-};
-struct FusedDecodeState;   // per-slot device tables (weight descriptors, sync counter base)
-bool fused_decode_supported(int M, int h, int heads, int d, int ffn);
-int fused_decode_launch(FusedDecodeState** state, const FusedDecodeArgs& a, cudaStream_t stream);
-void fused_decode_free(FusedDecodeState* state);
-
 int add_layernorm_launch(const void* x, const void* add, const void* add_bias, void* x_out, void* y,
                          const void* gamma, const void* beta, int rows, int h, int in_row_step, int in_row_off,
                          float eps, cudaStream_t stream);
-// add + LN whose added operand is the split-K sum of the preceding row-parallel GEMM
-// (launched with defer_fixup); bit-identical to splitk fixup -> add_layernorm_launch.
-int splitk_add_layernorm_launch(const float* ws, int64_t zstride, int splits, int m_tiles, int bn, const void* x,
-                                const void* add_bias, void* x_out, void* y, const void* gamma, const void* beta,
-                                int rows, int h, float eps, cudaStream_t stream);
 // add + LN whose added operand is the all-reduce (rank-ordered fp32 sum, RNE to bf16)
 // of the peers' staged partials of epoch far.epoch; waits for every peer's flag.
 int peer_add_layernorm_launch(const FusedARDesc& far, const void* x, const void* add_bias, void* x_out, void* y,
@@ -150,6 +113,5 @@ struct TraceRec;
 void trace_set_gemm(TraceRec* rec, unsigned int* n, unsigned int cap);
 void trace_set_norm(TraceRec* rec, unsigned int* n, unsigned int cap);
 void trace_set_attention(TraceRec* rec, unsigned int* n, unsigned int cap);
-void trace_set_fused(TraceRec* rec, unsigned int* n, unsigned int cap);
 
 }  // namespace liger

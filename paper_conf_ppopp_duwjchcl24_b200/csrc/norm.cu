@@ -43,34 +43,19 @@ __device__ __forceinline__ float block_sum(float v, float* red) {
   return s;
 }
 
-// Split-K partials of a row-parallel projection (gemm.cu layout): the fp32 partial
-// of chunk z for output (m, n) is at ws[z * zstride + tile(n, m) * 128 * bn +
-// (m % bn) * 128 + n % 128], tile(n, m) = (n / 128) * m_tiles + m / bn.
-struct SplitSrc {
-  const float* ws;
-  int64_t zstride;
-  int splits, m_tiles, bn;
-};
-
 // One CTA per output row; each thread owns up to MAXV 8-element vectors.  All
 // global loads of a row (x, add, bias, gamma, beta) are issued before any use so
 // the kernel pays one memory round trip (decode rows are latency-bound).
-// SPLIT: the added operand is not read from `add` but is the split-K sum of the
-// preceding GEMM, formed here exactly as the fixup kernel would have formed it
-// (chunks summed in z order from chunk 0, + 0 bias, RNE to bf16), so the result
-// is bit-identical to fixup -> add + LN with one kernel and one hand-off fewer.
 // PEER: the added operand is the fused all-reduce of the row-parallel partials the
 // peers staged for epoch far.epoch (peer_ar.cu protocol): wait for every peer's
 // flag, then sum the staged rows over ranks 0..t-1 in fp32 in that order and round
 // to bf16 -- the one-shot all-reduce's bits, without its kernel.
-template <int NT, int MAXV, int MODE>
+template <int NT, int MAXV, bool PEER>
 __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x, const bf16x8* __restrict__ add,
                                                     const bf16x8* __restrict__ add_bias, bf16x8* x_out,
                                                     bf16x8* __restrict__ y, const bf16x8* __restrict__ gamma,
                                                     const bf16x8* __restrict__ beta, int h, int in_row_step,
-                                                    int in_row_off, float eps, const SplitSrc sp,
-                                                    const FusedARDesc far) {
-  constexpr bool SPLIT = MODE == 1, PEER = MODE == 2;
+                                                    int in_row_off, float eps, const FusedARDesc far) {
   __shared__ float red[NT / 32];
   const uint64_t tr0 = trace_now();
   const int nv = h >> 3;
@@ -84,7 +69,7 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
   // (by the previous add + LN; the partial `add` comes from the preceding kernel):
   // their loads are issued before the wait.  Without `add`, x may come from the
   // preceding kernel (the embedding) and is loaded after it.
-  const bool x_early = SPLIT || PEER || add != nullptr;
+  const bool x_early = PEER || add != nullptr;
 #pragma unroll
   for (int j = 0; j < MAXV; ++j) {
     const int v = threadIdx.x + j * NT;
@@ -122,7 +107,7 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
     const int v = threadIdx.x + j * NT;
     if (v < nv) {
       if (!x_early) vx[j] = xr[v];
-      if (!SPLIT && !PEER && add) va[j] = add[in_row * nv + v];
+      if (!PEER && add) va[j] = add[in_row * nv + v];
     }
   }
   if (PEER) {
@@ -153,47 +138,6 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
       }
     }
   }
-  if (SPLIT) {
-    const int m = (int)in_row, mt = m / sp.bn, col = m % sp.bn;
-    float acc[MAXV][8];
-    for (int z0 = 0; z0 < sp.splits; z0 += 4) {
-      float4 t[4][MAXV][2];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < MAXV; ++j) {
-          const int v = threadIdx.x + j * NT;
-          if (z0 + i < sp.splits && v < nv) {
-            const int n = v * 8;
-            const float* src = sp.ws + (int64_t)(z0 + i) * sp.zstride +
-                               ((int64_t)((n >> 7) * sp.m_tiles + mt) * 128 * sp.bn) + col * 128 + (n & 127);
-            t[i][j][0] = __ldcg(reinterpret_cast<const float4*>(src));
-            t[i][j][1] = __ldcg(reinterpret_cast<const float4*>(src + 4));
-          }
-        }
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < MAXV; ++j) {
-          const int v = threadIdx.x + j * NT;
-          if (z0 + i < sp.splits && v < nv) {
-            const float f[8] = {t[i][j][0].x, t[i][j][0].y, t[i][j][0].z, t[i][j][0].w,
-                                t[i][j][1].x, t[i][j][1].y, t[i][j][1].z, t[i][j][1].w};
-#pragma unroll
-            for (int e = 0; e < 8; ++e) acc[j][e] = (z0 + i == 0) ? f[e] : acc[j][e] + f[e];
-          }
-        }
-    }
-#pragma unroll
-    for (int j = 0; j < MAXV; ++j) {
-      const int v = threadIdx.x + j * NT;
-      if (v < nv) {
-#pragma unroll
-        for (int e = 0; e < 8; ++e) acc[j][e] += 0.0f;   // the fixup's (zero) bias term
-        va[j] = pack8(acc[j]);
-      }
-    }
-  }
   float r[MAXV][8];
   float s = 0.f;
 #pragma unroll
@@ -201,7 +145,7 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
     const int v = threadIdx.x + j * NT;
     if (v < nv) {
       unpack8(vx[j], r[j]);
-      if (SPLIT || PEER || add) {
+      if (PEER || add) {
         float a[8];
         unpack8(va[j], a);
 #pragma unroll
@@ -259,34 +203,10 @@ int add_layernorm_launch(const void* x, const void* add, const void* add_bias, v
   const bf16x8* A = (const bf16x8*)add;
   const bf16x8* AB = (const bf16x8*)add_bias;
   const int nv = h / 8;
-  const SplitSrc none{};
   const FusedARDesc nofar{};
 #define LIGER_LN(NT, MV)                                                                                  \
-  launch_pdl(add_ln_kernel<NT, MV, 0>, dim3(rows), dim3(NT), 0, stream, X, A, AB, (bf16x8*)x_out,         \
-             (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, in_row_step, in_row_off, eps, none,  \
-             nofar)
-  int rc;
-  if (nv <= 128) rc = LIGER_LN(128, 1);
-  else if (nv <= 512) rc = LIGER_LN(128, 4);
-  else if (nv <= 1024) rc = LIGER_LN(256, 4);
-  else rc = LIGER_LN(512, 4);
-#undef LIGER_LN
-  return rc ? LIGER_ECUDA : 0;
-}
-
-int splitk_add_layernorm_launch(const float* ws, int64_t zstride, int splits, int m_tiles, int bn, const void* x,
-                                const void* add_bias, void* x_out, void* y, const void* gamma, const void* beta,
-                                int rows, int h, float eps, cudaStream_t stream) {
-  if (rows <= 0) return 0;
-  if (h % 128 || h > 16384 || !ws || splits < 1 || !x || !y || !gamma || !beta) return LIGER_EINVAL;
-  const SplitSrc sp{ws, zstride, splits, m_tiles, bn};
-  const FusedARDesc nofar{};
-  const bf16x8* X = (const bf16x8*)x;
-  const bf16x8* AB = (const bf16x8*)add_bias;
-  const int nv = h / 8;
-#define LIGER_LN(NT, MV)                                                                                      \
-  launch_pdl(add_ln_kernel<NT, MV, 1>, dim3(rows), dim3(NT), 0, stream, X, (const bf16x8*)nullptr, AB,        \
-             (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, 1, 0, eps, sp, nofar)
+  launch_pdl(add_ln_kernel<NT, MV, false>, dim3(rows), dim3(NT), 0, stream, X, A, AB, (bf16x8*)x_out,     \
+             (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, in_row_step, in_row_off, eps, nofar)
   int rc;
   if (nv <= 128) rc = LIGER_LN(128, 1);
   else if (nv <= 512) rc = LIGER_LN(128, 4);
@@ -300,13 +220,12 @@ int peer_add_layernorm_launch(const FusedARDesc& far, const void* x, const void*
                               const void* gamma, const void* beta, int rows, int h, float eps, cudaStream_t stream) {
   if (rows <= 0) return 0;
   if (h % 8 || h > 16384 || far.world < 1 || far.world > 8 || !x || !y || !gamma || !beta) return LIGER_EINVAL;
-  const SplitSrc none{};
   const bf16x8* X = (const bf16x8*)x;
   const bf16x8* AB = (const bf16x8*)add_bias;
   const int nv = h / 8;
 #define LIGER_LN(NT, MV)                                                                                      \
-  launch_pdl(add_ln_kernel<NT, MV, 2>, dim3(rows), dim3(NT), 0, stream, X, (const bf16x8*)nullptr, AB,        \
-             (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, 1, 0, eps, none, far)
+  launch_pdl(add_ln_kernel<NT, MV, true>, dim3(rows), dim3(NT), 0, stream, X, (const bf16x8*)nullptr, AB,     \
+             (bf16x8*)x_out, (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, 1, 0, eps, far)
   int rc;
   if (nv <= 128) rc = LIGER_LN(128, 1);
   else if (nv <= 512) rc = LIGER_LN(128, 4);

@@ -13,8 +13,7 @@ ACT = {"none": 0, "relu": 1, "gelu_tanh": 2}
 SYNC = {"hybrid": 0, "cpu_gpu": 1, "inter_stream": 2}
 MODE = {"serial": 0, "interleaved": 1, "pipeline": 2, "pipeline_th": 3}
 KV_BLOCK = 16
-KT_NAMES = ["gemm_decode", "attn", "ln", "allreduce", "gemm_prefill", "lm_head", "splitk_fixup",
-            "decode_fused"]   # LIGER_KT_*
+KT_NAMES = ["gemm_decode", "attn", "ln", "allreduce", "gemm_prefill", "lm_head", "splitk_fixup"]   # LIGER_KT_*
 OPS = ["embed", "ln1", "qkv", "attn", "out", "ar1", "ln2", "fc1", "fc2", "ar2", "head", "tokg", "pick",
        "recv_x", "send_x", "recv_tok", "send_tok"]
 
@@ -35,21 +34,6 @@ class liger_result(C.Structure):
     _fields_ = [("id", C.c_int64), ("batch", C.c_int32), ("seq_len", C.c_int32), ("n_new", C.c_int32),
                 ("done", C.c_int32), ("arrival_s", C.c_double), ("submit_s", C.c_double),
                 ("start_s", C.c_double), ("finish_s", C.c_double)]
-
-
-class liger_fused_layer(C.Structure):
-    _fields_ = [(n, C.c_void_p) for n in ("b_qkv", "b_o", "b_1", "b_2", "g1", "be1", "g2", "be2",
-                                          "w_qkv", "w_o", "w_1", "w_2")]
-
-
-class liger_fused_decode_args(C.Structure):
-    _fields_ = [("L", C.c_int32), ("M", C.c_int32), ("h", C.c_int32), ("heads", C.c_int32), ("d", C.c_int32),
-                ("ffn", C.c_int32), ("act", C.c_int32), ("pos", C.c_int32), ("eps", C.c_float),
-                ("qscale", C.c_float), ("first_no_add", C.c_int32), ("layers", C.POINTER(liger_fused_layer)),
-                ("x", C.c_void_p), ("y", C.c_void_p), ("qkv", C.c_void_p), ("attn", C.c_void_p),
-                ("part", C.c_void_p), ("hbuf", C.c_void_p), ("kv", C.c_void_p), ("kv_layer_elems", C.c_int64),
-                ("page_table", C.c_void_p), ("max_pages", C.c_int32), ("gemm_ws", C.c_void_p),
-                ("gemm_ws_bytes", C.c_size_t), ("attn_ws", C.c_void_p), ("attn_ws_bytes", C.c_size_t)]
 
 
 class liger_stats_t(C.Structure):
@@ -85,7 +69,6 @@ _SIGS = {
     "liger_op_gemm": (_I, [_P, _I64, _P, _I64, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),
     "liger_op_gemm_tiled": (_I, [_P, _I64, _P, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),
     "liger_op_tile_weight": (_I, [_P, _I64, _P, _I, _I, _P]),
-    "liger_op_gemm_tiled_add_layernorm": (_I, [_P, _P, _I, _I, _I, _P, _P, _P, _P, _P, _F, _P, _SZ, _P]),
     "liger_gemm_workspace_bytes": (_SZ, [_I, _I, _I]),
     "liger_gemm_plan": (_I, [_I, _I, _I, _P]),
     "liger_op_add_layernorm": (_I, [_P, _P, _P, _P, _P, _P, _P, _I, _I, _I, _I, _F, _P]),
@@ -99,7 +82,6 @@ _SIGS = {
     "liger_planner_submit": (_I, [_P, _I64, _I, _P, _P, _P]),
     "liger_plan_round": (_I, [_P, _P, _I, _P, _P, _P]),
     "liger_planner_destroy": (_I, [_P]),
-    "liger_op_decode_fused": (_I, [C.POINTER(liger_fused_decode_args), _P]),
     "liger_trace_start": (_I, [C.c_uint]),
     "liger_trace_stop": (_I, [_P, C.c_uint, _P]),
 }
@@ -171,16 +153,6 @@ def gemm_tiled(x, w_tiled, out, *, N, n0=0, n1=None, bias=None, act="none", scal
                                     _s(stream)), what="liger_op_gemm_tiled")
 
 
-def gemm_tiled_add_layernorm(x, w_tiled, x_res, y, gamma, beta, *, N, add_bias=None, eps=1e-5, workspace=None,
-                             stream=None):
-    """Row-parallel projection + residual add + LayerNorm in two kernels (t = 1)."""
-    M, K = x.shape
-    ws_b = workspace.numel() * workspace.element_size() if workspace is not None else 0
-    check(lib().liger_op_gemm_tiled_add_layernorm(_p(x), _p(w_tiled), M, N, K, _p(x_res), _p(add_bias), _p(y),
-                                                  _p(gamma), _p(beta), eps, _p(workspace), ws_b, _s(stream)),
-          what="liger_op_gemm_tiled_add_layernorm")
-
-
 def tile_weight(w, w_tiled, stream=None):
     N, K = w.shape
     check(lib().liger_op_tile_weight(_p(w), w.stride(0), _p(w_tiled), N, K, _s(stream)), what="liger_op_tile_weight")
@@ -195,9 +167,9 @@ def gemm_workspace_bytes(M, N, K):
 
 
 def gemm_plan(M, N, K):
-    out = (C.c_int32 * 7)()
+    out = (C.c_int32 * 5)()
     check(lib().liger_gemm_plan(M, N, K, out), what="liger_gemm_plan")
-    return dict(zip(("bn", "m_tiles", "kc", "splits", "stages", "cluster", "clusters"), list(out)))
+    return dict(zip(("bn", "m_tiles", "kc", "splits", "stages"), list(out)))
 
 
 def add_layernorm(x, gamma, beta, y, *, add=None, add_bias=None, x_out=None, rows=None, in_row_step=1,
@@ -241,23 +213,7 @@ def c0_fill(dst, *, seed, tensor_id, row_off=0, col_off=0, idx_row_stride, idx_c
                                  idx_row_stride, idx_col_stride, exp, kind, _s(stream)), what="liger_op_c0_fill")
 
 
-def decode_fused(layers, *, M, h, heads, d, ffn, act, pos, x, y, qkv, attn, part, hbuf, kv, kv_layer_elems,
-                 page_table, max_pages, gemm_ws, attn_ws, eps=1e-5, qscale=None, first_no_add=True, stream=None):
-    """liger_op_decode_fused: `layers` = list of dicts of torch tensors (tiled weights)."""
-    arr = (liger_fused_layer * len(layers))()
-    for i, w in enumerate(layers):
-        for n, _ in liger_fused_layer._fields_:
-            setattr(arr[i], n, w[n].data_ptr())
-    a = liger_fused_decode_args(len(layers), M, h, heads, d, ffn, ACT[act], pos, eps,
-                                qscale if qscale is not None else d ** -0.5, int(first_no_add), arr,
-                                x.data_ptr(), y.data_ptr(), qkv.data_ptr(), attn.data_ptr(), part.data_ptr(),
-                                hbuf.data_ptr(), kv.data_ptr(), kv_layer_elems, page_table.data_ptr(), max_pages,
-                                gemm_ws.data_ptr(), gemm_ws.numel() * gemm_ws.element_size(),
-                                attn_ws.data_ptr(), attn_ws.numel() * attn_ws.element_size())
-    check(lib().liger_op_decode_fused(C.byref(a), _s(stream)), None, "liger_op_decode_fused")
-
-
-TRACE_KIDS = {1: "gemm", 2: "fixup", 3: "attn_dec", 0x103: "attn_merge", 4: "attn_pre", 5: "add_ln", 9: "fused"}
+TRACE_KIDS = {1: "gemm", 2: "fixup", 3: "attn_dec", 0x103: "attn_merge", 4: "attn_pre", 5: "add_ln"}
 
 
 def trace_start(capacity=1 << 20):

@@ -337,162 +337,3 @@ def test_tp_layer_vs_oracle(L, name, t, b, s):
     for got, ref in ((out_pf, ref_pf.reshape(M, -1)), (out_dc, ref_dc.reshape(b, -1))):
         rel, mae = errs(to_np64(got), ref)
         assert rel <= REL and mae <= MAE, (rel, mae)
-
-
-_CLUSTER_CHILD = r"""
-import sys, numpy as np, torch
-sys.path.insert(0, {root!r})
-from liger_inputs import c0_values
-from paper_conf_ppopp_duwjchcl24_b200 import liger as L
-out = []
-for (M, N, K) in {shapes!r}:
-    x = torch.from_numpy(c0_values(4, 1, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K).astype(np.float32)).cuda().bfloat16()
-    w = torch.from_numpy(c0_values(4, 2, np.arange(N * K, dtype=np.uint64), -6).reshape(N, K).astype(np.float32)).cuda().bfloat16()
-    b = torch.from_numpy(c0_values(4, 3, np.arange(N, dtype=np.uint64), -4).astype(np.float32)).cuda().bfloat16()
-    ws = torch.zeros(max(L.gemm_workspace_bytes(M, N, K), 16384) // 4 + 16, dtype=torch.int32, device="cuda")
-    o = torch.zeros(M, N, dtype=torch.bfloat16, device="cuda")
-    L.gemm(x, w, o, bias=b, act="relu", workspace=ws)
-    torch.cuda.synchronize()
-    out.append((L.gemm_plan(M, N, K), o.view(torch.int16).cpu().numpy().tobytes().hex()))
-print(repr(out))
-"""
-
-
-def test_gemm_cluster_splitk_equals_fixup_kernel(L):
-    """Opt-in (LIGER_GEMM_CLUSTER=1): decode GEMMs reduce their split-K chunks inside
-    a thread-block cluster over DSMEM; the default fixup-kernel path sums the same
-    chunks in the same order, so the two must agree bit for bit (and both meet the oracle,
-    test_gemm_vs_oracle).  Shapes: OPT-13B decode projections at b = 8 and ragged M."""
-    import ast
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    shapes = [(8, 5120, 5120), (8, 5120, 20480), (8, 20480, 5120), (3, 1000, 2560), (33, 640, 4096)]
-    code = _CLUSTER_CHILD.format(root=root, shapes=shapes)
-    res = {}
-    runs = (("default", {"LIGER_GEMM_CLUSTER": "1"}),
-            ("cluster4", {"LIGER_GEMM_FORCE_SPLITS": "4", "LIGER_GEMM_CLUSTER": "1"}),
-            ("fixup4", {"LIGER_GEMM_FORCE_SPLITS": "4", "LIGER_GEMM_CLUSTER": "0"}))
-    for tag, env in runs:
-        p = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env}, capture_output=True, text=True,
-                           timeout=300)
-        assert p.returncode == 0, p.stderr[-2000:]
-        res[tag] = ast.literal_eval(p.stdout.strip().splitlines()[-1])
-    assert any(pl["cluster"] > 1 for pl, _ in res["default"]), res["default"]
-    assert all(pl["cluster"] == 4 for pl, _ in res["cluster4"]), res["cluster4"]
-    assert all(pl["cluster"] == 1 and pl["splits"] == 4 for pl, _ in res["fixup4"])
-    for (pc, hc), (pf, hf), s in zip(res["cluster4"], res["fixup4"], shapes):
-        assert pc["kc"] == pf["kc"]
-        assert hc == hf, (s, pc, pf)
-
-
-@pytest.mark.parametrize("M,N,K", [(2, 5120, 5120), (8, 5120, 20480), (5, 1024, 4096), (33, 9216, 1152)])
-def test_gemm_add_layernorm_fused_bit_exact(L, M, N, K):
-    """t = 1: the row-parallel projection's split-K partials summed inside the add + LN
-    kernel (liger_op_gemm_tiled_add_layernorm) equal the GEMM -> fixup -> add + LN
-    sequence bit for bit, and the oracle (P = x W^T, x1 = x_res + P + b, LN) within
-    the BASELINE.json tolerance.  Shapes: OPT-13B out-proj / FC2 at b = 2 / 8, a
-    small ragged case, OPT-66B TP = 8 out-proj shape at M = 33."""
-    if L.gemm_plan(M, N, K)["splits"] < 2:
-        pytest.skip("no split-K plan at this shape")
-    x = c0_values(6, 1, np.arange(M * K, dtype=np.uint64), -1).reshape(M, K)
-    w = c0_values(6, 2, np.arange(N * K, dtype=np.uint64), -6).reshape(N, K)
-    xr = c0_values(6, 3, np.arange(M * N, dtype=np.uint64), -2).reshape(M, N)
-    b = c0_values(6, 4, np.arange(N, dtype=np.uint64), -5)
-    g = 1 + c0_values(6, 5, np.arange(N, dtype=np.uint64), -4)
-    be = c0_values(6, 6, np.arange(N, dtype=np.uint64), -4)
-    wt = torch.empty(L.tiled_numel(N, K), dtype=torch.bfloat16, device="cuda")
-    L.tile_weight(bf16_dev(w), wt)
-    xd, bd, gd, bed = bf16_dev(x), bf16_dev(b), bf16_dev(g), bf16_dev(be)
-    ws = workspace(L.gemm_workspace_bytes(M, N, K))
-    # unfused: GEMM (with its fixup) into P, then add + LN
-    p = torch.empty(M, N, dtype=torch.bfloat16, device="cuda")
-    L.gemm_tiled(xd, wt, p, N=N, workspace=ws)
-    x1 = bf16_dev(xr)
-    y1 = torch.empty_like(x1)
-    L.add_layernorm(x1, gd, bed, y1, add=p, add_bias=bd, x_out=x1)
-    # fused
-    x2 = bf16_dev(xr)
-    y2 = torch.empty_like(x2)
-    L.gemm_tiled_add_layernorm(xd, wt, x2, y2, gd, bed, N=N, add_bias=bd, workspace=ws)
-    torch.cuda.synchronize()
-    assert torch.equal(x1.view(torch.int16), x2.view(torch.int16))
-    assert torch.equal(y1.view(torch.int16), y2.view(torch.int16))
-    ref_x = xr.astype(np.float64) + x.astype(np.float64) @ w.astype(np.float64).T + b
-    assert errs(to_np64(x2), ref_x)[0] <= REL
-    ref_y = om.layer_norm(to_np64(x2), g.astype(np.float64), be, 1e-5)
-    rel, mae = errs(to_np64(y2), ref_y)
-    assert rel <= REL and mae <= 1e-2
-
-
-_FUSE_CHILD = r"""
-import sys, numpy as np
-sys.path.insert(0, {root!r})
-from liger_inputs import make_trace
-from liger_inputs.configs import ModelConfig
-from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
-cfg = ModelConfig("mid3", 3, 1024, 8, 4096, 1024, 96, "relu")
-trace = make_trace(3, float("inf"), seed=4, batch_sizes=(2, 5), prompt_range=(20, 60), n_decode=6, vocab=cfg.vocab)
-eng = LigerEngine(cfg, mode="interleaved", max_batch=8, max_seq=64, max_new=8, seed=7)
-ids = [eng.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], 0.0) for t in trace]
-eng.drain()
-print(repr([eng.poll(i, want_tokens=True)[1].tolist() for i in ids]))
-eng.close()
-"""
-
-
-def test_engine_split_ln_fusion_bit_exact_and_oracle(L):
-    """Engine at t = 1 on a config whose decode projections split K (h = 1024,
-    ffn 4096, d = 128): LIGER_FUSE_SPLITK_LN=1 (out-proj / FC2 partials summed inside
-    the next add + LN) and the default fixup-kernel path give identical tokens,
-    equal to the fp64 oracle's greedy tokens where its top-2 margin is clear."""
-    import ast
-    import os
-    import subprocess
-    import sys
-    from liger_inputs.configs import ModelConfig
-    from liger_inputs import make_trace
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    assert L.gemm_plan(2, 1024, 4096)["splits"] > 1 and L.gemm_plan(5, 1024, 1024)["splits"] > 1
-    res = {}
-    for flag in ("1", "0"):
-        p = subprocess.run([sys.executable, "-c", _FUSE_CHILD.format(root=root)],
-                           env={**os.environ, "LIGER_FUSE_SPLITK_LN": flag}, capture_output=True, text=True,
-                           timeout=600)
-        assert p.returncode == 0, p.stderr[-2000:]
-        res[flag] = ast.literal_eval(p.stdout.strip().splitlines()[-1])
-    assert res["1"] == res["0"]
-    cfg = ModelConfig("mid3", 3, 1024, 8, 4096, 1024, 96, "relu")
-    trace = make_trace(3, float("inf"), seed=4, batch_sizes=(2, 5), prompt_range=(20, 60), n_decode=6,
-                       vocab=cfg.vocab)
-    t = trace[0]
-    pr = t["tokens"].reshape(t["batch"], t["seq_len"])
-    ref, logits = om.greedy_generate(cfg, 7, pr, t["n_decode"], return_logits=True)
-    ok = om.top2_margin(logits) > 0.02 * np.sqrt((logits ** 2).mean())
-    got = np.array(res["1"][0])
-    for i in range(t["batch"]):
-        n = int(np.argmin(ok[i])) if not ok[i].all() else t["n_decode"]
-        assert np.array_equal(got[i, :n], ref[i, :n])
-
-
-def test_gemm_early_fixup_bit_exact(L):
-    """Opt-in LIGER_EARLY_FIXUP=1: the split-K fixup reduces each tile as soon as its
-    chunks are counted in (per-tile readiness counters) instead of after the whole
-    GEMM grid -- same chunk order, so the same bits as the default fixup."""
-    import ast
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    shapes = [(8, 5120, 5120), (8, 5120, 20480), (8, 20480, 5120), (3, 1000, 2560), (33, 640, 4096)]
-    code = _CLUSTER_CHILD.format(root=root, shapes=shapes)
-    res = {}
-    for flag in ("1", "0"):
-        p = subprocess.run([sys.executable, "-c", code], env={**os.environ, "LIGER_EARLY_FIXUP": flag},
-                           capture_output=True, text=True, timeout=300)
-        assert p.returncode == 0, p.stderr[-2000:]
-        res[flag] = ast.literal_eval(p.stdout.strip().splitlines()[-1])
-    assert any(pl["splits"] > 1 for pl, _ in res["1"])
-    for (p1, h1), (p0, h0), s in zip(res["1"], res["0"], shapes):
-        assert p1 == p0 and h1 == h0, s
