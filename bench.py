@@ -1,29 +1,38 @@
 """Benchmark of the Liger hot path (driver contract).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--loopback]
 
 Workload (BASELINE.json configs[1]): OPT-13B random-init bf16, Poisson-shaped
 request batches (batch 2/4/8, prompt U[128, 512], 32 generated tokens), served
 through the C ABI (liger_submit / liger_step / liger_poll).  One "step" = one
 request batch through the whole hot path (prefill pass + 31 decode passes over
-all 40 layers).  N GPUs = tensor parallel degree N (one process per GPU).
+all 40 layers).  N GPUs = tensor-parallel degree N (one process per GPU).  Without
+torchrun, `--gpus N > 1` re-launches itself under torch.distributed.run with N
+processes; `--loopback` instead runs the N ranks as threads sharing ONE GPU (the
+loopback communicator: a functional dry run of the t > 1 path, not a speed claim).
 
-value    = requests (sequences) per second of the whole job with the prompts
-           already resident in HBM, all K batches offered at once (capacity;
-           device time between two synchronised barriers, max over ranks).
-e2e      = the same with host prompts copied in and generated tokens copied
-           out through the public API inside the timed region.
-latency  = mean / p99 request latency (pending + execution) of a
-           Poisson trace at a fixed rate of 0.5 x the measured capacity.
-roofline = the dominant kernel class (by device time) in a timed replay with
-           per-launch CUDA events inside the library.
+value     = requests (sequences) per second of the whole job with the prompts
+            already resident in HBM, all K batches offered at once (capacity;
+            device time between two synchronised barriers, max over ranks).
+e2e       = the same with host prompts copied in and generated tokens copied
+            out through the public API inside the timed region.
+operating_points = the BASELINE metric itself: Poisson
+            traces at rising arrival rates for serial intra-op TP and for the
+            interleaved mode on the same traces; L* = 1.5 x serial's mean latency at
+            the lowest rate; each mode's req/s at mean latency <= L* (interpolated)
+            and mean / p99 latency at 0.5 and 0.8 x serial's saturation rate.
+roofline  = the dominant kernel class (by device time) in a timed replay with
+            per-launch CUDA events inside the library; at N > 1 also the
+            all-reduce class (bus bandwidth) and an NCCL-tests-style sweep.
 """
 import argparse
 import json
 import math
 import os
+import socket
 import subprocess
 import sys
+import threading
 import time
 
 import numpy as np
@@ -31,7 +40,7 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 # stdout carries exactly one JSON line: NCCL prints a version banner at NCCL_DEBUG=WARN/VERSION
-os.environ["NCCL_DEBUG"] = "NONE"
+os.environ.setdefault("NCCL_DEBUG", "NONE")
 _JSON_FD = None
 
 
@@ -46,10 +55,12 @@ def _redirect_stdout():
     _JSON_FD = os.dup(1)
     os.dup2(2, 1)
 
+
 from liger_inputs import get_config, make_trace  # noqa: E402
 
 METRIC = "req/s at fixed mean latency; mean/p99 latency at fixed req/s (OPT, TP=1/2/4/8)"
 PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
+NVLINK_SPEC_GBS = 900.0   # NVLink 5 per direction per GPU (B200 spec)
 
 
 def load_peaks():
@@ -108,15 +119,115 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+# ----------------------------------------------------------------------------- rank groups
+class DistGroup:
+    """torch.distributed ranks (one process per GPU): gloo for host values."""
+
+    def __init__(self, world, rank):
+        import torch.distributed as dist
+        self.dist, self.world, self.rank = dist, world, rank
+        self.gloo = dist.new_group(backend="gloo") if world > 1 else None
+
+    def barrier(self):
+        import torch
+        if self.world > 1:
+            self.dist.barrier(group=self.gloo)
+        torch.cuda.synchronize()
+
+    def max(self, x):
+        if self.world == 1:
+            return x
+        import torch
+        t = torch.tensor([x], dtype=torch.float64)
+        self.dist.all_reduce(t, op=self.dist.ReduceOp.MAX, group=self.gloo)
+        return float(t.item())
+
+    def bcast(self, obj):
+        if self.world == 1:
+            return obj
+        o = [obj]
+        self.dist.broadcast_object_list(o, src=0, group=self.gloo)
+        return o[0]
+
+
+class ThreadShared:
+    def __init__(self, world):
+        self.world = world
+        self.bar = threading.Barrier(world)
+        self.slots = [None] * world
+
+
+class ThreadGroup:
+    """Loopback ranks: threads of this process sharing one GPU."""
+
+    def __init__(self, shared, rank):
+        self.s, self.world, self.rank = shared, shared.world, rank
+
+    def barrier(self):
+        import torch
+        torch.cuda.synchronize()
+        self.s.bar.wait()
+
+    def _gather(self, x):
+        self.s.bar.wait()
+        self.s.slots[self.rank] = x
+        self.s.bar.wait()
+        out = list(self.s.slots)
+        self.s.bar.wait()
+        return out
+
+    def max(self, x):
+        return max(self._gather(x))
+
+    def bcast(self, obj):
+        return self._gather(obj)[0]
+
+
 # ----------------------------------------------------------------------------- CPU oracle baseline
-def cpu_oracle_sample(cfg, b=2, s=256, n_new=32, budget_s=20.0):
-    """Time the fp64 oracle on a bounded sample of the workload: one decoder
-    layer's prefill over a [b, s] batch and one decode step at ctx s+16, then
-    extrapolate to L layers and n_new passes (labelled as such)."""
+def cpu_oracle_sample(cfg, b=2, s=128, n_new=32, threads=None):
+    """Time the CPU oracle on a bounded sample of the workload and extrapolate (labelled).
+
+    Preferred: the fp32 C++ OpenMP oracle binary (oracle/layer_ref.cpp; BASELINE.md
+    "CPU baseline plan") on one decoder layer -- a prefill over [b, s] and decode
+    steps at ctx s + 16 -- with weights generated on the fly, x L layers x n_new passes.
+    Fallback (binary not built): the fp64 numpy oracle on the same sample."""
+    nproc = os.cpu_count() or 1
+    exe = None
+    try:   # -march=native: compile for THIS host (the binary may not have been built here)
+        import tempfile
+        from paper_conf_ppopp_duwjchcl24_b200.build import build_oracle
+        exe, _ = build_oracle(os.path.join(tempfile.gettempdir(), f"liger_oracle_{os.getpid()}"))
+    except Exception as e:
+        print(f"bench.py: C++ oracle unavailable ({e}); timing the numpy oracle", file=sys.stderr)
+    if exe and os.path.exists(exe):
+        out = {}
+        for th in ([threads] if threads else [nproc, 1]):
+            cmd = [exe, "--hidden", str(cfg.hidden), "--heads", str(cfg.n_heads), "--ffn", str(cfg.ffn),
+                   "--act", cfg.act, "--batch", str(b), "--prompt", str(s), "--decode-steps", "4",
+                   "--ctx", str(s + 16), "--budget-s", "12"]
+            env = {**os.environ, "OMP_NUM_THREADS": str(th)}
+            r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env)
+            if r.returncode != 0:
+                out = None
+                break
+            out[th] = json.loads(r.stdout.strip().splitlines()[-1])
+        if out:
+            main = out[max(out)]
+            per_batch = cfg.n_layers * (main["prefill_s"] + (n_new - 1) * main["decode_step_s"])
+            res = {"value": b / per_batch, "unit": "req/s", "cores": main["threads"], "kind": "oracle",
+                   "sample": (f"fp32 C++ OpenMP oracle (oracle/layer_ref.cpp, -O3 -march=native), one {cfg.name} "
+                              f"layer: prefill b={b} s={s} ({main['prefill_s']:.2f} s) + decode steps at ctx "
+                              f"{s + 16} ({main['decode_step_s'] * 1e3:.1f} ms each); extrapolated x{cfg.n_layers} "
+                              f"layers x {n_new} passes"),
+                   "per_batch_s": per_batch}
+            if 1 in out and max(out) != 1:
+                one = out[1]
+                pb1 = cfg.n_layers * (one["prefill_s"] + (n_new - 1) * one["decode_step_s"])
+                res["one_thread"] = {"value": b / pb1, "unit": "req/s", "cores": 1}
+            return res
     from oracle import model as om
     rng = np.random.default_rng(0)
     h, f = cfg.hidden, cfg.ffn
-    # weights are inputs: a cheap normal generator (the oracle's arithmetic is what is timed)
     w = {"w_qkv": rng.standard_normal((h, 3 * h)) * h ** -0.5, "b_qkv": np.zeros(3 * h),
          "w_o": rng.standard_normal((h, h)) * h ** -0.5, "b_o": np.zeros(h),
          "w_1": rng.standard_normal((h, f)) * h ** -0.5, "b_1": np.zeros(f),
@@ -129,125 +240,154 @@ def cpu_oracle_sample(cfg, b=2, s=256, n_new=32, budget_s=20.0):
     xd = rng.standard_normal((b, 1, h)) * 0.1
     reps = 0
     t0 = time.perf_counter()
-    while True:
+    while reps < 4:
         om.decoder_layer(cfg, w, xd, k, v, start_pos=s)
         reps += 1
-        if time.perf_counter() - t0 > min(5.0, budget_s / 4) or reps >= 8:
-            break
     t_dc = (time.perf_counter() - t0) / reps
     per_batch = cfg.n_layers * (t_pf + (n_new - 1) * t_dc)
-    cores = os.cpu_count()
-    return {"value": b / per_batch, "unit": "req/s", "cores": cores, "kind": "oracle",
-            "sample": (f"fp64 numpy oracle, one {cfg.name} layer: prefill b={b} s={s} ({t_pf:.2f}s) + "
-                       f"{reps} decode steps at ctx {s + 1} ({t_dc * 1e3:.1f} ms each); extrapolated x{cfg.n_layers} "
-                       f"layers x {n_new} passes"),
+    return {"value": b / per_batch, "unit": "req/s", "cores": nproc, "kind": "oracle",
+            "sample": (f"fp64 numpy oracle, one {cfg.name} layer: prefill b={b} s={s} ({t_pf:.2f}s) + {reps} decode "
+                       f"steps at ctx {s + 1} ({t_dc * 1e3:.1f} ms each); extrapolated x{cfg.n_layers} layers x "
+                       f"{n_new} passes"),
             "per_batch_s": per_batch}
 
 
 def run_reference(args):
+    """The reference arm of this tier: the CPU oracle as it stands, on the box's host
+    cores; each step is one bounded sample (one layer prefill + decode steps) whose
+    wall time is ms_per_step; value is the extrapolated whole-workload req/s."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
     cfg = get_config(args.config)
-    vals = []
+    vals, walls = [], []
     for i in range(args.warmup + args.steps):
-        r = cpu_oracle_sample(cfg, budget_s=8.0)
+        t0 = time.perf_counter()
+        r = cpu_oracle_sample(cfg, threads=os.cpu_count() or 1)
         if i >= args.warmup:
             vals.append(r["value"])
+            walls.append(time.perf_counter() - t0)
     v = float(np.mean(vals))
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "req/s", "n_gpus": args.gpus,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * 2 / v, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{args.config} TP={args.gpus}: one layer prefill+decode sample, extrapolated",
-                       "model": args.config},
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * float(np.mean(walls)),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f32" if "C++" in r["sample"] else "f64", "data": "synthetic",
+            "config": {"workload": f"{args.config} TP={args.gpus}: one-layer prefill + decode sample per step, "
+                                   f"req/s extrapolated to {cfg.n_layers} layers x 32 passes (ms_per_step = the "
+                                   f"sample's wall time)", "model": args.config},
             "cpu_baseline": {**{k: r[k] for k in ("unit", "cores", "kind", "sample")}, "value": v},
             "e2e": {"value": v, "unit": "req/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     emit(line)
     return 0
 
 
-# ----------------------------------------------------------------------------- GPU arm
-def main():
-    ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=12)
-    ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="opt-13b")
-    ap.add_argument("--layers", type=int, default=None, help="debug only: fewer layers (invalid for reporting)")
-    ap.add_argument("--mode", default="interleaved", choices=["interleaved", "serial", "pipeline", "pipeline_th"],
-                    help="Liger (interleaved), Intra-Op (serial TP) or Inter-Op (pipeline) baseline")
-    ap.add_argument("--inflight", type=int, default=2)
-    ap.add_argument("--F", type=int, default=8)
-    ap.add_argument("--cf", type=float, default=1.1, help="contention factor; <= 0: use the calibrated one")
-    ap.add_argument("--n-new", type=int, default=32)
-    ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--no-latency", action="store_true")
-    ap.add_argument("--seed", type=int, default=0)
-    ap.add_argument("--fused-ar", action="store_true",
-                    help="serial TP competitor: row-parallel GEMM + all-reduce fused over peer memory "
-                         "(LIGER_FUSED_AR=1 with the one-shot peer backend; use with --mode serial)")
-    ap.add_argument("--sync", default="hybrid", choices=["hybrid", "cpu_gpu", "inter_stream"],
-                    help="Algorithm 1 round synchronisation (§3.4 Fig. 8; ablation §4.5)")
-    ap.add_argument("--workload", default="mixed", choices=["mixed", "generative"],
-                    help="mixed: batches of 2/4/8 x prompt U[128,512] + n_new generated tokens (BASELINE.json "
-                         "configs[1]); generative: the paper's sampling-phase task (P:316, Fig. 11) -- batches of "
-                         "32 sequences at start length 16, one sampling iteration each (the 16-token conditioning "
-                         "pass that fills the KV cache is included in the step)")
-    args = ap.parse_args()
-    if args.workload == "generative":
-        args.n_new = 2
-    if args.fused_ar:
-        os.environ["LIGER_FUSED_AR"] = "1"
-        os.environ["LIGER_ONESHOT_AR"] = "1"
-    _redirect_stdout()
-    if args.impl == "reference":
-        return run_reference(args)
+# ----------------------------------------------------------------------------- serving helpers
+def serve_poisson(eng, group, trace, t_offset=0.0):
+    """Open-loop serving of a trace (arrival times on the host clock); all ranks submit
+    identically (rank 0 decides which arrivals are due).  Returns per-sequence
+    latencies (pending + execution) and the throughput over the run."""
+    group.barrier()
+    t0 = time.monotonic()
+    ids, sizes = [], []
+    i = 0
+    while True:
+        now = time.monotonic() - t0
+        due = sum(1 for r in trace[i:] if r["arrival_s"] <= now) if group.rank == 0 else 0
+        due = group.bcast(due)
+        for r in trace[i:i + due]:
+            ids.append(eng.submit(r["tokens"], r["batch"], r["seq_len"], r["n_decode"], t0 + r["arrival_s"]))
+            sizes.append(r["batch"])
+        i += due
+        rc = eng.step()
+        if i >= len(trace):
+            break
+        if rc == 2:   # idle: wait for the next arrival
+            time.sleep(max(0.0, min(0.001, trace[i]["arrival_s"] - (time.monotonic() - t0))))
+    eng.drain()
+    lats, fin = [], []
+    for bid, bsz in zip(ids, sizes):
+        res, _ = eng.poll(bid)
+        lats += [res.finish_s - res.arrival_s] * bsz
+        fin.append(res.finish_s)
+    lats.sort()
+    span = max(fin) - t0
+    return {"mean_s": float(np.mean(lats)), "p99_s": float(lats[max(0, math.ceil(0.99 * len(lats)) - 1)]),
+            "req_s": sum(sizes) / span}
 
+
+def req_s_at_latency(points, L):
+    """Largest throughput with mean latency <= L, interpolating linearly between the
+    swept points in (throughput, mean latency); points sorted by rate."""
+    best = None
+    for a, b in zip(points, points[1:]):
+        if a["mean_s"] <= L:
+            best = a["req_s"]
+        if a["mean_s"] <= L < b["mean_s"]:
+            w = (L - a["mean_s"]) / (b["mean_s"] - a["mean_s"])
+            best = a["req_s"] + w * (b["req_s"] - a["req_s"])
+            break
+    else:
+        if points and points[-1]["mean_s"] <= L:
+            best = points[-1]["req_s"]
+    return best
+
+
+def allreduce_sweep(eng, group, torch, F=8):
+    """NCCL-tests-style bus bandwidth of the library's all-reduce (liger_op_allreduce)
+    on the communication stream, 8 B .. 1 GiB, whole vs decomposed into F atomic
+    units (P:254, P:270): busbw = S / t * 2 (t - 1) / t."""
+    t = group.world
+    st = torch.cuda.Stream()
+    out = []
+    buf = torch.zeros(1 << 29, dtype=torch.bfloat16, device="cuda")
+    for lg in range(3, 31, 3):
+        n = max(8, (1 << lg) // 2)
+        x = buf[:n]
+        row = {"bytes": 2 * n}
+        for name, ks in (("whole", [F]), ("chunked", [1] * F)):
+            reps = 20 if n < (1 << 24) else 5
+            for rep in range(reps + 3):
+                if rep == 3:
+                    group.barrier()
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(st)
+                u = 0
+                for k in ks:
+                    eng.allreduce(x, u, u + k, F, stream=st.cuda_stream)
+                    u += k
+            e1.record(st)
+            e1.synchronize()
+            us = group.max(e0.elapsed_time(e1) * 1e3 / reps)
+            row[name + "_us"] = round(us, 2)
+            row[name + "_busbw_gbs"] = round(2 * n / (us * 1e-6) * 2 * (t - 1) / t / 1e9, 2)
+        out.append(row)
+    del buf
+    return out
+
+
+# ----------------------------------------------------------------------------- one rank
+def rank_main(args, group, local, uid, result):
     import torch
-    import torch.distributed as dist
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        gloo = dist.new_group(backend="gloo")
     from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
+    torch.cuda.set_device(local)
+    world, rank = group.world, group.rank
     cfg = get_config(args.config, args.layers)
-    uid = None
-    if world > 1:
-        obj = [LigerEngine.unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0, group=gloo)
-        uid = obj[0]
     gen = args.workload == "generative"
     trace_kw = (dict(batch_sizes=(32,), prompt_range=(16, 16)) if gen else {})
-    eng = LigerEngine(cfg, world=world, rank=rank, nccl_uid=uid, mode=args.mode, max_batch=32 if gen else 8,
-                      max_seq=16 if gen else 512, max_new=args.n_new, max_inflight=args.inflight, decomp_factor=args.F,
-                      contention_factor=args.cf, seed=args.seed, sync=args.sync)
+    ekw = dict(world=world, rank=rank, nccl_uid=uid, max_batch=32 if gen else 8, max_seq=16 if gen else 512,
+               max_new=args.n_new, max_inflight=args.inflight, decomp_factor=args.F, contention_factor=args.cf,
+               seed=args.seed, sync=args.sync)
+    eng = LigerEngine(cfg, mode=args.mode, **ekw)
     eng.profile([8, 64, 256, 512, 1024, 2048, 4096])
     # contention factor (P:246-248): measured GEMM || all-reduce slowdown (1-rank proxy at N=1)
     cf_cal, _ = eng.calibrate_cf([8, 256, 1024], set_cf=args.cf <= 0)
-    # contention control: the same calibration with the GEMM grid
-    # leaving SMs to the communication kernel
     cf_reserve = {}
-    for rsv in (8, 16, 32):
-        eng.set_gemm_sm_reserve(rsv)
-        cf_reserve[rsv] = round(eng.calibrate_cf([8, 256, 1024], set_cf=False)[0], 4)
-    eng.set_gemm_sm_reserve(int(os.environ.get("LIGER_GEMM_SM_RESERVE", "0")))
+    if not args.quick:   # contention control (SURVEY §8(f) 3): GEMM grids leaving SMs to the all-reduce
+        for rsv in (8, 16, 32):
+            eng.set_gemm_sm_reserve(rsv)
+            cf_reserve[rsv] = round(eng.calibrate_cf([8, 256, 1024], set_cf=False)[0], 4)
+        eng.set_gemm_sm_reserve(int(os.environ.get("LIGER_GEMM_SM_RESERVE", "0")))
     cf_reserve[0] = round(cf_cal, 4)
-
-    def barrier():
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
-
-    def max_over_ranks(x):
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
 
     trace = make_trace(args.warmup + args.steps, float("inf"), seed=args.seed, vocab=cfg.vocab,
                        n_decode=args.n_new, **trace_kw)
@@ -262,7 +402,7 @@ def main():
 
     def timed_run(host_io):
         eng.reset_stats()
-        barrier()
+        group.barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         t_host0 = time.perf_counter()
@@ -274,26 +414,25 @@ def main():
                 ids.append(eng.submit(r["tokens"], r["batch"], r["seq_len"], r["n_decode"], 0.0))
             else:
                 ids.append(eng.submit(None, r["batch"], r["seq_len"], r["n_decode"], 0.0, device_tokens=dt))
-        toks = []
         eng.drain()
         if host_io:
             for bid in ids:
-                toks.append(eng.poll(bid, want_tokens=True)[1])
+                eng.poll(bid, want_tokens=True)
         torch.cuda.nvtx.range_pop()
         torch.cuda.synchronize()
         e1.record()
         e1.synchronize()
         wall = time.perf_counter() - t_host0
-        dev_s = max_over_ranks(e0.elapsed_time(e1) * 1e-3)
-        return dev_s, wall, eng.stats(), toks
+        group.barrier()
+        dev_s = group.max(e0.elapsed_time(e1) * 1e-3)
+        return dev_s, wall, eng.stats()
 
     clocks = ClockSampler(local)
     clocks.start()
-    dev_s, wall_s, st, _ = timed_run(False)
+    dev_s, wall_s, st = timed_run(False)
     clk = clocks.stop()
     value = seqs / dev_s
-
-    e2e_s, _, _, toks = timed_run(True)
+    e2e_s, _, _ = timed_run(True)
     h2d = sum(r["batch"] * r["seq_len"] * 4 for r in timed) / len(timed)
     d2h = sum(r["batch"] * r["n_decode"] * 4 for r in timed) / len(timed)
 
@@ -311,17 +450,20 @@ def main():
     for k, v in kt.items():
         if v["count"] == 0 or v["ms"] <= 0:
             continue
-        if k in ("gemm_prefill",):
+        if k == "gemm_prefill":
             ach = v["flops"] / (v["ms"] * 1e-3) / 1e12
             classes[k] = dict(bound="tensor", achieved=ach, peak=tc_sus, unit="TFLOP/s", frac=ach / tc_sus)
         elif k == "allreduce":
-            continue
+            # bytes = message bytes; bus bandwidth S/t * 2(t-1)/t against NVLink 5 (spec)
+            ach = v["bytes"] / (v["ms"] * 1e-3) / 1e9 * 2 * (world - 1) / world
+            classes[k] = dict(bound="nvlink", achieved=ach, peak=NVLINK_SPEC_GBS, unit="GB/s (busbw)",
+                              frac=ach / NVLINK_SPEC_GBS)
         else:
             ach = v["bytes"] / (v["ms"] * 1e-3) / 1e9
             classes[k] = dict(bound="hbm", achieved=ach, peak=hbm, unit="GB/s", frac=ach / hbm)
         classes[k].update(share=shares[k], launches=v["count"], avg_us=1e3 * v["ms"] / v["count"],
                           per_launch_bytes=v["bytes"] / v["count"], per_launch_flops=v["flops"] / v["count"])
-    dom = max(classes, key=lambda k: shares[k]) if classes else None
+    dom = max((k for k in classes if k != "allreduce"), key=lambda k: shares[k], default=None)
     roof = None
     traffic = {}
     try:   # dram bytes per launch of each kernel class from the committed `ncu --set full` capture
@@ -350,14 +492,14 @@ def main():
         def batch_ms(n_new):
             best = 1e30
             for _ in range(2):
-                barrier()
+                group.barrier()
                 a, z = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 a.record()
                 eng.submit(None, bsz, slen, n_new, 0.0, device_tokens=ids_d)
                 eng.drain()
                 z.record()
                 z.synchronize()
-                best = min(best, max_over_ranks(a.elapsed_time(z)))
+                best = min(best, group.max(a.elapsed_time(z)))
             return best
         t1, tn = batch_ms(1), batch_ms(args.n_new)
         pass_us = (tn - t1) / (args.n_new - 1) * 1e3
@@ -372,39 +514,48 @@ def main():
                        "note": "whole decode pass (all kernels, PDL chain intact), CUDA events around "
                                "batches with n_new and 1 generated tokens; bytes = weights + KV read"}
 
-    # ---- latency at a fixed request rate (Poisson, 0.5 x capacity)
-    lat = None
+    # ---- NVLink all-reduce sweep (N > 1)
+    ar_sweep = allreduce_sweep(eng, group, torch, F=args.F) if world > 1 and not args.quick else None
+    scheduler = eng.scheduler_name()
+    eng.close()
+
+    # ---- the BASELINE metric: operating points of serial TP vs the interleaved mode
+    ops = None
     if not args.no_latency:
+        modes = ["serial", "interleaved"] + (["pipeline"] if world > 1 and not args.quick else [])
+        n_b = max(8, min(args.steps, 16))
         cap_batches = len(timed) / dev_s
-        rate = 0.5 * cap_batches
-        tr = make_trace(len(timed), rate, seed=args.seed + 1, vocab=cfg.vocab, n_decode=args.n_new, **trace_kw)
-        barrier()
-        t0 = time.monotonic()
-        ids, arr = [], []
-        i = 0
-        while i < len(tr) or eng_pending(eng, ids):
-            now = time.monotonic() - t0
-            # all ranks must submit identically: rank 0 decides how many arrivals are due
-            due = sum(1 for r in tr[i:] if r["arrival_s"] <= now)
-            if world > 1 and i < len(tr):   # i advances identically on every rank; afterwards no collective
-                obj = [due]
-                dist.broadcast_object_list(obj, src=0, group=gloo)
-                due = obj[0]
-            for r in tr[i:i + due]:
-                ids.append(eng.submit(r["tokens"], r["batch"], r["seq_len"], r["n_decode"], t0 + r["arrival_s"]))
-                arr.append(r["batch"])
-            i += due
-            rc = eng.step()
-            if rc == 2 and i < len(tr):       # idle: wait for the next arrival
-                time.sleep(max(0.0, min(0.001, tr[i]["arrival_s"] - (time.monotonic() - t0))))
-        eng.drain()
-        lats, wts = [], []
-        for bid, bsz in zip(ids, arr):
-            res, _ = eng.poll(bid)
-            lats += [res.finish_s - res.arrival_s] * bsz
-        lats.sort()
-        lat = {"rate_req_s": rate * float(np.mean([r["batch"] for r in tr])),
-               "mean_s": float(np.mean(lats)), "p99_s": float(lats[max(0, math.ceil(0.99 * len(lats)) - 1)])}
+        fracs = (0.3, 0.5, 0.8) if args.quick else (0.2, 0.35, 0.5, 0.65, 0.8, 0.95)
+        sweep = {}
+        for mode in modes:
+            e = LigerEngine(cfg, mode=mode, **ekw)
+            e.profile([8, 64, 256, 512, 1024, 2048, 4096])
+            for r in warm[:2]:
+                e.submit(r["tokens"], r["batch"], r["seq_len"], r["n_decode"], 0.0)
+            e.drain()
+            pts = []
+            for fr in fracs:
+                tr = make_trace(n_b, fr * cap_batches, seed=args.seed + 1, vocab=cfg.vocab, n_decode=args.n_new,
+                                **trace_kw)
+                p = serve_poisson(e, group, tr)
+                p["rate_req_s"] = fr * cap_batches * float(np.mean([r["batch"] for r in tr]))
+                p["rate_frac_of_capacity"] = fr
+                pts.append(p)
+            sweep[mode] = {"scheduler": e.scheduler_name(), "points": pts}
+            e.close()
+        ser = sweep["serial"]["points"]
+        L_star = 1.5 * ser[0]["mean_s"]
+        # serial saturation: the highest swept rate it still keeps up with (completed >= 0.95 lambda)
+        sat = max((p["rate_req_s"] for p in ser if p["req_s"] >= 0.95 * p["rate_req_s"]),
+                  default=ser[0]["rate_req_s"])
+        ops = {"L_star_s": round(L_star, 4), "serial_saturation_req_s": round(sat, 3),
+               "req_s_at_L_star": {m: (round(v, 3) if v else None) for m, v in
+                                   ((m, req_s_at_latency(sweep[m]["points"], L_star)) for m in sweep)},
+               "sweep": {m: {"scheduler": sweep[m]["scheduler"],
+                             "points": [{k: round(v, 4) for k, v in p.items()} for p in sweep[m]["points"]]}
+                         for m in sweep},
+               "trace": f"Poisson, {n_b} batches per point, seed {args.seed + 1}, rates = fractions of the "
+                        f"measured capacity ({', '.join(str(f) for f in fracs)})"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -412,7 +563,10 @@ def main():
         cpu.pop("per_batch_s", None)
 
     if rank == 0:
-        line = {
+        t1_note = ("t = 1: no all-reduce to interleave (P:149); the interleaved mode runs the in-flight "
+                   "batches' kernel lists concurrently on its two streams (reading R31); Algorithm 1, the "
+                   "decomposition factor and the contention factor are inactive")
+        result["line"] = {
             "metric": METRIC, "value": round(value, 3), "unit": "req/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(1e3 * dev_s / len(timed), 3), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
@@ -421,17 +575,22 @@ def main():
                                      f"iteration (+ the conditioning pass)" if gen else
                                      f"batches of 2/4/8 x prompt U[128,512], {args.n_new} generated tokens") +
                                     f", all {len(timed)} batches offered at once (capacity)"),
-                       "model": cfg.name, "tp": world,
-                       "mode": args.mode, "sync": args.sync, "fused_ar": args.fused_ar, "max_inflight": args.inflight, "decomp_factor": args.F,
-                       "contention_factor": args.cf if args.cf > 0 else cf_cal,
+                       "model": cfg.name, "tp": world, "mode": args.mode, "scheduler": scheduler,
+                       "loopback": bool(args.loopback), "sync": args.sync, "fused_ar": args.fused_ar,
+                       "max_inflight": args.inflight,
+                       "decomp_factor": args.F if world > 1 else None,
+                       "contention_factor": (args.cf if args.cf > 0 else cf_cal) if world > 1 else None,
+                       "note": t1_note if world == 1 else None,
                        "contention_factor_calibrated": round(cf_cal, 4),
                        "contention_factor_vs_gemm_sm_reserve": {str(k): v for k, v in sorted(cf_reserve.items())},
                        "sequences": seqs, "batches": len(timed),
                        "l2": "inputs larger than L2 (weights 26 GB per TP=1 rank)"},
-            "latency": lat,
+            "operating_points": ops,
             "e2e": {"value": round(seqs / e2e_s, 3), "unit": "req/s", "h2d_bytes_per_step": int(h2d),
                     "d2h_bytes_per_step": int(d2h)},
             "roofline": roof,
+            "allreduce": classes.get("allreduce"),
+            "allreduce_sweep": ar_sweep,
             "decode_pass_in_situ": decode_pass,
             "kernel_classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv) for kk, vv in v.items()}
                                for k, v in classes.items()},
@@ -441,18 +600,107 @@ def main():
             "host": {"wall_s": round(wall_s, 3), "host_us": round(st["host_us"], 1),
                      "rounds": st["rounds"], "kernels": st["kernels"]},
         }
-        emit(line)
-    eng.close()
-    if world > 1:
-        dist.destroy_process_group()
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=12)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="opt-13b")
+    ap.add_argument("--layers", type=int, default=None, help="debug only: fewer layers (invalid for reporting)")
+    ap.add_argument("--mode", default="interleaved", choices=["interleaved", "serial", "pipeline", "pipeline_th"],
+                    help="Liger (interleaved), Intra-Op (serial TP) or Inter-Op (pipeline) baseline")
+    ap.add_argument("--inflight", type=int, default=2)
+    ap.add_argument("--F", type=int, default=8)
+    ap.add_argument("--cf", type=float, default=1.1, help="contention factor; <= 0: use the calibrated one")
+    ap.add_argument("--n-new", type=int, default=32)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-latency", action="store_true")
+    ap.add_argument("--quick", action="store_true", help="fewer operating points, no SM-reserve / AR sweeps")
+    ap.add_argument("--loopback", action="store_true",
+                    help="run the --gpus N ranks as threads sharing one GPU (loopback communicator dry run)")
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--fused-ar", action="store_true",
+                    help="serial TP competitor: row-parallel GEMM + all-reduce fused over peer memory "
+                         "(LIGER_FUSED_AR=1 with the one-shot peer backend; use with --mode serial)")
+    ap.add_argument("--sync", default="hybrid", choices=["hybrid", "cpu_gpu", "inter_stream"],
+                    help="Algorithm 1 round synchronisation (§3.4 Fig. 8; ablation §4.5)")
+    ap.add_argument("--workload", default="mixed", choices=["mixed", "generative"],
+                    help="mixed: batches of 2/4/8 x prompt U[128,512] + n_new generated tokens (BASELINE.json "
+                         "configs[1]); generative: the paper's sampling-phase task (P:316, Fig. 11) -- batches of "
+                         "32 sequences at start length 16, one sampling iteration each (the 16-token conditioning "
+                         "pass that fills the KV cache is included in the step)")
+    args = ap.parse_args()
+    if args.workload == "generative":
+        args.n_new = 2
+    if args.fused_ar:
+        os.environ["LIGER_FUSED_AR"] = "1"
+        os.environ["LIGER_ONESHOT_AR"] = "1"
+    # N > 1 without torchrun: re-launch under torch.distributed.run, one process per GPU
+    if (args.impl == "ours" and args.gpus > 1 and not args.loopback and "WORLD_SIZE" not in os.environ):
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+        return subprocess.call(cmd)
+    _redirect_stdout()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    result = {}
+    if args.loopback:
+        from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
+        world = args.gpus
+        shared = ThreadShared(world)
+        uid = LigerEngine.loopback_id() if world > 1 else None
+        errs = []
+
+        def th(r):
+            try:
+                rank_main(args, ThreadGroup(shared, r), 0, uid, result)
+            except Exception as e:
+                import traceback
+                errs.append(f"rank {r}: {e!r}\n{traceback.format_exc()}")
+                shared.bar.abort()
+        ths = [threading.Thread(target=th, args=(r,)) for r in range(world)]
+        for t in ths:
+            t.start()
+        for t in ths:
+            t.join()
+        if errs:
+            print("\n".join(errs), file=sys.stderr)
+            return 1
+    else:
+        import torch.distributed as dist
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        rank = int(os.environ.get("RANK", "0"))
+        local = int(os.environ.get("LOCAL_RANK", "0"))
+        if world != args.gpus:
+            print(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}", file=sys.stderr)
+            return 2
+        torch.cuda.set_device(local)
+        if world > 1:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        group = DistGroup(world, rank)
+        uid = None
+        if world > 1:
+            from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
+            uid = group.bcast(LigerEngine.unique_id() if rank == 0 else None)
+        rank_main(args, group, local, uid, result)
+        if world > 1:
+            dist.destroy_process_group()
+    if "line" in result:
+        emit(result["line"])
     return 0
-
-
-def eng_pending(eng, ids):
-    for bid in ids:
-        if eng.poll(bid) is None:
-            return True
-    return False
 
 
 if __name__ == "__main__":

@@ -177,9 +177,43 @@ int liger_drain(liger_ctx* ctx);
  * (copied device -> host on the first successful poll that passes it). */
 int liger_poll(liger_ctx* ctx, int64_t id, liger_result* out, int32_t* tokens_out);
 
-/* Device pointer to a finished batch's generated tokens [batch * n_new] int32
- * (valid until the batch's slot is reused by a later submit). */
+/* Device pointer to a finished batch's generated tokens [batch * n_new] int32.
+ * LIGER_PENDING until the batch has finished; LIGER_ESTATE once its slot has been
+ * reused by a later batch (the pointer is valid only until then). */
 int liger_result_tokens_device(liger_ctx* ctx, int64_t id, const int32_t** dev_tokens);
+
+/* The per-layer all-reduce (§8(a) a6 / a10) as a standalone call on the
+ * context's communicator, decomposed as the engine decomposes it (§3.6; a13):
+ * in-place bf16 sum over the tensor-parallel ranks of units [u0, u1) of F, unit u
+ * being the contiguous element range [count*u/F, count*(u+1)/F) of device buffer
+ * `buf` (bf16 [count]).  With atomic chunks (t > 2, R9) every unit is its
+ * own collective, so any split of [0, F) into pieces gives the bits of the whole.
+ * Messages up to the one-shot cap use the peer-memory kernel when the backend has
+ * it (rank-ordered fp32 sum, RNE to bf16).  stream: cudaStream_t or NULL (the
+ * context's communication stream).  A no-op at world == 1.  [collective] */
+int liger_op_allreduce(liger_ctx* ctx, void* buf, size_t count, int u0, int u1, int F, void* stream);
+
+/* Debug readback for parity tests (not part of the serving path).
+ * liger_set_debug_capture(ctx, arena_bytes) [collective]: arena_bytes > 0 turns capture
+ * on with a device arena of that size (allocated here, before serving: nothing is
+ * allocated while peers may spin in one-shot all-reduce kernels; freed by
+ * liger_finalize), 0 turns it off.  For a batch admitted while capture is on, every
+ * LM-head pass (pass j = 0 prefill, j >= 1 decode step j, reading R22) copies, after the
+ * argmax, this rank's fp32 logits shard and the LM-head input residual into the batch's
+ * part of the arena (device-to-device copies on the pass's stream; no kernel and no
+ * change to any computed value); a batch that no longer fits is not captured.  liger_debug_read copies
+ * a finished batch's capture to host_buf:
+ *   LIGER_DBG_LOGITS  fp32 [n_new][batch][V/t]: logits of vocabulary columns
+ *                     [tp_rank*V/t, (tp_rank+1)*V/t) (C7: LN_f(x_L) . E_tok^T)
+ *   LIGER_DBG_RESID   bf16 [n_new][batch][h]: the last token's residual stream x_L
+ *                     after the last decoder layer, before the final LayerNorm (C6)
+ * Errors: LIGER_PENDING (not finished), LIGER_ESTATE (the batch ran without capture or
+ * on a pipeline stage without the LM head), LIGER_EINVAL (bytes smaller than the
+ * capture: n_new * batch * 4 V/t resp. n_new * batch * 2 h bytes). */
+#define LIGER_DBG_LOGITS 1
+#define LIGER_DBG_RESID 2
+int liger_set_debug_capture(liger_ctx* ctx, size_t arena_bytes);
+int liger_debug_read(liger_ctx* ctx, int64_t id, int what, void* host_buf, size_t bytes);
 
 int liger_stats(liger_ctx* ctx, liger_stats_t* out);
 int liger_reset_stats(liger_ctx* ctx);
@@ -244,6 +278,14 @@ int liger_profile(liger_ctx* ctx, const int32_t* m_list, int n_m);
  * set_cf != 0 installs the result as the scheduler's cf. [collective] */
 int liger_calibrate_cf(liger_ctx* ctx, const int32_t* m_list, int n_m, int set_cf, double* cf_out,
                        double* detail);
+
+/* The schedule this context actually runs (a static string): "serial" (Intra-Op),
+ * "algorithm1_hybrid" / "algorithm1_cpu_gpu" / "algorithm1_inter_stream" (Liger at
+ * t > 1, by sync mode), "t1_two_stream" (interleaved mode at t = 1, reading R31:
+ * there is no communication to interleave, the in-flight batches' kernel lists run
+ * concurrently on the two streams), "t1_algorithm1" (t = 1 with LIGER_T1_STREAMS=0),
+ * "pipeline", "pipeline_th". */
+const char* liger_scheduler_name(const liger_ctx* ctx);
 
 const char* liger_last_error(const liger_ctx* ctx);
 int liger_finalize(liger_ctx* ctx); /* [collective] */

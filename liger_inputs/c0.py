@@ -2,7 +2,7 @@
 
 BASELINE.json asks for "identical seeded random weights" on the oracle and the
 GPU path without shared code.  Both sides therefore implement this exact
-definition independently (this numpy version; `csrc/init.cu` on the device):
+definition independently (this numpy version; `c0_fill_kernel` in `csrc/norm.cu` on the device):
 
     x   = seed*0x9E3779B97F4A7C15 + tensor_id*0xD1B54A32D192ED03 + idx + 0x9E3779B97F4A7C15   (mod 2^64)
     u   = mix64(x)     (SplitMix64 finaliser)
@@ -21,7 +21,12 @@ Scales (reading R16, chosen to keep per-layer output RMS well below
                               e = round(0.5*log2(3/K)) - 2   (output projections W_o, W_2,
                                   halving the residual-branch gain, as GPT-2 scales them)
   bias                      : e = -6
-  embeddings E_tok, E_pos   : e = -3
+  embeddings E_tok, E_pos   : e = round(-0.5*log2(h)) - 1   (emb_exp(h): RMS ~ 0.3/sqrt(h),
+                                  small against the layers' output so that the decoder
+                                  layers decide the tied head's argmax -- the self term
+                                  E[tok].E[tok] grows like sqrt(h) against the others; with
+                                  a fixed 2^-3 a model with zero layers gave the same greedy
+                                  tokens; R16)
   layer-input activations   : e = -2   (layer-level parity tests only)
 """
 import math
@@ -39,7 +44,6 @@ GLOBAL_ID = {"e_tok": 0xFFFF00, "e_pos": 0xFFFF01, "lnf_g": 0xFFFF02, "lnf_b": 0
 ACT_ID_BASE = 0xFFFF10   # + layer: activations for per-layer parity tests
 
 BIAS_EXP = -6
-EMB_EXP = -3
 ACT_EXP = -2
 
 
@@ -81,6 +85,11 @@ OUT_PROJ = ("w_o", "w_2")
 def weight_exp(k_in: int, kind: str = "w_qkv") -> int:
     """Round half to even (Python round); the CUDA side uses nearbyint."""
     return int(round(0.5 * math.log2(3.0 / k_in))) - (2 if kind in OUT_PROJ else 1)
+
+
+def emb_exp(hidden: int) -> int:
+    """Scale exponent of the embeddings E_tok / E_pos (round half to even; CUDA: nearbyint)."""
+    return int(round(-0.5 * math.log2(hidden))) - 1
 
 
 def c0_values(seed: int, tensor_id: int, idx: np.ndarray, exp: int) -> np.ndarray:
@@ -136,7 +145,7 @@ def global_tensor(cfg, seed: int, kind: str, rows=None) -> np.ndarray:
         nrows = cfg.vocab if kind == "e_tok" else cfg.max_pos + 2
         r = np.arange(nrows, dtype=np.uint64) if rows is None else np.asarray(rows, dtype=np.uint64)
         idx = r[:, None] * np.uint64(h) + np.arange(h, dtype=np.uint64)[None, :]
-        return c0_values(seed, tid, idx, EMB_EXP)
+        return c0_values(seed, tid, idx, emb_exp(h))
     idx = np.arange(h, dtype=np.uint64)
     return _gamma(seed, tid, idx) if kind == "lnf_g" else _beta(seed, tid, idx)
 

@@ -229,12 +229,13 @@ def lm_head(cfg, g, x_last):
     return y @ g["e_tok"].T
 
 
-def greedy_generate(cfg, seed, prompt, n_new, layers=None, g=None, return_logits=False):
+def greedy_generate(cfg, seed, prompt, n_new, layers=None, g=None, return_logits=False, return_hidden=False):
     """Greedy generation with a KV cache (reading R22).
 
     prompt int [b, s].  Pass 0 is the prefill over the prompt and yields token 1;
     pass j (1 <= j < n_new) feeds token j at position s + j - 1 (M = b) and
-    yields token j+1.  Returns tokens [b, n_new] (and per-pass logits)."""
+    yields token j+1.  Returns tokens [b, n_new] (and per-pass logits [b, n_new, V];
+    with return_hidden also the LM-head input x_L of the last token [b, n_new, h])."""
     layers = layers or [layer_weights(cfg, seed, l) for l in range(cfg.n_layers)]
     g = g or global_weights(cfg, seed)
     b, s = prompt.shape
@@ -244,6 +245,7 @@ def greedy_generate(cfg, seed, prompt, n_new, layers=None, g=None, return_logits
         x, k, v = decoder_layer(cfg, w, x, start_pos=0)
         cache.append((k, v))
     logits = [lm_head(cfg, g, x[:, -1])]
+    hidden = [x[:, -1]]
     toks = [np.argmax(logits[-1], axis=-1)]
     for j in range(1, n_new):
         pos = s + j - 1
@@ -252,8 +254,11 @@ def greedy_generate(cfg, seed, prompt, n_new, layers=None, g=None, return_logits
             x, k, v = decoder_layer(cfg, w, x, cache[l][0], cache[l][1], start_pos=pos)
             cache[l] = (k, v)
         logits.append(lm_head(cfg, g, x[:, -1]))
+        hidden.append(x[:, -1])
         toks.append(np.argmax(logits[-1], axis=-1))
     out = np.stack(toks, axis=1)
+    if return_hidden:
+        return out, np.stack(logits, axis=1), np.stack(hidden, axis=1)
     return (out, np.stack(logits, axis=1)) if return_logits else out
 
 

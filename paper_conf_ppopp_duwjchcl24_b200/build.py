@@ -56,6 +56,30 @@ def build(verbose=False):
     return LIB
 
 
+ORACLE_SRC = os.path.join(HERE, "..", "oracle", "layer_ref.cpp")
+
+
+def build_oracle(out_dir=None, verbose=False):
+    """Compile the fp32 C++ CPU oracle (oracle/layer_ref.cpp; test / baseline
+    infrastructure, never loaded by the product): the timing binary `layer_ref` and
+    the ctypes library `liblayer_ref.so` for its pin test.  -march=native: build it on
+    the host that runs it (bench.py compiles its own copy on the GPU box's host)."""
+    out_dir = out_dir or os.path.join(HERE, "..", "oracle")
+    exe = os.path.join(out_dir, "layer_ref")
+    so = os.path.join(out_dir, "liblayer_ref.so")
+    base = ["g++", "-O3", "-march=native", "-fopenmp", "-std=c++17", ORACLE_SRC]
+    for cmd, out in ((base + ["-o", exe], exe), (base + ["-DLAYER_REF_NO_MAIN", "-shared", "-fPIC", "-o", so], so)):
+        if os.path.exists(out) and os.path.getmtime(out) >= os.path.getmtime(ORACLE_SRC):
+            continue
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError(f"g++ failed for the CPU oracle:\n{r.stderr}")
+    if verbose:
+        print(exe)
+    return exe, so
+
+
 if __name__ == "__main__":
     build(verbose=True)
+    build_oracle(verbose=True)
     sys.exit(0)

@@ -7,14 +7,15 @@
 //    (m16n8k16, fp32 accumulate), 64 queries x 64 keys per step, online
 //    softmax in registers; the CTA on the diagonal tile also writes that key
 //    tile's K/V into the cache pages.
-//  * decode: one query per sequence; split over the context in fixed chunks
-//    of 256 positions (a function of ctx only), two-pass softmax per chunk
-//    with warp-shuffle dot products, deterministic merge of the chunk partials
-//    in chunk order by the last CTA to finish.
+//  * decode: one query per sequence; persistent CTAs stream 32-position chunks of
+//    the cache through a cp.async.bulk ring, online softmax per lane group in
+//    registers, deterministic merge of the split partials (attn_decode.cuh).
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
 #include <stdlib.h>
+
+#include <algorithm>
 
 #include "attn_decode.cuh"
 #include "common.cuh"
@@ -262,107 +263,261 @@ int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* 
 }
 
 // ================================================================== decode
-// CTA = (head, sequence, chunk of DC_CHUNK positions), 128 threads.  Thread 0
-// stages the chunk's K and V page blocks (16 tokens x d bf16 = 4 KiB each,
-// contiguous in the paged pool) into shared memory with cp.async.bulk (TMA bulk
-// engine), all issued at once on one mbarrier, so a CTA pays one DRAM round
-// trip.  The new token (position pos) is taken from the qkv buffer (and
-// appended to its page by the last chunk's CTA).  Phase 1: warp w scores
-// positions [32w, 32w+32) (a token row spread over d/8 lanes, shuffle dot
-// products); two-pass softmax over the chunk; phase 2: thread (slot, vec)
-// accumulates p_t V[t] over positions t = slot (mod SLOTS).  Chunks of one
-// (sequence, head) are merged in chunk order by the last CTA (deterministic).
+// See attn_decode.cuh for the design.  Persistent CTAs of 128 threads; CTA c takes
+// items c, c + G, ... (item = (sequence, head, split), split-major within a
+// (sequence, head) so that consecutive items of a CTA are different heads) and
+// streams their 32-position chunks through a DC_NS-stage ring.
+// Enough for every launch with at most b sequences and context at most ctx (the split
+// count depends on both), so one buffer serves all passes of a slot.
 size_t attn_decode_workspace_bytes(int b, int heads, int d, int ctx) {
-  const int ns = (ctx + DC_CHUNK_MIN - 1) / DC_CHUNK_MIN;   // worst case (32-position chunks)
-  return ATTN_COUNTER_BYTES + (size_t)b * heads * ns * (d + 2) * sizeof(float);
+  size_t rows = 0;
+  for (int bb = 1; bb <= b; ++bb)
+    for (int c = DC_CH; c < ctx + DC_CH; c += DC_CH) {
+      int cps, nsp;
+      dec_attn_plan(bb, heads, std::min(c, ctx), &cps, &nsp);
+      rows = std::max(rows, (size_t)bb * heads * nsp);
+    }
+  return ATTN_COUNTER_BYTES + rows * (d + 2) * sizeof(float);
 }
 
-struct CtaSync {
-  __device__ __forceinline__ void operator()() const { __syncthreads(); }
+template <int D>
+struct DecSmem {
+  __nv_bfloat16 kv[DC_NS][2][DC_CH * D];   // stage s: K rows then V rows of the chunk
+  float st_acc[4 * (32 / (D / 8))][D];     // per lane group: acc (item merge)
+  float st_m[4 * (32 / (D / 8))], st_l[4 * (32 / (D / 8))];
+  float mw[DC_MAX_SPLITS], lw[DC_MAX_SPLITS];
+  uint64_t full[DC_NS];
+  int last;
 };
 
-// One CTA per work item (head, sequence, chunk); see attn_decode.cuh.
-template <int D, int DC_CHUNK>
+template <int D>
 __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const DecAttnArgs a) {
-  constexpr int SLOTS = DecAttnSmem<D, DC_CHUNK>::SLOTS;
+  constexpr int LPT = D / 8;          // lanes per token row (16 B each)
+  constexpr int TPW = 32 / LPT;       // token rows per warp step
+  constexpr int NG = 4 * TPW;         // lane groups per CTA
   const uint64_t tr0 = trace_now();
   extern __shared__ __align__(128) uint8_t dsm[];
-  __shared__ float sc[DC_CHUNK];
-  __shared__ float red[DC_THREADS / 32];
-  __shared__ float part[SLOTS * D];
-  __shared__ float mw[DC_MAX_SPLITS], lw[DC_MAX_SPLITS];
-  __shared__ __align__(8) uint64_t bar;
-  __shared__ int last;
-  DecAttnSmem<D, DC_CHUNK> sm;
-  sm.sK = reinterpret_cast<__nv_bfloat16*>(dsm);
-  sm.sV = sm.sK + DC_CHUNK * D;
-  sm.bar = &bar;
-  sm.sc = sc;
-  sm.red = red;
-  sm.part = part;
-  sm.mw = mw;
-  sm.lw = lw;
-  sm.last = &last;
-  const int head = blockIdx.x, bi = blockIdx.y, sp = blockIdx.z, nsp = gridDim.z;
-  if (threadIdx.x == 0) {
-    mbar_init(&bar, 1);
+  DecSmem<D>& sm = *reinterpret_cast<DecSmem<D>*>(dsm);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int grp = warp * TPW + lane / LPT;   // lane group 0..NG-1
+  const int gl = lane % LPT;                 // lane within the group: dims [8 gl, 8 gl + 8)
+  const int G = gridDim.x;
+  const int pos = a.pos, ctx = pos + 1, heads = a.heads, nsp = a.nsp, cps = a.cps;
+  const int nch = (ctx + DC_CH - 1) / DC_CH;
+  const int n_items = a.b * heads * nsp;
+  // task t of this CTA = chunk j of its i-th item; items i = blockIdx.x + k G
+  auto item_chunks = [&](int it, int* c0) {
+    const int sp = it % nsp;
+    *c0 = sp * cps;
+    return max(0, min(nch, *c0 + cps) - *c0);
+  };
+  if (tid == 0) {
+    for (int s = 0; s < DC_NS; ++s) mbar_init(&sm.full[s], 1);
     fence_barrier_init();
   }
   __syncthreads();
-  // The cached positions (< pos) were written by earlier passes, and the page
-  // table at admission: staging them does not depend on the preceding kernel
-  // (QKV), so it is issued before griddepcontrol.wait.
-  if (threadIdx.x < 32) dec_attn_issue<D, DC_CHUNK>(a, head, bi, sp, sm.sK, sm.sV, &bar, threadIdx.x);
+  // producer state (thread 0): next task to issue
+  int p_it = blockIdx.x, p_j = 0, issued = 0;
+  auto issue_next = [&]() {   // thread 0: stage the next task (if any) into ring slot issued % NS
+    while (p_it < n_items) {
+      int c0;
+      const int nc = item_chunks(p_it, &c0);
+      if (p_j < nc) break;
+      p_it += G;
+      p_j = 0;
+    }
+    const int s = issued % DC_NS;
+    if (p_it >= n_items) {   // nothing left: complete the stage's phase with no bytes
+      mbar_arrive(&sm.full[s]);
+      ++issued;
+      return;
+    }
+    int c0;
+    item_chunks(p_it, &c0);
+    const int bh = p_it / nsp, bi = bh / heads, head = bh % heads;
+    const int t0 = (c0 + p_j) * DC_CH;
+    const int tc1 = min(t0 + DC_CH, pos);                       // cached positions [t0, tc1)
+    const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
+    const int32_t* pt = a.page_table + (int64_t)bi * a.max_pages + (t0 >> 4);
+    mbar_arrive_expect_tx(&sm.full[s], (uint32_t)npg * 2 * KVB * D * 2);
+    for (int g = 0; g < npg; ++g) {
+      const int page = pt[g];
+      bulk_load(&sm.kv[s][0][g * KVB * D], a.kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &sm.full[s]);
+      bulk_load(&sm.kv[s][1][g * KVB * D], a.kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &sm.full[s]);
+    }
+    ++p_j;
+    ++issued;
+  };
+  // The cached positions were written by earlier passes and the page table at
+  // admission: the first NS stages are requested before the PDL wait.
+  if (tid == 0)
+    for (int s = 0; s < DC_NS; ++s) issue_next();
   pdl_enter();   // q and the new token's k / v come from the QKV kernel
   const uint64_t tr1 = trace_now();
-  dec_attn_partial<D, DC_CHUNK>(a, head, bi, sp, nsp, sm, 0, threadIdx.x, CtaSync{});
-  bool merged = false;
-  if (nsp > 1) {   // the last chunk of (sequence, head) to finish merges (acq_rel counter)
-    const int64_t unit = (int64_t)bi * a.heads + head;
+  const int64_t ld = (int64_t)3 * heads * D;
+  int consumed = 0;
+  bool merged_any = false;
+  for (int it = blockIdx.x; it < n_items; it += G) {
+    int c0;
+    const int nc = item_chunks(it, &c0);
+    const int sp = it % nsp, bh = it / nsp, bi = bh / heads, head = bh % heads;
+    const __nv_bfloat16* row = a.qkv + (int64_t)bi * ld;
+    float q[8], kn[8], vn[8];
+    bf16x8_to_f32(__ldcg(reinterpret_cast<const uint4*>(row + head * D + gl * 8)), q);
+    const bool has_new = nc > 0 && (c0 + nc) * DC_CH > pos && c0 * DC_CH <= pos;
+    if (has_new) {   // the new token (position pos): from the QKV output, appended to its page
+      const uint4 kv4 = __ldcg(reinterpret_cast<const uint4*>(row + (int64_t)heads * D + head * D + gl * 8));
+      const uint4 vv4 = __ldcg(reinterpret_cast<const uint4*>(row + (int64_t)2 * heads * D + head * D + gl * 8));
+      bf16x8_to_f32(kv4, kn);
+      bf16x8_to_f32(vv4, vn);
+      if (grp == 0) {
+        const int page = a.page_table[(int64_t)bi * a.max_pages + pos / KVB];
+        *reinterpret_cast<uint4*>(a.kv_pool + kv_off(page, 0, heads, head, pos % KVB, D) + gl * 8) = kv4;
+        *reinterpret_cast<uint4*>(a.kv_pool + kv_off(page, 1, heads, head, pos % KVB, D) + gl * 8) = vv4;
+      }
+    }
+    float m = -INFINITY, l = 0.f, acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    for (int j = 0; j < nc; ++j, ++consumed) {
+      const int s = consumed % DC_NS;
+      mbar_wait(&sm.full[s], (uint32_t)(consumed / DC_NS) & 1u);
+      const int t0 = (c0 + j) * DC_CH;
+      const __nv_bfloat16* sK = sm.kv[s][0];
+      const __nv_bfloat16* sV = sm.kv[s][1];
+#pragma unroll
+      for (int r = 0; r < DC_CH / NG; ++r) {
+        const int lt = r * NG + grp;           // local position of this lane group
+        const int t = t0 + lt;
+        float kf[8], vf[8];
+        if (t < pos) {
+          bf16x8_to_f32(*reinterpret_cast<const uint4*>(sK + lt * D + gl * 8), kf);
+          bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + gl * 8), vf);
+        } else {
+#pragma unroll
+          for (int e = 0; e < 8; ++e) {
+            kf[e] = kn[e];
+            vf[e] = vn[e];
+          }
+        }
+        float dot = 0.f;
+#pragma unroll
+        for (int e = 0; e < 8; ++e) dot += q[e] * kf[e];
+#pragma unroll
+        for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
+        if (t <= pos) {   // group-uniform
+          const float mn = fmaxf(m, dot);
+          const float sc = __expf(m - mn), p = __expf(dot - mn);
+          l = l * sc + p;
+#pragma unroll
+          for (int e = 0; e < 8; ++e) acc[e] = acc[e] * sc + p * vf[e];
+          m = mn;
+        }
+      }
+      __syncthreads();   // every warp is done with stage s
+      if (tid == 0) issue_next();
+    }
+    // ---- merge the lane groups' states (fixed order), then the item's result
+    if (gl == 0) {
+      sm.st_m[grp] = m;
+      sm.st_l[grp] = l;
+    }
+#pragma unroll
+    for (int e = 0; e < 8; ++e) sm.st_acc[grp][gl * 8 + e] = acc[e];
+    __syncthreads();
+    float M = -INFINITY;
+#pragma unroll
+    for (int g = 0; g < NG; ++g) M = fmaxf(M, sm.st_m[g]);
+    float L = 0.f;
+#pragma unroll
+    for (int g = 0; g < NG; ++g) L += sm.st_m[g] == -INFINITY ? 0.f : sm.st_l[g] * __expf(sm.st_m[g] - M);
+    const int64_t unit = (int64_t)bi * heads + head;
+    if (nsp == 1) {
+      for (int e = tid; e < D; e += DC_THREADS) {
+        float v = 0.f;
+#pragma unroll
+        for (int g = 0; g < NG; ++g) v += sm.st_m[g] == -INFINITY ? 0.f : sm.st_acc[g][e] * __expf(sm.st_m[g] - M);
+        a.o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(v / L);
+      }
+      __syncthreads();
+      continue;
+    }
+    float* wp = a.ws + (unit * nsp + sp) * (D + 2);
+    for (int e = tid; e < D; e += DC_THREADS) {
+      float v = 0.f;
+#pragma unroll
+      for (int g = 0; g < NG; ++g) v += sm.st_m[g] == -INFINITY ? 0.f : sm.st_acc[g][e] * __expf(sm.st_m[g] - M);
+      wp[e] = v;
+    }
+    if (tid == 0) {
+      wp[D] = M;
+      wp[D + 1] = L;
+    }
     __threadfence();
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (tid == 0) {
       int prev;
       asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&a.counters[unit]) : "memory");
-      last = (prev == nsp - 1);
+      sm.last = (prev == nsp - 1);
     }
     __syncthreads();
-    if (last) {
-      dec_attn_merge<D, DC_CHUNK>(a, head, bi, nsp, sm, threadIdx.x, CtaSync{});
-      if (threadIdx.x == 0) a.counters[unit] = 0;
-      merged = true;
+    if (sm.last) {   // the last split of (sequence, head): merge the splits in split order
+      for (int z = tid; z < nsp; z += DC_THREADS) {
+        const float* w2 = a.ws + (unit * nsp + z) * (D + 2);
+        sm.mw[z] = __ldcg(&w2[D]);
+        sm.lw[z] = __ldcg(&w2[D + 1]);
+      }
+      __syncthreads();
+      float MM = -INFINITY;
+      for (int z = 0; z < nsp; ++z) MM = fmaxf(MM, sm.mw[z]);
+      float LL = 0.f;
+      for (int z = 0; z < nsp; ++z) LL += sm.lw[z] * __expf(sm.mw[z] - MM);
+      for (int e = tid; e < D; e += DC_THREADS) {
+        float v = 0.f;
+        for (int z0 = 0; z0 < nsp; z0 += 8) {
+          float w8[8];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) w8[i] = (z0 + i < nsp) ? __ldcg(&a.ws[(unit * nsp + z0 + i) * (D + 2) + e]) : 0.f;
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            if (z0 + i < nsp) v += w8[i] * __expf(sm.mw[z0 + i] - MM);
+        }
+        a.o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(v / LL);
+      }
+      if (tid == 0) a.counters[unit] = 0;
+      merged_any = true;
     }
+    __syncthreads();
   }
-  if (threadIdx.x == 0) trace_write(merged ? (TK_ATTN_DEC | 0x100) : TK_ATTN_DEC, tr0, tr1);
+  // drain the ring: the stages issued beyond the last consumed task (arrive-only or
+  // loads that were never needed) must complete before the CTA exits
+  for (; consumed < issued; ++consumed) mbar_wait(&sm.full[consumed % DC_NS], (uint32_t)(consumed / DC_NS) & 1u);
+  if (tid == 0) trace_write(merged_any ? (TK_ATTN_DEC | 0x100) : TK_ATTN_DEC, tr0, tr1);
 }
 
-template <int D, int CH>
-static int launch_decode(const DecAttnArgs& a, int b, cudaStream_t stream) {
-  const int ns = (a.pos + 1 + CH - 1) / CH;
-  const size_t dsmem = (size_t)2 * CH * D * 2;
+template <int D>
+static int launch_decode(const DecAttnArgs& a, cudaStream_t stream) {
+  const size_t dsmem = sizeof(DecSmem<D>) + 128;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(attn_decode_kernel<D, CH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
+    cudaFuncSetAttribute(attn_decode_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
     attr = true;
   }
-  return launch_pdl(attn_decode_kernel<D, CH>, dim3(a.heads, b, ns), dim3(DC_THREADS), dsmem, stream, a);
+  const int items = a.b * a.heads * a.nsp;
+  const int grid = std::min(items, 148 * DC_CTAS_PER_SM);
+  return launch_pdl(attn_decode_kernel<D>, dim3(grid), dim3(DC_THREADS), dsmem, stream, a);
 }
 
 int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
                        int pos, int heads, int d, void* workspace, size_t ws_bytes, cudaStream_t stream) {
   if (b <= 0) return 0;
   const int ctx = pos + 1;
-  int CH = dec_attn_chunk(b, heads, ctx);
-  static const int ch_env = getenv("LIGER_ATTN_CHUNK") ? atoi(getenv("LIGER_ATTN_CHUNK")) : 0;   // experiments
-  if ((ch_env == 32 || ch_env == 64 || ch_env == 128) && (ctx + ch_env - 1) / ch_env <= DC_MAX_SPLITS) CH = ch_env;
-  const int ns = (ctx + CH - 1) / CH;
-  if (ns > DC_MAX_SPLITS) return LIGER_EINVAL;   // context longer than 4096 positions
-  if (ns > 1) {
+  DecAttnArgs a;
+  dec_attn_plan(b, heads, ctx, &a.cps, &a.nsp);
+  if (a.nsp > DC_MAX_SPLITS || (d != 64 && d != 128)) return LIGER_EINVAL;
+  if (a.nsp > 1) {
     if (!workspace || ws_bytes < attn_decode_workspace_bytes(b, heads, d, ctx) ||
         (size_t)b * heads * 4 > ATTN_COUNTER_BYTES)
       return LIGER_EINVAL;
   }
-  DecAttnArgs a;
   a.qkv = (const __nv_bfloat16*)qkv;
   a.o = (__nv_bfloat16*)o;
   a.kv_pool = (__nv_bfloat16*)kv_pool;
@@ -370,17 +525,10 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   a.max_pages = max_pages;
   a.pos = pos;
   a.heads = heads;
+  a.b = b;
   a.counters = (int*)workspace;
   a.ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
-  int rc;
-  if (d == 128)
-    rc = CH == 32 ? launch_decode<128, 32>(a, b, stream)
-                  : CH == 64 ? launch_decode<128, 64>(a, b, stream) : launch_decode<128, 128>(a, b, stream);
-  else if (d == 64)
-    rc = CH == 32 ? launch_decode<64, 32>(a, b, stream)
-                  : CH == 64 ? launch_decode<64, 64>(a, b, stream) : launch_decode<64, 128>(a, b, stream);
-  else
-    return LIGER_EINVAL;
+  const int rc = d == 128 ? launch_decode<128>(a, stream) : launch_decode<64>(a, stream);
   return rc ? LIGER_ECUDA : 0;
 }
 

@@ -95,69 +95,78 @@ struct NcclComm : Comm {
     if (region) cudaFree(region);
     if (comm) nccl().CommDestroy(comm);
   }
-  // [collective] map every rank's staging region: CUDA IPC handles exchanged with an
-  // NCCL all-gather (same-node NVLink / NVSwitch peers).  The ranks then agree (NCCL
-  // min) on whether every rank mapped every peer; if any could not (e.g. peers not
-  // P2P-reachable from this process), all of them fall back to NCCL all-reduces.
+  // all ranks' min of a local flag (a collective every rank reaches, whatever its flag)
+  int agree_min(int v, cudaStream_t st, int* out) {
+    int32_t* d = nullptr;
+    if (cudaMalloc(&d, sizeof(int32_t)) != cudaSuccess) return LIGER_ENOMEM;
+    cudaMemcpy(d, &v, sizeof(int32_t), cudaMemcpyHostToDevice);
+    ncclResult_t r = nccl().AllReduce(d, d, 1, ncclInt32, ncclMin, comm, st);
+    if (r == ncclSuccess && cudaStreamSynchronize(st) == cudaSuccess)
+      cudaMemcpy(out, d, sizeof(int32_t), cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    return r == ncclSuccess ? 0 : LIGER_ENCCL;
+  }
+  // [collective, at communicator creation] map every rank's staging region: CUDA IPC
+  // handles exchanged with an NCCL all-gather (same-node NVLink / NVSwitch peers).  Every
+  // rank takes part in every collective whatever its local outcome, and the ranks agree
+  // (NCCL min) first on the allocation and then on every rank having mapped every peer;
+  // if any step failed anywhere, all of them use NCCL all-reduces (no rank returns early
+  // while its peers wait in a collective).
   int setup_oneshot(cudaStream_t st) {
     const size_t cap = oneshot_cap(), rb = peer_ar_region_bytes(cap);
-    if (world > 8 || cudaMalloc(&region, rb) != cudaSuccess || cudaMemset(region, 0, rb) != cudaSuccess)
-      return LIGER_ENOMEM;
-    cudaIpcMemHandle_t h;
-    int ok = cudaIpcGetMemHandle(&h, region) == cudaSuccess ? 1 : 0;
-    char* d = nullptr;
-    if (cudaMalloc(&d, (size_t)64 * (world + 1) + 16) != cudaSuccess) return LIGER_ENOMEM;
-    cudaMemcpy(d + (size_t)64 * world, &h, 64, cudaMemcpyHostToDevice);
-    ncclResult_t r = nccl().AllGather(d + (size_t)64 * world, d, 64, ncclUint8, comm, st);
-    std::vector<cudaIpcMemHandle_t> all(world);
-    if (r == ncclSuccess && cudaStreamSynchronize(st) == cudaSuccess)
-      cudaMemcpy(all.data(), d, (size_t)64 * world, cudaMemcpyDeviceToHost);
-    if (r != ncclSuccess) {
-      cudaFree(d);
-      return LIGER_ENCCL;
+    int ok = world <= 8 ? 1 : 0;
+    if (ok && (cudaMalloc(&region, rb) != cudaSuccess || cudaMemset(region, 0, rb) != cudaSuccess)) {
+      cudaGetLastError();
+      if (region) cudaFree(region);
+      region = nullptr;
+      ok = 0;
     }
-    for (int q = 0; q < world && ok; ++q) {
-      if (q == rank) {
-        mapped[q] = region;
-        continue;
-      }
-      if (cudaIpcOpenMemHandle(&mapped[q], all[q], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
-        cudaGetLastError();
-        mapped[q] = nullptr;
-        ok = 0;
-      }
+    cudaIpcMemHandle_t h{};
+    if (ok && cudaIpcGetMemHandle(&h, region) != cudaSuccess) {
+      cudaGetLastError();
+      ok = 0;
     }
-    int32_t* flag = reinterpret_cast<int32_t*>(d + (size_t)64 * (world + 1));
-    cudaMemcpy(flag, &ok, sizeof(int32_t), cudaMemcpyHostToDevice);
-    r = nccl().AllReduce(flag, flag, 1, ncclInt32, ncclMin, comm, st);
     int all_ok = 0;
-    if (r == ncclSuccess && cudaStreamSynchronize(st) == cudaSuccess)
-      cudaMemcpy(&all_ok, flag, sizeof(int32_t), cudaMemcpyDeviceToHost);
-    cudaFree(d);
-    if (r != ncclSuccess) return LIGER_ENCCL;
-    if (!all_ok) {   // agreed fallback: NCCL for every all-reduce from now on
+    if (int rc = agree_min(ok, st, &all_ok)) return rc;
+    if (all_ok) {
+      char* d = nullptr;
+      if (cudaMalloc(&d, (size_t)64 * (world + 1)) != cudaSuccess) return LIGER_ENOMEM;
+      cudaMemcpy(d + (size_t)64 * world, &h, 64, cudaMemcpyHostToDevice);
+      ncclResult_t r = nccl().AllGather(d + (size_t)64 * world, d, 64, ncclUint8, comm, st);
+      std::vector<cudaIpcMemHandle_t> all(world);
+      if (r == ncclSuccess && cudaStreamSynchronize(st) == cudaSuccess)
+        cudaMemcpy(all.data(), d, (size_t)64 * world, cudaMemcpyDeviceToHost);
+      cudaFree(d);
+      if (r != ncclSuccess) return LIGER_ENCCL;
+      for (int q = 0; q < world && ok; ++q) {
+        if (q == rank) {
+          mapped[q] = region;
+          continue;
+        }
+        if (cudaIpcOpenMemHandle(&mapped[q], all[q], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+          cudaGetLastError();
+          mapped[q] = nullptr;
+          ok = 0;
+        }
+      }
+      if (int rc = agree_min(ok, st, &all_ok)) return rc;
+    }
+    if (!all_ok) {   // agreed fallback: NCCL for every all-reduce
       for (int q = 0; q < world; ++q)
         if (mapped[q] && q != rank) cudaIpcCloseMemHandle(mapped[q]);
       for (int q = 0; q < world; ++q) mapped[q] = nullptr;
       oneshot = false;
-      err = "one-shot all-reduce disabled: a rank could not map its peers' staging buffers";
+      err = "one-shot all-reduce disabled: a rank could not set up or map the peers' staging buffers";
       return 0;
     }
     par = new PeerAR();
     return par->init(world, rank, cap, region, mapped);
   }
-  PeerAR* peer_ar(cudaStream_t st) override {
-    if (!oneshot) return nullptr;
-    if (!par && setup_oneshot(st)) return nullptr;
-    return par;   // nullptr after an agreed fallback
-  }
+  int init_peer(cudaStream_t st) override { return oneshot ? setup_oneshot(st) : 0; }
+  PeerAR* peer_ar(cudaStream_t) override { return oneshot ? par : nullptr; }
   int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
     if (!count) return 0;
-    if (oneshot && oneshot_eligible(count, dt, op, buf)) {
-      if (!par)
-        if (int rc = setup_oneshot(st)) return rc;
-      if (par) return par->allreduce_bf16(buf, count, st);
-    }
+    if (oneshot && par && oneshot_eligible(count, dt, op, buf)) return par->allreduce_bf16(buf, count, st);
     ncclResult_t r = nccl().AllReduce(buf, buf, count, nccl_dt(dt), op == CO_SUM ? ncclSum : ncclMax, comm, st);
     if (r != ncclSuccess) {
       err = std::string("ncclAllReduce: ") + nccl().GetErrorString(r);
@@ -351,31 +360,39 @@ struct LoopbackComm : Comm {
     scratch_bytes = bytes;
     return 0;
   }
-  // [collective] the ranks' staging regions are plain device pointers of one process
+  // [collective, at communicator creation] the ranks' staging regions are plain device
+  // pointers of one process; every rank reaches the rendezvous whatever its allocation
+  // outcome, and all fall back together if any rank has no region
   int setup_oneshot() {
     const size_t cap = oneshot_cap(), rb = peer_ar_region_bytes(cap);
-    if (cudaMalloc(&region, rb) != cudaSuccess || cudaMemset(region, 0, rb) != cudaSuccess) return LIGER_ENOMEM;
+    if (cudaMalloc(&region, rb) != cudaSuccess || cudaMemset(region, 0, rb) != cudaSuccess) {
+      cudaGetLastError();
+      if (region) cudaFree(region);
+      region = nullptr;
+    }
     cudaDeviceSynchronize();
     std::vector<const void*> xs, ys;
     std::vector<cudaEvent_t> es;
     rendezvous(region, nullptr, nullptr, &xs, &ys, &es);
     void* peers[8] = {};
-    for (int q = 0; q < world; ++q) peers[q] = const_cast<void*>(xs[q]);
+    bool all = true;
+    for (int q = 0; q < world; ++q) {
+      peers[q] = const_cast<void*>(xs[q]);
+      all = all && peers[q];
+    }
+    if (!all) {
+      oneshot = false;
+      err = "one-shot all-reduce disabled: a rank could not allocate its staging buffer";
+      return 0;
+    }
     par = new PeerAR();
     return par->init(world, rank, cap, region, peers);
   }
-  PeerAR* peer_ar(cudaStream_t) override {
-    if (!oneshot) return nullptr;
-    if (!par && setup_oneshot()) return nullptr;
-    return par;
-  }
+  int init_peer(cudaStream_t) override { return oneshot ? setup_oneshot() : 0; }
+  PeerAR* peer_ar(cudaStream_t) override { return oneshot ? par : nullptr; }
   int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
     if (!count) return 0;
-    if (oneshot && oneshot_eligible(count, dt, op, buf)) {
-      if (!par)
-        if (int rc = setup_oneshot()) return rc;
-      return par->allreduce_bf16(buf, count, st);
-    }
+    if (oneshot && par && oneshot_eligible(count, dt, op, buf)) return par->allreduce_bf16(buf, count, st);
     const size_t bytes = count * dt_size(dt);
     if (int rc = ensure_scratch(bytes)) return rc;
     std::vector<const void*> xs, ys;
@@ -520,6 +537,11 @@ Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err) {
       delete c;
       return nullptr;
     }
+    if (c->init_peer(nullptr)) {
+      *err = "loopback communicator: one-shot setup failed";
+      delete c;
+      return nullptr;
+    }
     return c;
   }
   if (!nccl().ok) {
@@ -536,6 +558,16 @@ Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err) {
   if (r != ncclSuccess) {
     *err = std::string("ncclCommInitRank: ") + nccl().GetErrorString(r);
     c->comm = nullptr;
+    delete c;
+    return nullptr;
+  }
+  // the one-shot staging buffers are set up here, eagerly (a collective of every rank),
+  // never lazily inside a serving call
+  cudaStream_t st = nullptr;
+  int rc = cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) == cudaSuccess ? c->init_peer(st) : LIGER_ECUDA;
+  if (st) cudaStreamDestroy(st);
+  if (rc) {
+    *err = "NCCL communicator: one-shot all-reduce setup failed (" + c->err + ")";
     delete c;
     return nullptr;
   }

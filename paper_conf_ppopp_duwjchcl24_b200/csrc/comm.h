@@ -65,8 +65,9 @@ struct Comm {
   virtual int check_async() = 0;
   // host-side barrier of the group (loopback: every rank's thread has arrived)
   virtual void barrier() {}
-  // the one-shot peer all-reduce state (set up on first use; [collective]), or
-  // nullptr when this backend does not use it
+  // [collective] set up the one-shot peer all-reduce (called once by comm_create)
+  virtual int init_peer(cudaStream_t) { return 0; }
+  // the one-shot peer all-reduce state, or nullptr when this backend does not use it
   virtual PeerAR* peer_ar(cudaStream_t) { return nullptr; }
 };
 

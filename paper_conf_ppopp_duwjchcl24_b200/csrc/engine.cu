@@ -49,7 +49,9 @@ double now_s() {
 int weight_exp(int K, bool out_proj = false) {
   return (int)std::nearbyint(0.5 * std::log2(3.0 / K)) - (out_proj ? 2 : 1);
 }
-constexpr int BIAS_EXP = -6, EMB_EXP = -3;
+constexpr int BIAS_EXP = -6;
+// embeddings: 2^(round(-log2(h)/2) - 1) (C0, reading R16)
+int emb_exp(int h) { return (int)std::nearbyint(-0.5 * std::log2((double)h)) - 1; }
 constexpr uint64_t GID_ETOK = 0xFFFF00, GID_EPOS = 0xFFFF01, GID_LNFG = 0xFFFF02, GID_LNFB = 0xFFFF03;
 
 // ------------------------------------------------------------------ ops of one pass
@@ -85,6 +87,7 @@ struct Batch;
 // Per in-flight batch slot device buffers.
 struct Slot {
   void *x, *y, *qkv, *attn, *part, *hbuf, *yhead;
+  void* xhead = nullptr;   // [B, h] bf16: the last token's residual after the last layer (LM-head input)
   float *logits, *vals_all;
   int32_t *idx_all, *cur_tok, *tok_out, *prompt, *page_table;
   void *gemm_ws, *attn_ws;
@@ -130,6 +133,11 @@ struct Batch {
   // cursor
   int pass = 0, idx = 0, done = 0;   // done = units of the current op already launched
   bool all_launched = false, finished = false, results_copied = false;
+  bool captured = false;   // the LM head ran with debug capture on (liger_debug_read)
+  // debug capture (liger_set_debug_capture), allocated at admission: per pass, this
+  // rank's fp32 logits shard [n_new][b][V/t] and the LM-head input rows [n_new][b][h] bf16
+  float* dbg_logits = nullptr;
+  void* dbg_resid = nullptr;
   cudaEvent_t last_ev = nullptr;
   int last_stream = -1;
   bool has_last_ev = false;
@@ -195,6 +203,11 @@ struct liger_ctx {
   // OPT-13B bench (24.96 vs 24.44 req/s, same box); bits per batch unchanged
   bool t1_streams = false;   // Inter-Th: projection GEMMs issued as this many partitioned kernels
   bool calibrating = false;   // liger_calibrate_cf at t = 1 (proxy communicator)
+  // debug capture arena (liger_set_debug_capture): batches admitted while it is on take
+  // their capture buffers from it in admission order (bump allocation, never reused)
+  char* dbg_arena = nullptr;
+  size_t dbg_arena_bytes = 0, dbg_arena_used = 0;
+  bool dbg_capture = false;
   int n_sms = 148;
   // stats / timing
   liger_stats_t st{};
@@ -589,7 +602,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       // residual add of the last layer + final LN on the last token of each sequence
       const int step = pass == 0 ? bt->s : 1, off = pass == 0 ? bt->s - 1 : 0;
       // (folded decode pass: the last FC2 already added its output and bias to x)
-      rc = add_layernorm_launch(S.x, fold ? nullptr : S.part, fold ? nullptr : Wl.b_2, nullptr, S.yhead, c->lnf_g,
+      rc = add_layernorm_launch(S.x, fold ? nullptr : S.part, fold ? nullptr : Wl.b_2, S.xhead, S.yhead, c->lnf_g,
                                 c->lnf_b, b, h, step, off, eps, st);
       if (rc) break;
       GemmArgs g{};
@@ -607,6 +620,13 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
                          S.idx_all + (size_t)c->tp_rank * b, st);
       if (rc) break;
       c->st.gpu_launches += 3;
+      if (bt->dbg_logits) {   // test readback (liger_debug_read): copies only
+        cudaMemcpyAsync(bt->dbg_logits + (size_t)pass * b * c->Vl, S.logits, (size_t)b * c->Vl * 4,
+                        cudaMemcpyDeviceToDevice, st);
+        cudaMemcpyAsync((char*)bt->dbg_resid + (size_t)pass * b * h * 2, S.xhead, (size_t)b * h * 2,
+                        cudaMemcpyDeviceToDevice, st);
+        bt->captured = true;
+      }
       if (c->tp == 1) {
         rc = argmax_pick_launch(S.vals_all, S.idx_all, 1, b, S.cur_tok, S.tok_out, bt->n_new, pass, st);
         c->st.gpu_launches++;
@@ -708,12 +728,24 @@ struct BatchCursor : Cursor {
 // ------------------------------------------------------------------ admission / completion
 void reap(liger_ctx* c);
 
-// Admission is a pure function of the submit order (round-robin slots with a
-// fixed page range each), so every rank admits the same batch at the same
-// liger_step and all ranks issue identical plans / collectives.  Reusing a
-// slot waits (host) for its previous occupant, whose kernels are all enqueued.
-void admit(liger_ctx* c, Batch* bt) {
-  const int slot = (int)(c->admitted++ % (int64_t)c->slots.size());
+// Admission is a pure function of the submit order and of the launch state (slots
+// with a fixed page range each, taken round-robin from the next one, skipping slots
+// whose owner has kernels left to launch -- the same on every rank, since all ranks
+// make identical plans), so every rank admits the same batch into the same slot at
+// the same liger_step and all ranks issue identical plans / collectives.  A slot is
+// reusable once its previous owner has launched everything (its final event is
+// recorded); the host waits for that event before overwriting the slot's pinned
+// staging buffers.  Returns false (batch stays waiting) when no slot is reusable.
+bool admit(liger_ctx* c, Batch* bt) {
+  const int ns = (int)c->slots.size();
+  int slot = -1;
+  for (int i = 0; i < ns && slot < 0; ++i) {
+    const int s = (int)((c->admitted + i) % ns);
+    const Batch* o = c->slots[s].owner;
+    if (!o || o->all_launched) slot = s;
+  }
+  if (slot < 0) return false;
+  c->admitted = slot + 1;
   Slot& S = c->slots[slot];
   if (S.owner && !S.owner->finished) {
     cudaEventSynchronize(S.owner->final_ev);
@@ -738,6 +770,19 @@ void admit(liger_ctx* c, Batch* bt) {
   bt->last_ev = pool_event(c);
   cudaEventRecord(bt->last_ev, st);
   bt->has_last_ev = true;
+  if (c->dbg_capture && c->l1 == c->L) {   // test readback buffers of this batch (liger_debug_read)
+    // (from the preallocated arena: no cudaMalloc while peers may spin in one-shot kernels)
+    const size_t nl = ((size_t)bt->n_new * bt->b * c->Vl * 4 + 255) / 256 * 256;
+    const size_t nr = ((size_t)bt->n_new * bt->b * c->h * 2 + 255) / 256 * 256;
+    if (c->dbg_arena_used + nl + nr <= c->dbg_arena_bytes) {
+      bt->dbg_logits = reinterpret_cast<float*>(c->dbg_arena + c->dbg_arena_used);
+      bt->dbg_resid = c->dbg_arena + c->dbg_arena_used + nl;
+      c->dbg_arena_used += nl + nr;
+    }
+  }
+  bt->host_tokens.clear();   // staged in the slot's pinned buffer (copied in stream order)
+  bt->host_tokens.shrink_to_fit();
+  return true;
 }
 
 void CUDART_CB host_finish(void* p) {
@@ -767,6 +812,8 @@ void reap(liger_ctx* c) {
       bt->results_copied = true;
     }
     if (bt->finish_s.load() == 0) bt->finish_s.store(now_s());
+    cudaEventDestroy(bt->final_ev);   // complete; nothing waits on it any more
+    bt->final_ev = nullptr;
   }
 }
 
@@ -780,7 +827,7 @@ void update_list(liger_ctx* c) {
   reap(c);
   while ((int)c->processing.size() < cap && !c->waiting.empty()) {
     Batch* bt = c->waiting.front().get();
-    admit(c, bt);
+    if (!admit(c, bt)) break;
     c->processing.push_back(bt);
     c->all_batches[bt->id] = std::move(c->waiting.front());
     c->waiting.pop_front();
@@ -974,6 +1021,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     S.ln_stats = (float*)dalloc(c, 2 * 64 * sizeof(float));
     S.hbuf = dalloc(c, (size_t)Mmax * c->fl * 2);
     S.yhead = dalloc(c, (size_t)B * h * 2);
+    S.xhead = dalloc(c, (size_t)B * h * 2);
     S.logits = (float*)dalloc(c, (size_t)B * c->Vl * 4);
     S.vals_all = (float*)dalloc(c, (size_t)tp * B * 4);
     S.idx_all = (int32_t*)dalloc(c, (size_t)tp * B * 4);
@@ -1102,8 +1150,8 @@ int liger_load_embed(liger_ctx* c, uint64_t seed) {
   if (!c) return LIGER_EINVAL;
   const int64_t h = c->h;
   cudaStream_t st = c->s_comp;
-  CKR(c0_fill_launch(c->e_tok, c->V, (int)h, h, seed, GID_ETOK, 0, 0, h, 1, EMB_EXP, 0, st));
-  CKR(c0_fill_launch(c->e_pos, c->cfg.max_pos + 2, (int)h, h, seed, GID_EPOS, 0, 0, h, 1, EMB_EXP, 0, st));
+  CKR(c0_fill_launch(c->e_tok, c->V, (int)h, h, seed, GID_ETOK, 0, 0, h, 1, emb_exp((int)h), 0, st));
+  CKR(c0_fill_launch(c->e_pos, c->cfg.max_pos + 2, (int)h, h, seed, GID_EPOS, 0, 0, h, 1, emb_exp((int)h), 0, st));
   CKR(c0_fill_launch(c->lnf_g, 1, (int)h, h, seed, GID_LNFG, 0, 0, 0, 1, 0, 1, st));
   CKR(c0_fill_launch(c->lnf_b, 1, (int)h, h, seed, GID_LNFB, 0, 0, 0, 1, 0, 2, st));
   CK(cudaStreamSynchronize(st));
@@ -1300,7 +1348,71 @@ int liger_result_tokens_device(liger_ctx* c, int64_t id, const int32_t** dev_tok
   if (!c || id < 0 || id >= (int64_t)c->all_batches.size() || !dev_tokens) return LIGER_EINVAL;
   Batch* bt = c->all_batches[id].get();
   if (!bt || bt->slot < 0) return LIGER_PENDING;
+  if (!bt->finished) reap(c);
+  if (!bt->finished) return LIGER_PENDING;
+  if (c->slots[bt->slot].owner != bt)
+    return fail(c, LIGER_ESTATE, "liger_result_tokens_device: the batch's slot was reused by a later batch");
   *dev_tokens = c->slots[bt->slot].tok_out;
+  return LIGER_OK;
+}
+
+int liger_op_allreduce(liger_ctx* c, void* buf, size_t count, int u0, int u1, int F, void* stream) {
+  if (!c || !buf || F < 1 || u0 < 0 || u1 > F || u0 > u1) return LIGER_EINVAL;
+  if (!c->comm || u0 == u1 || !count) return LIGER_OK;   // t = 1: the sum of one partial
+  cudaStream_t st = stream ? (cudaStream_t)stream : c->s_comm;
+  if (issue_ar(c, buf, count, u0, u1, F, st)) return fail(c, LIGER_ENCCL, c->comm->err);
+  c->st.comm_kernels++;
+  return LIGER_OK;
+}
+
+const char* liger_scheduler_name(const liger_ctx* c) {
+  if (!c) return "none";
+  if (c->cfg.mode == LIGER_MODE_PIPELINE) return "pipeline";
+  if (c->cfg.mode == LIGER_MODE_PIPELINE_TH) return "pipeline_th";
+  if (c->cfg.mode == LIGER_MODE_SERIAL) return "serial";
+  if (c->t1_streams) return "t1_two_stream";
+  if (c->tp == 1) return "t1_algorithm1";   // t = 1 without the two-stream schedule (LIGER_T1_STREAMS=0)
+  switch (c->cfg.sync_mode) {
+    case LIGER_SYNC_CPU_GPU: return "algorithm1_cpu_gpu";
+    case LIGER_SYNC_INTER_STREAM: return "algorithm1_inter_stream";
+  }
+  return "algorithm1_hybrid";
+}
+
+int liger_set_debug_capture(liger_ctx* c, size_t arena_bytes) {
+  if (!c) return LIGER_EINVAL;
+  if (arena_bytes > c->dbg_arena_bytes) {
+    if (!c->processing.empty()) return fail(c, LIGER_ESTATE, "liger_set_debug_capture: batches in flight");
+    if (c->dbg_arena) cudaFree(c->dbg_arena);
+    c->dbg_arena = nullptr;
+    c->dbg_arena_bytes = c->dbg_arena_used = 0;
+    if (cudaMalloc((void**)&c->dbg_arena, arena_bytes) != cudaSuccess) {
+      cudaGetLastError();
+      c->dbg_arena = nullptr;
+    } else {
+      c->dbg_arena_bytes = arena_bytes;
+    }
+  }
+  // [collective]: nobody starts serving (and spinning on peers) before every rank has allocated
+  if (c->comm) c->comm->barrier();
+  if (arena_bytes && !c->dbg_arena) return fail(c, LIGER_ENOMEM, "liger_set_debug_capture: capture arena");
+  c->dbg_capture = arena_bytes != 0;
+  return LIGER_OK;
+}
+
+int liger_debug_read(liger_ctx* c, int64_t id, int what, void* host_buf, size_t bytes) {
+  if (!c || id < 0 || id >= (int64_t)c->all_batches.size() || !host_buf) return LIGER_EINVAL;
+  if (what != LIGER_DBG_LOGITS && what != LIGER_DBG_RESID) return LIGER_EINVAL;
+  Batch* bt = c->all_batches[id].get();
+  if (!bt) return LIGER_PENDING;
+  if (!bt->finished) reap(c);
+  if (!bt->finished) return LIGER_PENDING;
+  if (!bt->captured) return fail(c, LIGER_ESTATE, "liger_debug_read: no capture for this batch on this rank");
+  const size_t need = what == LIGER_DBG_LOGITS ? (size_t)bt->n_new * bt->b * c->Vl * 4
+                                                : (size_t)bt->n_new * bt->b * c->h * 2;
+  if (bytes < need) return fail(c, LIGER_EINVAL, "liger_debug_read: host buffer too small");
+  CK(cudaMemcpy(host_buf, what == LIGER_DBG_LOGITS ? (const void*)bt->dbg_logits : bt->dbg_resid, need,
+                cudaMemcpyDeviceToHost));
   return LIGER_OK;
 }
 
@@ -1601,7 +1713,8 @@ int liger_finalize(liger_ctx* c) {
   for (auto e : c->ev_pool) cudaEventDestroy(e);
   for (auto e : c->timing_pool) cudaEventDestroy(e);
   for (auto& b : c->all_batches)
-    if (b) cudaEventDestroy(b->final_ev);
+    if (b && b->final_ev) cudaEventDestroy(b->final_ev);
+  if (c->dbg_arena) cudaFree(c->dbg_arena);
   for (auto& b : c->waiting) cudaEventDestroy(b->final_ev);
   cudaEventDestroy(c->e1);
   cudaEventDestroy(c->e2);

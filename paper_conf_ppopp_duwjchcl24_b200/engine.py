@@ -114,6 +114,37 @@ class LigerEngine:
             toks = buf[:res.batch * res.n_new].reshape(res.batch, res.n_new).copy()
         return res, toks
 
+    def allreduce(self, buf, u0=0, u1=1, F=1, stream=None):
+        """liger_op_allreduce: in-place bf16 sum over the ranks of units [u0, u1) of F."""
+        self._chk(L.lib().liger_op_allreduce(self.ctx, C.c_void_p(buf.data_ptr()), buf.numel(), u0, u1, F,
+                                             None if stream is None else C.c_void_p(stream)), "liger_op_allreduce")
+
+    def set_debug_capture(self, arena_bytes=256 << 20):
+        """Test readback (liger_set_debug_capture, [collective]): capture per-pass logits and
+        LM-head input rows of the batches admitted from now on (0 turns it off)."""
+        self._chk(L.lib().liger_set_debug_capture(self.ctx, C.c_size_t(int(arena_bytes))),
+                  "liger_set_debug_capture")
+
+    def debug_read(self, bid, what, batch, n_new):
+        """liger_debug_read -> numpy: 'logits' fp32 [batch, n_new, V/t] (this rank's shard)
+        or 'resid' float32 (bf16 values) [batch, n_new, h]."""
+        if what == "logits":
+            n = self.model.vocab // (1 if self.cfg.mode >= 2 else self.world)
+            buf = np.empty((n_new, batch, n), dtype=np.float32)
+            code = L.DBG_LOGITS
+        else:
+            buf = np.empty((n_new, batch, self.model.hidden), dtype=np.uint16)
+            code = L.DBG_RESID
+        self._chk(L.lib().liger_debug_read(self.ctx, bid, code, buf.ctypes.data_as(C.c_void_p), buf.nbytes),
+                  "liger_debug_read")
+        if what != "logits":
+            buf = (buf.astype(np.uint32) << 16).view(np.float32)
+        return np.ascontiguousarray(buf.transpose(1, 0, 2))
+
+    def scheduler_name(self):
+        """The schedule this context runs (liger_scheduler_name)."""
+        return L.lib().liger_scheduler_name(self.ctx).decode()
+
     def stats(self):
         s = L.liger_stats_t()
         self._chk(L.lib().liger_stats(self.ctx, C.byref(s)), "liger_stats")

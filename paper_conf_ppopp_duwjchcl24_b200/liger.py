@@ -9,6 +9,9 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libliger.so")
 
 LIGER_OK, LIGER_PENDING, LIGER_IDLE = 0, 1, 2
+LIGER_EINVAL, LIGER_ENOMEM, LIGER_ECUDA, LIGER_ENCCL, LIGER_ESTATE, LIGER_ETIMEOUT, LIGER_ENODEV = (
+    -22, -12, -1000, -1001, -1002, -1003, -1004)
+DBG_LOGITS, DBG_RESID = 1, 2
 ACT = {"none": 0, "relu": 1, "gelu_tanh": 2}
 SYNC = {"hybrid": 0, "cpu_gpu": 1, "inter_stream": 2}
 MODE = {"serial": 0, "interleaved": 1, "pipeline": 2, "pipeline_th": 3}
@@ -56,6 +59,9 @@ _SIGS = {
     "liger_drain": (_I, [_P]),
     "liger_poll": (_I, [_P, _I64, C.POINTER(liger_result), _P]),
     "liger_result_tokens_device": (_I, [_P, _I64, C.POINTER(_P)]),
+    "liger_set_debug_capture": (_I, [_P, _SZ]),
+    "liger_op_allreduce": (_I, [_P, _P, _SZ, _I, _I, _I, _P]),
+    "liger_debug_read": (_I, [_P, _I64, _I, _P, _SZ]),
     "liger_stats": (_I, [_P, C.POINTER(liger_stats_t)]),
     "liger_reset_stats": (_I, [_P]),
     "liger_set_gemm_sm_reserve": (_I, [_P, _I]),
@@ -65,6 +71,7 @@ _SIGS = {
     "liger_profile": (_I, [_P, _P, _I]),
     "liger_calibrate_cf": (_I, [_P, _P, _I, _I, _P, _P]),
     "liger_last_error": (C.c_char_p, [_P]),
+    "liger_scheduler_name": (C.c_char_p, [_P]),
     "liger_finalize": (_I, [_P]),
     "liger_op_gemm": (_I, [_P, _I64, _P, _I64, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),
     "liger_op_gemm_tiled": (_I, [_P, _I64, _P, _P, _I64, _I, _I, _I, _I, _I, _P, _I, _I, _F, _I, _P, _SZ, _P]),

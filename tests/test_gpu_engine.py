@@ -1,12 +1,18 @@
 """End-to-end serving through liger_init / liger_load_layer / liger_submit /
-liger_step / liger_poll on one GPU: greedy tokens identical to the fp64 oracle
-on the tiny config (BASELINE.json), and serial vs interleaved runs bit-exact."""
+liger_step / liger_poll on one GPU (t = 1), compared with the fp64 oracle element
+by element (tests/engine_check.py): the LM-head input residual and the logits of
+every pass through the C-ABI debug readback, and the greedy tokens.  The inputs are
+non-degenerate (the oracle's tokens are not the echo of the prompt a model without
+layers gives), and a deliberately broken layer makes the checks fail."""
+import os
+
 import numpy as np
 import pytest
 import torch
 
 from liger_inputs import get_config, make_trace
-from oracle import model as om
+from liger_inputs.configs import ModelConfig
+from engine_check import serve, check_vs_oracle, assert_bit_identical
 
 pytestmark = pytest.mark.gpu
 
@@ -19,55 +25,105 @@ def E():
     return LigerEngine
 
 
-def _serve(engine, trace, want_tokens=True):
-    ids = [engine.submit(r["tokens"], r["batch"], r["seq_len"], r["n_decode"], r["arrival_s"]) for r in trace]
-    engine.drain()
-    out = []
-    for bid in ids:
-        res = engine.poll(bid, want_tokens=want_tokens)
-        assert res is not None and res[0].done == 1
-        out.append(res[1])
-    return out
+def _with_env(env, fn):
+    old = {k: os.environ.get(k) for k in env}
+    os.environ.update(env)
+    try:
+        return fn()
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
 
 
-def test_tiny_greedy_tokens_match_oracle(E):
+def _mixed_trace(n, seed, cfg, batch_sizes, prompt_range, n_new_choices):
+    """make_trace with a per-batch number of generated tokens (mixed n_new)."""
+    tr = make_trace(n, float("inf"), seed=seed, batch_sizes=batch_sizes, prompt_range=prompt_range, n_decode=1,
+                    vocab=cfg.vocab)
+    rng = np.random.default_rng(seed + 1000)
+    for t in tr:
+        t["n_decode"] = int(rng.choice(n_new_choices))
+    return tr
+
+
+def test_tiny_serving_matches_oracle_elementwise(E):
+    """BASELINE.json configs[0] shape (tiny, batch 2, prompt 32 + 8 generated) at t = 1:
+    residual, logits and tokens of every pass against the oracle."""
     cfg = get_config("tiny")
-    seed = 0
-    prompt = np.random.default_rng(0).integers(0, cfg.vocab, size=(2, 32))
-    ref, logits = om.greedy_generate(cfg, seed, prompt, 8, return_logits=True)
-    margin = om.top2_margin(logits)
-    rms = np.sqrt((logits ** 2).mean())
-    assert margin.min() > 0.02 * rms, "seed gives near-tied logits (reading R17): pick another seed"
-    eng = E(cfg, mode="serial", max_batch=4, max_seq=64, max_new=8, seed=seed)
-    toks = _serve(eng, [dict(tokens=prompt.reshape(-1), batch=2, seq_len=32, n_decode=8, arrival_s=0.0)])[0]
-    eng.close()
-    assert np.array_equal(toks, ref)
+    prompt = np.random.default_rng(0).integers(0, cfg.vocab, size=(2, 32)).astype(np.int32)
+    trace = [dict(tokens=prompt.reshape(-1), batch=2, seq_len=32, n_decode=8)]
+    res = serve(E, cfg, 1, trace, mode="serial", max_batch=4, max_seq=64, max_new=8, seed=0)
+    check_vs_oracle(cfg, 0, trace, res)
 
 
 def test_modes_bit_exact_and_match_oracle(E):
+    """Serial intra-op, interleaved with F = 8 and a processing list of 3 (t = 1: the
+    two-stream schedule, reading R31) over a trace with mixed batch sizes and mixed
+    numbers of generated tokens: every mode equals the oracle element-wise and the
+    modes are bit-identical to each other (tokens, logits, residual)."""
     cfg = get_config("tiny")
-    trace = make_trace(6, float("inf"), seed=3, batch_sizes=(1, 2, 3), prompt_range=(5, 40), n_decode=6,
-                       vocab=cfg.vocab)
+    trace = _mixed_trace(6, 3, cfg, (1, 2, 3), (5, 40), (2, 6, 8))
     results = {}
     for mode, infl, F in (("serial", 1, 1), ("interleaved", 2, 8), ("interleaved", 3, 1)):
-        eng = E(cfg, mode=mode, max_batch=4, max_seq=64, max_new=8, max_inflight=infl, decomp_factor=F, seed=1)
-        results[(mode, infl, F)] = _serve(eng, trace)
-        st = eng.stats()
+        results[(mode, infl, F)] = serve(E, cfg, 1, trace, mode=mode, max_batch=4, max_seq=64, max_new=8,
+                                         max_inflight=infl, decomp_factor=F, seed=1)
+        st = results[(mode, infl, F)][0]["stats"]
         assert st["kernels"] > 0 and st["gpu_launches"] > 0
-        eng.close()
     base = results[("serial", 1, 1)]
+    check_vs_oracle(cfg, 1, trace, base)
     for k, v in results.items():
-        for a, b in zip(base, v):
-            assert np.array_equal(a, b), k
-    # the tokens are the oracle's greedy tokens (where the oracle's margin is unambiguous)
-    for r, toks in zip(trace[:3], base[:3]):
-        p = r["tokens"].reshape(r["batch"], r["seq_len"])
-        ref, logits = om.greedy_generate(cfg, 1, p, r["n_decode"], return_logits=True)
-        ok = om.top2_margin(logits) > 0.02 * np.sqrt((logits ** 2).mean())
-        # compare up to the first ambiguous step of each sequence
-        for i in range(r["batch"]):
-            n = np.argmin(ok[i]) if not ok[i].all() else r["n_decode"]
-            assert np.array_equal(toks[i, :n], ref[i, :n])
+        assert_bit_identical(base, v)
+
+
+FOLD_CFGS = [ModelConfig("tiny3g", 3, 256, 4, 1024, 512, 96, "gelu_tanh"),
+             ModelConfig("mid3", 3, 1024, 8, 4096, 1024, 96, "relu")]
+
+
+@pytest.mark.parametrize("cfg", FOLD_CFGS, ids=lambda c: c.name)
+@pytest.mark.parametrize("fold", ["1", "0"])
+def test_ln_fold_decode_matches_oracle(E, cfg, fold):
+    """The default t = 1 decode path -- LayerNorm folded into the QKV / FC1 GEMMs
+    (W*gamma weights, in-kernel row statistics, u / c epilogue vectors) and the
+    residual adds in the out-proj / FC2 epilogues -- and the unfolded path
+    (LIGER_LN_FOLD=0), at decode batches b = 1, 2, 8 and 16, element-wise against the
+    oracle.  h = 1024 exercises the split-K fixup epilogue, h = 256 the single-chunk one."""
+    trace = []
+    for i, b in enumerate((1, 2, 8, 16)):
+        trace += make_trace(1, float("inf"), seed=40 + i, batch_sizes=(b,), prompt_range=(20, 60), n_decode=6,
+                            vocab=cfg.vocab)
+    res = _with_env({"LIGER_LN_FOLD": fold}, lambda: serve(E, cfg, 1, trace, mode="interleaved", max_batch=16,
+                                                           max_seq=64, max_new=8, seed=7))
+    check_vs_oracle(cfg, 7, trace, res)
+
+
+def test_ln_fold_full_size_opt13b_layer(E):
+    """The bench's launch configuration at full width: an OPT-13B-shaped model cut to
+    one decoder layer (h = 5120, ffn 20480, vocab 50272, ReLU) served at t = 1 with the
+    default folded decode path (split-K QKV / FC1 with the folded LN, out-proj / FC2
+    fixups with the residual add), b = 2 and 8, element-wise against the oracle."""
+    cfg = ModelConfig("opt13b-L1", 1, 5120, 40, 20480, 50272, 64, "relu")
+    trace = (make_trace(1, float("inf"), seed=9, batch_sizes=(2,), prompt_range=(24, 24), n_decode=6,
+                        vocab=cfg.vocab) +
+             make_trace(1, float("inf"), seed=10, batch_sizes=(8,), prompt_range=(17, 17), n_decode=4,
+                        vocab=cfg.vocab))
+    res = serve(E, cfg, 1, trace, mode="interleaved", max_batch=8, max_seq=24, max_new=6, seed=1)
+    check_vs_oracle(cfg, 1, trace, res)
+
+
+@pytest.mark.parametrize("skip", ["fc2", "attn", "out"])
+def test_broken_layer_fails_the_check(E, skip):
+    """The checks can fail: a decoder-layer kernel skipped (LIGER_DBG_SKIP, a timing
+    experiment switch that leaves its output buffer stale) must break the
+    element-wise comparison with the oracle."""
+    cfg = get_config("tiny")
+    prompt = np.random.default_rng(0).integers(0, cfg.vocab, size=(2, 32)).astype(np.int32)
+    trace = [dict(tokens=prompt.reshape(-1), batch=2, seq_len=32, n_decode=8)]
+    res = _with_env({"LIGER_DBG_SKIP": skip},
+                    lambda: serve(E, cfg, 1, trace, mode="serial", max_batch=4, max_seq=64, max_new=8, seed=0))
+    with pytest.raises(AssertionError):
+        check_vs_oracle(cfg, 0, trace, res)
 
 
 def test_device_resident_tokens_and_latency_fields(E):
@@ -78,6 +134,29 @@ def test_device_resident_tokens_and_latency_fields(E):
     eng.drain()
     res, _ = eng.poll(bid)
     assert res.done == 1 and res.finish_s >= res.start_s >= res.submit_s > 0
+    eng.close()
+
+
+def test_result_tokens_device_states(E):
+    """liger_result_tokens_device: PENDING before the batch finished, the tokens after,
+    ESTATE once a later batch reused the slot."""
+    import ctypes as C
+    from paper_conf_ppopp_duwjchcl24_b200 import liger as L
+    cfg = get_config("tiny")
+    eng = E(cfg, mode="serial", max_batch=2, max_seq=16, max_new=4, seed=0)
+    p = np.random.default_rng(5).integers(0, cfg.vocab, size=2 * 16).astype(np.int32)
+    bid = eng.submit(p, 2, 16, 4, 0.0)
+    ptr = C.c_void_p()
+    assert L.lib().liger_result_tokens_device(eng.ctx, bid, C.byref(ptr)) == L.LIGER_PENDING
+    eng.drain()
+    assert L.lib().liger_result_tokens_device(eng.ctx, bid, C.byref(ptr)) == L.LIGER_OK
+    assert ptr.value
+    host = eng.poll(bid, want_tokens=True)[1]
+    for _ in range(3):   # serial mode: 2 slots -> the first one is reused
+        eng.submit(p, 2, 16, 4, 0.0)
+    eng.drain()
+    assert L.lib().liger_result_tokens_device(eng.ctx, bid, C.byref(ptr)) == L.LIGER_ESTATE
+    assert host.shape == (2, 4)
     eng.close()
 
 
@@ -105,101 +184,15 @@ def test_contention_factor_calibration(E):
 def test_nccl_oneshot_setup_and_kernel_single_rank(E):
     """The NCCL backend's one-shot path on real hardware at one rank: liger_calibrate_cf
     at t = 1 runs its all-reduces on a 1-rank NCCL communicator; with LIGER_ONESHOT_AR=1
-    that exercises the CUDA-IPC staging setup, the NCCL agreement on it and the
-    one-shot kernel (flags, staging, rank-ordered sum) -- with the GEMM SM reserve
-    on, so GEMM grids leave SMs to it."""
-    import os
+    its creation sets up the CUDA-IPC staging eagerly (with the NCCL agreement on it)
+    and the all-reduces run the one-shot kernel -- with the GEMM SM reserve on."""
     cfg = get_config("tiny")
-    os.environ["LIGER_ONESHOT_AR"] = "1"
-    try:
+
+    def run():
         eng = E(cfg, max_batch=2, max_seq=32, max_new=4, seed=0)
         eng.set_gemm_sm_reserve(16)
         cf, _ = eng.calibrate_cf([16, 64], set_cf=False)
-        toks_ok = True
-        prompt = np.random.default_rng(1).integers(0, cfg.vocab, size=(2, 16)).astype(np.int32)
-        bid = eng.submit(prompt.reshape(-1), 2, 16, 3, 0.0)
-        eng.drain()
-        res, toks = eng.poll(bid, want_tokens=True)
         eng.close()
-    finally:
-        os.environ.pop("LIGER_ONESHOT_AR", None)
+        return cf
+    cf = _with_env({"LIGER_ONESHOT_AR": "1"}, run)
     assert 1.0 <= cf < 10.0
-    assert res.done == 1 and toks.shape == (2, 3) and toks_ok
-
-
-_FOLD_CHILD = r"""
-import sys, numpy as np
-sys.path.insert(0, {root!r})
-from liger_inputs import make_trace, get_config
-from liger_inputs.configs import ModelConfig
-from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
-cfg = {cfg}
-trace = make_trace(3, float("inf"), seed=4, batch_sizes=(2, 5), prompt_range=(20, 60), n_decode=6, vocab=cfg.vocab)
-eng = LigerEngine(cfg, mode="interleaved", max_batch=8, max_seq=64, max_new=8, seed=7)
-ids = [eng.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], 0.0) for t in trace]
-eng.drain()
-print(repr([eng.poll(i, want_tokens=True)[1].tolist() for i in ids]))
-eng.close()
-"""
-
-
-@pytest.mark.parametrize("cfg_expr", ['ModelConfig("mid3", 3, 1024, 8, 4096, 1024, 96, "relu")',
-                                      'ModelConfig("tiny3g", 3, 256, 4, 1024, 512, 96, "gelu_tanh")'])
-def test_ln_fold_decode_matches_oracle(E, cfg_expr):
-    """t = 1 decode passes with LayerNorm folded into the QKV / FC1 GEMMs
-    (W*gamma weights, in-kernel row statistics, u / c epilogue vectors) and the
-    residual adds in the out-proj / FC2 epilogues -- default -- against the fp64
-    oracle's greedy tokens (where its top-2 margin is clear), and against the
-    unfolded path (LIGER_LN_FOLD=0).  h = 1024 exercises the split-K fixup path,
-    h = 256 the single-chunk epilogue path."""
-    import ast
-    import os
-    import subprocess
-    import sys
-    from liger_inputs.configs import ModelConfig
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    res = {}
-    for flag in ("1", "0"):
-        p = subprocess.run([sys.executable, "-c", _FOLD_CHILD.format(root=root, cfg=cfg_expr)],
-                           env={**os.environ, "LIGER_LN_FOLD": flag}, capture_output=True, text=True, timeout=600)
-        assert p.returncode == 0, p.stderr[-2000:]
-        res[flag] = ast.literal_eval(p.stdout.strip().splitlines()[-1])
-    cfg = eval(cfg_expr)
-    trace = make_trace(3, float("inf"), seed=4, batch_sizes=(2, 5), prompt_range=(20, 60), n_decode=6,
-                       vocab=cfg.vocab)
-    agree = total = 0
-    for t, got1, got0 in zip(trace, res["1"], res["0"]):
-        pr = t["tokens"].reshape(t["batch"], t["seq_len"])
-        ref, logits = om.greedy_generate(cfg, 7, pr, t["n_decode"], return_logits=True)
-        ok = om.top2_margin(logits) > 0.02 * np.sqrt((logits ** 2).mean())
-        for i in range(t["batch"]):
-            n = int(np.argmin(ok[i])) if not ok[i].all() else t["n_decode"]
-            assert np.array_equal(np.array(got1)[i, :n], ref[i, :n])
-            assert np.array_equal(np.array(got0)[i, :n], ref[i, :n])
-            agree += int(np.sum(np.array(got1)[i] == np.array(got0)[i]))
-            total += t["n_decode"]
-    assert agree >= 0.9 * total
-
-
-def test_ln_fold_full_size_opt13b_layer_tokens(E):
-    """The bench's launch configuration at full size: an OPT-13B-shaped model cut to one
-    decoder layer (h = 5120, ffn 20480, vocab 50272, ReLU) served at t = 1 -- decode
-    passes with the LayerNorms folded into the split-K QKV / FC1 GEMMs and the
-    residual adds in the out-proj / FC2 fixups (plans 1 / 3 / 10 / 7 chunks) -- gives
-    the fp64 oracle's greedy tokens wherever the oracle's top-2 margin is clear."""
-    from liger_inputs.configs import ModelConfig
-    cfg = ModelConfig("opt13b-L1", 1, 5120, 40, 20480, 50272, 64, "relu")
-    prompt = np.random.default_rng(9).integers(0, cfg.vocab, size=(2, 24))
-    eng = E(cfg, mode="interleaved", max_batch=2, max_seq=24, max_new=6, seed=1)
-    bid = eng.submit(prompt.reshape(-1).astype(np.int32), 2, 24, 6, 0.0)
-    eng.drain()
-    _, toks = eng.poll(bid, want_tokens=True)
-    eng.close()
-    ref, logits = om.greedy_generate(cfg, 1, prompt, 6, return_logits=True)
-    ok = om.top2_margin(logits) > 0.02 * np.sqrt((logits ** 2).mean())
-    checked = 0
-    for i in range(2):
-        n = int(np.argmin(ok[i])) if not ok[i].all() else 6
-        assert np.array_equal(toks[i, :n], ref[i, :n]), (toks, ref)
-        checked += n
-    assert checked >= 4
