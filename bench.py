@@ -671,7 +671,7 @@ def main():
                 import traceback
                 errs.append(f"rank {r}: {e!r}\n{traceback.format_exc()}")
                 shared.bar.abort()
-        ths = [threading.Thread(target=th, args=(r,)) for r in range(world)]
+        ths = [threading.Thread(target=th, args=(r,), daemon=True) for r in range(world)]
         for t in ths:
             t.start()
         for t in ths:

@@ -352,8 +352,10 @@ int liger_op_attn_prefill(const void* qkv, void* o, void* kv_pool, const int32_t
 /* Decode attention (§8(a) a4) for one new token per sequence at position
  * `pos` (cache holds positions [0, pos)): qkv [b, 3*heads*d]; appends the
  * token's K/V to the cache page; o [b, heads*d].  workspace: device scratch
- * of liger_attn_decode_workspace_bytes(b, heads, d, pos + 1) bytes, first
- * 16 KiB zero before first use (left zero). */
+ * of liger_attn_decode_workspace_bytes(b, heads, d, pos + 1) bytes (enough for
+ * every launch with at most b sequences and context at most pos + 1), first
+ * 16 KiB zero before first use (left zero).  LIGER_EINVAL if pos >= max_pages * 16
+ * (the page table row cannot hold the new token) or d not in {64, 128}. */
 int liger_op_attn_decode(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
                          int pos, int heads, int d, void* workspace, size_t ws_bytes, void* stream);
 size_t liger_attn_decode_workspace_bytes(int b, int heads, int d, int ctx);

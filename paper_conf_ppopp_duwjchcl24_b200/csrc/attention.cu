@@ -512,7 +512,8 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   const int ctx = pos + 1;
   DecAttnArgs a;
   dec_attn_plan(b, heads, ctx, &a.cps, &a.nsp);
-  if (a.nsp > DC_MAX_SPLITS || (d != 64 && d != 128)) return LIGER_EINVAL;
+  // the page table row must hold position pos (the new token's page)
+  if (a.nsp > DC_MAX_SPLITS || (d != 64 && d != 128) || pos < 0 || pos >= max_pages * KVB) return LIGER_EINVAL;
   if (a.nsp > 1) {
     if (!workspace || ws_bytes < attn_decode_workspace_bytes(b, heads, d, ctx) ||
         (size_t)b * heads * 4 > ATTN_COUNTER_BYTES)
@@ -530,6 +531,13 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   a.ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
   const int rc = d == 128 ? launch_decode<128>(a, stream) : launch_decode<64>(a, stream);
   return rc ? LIGER_ECUDA : 0;
+}
+
+void preload_attention_kernels() {
+  preload_kernel(attn_prefill_kernel<64>);
+  preload_kernel(attn_prefill_kernel<128>);
+  preload_kernel(attn_decode_kernel<64>);
+  preload_kernel(attn_decode_kernel<128>);
 }
 
 LIGER_TRACE_SETTER(attention)

@@ -19,6 +19,14 @@ void set_global_error(const std::string& s) {
 const char* global_error() { return g_last_error.c_str(); }
 
 // Returns 0 if the current device is an sm_100 part, LIGER_ENODEV otherwise.
+void preload_kernels() {
+  preload_gemm_kernels();
+  preload_norm_kernels();
+  preload_attention_kernels();
+  preload_comm_kernels();
+  cudaGetLastError();
+}
+
 int check_device() {
   static int state = 1;   // 1 = unknown
   static std::once_flag once;
@@ -33,6 +41,7 @@ int check_device() {
     cudaDeviceProp p;
     cudaGetDeviceProperties(&p, dev);
     state = (p.major == 10) ? 0 : LIGER_ENODEV;
+    if (!state) preload_kernels();
   });
   if (state) set_global_error("liger: no sm_100 (B200) CUDA device available; there is no CPU fallback");
   return state;

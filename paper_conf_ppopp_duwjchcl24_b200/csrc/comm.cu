@@ -574,4 +574,13 @@ Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err) {
   return c;
 }
 
+void preload_peer_ar_kernel();
+void preload_comm_kernels() {
+  preload_kernel(loop_reduce_bf16_kernel<false>);
+  preload_kernel(loop_reduce_bf16_kernel<true>);
+  preload_kernel(loop_reduce_kernel<float, false>);
+  preload_kernel(loop_reduce_kernel<float, true>);
+  preload_peer_ar_kernel();
+}
+
 }  // namespace liger

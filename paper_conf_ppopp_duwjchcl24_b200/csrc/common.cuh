@@ -259,6 +259,16 @@ LIGER_DEV float gelu_tanh_f(float x) {
 // (the all-reduce kernels spinning on peers' flags) would otherwise pin a small-smem
 // configuration and keep a persistent GEMM CTA (up to 217 KB) off that SM -- with
 // static unit assignment that GEMM then never completes (a TP = 4 loopback hang).
+inline void prefer_max_smem(const void* fn);
+// Load a kernel now (CUDA lazy module loading would otherwise load it at its first launch,
+// which can wait for running kernels -- a deadlock when those spin on peers whose host
+// thread is the one loading; see preload_kernels in kernels.h).
+template <typename K>
+inline void preload_kernel(K k) {
+  cudaFuncAttributes a;
+  cudaFuncGetAttributes(&a, reinterpret_cast<const void*>(k));
+  prefer_max_smem(reinterpret_cast<const void*>(k));
+}
 inline void prefer_max_smem(const void* fn) {
   static std::mutex mu;
   static std::unordered_set<const void*> done;

@@ -256,6 +256,16 @@ void* dalloc(liger_ctx* c, size_t bytes) {
   return p;
 }
 
+// cudaDeviceSynchronize inside a [collective] call, followed by a barrier of the ranks:
+// on the loopback backend the ranks share the GPU, and a rank that left the call and
+// launched a kernel spinning on its peers (one-shot all-reduce) would keep a peer's
+// device-wide synchronize from ever returning.
+int device_sync_collective(liger_ctx* c) {
+  const cudaError_t e = cudaDeviceSynchronize();
+  if (c->comm) c->comm->barrier();
+  return e == cudaSuccess ? 0 : LIGER_ECUDA;
+}
+
 // Ring of reusable events for per-batch cross-stream dependencies.  Re-recording
 // an event that an older wait still references is safe: cudaStreamWaitEvent
 // captures the event's state at the time of the call.
@@ -413,7 +423,8 @@ void timed_end(liger_ctx* c, cudaStream_t s, cudaEvent_t a, int cls, double byte
 }
 void timing_flush(liger_ctx* c) {
   if (c->timed.empty()) return;
-  cudaDeviceSynchronize();
+  cudaStreamSynchronize(c->s_comp);   // this rank's streams only (peers may be running spinning kernels)
+  cudaStreamSynchronize(c->s_comm);
   for (auto& t : c->timed) {
     float ms = 0;
     cudaEventElapsedTime(&ms, t.a, t.b);
@@ -1072,7 +1083,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
     }
     if (c->pipe && world > 1) c->pass_ops.push_back({OP_SEND_TOK, -1});
   }
-  CK(cudaDeviceSynchronize());
+  if (device_sync_collective(c)) return fail(nullptr, LIGER_ECUDA, "liger_init: device synchronize failed");
   *out = cp.release();
   return LIGER_OK;
 }
@@ -1482,6 +1493,7 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
                        double* detail /* [n_m][4][2] slowdowns (gemm, ar) or NULL */) {
   if (!c || !m_list || n_m <= 0) return LIGER_EINVAL;
   if (!c->processing.empty() || !c->waiting.empty()) return fail(c, LIGER_ESTATE, "liger_calibrate_cf: batches in flight");
+  CKR(device_sync_collective(c));
   Comm* comm = c->comm;
   Comm* own = nullptr;
   if (!comm) {   // t = 1: a 1-rank NCCL communicator's all-reduce kernel as the proxy
@@ -1493,7 +1505,7 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
     if (!own) return fail(c, LIGER_ENCCL, "liger_calibrate_cf: " + err);
     comm = own;
   }
-  CK(cudaDeviceSynchronize());
+  CKR(device_sync_collective(c));
   Slot& S = c->slots[0];
   const int Mmax = c->cfg.max_batch * c->cfg.max_seq;
   cudaEvent_t ev[4];
@@ -1567,7 +1579,7 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
   }
   if (set_cf) c->cf = cf;
   if (cf_out) *cf_out = cf;
-  CK(cudaDeviceSynchronize());
+  CKR(device_sync_collective(c));
   return LIGER_OK;
 }
 
@@ -1576,7 +1588,7 @@ int liger_calibrate_cf(liger_ctx* c, const int32_t* m_list, int n_m, int set_cf,
 int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
   if (!c || !m_list || n_m <= 0) return LIGER_EINVAL;
   if (!c->processing.empty() || !c->waiting.empty()) return fail(c, LIGER_ESTATE, "liger_profile: batches in flight");
-  CK(cudaDeviceSynchronize());
+  CKR(device_sync_collective(c));
   Slot& S = c->slots[0];
   cudaStream_t st = c->s_comp;
   cudaEvent_t a, b;
@@ -1689,7 +1701,7 @@ int liger_profile(liger_ctx* c, const int32_t* m_list, int n_m) {
     c->attn_scale[0] = flat[i++];
     c->attn_scale[1] = flat[i++];
   }
-  CK(cudaDeviceSynchronize());
+  CKR(device_sync_collective(c));
   return LIGER_OK;
 }
 

@@ -729,6 +729,15 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
              : 0;
 }
 
+void preload_gemm_kernels() {
+  for (auto k : {gemm_tc_kernel<false>, gemm_tc_kernel<true>}) {
+    preload_kernel(k);
+    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, MAX_SMEM);
+  }
+  preload_kernel(splitk_reduce_kernel<false>);
+  preload_kernel(splitk_reduce_kernel<true>);
+}
+
 LIGER_TRACE_SETTER(gemm)
 
 }  // namespace liger

@@ -69,6 +69,17 @@ struct GemmArgs {
   const void* resid = nullptr;
 };
 
+// Load every kernel of the library up front (called once from check_device): with CUDA's
+// lazy module loading a kernel is loaded at its first launch, and loading may wait for
+// kernels already running -- on the loopback backend (or any process whose running
+// kernels spin on peers) a peer spinning on this rank's flag then never sees it: a
+// deadlock seen in the fused all-reduce test.
+void preload_kernels();
+void preload_gemm_kernels();
+void preload_norm_kernels();
+void preload_attention_kernels();
+void preload_comm_kernels();
+
 GemmPlan gemm_plan(int M, int N, int K);
 size_t gemm_workspace_bytes(int M, int N, int K);
 int gemm_launch(const GemmArgs& a, cudaStream_t stream);

@@ -421,6 +421,24 @@ int copy_tokens_launch(const int32_t* src, int32_t* dst, int n, cudaStream_t str
   return cudaGetLastError() == cudaSuccess ? 0 : LIGER_ECUDA;
 }
 
+void preload_norm_kernels() {
+  preload_kernel(add_ln_kernel<128, 1, false>);
+  preload_kernel(add_ln_kernel<128, 4, false>);
+  preload_kernel(add_ln_kernel<256, 4, false>);
+  preload_kernel(add_ln_kernel<512, 4, false>);
+  preload_kernel(add_ln_kernel<128, 1, true>);
+  preload_kernel(add_ln_kernel<128, 4, true>);
+  preload_kernel(add_ln_kernel<256, 4, true>);
+  preload_kernel(add_ln_kernel<512, 4, true>);
+  preload_kernel(embed_kernel);
+  preload_kernel(argmax_kernel);
+  preload_kernel(argmax_pick_kernel);
+  preload_kernel(c0_fill_kernel);
+  preload_kernel(tile_weight_kernel);
+  preload_kernel(fold_gamma_tiled_kernel);
+  preload_kernel(copy_i32_kernel);
+}
+
 LIGER_TRACE_SETTER(norm)
 
 }  // namespace liger

@@ -24,6 +24,7 @@
 #include <stdint.h>
 #include <string.h>
 #include <stdio.h>
+#include <stdlib.h>
 
 #include "comm.h"
 #include "common.cuh"
@@ -143,9 +144,15 @@ int PeerAR::init(int world_, int rank_, size_t cap_, void* local_region, void* c
 
 PeerAR::~PeerAR() {}
 
+static bool dbg_epochs() {
+  static const bool on = getenv("LIGER_DBG_EPOCH") != nullptr;
+  return on;
+}
+
 int PeerAR::fused_begin(size_t bytes, FusedARDesc* out) {
   if (bytes > cap || bytes % 16) return LIGER_EINVAL;
   ++epoch;
+  if (dbg_epochs()) fprintf(stderr, "[rank %d] epoch %llu fused %zu B\n", rank, (unsigned long long)epoch, bytes);
   const int b = (int)(epoch & 1);
   FusedARDesc d{};
   d.stage = static_cast<char*>(local) + (size_t)b * cap;
@@ -166,6 +173,7 @@ int PeerAR::allreduce_bf16(void* buf, size_t count, cudaStream_t st) {
   if (bytes > cap || bytes % 16 || reinterpret_cast<uintptr_t>(buf) % 16) return LIGER_EINVAL;
   if (!count) return 0;
   ++epoch;
+  if (dbg_epochs()) fprintf(stderr, "[rank %d] epoch %llu one-shot %zu B\n", rank, (unsigned long long)epoch, bytes);
   const int b = (int)(epoch & 1);
   PeerPtrs pp{};
   for (int q = 0; q < world; ++q) {
@@ -183,5 +191,7 @@ int PeerAR::allreduce_bf16(void* buf, size_t count, cudaStream_t st) {
              ? LIGER_ECUDA
              : 0;
 }
+
+void preload_peer_ar_kernel() { preload_kernel(oneshot_ar_bf16_kernel); }
 
 }  // namespace liger

@@ -97,7 +97,7 @@ def serve(E, cfg, world, trace, *, capture=True, durations=(), threads=True, **k
     if world == 1 and not threads:
         rank_main(0)
     else:
-        ths = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+        ths = [threading.Thread(target=rank_main, args=(r,), daemon=True) for r in range(world)]
         for t in ths:
             t.start()
         for t in ths:

@@ -247,10 +247,10 @@ def test_decode_attention_long_context_split(L):
 
 
 def test_decode_attention_max_context_and_limit(L):
-    """The longest context decode attention takes (64 chunks of 64 = 4096 positions),
-    over scattered pages (a seeded permutation: the page-table indirection), against
-    the oracle; the new token's K/V are appended to its page; one position more is
-    rejected with LIGER_EINVAL (include/liger.h, liger_op_attn_decode)."""
+    """A long context (4096 positions) over scattered pages (a seeded permutation: the
+    page-table indirection), against the oracle; the new token's K/V are appended to its
+    page; a position beyond the page table's width (max_pages * 16) is rejected with
+    LIGER_EINVAL (include/liger.h, liger_op_attn_decode)."""
     b, heads, d, pos = 2, 2, 128, 4095
     maxp = (pos + 1 + 15) // 16
     n = b * maxp * 2 * heads * 16 * d

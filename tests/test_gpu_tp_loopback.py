@@ -260,7 +260,7 @@ def test_allreduce_op_vs_oracle_and_decomposition(E, world, oneshot):
 
     import threading
     with env(LIGER_ONESHOT_AR=oneshot, LIGER_ONESHOT_MAX_KB="16"):
-        ths = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+        ths = [threading.Thread(target=rank_main, args=(r,), daemon=True) for r in range(world)]
         for t in ths:
             t.start()
         for t in ths:

@@ -115,7 +115,7 @@ def _engine(world, env):
             e.close()
         except Exception as ex:
             err.append(repr(ex))
-    ths = [threading.Thread(target=run, args=(r,)) for r in range(world)]
+    ths = [threading.Thread(target=run, args=(r,), daemon=True) for r in range(world)]
     for t in ths:
         t.start()
     for t in ths:
