@@ -65,6 +65,7 @@ def build_oracle(out_dir=None, verbose=False):
     the ctypes library `liblayer_ref.so` for its pin test.  -march=native: build it on
     the host that runs it (bench.py compiles its own copy on the GPU box's host)."""
     out_dir = out_dir or os.path.join(HERE, "..", "oracle")
+    os.makedirs(out_dir, exist_ok=True)
     exe = os.path.join(out_dir, "layer_ref")
     so = os.path.join(out_dir, "liblayer_ref.so")
     base = ["g++", "-O3", "-march=native", "-fopenmp", "-std=c++17", ORACLE_SRC]

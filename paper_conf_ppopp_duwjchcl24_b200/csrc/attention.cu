@@ -286,85 +286,107 @@ struct DecSmem {
   float st_acc[4 * (32 / (D / 8))][D];     // per lane group: acc (item merge)
   float st_m[4 * (32 / (D / 8))], st_l[4 * (32 / (D / 8))];
   float mw[DC_MAX_SPLITS], lw[DC_MAX_SPLITS];
-  uint64_t full[DC_NS];
+  uint64_t full[DC_NS], empty[DC_NS];
   int last;
 };
 
+// Warps 0..3 compute, warp 4 (lane 0) is the producer: it walks the same task list
+// (chunk j of item i = blockIdx.x + k G) and keeps DC_NS chunks in flight, refilling a
+// stage as soon as the four compute warps have released it (empty[s]).
 template <int D>
-__global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const DecAttnArgs a) {
+__global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecAttnArgs a) {
   constexpr int LPT = D / 8;          // lanes per token row (16 B each)
   constexpr int TPW = 32 / LPT;       // token rows per warp step
   constexpr int NG = 4 * TPW;         // lane groups per CTA
+  constexpr int PPG = DC_CH / NG;     // positions per lane group per chunk
   const uint64_t tr0 = trace_now();
   extern __shared__ __align__(128) uint8_t dsm[];
   DecSmem<D>& sm = *reinterpret_cast<DecSmem<D>*>(dsm);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int grp = warp * TPW + lane / LPT;   // lane group 0..NG-1
-  const int gl = lane % LPT;                 // lane within the group: dims [8 gl, 8 gl + 8)
   const int G = gridDim.x;
   const int pos = a.pos, ctx = pos + 1, heads = a.heads, nsp = a.nsp, cps = a.cps;
   const int nch = (ctx + DC_CH - 1) / DC_CH;
   const int n_items = a.b * heads * nsp;
-  // task t of this CTA = chunk j of its i-th item; items i = blockIdx.x + k G
   auto item_chunks = [&](int it, int* c0) {
-    const int sp = it % nsp;
-    *c0 = sp * cps;
+    *c0 = (it % nsp) * cps;
     return max(0, min(nch, *c0 + cps) - *c0);
   };
   if (tid == 0) {
-    for (int s = 0; s < DC_NS; ++s) mbar_init(&sm.full[s], 1);
+    for (int s = 0; s < DC_NS; ++s) {
+      mbar_init(&sm.full[s], 1);
+      mbar_init(&sm.empty[s], 4);   // one arrive per compute warp
+    }
     fence_barrier_init();
   }
   __syncthreads();
-  // producer state (thread 0): next task to issue
-  int p_it = blockIdx.x, p_j = 0, issued = 0;
-  auto issue_next = [&]() {   // thread 0: stage the next task (if any) into ring slot issued % NS
-    while (p_it < n_items) {
+  if (warp == 4) {
+    // ---------------- producer warp: the page ids of up to 32 pages are fetched in one
+    // parallel load (no serial page-table round trips on the refill path); lane 0
+    // paces the ring, lanes 0 / 1 issue the two pages of a chunk
+    int k = 0;
+    bool waited = false;
+    for (int it = blockIdx.x; it < n_items; it += G) {
       int c0;
-      const int nc = item_chunks(p_it, &c0);
-      if (p_j < nc) break;
-      p_it += G;
-      p_j = 0;
+      const int nc = item_chunks(it, &c0);
+      const int bh = it / nsp, bi = bh / heads, head = bh % heads;
+      const int32_t* pt = a.page_table + (int64_t)bi * a.max_pages + c0 * (DC_CH / KVB);
+      const int npages_item = (min(ctx, (c0 + nc) * DC_CH) - c0 * DC_CH + KVB - 1) / KVB;
+      for (int j0 = 0; j0 < nc; j0 += 32 / (DC_CH / KVB)) {
+        const int pg0 = j0 * (DC_CH / KVB);
+        const int my_page = (pg0 + lane < npages_item) ? pt[pg0 + lane] : 0;
+        for (int j = j0; j < min(nc, j0 + 32 / (DC_CH / KVB)); ++j, ++k) {
+          const int s = k % DC_NS;
+          const int t0 = (c0 + j) * DC_CH;
+          const int tc1 = min(t0 + DC_CH, pos);                       // cached positions [t0, tc1)
+          const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
+          if (lane == 0) {
+            if (k >= DC_NS) mbar_wait(&sm.empty[s], (uint32_t)((k / DC_NS) - 1) & 1u);
+            mbar_arrive_expect_tx(&sm.full[s], (uint32_t)npg * 2 * KVB * D * 2);
+          }
+          __syncwarp();
+          const int page = __shfl_sync(0xffffffffu, my_page, ((j - j0) * (DC_CH / KVB) + lane) & 31);
+          if (lane < npg) {
+            bulk_load(&sm.kv[s][0][lane * KVB * D], a.kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2,
+                      &sm.full[s]);
+            bulk_load(&sm.kv[s][1][lane * KVB * D], a.kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2,
+                      &sm.full[s]);
+          }
+          // The cached positions were written by earlier passes and the page table at
+          // admission: the first stages are requested before the PDL wait.
+          if (k == DC_NS - 1) {
+            grid_dependency_wait();
+            waited = true;
+          }
+        }
+      }
     }
-    const int s = issued % DC_NS;
-    if (p_it >= n_items) {   // nothing left: complete the stage's phase with no bytes
-      mbar_arrive(&sm.full[s]);
-      ++issued;
-      return;
-    }
-    int c0;
-    item_chunks(p_it, &c0);
-    const int bh = p_it / nsp, bi = bh / heads, head = bh % heads;
-    const int t0 = (c0 + p_j) * DC_CH;
-    const int tc1 = min(t0 + DC_CH, pos);                       // cached positions [t0, tc1)
-    const int npg = tc1 > t0 ? (tc1 - t0 + KVB - 1) / KVB : 0;
-    const int32_t* pt = a.page_table + (int64_t)bi * a.max_pages + (t0 >> 4);
-    mbar_arrive_expect_tx(&sm.full[s], (uint32_t)npg * 2 * KVB * D * 2);
-    for (int g = 0; g < npg; ++g) {
-      const int page = pt[g];
-      bulk_load(&sm.kv[s][0][g * KVB * D], a.kv_pool + kv_off(page, 0, heads, head, 0, D), KVB * D * 2, &sm.full[s]);
-      bulk_load(&sm.kv[s][1][g * KVB * D], a.kv_pool + kv_off(page, 1, heads, head, 0, D), KVB * D * 2, &sm.full[s]);
-    }
-    ++p_j;
-    ++issued;
-  };
-  // The cached positions were written by earlier passes and the page table at
-  // admission: the first NS stages are requested before the PDL wait.
-  if (tid == 0)
-    for (int s = 0; s < DC_NS; ++s) issue_next();
+    if (!waited) grid_dependency_wait();
+    grid_dependency_trigger();   // after the wait ("trigger after wait", common.cuh)
+    return;
+  }
+  // ---------------- compute warps 0..3
+  const int grp = warp * TPW + lane / LPT;   // lane group 0..NG-1
+  const int gl = lane % LPT;                 // lane within the group: dims [8 gl, 8 gl + 8)
   pdl_enter();   // q and the new token's k / v come from the QKV kernel
   const uint64_t tr1 = trace_now();
   const int64_t ld = (int64_t)3 * heads * D;
-  int consumed = 0;
+  int k = 0;
   bool merged_any = false;
+  // q of the CTA's next item is loaded one item ahead (its latency hides behind the ring)
+  auto load_q = [&](int it) {
+    const int bh = it / nsp, bi = bh / heads, head = bh % heads;
+    return __ldcg(reinterpret_cast<const uint4*>(a.qkv + (int64_t)bi * ld + head * D + gl * 8));
+  };
+  uint4 q_next = blockIdx.x < n_items ? load_q(blockIdx.x) : make_uint4(0, 0, 0, 0);
   for (int it = blockIdx.x; it < n_items; it += G) {
     int c0;
     const int nc = item_chunks(it, &c0);
     const int sp = it % nsp, bh = it / nsp, bi = bh / heads, head = bh % heads;
     const __nv_bfloat16* row = a.qkv + (int64_t)bi * ld;
     float q[8], kn[8], vn[8];
-    bf16x8_to_f32(__ldcg(reinterpret_cast<const uint4*>(row + head * D + gl * 8)), q);
-    const bool has_new = nc > 0 && (c0 + nc) * DC_CH > pos && c0 * DC_CH <= pos;
+    bf16x8_to_f32(q_next, q);
+    if (it + G < n_items) q_next = load_q(it + G);
+    const bool has_new = (c0 + nc) * DC_CH > pos && c0 * DC_CH <= pos;
     if (has_new) {   // the new token (position pos): from the QKV output, appended to its page
       const uint4 kv4 = __ldcg(reinterpret_cast<const uint4*>(row + (int64_t)heads * D + head * D + gl * 8));
       const uint4 vv4 = __ldcg(reinterpret_cast<const uint4*>(row + (int64_t)2 * heads * D + head * D + gl * 8));
@@ -377,43 +399,61 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const DecAttnAr
       }
     }
     float m = -INFINITY, l = 0.f, acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    for (int j = 0; j < nc; ++j, ++consumed) {
-      const int s = consumed % DC_NS;
-      mbar_wait(&sm.full[s], (uint32_t)(consumed / DC_NS) & 1u);
+    for (int j = 0; j < nc; ++j, ++k) {
+      const int s = k % DC_NS;
+      mbar_wait(&sm.full[s], (uint32_t)(k / DC_NS) & 1u);
       const int t0 = (c0 + j) * DC_CH;
       const __nv_bfloat16* sK = sm.kv[s][0];
       const __nv_bfloat16* sV = sm.kv[s][1];
+      // scores of this lane group's PPG positions (independent chains), then one
+      // online-softmax update for all of them
+      float sc[PPG], vf[PPG][8];
 #pragma unroll
-      for (int r = 0; r < DC_CH / NG; ++r) {
-        const int lt = r * NG + grp;           // local position of this lane group
+      for (int r = 0; r < PPG; ++r) {
+        const int lt = r * NG + grp;
         const int t = t0 + lt;
-        float kf[8], vf[8];
+        float kf[8];
         if (t < pos) {
           bf16x8_to_f32(*reinterpret_cast<const uint4*>(sK + lt * D + gl * 8), kf);
-          bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + gl * 8), vf);
+          bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + gl * 8), vf[r]);
         } else {
 #pragma unroll
           for (int e = 0; e < 8; ++e) {
             kf[e] = kn[e];
-            vf[e] = vn[e];
+            vf[r][e] = vn[e];
           }
         }
         float dot = 0.f;
 #pragma unroll
         for (int e = 0; e < 8; ++e) dot += q[e] * kf[e];
-#pragma unroll
-        for (int off = LPT / 2; off > 0; off >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, off);
-        if (t <= pos) {   // group-uniform
-          const float mn = fmaxf(m, dot);
-          const float sc = __expf(m - mn), p = __expf(dot - mn);
-          l = l * sc + p;
-#pragma unroll
-          for (int e = 0; e < 8; ++e) acc[e] = acc[e] * sc + p * vf[e];
-          m = mn;
-        }
+        sc[r] = dot;
       }
-      __syncthreads();   // every warp is done with stage s
-      if (tid == 0) issue_next();
+#pragma unroll
+      for (int off = LPT / 2; off > 0; off >>= 1)
+#pragma unroll
+        for (int r = 0; r < PPG; ++r) sc[r] += __shfl_xor_sync(0xffffffffu, sc[r], off);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sm.empty[s]);   // this warp is done with stage s (values in registers)
+      float mn = m;
+#pragma unroll
+      for (int r = 0; r < PPG; ++r)
+        if (t0 + r * NG + grp <= pos) mn = fmaxf(mn, sc[r]);
+      if (mn != -INFINITY) {   // group-uniform: at least one valid position so far
+        const float scale = __expf(m - mn);
+        l *= scale;
+#pragma unroll
+        for (int e = 0; e < 8; ++e) acc[e] *= scale;
+#pragma unroll
+        for (int r = 0; r < PPG; ++r) {
+          if (t0 + r * NG + grp <= pos) {
+            const float p = __expf(sc[r] - mn);
+            l += p;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) acc[e] += p * vf[r][e];
+          }
+        }
+        m = mn;
+      }
     }
     // ---- merge the lane groups' states (fixed order), then the item's result
     if (gl == 0) {
@@ -422,7 +462,7 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const DecAttnAr
     }
 #pragma unroll
     for (int e = 0; e < 8; ++e) sm.st_acc[grp][gl * 8 + e] = acc[e];
-    __syncthreads();
+    named_bar_sync(1, DC_THREADS);
     float M = -INFINITY;
 #pragma unroll
     for (int g = 0; g < NG; ++g) M = fmaxf(M, sm.st_m[g]);
@@ -437,7 +477,7 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const DecAttnAr
         for (int g = 0; g < NG; ++g) v += sm.st_m[g] == -INFINITY ? 0.f : sm.st_acc[g][e] * __expf(sm.st_m[g] - M);
         a.o[(int64_t)bi * heads * D + head * D + e] = __float2bfloat16_rn(v / L);
       }
-      __syncthreads();
+      named_bar_sync(1, DC_THREADS);
       continue;
     }
     float* wp = a.ws + (unit * nsp + sp) * (D + 2);
@@ -451,21 +491,21 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const DecAttnAr
       wp[D] = M;
       wp[D + 1] = L;
     }
-    __threadfence();
-    __syncthreads();
+    named_bar_sync(1, DC_THREADS);   // the CTA's partial is written (CTA scope) ...
     if (tid == 0) {
+      __threadfence();               // ... and made visible device-wide by one cumulative fence
       int prev;
       asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(prev) : "l"(&a.counters[unit]) : "memory");
       sm.last = (prev == nsp - 1);
     }
-    __syncthreads();
+    named_bar_sync(1, DC_THREADS);
     if (sm.last) {   // the last split of (sequence, head): merge the splits in split order
       for (int z = tid; z < nsp; z += DC_THREADS) {
         const float* w2 = a.ws + (unit * nsp + z) * (D + 2);
         sm.mw[z] = __ldcg(&w2[D]);
         sm.lw[z] = __ldcg(&w2[D + 1]);
       }
-      __syncthreads();
+      named_bar_sync(1, DC_THREADS);
       float MM = -INFINITY;
       for (int z = 0; z < nsp; ++z) MM = fmaxf(MM, sm.mw[z]);
       float LL = 0.f;
@@ -485,11 +525,8 @@ __global__ void __launch_bounds__(DC_THREADS) attn_decode_kernel(const DecAttnAr
       if (tid == 0) a.counters[unit] = 0;
       merged_any = true;
     }
-    __syncthreads();
+    named_bar_sync(1, DC_THREADS);
   }
-  // drain the ring: the stages issued beyond the last consumed task (arrive-only or
-  // loads that were never needed) must complete before the CTA exits
-  for (; consumed < issued; ++consumed) mbar_wait(&sm.full[consumed % DC_NS], (uint32_t)(consumed / DC_NS) & 1u);
   if (tid == 0) trace_write(merged_any ? (TK_ATTN_DEC | 0x100) : TK_ATTN_DEC, tr0, tr1);
 }
 
@@ -503,7 +540,7 @@ static int launch_decode(const DecAttnArgs& a, cudaStream_t stream) {
   }
   const int items = a.b * a.heads * a.nsp;
   const int grid = std::min(items, 148 * DC_CTAS_PER_SM);
-  return launch_pdl(attn_decode_kernel<D>, dim3(grid), dim3(DC_THREADS), dsmem, stream, a);
+  return launch_pdl(attn_decode_kernel<D>, dim3(grid), dim3(DC_THREADS + 32), dsmem, stream, a);
 }
 
 int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,

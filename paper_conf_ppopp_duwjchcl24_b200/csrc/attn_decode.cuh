@@ -6,7 +6,7 @@
 // HBM-bound: every cached K and V byte is read once.  Design (B200, 148 SMs):
 //  * work = (sequence, head, split); a split is a run of 32-position chunks (two
 //    16-token pages of K and of V, 4 x 4 KiB at d = 128); the split count is chosen
-//    per launch so that there are ~2 items per CTA slot;
+//    per launch so that there is ~1 item per CTA slot;
 //  * a persistent grid of up to 3 CTAs per SM walks its items' chunks as one task
 //    stream through an NS-stage shared-memory ring filled by cp.async.bulk (the TMA
 //    bulk engine) on per-stage mbarriers: NS x 16 KiB in flight per CTA, ~192 KiB per
@@ -66,14 +66,17 @@ struct DecAttnArgs {
   int* counters;              // [b * heads], zero between uses
 };
 
-// Split plan of a launch: chunks per split and the split count.  Items (sequence,
-// head, split) ~ 2 per CTA slot of a full persistent grid.
+// Split plan of a launch: chunks per split and the split count.  Each CTA slot of a
+// full persistent grid gets about one item (an item's fixed costs -- q load, lane-group
+// merge, split partial + merge -- are paid once per CTA): (sequence, head) pairs are
+// split only while there are fewer items than slots, never below one chunk per split.
 inline void dec_attn_plan(int b, int heads, int ctx, int* cps, int* nsp) {
   const int nch = (ctx + DC_CH - 1) / DC_CH;
   const int slots = 148 * DC_CTAS_PER_SM;
-  const int want = (2 * slots + b * heads - 1) / (b * heads);     // splits per (sequence, head)
+  int want = slots / (b * heads);
+  if (want < 1) want = 1;
+  if (want > nch) want = nch;
   int c = (nch + want - 1) / want;
-  if (c < 1) c = 1;
   while ((nch + c - 1) / c > DC_MAX_SPLITS) ++c;
   *cps = c;
   *nsp = (nch + c - 1) / c;
