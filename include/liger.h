@@ -193,6 +193,24 @@ int liger_result_tokens_device(liger_ctx* ctx, int64_t id, const int32_t** dev_t
  * context's communication stream).  A no-op at world == 1.  [collective] */
 int liger_op_allreduce(liger_ctx* ctx, void* buf, size_t count, int u0, int u1, int F, void* stream);
 
+/* CUDA-IPC peer regions and the one-shot all-reduce kernel on them (§8(a) a6/a10 decode
+ * transport; what the NCCL backend sets up with LIGER_ONESHOT_AR=1, exposed so that the
+ * transport can be tested across processes with any bootstrap).  A region holds
+ * [2 staging buffers of cap bytes][epoch flag][counters] (zeroed at creation);
+ * liger_ipc_region_create allocates one on the current device and writes its 64-byte
+ * cudaIpcMemHandle to `handle`; liger_ipc_region_open maps a peer process's region.
+ * liger_op_oneshot_allreduce: in-place bf16 sum of buf[count] over `world` ranks whose
+ * regions are regions[0..world) (regions[rank] = this rank's own), call number `epoch`
+ * (1, 2, ... in the same order on every rank): stage, publish the epoch (system-scope
+ * release), wait for every peer's flag (10 s watchdog trap), sum in rank order in fp32,
+ * round to bf16.  count * 2 <= cap, 16-byte multiples.  LIGER_EINVAL / LIGER_ECUDA. */
+int liger_ipc_region_create(size_t cap, void** region, uint8_t* handle);
+int liger_ipc_region_open(const uint8_t* handle, void** peer);
+int liger_ipc_region_close(void* peer);
+int liger_ipc_region_free(void* region);
+int liger_op_oneshot_allreduce(void* buf, size_t count, void* const* regions, int world, int rank, size_t cap,
+                               uint64_t epoch, void* stream);
+
 /* Debug readback for parity tests (not part of the serving path).
  * liger_set_debug_capture(ctx, arena_bytes) [collective]: arena_bytes > 0 turns capture
  * on with a device arena of that size (allocated here, before serving: nothing is

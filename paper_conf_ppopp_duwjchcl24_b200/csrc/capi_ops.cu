@@ -5,6 +5,7 @@
 #include <mutex>
 #include <string>
 
+#include "comm.h"
 #include "kernels.h"
 
 namespace liger {
@@ -141,6 +142,49 @@ int liger_op_c0_fill(void* dst, int rows, int cols, int64_t ld, uint64_t seed, u
   return ret(c0_fill_launch(dst, rows, cols, ld, seed, tensor_id, row_off, col_off, idx_row_stride, idx_col_stride,
                             exp, kind, (cudaStream_t)stream),
              "liger_op_c0_fill");
+}
+
+// ------------------------------------------------------------------ CUDA-IPC peer regions (transport tests)
+int liger_ipc_region_create(size_t cap, void** region, uint8_t* handle) {
+  if (int rc = check_device()) return rc;
+  if (!region || !handle || cap == 0 || cap % 256) return LIGER_EINVAL;
+  const size_t rb = peer_ar_region_bytes(cap);
+  void* r = nullptr;
+  if (cudaMalloc(&r, rb) != cudaSuccess) return ret(LIGER_ENOMEM, "liger_ipc_region_create");
+  cudaIpcMemHandle_t h;
+  if (cudaMemset(r, 0, rb) != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess ||
+      cudaIpcGetMemHandle(&h, r) != cudaSuccess) {
+    cudaFree(r);
+    return ret(LIGER_ECUDA, "liger_ipc_region_create");
+  }
+  memcpy(handle, &h, sizeof(h));
+  *region = r;
+  return LIGER_OK;
+}
+
+int liger_ipc_region_open(const uint8_t* handle, void** peer) {
+  if (int rc = check_device()) return rc;
+  if (!handle || !peer) return LIGER_EINVAL;
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, sizeof(h));
+  if (cudaIpcOpenMemHandle(peer, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+    return ret(LIGER_ECUDA, "liger_ipc_region_open");
+  return LIGER_OK;
+}
+
+int liger_ipc_region_close(void* peer) { return cudaIpcCloseMemHandle(peer) == cudaSuccess ? LIGER_OK : LIGER_ECUDA; }
+
+int liger_ipc_region_free(void* region) { return cudaFree(region) == cudaSuccess ? LIGER_OK : LIGER_ECUDA; }
+
+int liger_op_oneshot_allreduce(void* buf, size_t count, void* const* regions, int world, int rank, size_t cap,
+                               uint64_t epoch, void* stream) {
+  if (int rc = check_device()) return rc;
+  if (!buf || !regions || world < 1 || world > 8 || rank < 0 || rank >= world || epoch == 0)
+    return LIGER_EINVAL;
+  PeerAR par;
+  if (int rc = par.init(world, rank, cap, regions[rank], regions)) return ret(rc, "liger_op_oneshot_allreduce");
+  par.epoch = epoch - 1;   // this call is epoch `epoch` (allreduce_bf16 pre-increments)
+  return ret(par.allreduce_bf16(buf, count, (cudaStream_t)stream), "liger_op_oneshot_allreduce");
 }
 
 }  // extern "C"

@@ -60,6 +60,11 @@ _SIGS = {
     "liger_poll": (_I, [_P, _I64, C.POINTER(liger_result), _P]),
     "liger_result_tokens_device": (_I, [_P, _I64, C.POINTER(_P)]),
     "liger_set_debug_capture": (_I, [_P, _SZ]),
+    "liger_ipc_region_create": (_I, [_SZ, C.POINTER(_P), _P]),
+    "liger_ipc_region_open": (_I, [_P, C.POINTER(_P)]),
+    "liger_ipc_region_close": (_I, [_P]),
+    "liger_ipc_region_free": (_I, [_P]),
+    "liger_op_oneshot_allreduce": (_I, [_P, _SZ, _P, _I, _I, _SZ, _U64, _P]),
     "liger_op_allreduce": (_I, [_P, _P, _SZ, _I, _I, _I, _P]),
     "liger_debug_read": (_I, [_P, _I64, _I, _P, _SZ]),
     "liger_stats": (_I, [_P, C.POINTER(liger_stats_t)]),
@@ -158,6 +163,28 @@ def gemm_tiled(x, w_tiled, out, *, N, n0=0, n1=None, bias=None, act="none", scal
     check(lib().liger_op_gemm_tiled(_p(x), x.stride(0), _p(w_tiled), _p(out), out.stride(0), M, N, K, n0, n1,
                                     _p(bias), ACT[act], scale_cols, scale, out_f32, _p(workspace), ws_b,
                                     _s(stream)), what="liger_op_gemm_tiled")
+
+
+def ipc_region_create(cap):
+    """(region pointer, 64-byte CUDA-IPC handle) of a fresh one-shot staging region."""
+    reg = C.c_void_p()
+    h = C.create_string_buffer(64)
+    check(lib().liger_ipc_region_create(cap, C.byref(reg), h), what="liger_ipc_region_create")
+    return reg.value, h.raw
+
+
+def ipc_region_open(handle):
+    p = C.c_void_p()
+    check(lib().liger_ipc_region_open(C.create_string_buffer(bytes(handle), 64), C.byref(p)),
+          what="liger_ipc_region_open")
+    return p.value
+
+
+def oneshot_allreduce(buf, regions, rank, cap, epoch, stream=None):
+    """liger_op_oneshot_allreduce on torch bf16 buffer `buf` (in place)."""
+    arr = (C.c_void_p * len(regions))(*regions)
+    check(lib().liger_op_oneshot_allreduce(_p(buf), buf.numel(), arr, len(regions), rank, cap, epoch, _s(stream)),
+          what="liger_op_oneshot_allreduce")
 
 
 def tile_weight(w, w_tiled, stream=None):

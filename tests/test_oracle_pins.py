@@ -172,3 +172,19 @@ def test_model_matches_hf_opt_fp64(act):
         gen = m.generate(torch.from_numpy(prompt), max_new_tokens=8, do_sample=False,
                          attention_mask=torch.ones_like(torch.from_numpy(prompt)))
     assert np.array_equal(gen[:, 32:].numpy(), toks)
+
+
+def test_top2_margin_hand_computed():
+    """om.top2_margin (the near-tie gate of the token comparisons, reading R17) on
+    hand-worked rows: the gap between the largest and the second-largest logit, a tie
+    gives 0, order within the row does not matter, leading axes are kept."""
+    from oracle import model as om
+    x = np.array([[[1.0, 5.0, 3.0, -2.0], [0.5, 0.5, 0.1, 0.0]],
+                  [[-1.0, -3.0, -0.25, -7.0], [2.0, 9.0, 9.0, 1.0]]])
+    m = om.top2_margin(x)
+    assert m.shape == (2, 2)
+    assert np.array_equal(m, np.array([[2.0, 0.0], [0.75, 0.0]]))
+    rng = np.random.default_rng(0)
+    y = rng.standard_normal((3, 17))
+    srt = -np.sort(-y, axis=-1)
+    assert np.allclose(om.top2_margin(y[:, rng.permutation(17)]), srt[:, 0] - srt[:, 1])
