@@ -64,6 +64,7 @@ struct DecAttnArgs {
   int cps;                    // chunks per split
   float* ws;                  // split partials [b * heads][nsp][D + 2]
   int* counters;              // [b * heads], zero between uses
+  int early_trigger;          // release the dependent before the PDL wait (pdl_enter_early)
 };
 
 // Split plan of a launch: chunks per split and the split count.  Each CTA slot of a
