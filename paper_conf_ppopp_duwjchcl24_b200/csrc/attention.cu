@@ -367,7 +367,7 @@ __global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecA
   // ---------------- compute warps 0..3
   const int grp = warp * TPW + lane / LPT;   // lane group 0..NG-1
   const int gl = lane % LPT;                 // lane within the group: dims [8 gl, 8 gl + 8)
-  pdl_enter_early(a.early_trigger);   // q and the new token's k / v come from the QKV kernel
+  pdl_enter();   // q and the new token's k / v come from the QKV kernel
   const uint64_t tr1 = trace_now();
   const int64_t ld = (int64_t)3 * heads * D;
   int k = 0;
@@ -564,10 +564,6 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
   a.pos = pos;
   a.heads = heads;
   a.b = b;
-  {
-    static const int et = getenv("LIGER_EARLY_TRIGGER") ? atoi(getenv("LIGER_EARLY_TRIGGER")) : 0;
-    a.early_trigger = (et & 2) != 0;
-  }
   a.counters = (int*)workspace;
   a.ws = workspace ? (float*)((char*)workspace + ATTN_COUNTER_BYTES) : nullptr;
   const int rc = d == 128 ? launch_decode<128>(a, stream) : launch_decode<64>(a, stream);

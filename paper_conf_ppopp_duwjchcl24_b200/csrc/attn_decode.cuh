@@ -27,6 +27,7 @@
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "../../include/liger.h"
 #include "common.cuh"
@@ -64,7 +65,6 @@ struct DecAttnArgs {
   int cps;                    // chunks per split
   float* ws;                  // split partials [b * heads][nsp][D + 2]
   int* counters;              // [b * heads], zero between uses
-  int early_trigger;          // release the dependent before the PDL wait (pdl_enter_early)
 };
 
 // Split plan of a launch: chunks per split and the split count.  Each CTA slot of a
@@ -73,7 +73,7 @@ struct DecAttnArgs {
 // split only while there are fewer items than slots, never below one chunk per split.
 inline void dec_attn_plan(int b, int heads, int ctx, int* cps, int* nsp) {
   const int nch = (ctx + DC_CH - 1) / DC_CH;
-  const int slots = 148 * DC_CTAS_PER_SM;
+  static const int slots = getenv("LIGER_ATTN_SLOTS") ? atoi(getenv("LIGER_ATTN_SLOTS")) : 148 * DC_CTAS_PER_SM;
   int want = slots / (b * heads);
   if (want < 1) want = 1;
   if (want > nch) want = nch;

@@ -202,16 +202,6 @@ LIGER_DEV void pdl_enter() {
   grid_dependency_wait();
   grid_dependency_trigger();
 }
-// For a kernel that never spins on other ranks and whose dependent's pre-wait part reads
-// only immutable data (a projection GEMM prefetching weights): trigger first, so the
-// dependent is launched while this kernel still waits -- its CTAs take each SM as soon
-// as the kernels there exit and start their weight stream, instead of after this
-// kernel's wait plus the launch latency.  (LIGER_EARLY_TRIGGER experiment.)
-LIGER_DEV void pdl_enter_early(bool early) {
-  if (early) grid_dependency_trigger();
-  grid_dependency_wait();
-  if (!early) grid_dependency_trigger();
-}
 
 // ---------------------------------------------------------------- timeline trace
 // Development diagnostics (liger_trace_start / liger_trace_stop): thread 0 of every

@@ -90,7 +90,6 @@ struct GemmParams {
   float ln_eps;
   // residual add in the final store: out[m, n] = resid[m, n] + v (may alias out)
   const __nv_bfloat16* resid;
-  int early_trigger;                // fixup: release the dependent before the wait (pdl_enter_early)
 };
 
 // mean / rstd (population variance, eps inside the sqrt) of rows m < M of X[M, K]
@@ -400,7 +399,7 @@ __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) 
       }
     }
   }
-  pdl_enter_early(p.early_trigger);
+  pdl_enter();
   const uint64_t tr1 = trace_now();
   const float* lnst = p.ln_stats;
   for (int64_t t = t_first; t < total; t += (int64_t)gridDim.x * blockDim.x) {
@@ -707,10 +706,6 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
     p.pub_epoch = a.far->epoch;
   }
   p.ws = a.workspace ? reinterpret_cast<float*>(reinterpret_cast<char*>(a.workspace) + GEMM_COUNTER_BYTES) : nullptr;
-  {
-    static const int et = getenv("LIGER_EARLY_TRIGGER") ? atoi(getenv("LIGER_EARLY_TRIGGER")) : 0;
-    p.early_trigger = (et & 1) && !a.far;   // the fused all-reduce producer publishes to spinning peers
-  }
   p.w_tiled = a.w_tiled;
   p.nkb_total = (a.K + BK - 1) / BK;
   p.n_tiles = ntiles;
