@@ -240,23 +240,36 @@ def test_allreduce_op_vs_oracle_and_decomposition(E, world, oneshot):
     parts = {n: [part(q, n) for q in range(world)] for n in sizes}
     got = {}
     err = []
+    import threading
+    bar = threading.Barrier(world)
 
     def rank_main(r):
+        # On the loopback backend the ranks share one GPU: a device-wide synchronize (or a
+        # synchronous copy) on one rank while a peer's one-shot kernel spins on this
+        # rank's next epoch never returns.  Inputs are staged before any all-reduce, the
+        # all-reduces run on the rank's own stream, and results are read after a barrier.
         try:
             torch.cuda.set_device(0)
             eng = E(cfg, world=world, rank=r, nccl_uid=uid, max_batch=2, max_seq=16, max_new=2, seed=0, load=False)
+            bufs = {(n, tuple(ks)): torch.from_numpy(parts[n][r]).cuda().bfloat16() for n in sizes for ks in splits}
+            torch.cuda.synchronize()
+            bar.wait()
+            st = torch.cuda.Stream()
             for n in sizes:
                 for ks in splits:
-                    buf = torch.from_numpy(parts[n][r]).cuda().bfloat16()
                     u = 0
                     for k in ks:
-                        eng.allreduce(buf, u, u + k, F)
+                        eng.allreduce(bufs[(n, tuple(ks))], u, u + k, F, stream=st.cuda_stream)
                         u += k
-                    torch.cuda.synchronize()
-                    got[(r, n, tuple(ks))] = buf.float().cpu().numpy()
+            st.synchronize()
+            bar.wait()
+            for key, b in bufs.items():
+                got[(r,) + key] = b.float().cpu().numpy()
+            bar.wait()
             eng.close()
         except Exception as e:
             err.append(repr(e))
+            bar.abort()
 
     import threading
     with env(LIGER_ONESHOT_AR=oneshot, LIGER_ONESHOT_MAX_KB="16"):
