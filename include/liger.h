@@ -150,6 +150,33 @@ int liger_load_layer(liger_ctx* ctx, int layer, uint64_t seed);
 /* Initialise embeddings (token + learned positions), final LN. [collective] */
 int liger_load_embed(liger_ctx* ctx, uint64_t seed);
 
+/* Load caller-owned weights instead of the seeded init (e.g. torch tensors; the library
+ * copies them into its own layout -- the tiled projection weights, the folded-LN copies
+ * at t = 1 -- and never keeps or frees the caller's pointers; the copies are complete
+ * when the call returns).  All device pointers, bf16, row-major, THIS RANK's shard in the
+ * nn.Linear layout of the Megatron partition (C8):
+ *   w_qkv [3h/t, h]: rows = this rank's q heads | k heads | v heads (h/t rows each);
+ *   b_qkv [3h/t] (same order); w_o [h, h/t] (columns = this rank's heads); b_o [h];
+ *   w_1 [f/t, h] (rows = this rank's FFN columns); b_1 [f/t]; w_2 [h, f/t]; b_2 [h];
+ *   ln1_g, ln1_b, ln2_g, ln2_b [h] (replicated).
+ * In the pipeline modes t = 1 and the rank loads only its stage's layers (others: no-op).
+ * LIGER_EINVAL for a null pointer or a layer out of range. [collective] */
+typedef struct {
+  const void *w_qkv, *b_qkv, *w_o, *b_o, *w_1, *b_1, *w_2, *b_2, *ln1_g, *ln1_b, *ln2_g, *ln2_b;
+} liger_layer_weights;
+int liger_load_layer_weights(liger_ctx* ctx, int layer, const liger_layer_weights* w);
+/* Caller-owned embeddings: e_tok [V, h], e_pos [max_pos + 2, h] (OPT's offset 2 included),
+ * lnf_g, lnf_b [h]; device bf16, replicated on every rank; copied. [collective] */
+int liger_load_embed_weights(liger_ctx* ctx, const void* e_tok, const void* e_pos, const void* lnf_g,
+                             const void* lnf_b);
+
+/* Run on caller-owned CUDA streams (e.g. torch streams) instead of the two the context
+ * created: compute_stream carries the computation kernels, comm_stream the collectives
+ * (Algorithm 1's two streams).  Borrowed: the library never destroys them; they must
+ * outlive the context and be distinct, non-null streams.  Only while no batch is in flight
+ * (LIGER_ESTATE otherwise); the context's own streams are synchronised first. */
+int liger_set_streams(liger_ctx* ctx, void* compute_stream, void* comm_stream);
+
 /* Enqueue one pre-packed batch in the waiting queue.
  * tokens: [batch * seq_len] int32 prompt ids, sequence-major; host pointer
  * (copied to the device inside the library) or device pointer when

@@ -160,6 +160,7 @@ struct liger_ctx {
   std::string err;
   Comm* comm = nullptr;   // NCCL or loopback (comm.cu); nullptr at world == 1
   cudaStream_t s_comp = nullptr, s_comm = nullptr;
+  bool own_streams = true;   // false after liger_set_streams (borrowed: never destroyed)
   std::vector<LayerW> layers;
   void *e_tok = nullptr, *e_pos = nullptr, *lnf_g = nullptr, *lnf_b = nullptr;
   std::vector<void*> allocs;
@@ -1157,6 +1158,65 @@ int liger_load_layer(liger_ctx* c, int l, uint64_t seed) {
   return LIGER_OK;
 }
 
+int liger_load_layer_weights(liger_ctx* c, int l, const liger_layer_weights* w) {
+  if (!c || !w || l < 0 || l >= c->L) return LIGER_EINVAL;
+  if (l < c->l0 || l >= c->l1) return LIGER_OK;   // another pipeline stage's layer
+  const void* need[] = {w->w_qkv, w->b_qkv, w->w_o, w->b_o, w->w_1, w->b_1, w->w_2, w->b_2,
+                        w->ln1_g, w->ln1_b, w->ln2_g, w->ln2_b};
+  for (const void* q : need)
+    if (!q) return fail(c, LIGER_EINVAL, "liger_load_layer_weights: null pointer");
+  const int64_t h = c->h, hl = c->hl, fl = c->fl;
+  LayerW& W = c->layers[l];
+  cudaStream_t st = c->s_comp;
+  CK(cudaMemsetAsync(W.w_qkv, 0, (size_t)pad128(3 * (int)hl) * h * 2, st));
+  CK(cudaMemsetAsync(W.w_1, 0, (size_t)pad128((int)fl) * h * 2, st));
+  CKR(tile_weight_launch(w->w_qkv, h, W.w_qkv, (int)(3 * hl), (int)h, st));
+  CKR(tile_weight_launch(w->w_o, hl, W.w_o, (int)h, (int)hl, st));
+  CKR(tile_weight_launch(w->w_1, h, W.w_1, (int)fl, (int)h, st));
+  CKR(tile_weight_launch(w->w_2, fl, W.w_2, (int)h, (int)fl, st));
+  CK(cudaMemcpyAsync(W.b_qkv, w->b_qkv, (size_t)3 * hl * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(W.b_o, w->b_o, (size_t)h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(W.b_1, w->b_1, (size_t)fl * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(W.b_2, w->b_2, (size_t)h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(W.g1, w->ln1_g, (size_t)h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(W.be1, w->ln1_b, (size_t)h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(W.g2, w->ln2_g, (size_t)h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(W.be2, w->ln2_b, (size_t)h * 2, cudaMemcpyDeviceToDevice, st));
+  if (c->ln_fold) CKR(fold_layer_norms(c, W, st));
+  CK(cudaStreamSynchronize(st));
+  return LIGER_OK;
+}
+
+int liger_load_embed_weights(liger_ctx* c, const void* e_tok, const void* e_pos, const void* lnf_g,
+                             const void* lnf_b) {
+  if (!c || !e_tok || !e_pos || !lnf_g || !lnf_b) return LIGER_EINVAL;
+  const size_t h = c->h;
+  cudaStream_t st = c->s_comp;
+  CK(cudaMemcpyAsync(c->e_tok, e_tok, (size_t)c->V * h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(c->e_pos, e_pos, (size_t)(c->cfg.max_pos + 2) * h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(c->lnf_g, lnf_g, h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(c->lnf_b, lnf_b, h * 2, cudaMemcpyDeviceToDevice, st));
+  CK(cudaStreamSynchronize(st));
+  return LIGER_OK;
+}
+
+int liger_set_streams(liger_ctx* c, void* compute_stream, void* comm_stream) {
+  if (!c || !compute_stream || !comm_stream || compute_stream == comm_stream) return LIGER_EINVAL;
+  if (!c->processing.empty() || !c->waiting.empty())
+    return fail(c, LIGER_ESTATE, "liger_set_streams: batches in flight");
+  CK(cudaStreamSynchronize(c->s_comp));
+  CK(cudaStreamSynchronize(c->s_comm));
+  if (c->own_streams) {
+    cudaStreamDestroy(c->s_comp);
+    cudaStreamDestroy(c->s_comm);
+    c->own_streams = false;
+  }
+  c->s_comp = (cudaStream_t)compute_stream;
+  c->s_comm = (cudaStream_t)comm_stream;
+  c->have_round = false;
+  return LIGER_OK;
+}
+
 int liger_load_embed(liger_ctx* c, uint64_t seed) {
   if (!c) return LIGER_EINVAL;
   const int64_t h = c->h;
@@ -1732,8 +1792,10 @@ int liger_finalize(liger_ctx* c) {
   cudaEventDestroy(c->e2);
   cudaEventDestroy(c->e_end[0]);
   cudaEventDestroy(c->e_end[1]);
-  cudaStreamDestroy(c->s_comp);
-  cudaStreamDestroy(c->s_comm);
+  if (c->own_streams) {
+    cudaStreamDestroy(c->s_comp);
+    cudaStreamDestroy(c->s_comm);
+  }
   gemm_forget_pointer_range(nullptr, ~size_t(0));
   delete c;
   return LIGER_OK;

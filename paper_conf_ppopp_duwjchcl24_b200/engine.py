@@ -61,6 +61,25 @@ class LigerEngine:
             self._chk(lib.liger_load_layer(self.ctx, l, seed), "liger_load_layer")
         self._chk(lib.liger_load_embed(self.ctx, seed), "liger_load_embed")
 
+    def load_weights(self, layers, embed):
+        """Caller-owned weights (liger_load_layer_weights / liger_load_embed_weights): `layers`
+        = list of dicts of this rank's bf16 device tensors (nn.Linear layout, see liger.h),
+        `embed` = dict(e_tok, e_pos, lnf_g, lnf_b).  The library copies them."""
+        lib = L.lib()
+        for l, w in enumerate(layers):
+            if w is None:
+                continue
+            st = L.liger_layer_weights(*[w[n].data_ptr() for n, _ in L.liger_layer_weights._fields_])
+            self._chk(lib.liger_load_layer_weights(self.ctx, l, C.byref(st)), "liger_load_layer_weights")
+        self._chk(lib.liger_load_embed_weights(self.ctx, *[C.c_void_p(embed[k].data_ptr()) for k in
+                                                             ("e_tok", "e_pos", "lnf_g", "lnf_b")]),
+                  "liger_load_embed_weights")
+
+    def set_streams(self, compute_stream, comm_stream):
+        """Run on caller-owned streams (e.g. torch.cuda.Stream().cuda_stream); liger_set_streams."""
+        self._chk(L.lib().liger_set_streams(self.ctx, C.c_void_p(compute_stream), C.c_void_p(comm_stream)),
+                  "liger_set_streams")
+
     def profile(self, m_list):
         arr = (C.c_int32 * len(m_list))(*m_list)
         self._chk(L.lib().liger_profile(self.ctx, arr, len(m_list)), "liger_profile")

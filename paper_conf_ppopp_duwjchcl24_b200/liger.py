@@ -39,6 +39,11 @@ class liger_result(C.Structure):
                 ("start_s", C.c_double), ("finish_s", C.c_double)]
 
 
+class liger_layer_weights(C.Structure):
+    _fields_ = [(n, C.c_void_p) for n in ("w_qkv", "b_qkv", "w_o", "b_o", "w_1", "b_1", "w_2", "b_2", "ln1_g",
+                                          "ln1_b", "ln2_g", "ln2_b")]
+
+
 class liger_stats_t(C.Structure):
     _fields_ = [("rounds", C.c_int64), ("kernels", C.c_int64), ("comm_kernels", C.c_int64),
                 ("split_pieces", C.c_int64), ("overlapped_rounds", C.c_int64), ("host_us", C.c_double),
@@ -54,6 +59,9 @@ _SIGS = {
     "liger_loopback_unique_id": (_I, [_P]),
     "liger_load_layer": (_I, [_P, _I, _U64]),
     "liger_load_embed": (_I, [_P, _U64]),
+    "liger_load_layer_weights": (_I, [_P, _I, C.POINTER(liger_layer_weights)]),
+    "liger_load_embed_weights": (_I, [_P, _P, _P, _P, _P]),
+    "liger_set_streams": (_I, [_P, _P, _P]),
     "liger_submit": (_I64, [_P, _I, _I, _P, _I, _I, _D]),
     "liger_step": (_I, [_P]),
     "liger_drain": (_I, [_P]),

@@ -285,3 +285,74 @@ def test_allreduce_op_vs_oracle_and_decomposition(E, world, oneshot):
             want = bf16_rne(ref.astype(np.float32))
             for r in range(world):
                 assert np.array_equal(got[(r, n, tuple(ks))].view(np.uint32), want.view(np.uint32)), (r, n, ks)
+
+
+def _host_shard(cfg, seed, t, r):
+    """Rank r's shard of every layer and the embeddings as bf16 torch tensors on the GPU,
+    built on the HOST from the numpy C0 generator (liger_inputs; not the library's init)."""
+    from liger_inputs import layer_tensor, global_tensor
+    h, a, f = cfg.hidden, cfg.n_heads, cfg.ffn
+    hl, fl = h // t, f // t
+    dev = lambda x: torch.from_numpy(np.ascontiguousarray(x, dtype=np.float32)).cuda().bfloat16()
+    layers = []
+    for l in range(cfg.n_layers):
+        wq = layer_tensor(cfg, seed, l, "w_qkv")                 # [h, 3h] logical
+        bq = layer_tensor(cfg, seed, l, "b_qkv")
+        cols = np.r_[r * hl:(r + 1) * hl, h + r * hl:h + (r + 1) * hl, 2 * h + r * hl:2 * h + (r + 1) * hl]
+        layers.append(dict(
+            w_qkv=dev(wq[:, cols].T), b_qkv=dev(bq[cols]),
+            w_o=dev(layer_tensor(cfg, seed, l, "w_o")[r * hl:(r + 1) * hl, :].T), b_o=dev(layer_tensor(cfg, seed, l, "b_o")),
+            w_1=dev(layer_tensor(cfg, seed, l, "w_1")[:, r * fl:(r + 1) * fl].T),
+            b_1=dev(layer_tensor(cfg, seed, l, "b_1")[r * fl:(r + 1) * fl]),
+            w_2=dev(layer_tensor(cfg, seed, l, "w_2")[r * fl:(r + 1) * fl, :].T), b_2=dev(layer_tensor(cfg, seed, l, "b_2")),
+            ln1_g=dev(layer_tensor(cfg, seed, l, "ln1_g")), ln1_b=dev(layer_tensor(cfg, seed, l, "ln1_b")),
+            ln2_g=dev(layer_tensor(cfg, seed, l, "ln2_g")), ln2_b=dev(layer_tensor(cfg, seed, l, "ln2_b"))))
+    embed = {k: dev(global_tensor(cfg, seed, k)) for k in ("e_tok", "e_pos", "lnf_g", "lnf_b")}
+    return layers, embed
+
+
+@pytest.mark.parametrize("world", [1, 2])
+def test_caller_owned_weights_and_streams(E, world):
+    """§8(b) boundary: weights passed in as caller-owned torch tensors
+    (liger_load_layer_weights / liger_load_embed_weights, copied by the library) and the
+    serving run on caller-owned torch streams (liger_set_streams) give the bits of the
+    seeded-init engine and the oracle element-wise, at t = 1 (LN fold) and loopback t = 2."""
+    import threading
+    cfg = get_config("tiny")
+    trace = _mixed_trace(3, 9, cfg, (1, 2), (8, 30), (3, 5))
+    kw = dict(mode="interleaved", max_batch=2, max_seq=32, max_new=8, seed=11)
+    ref = serve(E, cfg, world, trace, **kw)
+    uid = E.loopback_id() if world > 1 else None
+    out = [None] * world
+    err = []
+    bar = threading.Barrier(world)
+
+    def rank_main(r):
+        try:
+            torch.cuda.set_device(0)
+            layers, embed = _host_shard(cfg, 11, world, r)
+            eng = E(cfg, world=world, rank=r, nccl_uid=uid, load=False, **kw)
+            eng.load_weights(layers, embed)
+            s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+            eng.set_streams(s1.cuda_stream, s2.cuda_stream)
+            eng.set_debug_capture()
+            ids = [eng.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], 0.0) for t in trace]
+            eng.drain()
+            out[r] = dict(tokens=[eng.poll(i, want_tokens=True)[1] for i in ids], stats=eng.stats(),
+                          logits=[eng.debug_read(i, "logits", t["batch"], t["n_decode"]) for i, t in zip(ids, trace)],
+                          resid=[eng.debug_read(i, "resid", t["batch"], t["n_decode"]) for i, t in zip(ids, trace)])
+            bar.wait()
+            eng.close()
+            del layers, embed
+        except Exception as e:
+            err.append(repr(e))
+            bar.abort()
+
+    ths = [threading.Thread(target=rank_main, args=(r,), daemon=True) for r in range(world)]
+    for t in ths:
+        t.start()
+    for t in ths:
+        t.join(timeout=300)
+    assert not err, err
+    assert_bit_identical(ref, out)
+    check_vs_oracle(cfg, 11, trace, out, world=world)
