@@ -184,6 +184,24 @@ class ThreadGroup:
 
 
 # ----------------------------------------------------------------------------- CPU oracle baseline
+_CPP_ORACLE = []
+
+
+def _cpp_oracle():
+    """The fp32 C++ oracle binary compiled (once per process) for THIS host (-march=native:
+    the repo's copy may have been built elsewhere), or None."""
+    if not _CPP_ORACLE:
+        exe = None
+        try:
+            import tempfile
+            from paper_conf_ppopp_duwjchcl24_b200.build import build_oracle
+            exe, _ = build_oracle(os.path.join(tempfile.gettempdir(), f"liger_oracle_{os.getpid()}"))
+        except Exception as e:
+            print(f"bench.py: C++ oracle unavailable ({e}); timing the numpy oracle", file=sys.stderr)
+        _CPP_ORACLE.append(exe)
+    return _CPP_ORACLE[0]
+
+
 def cpu_oracle_sample(cfg, b=2, s=128, n_new=32, threads=None):
     """Time the CPU oracle on a bounded sample of the workload and extrapolate (labelled).
 
@@ -192,13 +210,7 @@ def cpu_oracle_sample(cfg, b=2, s=128, n_new=32, threads=None):
     steps at ctx s + 16 -- with weights generated on the fly, x L layers x n_new passes.
     Fallback (binary not built): the fp64 numpy oracle on the same sample."""
     nproc = os.cpu_count() or 1
-    exe = None
-    try:   # -march=native: compile for THIS host (the binary may not have been built here)
-        import tempfile
-        from paper_conf_ppopp_duwjchcl24_b200.build import build_oracle
-        exe, _ = build_oracle(os.path.join(tempfile.gettempdir(), f"liger_oracle_{os.getpid()}"))
-    except Exception as e:
-        print(f"bench.py: C++ oracle unavailable ({e}); timing the numpy oracle", file=sys.stderr)
+    exe = _cpp_oracle()
     if exe and os.path.exists(exe):
         out = {}
         for th in ([threads] if threads else [nproc, 1]):

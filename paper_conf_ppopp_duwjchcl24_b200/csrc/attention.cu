@@ -398,7 +398,11 @@ __global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecA
         *reinterpret_cast<uint4*>(a.kv_pool + kv_off(page, 1, heads, head, pos % KVB, D) + gl * 8) = vv4;
       }
     }
-    float m = -INFINITY, l = 0.f, acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    float m = -INFINITY, l = 0.f;
+    float2 acc2[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+    float2 q2[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) q2[e] = make_float2(q[2 * e], q[2 * e + 1]);
     for (int j = 0; j < nc; ++j, ++k) {
       const int s = k % DC_NS;
       mbar_wait(&sm.full[s], (uint32_t)(k / DC_NS) & 1u);
@@ -407,26 +411,36 @@ __global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecA
       const __nv_bfloat16* sV = sm.kv[s][1];
       // scores of this lane group's PPG positions (independent chains), then one
       // online-softmax update for all of them
-      float sc[PPG], vf[PPG][8];
+      // packed fp32x2 arithmetic (FFMA2 / FMUL2): a K or V row slice of 8 bf16 is 4 bf16x2
+      // words, unpacked to 4 float2 (element 2i in the low half of word i)
+      float sc[PPG];
+      float2 vf[PPG][4];
+      const bool full_chunk = t0 + DC_CH <= pos;   // every position cached (block-uniform)
 #pragma unroll
       for (int r = 0; r < PPG; ++r) {
         const int lt = r * NG + grp;
         const int t = t0 + lt;
-        float kf[8];
-        if (t < pos) {
-          bf16x8_to_f32(*reinterpret_cast<const uint4*>(sK + lt * D + gl * 8), kf);
-          bf16x8_to_f32(*reinterpret_cast<const uint4*>(sV + lt * D + gl * 8), vf[r]);
+        float2 kf[4];
+        if (full_chunk || t < pos) {
+          const uint4 kw = *reinterpret_cast<const uint4*>(sK + lt * D + gl * 8);
+          const uint4 vw = *reinterpret_cast<const uint4*>(sV + lt * D + gl * 8);
+          const uint32_t kk[4] = {kw.x, kw.y, kw.z, kw.w}, vv[4] = {vw.x, vw.y, vw.z, vw.w};
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            kf[e] = make_float2(__uint_as_float(kk[e] << 16), __uint_as_float(kk[e] & 0xFFFF0000u));
+            vf[r][e] = make_float2(__uint_as_float(vv[e] << 16), __uint_as_float(vv[e] & 0xFFFF0000u));
+          }
         } else {
 #pragma unroll
-          for (int e = 0; e < 8; ++e) {
-            kf[e] = kn[e];
-            vf[r][e] = vn[e];
+          for (int e = 0; e < 4; ++e) {
+            kf[e] = make_float2(kn[2 * e], kn[2 * e + 1]);
+            vf[r][e] = make_float2(vn[2 * e], vn[2 * e + 1]);
           }
         }
-        float dot = 0.f;
+        float2 d2 = __fmul2_rn(q2[0], kf[0]);
 #pragma unroll
-        for (int e = 0; e < 8; ++e) dot += q[e] * kf[e];
-        sc[r] = dot;
+        for (int e = 1; e < 4; ++e) d2 = __ffma2_rn(q2[e], kf[e], d2);
+        sc[r] = d2.x + d2.y;
       }
 #pragma unroll
       for (int off = LPT / 2; off > 0; off >>= 1)
@@ -437,19 +451,21 @@ __global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecA
       float mn = m;
 #pragma unroll
       for (int r = 0; r < PPG; ++r)
-        if (t0 + r * NG + grp <= pos) mn = fmaxf(mn, sc[r]);
+        if (full_chunk || t0 + r * NG + grp <= pos) mn = fmaxf(mn, sc[r]);
       if (mn != -INFINITY) {   // group-uniform: at least one valid position so far
         const float scale = __expf(m - mn);
         l *= scale;
+        const float2 sc2 = make_float2(scale, scale);
 #pragma unroll
-        for (int e = 0; e < 8; ++e) acc[e] *= scale;
+        for (int e = 0; e < 4; ++e) acc2[e] = __fmul2_rn(acc2[e], sc2);
 #pragma unroll
         for (int r = 0; r < PPG; ++r) {
-          if (t0 + r * NG + grp <= pos) {
+          if (full_chunk || t0 + r * NG + grp <= pos) {
             const float p = __expf(sc[r] - mn);
             l += p;
+            const float2 p2 = make_float2(p, p);
 #pragma unroll
-            for (int e = 0; e < 8; ++e) acc[e] += p * vf[r][e];
+            for (int e = 0; e < 4; ++e) acc2[e] = __ffma2_rn(p2, vf[r][e], acc2[e]);
           }
         }
         m = mn;
@@ -461,7 +477,10 @@ __global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecA
       sm.st_l[grp] = l;
     }
 #pragma unroll
-    for (int e = 0; e < 8; ++e) sm.st_acc[grp][gl * 8 + e] = acc[e];
+    for (int e = 0; e < 4; ++e) {
+      sm.st_acc[grp][gl * 8 + 2 * e] = acc2[e].x;
+      sm.st_acc[grp][gl * 8 + 2 * e + 1] = acc2[e].y;
+    }
     named_bar_sync(1, DC_THREADS);
     float M = -INFINITY;
 #pragma unroll
