@@ -356,3 +356,48 @@ def test_caller_owned_weights_and_streams(E, world):
     assert not err, err
     assert_bit_identical(ref, out)
     check_vs_oracle(cfg, 11, trace, out, world=world)
+
+
+def test_profile_and_contention_factor_across_ranks(E):
+    """a16: the offline profile and the contention-factor calibration run
+    with real cross-rank all-reduces (loopback TP = 2: every all-reduce a collective of the
+    two rank threads); the ranks agree on the result (max over ranks), cf >= 1, and the
+    agreed tables drive identical plans: interleaved serving on both ranks afterwards stays
+    bit-identical to serial TP and equal to the oracle."""
+    import threading
+    cfg = get_config("tiny")
+    uid = E.loopback_id()
+    trace = _mixed_trace(3, 9, cfg, (1, 2), (8, 30), (3, 5))
+    cfs = [None, None]
+    res = [None, None]
+    err = []
+
+    def rank_main(r):
+        try:
+            torch.cuda.set_device(0)
+            eng = E(cfg, world=2, rank=r, nccl_uid=uid, mode="interleaved", max_batch=2, max_seq=32, max_new=8,
+                    max_inflight=2, seed=11)
+            eng.profile([2, 16, 64])
+            cf, detail = eng.calibrate_cf([16, 64], set_cf=True)
+            cfs[r] = (cf, detail)
+            eng.set_debug_capture()
+            ids = [eng.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], 0.0) for t in trace]
+            eng.drain()
+            res[r] = dict(tokens=[eng.poll(i, want_tokens=True)[1] for i in ids], stats=eng.stats(),
+                          logits=[eng.debug_read(i, "logits", t["batch"], t["n_decode"]) for i, t in zip(ids, trace)],
+                          resid=[eng.debug_read(i, "resid", t["batch"], t["n_decode"]) for i, t in zip(ids, trace)])
+            eng.close()
+        except Exception as e:
+            err.append(repr(e))
+
+    ths = [threading.Thread(target=rank_main, args=(r,), daemon=True) for r in range(2)]
+    for t in ths:
+        t.start()
+    for t in ths:
+        t.join(timeout=300)
+    assert not err, err
+    assert cfs[0][0] == cfs[1][0] and 1.0 <= cfs[0][0] < 100.0, cfs
+    assert set(cfs[0][1]) == {16, 64}
+    base = serve(E, cfg, 2, trace, mode="serial", max_batch=2, max_seq=32, max_new=8, seed=11)
+    assert_bit_identical(base, res)
+    check_vs_oracle(cfg, 11, trace, res, world=2)
