@@ -590,7 +590,7 @@ GemmPlan gemm_plan(int M, int N, int K) {
   const int G = num_sms();
   const int n_tiles = (N + BM - 1) / BM;
   const int nkb = (K + BK - 1) / BK;
-  const int mt = (M + 255) / 256;
+  int mt = (M + 255) / 256;
   int bn = (M + mt - 1) / mt;
   bn = (bn + 15) / 16 * 16;
   if (bn < 16) bn = 16;
@@ -632,6 +632,38 @@ GemmPlan gemm_plan(int M, int N, int K) {
     if (cost < best - 1e-9) {
       best = cost;
       best_s = S;
+    }
+  }
+  // Prefill token tiling: an unsplit prefill GEMM also tries smaller token tiles, down
+  // to bn = 144, so that its units fill the waves of G persistent CTAs better (e.g.
+  // M = 1024, N = 5120: 4 x 256 gives 160 units = 2 rounds of which the second is 8%
+  // full; 7 x 160 gives 280 units in 2 rounds of shorter units: 75 -> 56 us on B200,
+  // profiles/r02/gemm_prefill_tiling.txt).  Per-k-block cost 430 + 1.8 bn cycles,
+  // fitted to the large-M bn = 256 / 192 / 128 times there; a smaller tile must win
+  // by 5% (model error).  Below 144 the fixed 16 KiB weight tile per k-block
+  // dominates (bn = 128 measured up to 1.45x slower per flop than 256).
+  static const bool bn_fixed = getenv("LIGER_GEMM_BN_FIXED") != nullptr;   // experiments only
+  constexpr int BN_MIN_PREFILL = 144;
+  if (M > 64 && best_s == 1 && !bn_fixed) {
+    auto cost1 = [&](int mt_, int bn_) {
+      return ceil((double)n_tiles * mt_ / G) * (nkb * (430.0 + 1.8 * bn_) + 300.0);
+    };
+    const double base = cost1(mt, bn);
+    double cbest = base;
+    int mt_b = mt, bn_b = bn;
+    for (int m2 = mt + 1; m2 <= (M + BN_MIN_PREFILL - 1) / BN_MIN_PREFILL; ++m2) {
+      const int b2 = ((M + m2 - 1) / m2 + 15) / 16 * 16;
+      if ((M + b2 - 1) / b2 != m2 || b2 < BN_MIN_PREFILL) continue;
+      const double c2 = cost1(m2, b2);
+      if (c2 < cbest) {
+        cbest = c2;
+        mt_b = m2;
+        bn_b = b2;
+      }
+    }
+    if (cbest < 0.95 * base) {
+      mt = mt_b;
+      bn = bn_b;
     }
   }
   if (const char* e = getenv("LIGER_GEMM_FORCE_SPLITS")) {   // experiments only
