@@ -577,7 +577,7 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
                     (double)pl.splits * M * n * 4 + (double)M * n * 2, 0);
         }
       }
-      c->st.gpu_launches++;
+      c->st.gpu_launches += fix ? 2 : 1;   // the GEMM (+ its split-K fixup kernel)
       break;
     }
     case OP_ATTN: {
