@@ -3,10 +3,10 @@
 // Paged pool layout: [n_pages][2 (K,V)][heads][16 tokens][d] bf16; a sequence's
 // page_table row maps token position p to page page_table[p / 16].
 //
-//  * prefill: flash-style causal attention with bf16 tensor-core mma.sync
-//    (m16n8k16, fp32 accumulate), 64 queries x 64 keys per step, online
-//    softmax in registers; the CTA on the diagonal tile also writes that key
-//    tile's K/V into the cache pages.
+//  * prefill: flash-style causal attention on the tcgen05 tensor cores (TMA-loaded
+//    Q / K / V tiles, S and O accumulators in TMEM, softmax warps owning one query
+//    row each; persistent CTAs over (query tile, sequence, head) items), which also
+//    appends the prompt's K / V to the cache pages (attn_prefill_tc.cuh).
 //  * decode: one query per sequence; persistent CTAs stream 32-position chunks of
 //    the cache through a cp.async.bulk ring, online softmax per lane group in
 //    registers, deterministic merge of the split partials (attn_decode.cuh).
@@ -18,248 +18,41 @@
 #include <algorithm>
 
 #include "attn_decode.cuh"
+#include "attn_prefill_tc.cuh"
 #include "common.cuh"
 #include "kernels.h"
 
 namespace liger {
 
 // ================================================================== prefill
-constexpr int PF_BQ = 128, PF_BK = 64;
+// tcgen05 / TMEM / TMA kernel: attn_prefill_tc.cuh.
 
-__device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
-  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
-               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
-               : "r"(addr));
-}
-__device__ __forceinline__ void ldsm_x4_t(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
-  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];"
-               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
-               : "r"(addr));
-}
-__device__ __forceinline__ void mma_bf16_16816(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
-                                               uint32_t b0, uint32_t b1) {
-  asm volatile(
-      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
-      "{%0,%1,%2,%3};"
-      : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
-      : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
-}
-__device__ __forceinline__ uint32_t pack_bf16(float lo, float hi) {
-  __nv_bfloat162 v = __floats2bfloat162_rn(lo, hi);
-  return *reinterpret_cast<uint32_t*>(&v);
-}
-
-__device__ __forceinline__ void cp_async16(void* smem_dst, const void* gsrc, bool valid) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(smem_dst)), "l"(gsrc),
-               "r"(valid ? 16 : 0)
-               : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-
-// Prefill causal attention, flash-style: CTA = (128-query tile, head, sequence),
-// 8 warps x 16 query rows; 64-key tiles of K and V double-buffered in shared
-// memory with cp.async (the next tile loads while the current one is
-// computed); S = Q K^T and O += P V on bf16 tensor cores (mma.sync m16n8k16,
-// fp32 accumulate); online softmax in registers.  The CTA whose query range
-// contains a key tile also writes that tile's K/V into the paged cache.
-constexpr int PF_THREADS = 256;
 template <int D>
-__global__ void __launch_bounds__(PF_THREADS) attn_prefill_kernel(const __nv_bfloat16* __restrict__ qkv,
-                                                                  __nv_bfloat16* __restrict__ o,
-                                                                  __nv_bfloat16* __restrict__ kv_pool,
-                                                                  const int32_t* __restrict__ page_table,
-                                                                  int max_pages, int s, int heads) {
-  constexpr int LDS = D + 8;   // padded smem row (bank-conflict-free ldmatrix)
-  constexpr int NV = D / 8;    // 16-byte vectors per row
-  extern __shared__ __align__(16) uint8_t pf_smem[];
-  __nv_bfloat16* sQ = reinterpret_cast<__nv_bfloat16*>(pf_smem);       // [PF_BQ][LDS]
-  __nv_bfloat16* sK = sQ + PF_BQ * LDS;                                  // [2][PF_BK][LDS]
-  __nv_bfloat16* sV = sK + 2 * PF_BK * LDS;                              // [2][PF_BK][LDS]
-
-  const int nqt = gridDim.x;
-  const int qt = nqt - 1 - blockIdx.x;   // longest (most key tiles) first
-  const int head = blockIdx.y, bi = blockIdx.z;
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int64_t ld = (int64_t)3 * heads * D;
-  const __nv_bfloat16* base = qkv + (int64_t)bi * s * ld;
-  const int q0 = qt * PF_BQ;
-  const int q_hi = min(s, q0 + PF_BQ);            // rows [q0, q_hi)
-  const int nkt = (q_hi - 1) / PF_BK + 1;         // key tiles with k0 <= last row
-  pdl_enter();
-
-  auto load_kv = [&](int kt, int buf) {
-    const int k0 = kt * PF_BK;
-    for (int i = tid; i < PF_BK * NV; i += PF_THREADS) {
-      const int r = i / NV, c = (i % NV) * 8;
-      const bool ok = k0 + r < s;
-      const __nv_bfloat16* rowp = base + (int64_t)(ok ? k0 + r : 0) * ld;
-      cp_async16(&sK[(buf * PF_BK + r) * LDS + c], rowp + (int64_t)heads * D + head * D + c, ok);
-      cp_async16(&sV[(buf * PF_BK + r) * LDS + c], rowp + (int64_t)2 * heads * D + head * D + c, ok);
-    }
-  };
-  for (int i = tid; i < PF_BQ * NV; i += PF_THREADS) {
-    const int r = i / NV, c = (i % NV) * 8;
-    const bool ok = q0 + r < s;
-    cp_async16(&sQ[r * LDS + c], base + (int64_t)(ok ? q0 + r : 0) * ld + head * D + c, ok);
+static int launch_prefill_tc(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages,
+                             int b, int s, int heads, cudaStream_t stream) {
+  CUtensorMap tm;
+  if (gemm_act_map(&tm, qkv, b * s, 3 * heads * D, (int64_t)3 * heads * D, PT_BQ)) return LIGER_ECUDA;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(attn_prefill_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, PtSmem<D>::ALLOC);
+    attr = true;
   }
-  load_kv(0, 0);
-  cp_async_commit();
-
-  const int g = lane >> 2, tig = lane & 3;
-  float m_r[2] = {-INFINITY, -INFINITY}, l_r[2] = {0.f, 0.f};
-  float acc[D / 8][4];
-#pragma unroll
-  for (int j = 0; j < D / 8; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
-  const float L2E = 1.4426950408889634f;
-  const int wrow0 = q0 + warp * 16;        // this warp's rows [wrow0, wrow0 + 16)
-  const int row0 = wrow0 + g;              // this thread's rows: row0, row0 + 8
-
-  for (int kt = 0; kt < nkt; ++kt) {
-    const int buf = kt & 1;
-    const int k0 = kt * PF_BK;
-    if (kt + 1 < nkt) load_kv(kt + 1, buf ^ 1);
-    cp_async_commit();
-    cp_async_wait<1>();   // tile kt (and Q) landed
-    __syncthreads();
-    const __nv_bfloat16* cK = sK + buf * PF_BK * LDS;
-    const __nv_bfloat16* cV = sV + buf * PF_BK * LDS;
-    if (k0 >= q0 && k0 < q0 + PF_BQ) {   // this CTA appends key tile kt to the paged cache
-      for (int i = tid; i < PF_BK * NV; i += PF_THREADS) {
-        const int r = i / NV, c = (i % NV) * 8;
-        const int p = k0 + r;
-        if (p < s) {
-          const int page = page_table[(int64_t)bi * max_pages + p / KVB];
-          *reinterpret_cast<uint4*>(kv_pool + kv_off(page, 0, heads, head, p % KVB, D) + c) =
-              *reinterpret_cast<const uint4*>(&cK[r * LDS + c]);
-          *reinterpret_cast<uint4*>(kv_pool + kv_off(page, 1, heads, head, p % KVB, D) + c) =
-              *reinterpret_cast<const uint4*>(&cV[r * LDS + c]);
-        }
-      }
-    }
-    if (k0 <= wrow0 + 15 && wrow0 < s) {   // warp-uniform: some key of this tile is visible to the warp
-      float sc[8][4];
-#pragma unroll
-      for (int j = 0; j < 8; ++j) sc[j][0] = sc[j][1] = sc[j][2] = sc[j][3] = 0.f;
-#pragma unroll
-      for (int kc = 0; kc < D; kc += 16) {
-        uint32_t a0, a1, a2, a3;
-        const int ar = warp * 16 + (lane % 8) + ((lane / 8) % 2) * 8;
-        const int ac = kc + (lane / 16) * 8;
-        ldsm_x4(smem_u32(&sQ[ar * LDS + ac]), a0, a1, a2, a3);
-#pragma unroll
-        for (int nb = 0; nb < 8; nb += 2) {
-          uint32_t b0, b1, b2, b3;
-          const int br = nb * 8 + (lane % 8) + (lane / 16) * 8;
-          const int bc = kc + ((lane / 8) % 2) * 8;
-          ldsm_x4(smem_u32(&cK[br * LDS + bc]), b0, b1, b2, b3);
-          mma_bf16_16816(sc[nb], a0, a1, a2, a3, b0, b1);
-          mma_bf16_16816(sc[nb + 1], a0, a1, a2, a3, b2, b3);
-        }
-      }
-      if (k0 + PF_BK - 1 > wrow0 || k0 + PF_BK > s) {   // diagonal / ragged tile: mask
-#pragma unroll
-        for (int nb = 0; nb < 8; ++nb) {
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const int key = k0 + nb * 8 + tig * 2 + (e & 1);
-            const int row = row0 + (e >> 1) * 8;
-            if (key > row || key >= s) sc[nb][e] = -INFINITY;
-          }
-        }
-      }
-#pragma unroll
-      for (int h2 = 0; h2 < 2; ++h2) {
-        float mx = -INFINITY;
-#pragma unroll
-        for (int nb = 0; nb < 8; ++nb) mx = fmaxf(mx, fmaxf(sc[nb][2 * h2], sc[nb][2 * h2 + 1]));
-        mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
-        mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
-        const float m_new = fmaxf(m_r[h2], mx);
-        const float corr = (m_new == -INFINITY) ? 1.f : exp2f((m_r[h2] - m_new) * L2E);
-        float sum = 0.f;
-#pragma unroll
-        for (int nb = 0; nb < 8; ++nb) {
-#pragma unroll
-          for (int e = 0; e < 2; ++e) {
-            const float v = sc[nb][2 * h2 + e];
-            const float pv = (v == -INFINITY) ? 0.f : exp2f((v - m_new) * L2E);
-            sc[nb][2 * h2 + e] = pv;
-            sum += pv;
-          }
-        }
-        sum += __shfl_xor_sync(0xffffffffu, sum, 1);
-        sum += __shfl_xor_sync(0xffffffffu, sum, 2);
-        l_r[h2] = l_r[h2] * corr + sum;
-        m_r[h2] = m_new;
-#pragma unroll
-        for (int j = 0; j < D / 8; ++j) {
-          acc[j][2 * h2] *= corr;
-          acc[j][2 * h2 + 1] *= corr;
-        }
-      }
-#pragma unroll
-      for (int kc = 0; kc < 4; ++kc) {   // 16 keys per step
-        const uint32_t a0 = pack_bf16(sc[2 * kc][0], sc[2 * kc][1]);
-        const uint32_t a1 = pack_bf16(sc[2 * kc][2], sc[2 * kc][3]);
-        const uint32_t a2 = pack_bf16(sc[2 * kc + 1][0], sc[2 * kc + 1][1]);
-        const uint32_t a3 = pack_bf16(sc[2 * kc + 1][2], sc[2 * kc + 1][3]);
-#pragma unroll
-        for (int nb = 0; nb < D / 8; nb += 2) {
-          uint32_t b0, b1, b2, b3;
-          const int vr = kc * 16 + (lane % 8) + ((lane / 8) % 2) * 8;
-          const int vc = nb * 8 + (lane / 16) * 8;
-          ldsm_x4_t(smem_u32(&cV[vr * LDS + vc]), b0, b1, b2, b3);
-          mma_bf16_16816(acc[nb], a0, a1, a2, a3, b0, b1);
-          mma_bf16_16816(acc[nb + 1], a0, a1, a2, a3, b2, b3);
-        }
-      }
-    }
-    __syncthreads();   // buffer `buf` is refilled at iteration kt + 2
-  }
-  cp_async_wait<0>();
-#pragma unroll
-  for (int h2 = 0; h2 < 2; ++h2) {
-    const int row = row0 + h2 * 8;
-    if (row < s) {
-      const float inv = 1.0f / l_r[h2];
-      __nv_bfloat16* orow = o + ((int64_t)bi * s + row) * ((int64_t)heads * D) + head * D;
-#pragma unroll
-      for (int nb = 0; nb < D / 8; ++nb) {
-        const int c = nb * 8 + tig * 2;
-        *reinterpret_cast<__nv_bfloat162*>(orow + c) =
-            __floats2bfloat162_rn(acc[nb][2 * h2] * inv, acc[nb][2 * h2 + 1] * inv);
-      }
-    }
-  }
+  const int items = (s + PT_BQ - 1) / PT_BQ * b * heads;
+  const int grid = std::min(items, sm_count());
+  return launch_pdl(attn_prefill_tc_kernel<D>, dim3(grid), dim3(PT_THREADS), (size_t)PtSmem<D>::ALLOC, stream, tm,
+                    (__nv_bfloat16*)o, (const __nv_bfloat16*)qkv, (__nv_bfloat16*)kv_pool, page_table, max_pages, b,
+                    s, heads)
+             ? LIGER_ECUDA
+             : 0;
 }
 
 int attn_prefill_launch(const void* qkv, void* o, void* kv_pool, const int32_t* page_table, int max_pages, int b,
                         int s, int heads, int d, cudaStream_t stream) {
   if (b <= 0 || s <= 0) return 0;
-  dim3 grid((s + PF_BQ - 1) / PF_BQ, heads, b);
-  const size_t smem = (size_t)(PF_BQ + 4 * PF_BK) * (d + 8) * 2;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(attn_prefill_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (PF_BQ + 4 * PF_BK) * (128 + 8) * 2);
-    cudaFuncSetAttribute(attn_prefill_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (PF_BQ + 4 * PF_BK) * (64 + 8) * 2);
-    attr = true;
-  }
-  int rc;
-  if (d == 128)
-    rc = launch_pdl(attn_prefill_kernel<128>, grid, dim3(PF_THREADS), smem, stream, (const __nv_bfloat16*)qkv,
-                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
-  else if (d == 64)
-    rc = launch_pdl(attn_prefill_kernel<64>, grid, dim3(PF_THREADS), smem, stream, (const __nv_bfloat16*)qkv,
-                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, s, heads);
-  else
-    return LIGER_EINVAL;
-  return rc ? LIGER_ECUDA : 0;
+  if (d != 64 && d != 128) return LIGER_EINVAL;
+  if ((int64_t)b * s > (int64_t)1 << 30) return LIGER_EINVAL;
+  return d == 128 ? launch_prefill_tc<128>(qkv, o, kv_pool, page_table, max_pages, b, s, heads, stream)
+                  : launch_prefill_tc<64>(qkv, o, kv_pool, page_table, max_pages, b, s, heads, stream);
 }
 
 // ================================================================== decode
@@ -590,8 +383,8 @@ int attn_decode_launch(const void* qkv, void* o, void* kv_pool, const int32_t* p
 }
 
 void preload_attention_kernels() {
-  preload_kernel(attn_prefill_kernel<64>);
-  preload_kernel(attn_prefill_kernel<128>);
+  preload_kernel(attn_prefill_tc_kernel<64>);
+  preload_kernel(attn_prefill_tc_kernel<128>);
   preload_kernel(attn_decode_kernel<64>);
   preload_kernel(attn_decode_kernel<128>);
 }

@@ -281,6 +281,18 @@ inline void prefer_max_smem(const void* fn) {
 // Launch with programmatic stream serialization so the kernel's prologue overlaps
 // the tail of the previous kernel on the stream (the kernel calls
 // grid_dependency_wait() before touching data produced or consumed upstream).
+// SMs of the current device (host).
+inline int sm_count() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
 template <typename... KArgs, typename... Args>
 inline int launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
                       Args&&... args) {

@@ -219,6 +219,38 @@ def test_attention_prefill_and_decode_vs_oracle(L, b, s, heads, d):
         assert errs(to_np64(o1), ref1)[0] <= REL
 
 
+@pytest.mark.parametrize("b,s,heads,d,growth", [(2, 300, 40, 128, 0.0), (1, 400, 4, 64, 40.0), (3, 129, 50, 128, 0.0)])
+def test_attention_prefill_persistent_items_and_rescale(L, b, s, heads, d, growth):
+    """The tcgen05 prefill kernel's persistent item loop (more (query tile, sequence,
+    head) items than SMs: 240 / 450 items, so CTAs carry Q / K / V stages, S / O
+    accumulators and barrier phases across items) and its lazy O rescale (growth > 0:
+    key rows scaled by 1 + growth * p / s, so later key blocks raise the row max by far
+    more than 2^8 and the TMEM accumulator is rescaled), against the oracle; the paged
+    cache holds exactly K and V."""
+    qkv = _qkv(b, s, heads, d, 31)
+    hd = heads * d
+    if growth:
+        scale = (1.0 + growth * np.arange(s) / s).astype(np.float32)
+        qkv[:, hd:2 * hd] *= np.tile(scale, b)[:, None]
+    qkvd = bf16_dev(qkv)
+    qkv = to_np64(qkvd)
+    o = torch.empty(b * s, hd, dtype=torch.bfloat16, device="cuda")
+    maxp = (s + 15) // 16 + 1
+    pt = torch.from_numpy(np.random.default_rng(3).permutation(b * maxp).astype(np.int32).reshape(b, maxp)).cuda()
+    pool = torch.zeros(b * maxp, 2, heads, 16, d, dtype=torch.bfloat16, device="cuda")
+    L.attn_prefill(qkvd, o, pool, pt, b=b, s=s, heads=heads, d=d)
+    torch.cuda.synchronize()
+    q, k, v = (_split(qkv[:, i * hd:(i + 1) * hd], b, s, heads, d) for i in range(3))
+    ref = om.causal_attention(q, k, v, np.arange(s), np.arange(s)).transpose(0, 2, 1, 3).reshape(b * s, hd)
+    assert errs(to_np64(o), ref)[0] <= REL
+    ptn = pt.cpu().numpy()
+    pl = pool.float().cpu().numpy()
+    for bi in range(b):
+        pages = ptn[bi, np.arange(s) // 16]
+        assert np.array_equal(pl[pages, 0, :, np.arange(s) % 16, :], k[bi].transpose(1, 0, 2))
+        assert np.array_equal(pl[pages, 1, :, np.arange(s) % 16, :], v[bi].transpose(1, 0, 2))
+
+
 def test_decode_attention_long_context_split(L):
     """ctx > 256 exercises the deterministic multi-chunk merge; the result must not
     depend on scheduling (run twice, bit-identical)."""
