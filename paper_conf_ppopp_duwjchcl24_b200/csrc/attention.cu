@@ -40,7 +40,7 @@ static int launch_prefill_tc(const void* qkv, void* o, void* kv_pool, const int3
   const int items = (s + PT_BQ - 1) / PT_BQ * b * heads;
   const int grid = std::min(items, sm_count());
   return launch_pdl(attn_prefill_tc_kernel<D>, dim3(grid), dim3(PT_THREADS), (size_t)PtSmem<D>::ALLOC, stream, tm,
-                    (__nv_bfloat16*)o, (const __nv_bfloat16*)qkv, (__nv_bfloat16*)kv_pool, page_table, max_pages, b,
+                    (__nv_bfloat16*)o, (__nv_bfloat16*)kv_pool, page_table, max_pages, b,
                     s, heads)
              ? LIGER_ECUDA
              : 0;

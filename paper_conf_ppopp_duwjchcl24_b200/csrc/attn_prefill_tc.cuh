@@ -73,7 +73,7 @@ LIGER_DEV uint64_t umma_desc_sw128_mn(uint32_t smem_addr, uint32_t lbo, uint32_t
 template <int D>
 __global__ void __launch_bounds__(PT_THREADS, 1)
     attn_prefill_tc_kernel(const __grid_constant__ CUtensorMap tm, __nv_bfloat16* __restrict__ o,
-                           const __nv_bfloat16* __restrict__ qkv, __nv_bfloat16* __restrict__ kv_pool,
+                           __nv_bfloat16* __restrict__ kv_pool,
                            const int32_t* __restrict__ page_table, int max_pages, int b, int s, int heads) {
   using L = PtSmem<D>;
   extern __shared__ uint8_t pt_raw[];

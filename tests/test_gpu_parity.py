@@ -41,7 +41,9 @@ def test_c0_device_matches_numpy_bit_exact(L):
 
 # ---------------------------------------------------------------- GEMM
 GEMM_SHAPES = [(1, 128, 64), (2, 384, 256), (16, 256, 128), (37, 200, 320), (64, 512, 1024), (65, 640, 768),
-               (300, 384, 512), (513, 256, 256), (1024, 1024, 512)]
+               (300, 384, 512), (513, 256, 256), (1024, 1024, 512),
+               # prefill token tiles below 256 chosen for wave fill (bn 144 / 224, ragged last tile)
+               (1000, 5120, 512), (1500, 2560, 1024)]
 
 
 @pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
@@ -85,7 +87,8 @@ def test_gemm_decomposition_bit_exact(L, M, N, K):
         assert torch.equal(out, full), ks
 
 
-@pytest.mark.parametrize("name,t,M", [("opt-13b", 1, 8), ("opt-13b", 1, 512), ("opt-13b", 1, 4096),
+@pytest.mark.parametrize("name,t,M", [("opt-13b", 1, 8), ("opt-13b", 1, 512), ("opt-13b", 1, 1024),
+                                      ("opt-13b", 1, 2048), ("opt-13b", 1, 4096),
                                       ("opt-30b", 4, 8), ("opt-66b", 8, 2), ("glm-130b", 8, 2),
                                       ("glm-130b", 8, 2048)])
 def test_gemm_full_size_sampled(L, name, t, M):

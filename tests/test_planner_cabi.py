@@ -208,12 +208,24 @@ def test_gemm_plan_host_logic(L):
             tiles = -(-N // 128) * pl["m_tiles"]
             if M > 64 and tiles >= 148:
                 assert pl["splits"] == 1
+            # token tiling: decode one tile of M rounded to 16; prefill m_tiles = ceil(M / bn)
+            # with bn = 256-wide tiles, or (unsplit only) a smaller tile of at least 144
+            if M <= 64:
+                assert pl["m_tiles"] == 1 and pl["bn"] == max(16, -(-M // 16) * 16)
+            else:
+                assert pl["m_tiles"] == -(-M // pl["bn"])
+                assert pl["m_tiles"] == -(-M // 256) or (pl["bn"] >= 144 and pl["splits"] == 1)
     # decode shapes (profiles/r01/split_sweep_decode.txt): QKV one chunk, out-proj 3,
     # FC1 8-10, FC2 3-7 -- within 3 % of the best measured at every shape
     assert L.gemm_plan(8, 15360, 5120)["splits"] == 1
     assert L.gemm_plan(8, 5120, 5120)["splits"] == 3
     assert 8 <= L.gemm_plan(8, 20480, 5120)["splits"] <= 10
     assert 3 <= L.gemm_plan(8, 5120, 20480)["splits"] <= 7
+    # prefill wave fill (profiles/r02/gemm_prefill_tiling.txt): out-proj at M = 1024 runs
+    # 7 tiles of 160 tokens (280 units in 2 rounds; 4 x 256 left the second round 8 % full,
+    # 75 -> 56-58 us on B200); QKV at M = 4096 keeps 256-token tiles
+    assert L.gemm_plan(1024, 5120, 5120)["bn"] == 160
+    assert L.gemm_plan(4096, 15360, 5120)["bn"] == 256
 
 
 def test_missing_library_fails_loudly(monkeypatch, tmp_path):
