@@ -656,6 +656,8 @@ def main():
     if args.workload == "generative":
         args.n_new = 2
     if args.fused_ar:
+        if args.loopback:   # loopback ranks share one GPU: no peer-memory kernels there
+            ap.error("--fused-ar needs one GPU per rank (not --loopback)")
         os.environ["LIGER_FUSED_AR"] = "1"
         os.environ["LIGER_ONESHOT_AR"] = "1"
     # N > 1 without torchrun: re-launch under torch.distributed.run, one process per GPU

@@ -230,13 +230,43 @@ int liger_op_allreduce(liger_ctx* ctx, void* buf, size_t count, int u0, int u1, 
  * regions are regions[0..world) (regions[rank] = this rank's own), call number `epoch`
  * (1, 2, ... in the same order on every rank): stage, publish the epoch (system-scope
  * release), wait for every peer's flag (10 s watchdog trap), sum in rank order in fp32,
- * round to bf16.  count * 2 <= cap, 16-byte multiples.  LIGER_EINVAL / LIGER_ECUDA. */
+ * round to bf16.  count * 2 <= cap, 16-byte multiples.  LIGER_EINVAL / LIGER_ECUDA.
+ * phases selects the kernel's halves: LIGER_AR_PHASE_STAGE (copy buf into this rank's
+ * staging buffer of the epoch and publish the flag), LIGER_AR_PHASE_REDUCE (wait for all
+ * flags, sum), or both (what the serving path runs, one launch per rank with the ranks on
+ * different GPUs).  Ranks that share ONE GPU must not run kernels that wait on each other
+ * concurrently (nothing guarantees they are co-scheduled; B200_PROFILING.md): there every
+ * rank runs STAGE, the host synchronises, then every rank runs REDUCE (whose waits are
+ * then already satisfied) -- the same kernel code, the same bits. */
+#define LIGER_AR_PHASE_STAGE 1
+#define LIGER_AR_PHASE_REDUCE 2
 int liger_ipc_region_create(size_t cap, void** region, uint8_t* handle);
 int liger_ipc_region_open(const uint8_t* handle, void** peer);
 int liger_ipc_region_close(void* peer);
 int liger_ipc_region_free(void* region);
 int liger_op_oneshot_allreduce(void* buf, size_t count, void* const* regions, int world, int rank, size_t cap,
-                               uint64_t epoch, void* stream);
+                               uint64_t epoch, int phases, void* stream);
+
+/* The fused row-parallel GEMM + all-reduce of serial TP (§8(f) next row 4; DESIGN.md §8
+ * "Fused row-parallel GEMM + all-reduce"), its two halves on explicit regions, call number
+ * `epoch` as above (one epoch per fused all-reduce, the same sequence as the one-shot's).
+ * liger_op_gemm_fused_ar_stage: the split-K GEMM P = x[M, K] . W^T (W tiled as for
+ * liger_op_gemm_tiled, no bias / activation: the row-parallel partial) whose
+ * split-K fixup writes bf16(P) row-major [M, N] into this rank's staging buffer of the
+ * epoch and, once every fixup CTA's stores are visible, publishes the epoch flag.
+ * LIGER_EINVAL unless the plan of (M, N, K) splits K (the fixup is the producer) and
+ * M * N * 2 <= cap.
+ * liger_op_add_layernorm_fused_ar: waits for every rank's flag, then for each row i < rows
+ *   r = x[i] + sum_{q = 0..world-1} staged_q[i] (fp32, in rank order, bf16 of the sum as
+ *       the one-shot all-reduce rounds it) + add_bias,
+ * and x_out / y as liger_op_add_layernorm (h = N).  Same one-GPU rule as the one-shot:
+ * every rank's stage call completes before any rank's add + LN call is launched. */
+int liger_op_gemm_fused_ar_stage(const void* x, int64_t ldx, const void* w_tiled, int M, int N, int K,
+                                 void* const* regions, int world, int rank, size_t cap, uint64_t epoch,
+                                 void* workspace, size_t ws_bytes, void* stream);
+int liger_op_add_layernorm_fused_ar(void* const* regions, int world, int rank, size_t cap, uint64_t epoch,
+                                    const void* x, const void* add_bias, void* x_out, void* y, const void* gamma,
+                                    const void* beta, int rows, int h, float eps, void* stream);
 
 /* Debug readback for parity tests (not part of the serving path).
  * liger_set_debug_capture(ctx, arena_bytes) [collective]: arena_bytes > 0 turns capture

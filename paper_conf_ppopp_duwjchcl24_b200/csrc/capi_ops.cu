@@ -177,14 +177,49 @@ int liger_ipc_region_close(void* peer) { return cudaIpcCloseMemHandle(peer) == c
 int liger_ipc_region_free(void* region) { return cudaFree(region) == cudaSuccess ? LIGER_OK : LIGER_ECUDA; }
 
 int liger_op_oneshot_allreduce(void* buf, size_t count, void* const* regions, int world, int rank, size_t cap,
-                               uint64_t epoch, void* stream) {
+                               uint64_t epoch, int phases, void* stream) {
   if (int rc = check_device()) return rc;
-  if (!buf || !regions || world < 1 || world > 8 || rank < 0 || rank >= world || epoch == 0)
+  if (!buf || !regions || world < 1 || world > 8 || rank < 0 || rank >= world || epoch == 0 || phases < 1 ||
+      phases > 3)
     return LIGER_EINVAL;
   PeerAR par;
   if (int rc = par.init(world, rank, cap, regions[rank], regions)) return ret(rc, "liger_op_oneshot_allreduce");
   par.epoch = epoch - 1;   // this call is epoch `epoch` (allreduce_bf16 pre-increments)
-  return ret(par.allreduce_bf16(buf, count, (cudaStream_t)stream), "liger_op_oneshot_allreduce");
+  return ret(par.allreduce_bf16(buf, count, (cudaStream_t)stream, phases), "liger_op_oneshot_allreduce");
+}
+
+// the fused producer / consumer descriptor of call `epoch` on explicit regions
+static int fused_desc(void* const* regions, int world, int rank, size_t cap, uint64_t epoch, size_t bytes,
+                      FusedARDesc* far) {
+  if (!regions || world < 1 || world > 8 || rank < 0 || rank >= world || epoch == 0) return LIGER_EINVAL;
+  PeerAR par;
+  if (int rc = par.init(world, rank, cap, regions[rank], regions)) return rc;
+  par.epoch = epoch - 1;   // fused_begin pre-increments
+  return par.fused_begin(bytes, far);
+}
+
+int liger_op_gemm_fused_ar_stage(const void* x, int64_t ldx, const void* w_tiled, int M, int N, int K,
+                                 void* const* regions, int world, int rank, size_t cap, uint64_t epoch,
+                                 void* workspace, size_t ws_bytes, void* stream) {
+  if (int rc = check_device()) return rc;
+  FusedARDesc far{};
+  if (int rc = fused_desc(regions, world, rank, cap, epoch, (size_t)M * N * 2, &far))
+    return ret(rc, "liger_op_gemm_fused_ar_stage");
+  GemmArgs a{x, ldx, w_tiled, 64, nullptr, N, M, N, K, 0, N, nullptr, LIGER_ACT_NONE, 0, 1.0f, 0, workspace,
+             ws_bytes, 1};
+  a.far = &far;
+  return ret(gemm_launch(a, (cudaStream_t)stream), "liger_op_gemm_fused_ar_stage");
+}
+
+int liger_op_add_layernorm_fused_ar(void* const* regions, int world, int rank, size_t cap, uint64_t epoch,
+                                    const void* x, const void* add_bias, void* x_out, void* y, const void* gamma,
+                                    const void* beta, int rows, int h, float eps, void* stream) {
+  if (int rc = check_device()) return rc;
+  FusedARDesc far{};
+  if (int rc = fused_desc(regions, world, rank, cap, epoch, (size_t)rows * h * 2, &far))
+    return ret(rc, "liger_op_add_layernorm_fused_ar");
+  return ret(peer_add_layernorm_launch(far, x, add_bias, x_out, y, gamma, beta, rows, h, eps, (cudaStream_t)stream),
+             "liger_op_add_layernorm_fused_ar");
 }
 
 }  // extern "C"

@@ -313,13 +313,8 @@ struct LoopbackComm : Comm {
   cudaEvent_t ev_ready = nullptr, ev_done = nullptr;
   void* scratch = nullptr;
   size_t scratch_bytes = 0;
-  bool oneshot = true;
-  PeerAR* par = nullptr;
-  void* region = nullptr;
   ~LoopbackComm() override {
     cudaDeviceSynchronize();
-    delete par;
-    if (region) cudaFree(region);
     if (ev_ready) cudaEventDestroy(ev_ready);
     if (ev_done) cudaEventDestroy(ev_done);
     if (scratch) cudaFree(scratch);
@@ -360,39 +355,13 @@ struct LoopbackComm : Comm {
     scratch_bytes = bytes;
     return 0;
   }
-  // [collective, at communicator creation] the ranks' staging regions are plain device
-  // pointers of one process; every rank reaches the rendezvous whatever its allocation
-  // outcome, and all fall back together if any rank has no region
-  int setup_oneshot() {
-    const size_t cap = oneshot_cap(), rb = peer_ar_region_bytes(cap);
-    if (cudaMalloc(&region, rb) != cudaSuccess || cudaMemset(region, 0, rb) != cudaSuccess) {
-      cudaGetLastError();
-      if (region) cudaFree(region);
-      region = nullptr;
-    }
-    cudaDeviceSynchronize();
-    std::vector<const void*> xs, ys;
-    std::vector<cudaEvent_t> es;
-    rendezvous(region, nullptr, nullptr, &xs, &ys, &es);
-    void* peers[8] = {};
-    bool all = true;
-    for (int q = 0; q < world; ++q) {
-      peers[q] = const_cast<void*>(xs[q]);
-      all = all && peers[q];
-    }
-    if (!all) {
-      oneshot = false;
-      err = "one-shot all-reduce disabled: a rank could not allocate its staging buffer";
-      return 0;
-    }
-    par = new PeerAR();
-    return par->init(world, rank, cap, region, peers);
-  }
-  int init_peer(cudaStream_t) override { return oneshot ? setup_oneshot() : 0; }
-  PeerAR* peer_ar(cudaStream_t) override { return oneshot ? par : nullptr; }
+  // No peer-memory kernels on this backend: its ranks share one GPU, and kernels that
+  // wait on each other are not guaranteed to be co-scheduled there (B200_PROFILING.md).
+  // The one-shot / fused kernels are tested phase by phase through the op-level C-ABI.
+  int init_peer(cudaStream_t) override { return 0; }
+  PeerAR* peer_ar(cudaStream_t) override { return nullptr; }
   int allreduce(void* buf, size_t count, CommDType dt, CommOp op, cudaStream_t st) override {
     if (!count) return 0;
-    if (oneshot && par && oneshot_eligible(count, dt, op, buf)) return par->allreduce_bf16(buf, count, st);
     const size_t bytes = count * dt_size(dt);
     if (int rc = ensure_scratch(bytes)) return rc;
     std::vector<const void*> xs, ys;
@@ -504,7 +473,6 @@ Comm* comm_create(int world, int rank, const uint8_t* uid, std::string* err) {
     auto* c = new LoopbackComm();
     c->world = world;
     c->rank = rank;
-    c->oneshot = oneshot_enabled(true);
     c->key.assign((const char*)uid, 48);
     {
       std::lock_guard<std::mutex> l(g_groups_mu);

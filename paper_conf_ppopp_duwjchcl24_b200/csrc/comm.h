@@ -40,7 +40,9 @@ struct PeerAR {
   unsigned int* counter = nullptr;
   uint64_t epoch = 0;
   int init(int world, int rank, size_t cap, void* local_region, void* const* peer_regions);
-  int allreduce_bf16(void* buf, size_t count, cudaStream_t st);   // in place, sum in rank order
+  // in place, sum in rank order; phases = LIGER_AR_PHASE_STAGE (stage + publish) |
+  // LIGER_AR_PHASE_REDUCE (wait for every flag + sum); the serving path runs both
+  int allreduce_bf16(void* buf, size_t count, cudaStream_t st, int phases = 3);
   unsigned int* fused_counter = nullptr;
   // take the next epoch for a fused producer/consumer pair (same order on all ranks)
   int fused_begin(size_t bytes, FusedARDesc* out);

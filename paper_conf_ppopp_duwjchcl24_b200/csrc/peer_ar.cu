@@ -16,9 +16,12 @@
 // rewritten at call e + 2 only after this rank passed call e + 1's flag wait, i.e.
 // after every peer finished call e (stream order), so two buffers suffice.
 //
-// Transports: NVLink peers map each other's staging with CUDA IPC handles
-// (exchanged by the NCCL communicator); the loopback test backend (t ranks as
-// threads on one GPU) shares plain device pointers -- the kernel is the same.
+// Transport: NVLink peers map each other's staging with CUDA IPC handles
+// (exchanged by the NCCL communicator), one rank per GPU.  The loopback test
+// backend (t ranks sharing one GPU) never uses it: kernels that wait on each other
+// are not guaranteed to be co-scheduled on one GPU.  There the kernel is tested
+// phase by phase (`phases`): every rank's STAGE launch, a host sync, then every
+// rank's REDUCE launch, whose flag waits are already satisfied.
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
@@ -55,24 +58,33 @@ __device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned l
 __global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf, size_t n8, uint4* my_stage,
                                                                       unsigned long long* my_flag,
                                                                       unsigned int* counter, PeerPtrs peers,
-                                                                      int world, unsigned long long epoch) {
+                                                                      int world, unsigned long long epoch,
+                                                                      int phases) {
   const size_t stride = (size_t)gridDim.x * blockDim.x;
   // The partials come from the preceding GEMM.  Dependents are released only after
   // every peer has arrived (below): a kernel parked at its griddepcontrol.wait
   // must not hold SM resources while this one spins on other ranks -- on the
   // loopback backend those ranks share this GPU and would need them to progress.
   grid_dependency_wait();
-  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += stride) my_stage[i] = buf[i];
-  __threadfence_system();   // every thread's staging stores before the block's publish
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence_system();
-    const unsigned int prev = atomicAdd(counter, 1u);
-    if (prev == gridDim.x - 1) {   // every block's staging copy is done: publish
-      *counter = 0;
+  if (phases & LIGER_AR_PHASE_STAGE) {
+    for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += stride) my_stage[i] = buf[i];
+    __threadfence_system();   // every thread's staging stores before the block's publish
+    __syncthreads();
+    if (threadIdx.x == 0) {
       __threadfence_system();
-      st_release_sys(my_flag, epoch);
+      const unsigned int prev = atomicAdd(counter, 1u);
+      if (prev == gridDim.x - 1) {   // every block's staging copy is done: publish
+        *counter = 0;
+        __threadfence_system();
+        st_release_sys(my_flag, epoch);
+      }
     }
+  }
+  if (!(phases & LIGER_AR_PHASE_REDUCE)) {
+    grid_dependency_trigger();
+    return;
+  }
+  if (threadIdx.x == 0) {
     const uint64_t t0 = trace_now();
     for (int q = 0; q < world; ++q)
       while (ld_acquire_sys(peers.flag[q]) < epoch) {
@@ -168,9 +180,10 @@ int PeerAR::fused_begin(size_t bytes, FusedARDesc* out) {
   return 0;
 }
 
-int PeerAR::allreduce_bf16(void* buf, size_t count, cudaStream_t st) {
+int PeerAR::allreduce_bf16(void* buf, size_t count, cudaStream_t st, int phases) {
   const size_t bytes = count * 2;
-  if (bytes > cap || bytes % 16 || reinterpret_cast<uintptr_t>(buf) % 16) return LIGER_EINVAL;
+  if (bytes > cap || bytes % 16 || reinterpret_cast<uintptr_t>(buf) % 16 || phases < 1 || phases > 3)
+    return LIGER_EINVAL;
   if (!count) return 0;
   ++epoch;
   if (dbg_epochs()) fprintf(stderr, "[rank %d] epoch %llu one-shot %zu B\n", rank, (unsigned long long)epoch, bytes);
@@ -187,7 +200,7 @@ int PeerAR::allreduce_bf16(void* buf, size_t count, cudaStream_t st) {
   uint4* stage = reinterpret_cast<uint4*>(static_cast<char*>(local) + (size_t)b * cap);
   unsigned long long* flag = reinterpret_cast<unsigned long long*>(static_cast<char*>(local) + 2 * cap);
   return launch_pdl(oneshot_ar_bf16_kernel, dim3(blocks), dim3(PAR_THREADS), 0, st, reinterpret_cast<uint4*>(buf),
-                    n8, stage, flag, counter, pp, world, (unsigned long long)epoch)
+                    n8, stage, flag, counter, pp, world, (unsigned long long)epoch, phases)
              ? LIGER_ECUDA
              : 0;
 }

@@ -72,7 +72,9 @@ _SIGS = {
     "liger_ipc_region_open": (_I, [_P, C.POINTER(_P)]),
     "liger_ipc_region_close": (_I, [_P]),
     "liger_ipc_region_free": (_I, [_P]),
-    "liger_op_oneshot_allreduce": (_I, [_P, _SZ, _P, _I, _I, _SZ, _U64, _P]),
+    "liger_op_oneshot_allreduce": (_I, [_P, _SZ, _P, _I, _I, _SZ, _U64, _I, _P]),
+    "liger_op_gemm_fused_ar_stage": (_I, [_P, _I64, _P, _I, _I, _I, _P, _I, _I, _SZ, _U64, _P, _SZ, _P]),
+    "liger_op_add_layernorm_fused_ar": (_I, [_P, _I, _I, _SZ, _U64, _P, _P, _P, _P, _P, _P, _I, _I, _F, _P]),
     "liger_op_allreduce": (_I, [_P, _P, _SZ, _I, _I, _I, _P]),
     "liger_debug_read": (_I, [_P, _I64, _I, _P, _SZ]),
     "liger_stats": (_I, [_P, C.POINTER(liger_stats_t)]),
@@ -188,11 +190,33 @@ def ipc_region_open(handle):
     return p.value
 
 
-def oneshot_allreduce(buf, regions, rank, cap, epoch, stream=None):
+AR_PHASE_STAGE, AR_PHASE_REDUCE = 1, 2
+
+
+def oneshot_allreduce(buf, regions, rank, cap, epoch, phases=AR_PHASE_STAGE | AR_PHASE_REDUCE, stream=None):
     """liger_op_oneshot_allreduce on torch bf16 buffer `buf` (in place)."""
     arr = (C.c_void_p * len(regions))(*regions)
-    check(lib().liger_op_oneshot_allreduce(_p(buf), buf.numel(), arr, len(regions), rank, cap, epoch, _s(stream)),
+    check(lib().liger_op_oneshot_allreduce(_p(buf), buf.numel(), arr, len(regions), rank, cap, epoch, phases,
+                                           _s(stream)),
           what="liger_op_oneshot_allreduce")
+
+
+def gemm_fused_ar_stage(x, w_tiled, M, N, K, regions, rank, cap, epoch, workspace, stream=None):
+    """liger_op_gemm_fused_ar_stage: split-K GEMM whose fixup stages bf16(x W^T) and publishes."""
+    arr = (C.c_void_p * len(regions))(*regions)
+    check(lib().liger_op_gemm_fused_ar_stage(_p(x), x.stride(0), _p(w_tiled), M, N, K, arr, len(regions), rank, cap,
+                                             epoch, _p(workspace), workspace.numel() * workspace.element_size(),
+                                             _s(stream)),
+          what="liger_op_gemm_fused_ar_stage")
+
+
+def add_layernorm_fused_ar(regions, rank, cap, epoch, x, add_bias, x_out, y, gamma, beta, eps=1e-5, stream=None):
+    """liger_op_add_layernorm_fused_ar: x + sum of the ranks' staged rows + bias, then LN."""
+    arr = (C.c_void_p * len(regions))(*regions)
+    rows, h = x.shape
+    check(lib().liger_op_add_layernorm_fused_ar(arr, len(regions), rank, cap, epoch, _p(x), _p(add_bias), _p(x_out),
+                                                _p(y), _p(gamma), _p(beta), rows, h, eps, _s(stream)),
+          what="liger_op_add_layernorm_fused_ar")
 
 
 def tile_weight(w, w_tiled, stream=None):

@@ -4,7 +4,14 @@ peer-visible staging region (liger_ipc_region_create), exchange the 64-byte IPC 
 a gloo process group, map the peer's region (liger_ipc_region_open) and run
 liger_op_oneshot_allreduce -- stage, system-scope epoch flag, rank-ordered fp32 sum -- on
 seeded bf16 partials, element-wise against the oracle's sum (bit-exact at t = 2: the sum of
-two bf16 values is exact in fp32 and rounds once).  Both ranks must end with the same bits."""
+two bf16 values is exact in fp32 and rounds once).  Both ranks must end with the same bits.
+
+The two processes share one GPU, where kernels that wait on each other are not guaranteed
+to be co-scheduled (B200_PROFILING.md: such process pairs raised Xid 109).  Each call
+therefore runs in two phases: both ranks stage + publish (LIGER_AR_PHASE_STAGE) and
+synchronise, a gloo barrier, then both wait + sum (LIGER_AR_PHASE_REDUCE) -- whose flag
+waits are already satisfied -- so the peer loads, flags and IPC mappings are exercised
+across processes without any kernel spinning on another process's kernel."""
 import os
 
 import numpy as np
@@ -32,8 +39,12 @@ def _rank(r, port, q):
         for e, n in enumerate((8 * 5120, 16 * 1024, 256), start=1):
             x = c0_values(5, 200 + r, np.arange(n, dtype=np.uint64) + 1000 * e, -3)
             buf = torch.from_numpy(x.astype(np.float32)).cuda().bfloat16()
-            L.oneshot_allreduce(buf, regions, r, CAP, e)
+            L.oneshot_allreduce(buf, regions, r, CAP, e, phases=L.AR_PHASE_STAGE)
             torch.cuda.synchronize()
+            dist.barrier()
+            L.oneshot_allreduce(buf, regions, r, CAP, e, phases=L.AR_PHASE_REDUCE)
+            torch.cuda.synchronize()
+            dist.barrier()
             out.append(buf.view(torch.int16).cpu().numpy().tobytes())
         dist.barrier()
         for k in range(2):

@@ -97,7 +97,7 @@ def _engine(world, env):
     from liger_inputs import get_config, make_trace
     from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
     from liger_inputs.configs import ModelConfig
-    cfg = ModelConfig("mid2", 2, 1024, 8, 4096, 1024, 96, "relu") if env.get("LIGER_FUSED_AR") else get_config("tiny")
+    cfg = get_config("tiny")
     trace = make_trace(2, float("inf"), seed=1, batch_sizes=(1, 2), prompt_range=(8, 24), n_decode=3,
                        vocab=cfg.vocab)
     uid = LigerEngine.loopback_id() if world > 1 else None
@@ -107,8 +107,8 @@ def _engine(world, env):
     def run(r):
         try:
             torch.cuda.set_device(0)
-            e = LigerEngine(cfg, world=world, rank=r, nccl_uid=uid, mode="serial" if env.get("LIGER_FUSED_AR") else
-                            "interleaved", max_batch=2, max_seq=32, max_new=4, seed=0)
+            e = LigerEngine(cfg, world=world, rank=r, nccl_uid=uid, mode="interleaved", max_batch=2, max_seq=32,
+                            max_new=4, seed=0)
             ids = [e.submit(t["tokens"], t["batch"], t["seq_len"], t["n_decode"], 0.0) for t in trace]
             e.drain()
             toks[r] = [e.poll(i, want_tokens=True)[1].tolist() for i in ids]
@@ -125,11 +125,22 @@ def _engine(world, env):
     print(f"engine world={world} {env}: tokens {toks[0]}")
 
 
+def _peer_ar_phased():
+    """One-shot and fused GEMM + all-reduce kernels at t = 2, phase by phase on one GPU
+    (every rank's stage / publish launch completes before any rank's wait / sum launch)."""
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+    import test_gpu_peer_ar as T
+    from paper_conf_ppopp_duwjchcl24_b200 import liger
+    T.test_oneshot_allreduce_phased_vs_oracle(liger, 2)
+    T.test_fused_gemm_allreduce_phased_vs_oracle(liger, 2)
+    print("peer_ar phased ok")
+
+
 CASES = {
     "gemm_splitk": gemm_splitk, "attn_decode": attn_decode, "attn_prefill": attn_prefill, "add_ln": add_ln,
     "engine_t1": lambda: _engine(1, {}),
-    "engine_tp2_oneshot": lambda: _engine(2, {"LIGER_ONESHOT_AR": "1"}),
-    "engine_tp2_fused": lambda: _engine(2, {"LIGER_FUSED_AR": "1"}),
+    "engine_tp2_loopback": lambda: _engine(2, {}),
+    "peer_ar_phased": lambda: _peer_ar_phased(),
 }
 
 if __name__ == "__main__":
