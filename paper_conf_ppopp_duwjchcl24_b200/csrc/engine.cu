@@ -1296,13 +1296,18 @@ int liger_step(liger_ctx* c) {
     c->have_round = false;
     n = (int)pieces.size();
   } else if (c->t1_streams && !c->timing) {
-    // t = 1: every in-flight batch's whole list, in order, on the stream of its slot
-    // (per-launch kernel timing runs the batches one at a time instead)
+    // t = 1: one pass of every in-flight batch per step, in turn, each on the stream of
+    // its slot (per-launch kernel timing runs the batches one at a time instead).  A
+    // stream's launch queue is bounded: enqueueing one batch's whole list at once blocked
+    // the host on that stream until the batch had nearly finished, so the other stream
+    // stayed empty and the two batches' kernels never overlapped (in-kernel trace,
+    // tools/timeline_capacity.py); pass by pass, both streams always hold work.
     for (Batch* bt : c->processing) {
       if (bt->all_launched) continue;
       const size_t p0 = pieces.size();
       BatchCursor cur(c, bt, &pieces);
-      while (!cur.empty()) cur.take(cur.head_left());
+      const int pass = bt->pass;
+      while (!cur.empty() && bt->pass == pass) cur.take(cur.head_left());
       std::vector<int> mine;
       for (size_t i = p0; i < pieces.size(); ++i) mine.push_back((int)i);
       CKR(launch_run(c, pieces, mine, bt->slot & 1));
