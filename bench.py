@@ -501,13 +501,14 @@ def rank_main(args, group, local, uid, result):
         ids_d = torch.from_numpy(np.random.default_rng(3).integers(0, cfg.vocab, size=bsz * slen)
                                  .astype(np.int32)).cuda()
 
-        def batch_ms(n_new):
+        def batch_ms(n_new, k=1):
             best = 1e30
             for _ in range(2):
                 group.barrier()
                 a, z = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 a.record()
-                eng.submit(None, bsz, slen, n_new, 0.0, device_tokens=ids_d)
+                for _ in range(k):
+                    eng.submit(None, bsz, slen, n_new, 0.0, device_tokens=ids_d)
                 eng.drain()
                 z.record()
                 z.synchronize()
@@ -525,6 +526,17 @@ def rank_main(args, group, local, uid, result):
                        "unit": "GB/s", "frac": round(gbs / hbm, 4),
                        "note": "whole decode pass (all kernels, PDL chain intact), CUDA events around "
                                "batches with n_new and 1 generated tokens; bytes = weights + KV read"}
+        if args.inflight >= 2 and args.mode == "interleaved":
+            # the same with two such batches served together: what the schedule that ran
+            # streams while both batches decode (at t = 1 their passes run concurrently on
+            # the two streams, R31), per pass of one batch
+            t1b, tnb = batch_ms(1, 2), batch_ms(args.n_new, 2)
+            pass2 = (tnb - t1b) / (2 * (args.n_new - 1)) * 1e3
+            gbs2 = (w_bytes + kv_bytes) / (pass2 * 1e-6) / 1e9
+            decode_pass["two_batches"] = {"us_per_pass_per_batch": round(pass2, 1), "achieved": round(gbs2, 1),
+                                          "frac": round(gbs2 / hbm, 4),
+                                          "note": "two equal batches served together (both decode "
+                                                  "concurrently); aggregate weight + KV stream"}
 
     # ---- NVLink all-reduce sweep (N > 1)
     ar_sweep = allreduce_sweep(eng, group, torch, F=args.F) if world > 1 and not args.quick else None
