@@ -59,7 +59,6 @@ struct GemmParams {
   int kc, splits;
   int bn;
   int stages;
-  int acc_stages;       // TMEM accumulator stages (1, 2 or 4)
   int n_tiles, m_tiles;
   int units;            // n_tiles * m_tiles * splits
   int w_tiled;          // W stored as [N/128][K/64][128][64] (each TMA box contiguous)
@@ -199,7 +198,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
   const int lane = threadIdx.x & 31;
   const int G = gridDim.x;
   const uint32_t acc_cols = p.bn <= 32 ? 32 : (p.bn <= 64 ? 64 : (p.bn <= 128 ? 128 : 256));
-  const int TS = p.acc_stages;                     // TMEM accumulator stages (epilogue slack)
+  const int TS = acc_cols >= 256 ? 2 : 4;          // TMEM accumulator stages (epilogue slack)
   const uint32_t tmem_cols = (uint32_t)TS * acc_cols;
 
   if (threadIdx.x == 0) {
@@ -576,14 +575,6 @@ static int stages_for(int bn, int extra_smem, int budget) {
 }
 
 constexpr int LN_STATS_SMEM = 2 * 64 * 4;   // folded-LayerNorm row statistics (M <= 64)
-constexpr int SM_SMEM = 228 * 1024;          // shared memory of one SM (all its CTAs)
-constexpr int COLOC_DECODE_STAGES = 4;
-
-// experiment: plans that let a prefill GEMM CTA and a decode GEMM CTA share an SM
-static bool coloc_enabled() {
-  static const bool on = getenv("LIGER_COLOC") && atoi(getenv("LIGER_COLOC")) != 0;
-  return on;
-}
 
 // Tiling policy.  A decomposition piece of a GEMM (a column slice [n0, n1)) keeps
 // the full GEMM's (M, N, K), so every per-element quantity -- the token tiling
@@ -684,21 +675,7 @@ GemmPlan gemm_plan(int M, int N, int K) {
   pl.m_tiles = mt;
   pl.kc = kcb * BK;
   pl.splits = (nkb + kcb - 1) / kcb;
-  const int acc_cols = bn <= 32 ? 32 : (bn <= 64 ? 64 : (bn <= 128 ? 128 : 256));
-  pl.acc_stages = acc_cols >= 256 ? 2 : 4;
-  int budget = MAX_SMEM;
-  if (coloc_enabled()) {
-    // co-residency of a prefill GEMM CTA with a decode GEMM CTA of the other stream on
-    // one SM: decode <= COLOC_DECODE_STAGES stages, prefill in the rest of the SM's
-    // shared memory and <= 256 TMEM columns (one accumulator stage)
-    if (M <= 64) {
-      budget = std::min(budget, 1024 + COLOC_DECODE_STAGES * (A_BYTES + bn * BK * 2) + 512 + LN_STATS_SMEM);
-    } else {
-      budget = SM_SMEM - 2048 - (1024 + COLOC_DECODE_STAGES * (A_BYTES + 16 * BK * 2) + 512 + LN_STATS_SMEM);
-      if (acc_cols >= 256) pl.acc_stages = 1;
-    }
-  }
-  pl.stages = stages_for(bn, LN_STATS_SMEM, budget);
+  pl.stages = stages_for(bn, LN_STATS_SMEM, MAX_SMEM);
   pl.smem = 1024 + pl.stages * (A_BYTES + pl.bn * BK * 2) + 512 + LN_STATS_SMEM;
   return pl;
 }
@@ -742,7 +719,7 @@ int gemm_launch(const GemmArgs& a, cudaStream_t stream) {
   }
   GemmParams p;
   p.M = a.M; p.N = a.N; p.K = a.K; p.n0 = a.n0; p.n1 = a.n1;
-  p.kc = pl.kc; p.splits = pl.splits; p.bn = pl.bn; p.stages = pl.stages; p.acc_stages = pl.acc_stages;
+  p.kc = pl.kc; p.splits = pl.splits; p.bn = pl.bn; p.stages = pl.stages;
   p.bias = reinterpret_cast<const __nv_bfloat16*>(a.bias);
   p.act = a.act; p.scale_cols = a.scale_cols; p.scale = a.scale;
   p.out = a.out; p.ldo = a.ldo; p.out_f32 = a.out_f32;

@@ -13,7 +13,6 @@ constexpr size_t ATTN_COUNTER_BYTES = 16384;
 
 struct GemmPlan {
   int bn, m_tiles, kc, splits, stages, smem;
-  int acc_stages;   // TMEM accumulator stages (epilogue / next-unit MMA overlap)
 };
 
 // Descriptor of one fused all-reduce (epoch) for kernels that do the one-shot
