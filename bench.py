@@ -378,6 +378,49 @@ def allreduce_sweep(eng, group, torch, F=8):
 
 
 # ----------------------------------------------------------------------------- one rank
+TRACE_KINDS = {1: "gemm", 2: "splitk_fixup", 3: "attn_decode", 4: "attn_prefill", 5: "add_ln", 6: "embed",
+               7: "argmax", 8: "argmax_pick", 9: "fused_ar", 3 | 256: "attn_decode_merge"}
+
+
+def capacity_trace(eng, trace, torch):
+    """Where the schedule that ran spends the GPU: the in-kernel %globaltimer record of every
+    CTA (kind, SM, PDL-wait release, exit) while `trace` is served as in the timed region.
+    Per kernel kind, its share of the SMs' time (sum over CTAs of release -> exit, divided
+    by SMs x span), and the fraction of the span in which no GEMM CTA works."""
+    from paper_conf_ppopp_duwjchcl24_b200 import liger as L
+    cap = 1 << 23
+    torch.cuda.synchronize()
+    L.trace_start(cap)
+    for r in trace:
+        eng.submit(r["tokens"], r["batch"], r["seq_len"], r["n_decode"], 0.0)
+    eng.drain()
+    torch.cuda.synchronize()
+    rec = L.trace_stop(cap)
+    if len(rec) == 0 or len(rec) >= cap:
+        return None
+    t0 = int(rec["t0"].min())
+    a = (rec["t1"].astype(np.int64) - t0).astype(np.float64)
+    z = (rec["t2"].astype(np.int64) - t0).astype(np.float64)
+    span = float(z.max())
+    nsm = int(rec["smid"].max()) + 1
+    share = {}
+    for k in np.unique(rec["kid"]):
+        m = rec["kid"] == k
+        share[TRACE_KINDS.get(int(k), str(int(k)))] = round(float((z[m] - a[m]).sum()) / (nsm * span), 4)
+    g = rec["kid"] == 1
+    ev = np.concatenate([a[g], z[g]])
+    dv = np.concatenate([np.ones(int(g.sum())), -np.ones(int(g.sum()))])
+    o = np.argsort(ev, kind="stable")
+    busy = np.cumsum(dv[o])[:-1] > 0
+    gemm_cov = float(np.diff(ev[o])[busy].sum()) / span
+    return {"batches": len(trace), "span_ms": round(span / 1e6, 2), "sms": nsm, "cta_records": int(len(rec)),
+            "sm_time_share": share, "no_gemm_working_frac": round(1.0 - gemm_cov, 4),
+            "note": "in-kernel %globaltimer trace of every CTA while these batches are served as in the timed "
+                    "region (release of the PDL wait -> exit); sm_time_share = CTA-time / (SMs x span); "
+                    "embedding and argmax kernels are not traced; attn_decode_merge = decode-attention CTAs "
+                    "that also merged the splits"}
+
+
 def rank_main(args, group, local, uid, result):
     import torch
     from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
@@ -538,6 +581,12 @@ def rank_main(args, group, local, uid, result):
                                           "note": "two equal batches served together (both decode "
                                                   "concurrently); aggregate weight + KV stream"}
 
+    # ---- where the GPU time goes in the schedule that ran (N = 1: one traced run of 4 batches)
+    cap_trace = None
+    if world == 1 and not gen and not args.quick:
+        cap_trace = capacity_trace(eng, make_trace(4, float("inf"), seed=args.seed, vocab=cfg.vocab,
+                                                   n_decode=args.n_new), torch)
+
     # ---- NVLink all-reduce sweep (N > 1)
     ar_sweep = allreduce_sweep(eng, group, torch, F=args.F) if world > 1 and not args.quick else None
     scheduler = eng.scheduler_name()
@@ -616,6 +665,7 @@ def rank_main(args, group, local, uid, result):
             "allreduce": classes.get("allreduce"),
             "allreduce_sweep": ar_sweep,
             "decode_pass_in_situ": decode_pass,
+            "capacity_trace": cap_trace,
             "kernel_classes": {k: {kk: (round(vv, 4) if isinstance(vv, float) else vv) for kk, vv in v.items()}
                                for k, v in classes.items()},
             "cpu_baseline": cpu,

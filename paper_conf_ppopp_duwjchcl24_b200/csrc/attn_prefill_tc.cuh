@@ -76,6 +76,7 @@ __global__ void __launch_bounds__(PT_THREADS, 1)
                            __nv_bfloat16* __restrict__ kv_pool,
                            const int32_t* __restrict__ page_table, int max_pages, int b, int s, int heads) {
   using L = PtSmem<D>;
+  const uint64_t tr0 = trace_now();
   extern __shared__ uint8_t pt_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(pt_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + L::BARS);
@@ -124,6 +125,7 @@ __global__ void __launch_bounds__(PT_THREADS, 1)
   const uint32_t tmem = *tmem_slot;
   const uint32_t tS = tmem, tO = tmem + 128;
   pdl_enter();   // Q / K / V come from the QKV GEMM
+  const uint64_t tr1 = trace_now();
 
   if (warp == 0) {
     if (lane == 0) {
@@ -349,6 +351,7 @@ __global__ void __launch_bounds__(PT_THREADS, 1)
     tc_fence_after();
     tmem_dealloc(tmem, 256);
   }
+  if (threadIdx.x == 0) trace_write(TK_ATTN_PRE, tr0, tr1);
 }
 
 }  // namespace liger
