@@ -421,7 +421,18 @@ def capacity_trace(eng, trace, torch):
                     "that also merged the splits"}
 
 
-def rank_main(args, group, local, uid, result):
+def uid_factory(group, make):
+    """new_uid() for rank_main: at world > 1 every call is a collective in which rank 0
+    makes a fresh id (make()) and every rank receives it; None at world 1."""
+    if group.world == 1:
+        return lambda: None
+    return lambda: group.bcast(make() if group.rank == 0 else None)
+
+
+def rank_main(args, group, local, new_uid, result):
+    """One rank.  new_uid(): a fresh communicator id agreed by all ranks (a collective), or
+    None at world 1 -- every engine this rank creates gets its own, since an ncclUniqueId
+    bootstraps exactly one communicator."""
     import torch
     from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
     torch.cuda.set_device(local)
@@ -429,7 +440,7 @@ def rank_main(args, group, local, uid, result):
     cfg = get_config(args.config, args.layers)
     gen = args.workload == "generative"
     trace_kw = (dict(batch_sizes=(32,), prompt_range=(16, 16)) if gen else {})
-    ekw = dict(world=world, rank=rank, nccl_uid=uid, max_batch=32 if gen else 8, max_seq=16 if gen else 512,
+    ekw = dict(world=world, rank=rank, nccl_uid=new_uid(), max_batch=32 if gen else 8, max_seq=16 if gen else 512,
                max_new=args.n_new, max_inflight=args.inflight, decomp_factor=args.F, contention_factor=args.cf,
                seed=args.seed, sync=args.sync)
     eng = LigerEngine(cfg, mode=args.mode, **ekw)
@@ -601,6 +612,7 @@ def rank_main(args, group, local, uid, result):
         fracs = (0.3, 0.5, 0.8) if args.quick else (0.2, 0.35, 0.5, 0.65, 0.8, 0.95)
         sweep = {}
         for mode in modes:
+            ekw["nccl_uid"] = new_uid()
             e = LigerEngine(cfg, mode=mode, **ekw)
             e.profile([8, 64, 256, 512, 1024, 2048, 4096])
             for r in warm[:2]:
@@ -737,12 +749,12 @@ def main():
         from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
         world = args.gpus
         shared = ThreadShared(world)
-        uid = LigerEngine.loopback_id() if world > 1 else None
         errs = []
 
         def th(r):
             try:
-                rank_main(args, ThreadGroup(shared, r), 0, uid, result)
+                g = ThreadGroup(shared, r)
+                rank_main(args, g, 0, uid_factory(g, LigerEngine.loopback_id), result)
             except Exception as e:
                 import traceback
                 errs.append(f"rank {r}: {e!r}\n{traceback.format_exc()}")
@@ -767,11 +779,8 @@ def main():
         if world > 1:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         group = DistGroup(world, rank)
-        uid = None
-        if world > 1:
-            from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
-            uid = group.bcast(LigerEngine.unique_id() if rank == 0 else None)
-        rank_main(args, group, local, uid, result)
+        from paper_conf_ppopp_duwjchcl24_b200.engine import LigerEngine
+        rank_main(args, group, local, uid_factory(group, LigerEngine.unique_id), result)
         if world > 1:
             dist.destroy_process_group()
     if "line" in result:

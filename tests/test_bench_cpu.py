@@ -72,7 +72,11 @@ def _rank(r, port, q):
     eng = FakeEngine()
     res = B.serve_poisson(eng, g, tr)
     mx = g.max(float(r + 1))
-    q.put((r, eng.subs, mx, res["req_s"] > 0))
+    # every engine a rank creates gets a fresh communicator id, the same on all ranks
+    made = iter(range(100, 200))
+    new_uid = B.uid_factory(g, lambda: b"uid-%d" % next(made))
+    uids = [new_uid() for _ in range(3)]
+    q.put((r, eng.subs, mx, res["req_s"] > 0, uids))
     dist.destroy_process_group()
 
 
@@ -86,7 +90,10 @@ def test_serve_poisson_submits_identically_on_two_gloo_ranks():
     out = sorted(q.get(timeout=120) for _ in range(2))
     for p in ps:
         p.join(timeout=60)
-    (_, s0, m0, ok0), (_, s1, m1, ok1) = out
+    (_, s0, m0, ok0, u0), (_, s1, m1, ok1, u1) = out
     assert s0 == s1 and len(s0) == 6     # the same batches in the same order on both ranks
     assert m0 == m1 == 2.0               # max over ranks
     assert ok0 and ok1
+    # one fresh communicator id per engine (an ncclUniqueId bootstraps one communicator),
+    # identical on both ranks
+    assert u0 == u1 == [b"uid-100", b"uid-101", b"uid-102"]
