@@ -398,6 +398,12 @@ def capacity_trace(eng, trace, torch):
     rec = L.trace_stop(cap)
     if len(rec) == 0 or len(rec) >= cap:
         return None
+    return {"batches": len(trace), **trace_summary(rec)}
+
+
+def trace_summary(rec):
+    """Per kernel kind: sum over CTAs of (PDL-wait release t1 -> exit t2) / (SMs x span); and
+    the fraction of the span [min t0, max t2] in which no GEMM CTA (kid 1) works."""
     t0 = int(rec["t0"].min())
     a = (rec["t1"].astype(np.int64) - t0).astype(np.float64)
     z = (rec["t2"].astype(np.int64) - t0).astype(np.float64)
@@ -412,8 +418,8 @@ def capacity_trace(eng, trace, torch):
     dv = np.concatenate([np.ones(int(g.sum())), -np.ones(int(g.sum()))])
     o = np.argsort(ev, kind="stable")
     busy = np.cumsum(dv[o])[:-1] > 0
-    gemm_cov = float(np.diff(ev[o])[busy].sum()) / span
-    return {"batches": len(trace), "span_ms": round(span / 1e6, 2), "sms": nsm, "cta_records": int(len(rec)),
+    gemm_cov = float(np.diff(ev[o])[busy].sum()) / span if g.any() else 0.0
+    return {"span_ms": round(span / 1e6, 2), "sms": nsm, "cta_records": int(len(rec)),
             "sm_time_share": share, "no_gemm_working_frac": round(1.0 - gemm_cov, 4),
             "note": "in-kernel %globaltimer trace of every CTA while these batches are served as in the timed "
                     "region (release of the PDL wait -> exit); sm_time_share = CTA-time / (SMs x span); "

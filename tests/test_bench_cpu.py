@@ -97,3 +97,16 @@ def test_serve_poisson_submits_identically_on_two_gloo_ranks():
     # one fresh communicator id per engine (an ncclUniqueId bootstraps one communicator),
     # identical on both ranks
     assert u0 == u1 == [b"uid-100", b"uid-101", b"uid-102"]
+
+
+def test_trace_summary_hand_computed():
+    """bench.trace_summary on hand-made CTA records (2 SMs, span 100 ns): GEMM CTAs work in
+    [10, 40] and [30, 60] (union 50 ns -> no GEMM working 0.5 of the span), a fixup CTA in
+    [60, 100] (its entry t0 = 0 starts the span); SM-time shares 60 / 200 and 40 / 200."""
+    dt = np.dtype([("kid", "<u4"), ("cta", "<u4"), ("smid", "<u4"), ("pad", "<u4"),
+                   ("t0", "<u8"), ("t1", "<u8"), ("t2", "<u8")])
+    rec = np.array([(1, 0, 0, 0, 5, 10, 40), (1, 1, 1, 0, 5, 30, 60), (2, 0, 1, 0, 0, 60, 100)], dtype=dt)
+    out = bench.trace_summary(rec)
+    assert out["sms"] == 2 and out["span_ms"] == round(100 / 1e6, 2)
+    assert out["sm_time_share"] == {"gemm": 0.3, "splitk_fixup": 0.2}
+    assert out["no_gemm_working_frac"] == 0.5
