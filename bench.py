@@ -653,6 +653,8 @@ def rank_main(args, group, local, new_uid, result):
         cpu = cpu_oracle_sample(cfg)
         cpu.pop("per_batch_s", None)
 
+    w_rank_gb = (cfg.n_layers * (4 * cfg.hidden ** 2 + 2 * cfg.hidden * cfg.ffn) + cfg.vocab * cfg.hidden) * 2 \
+        / world / 1e9
     if rank == 0:
         t1_note = ("t = 1: no all-reduce to interleave (P:149); the interleaved mode runs the in-flight "
                    "batches' kernel lists concurrently on its two streams (reading R31); Algorithm 1, the "
@@ -675,7 +677,7 @@ def rank_main(args, group, local, new_uid, result):
                        "contention_factor_calibrated": round(cf_cal, 4),
                        "contention_factor_vs_gemm_sm_reserve": {str(k): v for k, v in sorted(cf_reserve.items())},
                        "sequences": seqs, "batches": len(timed),
-                       "l2": "inputs larger than L2 (weights 26 GB per TP=1 rank)"},
+                       "l2": f"inputs larger than L2 (weights {w_rank_gb:.1f} GB per rank)"},
             "operating_points": ops,
             "e2e": {"value": round(seqs / e2e_s, 3), "unit": "req/s", "h2d_bytes_per_step": int(h2d),
                     "d2h_bytes_per_step": int(d2h)},
@@ -690,7 +692,9 @@ def rank_main(args, group, local, new_uid, result):
             "clocks": clk,
             "gpu_launches": int(st["gpu_launches"]),
             "host": {"wall_s": round(wall_s, 3), "host_us": round(st["host_us"], 1),
-                     "rounds": st["rounds"], "kernels": st["kernels"]},
+                     "wait_us": round(st["wait_us"], 1), "rounds": st["rounds"], "kernels": st["kernels"],
+                     "host_us_per_round_excl_wait": round((st["host_us"] - st["wait_us"]) / max(1, st["rounds"]),
+                                                          2)},
         }
 
 

@@ -178,6 +178,10 @@ struct liger_ctx {
   cudaEvent_t e1 = nullptr, e2 = nullptr;
   cudaEvent_t e_end[2] = {nullptr, nullptr};   // CPU_GPU sync: end of the round on each stream
   bool have_round = false;
+  // E1 placement (liger_step): host time of one round after its E1 wait (EMA, us), and a
+  // fixed lead from LIGER_E1_LEAD_US (< 0: use the EMA)
+  double host_round_us = 0.0;
+  double e1_lead_us = -1.0;
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_next = 0;
   DurTable dur;
@@ -953,6 +957,7 @@ int liger_init(int world, int rank, const liger_cfg* cfg, const uint8_t* nccl_ui
   const char* env = getenv("LIGER_AR_ATOMIC_CHUNKS");
   c->ar_atomic_chunks = env ? atoi(env) != 0 : (tp > 2);
   if (const char* e = getenv("LIGER_AR_DECOMP_MIN_KB")) c->ar_decomp_min_bytes = (size_t)atoll(e) * 1024;
+  if (const char* e = getenv("LIGER_E1_LEAD_US")) c->e1_lead_us = atof(e);   // 0: the paper's placement
   if (world > 1) {
     if (!nccl_uid) return fail(nullptr, LIGER_EINVAL, "liger_init: nccl_uid required for world > 1");
     std::string err;
@@ -1272,6 +1277,7 @@ int liger_step(liger_ctx* c) {
     }
     c->st.wait_us += (now_s() - w0) * 1e6;
   }
+  const double t_woke = now_s();
   update_list(c);
   if (c->processing.empty()) {
     c->st.host_us += (now_s() - t0) * 1e6;
@@ -1346,16 +1352,35 @@ int liger_step(liger_ctx* c) {
       cudaStreamWaitEvent(c->s_comp, c->e2, 0);
       cudaStreamWaitEvent(c->s_comm, c->e2, 0);
     }
+    // E1 placement.  The paper records E1 before the switch kernel (the last of SubSet0,
+    // P:236) so the host plans and launches the next round while that kernel runs -- on
+    // its V100s kernels took milliseconds.  B200 decode kernels take 3-30 us, the order of
+    // the host's own work per round, so E1 goes before the first SubSet0 kernel from which
+    // the profiled durations of the kernels still to run cover the host's measured time
+    // per round (x1.5), and never after the switch kernel.  Only the time at which the
+    // host wakes up moves: plans and kernels are the same (they depend on the launch state
+    // alone, identical on every rank).
+    size_t e1_at = w0.empty() ? 0 : w0.size() - 1;
+    {
+      const double lead = c->e1_lead_us >= 0 ? c->e1_lead_us : 1.5 * c->host_round_us;
+      double rem = 0.0;
+      for (size_t i = w0.size(); i-- > 0;) {
+        const Piece& p = pieces[w0[i]];
+        rem += 1e6 * op_dur(c, p.bt, p.pass, c->pass_ops[p.idx].op, p.u1 - p.u0);   // s -> us
+        if (i < e1_at) e1_at = i;
+        if (rem >= lead) break;
+      }
+    }
     // communication subset first
     auto launch_sub0 = [&]() -> int {
       if (w0.empty()) return 0;
-      std::vector<int> head(w0.begin(), w0.end() - 1), last(1, w0.back());
+      std::vector<int> head(w0.begin(), w0.begin() + e1_at), tail(w0.begin() + e1_at, w0.end());
       int rc = launch_run(c, pieces, head, s0);
       if (rc < 0) return rc;
-      cudaEventRecord(c->e1, stream_of(c, s0));   // E1: before the switch kernel
-      rc = launch_run(c, pieces, last, s0);
+      cudaEventRecord(c->e1, stream_of(c, s0));   // E1: before the kernels that cover the host's round
+      rc = launch_run(c, pieces, tail, s0);
       if (rc < 0) return rc;
-      cudaEventRecord(c->e2, stream_of(c, s0));   // E2: after it
+      cudaEventRecord(c->e2, stream_of(c, s0));   // E2: after the switch kernel
       return 0;
     };
     if (s1 == 1) {
@@ -1373,6 +1398,8 @@ int liger_step(liger_ctx* c) {
     c->st.rounds++;
     if (!w1.empty()) c->st.overlapped_rounds++;
     n = (int)pieces.size();
+    const double us = (now_s() - t_woke) * 1e6;
+    c->host_round_us = c->host_round_us > 0 ? 0.9 * c->host_round_us + 0.1 * us : us;
   }
   c->st.host_us += (now_s() - t0) * 1e6;
   (void)n;
