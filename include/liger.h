@@ -240,12 +240,21 @@ int liger_op_allreduce(liger_ctx* ctx, void* buf, size_t count, int u0, int u1, 
  * then already satisfied) -- the same kernel code, the same bits. */
 #define LIGER_AR_PHASE_STAGE 1
 #define LIGER_AR_PHASE_REDUCE 2
+/* Test vehicle for the one-shot kernel's cross-rank protocol on ONE GPU: the `world` ranks of
+ * call `epoch` -- rank q's buffer bufs[q] (bf16 [count], summed in place) and region
+ * regions[q] (as above: liger_ipc_region_create'd or any zeroed device allocation of
+ * liger's region size) -- run as ONE cooperative launch whose block group q executes rank
+ * q's device code (stage, publish, spin on every flag, rank-ordered sum): the ranks' spins
+ * run concurrently with every block co-resident, as ranks on different GPUs do.
+ * LIGER_EINVAL if the blocks cannot all be co-resident. */
 int liger_ipc_region_create(size_t cap, void** region, uint8_t* handle);
 int liger_ipc_region_open(const uint8_t* handle, void** peer);
 int liger_ipc_region_close(void* peer);
 int liger_ipc_region_free(void* region);
 int liger_op_oneshot_allreduce(void* buf, size_t count, void* const* regions, int world, int rank, size_t cap,
                                uint64_t epoch, int phases, void* stream);
+int liger_op_oneshot_allreduce_emulated(void* const* bufs, size_t count, void* const* regions, int world, size_t cap,
+                                        uint64_t epoch, void* stream);
 
 /* The fused row-parallel GEMM + all-reduce of serial TP (§8(f) next row 4; DESIGN.md §8
  * "Fused row-parallel GEMM + all-reduce"), its two halves on explicit regions, call number

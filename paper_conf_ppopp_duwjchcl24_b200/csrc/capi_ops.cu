@@ -188,6 +188,14 @@ int liger_op_oneshot_allreduce(void* buf, size_t count, void* const* regions, in
   return ret(par.allreduce_bf16(buf, count, (cudaStream_t)stream, phases), "liger_op_oneshot_allreduce");
 }
 
+int liger_op_oneshot_allreduce_emulated(void* const* bufs, size_t count, void* const* regions, int world, size_t cap,
+                                        uint64_t epoch, void* stream) {
+  if (int rc = check_device()) return rc;
+  if (!bufs || !regions) return LIGER_EINVAL;
+  return ret(oneshot_allreduce_emulated(bufs, count, regions, world, cap, epoch, (cudaStream_t)stream),
+             "liger_op_oneshot_allreduce_emulated");
+}
+
 // the fused producer / consumer descriptor of call `epoch` on explicit regions
 static int fused_desc(void* const* regions, int world, int rank, size_t cap, uint64_t epoch, size_t bytes,
                       FusedARDesc* far) {

@@ -49,6 +49,9 @@ struct PeerAR {
   ~PeerAR();
 };
 size_t peer_ar_region_bytes(size_t cap);
+// test vehicle: `world` ranks' one-shot all-reduces (call `epoch`) as one cooperative launch
+int oneshot_allreduce_emulated(void* const* bufs, size_t count, void* const* regions, int world, size_t cap,
+                               uint64_t epoch, cudaStream_t st);
 
 enum CommDType { CD_BF16, CD_F32, CD_I32 };
 enum CommOp { CO_SUM, CO_MAX };

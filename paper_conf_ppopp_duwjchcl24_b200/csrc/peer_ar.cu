@@ -54,26 +54,25 @@ __device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned l
   asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
+// One rank's one-shot all-reduce, run by `nblk` blocks (block index `bid` of them).
 // n8 = number of 8-element (16-byte) vectors
-__global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf, size_t n8, uint4* my_stage,
-                                                                      unsigned long long* my_flag,
-                                                                      unsigned int* counter, PeerPtrs peers,
-                                                                      int world, unsigned long long epoch,
-                                                                      int phases) {
-  const size_t stride = (size_t)gridDim.x * blockDim.x;
+__device__ __forceinline__ void oneshot_rank(uint4* buf, size_t n8, uint4* my_stage, unsigned long long* my_flag,
+                                             unsigned int* counter, const PeerPtrs& peers, int world,
+                                             unsigned long long epoch, int phases, int bid, int nblk) {
+  const size_t stride = (size_t)nblk * blockDim.x;
   // The partials come from the preceding GEMM.  Dependents are released only after
   // every peer has arrived (below): a kernel parked at its griddepcontrol.wait
   // must not hold SM resources while this one spins on other ranks -- on the
   // loopback backend those ranks share this GPU and would need them to progress.
   grid_dependency_wait();
   if (phases & LIGER_AR_PHASE_STAGE) {
-    for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += stride) my_stage[i] = buf[i];
+    for (size_t i = (size_t)bid * blockDim.x + threadIdx.x; i < n8; i += stride) my_stage[i] = buf[i];
     __threadfence_system();   // every thread's staging stores before the block's publish
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence_system();
       const unsigned int prev = atomicAdd(counter, 1u);
-      if (prev == gridDim.x - 1) {   // every block's staging copy is done: publish
+      if (prev == (unsigned int)nblk - 1) {   // every block's staging copy is done: publish
         *counter = 0;
         __threadfence_system();
         st_release_sys(my_flag, epoch);
@@ -91,14 +90,14 @@ __global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf
         __nanosleep(64);
         if (trace_now() - t0 > 10000000000ull) {   // a peer never arrived: fail, do not hang
           printf("liger one-shot all-reduce: epoch %llu, waited 10 s for peer %d (flag %llu), block %d of %d\n",
-                 epoch, q, ld_acquire_sys(peers.flag[q]), blockIdx.x, gridDim.x);
+                 epoch, q, ld_acquire_sys(peers.flag[q]), bid, nblk);
           __trap();
         }
       }
   }
   __syncthreads();
   grid_dependency_trigger();
-  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += stride) {
+  for (size_t i = (size_t)bid * blockDim.x + threadIdx.x; i < n8; i += stride) {
     uint4 v[PAR_MAX_WORLD];
 #pragma unroll
     for (int q = 0; q < PAR_MAX_WORLD; ++q)
@@ -133,6 +132,32 @@ __global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf
   }
 }
 
+
+__global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_bf16_kernel(uint4* buf, size_t n8, uint4* my_stage,
+                                                                      unsigned long long* my_flag,
+                                                                      unsigned int* counter, PeerPtrs peers,
+                                                                      int world, unsigned long long epoch,
+                                                                      int phases) {
+  oneshot_rank(buf, n8, my_stage, my_flag, counter, peers, world, epoch, phases, blockIdx.x, gridDim.x);
+}
+
+// Test vehicle: the `world` ranks of one all-reduce as ONE cooperative launch on one GPU
+// (block group q = blocks [q nblk, (q + 1) nblk) runs rank q's oneshot_rank), so the ranks'
+// spins on each other's flags run concurrently with every block co-resident -- the way
+// ranks on different GPUs run, which separate launches on one GPU cannot guarantee.
+struct EmuRanks {
+  uint4* buf[PAR_MAX_WORLD];
+  uint4* stage[PAR_MAX_WORLD];
+  unsigned long long* flag[PAR_MAX_WORLD];
+  unsigned int* counter[PAR_MAX_WORLD];
+};
+__global__ void __launch_bounds__(PAR_THREADS) oneshot_ar_emulated_kernel(EmuRanks r, size_t n8, PeerPtrs peers,
+                                                                          int world, unsigned long long epoch,
+                                                                          int nblk) {
+  const int q = blockIdx.x / nblk;
+  oneshot_rank(r.buf[q], n8, r.stage[q], r.flag[q], r.counter[q], peers, world, epoch,
+               LIGER_AR_PHASE_STAGE | LIGER_AR_PHASE_REDUCE, blockIdx.x % nblk, nblk);
+}
 }  // namespace
 
 // [2 buffers][cap] | epoch flag (+0) | one-shot block counter (+128) | fused-producer
@@ -205,6 +230,46 @@ int PeerAR::allreduce_bf16(void* buf, size_t count, cudaStream_t st, int phases)
              : 0;
 }
 
-void preload_peer_ar_kernel() { preload_kernel(oneshot_ar_bf16_kernel); }
+// world ranks' regions[q] (each [2 staging buffers of cap][flag][counters], zeroed before the
+// first use) and buffers bufs[q]; call number `epoch`: one cooperative launch
+int oneshot_allreduce_emulated(void* const* bufs, size_t count, void* const* regions, int world, size_t cap,
+                               uint64_t epoch, cudaStream_t st) {
+  const size_t bytes = count * 2;
+  if (world < 1 || world > PAR_MAX_WORLD || bytes > cap || bytes % 16 || cap % 256 || epoch == 0) return LIGER_EINVAL;
+  if (!count) return 0;
+  const int b = (int)(epoch & 1);
+  EmuRanks r{};
+  PeerPtrs pp{};
+  for (int q = 0; q < world; ++q) {
+    if (!bufs[q] || !regions[q] || reinterpret_cast<uintptr_t>(bufs[q]) % 16) return LIGER_EINVAL;
+    char* reg = static_cast<char*>(regions[q]);
+    r.buf[q] = static_cast<uint4*>(bufs[q]);
+    r.stage[q] = reinterpret_cast<uint4*>(reg + (size_t)b * cap);
+    r.flag[q] = reinterpret_cast<unsigned long long*>(reg + 2 * cap);
+    r.counter[q] = reinterpret_cast<unsigned int*>(reg + 2 * cap + 128);
+    pp.data[q] = r.stage[q];
+    pp.flag[q] = r.flag[q];
+  }
+  const size_t n8 = bytes / 16;
+  int nblk = (int)((n8 + PAR_THREADS - 1) / PAR_THREADS);
+  nblk = nblk < 1 ? 1 : (nblk > 8 ? 8 : nblk);
+  int dev = 0, per_sm = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, oneshot_ar_emulated_kernel, PAR_THREADS, 0);
+  if (world * nblk > per_sm * sms) return LIGER_EINVAL;   // every block must be co-resident
+  unsigned long long ep = epoch;
+  int w = world;
+  void* args[] = {&r, (void*)&n8, &pp, &w, &ep, &nblk};
+  return cudaLaunchCooperativeKernel((const void*)oneshot_ar_emulated_kernel, dim3(world * nblk), dim3(PAR_THREADS),
+                                     args, 0, st) == cudaSuccess
+             ? 0
+             : LIGER_ECUDA;
+}
+
+void preload_peer_ar_kernel() {
+  preload_kernel(oneshot_ar_bf16_kernel);
+  preload_kernel(oneshot_ar_emulated_kernel);
+}
 
 }  // namespace liger

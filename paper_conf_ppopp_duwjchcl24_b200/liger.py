@@ -73,6 +73,7 @@ _SIGS = {
     "liger_ipc_region_close": (_I, [_P]),
     "liger_ipc_region_free": (_I, [_P]),
     "liger_op_oneshot_allreduce": (_I, [_P, _SZ, _P, _I, _I, _SZ, _U64, _I, _P]),
+    "liger_op_oneshot_allreduce_emulated": (_I, [_P, _SZ, _P, _I, _SZ, _U64, _P]),
     "liger_op_gemm_fused_ar_stage": (_I, [_P, _I64, _P, _I, _I, _I, _P, _I, _I, _SZ, _U64, _P, _SZ, _P]),
     "liger_op_add_layernorm_fused_ar": (_I, [_P, _I, _I, _SZ, _U64, _P, _P, _P, _P, _P, _P, _I, _I, _F, _P]),
     "liger_op_allreduce": (_I, [_P, _P, _SZ, _I, _I, _I, _P]),
@@ -199,6 +200,16 @@ def oneshot_allreduce(buf, regions, rank, cap, epoch, phases=AR_PHASE_STAGE | AR
     check(lib().liger_op_oneshot_allreduce(_p(buf), buf.numel(), arr, len(regions), rank, cap, epoch, phases,
                                            _s(stream)),
           what="liger_op_oneshot_allreduce")
+
+
+def oneshot_allreduce_emulated(bufs, regions, cap, epoch, stream=None):
+    """liger_op_oneshot_allreduce_emulated: every rank's one-shot all-reduce of call `epoch` as one
+    cooperative launch (test vehicle for the cross-rank protocol on one GPU); bufs summed in place."""
+    w = len(bufs)
+    pb = (C.c_void_p * w)(*[b.data_ptr() for b in bufs])
+    pr = (C.c_void_p * w)(*regions)
+    check(lib().liger_op_oneshot_allreduce_emulated(pb, bufs[0].numel(), pr, w, cap, epoch, _s(stream)),
+          what="liger_op_oneshot_allreduce_emulated")
 
 
 def gemm_fused_ar_stage(x, w_tiled, M, N, K, regions, rank, cap, epoch, workspace, stream=None):

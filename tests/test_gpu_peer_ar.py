@@ -8,6 +8,9 @@ B200_PROFILING.md).  Every test therefore runs each kernel phase by phase throug
 C-ABI: all ranks' staging / publishing launches first, a host synchronisation, then all
 ranks' waiting / summing launches, whose waits are already satisfied.  The kernels are the
 ones the serving path launches with both phases in one launch per rank (one rank per GPU).
+The one-shot protocol with the ranks truly concurrent (spinning on each other) runs as ONE
+cooperative launch holding every rank's blocks (liger_op_oneshot_allreduce_emulated), the
+emulation B200_PROFILING.md prescribes when there are fewer GPUs than ranks.
 
 Oracle: oracle.model.allreduce_decomposed (the per-layer all-reduce of P:286 as a
 sum of the ranks' bf16 partials) and oracle.model.layer_norm (C2)."""
@@ -88,6 +91,29 @@ def test_oneshot_allreduce_phased_vs_oracle(L, world):
                 want_bits = (want.view(np.uint32) >> 16).astype(np.uint16).view(np.int16)
                 for q in range(world):
                     assert np.array_equal(_bits(bufs[q]), want_bits), (world, n, ks, q)
+    finally:
+        _free(L, regions)
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_oneshot_allreduce_concurrent_ranks_vs_oracle(L, world):
+    """The same kernel code with the ranks truly concurrent: every rank's one-shot all-reduce
+    of a call as ONE cooperative launch (block group q = rank q: stage, publish its epoch,
+    spin until all t flags arrive, rank-ordered fp32 sum), 6 consecutive calls alternating
+    the staging buffers and reusing the flags and counters -- what ranks on t GPUs do, run
+    with every block co-resident.  Every rank ends with bf16_rne(oracle sum), bit for bit."""
+    regions = _regions(L, world)
+    try:
+        for epoch, n in enumerate((8 * 5120, 16 * 1024 + 8, 256, 8 * 5120, 40, 4096), start=1):
+            parts = [_part(q, n, seed=90 + epoch) for q in range(world)]
+            bufs = [bf16_dev(parts[q]) for q in range(world)]
+            L.oneshot_allreduce_emulated(bufs, regions, CAP, epoch)
+            torch.cuda.synchronize()
+            ref = om.allreduce_decomposed([p.astype(np.float64) for p in parts], 1, [1])
+            want = bf16_rne(ref.astype(np.float32))
+            want_bits = (want.view(np.uint32) >> 16).astype(np.uint16).view(np.int16)
+            for q in range(world):
+                assert np.array_equal(_bits(bufs[q]), want_bits), (world, epoch, n, q)
     finally:
         _free(L, regions)
 
