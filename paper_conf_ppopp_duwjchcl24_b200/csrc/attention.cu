@@ -92,7 +92,7 @@ __global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecA
   constexpr int TPW = 32 / LPT;       // token rows per warp step
   constexpr int NG = 4 * TPW;         // lane groups per CTA
   constexpr int PPG = DC_CH / NG;     // positions per lane group per chunk
-  const uint64_t tr0 = trace_now();
+  const TraceStart tr0 = trace_begin();
   extern __shared__ __align__(128) uint8_t dsm[];
   DecSmem<D>& sm = *reinterpret_cast<DecSmem<D>*>(dsm);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;

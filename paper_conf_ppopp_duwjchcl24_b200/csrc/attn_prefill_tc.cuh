@@ -76,7 +76,7 @@ __global__ void __launch_bounds__(PT_THREADS, 1)
                            __nv_bfloat16* __restrict__ kv_pool,
                            const int32_t* __restrict__ page_table, int max_pages, int b, int s, int heads) {
   using L = PtSmem<D>;
-  const uint64_t tr0 = trace_now();
+  const TraceStart tr0 = trace_begin();
   extern __shared__ uint8_t pt_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(pt_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + L::BARS);

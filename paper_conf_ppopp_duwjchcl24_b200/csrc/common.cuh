@@ -205,7 +205,7 @@ LIGER_DEV void pdl_enter() {
 
 // ---------------------------------------------------------------- timeline trace
 // Development diagnostics (liger_trace_start / liger_trace_stop): thread 0 of every
-// CTA of a traced kernel appends {kernel id, CTA, SM, entry, after-PDL-wait, exit}
+// CTA of a traced kernel writes {kernel id, CTA, SM, entry, after-PDL-wait, exit}
 // %globaltimer stamps.  Off (one predicated load) unless a buffer is installed.
 // Each translation unit holds its own copy of the buffer descriptor.
 struct TraceRec {
@@ -223,11 +223,22 @@ LIGER_DEV uint64_t trace_now() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
-LIGER_DEV void trace_write(uint32_t kid, uint64_t t0, uint64_t t1) {
-  if (g_trace.rec == nullptr) return;
+// Entry stamp; thread 0 of a traced CTA also reserves its record slot here, so the atomic's
+// round trip overlaps the kernel's work instead of delaying the CTA's exit.
+struct TraceStart {
+  uint64_t t0;
+  unsigned int slot;
+};
+LIGER_DEV TraceStart trace_begin() {
+  TraceStart r{trace_now(), 0xFFFFFFFFu};
+  if (threadIdx.x == 0 && g_trace.rec != nullptr) r.slot = atomicAdd(g_trace.n, 1u);
+  return r;
+}
+LIGER_DEV void trace_write(uint32_t kid, TraceStart s0, uint64_t t1) {
+  if (g_trace.rec == nullptr || s0.slot >= g_trace.cap) return;
+  const uint64_t t0 = s0.t0;
   const uint64_t t2 = trace_now();
-  const unsigned int i = atomicAdd(g_trace.n, 1u);
-  if (i >= g_trace.cap) return;
+  const unsigned int i = s0.slot;
   uint32_t sm;
   asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
   TraceRec r;

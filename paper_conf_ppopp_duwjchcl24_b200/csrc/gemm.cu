@@ -179,8 +179,8 @@ template <bool EXT>
 __global__ void __launch_bounds__(GEMM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmParams p) {
-  const uint64_t tr0 = trace_now();
-  uint64_t tr1 = tr0;
+  const TraceStart tr0 = trace_begin();
+  uint64_t tr1 = tr0.t0;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int S = p.stages;
@@ -369,7 +369,7 @@ __global__ void __launch_bounds__(GEMM_THREADS, 1)
 // reading the column-major per-tile partials coalesced.
 template <bool EXT>
 __global__ void __launch_bounds__(256) splitk_reduce_kernel(const GemmParams p) {
-  const uint64_t tr0 = trace_now();
+  const TraceStart tr0 = trace_begin();
   const int tiles = p.n_tiles * p.m_tiles;
   const int64_t zstride = (int64_t)tiles * (BM * p.bn);
   const int slice_w = p.n1 - p.n0;

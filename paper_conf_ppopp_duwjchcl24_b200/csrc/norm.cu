@@ -57,7 +57,7 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
                                                     const bf16x8* __restrict__ beta, int h, int in_row_step,
                                                     int in_row_off, float eps, const FusedARDesc far) {
   __shared__ float red[NT / 32];
-  const uint64_t tr0 = trace_now();
+  const TraceStart tr0 = trace_begin();
   const int nv = h >> 3;
   const int64_t in_row = (int64_t)blockIdx.x * in_row_step + in_row_off;
   const bf16x8* xr = x + in_row * nv;
