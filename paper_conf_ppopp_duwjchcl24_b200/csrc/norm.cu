@@ -50,7 +50,11 @@ __device__ __forceinline__ float block_sum(float v, float* red) {
 // peers staged for epoch far.epoch (peer_ar.cu protocol): wait for every peer's
 // flag, then sum the staged rows over ranks 0..t-1 in fp32 in that order and round
 // to bf16 -- the one-shot all-reduce's bits, without its kernel.
-template <int NT, int MAXV, bool PEER>
+// LATE: gamma / beta are loaded where they are used (after the statistics) instead of
+// being held in registers from the start -- fewer live registers, more resident rows per
+// SM: the variant for many-row (prefill) launches, where occupancy, not one row's
+// latency, bounds the kernel.
+template <int NT, int MAXV, bool PEER, bool LATE = false>
 __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x, const bf16x8* __restrict__ add,
                                                     const bf16x8* __restrict__ add_bias, bf16x8* x_out,
                                                     bf16x8* __restrict__ y, const bf16x8* __restrict__ gamma,
@@ -76,8 +80,10 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
     if (v < nv) {
       if (x_early) vx[j] = xr[v];
       if (add_bias) vb[j] = add_bias[v];
-      vg[j] = gamma[v];
-      vbe[j] = beta[v];
+      if (!LATE) {
+        vg[j] = gamma[v];
+        vbe[j] = beta[v];
+      }
     }
   }
   if (PEER) {
@@ -184,8 +190,8 @@ __global__ void __launch_bounds__(NT) add_ln_kernel(const bf16x8* __restrict__ x
     const int v = threadIdx.x + j * NT;
     if (v < nv) {
       float g[8], b[8], o[8];
-      unpack8(vg[j], g);
-      unpack8(vbe[j], b);
+      unpack8(LATE ? gamma[v] : vg[j], g);
+      unpack8(LATE ? beta[v] : vbe[j], b);
 #pragma unroll
       for (int e = 0; e < 8; ++e) o[e] = (r[j][e] - mean) * rstd * g[e] + b[e];
       y[(int64_t)blockIdx.x * nv + v] = pack8(o);
@@ -208,7 +214,16 @@ int add_layernorm_launch(const void* x, const void* add, const void* add_bias, v
   launch_pdl(add_ln_kernel<NT, MV, false>, dim3(rows), dim3(NT), 0, stream, X, A, AB, (bf16x8*)x_out,     \
              (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, in_row_step, in_row_off, eps, nofar)
   int rc;
-  if (nv <= 128) rc = LIGER_LN(128, 1);
+  // many rows (prefill): the LATE variant with NT = nv / 4 rounded up to a warp (fewer
+  // live registers: 4 rows per SM instead of 2 at h = 5120; tools/kbench_ln.py, 4096
+  // rows: 68.5 -> 47.9 us); few rows (decode): everything loaded before the PDL wait
+  if (rows > 2 * 148 && nv > 512 && nv <= 1536) {
+#define LIGER_LN_L(NT)                                                                                          \
+  launch_pdl(add_ln_kernel<NT, 4, false, true>, dim3(rows), dim3(NT), 0, stream, X, A, AB, (bf16x8*)x_out,  \
+             (bf16x8*)y, (const bf16x8*)gamma, (const bf16x8*)beta, h, in_row_step, in_row_off, eps, nofar)
+    rc = nv <= 640 ? LIGER_LN_L(160) : nv <= 896 ? LIGER_LN_L(224) : nv <= 1152 ? LIGER_LN_L(288) : LIGER_LN_L(384);
+#undef LIGER_LN_L
+  } else if (nv <= 128) rc = LIGER_LN(128, 1);
   else if (nv <= 512) rc = LIGER_LN(128, 4);
   else if (nv <= 1024) rc = LIGER_LN(256, 4);
   else rc = LIGER_LN(512, 4);
@@ -426,6 +441,10 @@ void preload_norm_kernels() {
   preload_kernel(add_ln_kernel<128, 4, false>);
   preload_kernel(add_ln_kernel<256, 4, false>);
   preload_kernel(add_ln_kernel<512, 4, false>);
+  preload_kernel(add_ln_kernel<160, 4, false, true>);
+  preload_kernel(add_ln_kernel<224, 4, false, true>);
+  preload_kernel(add_ln_kernel<288, 4, false, true>);
+  preload_kernel(add_ln_kernel<384, 4, false, true>);
   preload_kernel(add_ln_kernel<128, 1, true>);
   preload_kernel(add_ln_kernel<128, 4, true>);
   preload_kernel(add_ln_kernel<256, 4, true>);

@@ -123,7 +123,8 @@ def test_gemm_empty_and_errors(L):
 
 
 # ---------------------------------------------------------------- LayerNorm
-@pytest.mark.parametrize("R,h", [(1, 256), (7, 1024), (33, 5120), (3, 12288)])
+@pytest.mark.parametrize("R,h", [(1, 256), (7, 1024), (33, 5120), (3, 12288),
+                                 (300, 5120), (301, 7168), (400, 9216), (297, 12288)])   # many rows: LATE variant
 def test_add_layernorm_vs_oracle(L, R, h):
     x = c0_values(3, 1, np.arange(R * h, dtype=np.uint64), 0).reshape(R, h)
     a = c0_values(3, 2, np.arange(R * h, dtype=np.uint64), -1).reshape(R, h)
