@@ -296,7 +296,42 @@ __global__ void argmax_kernel(const float* __restrict__ logits, int64_t ld, int 
   const float* row = logits + (int64_t)blockIdx.x * ld;
   float bv = -INFINITY;
   int bi = 0x7fffffff;
-  for (int i = threadIdx.x; i < n; i += blockDim.x) better(bv, bi, row[i], i);
+  // 16-byte loads, four independent (max, index) states per thread so that several loads
+  // are in flight (a scalar loop was one dependent L2 / HBM round trip per element);
+  // `better` is a total order (larger value, then lower index), so the result does not
+  // depend on the visiting order
+  int done = 0;
+  if ((reinterpret_cast<uintptr_t>(row) & 15) == 0) {
+    const int n4 = n >> 2;
+    const float4* r4 = reinterpret_cast<const float4*>(row);
+    float v4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+    int i4[4] = {0x7fffffff, 0x7fffffff, 0x7fffffff, 0x7fffffff};
+    int k = threadIdx.x;
+    for (; k + 3 * (int)blockDim.x < n4; k += 4 * blockDim.x) {
+      float4 q[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) q[u] = __ldcg(r4 + k + u * blockDim.x);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int e = 4 * (k + u * (int)blockDim.x);
+        better(v4[u], i4[u], q[u].x, e);
+        better(v4[u], i4[u], q[u].y, e + 1);
+        better(v4[u], i4[u], q[u].z, e + 2);
+        better(v4[u], i4[u], q[u].w, e + 3);
+      }
+    }
+    for (; k < n4; k += blockDim.x) {
+      const float4 q = __ldcg(r4 + k);
+      better(v4[0], i4[0], q.x, 4 * k);
+      better(v4[0], i4[0], q.y, 4 * k + 1);
+      better(v4[0], i4[0], q.z, 4 * k + 2);
+      better(v4[0], i4[0], q.w, 4 * k + 3);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) better(bv, bi, v4[u], i4[u]);
+    done = n4 << 2;
+  }
+  for (int i = done + threadIdx.x; i < n; i += blockDim.x) better(bv, bi, row[i], i);
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
     float ov = __shfl_xor_sync(0xffffffffu, bv, o);

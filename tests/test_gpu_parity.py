@@ -327,6 +327,26 @@ def test_argmax_lowest_index_on_ties(L):
     assert np.array_equal(mx.cpu().numpy(), logits.max(axis=1))
 
 
+@pytest.mark.parametrize("rows,n,ld", [(8, 50272, 50272), (3, 50272, 50275), (2, 6284, 6284), (4, 18817, 18820)])
+def test_argmax_vocab_sizes_ties_and_strides(L, rows, n, ld):
+    """LM-head argmax at vocabulary-shard sizes (OPT 50272 at t = 1, 6284 at t = 8, a ragged
+    18817), 16-byte-aligned and unaligned row strides: lowest index on ties, wherever the tied
+    maxima fall (same 16-byte group, different unrolled load groups, the scalar tail)."""
+    rng = np.random.default_rng(rows * n)
+    buf = rng.standard_normal((rows, ld)).astype(np.float32)
+    logits = buf[:, :n]
+    ties = [(5, 6), (4100 % n, (n * 4) // 5), (n - 1, 3), (n - 2, n - 1)]
+    for r in range(rows):
+        logits[r, list(ties[r % 4])] = 60.0 + r
+    d = torch.from_numpy(np.ascontiguousarray(buf)).cuda()
+    mx = torch.empty(rows, device="cuda")
+    ix = torch.empty(rows, dtype=torch.int32, device="cuda")
+    L.lib().liger_op_argmax(L._p(d), ld, rows, n, 7, L._p(mx), L._p(ix), None)
+    torch.cuda.synchronize()
+    assert np.array_equal(ix.cpu().numpy(), np.argmax(logits, axis=1) + 7)
+    assert np.array_equal(mx.cpu().numpy(), logits.max(axis=1))
+
+
 # ---------------------------------------------------------------- full TP decoder layer through the C ABI
 @pytest.mark.parametrize("name,t,b,s", [("tiny", 1, 2, 32), ("tiny", 2, 2, 32), ("tiny", 4, 3, 17),
                                         ("opt-13b", 1, 2, 24), ("opt-13b", 2, 1, 64), ("opt-30b", 4, 1, 12)])
