@@ -132,6 +132,23 @@ def test_pipeline_baselines_match_oracle(E, world, mode):
     assert pipe[world - 1]["stats"]["comm_kernels"] > 0
 
 
+@pytest.mark.parametrize("lead", ["0", "1000000"])
+def test_e1_placement_bit_exact(E, lead):
+    """Hybrid sync E1 placement (DESIGN R8): the paper's (before the switch kernel, lead 0)
+    and the earliest (before the first SubSet0 kernel, a lead no round reaches) change only
+    when the host wakes up -- bit-identical to the default duration-aware placement, which
+    matches the oracle element-wise, at TP = 2 with decomposition."""
+    cfg = get_config("tiny")
+    trace = _mixed_trace(4, 23, cfg, (1, 2, 3), (8, 40), (3, 5))
+    kw = dict(mode="interleaved", max_batch=4, max_seq=48, max_new=8, max_inflight=3, decomp_factor=8, seed=7)
+    ref = serve(E, cfg, 2, trace, **kw)
+    with env(LIGER_E1_LEAD_US=lead):
+        alt = serve(E, cfg, 2, trace, **kw)
+    check_vs_oracle(cfg, 7, trace, ref, world=2)
+    assert_bit_identical(ref, alt)
+    assert alt[0]["stats"]["overlapped_rounds"] > 0
+
+
 @pytest.mark.parametrize("sync", ["cpu_gpu", "inter_stream"])
 def test_sync_ablation_modes_bit_exact(E, sync):
     """§3.4 Fig. 8 / §4.5 ablation: the CPU-GPU-only and inter-stream-only
