@@ -112,6 +112,25 @@ def test_ln_fold_full_size_opt13b_layer(E):
     check_vs_oracle(cfg, 1, trace, res)
 
 
+def test_full_size_opt13b_two_stream_equals_serial(E):
+    """bench.py's launch configuration at full size (OPT-13B, 40 layers, t = 1): 4 batches of
+    the bench's mixed trace (b in {2, 4, 8}, prompts U[128, 512], 32 generated tokens) served
+    by the interleaved mode (the pass-by-pass two-stream schedule, folded LN) and by serial
+    intra-op TP give identical tokens, logits and last-layer residuals bit for bit (a
+    property that holds at any size; the oracle's element-wise checks run at the sizes it
+    finishes in seconds).  The tokens are valid ids, not the echo of the last prompt token."""
+    cfg = get_config("opt-13b")
+    trace = make_trace(4, float("inf"), seed=3, vocab=cfg.vocab, n_decode=32)
+    kw = dict(max_batch=8, max_seq=512, max_new=32, seed=0)
+    two = serve(E, cfg, 1, trace, mode="interleaved", **kw)
+    ser = serve(E, cfg, 1, trace, mode="serial", **kw)
+    assert_bit_identical(two, ser)
+    for t, toks, lg in zip(trace, two[0]["tokens"], two[0]["logits"]):
+        assert toks.shape == (t["batch"], 32) and toks.min() >= 0 and toks.max() < cfg.vocab
+        assert np.isfinite(lg).all()
+        assert np.mean(toks != t["tokens"].reshape(t["batch"], -1)[:, -1:]) >= 0.5
+
+
 @pytest.mark.parametrize("skip", ["fc2", "attn", "out"])
 def test_broken_layer_fails_the_check(E, skip):
     """The checks can fail: a decoder-layer kernel skipped (LIGER_DBG_SKIP, a timing
