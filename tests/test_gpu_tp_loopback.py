@@ -150,6 +150,26 @@ def test_full_size_opt13b_tp2_interleaved_equals_serial(E):
     assert st["overlapped_rounds"] > 0 and st["split_pieces"] > 0 and st["comm_kernels"] > 0
 
 
+def test_full_size_opt30b_tp4_modes(E):
+    """BASELINE.json configs[2] at full size: OPT-30B (48 layers, h = 7168) with 2 request
+    batches -- Algorithm 1 interleaving at TP = 4 equals serial TP = 4 bit for bit (tokens,
+    logits shards, residuals; all ranks the same residual), and the 4-stage Inter-Op
+    pipeline equals the unsharded single-GPU run bit for bit."""
+    cfg = get_config("opt-30b")
+    trace = make_trace(2, float("inf"), seed=6, vocab=cfg.vocab, n_decode=4, prompt_range=(128, 256))
+    kw = dict(max_batch=8, max_seq=256, max_new=4, seed=0)
+    inter = serve(E, cfg, 4, trace, mode="interleaved", max_inflight=2, decomp_factor=8, **kw)
+    ser = serve(E, cfg, 4, trace, mode="serial", **kw)
+    assert_bit_identical(inter, ser)
+    for r in range(1, 4):
+        for a, b in zip(inter[0]["tokens"] + inter[0]["resid"], inter[r]["tokens"] + inter[r]["resid"]):
+            assert np.array_equal(a, b)
+    del inter, ser
+    pipe = serve(E, cfg, 4, trace, mode="pipeline", max_inflight=4, **kw)
+    single = serve(E, cfg, 1, trace, mode="serial", **kw)
+    assert_bit_identical(single, [pipe[3]])
+
+
 @pytest.mark.parametrize("lead", ["0", "1000000"])
 def test_e1_placement_bit_exact(E, lead):
     """Hybrid sync E1 placement (DESIGN R8): the paper's (before the switch kernel, lead 0)
