@@ -170,6 +170,23 @@ def test_full_size_opt30b_tp4_modes(E):
     assert_bit_identical(single, [pipe[3]])
 
 
+def test_full_size_opt66b_tp8_interleaved_equals_serial(E):
+    """BASELINE.json configs[3] at full size: OPT-66B (64 layers, h = 9216) at TP = 8 (eight
+    loopback ranks, 16.5 GB of weights each, on the one GPU), kernel decomposition on:
+    Algorithm 1 interleaving equals serial TP bit for bit, every rank the same residual."""
+    cfg = get_config("opt-66b")
+    trace = make_trace(2, float("inf"), seed=8, vocab=cfg.vocab, n_decode=3, batch_sizes=(2, 4),
+                       prompt_range=(64, 128))
+    kw = dict(max_batch=4, max_seq=128, max_new=3, seed=0)
+    inter = serve(E, cfg, 8, trace, mode="interleaved", max_inflight=2, decomp_factor=8, **kw)
+    ser = serve(E, cfg, 8, trace, mode="serial", **kw)
+    assert_bit_identical(inter, ser)
+    for r in range(1, 8):
+        for a, b in zip(inter[0]["tokens"] + inter[0]["resid"], inter[r]["tokens"] + inter[r]["resid"]):
+            assert np.array_equal(a, b)
+    assert inter[0]["stats"]["overlapped_rounds"] > 0
+
+
 @pytest.mark.parametrize("lead", ["0", "1000000"])
 def test_e1_placement_bit_exact(E, lead):
     """Hybrid sync E1 placement (DESIGN R8): the paper's (before the switch kernel, lead 0)
