@@ -187,6 +187,27 @@ def test_full_size_opt66b_tp8_interleaved_equals_serial(E):
     assert inter[0]["stats"]["overlapped_rounds"] > 0
 
 
+def test_glm130b_layer_stack_tp8_cf_sweep(E):
+    """BASELINE.json configs[4] shape: a GLM-130B-shaped layer stack (h = 12288, 96 heads,
+    FFN 49152, tanh-GELU, vocab 150528; 6 of the 70 layers, which is what fits eight ranks on
+    one GPU) at TP = 8 with long prompts of 2048 tokens (100 MB prefill all-reduces,
+    decomposed): the contention-factor sweep of the scheduler (cf 1.0 / 1.1 / 1.3)
+    changes which kernels overlap, never the results -- every cf's run equals serial TP bit
+    for bit."""
+    cfg = get_config("glm-130b", 6)
+    trace = make_trace(2, float("inf"), seed=12, vocab=cfg.vocab, n_decode=3, batch_sizes=(1, 2),
+                       prompt_range=(2048, 2048))
+    kw = dict(max_batch=2, max_seq=2048, max_new=3, seed=0)
+    ser = serve(E, cfg, 8, trace, mode="serial", **kw)
+    rounds = {}
+    for cf in (1.0, 1.1, 1.3):
+        inter = serve(E, cfg, 8, trace, mode="interleaved", max_inflight=2, decomp_factor=8, contention_factor=cf,
+                      **kw)
+        assert_bit_identical(inter, ser)
+        rounds[cf] = inter[0]["stats"]["overlapped_rounds"]
+    assert all(v > 0 for v in rounds.values()), rounds
+
+
 @pytest.mark.parametrize("lead", ["0", "1000000"])
 def test_e1_placement_bit_exact(E, lead):
     """Hybrid sync E1 placement (DESIGN R8): the paper's (before the switch kernel, lead 0)
