@@ -76,21 +76,21 @@ size_t attn_decode_workspace_bytes(int b, int heads, int d, int ctx) {
 template <int D>
 struct DecSmem {
   __nv_bfloat16 kv[DC_NS][2][DC_CH * D];   // stage s: K rows then V rows of the chunk
-  float st_acc[4 * (32 / (D / 8))][D];     // per lane group: acc (item merge)
-  float st_m[4 * (32 / (D / 8))], st_l[4 * (32 / (D / 8))];
+  float st_acc[DC_CWARPS * (32 / (D / 8))][D];     // per lane group: acc (item merge)
+  float st_m[DC_CWARPS * (32 / (D / 8))], st_l[DC_CWARPS * (32 / (D / 8))];
   float mw[DC_MAX_SPLITS], lw[DC_MAX_SPLITS];
   uint64_t full[DC_NS], empty[DC_NS];
   int last;
 };
 
-// Warps 0..3 compute, warp 4 (lane 0) is the producer: it walks the same task list
+// Warps 0..DC_CWARPS-1 compute, warp DC_CWARPS (lane 0) is the producer: it walks the same task list
 // (chunk j of item i = blockIdx.x + k G) and keeps DC_NS chunks in flight, refilling a
 // stage as soon as the four compute warps have released it (empty[s]).
 template <int D>
-__global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecAttnArgs a) {
+__global__ void __launch_bounds__(DC_THREADS + 32, DC_CTAS_PER_SM) attn_decode_kernel(const DecAttnArgs a) {
   constexpr int LPT = D / 8;          // lanes per token row (16 B each)
   constexpr int TPW = 32 / LPT;       // token rows per warp step
-  constexpr int NG = 4 * TPW;         // lane groups per CTA
+  constexpr int NG = DC_CWARPS * TPW; // lane groups per CTA
   constexpr int PPG = DC_CH / NG;     // positions per lane group per chunk
   const TraceStart tr0 = trace_begin();
   extern __shared__ __align__(128) uint8_t dsm[];
@@ -107,12 +107,12 @@ __global__ void __launch_bounds__(DC_THREADS + 32) attn_decode_kernel(const DecA
   if (tid == 0) {
     for (int s = 0; s < DC_NS; ++s) {
       mbar_init(&sm.full[s], 1);
-      mbar_init(&sm.empty[s], 4);   // one arrive per compute warp
+      mbar_init(&sm.empty[s], DC_CWARPS);   // one arrive per compute warp
     }
     fence_barrier_init();
   }
   __syncthreads();
-  if (warp == 4) {
+  if (warp == DC_CWARPS) {
     // ---------------- producer warp: the page ids of up to 32 pages are fetched in one
     // parallel load (no serial page-table round trips on the refill path); lane 0
     // paces the ring, lanes 0 / 1 issue the two pages of a chunk

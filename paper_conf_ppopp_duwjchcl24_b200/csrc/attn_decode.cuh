@@ -37,7 +37,8 @@ namespace liger {
 constexpr int KVB = LIGER_KV_BLOCK;
 constexpr int DC_CH = 32;          // positions per chunk (two pages)
 constexpr int DC_NS = 4;           // ring stages per CTA
-constexpr int DC_THREADS = 128;
+constexpr int DC_THREADS = 128;      // compute threads (the producer warp comes on top)
+constexpr int DC_CWARPS = DC_THREADS / 32;
 constexpr int DC_CTAS_PER_SM = 3;
 constexpr int DC_MAX_SPLITS = 64;  // splits per (sequence, head)
 
