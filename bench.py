@@ -645,7 +645,8 @@ def rank_main(args, group, local, new_uid, result):
                                           "note": "two equal batches served together (both decode "
                                                   "concurrently); aggregate weight + KV stream"}
 
-    gemm_situ = decode_gemm_in_situ(eng, cfg, world, torch) if not gen else None
+    # (the in-kernel trace buffer is per process: not with loopback ranks sharing one)
+    gemm_situ = decode_gemm_in_situ(eng, cfg, world, torch) if not gen and not args.loopback else None
     if roof is not None and gemm_situ is not None and roof["kernel"] == "gemm_decode":
         gemm_situ["peak"] = hbm
         gemm_situ["frac"] = round(gemm_situ["achieved"] / hbm, 4)
@@ -746,8 +747,11 @@ def rank_main(args, group, local, new_uid, result):
             "gpu_launches": int(st["gpu_launches"]),
             "host": {"wall_s": round(wall_s, 3), "host_us": round(st["host_us"], 1),
                      "wait_us": round(st["wait_us"], 1), "rounds": st["rounds"], "kernels": st["kernels"],
+                     "comm_host_us": round(st["comm_host_us"], 1),
                      "host_us_per_round_excl_wait": round((st["host_us"] - st["wait_us"]) / max(1, st["rounds"]),
-                                                          2)},
+                                                          2),
+                     "host_us_per_round_excl_wait_and_comm": round(
+                         (st["host_us"] - st["wait_us"] - st["comm_host_us"]) / max(1, st["rounds"]), 2)},
         }
 
 

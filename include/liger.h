@@ -116,6 +116,8 @@ typedef struct {
   double host_us;           /* host time spent in liger_step (plan + launch + waits)          */
   double wait_us;           /* host time spent waiting on E1 events                            */
   int64_t gpu_launches;     /* CUDA kernel launches issued by the library                     */
+  double comm_host_us;      /* host time inside communication calls (NCCL enqueue; the loopback
+                               backend's rendezvous) -- part of host_us                          */
 } liger_stats_t;
 
 /* ------------------------------------------------------------------ lifecycle */

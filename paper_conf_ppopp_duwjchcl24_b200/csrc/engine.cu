@@ -606,7 +606,9 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
       const int F = op_units(c, po.op, M);
       const size_t E = (size_t)M * h;
       timed_begin(c, st, &ta);
+      const double h0 = now_s();
       if (issue_ar(c, S.part, E, u0, u1, F, st)) return fail(c, LIGER_ENCCL, c->comm->err);
+      c->st.comm_host_us += (now_s() - h0) * 1e6;
       timed_end(c, st, ta, LIGER_KT_ALLREDUCE, (double)(E * u1 / F - E * u0 / F) * 2, 0);
       c->st.comm_kernels++;
       c->st.gpu_launches++;
@@ -651,9 +653,11 @@ int launch_piece(liger_ctx* c, Batch* bt, int pass, int pidx, int u0, int u1, cu
     }
     case OP_TOKG: {
       const int b = bt->b;
+      const double h0 = now_s();
       if (c->comm->allgather2(S.vals_all + (size_t)c->rank * b, S.vals_all, b, CD_F32,
                               S.idx_all + (size_t)c->rank * b, S.idx_all, b, CD_I32, st))
         return fail(c, LIGER_ENCCL, c->comm->err);
+      c->st.comm_host_us += (now_s() - h0) * 1e6;
       c->st.comm_kernels++;
       c->st.gpu_launches++;
       break;

@@ -585,7 +585,25 @@ constexpr int LN_STATS_SMEM = 2 * 64 * 4;   // folded-LayerNorm row statistics (
 // are summed by the PDL-chained fixup kernel.  (An in-cluster DSMEM reduction, a
 // last-CTA reduction and an early fixup were built, measured slower and removed:
 // profiles/r01/cluster_splitk.txt.)
+static GemmPlan gemm_plan_compute(int M, int N, int K);
+
+// The plan of a shape is computed once per host thread (the cost model loops over split
+// counts: ~1-2 us, paid on every launch otherwise -- host time Algorithm 1's rounds
+// cannot afford when kernels run for a few microseconds)
 GemmPlan gemm_plan(int M, int N, int K) {
+  static thread_local std::unordered_map<uint64_t, GemmPlan> cache;
+  const uint64_t key = ((uint64_t)(uint32_t)M << 42) ^ ((uint64_t)(uint32_t)N << 21) ^ (uint64_t)(uint32_t)K;
+  if (M >= 0 && N >= 0 && K >= 0 && M < (1 << 21) && N < (1 << 21) && K < (1 << 21)) {
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+    const GemmPlan pl = gemm_plan_compute(M, N, K);
+    if (cache.size() < 4096) cache.emplace(key, pl);
+    return pl;
+  }
+  return gemm_plan_compute(M, N, K);
+}
+
+static GemmPlan gemm_plan_compute(int M, int N, int K) {
   GemmPlan pl{};
   const int G = num_sms();
   const int n_tiles = (N + BM - 1) / BM;

@@ -47,7 +47,7 @@ class liger_layer_weights(C.Structure):
 class liger_stats_t(C.Structure):
     _fields_ = [("rounds", C.c_int64), ("kernels", C.c_int64), ("comm_kernels", C.c_int64),
                 ("split_pieces", C.c_int64), ("overlapped_rounds", C.c_int64), ("host_us", C.c_double),
-                ("wait_us", C.c_double), ("gpu_launches", C.c_int64)]
+                ("wait_us", C.c_double), ("gpu_launches", C.c_int64), ("comm_host_us", C.c_double)]
 
 
 _lib = None
