@@ -110,3 +110,16 @@ def test_trace_summary_hand_computed():
     assert out["sms"] == 2 and out["span_ms"] == round(100 / 1e6, 2)
     assert out["sm_time_share"] == {"gemm": 0.3, "splitk_fixup": 0.2}
     assert out["no_gemm_working_frac"] == 0.5
+
+
+def test_trace_launches_groups_by_cta_repeat():
+    """bench.trace_launches: CTA records of one kernel kind, in entry order, split into launches
+    where a CTA index repeats (PDL: the next launch's CTAs enter before this one's exit); each
+    launch -> (first PDL-wait release, last exit, CTAs)."""
+    dt = np.dtype([("kid", "<u4"), ("cta", "<u4"), ("smid", "<u4"), ("pad", "<u4"),
+                   ("t0", "<u8"), ("t1", "<u8"), ("t2", "<u8")])
+    rows = [(1, 0, 0, 0, 10, 20, 50), (1, 1, 1, 0, 11, 21, 55), (2, 0, 0, 0, 12, 56, 60),
+            (1, 0, 2, 0, 40, 61, 90), (1, 1, 3, 0, 41, 62, 95), (1, 2, 4, 0, 42, 63, 99)]
+    rec = np.array(rows, dtype=dt)
+    assert bench.trace_launches(rec, 1) == [(20, 55, 2), (61, 99, 3)]
+    assert bench.trace_launches(rec, 2) == [(56, 60, 1)]
