@@ -763,6 +763,21 @@ def _free_port():
     return p
 
 
+def _watchdog(seconds):
+    """Fail loudly instead of hanging: a rank still running after `seconds` (e.g. a peer
+    lost in a collective) prints why and exits non-zero, so torchrun ends the job."""
+    if seconds <= 0:
+        return
+
+    def fire():
+        print(f"bench.py: rank {os.environ.get('RANK', '0')} still running after {seconds:.0f} s "
+              f"(LIGER_BENCH_TIMEOUT_S); exiting", file=sys.stderr, flush=True)
+        os._exit(3)
+    t = threading.Timer(seconds, fire)
+    t.daemon = True
+    t.start()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -809,6 +824,7 @@ def main():
     _redirect_stdout()
     if args.impl == "reference":
         return run_reference(args)
+    _watchdog(float(os.environ.get("LIGER_BENCH_TIMEOUT_S", "1800")))
 
     import torch
     result = {}
