@@ -7,7 +7,7 @@
 //  * work = (sequence, head, split); a split is a run of 32-position chunks (two
 //    16-token pages of K and of V, 4 x 4 KiB at d = 128); the split count is chosen
 //    per launch so that there is ~1 item per CTA slot;
-//  * a persistent grid of up to 3 CTAs per SM walks its items' chunks as one task
+//  * a persistent grid (about 2 items per SM, up to 3 CTAs resident) walks its items' chunks as one task
 //    stream through an NS-stage shared-memory ring filled by cp.async.bulk (the TMA
 //    bulk engine) on per-stage mbarriers: NS x 16 KiB in flight per CTA, ~192 KiB per
 //    SM, enough to cover the DRAM latency at the SM's share of HBM bandwidth; the
@@ -74,7 +74,11 @@ struct DecAttnArgs {
 // split only while there are fewer items than slots, never below one chunk per split.
 inline void dec_attn_plan(int b, int heads, int ctx, int* cps, int* nsp) {
   const int nch = (ctx + DC_CH - 1) / DC_CH;
-  static const int slots = getenv("LIGER_ATTN_SLOTS") ? atoi(getenv("LIGER_ATTN_SLOTS")) : 148 * DC_CTAS_PER_SM;
+  // 2 items per SM: with two batches decoding on the two streams, fewer attention CTAs
+  // leave more of each SM to the other batch's weight-streaming GEMM (bench capacity
+  // 30.35-30.49 vs 29.86-30.06 req/s with 3 per SM; one batch alone: equal within noise,
+  // profiles/r02/knob_sweeps_two_stream.txt)
+  static const int slots = getenv("LIGER_ATTN_SLOTS") ? atoi(getenv("LIGER_ATTN_SLOTS")) : 148 * 2;
   int want = slots / (b * heads);
   if (want < 1) want = 1;
   if (want > nch) want = nch;
